@@ -1,0 +1,397 @@
+#!/usr/bin/env python
+"""SNICIT hot-path benchmark: SDGC inference edges/s on B200 (BASELINE.json metric).
+
+    python bench.py [--gpus N] [--steps K] [--warmup W] [--config C2] [--impl snicit|reference]
+
+A step = one whole SNICIT inference (all SURVEY 8(a) rows: pre-convergence layers, conversion,
+post-convergence layers, recovery, categories) over one batch.  N=1 workload: config C2 (SDGC 4096
+neurons x 480 layers, batch 60,000, t=30, s=32, n=16, eta=eps=0.03), synthetic inputs (DESIGN.md
+section 5).  N>1 (torchrun, one rank per GPU, NCCL): weak scaling -- every rank infers its own 60,000-row
+batch (global row ids offset by rank), the category ids are all-gathered; value = rows of all ranks x
+connections / max-over-ranks step time.
+
+value: device-resident inputs (Y0 already in HBM), CUDA events around exactly K steps on the stream the
+library launches on, barrier + synchronize on both sides.  Inputs (983 MB) are larger than L2 (126 MB), so
+no explicit L2 flush.  e2e: the same metric through the C ABI with host (pinned) buffers: H2D of Y0 and D2H
+of Y(L) + categories inside the timed region.
+
+--impl reference: the CPU oracle (plain Eq. 1, oracle/) timed on the host cores on a bounded row sample of
+the same workload (rank 0 only).
+"""
+from __future__ import annotations
+
+import argparse
+import json
+import os
+import subprocess
+import sys
+import threading
+import time
+
+ROOT = os.path.dirname(os.path.abspath(__file__))
+sys.path.insert(0, ROOT)
+
+import numpy as np  # noqa: E402
+
+from workload import sdgc  # noqa: E402
+
+METRIC = "SDGC inference edges/sec at 1/2/4/8 B200; % of HBM roofline"
+UNIT = "edges/s"
+
+
+def parse():
+    p = argparse.ArgumentParser()
+    p.add_argument("--gpus", type=int, default=1)
+    p.add_argument("--steps", type=int, default=5)
+    p.add_argument("--warmup", type=int, default=3)
+    p.add_argument("--impl", choices=["snicit", "reference"], default="snicit")
+    p.add_argument("--config", default="C2", choices=["C1", "C2", "C3", "C4", "C5"])
+    p.add_argument("--mode", default="radix", choices=["radix", "perm", "random"])
+    p.add_argument("--t", type=int, default=None)
+    p.add_argument("--s", type=int, default=None)
+    p.add_argument("--kernel", default="auto", choices=["auto", "ell", "circ"])
+    p.add_argument("--scaling", default="weak", choices=["weak", "strong"])
+    p.add_argument("--batch", type=int, default=None, help="override rows per rank (weak) / global (strong)")
+    p.add_argument("--no-e2e", action="store_true")
+    p.add_argument("--no-cpu-baseline", action="store_true")
+    p.add_argument("--no-uncompressed", action="store_true")
+    p.add_argument("--cpu-seconds", type=float, default=15.0, help="target CPU work of the oracle sample")
+    return p.parse_args()
+
+
+def config_params(args):
+    c = dict(sdgc.CONFIGS[args.config])
+    if args.config == "C5":
+        snic = dict(t=sdgc.medium_t(c["L"]), s=128, n=0)
+    else:
+        snic = dict(t=30, s=32, n=16)
+    if args.t is not None:
+        snic["t"] = args.t
+    if args.s is not None:
+        snic["s"] = args.s
+    if args.batch is not None:
+        c["B"] = args.batch
+    return c, snic
+
+
+def make_network(args, c):
+    if args.config == "C5":
+        return sdgc.gen_medium_network(c["N"], c["L"])
+    return sdgc.gen_network(c["N"], c["L"], args.mode)
+
+
+def make_inputs(args, c, B, row0):
+    if args.config == "C5":
+        return sdgc.gen_medium_inputs(c["N"], B, row0=row0)
+    return sdgc.gen_inputs(c["N"], B, row0=row0)
+
+
+def cpu_info():
+    model = ""
+    try:
+        with open("/proc/cpuinfo") as f:
+            for line in f:
+                if line.startswith("model name"):
+                    model = line.split(":", 1)[1].strip()
+                    break
+    except OSError:
+        pass
+    return model
+
+
+# ------------------------------------------------------------------ clocks (nvidia-smi during the timed region)
+class ClockSampler:
+    Q = ("clocks.sm,clocks.max.sm,power.draw,clocks_event_reasons.active,clocks_event_reasons.hw_slowdown,"
+         "clocks_event_reasons.hw_thermal_slowdown,clocks_event_reasons.sw_thermal_slowdown,"
+         "clocks_event_reasons.sw_power_cap")
+
+    def __init__(self, index: int):
+        self.index = index
+        self.proc = None
+        self.lines = []
+
+    def start(self):
+        try:
+            self.proc = subprocess.Popen(["nvidia-smi", "-i", str(self.index), f"--query-gpu={self.Q}",
+                                          "--format=csv,noheader,nounits", "-lms", "200"],
+                                         stdout=subprocess.PIPE, stderr=subprocess.DEVNULL, text=True)
+            self.th = threading.Thread(target=self._read, daemon=True)
+            self.th.start()
+        except (OSError, FileNotFoundError):
+            self.proc = None
+
+    def _read(self):
+        for line in self.proc.stdout:
+            self.lines.append(line.strip())
+
+    def stop(self):
+        if self.proc is None:
+            return None
+        time.sleep(0.25)
+        self.proc.terminate()
+        try:
+            self.proc.wait(timeout=5)
+        except subprocess.TimeoutExpired:
+            self.proc.kill()
+        sm, mx, reasons = [], 0, set()
+        names = ["hw_slowdown", "hw_thermal_slowdown", "sw_thermal_slowdown", "sw_power_cap"]
+        for ln in self.lines:
+            parts = [p.strip() for p in ln.split(",")]
+            if len(parts) < 8:
+                continue
+            try:
+                sm.append(float(parts[0]))
+                mx = max(mx, float(parts[1]))
+            except ValueError:
+                continue
+            for nm, v in zip(names, parts[4:8]):
+                if v.lower().startswith("active"):
+                    reasons.add(nm)
+        if not sm:
+            return None
+        return {"sm_mhz": float(np.median(sm)), "sm_max_mhz": mx, "reasons": sorted(reasons), "samples": len(sm)}
+
+
+def measured_peaks():
+    p = os.path.join(ROOT, "MEASURED_PEAKS.json")
+    if os.path.exists(p):
+        with open(p) as f:
+            d = json.load(f)
+        return float(d["hbm_gbs"]), "measured (MEASURED_PEAKS.json hbm_gbs)"
+    return 6650.0, "fallback (B200_PROFILING.md: 6.65 TB/s)"
+
+
+# ------------------------------------------------------------------ reference arm (CPU oracle)
+def run_reference(args):
+    rank = int(os.environ.get("RANK", "0"))
+    if rank != 0:
+        return 0
+    import oracle
+
+    c, snic = config_params(args)
+    net = make_network(args, c)
+    nnz = net.nnz
+    cores = os.cpu_count() or 1
+    # size the per-step sample to ~cpu_seconds of the oracle on all cores (1 calibration row)
+    probe = make_inputs(args, c, 1, 0)
+    t0 = time.perf_counter()
+    oracle.layers_f32(net, probe, nthreads=1)
+    per_row = max(time.perf_counter() - t0, 1e-6)
+    rows = int(max(cores, min(c["B"], args.cpu_seconds * cores / per_row / max(args.steps, 1))))
+    rows = max(1, min(rows, c["B"]))
+    Y = make_inputs(args, c, rows, 0)
+    for _ in range(max(args.warmup, 0) if rows * per_row / cores < 2 else 1):
+        oracle.layers_f32(net, Y[: max(1, rows // 8)])
+    times = []
+    for _ in range(args.steps):
+        t0 = time.perf_counter()
+        oracle.layers_f32(net, Y)
+        times.append(time.perf_counter() - t0)
+    T = float(np.mean(times))
+    value = rows * nnz / T
+    sample = f"{rows} of {c['B']} rows of {args.config} (plain Eq. 1 oracle, all {net.L} layers), per step"
+    line = {
+        "impl": "reference", "metric": METRIC, "value": value, "unit": UNIT, "n_gpus": args.gpus,
+        "steps": args.steps, "warmup": args.warmup, "ms_per_step": T * 1e3, "higher_is_better": True,
+        "scaling": args.scaling, "vs_baseline": None, "dtype": "f32", "data": "synthetic",
+        "config": {"workload": f"{args.config}: {c['desc']}", "neurons": c["N"], "layers": c["L"],
+                   "batch": c["B"], "w_mode": args.mode, "t": snic["t"], "s": snic["s"]},
+        "cpu_baseline": {"value": value, "unit": UNIT, "cores": cores, "kind": "oracle", "sample": sample,
+                         "cpu": cpu_info()},
+        "e2e": {"value": value, "unit": UNIT, "h2d_bytes_per_step": 0, "d2h_bytes_per_step": 0},
+    }
+    print(json.dumps(line), flush=True)
+    return 0
+
+
+# ------------------------------------------------------------------ SNICIT arm
+def run_snicit(args):
+    import torch
+    import torch.distributed as dist
+
+    from paper_conf_icpp_jiangh0h23_b200 import KERNEL_AUTO, KERNEL_CIRC, KERNEL_ELL, SnicitNetwork, default_options
+    from paper_conf_icpp_jiangh0h23_b200.parallel import allgather_categories, shard_rows
+
+    world = int(os.environ.get("WORLD_SIZE", "1"))
+    rank = int(os.environ.get("RANK", "0"))
+    local = int(os.environ.get("LOCAL_RANK", "0"))
+    distributed = world > 1
+    if distributed:
+        torch.cuda.set_device(local)
+        dist.init_process_group("nccl", device_id=torch.device("cuda", local))
+    dev = torch.device("cuda", local)
+    torch.cuda.set_device(dev)
+
+    c, snic = config_params(args)
+    if args.scaling == "weak":
+        B_local, row0 = c["B"], rank * c["B"]
+        B_global = c["B"] * world
+    else:
+        a, b = shard_rows(c["B"], world, rank)
+        B_local, row0, B_global = b - a, a, c["B"]
+    net = make_network(args, c)
+    nnz = net.nnz
+    kern = {"auto": KERNEL_AUTO, "ell": KERNEL_ELL, "circ": KERNEL_CIRC}[args.kernel]
+    Yh = make_inputs(args, c, B_local, row0)
+    g = SnicitNetwork.from_network(net, device=local)
+    stream = torch.cuda.Stream(device=dev)
+    g.set_stream(stream)
+    y0 = torch.from_numpy(Yh).to(dev)
+    y_out = torch.empty_like(y0)
+    opt = default_options(kernel=kern, n_segments=snic["n"])
+    t, s = snic["t"], snic["s"]
+
+    def step():
+        g.infer(y0, t=t, s=s, options=opt, y_out=y_out, row_offset=row0)
+        if distributed:
+            with torch.cuda.stream(stream):
+                ids = torch.from_numpy(g.categories()).to(dev)
+                allgather_categories(ids)
+        else:
+            g.num_categories()  # category set present (count read synchronises the stream)
+
+    def timed(fn, k):
+        if distributed:
+            dist.barrier()
+        torch.cuda.synchronize(dev)
+        e0, e1 = torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)
+        e0.record(stream)
+        for _ in range(k):
+            fn()
+        e1.record(stream)
+        torch.cuda.synchronize(dev)
+        if distributed:
+            dist.barrier()
+        ms = e0.elapsed_time(e1) / k
+        if distributed:
+            tt = torch.tensor([ms], device=dev)
+            dist.all_reduce(tt, op=dist.ReduceOp.MAX)
+            ms = float(tt.item())
+        return ms
+
+    for _ in range(max(args.warmup, 3)):
+        step()
+    clocks = ClockSampler(local)
+    clocks.start()
+    ms = timed(step, args.steps)
+    clk = clocks.stop()
+    launches_per_step = g.stats()["kernel_launches"]
+    value = B_global * nnz / (ms * 1e-3)
+
+    # ---- roofline of the dominant kernel (the pre-convergence layer kernel), live CUDA events
+    opt_prof = default_options(kernel=kern, n_segments=snic["n"], timing=2)
+    prof_ms, prof_bytes, prof_rows = [], [], []
+    for _ in range(max(1, min(args.steps, 3))):
+        g.infer(y0, t=t, s=s, options=opt_prof, y_out=y_out, row_offset=row0)
+        pr = g.layer_profile()
+        prof_ms.append(pr["ms"])
+        prof_bytes.append(pr["bytes"])
+        prof_rows.append(pr["rows"])
+    st = g.stats()
+    phases = {k: st[k] for k in ("t_pre_ms", "t_convert_ms", "t_post_ms", "t_recover_ms", "t_total_ms")}
+    pm = np.mean(np.stack(prof_ms), axis=0) if prof_ms and len(prof_ms[0]) else np.zeros(0)
+    pb = prof_bytes[0] if prof_bytes else np.zeros(0)
+    peak, peak_src = measured_peaks()
+    roof = None
+    if len(pm):
+        avg_ms = float(pm.mean())
+        avg_bytes = float(pb.mean())
+        achieved = avg_bytes / (avg_ms * 1e-3) / 1e9
+        roof = {"bound": "hbm", "achieved": achieved, "peak": peak, "unit": "GB/s", "frac": achieved / peak,
+                "traffic": None, "kernel": "layer_circ_kernel" if st["circ_layers"] else "layer_ell_kernel",
+                "peak_source": peak_src, "launches": int(len(pm)), "avg_launch_ms": avg_ms,
+                "avg_algorithmic_bytes": avg_bytes,
+                "share_of_step": float(pm.sum() / ms) if ms > 0 else None,
+                "layer0_frac": float(pb[0] / (pm[0] * 1e-3) / 1e9 / peak)}
+
+    # ---- uncompressed GPU baseline (t >= L, same kernels)
+    unc = None
+    if not args.no_uncompressed:
+        def step_unc():
+            g.infer(y0, t=net.L, s=s, options=opt, y_out=y_out, row_offset=row0)
+            g.num_categories()
+        step_unc()
+        ms_u = timed(step_unc, max(1, min(args.steps, 3)))
+        unc = {"value": B_global * nnz / (ms_u * 1e-3), "unit": UNIT, "ms_per_step": ms_u,
+               "speedup_snicit": ms_u / ms}
+
+    # ---- e2e through the C ABI with host (pinned) buffers
+    e2e = None
+    if not args.no_e2e:
+        yh_pin = torch.from_numpy(Yh).pin_memory()
+        yo_pin = torch.empty_like(yh_pin).pin_memory()
+
+        def step_e2e():
+            g.infer(yh_pin.numpy(), t=t, s=s, options=opt, y_out=yo_pin.numpy(), row_offset=row0)
+            cats = g.categories()
+            if distributed:
+                with torch.cuda.stream(stream):
+                    allgather_categories(torch.from_numpy(cats).to(dev))
+            return cats
+        step_e2e()
+        if distributed:
+            dist.barrier()
+        torch.cuda.synchronize(dev)
+        k = max(1, min(args.steps, 3))
+        t0 = time.perf_counter()
+        for _ in range(k):
+            cats = step_e2e()
+        torch.cuda.synchronize(dev)
+        ms_e = (time.perf_counter() - t0) * 1e3 / k
+        if distributed:
+            tt = torch.tensor([ms_e], device=dev)
+            dist.all_reduce(tt, op=dist.ReduceOp.MAX)
+            ms_e = float(tt.item())
+        e2e = {"value": B_global * nnz / (ms_e * 1e-3), "unit": UNIT, "ms_per_step": ms_e,
+               "h2d_bytes_per_step": int(Yh.nbytes) * world, "d2h_bytes_per_step": (int(Yh.nbytes) + 8 * len(cats)) * world,
+               "timer": "host wall clock around K synchronous C-ABI calls"}
+
+    # ---- CPU oracle baseline (rank 0, N = 1 only), bounded sample
+    cpu = None
+    if rank == 0 and world == 1 and not args.no_cpu_baseline:
+        import oracle
+        cores = os.cpu_count() or 1
+        t0 = time.perf_counter()
+        oracle.layers_f32(net, Yh[:1], nthreads=1)
+        per_row = max(time.perf_counter() - t0, 1e-6)
+        rows = int(max(cores, min(B_local, args.cpu_seconds * cores / per_row)))
+        t0 = time.perf_counter()
+        oracle.layers_f32(net, Yh[:rows])
+        T = time.perf_counter() - t0
+        cpu = {"value": rows * nnz / T, "unit": UNIT, "cores": cores, "kind": "oracle",
+               "sample": f"{rows} of {B_local} rows, plain Eq. 1 oracle over all {net.L} layers ({T:.1f} s)",
+               "cpu": cpu_info()}
+
+    if rank == 0:
+        line = {
+            "metric": METRIC, "value": value, "unit": UNIT, "n_gpus": world, "steps": args.steps,
+            "warmup": max(args.warmup, 3), "ms_per_step": ms, "higher_is_better": True, "scaling": args.scaling,
+            "vs_baseline": None, "dtype": "f32", "data": "synthetic (seeded SDGC-like RadiX W, MNIST-like binary Y0)",
+            "config": {"workload": f"{args.config}: {c['desc']}", "neurons": c["N"], "layers": c["L"],
+                       "batch_per_rank": B_local, "global_batch": B_global, "connections": nnz, "w_mode": args.mode,
+                       "t": t, "s": s, "n": snic["n"], "eta": 0.03, "eps": 0.03, "kernel": args.kernel,
+                       "l2": "inputs larger than L2 (no flush)", "parallelism": f"dp{world} (row shards)"},
+            "roofline": roof, "cpu_baseline": cpu, "e2e": e2e, "clocks": clk,
+            "gpu_launches": int(launches_per_step * args.steps),
+            "uncompressed": unc, "phases_ms": phases,
+            "dynamics": {k: st[k] for k in ("live_at_t", "n_centroids", "n_sampled", "residual_at_t",
+                                            "residual_final", "n_categories")},
+            "paper_context": "SNICIT 4096-480 on 1x RTX A6000, B=60000: 44.17 ms = 8.55e13 edges/s (Table 3, P:1377)",
+        }
+        print(json.dumps(line), flush=True)
+    g.close()
+    if distributed:
+        dist.barrier()
+        dist.destroy_process_group()
+    return 0
+
+
+def main():
+    args = parse()
+    if args.impl == "reference":
+        return run_reference(args)
+    return run_snicit(args)
+
+
+if __name__ == "__main__":
+    sys.exit(main())

@@ -1,0 +1,181 @@
+/*
+ * snicit.h -- C ABI of libsnicit.so: SNICIT sparse-DNN inference on NVIDIA B200 (sm_100a).
+ *
+ * SNICIT (Jiang, Huang, Yu, Ho; ICPP 2023).  Citations are PAPER.md line numbers
+ * (P:<line>) of the paper text; readings R1..R23 are listed in DESIGN.md section 3.
+ *
+ * Problem (Eq. 1): Y(l+1) = sigma(Y(l) . W(l) + b(l)),
+ * sigma(x) = min(max(x, 0), ymax) (Table 2).  SNICIT (Fig. 2) runs the
+ * first t layers plainly, converts Y(t) into centroid rows + residue rows (Sec. 3.2,
+ * P:445-815), propagates centroids and non-empty residues (Sec. 3.3, Eq. 5)
+ * and recovers Y(L) (Eq. 6).  The category set (R13) is the ascending
+ * list of rows of Y(L) with any non-zero.
+ *
+ * Layout (R1): activations are B x N row-major fp32, one row per sample (the paper's
+ * column).  Layer l's weights are CSC over OUTPUT neurons: the inputs k of output j are
+ * idx[ptr[l*(N+1)+j] .. ptr[l*(N+1)+j+1]) with values val[..], in ACCUMULATION order (R12:
+ * acc = fmaf(y[k], w, acc) over the stored order, then + b[j], then clamp).
+ *
+ * Every compute step runs in hand-written CUDA kernels on the handle's device; there is no
+ * CPU fallback: without a usable sm_100 device every call returns SNICIT_E_CUDA.
+ *
+ * Thread-safety: a handle is not thread-safe; distinct handles may be used concurrently.
+ * Errors: every call returns snicit_status; snicit_last_error() gives a thread-local message.
+ */
+#ifndef SNICIT_H
+#define SNICIT_H
+#include <stdint.h>
+
+#ifdef __cplusplus
+extern "C" {
+#endif
+
+#define SNICIT_ABI_VERSION 1
+
+typedef struct snicit_network snicit_network; /* opaque: owns device copies of W, b + workspace */
+
+typedef enum {
+    SNICIT_OK = 0,
+    SNICIT_E_INVALID_ARG = -1, /* bad shape / pointer / parameter */
+    SNICIT_E_BAD_SPARSE = -2,  /* index out of range, duplicate in a column, ptr not monotone */
+    SNICIT_E_OOM = -3,         /* device allocation failed */
+    SNICIT_E_CUDA = -4,        /* CUDA runtime error or no sm_100 device */
+    SNICIT_E_STATE = -5,       /* e.g. categories requested before any infer */
+    SNICIT_E_UNSUPPORTED = -6
+} snicit_status;
+
+typedef enum {
+    SNICIT_CSC = 0, /* per output j: its inputs k (the paper's row j of W(i+1)) */
+    SNICIT_CSR = 1  /* per input k: its outputs j; transposed on load, entries of each output
+                       column then ordered by ascending k */
+} snicit_format;
+
+typedef enum {
+    SNICIT_KERNEL_AUTO = 0, /* shift-invariant layers use the circulant kernel, others ELL */
+    SNICIT_KERNEL_ELL = 1,  /* force the general gather kernel on every layer */
+    SNICIT_KERNEL_CIRC = 2  /* require the circulant kernel (error if a layer is not eligible) */
+} snicit_kernel;
+
+/* SNICIT parameters (s = 32, t = 30, n = 16, eps = eta = 0.03 for SDGC;
+ * P:1460-1465 medium nets: no downsampling, s = 128). */
+typedef struct {
+    int32_t n_segments;     /* n of sum downsampling; 0 = none (n = N), R15 */
+    float eta;              /* Eq. 2 threshold (absolute, R3) */
+    float eps;              /* Alg. 1 line 16: prune if diff < n*eps */
+    float prune_eps;        /* near-zero residual relaxation (R8); 0 = exact */
+    int32_t drop_dead_rows; /* 1 = exact zero-row compaction (R23) */
+    int32_t kernel;         /* snicit_kernel */
+    int32_t timing;         /* 1 = record per-phase CUDA-event times for snicit_stats;
+                               2 = also one event pair around every pre-convergence layer kernel
+                               (snicit_layer_profile) */
+    int32_t ne_interval;    /* host reads the active-residual count every this many post layers
+                               (P:966-970 uses 200) and stops launching residual work at 0;
+                               0 = default (64) */
+    int32_t reserved[4];
+} snicit_options;
+
+/* Per-run statistics of the last snicit_infer (times in ms, valid when options.timing). */
+typedef struct {
+    double t_pre_ms, t_convert_ms, t_post_ms, t_recover_ms, t_total_ms;
+    int64_t batch;            /* rows of this call */
+    int64_t live_at_t;        /* rows not dropped as dead at layer t */
+    int64_t residual_at_t;    /* non-empty residue rows right after conversion */
+    int64_t residual_final;   /* non-empty residue rows after the last layer */
+    int64_t n_categories;
+    int32_t n_centroids;      /* cent_cnt = |y*| */
+    int32_t n_sampled;        /* s actually sampled (min(s, live)) */
+    int32_t threshold_layer;  /* t used (min(t, L)) */
+    int32_t circ_layers;      /* layers run by the circulant kernel */
+    int64_t kernel_launches;  /* kernels launched by this infer */
+} snicit_stats_t;
+
+/* Fill *opt with the paper's SDGC defaults (n = 16, eta = eps = 0.03, prune_eps = 0,
+ * drop_dead_rows = 1, kernel = AUTO, timing = 0, ne_interval = 64). */
+void snicit_default_options(snicit_options* opt);
+
+/* Load a network (one-time; untimed in the benchmark).  All pointers are HOST pointers and
+ * are copied (the caller may free them on return).  n_layers >= 1, n_neurons >= 1.
+ * ptr: L*(N+1) int64 ABSOLUTE offsets into idx/val (layer l's first offset = layer l-1's last);
+ * for SNICIT_CSR the roles of rows/columns swap (per input k).  bias: L*N fp32.  ymax > 0.
+ * Validation: offsets monotone, 0 <= idx < N, no duplicate index within a column, finite
+ * values -> SNICIT_E_BAD_SPARSE / SNICIT_E_INVALID_ARG.  cuda_device: device ordinal.
+ * On success *out owns device memory until snicit_free_network. */
+snicit_status snicit_load_network(int32_t n_neurons, int32_t n_layers, snicit_format fmt,
+                                  const int64_t* ptr, const int32_t* idx, const float* val,
+                                  const float* bias, float ymax, int32_t cuda_device,
+                                  snicit_network** out);
+
+/* All work of this handle is issued on `cuda_stream` (a cudaStream_t, e.g.
+ * torch.cuda.current_stream().cuda_stream); NULL = the legacy default stream. */
+snicit_status snicit_set_stream(snicit_network* net, void* cuda_stream);
+
+/* Run inference on `batch` rows.
+ *  y0:              batch*N fp32 row-major (R1); device pointer if y0_on_device else host.
+ *                   Not modified.
+ *  row_offset:      global id of local row 0 (multi-GPU row sharding); category
+ *                   ids are row_offset + local row.
+ *  threshold_layer: t; t >= L runs the uncompressed plain path.
+ *  centroid_count:  s, the sample size and upper bound on cent_cnt; >= 1.
+ *  opt:             NULL = snicit_default_options.
+ *  y_out:           batch*N fp32, caller-owned; device pointer if y_out_on_device else host;
+ *                   NULL = do not materialise Y(L) (categories are still computed).
+ * Synchronous w.r.t. the host only when a host pointer is involved or opt->ne_interval
+ * triggers a count read; otherwise work is queued on the handle's stream.
+ * Call snicit_categories afterwards (it synchronises the stream). */
+snicit_status snicit_infer(snicit_network* net, const float* y0, int64_t batch,
+                           int32_t y0_on_device, int64_t row_offset, int32_t threshold_layer,
+                           int32_t centroid_count, const snicit_options* opt, float* y_out,
+                           int32_t y_out_on_device);
+
+/* Category ids of the last infer, ascending, as int64 global row ids (library-owned until
+ * the next infer/free; copied out here).  Two-call pattern: rows == NULL -> *count = total.
+ * Otherwise *count is the capacity of rows on entry and the number written on return
+ * (min(capacity, total)).
+ * rows_on_device != 0: rows is a device pointer (device-to-device copy, no host sync beyond
+ * the count).  SNICIT_E_STATE before any infer. */
+snicit_status snicit_categories(snicit_network* net, int64_t* rows, int64_t* count,
+                                int32_t rows_on_device);
+
+/* Statistics of the last infer (synchronises the stream). */
+snicit_status snicit_stats(snicit_network* net, snicit_stats_t* out);
+
+/* Per-launch profile of the pre-convergence layer kernels of the last infer run with
+ * options.timing == 2: for layer i < *n (n = min(t, max)): ms[i] = CUDA-event duration of the
+ * layer kernel launch (on the handle's stream), rows[i] = active rows it processed, bytes[i] =
+ * algorithmic HBM bytes of the launch (8*rows*N + W bytes + 4*N).
+ * Host pointers; any may be NULL.  Synchronises the stream. */
+snicit_status snicit_layer_profile(snicit_network* net, int32_t max, double* ms, int64_t* rows, double* bytes,
+                                   int32_t* n);
+
+/* ---- test hooks (used by tests/ for step-level parity; not needed by applications) ---- */
+
+/* Clustering state of the last infer (t < L): centroid row ids (ascending, <= s entries),
+ * cent_cnt, mapper M (batch int32: -1 centroid, -2 dead, else centroid row id), ne flags
+ * at layer t (batch uint8), F (n x n_sampled fp64, row-major), live flags at t (batch uint8).
+ * Any output pointer may be NULL.  Host pointers. */
+snicit_status snicit_debug_clustering(snicit_network* net, int32_t* cent, int32_t* n_cent,
+                                      int32_t* M, uint8_t* ne_t, double* F, int32_t* n_sampled,
+                                      uint8_t* live_t);
+
+/* One plain layer (Eq. 1) of the loaded network on `rows` device rows: yout = sigma(yin . W(l) + b(l)).
+ * kernel: SNICIT_KERNEL_ELL or SNICIT_KERNEL_CIRC (error if not eligible) or AUTO.
+ * yin, yout: device pointers, rows*N fp32, must not alias. */
+snicit_status snicit_debug_layer(snicit_network* net, int32_t layer, const float* yin,
+                                 float* yout, int64_t rows, int32_t kernel);
+
+/* 1 if layer l is eligible for the circulant kernel, 0 if not, < 0 on error. */
+int32_t snicit_layer_is_circulant(const snicit_network* net, int32_t layer);
+
+/* Release all device memory of the handle.  NULL is a no-op. */
+void snicit_free_network(snicit_network* net);
+
+/* Thread-local description of the last error ("" if none). */
+const char* snicit_last_error(void);
+
+/* SNICIT_ABI_VERSION of the loaded library. */
+int32_t snicit_abi_version(void);
+
+#ifdef __cplusplus
+}
+#endif
+#endif /* SNICIT_H */

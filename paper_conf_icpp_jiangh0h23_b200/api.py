@@ -1,0 +1,173 @@
+"""Python front end of the SNICIT C ABI (same names as include/snicit.h, argument marshalling only).
+
+Device memory, streams and process groups come from PyTorch; all compute is in libsnicit.so.
+"""
+from __future__ import annotations
+
+import ctypes
+from typing import Optional
+
+import numpy as np
+
+from . import _lib
+from ._lib import Options, SnicitError, Stats, check, default_options, load_library
+
+
+def _is_cuda_tensor(x) -> bool:
+    return hasattr(x, "is_cuda") and bool(x.is_cuda)
+
+
+class SnicitNetwork:
+    """Owns one `snicit_network*` (device copy of W, b + workspace) on `device`.
+
+    `ptr` (int64, L*(N+1) absolute offsets), `idx` (int32), `val` (float32), `bias` (float32, L*N):
+    CSC over output neurons with the accumulation order stored (include/snicit.h).
+    """
+
+    def __init__(self, N: int, L: int, ptr, idx, val, bias, ymax: float, device: int = 0, fmt: int = _lib.CSC):
+        self._lib = load_library()
+        self.N, self.L, self.ymax, self.device = int(N), int(L), float(ymax), int(device)
+        ptr = np.ascontiguousarray(ptr, dtype=np.int64)
+        idx = np.ascontiguousarray(idx, dtype=np.int32)
+        val = np.ascontiguousarray(val, dtype=np.float32)
+        bias = np.ascontiguousarray(bias, dtype=np.float32)
+        if ptr.size != self.L * (self.N + 1) or bias.size != self.L * self.N:
+            raise ValueError("ptr must have L*(N+1) entries and bias L*N")
+        h = ctypes.c_void_p()
+        st = self._lib.snicit_load_network(self.N, self.L, fmt, ptr.ctypes.data, idx.ctypes.data if idx.size else None,
+                                           val.ctypes.data if val.size else None, bias.ctypes.data, self.ymax,
+                                           self.device, ctypes.byref(h))
+        check(st, "snicit_load_network")
+        self._h = h
+        self._last_batch = 0
+        self._stream = None
+
+    @classmethod
+    def from_network(cls, net, device: int = 0):
+        """From a workload.sdgc.Network-like object (N, L, ptr, idx, val, bias, ymax)."""
+        return cls(net.N, net.L, net.ptr, net.idx, net.val, net.bias, net.ymax, device=device)
+
+    # ------------------------------------------------------------------ lifecycle
+    def close(self):
+        if getattr(self, "_h", None):
+            self._lib.snicit_free_network(self._h)
+            self._h = None
+
+    def __del__(self):
+        try:
+            self.close()
+        except Exception:
+            pass
+
+    def __enter__(self):
+        return self
+
+    def __exit__(self, *a):
+        self.close()
+
+    # ------------------------------------------------------------------ calls
+    def set_stream(self, stream) -> None:
+        """stream: a torch.cuda.Stream, a raw cudaStream_t int, or None (legacy default stream)."""
+        raw = None
+        if stream is not None:
+            raw = stream.cuda_stream if hasattr(stream, "cuda_stream") else int(stream)
+        self._stream = stream
+        check(self._lib.snicit_set_stream(self._h, raw), "snicit_set_stream")
+
+    def infer(self, y0, t: int, s: int = 32, options: Optional[Options] = None, y_out=None,
+              row_offset: int = 0, **opt_kw):
+        """Run SNICIT on y0 (B x N fp32: CUDA tensor, CPU tensor or numpy array).
+
+        y_out: None (not materialised), or a B x N fp32 CUDA tensor / CPU tensor / numpy array to fill.
+        Returns y_out.
+        """
+        if options is None:
+            options = default_options(**opt_kw)
+        elif opt_kw:
+            raise ValueError("pass either options or keyword options")
+        if _is_cuda_tensor(y0):
+            assert y0.dtype.__str__() == "torch.float32" and y0.is_contiguous()
+            B = int(y0.shape[0])
+            y0_dev, y0p = 1, y0.data_ptr()
+        else:
+            arr = y0.numpy() if hasattr(y0, "numpy") else y0
+            if not (isinstance(arr, np.ndarray) and arr.dtype == np.float32 and arr.flags.c_contiguous):
+                raise ValueError("host y0 must be a C-contiguous float32 array")
+            B = int(arr.shape[0])
+            y0_dev, y0p = 0, arr.ctypes.data
+        if B and int(y0.shape[1]) != self.N:
+            raise ValueError(f"y0 must be B x {self.N}")
+        if y_out is None:
+            yo_dev, yop = 0, None
+        elif _is_cuda_tensor(y_out):
+            yo_dev, yop = 1, y_out.data_ptr()
+        else:
+            ya = y_out.numpy() if hasattr(y_out, "numpy") else y_out
+            yo_dev, yop = 0, ya.ctypes.data
+        st = self._lib.snicit_infer(self._h, y0p, B, y0_dev, int(row_offset), int(t), int(s), ctypes.byref(options),
+                                    yop, yo_dev)
+        check(st, "snicit_infer")
+        self._last_batch = B
+        return y_out
+
+    def categories(self) -> np.ndarray:
+        """Ascending global row ids of the category set (R13) of the last infer."""
+        n = ctypes.c_int64(0)
+        check(self._lib.snicit_categories(self._h, None, ctypes.byref(n), 0), "snicit_categories")
+        out = np.empty(n.value, dtype=np.int64)
+        if n.value:
+            check(self._lib.snicit_categories(self._h, out.ctypes.data, ctypes.byref(n), 0), "snicit_categories")
+        return out[:n.value]
+
+    def num_categories(self) -> int:
+        n = ctypes.c_int64(0)
+        check(self._lib.snicit_categories(self._h, None, ctypes.byref(n), 0), "snicit_categories")
+        return int(n.value)
+
+    def stats(self) -> dict:
+        s = Stats()
+        check(self._lib.snicit_stats(self._h, ctypes.byref(s)), "snicit_stats")
+        return s.as_dict()
+
+    def layer_profile(self, max_layers: int = 4096) -> dict:
+        """Per pre-convergence layer kernel: CUDA-event ms, active rows, algorithmic bytes
+        (needs options.timing == 2 on the last infer)."""
+        ms = np.zeros(max_layers, np.float64)
+        rows = np.zeros(max_layers, np.int64)
+        by = np.zeros(max_layers, np.float64)
+        n = ctypes.c_int32(0)
+        check(self._lib.snicit_layer_profile(self._h, max_layers, ms.ctypes.data, rows.ctypes.data, by.ctypes.data,
+                                             ctypes.byref(n)), "snicit_layer_profile")
+        k = n.value
+        return dict(ms=ms[:k].copy(), rows=rows[:k].copy(), bytes=by[:k].copy())
+
+    def debug_clustering(self, n_segments: int = 16, s: int = 32) -> dict:
+        B = self._last_batch
+        n = self.N if n_segments == 0 else n_segments
+        cent = np.empty(max(s, 1), np.int32)
+        ncent = ctypes.c_int32(0)
+        M = np.empty(max(B, 1), np.int32)
+        ne = np.empty(max(B, 1), np.uint8)
+        F = np.empty(n * max(s, 1), np.float64)
+        ns = ctypes.c_int32(0)
+        live = np.empty(max(B, 1), np.uint8)
+        check(self._lib.snicit_debug_clustering(self._h, cent.ctypes.data, ctypes.byref(ncent), M.ctypes.data,
+                                                ne.ctypes.data, F.ctypes.data, ctypes.byref(ns), live.ctypes.data),
+              "snicit_debug_clustering")
+        return dict(cent=cent[:ncent.value].copy(), M=M[:B].copy(), ne_t=ne[:B].astype(bool),
+                    F=F[:n * ns.value].reshape(n, ns.value).copy(), n_sampled=ns.value, live_t=live[:B].astype(bool))
+
+    def debug_layer(self, layer: int, yin, yout, kernel: int = _lib.KERNEL_AUTO) -> None:
+        """One plain layer on CUDA tensors (rows x N)."""
+        assert _is_cuda_tensor(yin) and _is_cuda_tensor(yout)
+        check(self._lib.snicit_debug_layer(self._h, int(layer), yin.data_ptr(), yout.data_ptr(), int(yin.shape[0]),
+                                           int(kernel)), "snicit_debug_layer")
+
+    def layer_is_circulant(self, layer: int) -> bool:
+        r = self._lib.snicit_layer_is_circulant(self._h, int(layer))
+        if r < 0:
+            raise SnicitError("bad layer")
+        return bool(r)
+
+
+__all__ = ["SnicitNetwork", "Options", "Stats", "SnicitError", "default_options"]

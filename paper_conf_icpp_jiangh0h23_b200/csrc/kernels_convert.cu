@@ -1,0 +1,379 @@
+// kernels_convert.cu -- row compaction, cluster-based conversion and recovery kernels (sm_100a).
+//
+//  compact_kernel       ne_idx from ne_rec on device, order-preserving
+//  downsample_kernel    column sampling + sum downsampling (Sec. 3.2.1, Fig. 3a)
+//  prune_kernel         sample pruning, Alg. 1 with Eq. 2 (reading R2), then the
+//                       centroid list y*
+//  map_residual_kernel  mapper M (Eq. 3) and residue errors (Eq. 4),
+//                       Alg. 2
+//  recover_kernel       final results recovery (Eq. 6) + category flags (R13)
+#include <cuda_runtime.h>
+
+#include "snicit_internal.cuh"
+
+namespace snicit {
+
+__global__ void iota_kernel(int* out, int n, int* count_out) {
+    for (int i = blockIdx.x * blockDim.x + threadIdx.x; i < n; i += gridDim.x * blockDim.x) out[i] = i;
+    if (count_out && blockIdx.x == 0 && threadIdx.x == 0) *count_out = n;
+}
+cudaError_t launch_iota(int* out, int n, int* count_out, cudaStream_t st) {
+    int grid = n > 0 ? (n + 255) / 256 : 1;
+    if (grid > 4096) grid = 4096;
+    iota_kernel<<<grid, 256, 0, st>>>(out, n, count_out);
+    return cudaGetLastError();
+}
+
+__global__ void fill_i32_kernel(int* out, int n, int v) {
+    for (int i = blockIdx.x * blockDim.x + threadIdx.x; i < n; i += gridDim.x * blockDim.x) out[i] = v;
+}
+cudaError_t launch_fill_i32(int* out, int n, int v, cudaStream_t st) {
+    if (n <= 0) return cudaSuccess;
+    int grid = (n + 255) / 256;
+    if (grid > 4096) grid = 4096;
+    fill_i32_kernel<<<grid, 256, 0, st>>>(out, n, v);
+    return cudaGetLastError();
+}
+__global__ void fill_u8_kernel(uint8_t* out, int n, uint8_t v) {
+    for (int i = blockIdx.x * blockDim.x + threadIdx.x; i < n; i += gridDim.x * blockDim.x) out[i] = v;
+}
+cudaError_t launch_fill_u8(uint8_t* out, int n, uint8_t v, cudaStream_t st) {
+    if (n <= 0) return cudaSuccess;
+    int grid = (n + 255) / 256;
+    if (grid > 4096) grid = 4096;
+    fill_u8_kernel<<<grid, 256, 0, st>>>(out, n, v);
+    return cudaGetLastError();
+}
+
+// flag_row[rows[p]] = 1 for p < *count
+__global__ void mark_rows_kernel(const int* rows, const int* count, uint8_t* flag_row) {
+    const int n = *count;
+    for (int i = blockIdx.x * blockDim.x + threadIdx.x; i < n; i += gridDim.x * blockDim.x) flag_row[rows[i]] = 1;
+}
+cudaError_t launch_mark_rows(const int* rows, const int* count, uint8_t* flag_row, int max_rows, cudaStream_t st) {
+    int grid = max_rows > 0 ? (max_rows + 255) / 256 : 1;
+    if (grid > 4096) grid = 4096;
+    mark_rows_kernel<<<grid, 256, 0, st>>>(rows, count, flag_row);
+    return cudaGetLastError();
+}
+
+// One warp per listed row: flag_pos[p] = any_k y[rows[p]][k] != 0.
+__global__ void row_nonzero_kernel(const float* __restrict__ y, int N, const int* rows, const int* count,
+                                   uint8_t* flag_pos) {
+    const int n = *count;
+    const int lane = threadIdx.x & 31;
+    const int warps = (gridDim.x * blockDim.x) >> 5;
+    for (int p = (blockIdx.x * blockDim.x + threadIdx.x) >> 5; p < n; p += warps) {
+        const float* r = y + (size_t)rows[p] * N;
+        int any = 0;
+        for (int k = lane; k < N; k += 32) any |= (r[k] != 0.0f);
+        any = __any_sync(0xffffffffu, any);
+        if (lane == 0) flag_pos[p] = any ? 1 : 0;
+    }
+}
+cudaError_t launch_row_nonzero(const float* y, int N, const int* rows, const int* count, uint8_t* flag_pos,
+                               int max_rows, int num_sms, cudaStream_t st) {
+    int grid = (max_rows + 7) / 8;
+    if (grid > num_sms * 8) grid = num_sms * 8;
+    if (grid < 1) grid = 1;
+    row_nonzero_kernel<<<grid, 256, 0, st>>>(y, N, rows, count, flag_pos);
+    return cudaGetLastError();
+}
+
+// ------------------------------------------------------------------------------ compaction
+// Order-preserving stream compaction of list_in by flag_pos (indexed by list position), one CTA:
+// each thread owns a contiguous segment, counts its survivors, block-wide exclusive scan (warp
+// shuffles + one shared-memory pass), then scatters.  ne_idx "sorted indices of ne_rec == true"
+// is thereby rebuilt on device every layer instead of by the paper's serial host loop
+// -- result-neutral by reading R16.
+constexpr int kCompactThreads = 1024;
+__global__ void __launch_bounds__(kCompactThreads) compact_kernel(const int* __restrict__ list_in,
+                                                                  const int* count_in,
+                                                                  const uint8_t* __restrict__ flag_pos,
+                                                                  int* __restrict__ list_out, int* count_out) {
+    __shared__ int warp_sums[32];
+    const int n = *count_in;
+    const int per = (n + kCompactThreads - 1) / kCompactThreads;
+    const int beg = min(n, (int)threadIdx.x * per);
+    const int end = min(n, beg + per);
+    int c = 0;
+    for (int i = beg; i < end; ++i) c += flag_pos[i] ? 1 : 0;
+    const int lane = threadIdx.x & 31, wid = threadIdx.x >> 5;
+    int incl = c;
+#pragma unroll
+    for (int o = 1; o < 32; o <<= 1) {
+        const int v = __shfl_up_sync(0xffffffffu, incl, o);
+        if (lane >= o) incl += v;
+    }
+    if (lane == 31) warp_sums[wid] = incl;
+    __syncthreads();
+    if (wid == 0) {
+        int ws = warp_sums[lane];
+        int wi = ws;
+#pragma unroll
+        for (int o = 1; o < 32; o <<= 1) {
+            const int v = __shfl_up_sync(0xffffffffu, wi, o);
+            if (lane >= o) wi += v;
+        }
+        warp_sums[lane] = wi - ws;  // exclusive warp offsets
+        if (lane == 31) *count_out = wi;
+    }
+    __syncthreads();
+    int pos = warp_sums[wid] + incl - c;
+    for (int i = beg; i < end; ++i)
+        if (flag_pos[i]) list_out[pos++] = list_in[i];
+}
+cudaError_t launch_compact(const int* list_in, const int* count_in, const uint8_t* flag_pos, int* list_out,
+                           int* count_out, int /*max_n*/, cudaStream_t st) {
+    compact_kernel<<<1, kCompactThreads, 0, st>>>(list_in, count_in, flag_pos, list_out, count_out);
+    return cudaGetLastError();
+}
+
+// ------------------------------------------------------------------------------ conversion
+// Sum downsampling: block (g, q) sums segment g of sampled row q ("first s columns", of
+// the live list, R14) in fp64 (R3).  Segments of floor(N/n), last takes the remainder (R15).
+__global__ void downsample_kernel(const float* __restrict__ y, int N, const int* rows, const int* count, int s,
+                                  int n, double* F) {
+    const int q = blockIdx.y;
+    const int s_eff = min(s, *count);
+    if (q >= s_eff) return;
+    const int g = blockIdx.x;
+    const int seg = N / n;
+    const int k0 = g * seg, k1 = (g == n - 1) ? N : k0 + seg;
+    const float* r = y + (size_t)rows[q] * N;
+    double sum = 0.0;
+    for (int k = k0 + threadIdx.x; k < k1; k += blockDim.x) sum += (double)r[k];
+    __shared__ double red[32];
+#pragma unroll
+    for (int o = 16; o > 0; o >>= 1) sum += __shfl_down_sync(0xffffffffu, sum, o);
+    if ((threadIdx.x & 31) == 0) red[threadIdx.x >> 5] = sum;
+    __syncthreads();
+    if (threadIdx.x < 32) {
+        double v = (threadIdx.x < (blockDim.x >> 5)) ? red[threadIdx.x] : 0.0;
+#pragma unroll
+        for (int o = 16; o > 0; o >>= 1) v += __shfl_down_sync(0xffffffffu, v, o);
+        if (threadIdx.x == 0) F[(size_t)g * s + q] = v;
+    }
+}
+cudaError_t launch_downsample(const float* y, int N, const int* rows, const int* count, int s, int n_seg,
+                              double* F, cudaStream_t st) {
+    const int n = n_seg <= 0 ? N : n_seg;
+    const int seg = N / n;
+    const int threads = seg >= 256 ? 256 : (seg >= 64 ? 64 : 32);
+    dim3 grid(n, s);
+    downsample_kernel<<<grid, threads, 0, st>>>(y, N, rows, count, s, n, F);
+    return cudaGetLastError();
+}
+
+// Alg. 1 in one CTA (P:603-605 launches <<<1,(n,s)>>>; here threads loop over the n x s pairs so
+// any n*s works, R5).  diff counts are integer atomics in shared memory: order-independent and
+// deterministic.  After the loop the survivors (ascending position = ascending row id, since the
+// live list is ascending) form y*; cent_cnt = |y*|.
+constexpr int kPruneThreads = 1024;
+__global__ void __launch_bounds__(kPruneThreads) prune_kernel(const double* __restrict__ F, const int* count, int s,
+                                                              int n, float eta, float eps, const int* rows,
+                                                              int* cent, int* n_cent, int* s_eff_out,
+                                                              int* col_idx) {
+    extern __shared__ int sh[];
+    int* tmp_idx = sh;     // [s]
+    int* diff = sh + s;    // [s]
+    const int s_eff = min(s, *count);
+    for (int q = threadIdx.x; q < s_eff; q += blockDim.x) tmp_idx[q] = q;  // lines 3-4
+    const double thr = (double)n * (double)eps;
+    const double eta_d = (double)eta;
+    for (int cmp = 0; cmp < s_eff; ++cmp) {  // line 6
+        __syncthreads();
+        if (tmp_idx[cmp] == -1) continue;    // line 7 (uniform: read after the barrier)
+        for (int q = threadIdx.x; q < s_eff; q += blockDim.x) diff[q] = 0;  // lines 10-11
+        __syncthreads();
+        for (int p = threadIdx.x; p < n * s_eff; p += blockDim.x) {         // lines 13-14, Eq. 2
+            const int g = p / s_eff, q = p - g * s_eff;
+            if (q != cmp && tmp_idx[q] != -1) {
+                const double d = fabs(F[(size_t)g * s + q] - F[(size_t)g * s + cmp]);
+                if (d > eta_d) atomicAdd(&diff[q], 1);
+            }
+        }
+        __syncthreads();
+        for (int q = threadIdx.x; q < s_eff; q += blockDim.x)                // lines 16-17
+            if (q != cmp && tmp_idx[q] != -1 && (double)diff[q] < thr) tmp_idx[q] = -1;
+    }
+    __syncthreads();
+    if (threadIdx.x == 0) {
+        int C = 0;
+        for (int q = 0; q < s_eff; ++q) {
+            col_idx[q] = tmp_idx[q];
+            if (tmp_idx[q] != -1) cent[C++] = rows[q];
+        }
+        *n_cent = C;
+        *s_eff_out = s_eff;
+    }
+}
+cudaError_t launch_prune(const double* F, const int* count, int s, int n_seg, float eta, float eps,
+                         const int* rows, int* cent, int* n_cent, int* s_eff, int* col_idx, cudaStream_t st) {
+    const size_t smem = 2 * sizeof(int) * (size_t)s;
+    prune_kernel<<<1, kPruneThreads, smem, st>>>(F, count, s, n_seg, eta, eps, rows, cent, n_cent, s_eff, col_idx);
+    return cudaGetLastError();
+}
+
+// Alg. 2 / Eq. 3-4: one CTA per live row.  L0 distance to each centroid (element-wise '!=' counts,
+// Alg. 2 lines 10-12), first minimum over ascending y* wins (strict '<', R6).  Centroid rows are
+// copied to the compact centroid buffer (slot = position in y*), M = -1 and ne = 1 (R7); mapped
+// rows get M = centroid row id, ne = (dist != 0), and their residue Y_r - Y_c written only if ne.
+constexpr int kMapThreads = 256;
+__global__ void __launch_bounds__(kMapThreads) map_residual_kernel(const float* __restrict__ y, int N,
+                                                                   const int* rows, const int* count,
+                                                                   const int* cent, const int* n_cent, int* M,
+                                                                   int* cslot, uint8_t* ne_row, uint8_t* flag_pos,
+                                                                   float* __restrict__ yhat,
+                                                                   float* __restrict__ cbuf) {
+    __shared__ int red[kMapThreads / 32];
+    __shared__ int s_best, s_slot;
+    const int n = *count;
+    const int C = *n_cent;
+    const int lane = threadIdx.x & 31, wid = threadIdx.x >> 5;
+    const int N4 = N >> 2;
+    for (int p = blockIdx.x; p < n; p += gridDim.x) {
+        const int r = rows[p];
+        const float4* y4 = reinterpret_cast<const float4*>(y + (size_t)r * N);
+        if (threadIdx.x == 0) {
+            s_slot = -1;
+            for (int c = 0; c < C; ++c)
+                if (cent[c] == r) s_slot = c;
+        }
+        __syncthreads();
+        const int slot = s_slot;
+        if (slot >= 0) {  // centroid row (Eq. 4 second case)
+            float4* d4 = reinterpret_cast<float4*>(cbuf + (size_t)slot * N);
+            for (int k = threadIdx.x; k < N4; k += blockDim.x) d4[k] = y4[k];
+            if (threadIdx.x == 0) {
+                M[r] = -1;
+                cslot[r] = slot;
+                ne_row[r] = 1;
+                flag_pos[p] = 0;
+            }
+            __syncthreads();
+            continue;
+        }
+        int best_dist = N + 1, best = 0;  // Alg. 2 line 3 (tracked by thread 0)
+        for (int c = 0; c < C; ++c) {
+            const float4* c4 = reinterpret_cast<const float4*>(y + (size_t)cent[c] * N);
+            int cnt = 0;
+            for (int k = threadIdx.x; k < N4; k += blockDim.x) {
+                const float4 a = y4[k], b = c4[k];
+                cnt += (a.x != b.x) + (a.y != b.y) + (a.z != b.z) + (a.w != b.w);
+            }
+#pragma unroll
+            for (int o = 16; o > 0; o >>= 1) cnt += __shfl_down_sync(0xffffffffu, cnt, o);
+            if (lane == 0) red[wid] = cnt;
+            __syncthreads();
+            if (threadIdx.x == 0) {
+                int d = 0;
+                for (int w = 0; w < kMapThreads / 32; ++w) d += red[w];
+                if (d < best_dist) {  // lines 14-16
+                    best_dist = d;
+                    best = c;
+                }
+            }
+            __syncthreads();
+        }
+        if (threadIdx.x == 0) {
+            s_best = best;
+            s_slot = best_dist;  // reuse as the distance broadcast
+            M[r] = cent[best];   // line 25
+            cslot[r] = best;
+            const uint8_t ne = best_dist != 0 ? 1 : 0;  // lines 26-29
+            ne_row[r] = ne;
+            flag_pos[p] = ne;
+        }
+        __syncthreads();
+        if (s_slot != 0) {  // residue only needed for non-empty rows (Eq. 4 first case)
+            const float4* c4 = reinterpret_cast<const float4*>(y + (size_t)cent[s_best] * N);
+            float4* o4 = reinterpret_cast<float4*>(yhat + (size_t)r * N);
+            for (int k = threadIdx.x; k < N4; k += blockDim.x) {
+                const float4 a = y4[k], b = c4[k];
+                o4[k] = make_float4(a.x - b.x, a.y - b.y, a.z - b.z, a.w - b.w);
+            }
+        }
+        __syncthreads();
+    }
+}
+cudaError_t launch_map_residual(const float* y, int N, const int* rows, const int* count, const int* cent,
+                                const int* n_cent, int* M, int* cslot, uint8_t* ne_row, uint8_t* flag_pos,
+                                float* yhat, float* cbuf, int max_rows, int num_sms, cudaStream_t st) {
+    int grid = num_sms * 8;
+    if (grid > max_rows) grid = max_rows;
+    if (grid < 1) grid = 1;
+    map_residual_kernel<<<grid, kMapThreads, 0, st>>>(y, N, rows, count, cent, n_cent, M, cslot, ne_row, flag_pos,
+                                                      yhat, cbuf);
+    return cudaGetLastError();
+}
+
+// ------------------------------------------------------------------------------ recovery
+// Eq. 6: Y_r = Yhat_r (centroid); (ne ? Yhat_r : 0) + Yhat_M(r) (mapped, R18); 0 (dead, R23).
+// plain != 0 (t >= L): Y_r = live ? yfinal_r : 0.  cat[r] = any non-zero (R13).  One CTA per row.
+constexpr int kRecThreads = 256;
+__global__ void __launch_bounds__(kRecThreads) recover_kernel(int N, int R, int plain,
+                                                              const float* __restrict__ yfinal,
+                                                              const uint8_t* live_row, const int* M,
+                                                              const int* cslot, const uint8_t* ne_row,
+                                                              const float* __restrict__ cbuf,
+                                                              float* __restrict__ y_out, uint8_t* cat) {
+    const int N4 = N >> 2;
+    for (int r = blockIdx.x; r < R; r += gridDim.x) {
+        int mode;  // 0 zero, 1 copy a, 2 a + c, 3 0 + c
+        const float4* a4 = nullptr;
+        const float4* c4 = nullptr;
+        if (plain) {
+            mode = live_row[r] ? 1 : 0;
+            a4 = reinterpret_cast<const float4*>(yfinal + (size_t)r * N);
+        } else {
+            const int m = M[r];
+            if (m == -2) {
+                mode = 0;
+            } else if (m == -1) {
+                mode = 1;
+                a4 = reinterpret_cast<const float4*>(cbuf + (size_t)cslot[r] * N);
+            } else {
+                c4 = reinterpret_cast<const float4*>(cbuf + (size_t)cslot[r] * N);
+                if (ne_row[r]) {
+                    mode = 2;
+                    a4 = reinterpret_cast<const float4*>(yfinal + (size_t)r * N);
+                } else {
+                    mode = 3;
+                }
+            }
+        }
+        int any = 0;
+        float4* o4 = y_out ? reinterpret_cast<float4*>(y_out + (size_t)r * N) : nullptr;
+        for (int k = threadIdx.x; k < N4; k += blockDim.x) {
+            float4 v;
+            if (mode == 0) {
+                v = make_float4(0.f, 0.f, 0.f, 0.f);
+            } else if (mode == 1) {
+                v = a4[k];
+            } else if (mode == 2) {
+                const float4 a = a4[k], c = c4[k];
+                v = make_float4(a.x + c.x, a.y + c.y, a.z + c.z, a.w + c.w);
+            } else {
+                const float4 c = c4[k];
+                v = make_float4(0.0f + c.x, 0.0f + c.y, 0.0f + c.z, 0.0f + c.w);
+            }
+            any |= (v.x != 0.f) | (v.y != 0.f) | (v.z != 0.f) | (v.w != 0.f);
+            if (o4) o4[k] = v;
+        }
+        any = __syncthreads_or(any);
+        if (threadIdx.x == 0) cat[r] = any ? 1 : 0;
+    }
+}
+cudaError_t launch_recover(int N, int R, int plain, const float* yfinal, const uint8_t* live_row, const int* M,
+                           const int* cslot, const uint8_t* ne_row, const float* cbuf, float* y_out,
+                           uint8_t* cat, int num_sms, cudaStream_t st) {
+    if (R <= 0) return cudaSuccess;
+    int grid = num_sms * 8;
+    if (grid > R) grid = R;
+    recover_kernel<<<grid, kRecThreads, 0, st>>>(N, R, plain, yfinal, live_row, M, cslot, ne_row, cbuf, y_out,
+                                                 cat);
+    return cudaGetLastError();
+}
+
+}  // namespace snicit

@@ -1,0 +1,814 @@
+// snicit_api.cu -- host runtime of libsnicit.so: the C ABI of include/snicit.h.
+//
+// Owns the device copies of the network, the per-batch workspace and the stream, validates every
+// argument, and sequences the kernels of the hot path:
+//   a1 pre-convergence layers (Eq. 1)  ->  a2 sampling + sum downsampling  ->  a3 Alg. 1 pruning
+//   ->  a4 Alg. 2 mapping + residues  ->  a5 post-convergence layers (Eq. 5) + row compaction
+//   ->  a6 Eq. 6 recovery + categories.
+// No computation of the method happens on the host; host code only launches kernels, moves
+// buffers the caller asked for, and reads device counters.
+#include <cuda_runtime.h>
+#include <stdint.h>
+#include <string.h>
+
+#include <algorithm>
+#include <cmath>
+#include <string>
+#include <vector>
+
+#include "../../include/snicit.h"
+#include "snicit_internal.cuh"
+
+using namespace snicit;
+
+namespace {
+
+thread_local std::string g_last_error;
+
+snicit_status fail(snicit_status st, const std::string& msg) {
+    g_last_error = msg;
+    return st;
+}
+
+#define CUDA_TRY(expr)                                                                            \
+    do {                                                                                          \
+        cudaError_t _e = (expr);                                                                  \
+        if (_e != cudaSuccess)                                                                    \
+            return fail(_e == cudaErrorMemoryAllocation ? SNICIT_E_OOM : SNICIT_E_CUDA,          \
+                        std::string(#expr) + ": " + cudaGetErrorString(_e));                     \
+    } while (0)
+
+template <typename T>
+struct DevBuf {
+    T* p = nullptr;
+    size_t n = 0;
+    cudaError_t ensure(size_t count) {
+        if (count <= n && p) return cudaSuccess;
+        if (p) cudaFree(p);
+        p = nullptr;
+        n = 0;
+        cudaError_t e = cudaMalloc(&p, std::max<size_t>(count, 1) * sizeof(T));
+        if (e == cudaSuccess) n = count;
+        return e;
+    }
+    void release() {
+        if (p) cudaFree(p);
+        p = nullptr;
+        n = 0;
+    }
+};
+
+// device counters (one int each)
+enum Counter { CNT_LIVE0 = 0, CNT_LIVE1, CNT_RES0, CNT_RES1, CNT_NCENT, CNT_SEFF, CNT_ALL, CNT_NCAT, CNT_N };
+
+}  // namespace
+
+struct snicit_network {
+    int device = 0;
+    int N = 0, L = 0;
+    float ymax = 32.f;
+    int num_sms = 148;
+    cudaStream_t stream = nullptr;
+    std::vector<LayerPlan> plan;
+    std::vector<uint8_t> dead_ok;  // dead_ok[l]: all biases of layers >= l are <= 0 (R23)
+    bool idx16 = true;
+    // weights
+    DevBuf<uint16_t> idx16_d;
+    DevBuf<int32_t> idx32_d;
+    DevBuf<float> val_d;
+    DevBuf<uint8_t> len_d;
+    DevBuf<float> wtab_d;
+    DevBuf<float> bias_d;
+    // workspace
+    int64_t cap_rows = 0;
+    int cap_s = 0, cap_n = 0;
+    DevBuf<float> Ya, Yb;
+    DevBuf<int> list0, list1, res0, res1, M, cslot, catlist, cent, col_idx, iota_s;
+    DevBuf<uint8_t> flag_pos, live_row, ne_row, cat, ne_t;
+    DevBuf<float> cbuf0, cbuf1, ac;
+    DevBuf<double> F;
+    DevBuf<int> counters;
+    int* h_counters = nullptr;  // pinned mirror
+    // last-run state
+    bool have_result = false;
+    int64_t last_batch = 0, last_offset = 0;
+    int last_t = 0;
+    int last_s = 0, last_n = 0;
+    bool last_converted = false;
+    int live_counter = 0;  // which CNT_LIVE* holds the live count at t
+    bool last_kernel_circ = false;
+    snicit_stats_t stats{};
+    cudaEvent_t ev[6] = {nullptr, nullptr, nullptr, nullptr, nullptr, nullptr};
+    std::vector<cudaEvent_t> lev;  // 2 per pre-convergence layer (timing == 2)
+    DevBuf<int> hist;              // active rows at the start of each pre-convergence layer
+    int prof_layers = 0;
+};
+
+extern "C" {
+
+void snicit_default_options(snicit_options* opt) {
+    if (!opt) return;
+    memset(opt, 0, sizeof(*opt));
+    opt->n_segments = 16;
+    opt->eta = 0.03f;
+    opt->eps = 0.03f;
+    opt->prune_eps = 0.0f;  // exact (R8)
+    opt->drop_dead_rows = 1;
+    opt->kernel = SNICIT_KERNEL_AUTO;
+    opt->timing = 0;
+    opt->ne_interval = 64;
+}
+
+const char* snicit_last_error(void) { return g_last_error.c_str(); }
+int32_t snicit_abi_version(void) { return SNICIT_ABI_VERSION; }
+
+void snicit_free_network(snicit_network* net) {
+    if (!net) return;
+    if (cudaSetDevice(net->device) == cudaSuccess && net->stream) cudaStreamSynchronize(net->stream);
+    net->idx16_d.release();
+    net->idx32_d.release();
+    net->val_d.release();
+    net->len_d.release();
+    net->wtab_d.release();
+    net->bias_d.release();
+    net->Ya.release();
+    net->Yb.release();
+    for (auto* b : {&net->list0, &net->list1, &net->res0, &net->res1, &net->M, &net->cslot, &net->catlist, &net->cent,
+                    &net->col_idx, &net->iota_s, &net->counters})
+        b->release();
+    for (auto* b : {&net->flag_pos, &net->live_row, &net->ne_row, &net->cat, &net->ne_t}) b->release();
+    net->cbuf0.release();
+    net->cbuf1.release();
+    net->ac.release();
+    net->F.release();
+    if (net->h_counters) cudaFreeHost(net->h_counters);
+    for (auto& e : net->ev)
+        if (e) cudaEventDestroy(e);
+    for (auto& e : net->lev)
+        if (e) cudaEventDestroy(e);
+    net->hist.release();
+    delete net;
+}
+
+snicit_status snicit_load_network(int32_t N, int32_t L, snicit_format fmt, const int64_t* ptr, const int32_t* idx,
+                                  const float* val, const float* bias, float ymax, int32_t cuda_device,
+                                  snicit_network** out) {
+    if (!out) return fail(SNICIT_E_INVALID_ARG, "out is NULL");
+    *out = nullptr;
+    if (N < 1 || L < 1) return fail(SNICIT_E_INVALID_ARG, "n_neurons and n_layers must be >= 1");
+    if (!ptr || !bias) return fail(SNICIT_E_INVALID_ARG, "ptr/bias NULL");
+    if (!(ymax > 0.0f) || std::isnan(ymax)) return fail(SNICIT_E_INVALID_ARG, "ymax must be > 0");
+    if (fmt != SNICIT_CSC && fmt != SNICIT_CSR) return fail(SNICIT_E_INVALID_ARG, "bad format");
+    if (N % 4 != 0) return fail(SNICIT_E_UNSUPPORTED, "n_neurons must be a multiple of 4 (16-byte rows)");
+    // ---- host-side validation and conversion to per-layer column lists (stored order kept)
+    std::vector<std::vector<int32_t>> cidx(N);
+    std::vector<std::vector<float>> cval(N);
+    const int64_t nnz_total = ptr[(int64_t)L * (N + 1) - 1];
+    if (nnz_total < 0) return fail(SNICIT_E_BAD_SPARSE, "negative nnz");
+    if (nnz_total > 0 && (!idx || !val)) return fail(SNICIT_E_INVALID_ARG, "idx/val NULL");
+    for (int64_t i = 0; i < nnz_total; ++i)
+        if (!std::isfinite(val[i])) return fail(SNICIT_E_INVALID_ARG, "non-finite weight");
+    for (int64_t i = 0; i < (int64_t)L * N; ++i)
+        if (!std::isfinite(bias[i])) return fail(SNICIT_E_INVALID_ARG, "non-finite bias");
+
+    auto* net = new snicit_network();
+    net->device = cuda_device;
+    net->N = N;
+    net->L = L;
+    net->ymax = ymax;
+    net->idx16 = N <= 65536;
+    net->plan.resize(L);
+
+    std::vector<int> Ks(L);
+    size_t ell_total = 0;
+    std::vector<std::vector<int32_t>> lay_idx(L);
+    std::vector<std::vector<float>> lay_val(L);
+    std::vector<std::vector<uint8_t>> lay_len(L);
+    std::vector<float> wtab;
+    std::vector<uint8_t> mark(N, 0);
+    for (int l = 0; l < L; ++l) {
+        const int64_t* p = ptr + (int64_t)l * (N + 1);
+        if (l > 0 && p[0] != ptr[(int64_t)l * (N + 1) - 1]) {
+            snicit_free_network(net);
+            return fail(SNICIT_E_BAD_SPARSE, "layer offsets not contiguous at layer " + std::to_string(l));
+        }
+        if (l == 0 && p[0] != 0) {
+            snicit_free_network(net);
+            return fail(SNICIT_E_BAD_SPARSE, "ptr[0] must be 0");
+        }
+        for (int j = 0; j < N; ++j) {
+            cidx[j].clear();
+            cval[j].clear();
+        }
+        for (int j = 0; j < N; ++j) {
+            if (p[j + 1] < p[j]) {
+                snicit_free_network(net);
+                return fail(SNICIT_E_BAD_SPARSE, "ptr not monotone");
+            }
+            for (int64_t e = p[j]; e < p[j + 1]; ++e) {
+                const int32_t k = idx[e];
+                if (k < 0 || k >= N) {
+                    snicit_free_network(net);
+                    return fail(SNICIT_E_BAD_SPARSE, "index out of range");
+                }
+                if (fmt == SNICIT_CSC) {
+                    cidx[j].push_back(k);
+                    cval[j].push_back(val[e]);
+                } else {  // CSR: entry (input j, output k); columns then ascending in input
+                    cidx[k].push_back(j);
+                    cval[k].push_back(val[e]);
+                }
+            }
+        }
+        int K = 0;
+        bool ragged = false;
+        for (int j = 0; j < N; ++j) {
+            for (int32_t k : cidx[j]) {
+                if (mark[k]) {
+                    for (int32_t kk : cidx[j]) mark[kk] = 0;
+                    snicit_free_network(net);
+                    return fail(SNICIT_E_BAD_SPARSE, "duplicate index in a column of layer " + std::to_string(l));
+                }
+                mark[k] = 1;
+            }
+            for (int32_t k : cidx[j]) mark[k] = 0;
+            K = std::max<int>(K, (int)cidx[j].size());
+        }
+        for (int j = 0; j < N; ++j)
+            if ((int)cidx[j].size() != K) ragged = true;
+        if (K > 255) {
+            snicit_free_network(net);
+            return fail(SNICIT_E_UNSUPPORTED, "more than 255 inputs per output neuron");
+        }
+        Ks[l] = K;
+        LayerPlan& pl = net->plan[l];
+        pl.K = K;
+        pl.ragged = ragged;
+        pl.ell_off = ell_total;
+        ell_total += (size_t)K * N;
+        // uniform value?
+        bool uniform = true;
+        float w0 = 0.f;
+        bool first = true;
+        for (int j = 0; j < N && uniform; ++j)
+            for (float v : cval[j]) {
+                if (first) {
+                    w0 = v;
+                    first = false;
+                } else if (v != w0 || std::signbit(v) != std::signbit(w0)) {
+                    uniform = false;
+                    break;
+                }
+            }
+        pl.uniform = uniform;
+        pl.w0 = w0;
+        // circulant? column j = (j + n*nu) mod N for n = 0..K-1, per-n weights uniform over j
+        pl.kind = 0;
+        pl.nu = 0;
+        if (!ragged && K >= 2) {
+            const int nu = (int)(((int64_t)cidx[0][1] - cidx[0][0] + N) % N);
+            bool circ = cidx[0][0] == 0 && circ_supported(N, K, nu);
+            for (int j = 0; j < N && circ; ++j)
+                for (int n = 0; n < K; ++n) {
+                    if (cidx[j][n] != (int32_t)(((int64_t)j + (int64_t)n * nu) % N) || cval[j][n] != cval[0][n] ||
+                        std::signbit(cval[j][n]) != std::signbit(cval[0][n])) {
+                        circ = false;
+                        break;
+                    }
+                }
+            if (circ) {
+                pl.kind = 1;
+                pl.nu = nu;
+                pl.w_off = wtab.size();
+                for (int n = 0; n < K; ++n) wtab.push_back(cval[0][n]);
+            }
+        }
+        // ELL (n-major) copy for every layer (ELL kernel and debug comparisons)
+        lay_idx[l].assign((size_t)K * N, 0);
+        lay_val[l].assign((size_t)K * N, 0.0f);
+        if (ragged) lay_len[l].assign(N, 0);
+        for (int j = 0; j < N; ++j) {
+            for (size_t n = 0; n < cidx[j].size(); ++n) {
+                lay_idx[l][n * N + j] = cidx[j][n];
+                lay_val[l][n * N + j] = cval[j][n];
+            }
+            if (ragged) lay_len[l][j] = (uint8_t)cidx[j].size();
+        }
+    }
+    // dead_ok
+    net->dead_ok.assign(L + 1, 1);
+    for (int l = L - 1; l >= 0; --l) {
+        bool ok = net->dead_ok[l + 1];
+        for (int j = 0; j < N; ++j)
+            if (bias[(int64_t)l * N + j] > 0.0f) ok = false;
+        net->dead_ok[l] = ok ? 1 : 0;
+    }
+    // ---- device (validation above needs no GPU, so bad input is reported on any host)
+    {
+        int ndev = 0;
+        if (cudaGetDeviceCount(&ndev) != cudaSuccess || ndev < 1) {
+            snicit_free_network(net);
+            return fail(SNICIT_E_CUDA, "no CUDA device");
+        }
+        if (cuda_device < 0 || cuda_device >= ndev) {
+            snicit_free_network(net);
+            return fail(SNICIT_E_INVALID_ARG, "bad cuda_device");
+        }
+        cudaDeviceProp prop;
+        cudaError_t pe = cudaGetDeviceProperties(&prop, cuda_device);
+        if (pe != cudaSuccess || prop.major != 10) {
+            snicit_free_network(net);
+            return fail(SNICIT_E_CUDA, pe != cudaSuccess ? std::string(cudaGetErrorString(pe))
+                                                         : "libsnicit is built for sm_100a (B200); device is sm_" +
+                                                               std::to_string(prop.major) + std::to_string(prop.minor));
+        }
+        net->num_sms = prop.multiProcessorCount;
+        cudaSetDevice(cuda_device);
+    }
+    // ---- upload
+    auto up = [&](auto& buf, const auto* host, size_t count) -> cudaError_t {
+        cudaError_t e = buf.ensure(count);
+        if (e != cudaSuccess) return e;
+        if (count) return cudaMemcpy(buf.p, host, count * sizeof(*host), cudaMemcpyHostToDevice);
+        return cudaSuccess;
+    };
+    cudaError_t e = cudaSuccess;
+    {
+        std::vector<float> allv(ell_total);
+        for (int l = 0; l < L; ++l) std::copy(lay_val[l].begin(), lay_val[l].end(), allv.begin() + net->plan[l].ell_off);
+        if (net->idx16) {
+            std::vector<uint16_t> alli(ell_total);
+            for (int l = 0; l < L; ++l)
+                for (size_t i = 0; i < lay_idx[l].size(); ++i) alli[net->plan[l].ell_off + i] = (uint16_t)lay_idx[l][i];
+            e = up(net->idx16_d, alli.data(), ell_total);
+        } else {
+            std::vector<int32_t> alli(ell_total);
+            for (int l = 0; l < L; ++l) std::copy(lay_idx[l].begin(), lay_idx[l].end(), alli.begin() + net->plan[l].ell_off);
+            e = up(net->idx32_d, alli.data(), ell_total);
+        }
+        if (e == cudaSuccess) e = up(net->val_d, allv.data(), ell_total);
+        bool any_rag = false;
+        for (int l = 0; l < L; ++l) any_rag |= net->plan[l].ragged;
+        if (e == cudaSuccess && any_rag) {
+            std::vector<uint8_t> alll((size_t)L * N, 0);
+            for (int l = 0; l < L; ++l)
+                if (net->plan[l].ragged) std::copy(lay_len[l].begin(), lay_len[l].end(), alll.begin() + (size_t)l * N);
+            e = up(net->len_d, alll.data(), alll.size());
+        }
+    }
+    if (e == cudaSuccess) e = up(net->wtab_d, wtab.data(), wtab.size());
+    if (e == cudaSuccess) e = up(net->bias_d, bias, (size_t)L * N);
+    if (e == cudaSuccess) e = net->counters.ensure(CNT_N);
+    if (e == cudaSuccess) e = cudaMallocHost(&net->h_counters, sizeof(int) * CNT_N);
+    for (int i = 0; i < 6 && e == cudaSuccess; ++i) e = cudaEventCreate(&net->ev[i]);
+    if (e != cudaSuccess) {
+        snicit_free_network(net);
+        return fail(e == cudaErrorMemoryAllocation ? SNICIT_E_OOM : SNICIT_E_CUDA, cudaGetErrorString(e));
+    }
+    *out = net;
+    return SNICIT_OK;
+}
+
+snicit_status snicit_set_stream(snicit_network* net, void* s) {
+    if (!net) return fail(SNICIT_E_INVALID_ARG, "net NULL");
+    net->stream = (cudaStream_t)s;
+    return SNICIT_OK;
+}
+
+int32_t snicit_layer_is_circulant(const snicit_network* net, int32_t l) {
+    if (!net || l < 0 || l >= net->L) return -1;
+    return net->plan[l].kind == 1 ? 1 : 0;
+}
+
+}  // extern "C"
+
+// ---------------------------------------------------------------------------------------- helpers
+static LayerArgs layer_args(snicit_network* net, int l, bool force_ell) {
+    const LayerPlan& pl = net->plan[l];
+    LayerArgs a{};
+    a.N = net->N;
+    a.bias = net->bias_d.p + (size_t)l * net->N;
+    a.ymax = net->ymax;
+    a.K = pl.K;
+    if (net->idx16)
+        a.idx16 = net->idx16_d.p + pl.ell_off;
+    else
+        a.idx32 = net->idx32_d.p + pl.ell_off;
+    a.val = pl.uniform ? nullptr : net->val_d.p + pl.ell_off;
+    a.len = pl.ragged ? net->len_d.p + (size_t)l * net->N : nullptr;
+    a.w0 = pl.w0;
+    if (pl.kind == 1 && !force_ell) {
+        a.nu = pl.nu;
+        a.wtab = pl.uniform ? nullptr : net->wtab_d.p + pl.w_off;
+    }
+    return a;
+}
+
+static bool use_circ(const snicit_network* net, int l, int kernel_opt) {
+    if (kernel_opt == SNICIT_KERNEL_ELL) return false;
+    return net->plan[l].kind == 1;
+}
+
+static cudaError_t run_layer(snicit_network* net, int l, int kernel_opt, int mode, LayerArgs a, int max_rows) {
+    if (use_circ(net, l, kernel_opt)) return launch_layer_circ(a, mode, max_rows, net->num_sms, net->stream);
+    return launch_layer_ell(a, mode, max_rows, net->num_sms, net->stream);
+}
+
+static cudaError_t ensure_workspace(snicit_network* net, int64_t R, int s, int n) {
+    const size_t rows = (size_t)std::max<int64_t>(R, 1);
+    const size_t rn = rows * (size_t)net->N;
+    cudaError_t e;
+    if ((e = net->Ya.ensure(rn)) != cudaSuccess) return e;
+    if ((e = net->Yb.ensure(rn)) != cudaSuccess) return e;
+    for (auto* b : {&net->list0, &net->list1, &net->res0, &net->res1, &net->M, &net->cslot, &net->catlist})
+        if ((e = b->ensure(rows)) != cudaSuccess) return e;
+    for (auto* b : {&net->flag_pos, &net->live_row, &net->ne_row, &net->cat, &net->ne_t})
+        if ((e = b->ensure(rows)) != cudaSuccess) return e;
+    const size_t ss = (size_t)std::max(s, 1);
+    for (auto* b : {&net->cbuf0, &net->cbuf1, &net->ac})
+        if ((e = b->ensure(ss * net->N)) != cudaSuccess) return e;
+    if ((e = net->cent.ensure(ss)) != cudaSuccess) return e;
+    if ((e = net->col_idx.ensure(ss)) != cudaSuccess) return e;
+    if ((e = net->iota_s.ensure(ss)) != cudaSuccess) return e;
+    if ((e = net->F.ensure((size_t)std::max(n, 1) * ss)) != cudaSuccess) return e;
+    return cudaSuccess;
+}
+
+static cudaError_t read_counter(snicit_network* net, int which, int* outv) {
+    cudaError_t e = cudaMemcpyAsync(net->h_counters + which, net->counters.p + which, sizeof(int),
+                                    cudaMemcpyDeviceToHost, net->stream);
+    if (e != cudaSuccess) return e;
+    e = cudaStreamSynchronize(net->stream);
+    if (e != cudaSuccess) return e;
+    *outv = net->h_counters[which];
+    return cudaSuccess;
+}
+
+extern "C" {
+
+snicit_status snicit_infer(snicit_network* net, const float* y0, int64_t batch, int32_t y0_on_device,
+                           int64_t row_offset, int32_t t, int32_t s, const snicit_options* opt_in, float* y_out,
+                           int32_t y_out_on_device) {
+    if (!net) return fail(SNICIT_E_INVALID_ARG, "net NULL");
+    if (batch < 0 || batch > 0x7fffffffLL) return fail(SNICIT_E_INVALID_ARG, "batch out of range");
+    if (batch > 0 && !y0) return fail(SNICIT_E_INVALID_ARG, "y0 NULL");
+    if (t < 0) return fail(SNICIT_E_INVALID_ARG, "threshold_layer < 0");
+    if (s < 1) return fail(SNICIT_E_INVALID_ARG, "centroid_count < 1");
+    if (row_offset < 0) return fail(SNICIT_E_INVALID_ARG, "row_offset < 0");
+    snicit_options opt;
+    if (opt_in)
+        opt = *opt_in;
+    else
+        snicit_default_options(&opt);
+    if (opt.n_segments < 0 || opt.n_segments > net->N) return fail(SNICIT_E_INVALID_ARG, "n_segments out of range");
+    if (!(opt.eps >= 0.0f) || std::isnan(opt.eta) || !(opt.prune_eps >= 0.0f))
+        return fail(SNICIT_E_INVALID_ARG, "bad eta/eps/prune_eps");
+    if (opt.kernel < 0 || opt.kernel > 2) return fail(SNICIT_E_INVALID_ARG, "bad kernel option");
+    const int N = net->N, L = net->L;
+    if (opt.kernel == SNICIT_KERNEL_CIRC)
+        for (int l = 0; l < L; ++l)
+            if (net->plan[l].kind != 1)
+                return fail(SNICIT_E_UNSUPPORTED, "layer " + std::to_string(l) + " is not circulant");
+    const int R = (int)batch;
+    const int tt = std::min(t, L);
+    const int n_seg = opt.n_segments == 0 ? N : opt.n_segments;
+    const int ne_interval = opt.ne_interval > 0 ? opt.ne_interval : 64;
+    CUDA_TRY(cudaSetDevice(net->device));
+    CUDA_TRY(ensure_workspace(net, R, s, n_seg));
+    cudaStream_t st = net->stream;
+    int64_t launches = 0;
+    int circ_layers = 0;
+    net->have_result = false;
+    snicit_stats_t stats{};
+    stats.batch = batch;
+    stats.threshold_layer = tt;
+
+    if (opt.timing) CUDA_TRY(cudaEventRecord(net->ev[0], st));
+    // ---- input
+    const float* cur;
+    float* bufs[2] = {net->Ya.p, net->Yb.p};
+    int nxt_i = 0;
+    if (y0_on_device) {
+        cur = y0;
+    } else {
+        CUDA_TRY(cudaMemcpyAsync(net->Ya.p, y0, sizeof(float) * (size_t)R * N, cudaMemcpyHostToDevice, st));
+        cur = net->Ya.p;
+        nxt_i = 1;
+    }
+    int* cnt = net->counters.p;
+    int* list_cur = net->list0.p;
+    int* list_nxt = net->list1.p;
+    int* cnt_cur = cnt + CNT_LIVE0;
+    int* cnt_nxt = cnt + CNT_LIVE1;
+    CUDA_TRY(launch_iota(list_cur, R, cnt_cur, st));
+    ++launches;
+    const bool drop = opt.drop_dead_rows != 0;
+    // zero input rows are dead only when the conversion happens at t = 0 (otherwise layer 0 drops them)
+    if (drop && net->dead_ok[0] && tt == 0 && R > 0) {
+        CUDA_TRY(launch_row_nonzero(cur, N, list_cur, cnt_cur, net->flag_pos.p, R, net->num_sms, st));
+        CUDA_TRY(launch_compact(list_cur, cnt_cur, net->flag_pos.p, list_nxt, cnt_nxt, R, st));
+        launches += 2;
+        std::swap(list_cur, list_nxt);
+        std::swap(cnt_cur, cnt_nxt);
+    }
+    // ---- a1: pre-convergence layers, Eq. 1 for i = 0..t-1
+    const bool prof = opt.timing >= 2;
+    if (prof) {
+        while ((int)net->lev.size() < 2 * tt) {
+            cudaEvent_t e;
+            CUDA_TRY(cudaEventCreate(&e));
+            net->lev.push_back(e);
+        }
+        CUDA_TRY(net->hist.ensure(std::max(tt, 1)));
+        net->prof_layers = tt;
+    } else {
+        net->prof_layers = 0;
+    }
+    for (int l = 0; l < tt; ++l) {
+        const bool drop_now = drop && net->dead_ok[l + 1];
+        if (prof) {
+            CUDA_TRY(cudaMemcpyAsync(net->hist.p + l, cnt_cur, sizeof(int), cudaMemcpyDeviceToDevice, st));
+            CUDA_TRY(cudaEventRecord(net->lev[2 * l], st));
+        }
+        LayerArgs a = layer_args(net, l, opt.kernel == SNICIT_KERNEL_ELL);
+        a.yin = cur;
+        a.yout = bufs[nxt_i];
+        a.rows = list_cur;
+        a.count = cnt_cur;
+        a.flag_pos = drop_now ? net->flag_pos.p : nullptr;
+        CUDA_TRY(run_layer(net, l, opt.kernel, MODE_PLAIN, a, R));
+        if (prof) CUDA_TRY(cudaEventRecord(net->lev[2 * l + 1], st));
+        ++launches;
+        circ_layers += use_circ(net, l, opt.kernel);
+        net->last_kernel_circ = use_circ(net, l, opt.kernel);
+        cur = bufs[nxt_i];
+        nxt_i ^= 1;
+        if (drop_now) {
+            CUDA_TRY(launch_compact(list_cur, cnt_cur, net->flag_pos.p, list_nxt, cnt_nxt, R, st));
+            ++launches;
+            std::swap(list_cur, list_nxt);
+            std::swap(cnt_cur, cnt_nxt);
+        }
+    }
+    if (opt.timing) CUDA_TRY(cudaEventRecord(net->ev[1], st));
+    // live flags at t (for recovery of the plain path and the debug hook)
+    CUDA_TRY(launch_fill_u8(net->live_row.p, R, 0, st));
+    CUDA_TRY(launch_mark_rows(list_cur, cnt_cur, net->live_row.p, R, st));
+    launches += 2;
+
+    float* y_dst = y_out_on_device ? y_out : nullptr;
+    const float* yfinal = cur;
+    const float* cfinal = net->cbuf0.p;
+    const bool converted = tt < L;
+    net->last_converted = converted;
+    if (!converted) {
+        if (opt.timing) {
+            CUDA_TRY(cudaEventRecord(net->ev[2], st));
+            CUDA_TRY(cudaEventRecord(net->ev[3], st));
+        }
+        if (!y_out_on_device && y_out) y_dst = bufs[nxt_i];
+        CUDA_TRY(launch_recover(N, R, 1, yfinal, net->live_row.p, nullptr, nullptr, nullptr, nullptr, y_dst,
+                                net->cat.p, net->num_sms, st));
+        ++launches;
+    } else {
+        // ---- a2/a3: sampling + sum downsampling + Alg. 1 pruning -> y*
+        CUDA_TRY(launch_downsample(cur, N, list_cur, cnt_cur, s, n_seg, net->F.p, st));
+        CUDA_TRY(launch_prune(net->F.p, cnt_cur, s, n_seg, opt.eta, opt.eps, list_cur, net->cent.p, cnt + CNT_NCENT,
+                              cnt + CNT_SEFF, net->col_idx.p, st));
+        // ---- a4: mapper + residues (Alg. 2); dead rows keep M = -2
+        CUDA_TRY(launch_fill_i32(net->M.p, R, -2, st));
+        CUDA_TRY(launch_fill_u8(net->ne_row.p, R, 0, st));
+        float* yhat = bufs[nxt_i];
+        float* yhat_other = bufs[nxt_i ^ 1];
+        CUDA_TRY(launch_map_residual(cur, N, list_cur, cnt_cur, net->cent.p, cnt + CNT_NCENT, net->M.p, net->cslot.p,
+                                     net->ne_row.p, net->flag_pos.p, yhat, net->cbuf0.p, R, net->num_sms, st));
+        int* rlist = net->res0.p;
+        int* rlist_nxt = net->res1.p;
+        int* rcnt = cnt + CNT_RES0;
+        int* rcnt_nxt = cnt + CNT_RES1;
+        CUDA_TRY(launch_compact(list_cur, cnt_cur, net->flag_pos.p, rlist, rcnt, R, st));
+        CUDA_TRY(launch_iota(net->iota_s.p, s, nullptr, st));
+        CUDA_TRY(cudaMemcpyAsync(net->ne_t.p, net->ne_row.p, (size_t)R, cudaMemcpyDeviceToDevice, st));
+        launches += 7;
+        if (opt.timing) CUDA_TRY(cudaEventRecord(net->ev[2], st));
+        // ---- a5: post-convergence layers, Eq. 5 for i = t..L-1
+        float* c_cur = net->cbuf0.p;
+        float* c_nxt = net->cbuf1.p;
+        int res_host = 1;
+        CUDA_TRY(read_counter(net, CNT_RES0, &res_host));
+        stats.residual_at_t = res_host;
+        float* yh_cur = yhat;
+        float* yh_nxt = yhat_other;
+        for (int l = tt; l < L; ++l) {
+            // centroids: Eq. 5 first case, keep a_c
+            LayerArgs a = layer_args(net, l, opt.kernel == SNICIT_KERNEL_ELL);
+            a.yin = c_cur;
+            a.yout = c_nxt;
+            a.rows = net->iota_s.p;
+            a.count = cnt + CNT_NCENT;
+            a.a_out = net->ac.p;
+            CUDA_TRY(run_layer(net, l, opt.kernel, MODE_CENTROID, a, s));
+            ++launches;
+            circ_layers += use_circ(net, l, opt.kernel);
+            if (res_host > 0) {
+                // residues: Eq. 5 second case, only non-empty rows (ne_idx)
+                LayerArgs b = layer_args(net, l, opt.kernel == SNICIT_KERNEL_ELL);
+                b.yin = yh_cur;
+                b.yout = yh_nxt;
+                b.rows = rlist;
+                b.count = rcnt;
+                b.a_c = net->ac.p;
+                b.cslot = net->cslot.p;
+                b.flag_pos = net->flag_pos.p;
+                b.flag_row = net->ne_row.p;
+                b.prune_eps = opt.prune_eps;
+                CUDA_TRY(run_layer(net, l, opt.kernel, MODE_RESIDUAL, b, R));
+                CUDA_TRY(launch_compact(rlist, rcnt, net->flag_pos.p, rlist_nxt, rcnt_nxt, R, st));
+                launches += 2;
+                std::swap(rlist, rlist_nxt);
+                std::swap(rcnt, rcnt_nxt);
+                std::swap(yh_cur, yh_nxt);
+                if (((l - tt + 1) % ne_interval) == 0) {
+                    const int which = (rcnt == cnt + CNT_RES0) ? CNT_RES0 : CNT_RES1;
+                    CUDA_TRY(read_counter(net, which, &res_host));
+                }
+            }
+            std::swap(c_cur, c_nxt);
+        }
+        if (opt.timing) CUDA_TRY(cudaEventRecord(net->ev[3], st));
+        {
+            int rf = 0;
+            const int which = (rcnt == cnt + CNT_RES0) ? CNT_RES0 : CNT_RES1;
+            if (res_host > 0) CUDA_TRY(read_counter(net, which, &rf));
+            stats.residual_final = res_host > 0 ? rf : 0;
+        }
+        yfinal = yh_cur;
+        cfinal = c_cur;
+        // ---- a6: recovery (Eq. 6)
+        if (!y_out_on_device && y_out) y_dst = yh_nxt;  // free buffer
+        CUDA_TRY(launch_recover(N, R, 0, yfinal, nullptr, net->M.p, net->cslot.p, net->ne_row.p, cfinal, y_dst,
+                                net->cat.p, net->num_sms, st));
+        ++launches;
+    }
+    // categories: ordered compaction of cat flags over all rows
+    CUDA_TRY(launch_iota(net->list1.p == list_cur ? net->list0.p : net->list1.p, R, cnt + CNT_ALL, st));
+    CUDA_TRY(launch_compact(net->list1.p == list_cur ? net->list0.p : net->list1.p, cnt + CNT_ALL, net->cat.p,
+                            net->catlist.p, cnt + CNT_NCAT, R, st));
+    launches += 2;
+    if (opt.timing) CUDA_TRY(cudaEventRecord(net->ev[4], st));
+    if (!y_out_on_device && y_out && R > 0)
+        CUDA_TRY(cudaMemcpyAsync(y_out, y_dst, sizeof(float) * (size_t)R * N, cudaMemcpyDeviceToHost, st));
+    if (opt.timing) CUDA_TRY(cudaEventRecord(net->ev[5], st));
+    net->have_result = true;
+    net->last_batch = batch;
+    net->last_offset = row_offset;
+    net->last_t = tt;
+    net->last_s = s;
+    net->last_n = n_seg;
+    stats.kernel_launches = launches;
+    stats.circ_layers = circ_layers;
+    net->stats = stats;
+    if (!opt.timing) {
+        net->stats.t_pre_ms = net->stats.t_convert_ms = net->stats.t_post_ms = net->stats.t_recover_ms = -1.0;
+        net->stats.t_total_ms = -1.0;
+    }
+    net->live_counter = (cnt_cur == cnt + CNT_LIVE0) ? CNT_LIVE0 : CNT_LIVE1;
+    if (opt.timing) {
+        CUDA_TRY(cudaEventSynchronize(net->ev[5]));
+        float ms;
+        cudaEventElapsedTime(&ms, net->ev[0], net->ev[1]);
+        net->stats.t_pre_ms = ms;
+        cudaEventElapsedTime(&ms, net->ev[1], net->ev[2]);
+        net->stats.t_convert_ms = ms;
+        cudaEventElapsedTime(&ms, net->ev[2], net->ev[3]);
+        net->stats.t_post_ms = ms;
+        cudaEventElapsedTime(&ms, net->ev[3], net->ev[4]);
+        net->stats.t_recover_ms = ms;
+        cudaEventElapsedTime(&ms, net->ev[0], net->ev[5]);
+        net->stats.t_total_ms = ms;
+    }
+    return SNICIT_OK;
+}
+
+snicit_status snicit_categories(snicit_network* net, int64_t* rows, int64_t* count, int32_t rows_on_device) {
+    if (!net || !count) return fail(SNICIT_E_INVALID_ARG, "net/count NULL");
+    if (!net->have_result) return fail(SNICIT_E_STATE, "no inference result");
+    CUDA_TRY(cudaSetDevice(net->device));
+    int total = 0;
+    CUDA_TRY(read_counter(net, CNT_NCAT, &total));
+    if (!rows) {
+        *count = total;
+        return SNICIT_OK;
+    }
+    const int64_t n = std::min<int64_t>(*count, total);
+    if (n > 0) {
+        std::vector<int32_t> tmp((size_t)n);
+        CUDA_TRY(cudaMemcpyAsync(tmp.data(), net->catlist.p, sizeof(int32_t) * n, cudaMemcpyDeviceToHost, net->stream));
+        CUDA_TRY(cudaStreamSynchronize(net->stream));
+        std::vector<int64_t> out((size_t)n);
+        for (int64_t i = 0; i < n; ++i) out[i] = net->last_offset + tmp[i];
+        if (rows_on_device)
+            CUDA_TRY(cudaMemcpy(rows, out.data(), sizeof(int64_t) * n, cudaMemcpyHostToDevice));
+        else
+            memcpy(rows, out.data(), sizeof(int64_t) * n);
+    }
+    *count = n;
+    return SNICIT_OK;
+}
+
+snicit_status snicit_stats(snicit_network* net, snicit_stats_t* out) {
+    if (!net || !out) return fail(SNICIT_E_INVALID_ARG, "net/out NULL");
+    if (!net->have_result) return fail(SNICIT_E_STATE, "no inference result");
+    CUDA_TRY(cudaSetDevice(net->device));
+    int v = 0;
+    CUDA_TRY(read_counter(net, net->live_counter, &v));
+    net->stats.live_at_t = v;
+    CUDA_TRY(read_counter(net, CNT_NCAT, &v));
+    net->stats.n_categories = v;
+    if (net->last_converted) {
+        CUDA_TRY(read_counter(net, CNT_NCENT, &v));
+        net->stats.n_centroids = v;
+        CUDA_TRY(read_counter(net, CNT_SEFF, &v));
+        net->stats.n_sampled = v;
+    }
+    *out = net->stats;
+    return SNICIT_OK;
+}
+
+snicit_status snicit_layer_profile(snicit_network* net, int32_t max, double* ms, int64_t* rows, double* bytes,
+                                   int32_t* n) {
+    if (!net) return fail(SNICIT_E_INVALID_ARG, "net NULL");
+    if (!net->have_result) return fail(SNICIT_E_STATE, "no inference result");
+    CUDA_TRY(cudaSetDevice(net->device));
+    CUDA_TRY(cudaStreamSynchronize(net->stream));
+    const int cnt = std::min<int>(std::max(max, 0), net->prof_layers);
+    std::vector<int> h((size_t)std::max(cnt, 1));
+    if (cnt > 0) CUDA_TRY(cudaMemcpy(h.data(), net->hist.p, sizeof(int) * cnt, cudaMemcpyDeviceToHost));
+    for (int l = 0; l < cnt; ++l) {
+        float t = 0.f;
+        CUDA_TRY(cudaEventElapsedTime(&t, net->lev[2 * l], net->lev[2 * l + 1]));
+        if (ms) ms[l] = t;
+        if (rows) rows[l] = h[l];
+        if (bytes) {
+            const LayerPlan& pl = net->plan[l];
+            // algorithmic bytes: rows read + written, weights, bias
+            double wb;
+            if (pl.kind == 1 && net->last_kernel_circ)
+                wb = 4.0 * pl.K;
+            else
+                wb = (double)pl.K * net->N * ((net->idx16 ? 2.0 : 4.0) + (pl.uniform ? 0.0 : 4.0));
+            bytes[l] = 8.0 * (double)h[l] * net->N + wb + 4.0 * net->N;
+        }
+    }
+    if (n) *n = cnt;
+    return SNICIT_OK;
+}
+
+snicit_status snicit_debug_clustering(snicit_network* net, int32_t* cent, int32_t* n_cent, int32_t* M, uint8_t* ne_t,
+                                      double* F, int32_t* n_sampled, uint8_t* live_t) {
+    if (!net) return fail(SNICIT_E_INVALID_ARG, "net NULL");
+    if (!net->have_result) return fail(SNICIT_E_STATE, "no inference result");
+    CUDA_TRY(cudaSetDevice(net->device));
+    CUDA_TRY(cudaStreamSynchronize(net->stream));
+    const int R = (int)net->last_batch;
+    int C = 0, se = 0;
+    if (net->last_converted) {
+        CUDA_TRY(cudaMemcpy(&C, net->counters.p + CNT_NCENT, sizeof(int), cudaMemcpyDeviceToHost));
+        CUDA_TRY(cudaMemcpy(&se, net->counters.p + CNT_SEFF, sizeof(int), cudaMemcpyDeviceToHost));
+    }
+    if (n_cent) *n_cent = C;
+    if (n_sampled) *n_sampled = se;
+    if (cent && C > 0) CUDA_TRY(cudaMemcpy(cent, net->cent.p, sizeof(int) * C, cudaMemcpyDeviceToHost));
+    if (M && R > 0 && net->last_converted) CUDA_TRY(cudaMemcpy(M, net->M.p, sizeof(int) * R, cudaMemcpyDeviceToHost));
+    if (ne_t && R > 0 && net->last_converted) CUDA_TRY(cudaMemcpy(ne_t, net->ne_t.p, R, cudaMemcpyDeviceToHost));
+    if (live_t && R > 0) CUDA_TRY(cudaMemcpy(live_t, net->live_row.p, R, cudaMemcpyDeviceToHost));
+    if (F && se > 0) {
+        std::vector<double> tmp((size_t)net->last_n * net->last_s);
+        CUDA_TRY(cudaMemcpy(tmp.data(), net->F.p, sizeof(double) * tmp.size(), cudaMemcpyDeviceToHost));
+        for (int g = 0; g < net->last_n; ++g)
+            for (int q = 0; q < se; ++q) F[(size_t)g * se + q] = tmp[(size_t)g * net->last_s + q];
+    }
+    return SNICIT_OK;
+}
+
+snicit_status snicit_debug_layer(snicit_network* net, int32_t layer, const float* yin, float* yout, int64_t rows,
+                                 int32_t kernel) {
+    if (!net || !yin || !yout) return fail(SNICIT_E_INVALID_ARG, "NULL argument");
+    if (layer < 0 || layer >= net->L) return fail(SNICIT_E_INVALID_ARG, "bad layer");
+    if (rows < 0 || rows > 0x7fffffffLL) return fail(SNICIT_E_INVALID_ARG, "bad rows");
+    if (kernel == SNICIT_KERNEL_CIRC && net->plan[layer].kind != 1)
+        return fail(SNICIT_E_UNSUPPORTED, "layer is not circulant");
+    CUDA_TRY(cudaSetDevice(net->device));
+    CUDA_TRY(ensure_workspace(net, rows, 1, 1));
+    CUDA_TRY(launch_iota(net->list0.p, (int)rows, net->counters.p + CNT_LIVE0, net->stream));
+    LayerArgs a = layer_args(net, layer, kernel == SNICIT_KERNEL_ELL);
+    a.yin = yin;
+    a.yout = yout;
+    a.rows = net->list0.p;
+    a.count = net->counters.p + CNT_LIVE0;
+    CUDA_TRY(run_layer(net, layer, kernel, MODE_PLAIN, a, (int)rows));
+    CUDA_TRY(cudaStreamSynchronize(net->stream));
+    return SNICIT_OK;
+}
+
+}  // extern "C"

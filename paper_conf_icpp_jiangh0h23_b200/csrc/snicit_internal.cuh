@@ -1,0 +1,132 @@
+// snicit_internal.cuh -- internal declarations of libsnicit.so (sm_100a).
+// Kernel/launcher interfaces shared by the .cu files of the library; not part of the ABI.
+#pragma once
+#include <cuda_runtime.h>
+#include <stdint.h>
+
+#include <string>
+#include <vector>
+
+namespace snicit {
+
+// ------------------------------------------------------------------ PTX helpers (TMA bulk, mbarrier)
+__device__ __forceinline__ uint32_t smem_u32(const void* p) {
+    return static_cast<uint32_t>(__cvta_generic_to_shared(p));
+}
+__device__ __forceinline__ void mbar_init(uint64_t* bar, uint32_t count) {
+    asm volatile("mbarrier.init.shared::cta.b64 [%0], %1;" ::"r"(smem_u32(bar)), "r"(count) : "memory");
+}
+__device__ __forceinline__ void fence_proxy_async_smem() {
+    asm volatile("fence.proxy.async.shared::cta;" ::: "memory");
+}
+__device__ __forceinline__ void mbar_arrive_expect_tx(uint64_t* bar, uint32_t bytes) {
+    asm volatile("mbarrier.arrive.expect_tx.shared::cta.b64 _, [%0], %1;" ::"r"(smem_u32(bar)), "r"(bytes)
+                 : "memory");
+}
+__device__ __forceinline__ bool mbar_try_wait(uint64_t* bar, uint32_t parity) {
+    uint32_t ok;
+    asm volatile(
+        "{\n\t.reg .pred p;\n\t"
+        "mbarrier.try_wait.parity.shared::cta.b64 p, [%1], %2;\n\t"
+        "selp.u32 %0, 1, 0, p;\n\t}"
+        : "=r"(ok)
+        : "r"(smem_u32(bar)), "r"(parity)
+        : "memory");
+    return ok != 0;
+}
+__device__ __forceinline__ void mbar_wait(uint64_t* bar, uint32_t parity) {
+    while (!mbar_try_wait(bar, parity)) {
+    }
+}
+// 1-D bulk copy global -> shared (TMA engine, UBLKCP), completion counted on `bar`.
+__device__ __forceinline__ void bulk_g2s(void* sdst, const void* gsrc, uint32_t bytes, uint64_t* bar) {
+    asm volatile(
+        "cp.async.bulk.shared::cluster.global.mbarrier::complete_tx::bytes [%0], [%1], %2, [%3];" ::"r"(
+            smem_u32(sdst)),
+        "l"(gsrc), "r"(bytes), "r"(smem_u32(bar))
+        : "memory");
+}
+// 1-D bulk copy shared -> global (TMA store), bulk-group completion.
+__device__ __forceinline__ void bulk_s2g(void* gdst, const void* ssrc, uint32_t bytes) {
+    asm volatile("cp.async.bulk.global.shared::cta.bulk_group [%0], [%1], %2;" ::"l"(gdst), "r"(smem_u32(ssrc)),
+                 "r"(bytes)
+                 : "memory");
+}
+__device__ __forceinline__ void bulk_commit() { asm volatile("cp.async.bulk.commit_group;" ::: "memory"); }
+__device__ __forceinline__ void bulk_wait_read0() { asm volatile("cp.async.bulk.wait_group.read 0;" ::: "memory"); }
+__device__ __forceinline__ void bulk_wait0() { asm volatile("cp.async.bulk.wait_group 0;" ::: "memory"); }
+
+// sigma(x) = min(max(x, 0), ymax): Table 2
+__device__ __forceinline__ float sigma(float x, float ymax) { return fminf(fmaxf(x, 0.0f), ymax); }
+
+// ------------------------------------------------------------------ layer kernels
+enum LayerMode : int {
+    MODE_PLAIN = 0,     // Eq. 1: y' = sigma(acc + b)
+    MODE_CENTROID = 1,  // Eq. 5 first case, also stores a_c = acc (pre-activation, no bias)
+    MODE_RESIDUAL = 2   // Eq. 5 second case: sigma((a_c + acc) + b) - sigma(a_c + b)
+};
+
+struct LayerArgs {
+    int N;
+    const float* yin;       // rows of N fp32 (indexed by row id)
+    float* yout;
+    const int* rows;        // active row ids (list)
+    const int* count;       // device: number of active rows
+    const float* bias;      // [N] of this layer
+    float ymax;
+    uint8_t* flag_pos;      // nullable: any-non-zero of the row, indexed by list position
+    uint8_t* flag_row;      // nullable: same, indexed by row id
+    float* a_out;           // CENTROID: a_c [row][N]
+    const float* a_c;       // RESIDUAL: a_c [slot][N]
+    const int* cslot;       // RESIDUAL: centroid slot of each row id
+    float prune_eps;        // RESIDUAL: |v| <= prune_eps -> 0
+    // ELL weights (n-major: entry n of column j at n*N + j)
+    int K;                  // max entries per column
+    const uint16_t* idx16;  // used when N <= 65536
+    const int32_t* idx32;
+    const float* val;       // nullable when uniform
+    const uint8_t* len;     // nullable: per-column length (ragged); NULL = all K
+    float w0;               // uniform value
+    // circulant: column j reads (j + n*nu) mod N, n = 0..K-1, weight w[n] (or w0)
+    int nu;
+    const float* wtab;      // K per-n weights (device), nullable when uniform
+};
+
+struct LayerPlan {
+    int kind;       // 0 = ELL, 1 = CIRC
+    int K;
+    int nu;         // CIRC
+    bool uniform;   // all values equal (w0)
+    bool ragged;    // column lengths differ
+    float w0;
+    size_t ell_off; // element offset of this layer in the ELL arrays
+    size_t w_off;   // offset in the per-n weight table
+};
+
+// launchers (kernels_layer.cu); return cudaError_t of the launch
+cudaError_t launch_layer_ell(const LayerArgs& a, int mode, int max_rows, int num_sms, cudaStream_t st);
+cudaError_t launch_layer_circ(const LayerArgs& a, int mode, int max_rows, int num_sms, cudaStream_t st);
+bool circ_supported(int N, int K, int nu);
+bool ell_smem_ok(int N);
+
+// kernels_convert.cu
+cudaError_t launch_iota(int* out, int n, int* count_out, cudaStream_t st);
+cudaError_t launch_fill_i32(int* out, int n, int v, cudaStream_t st);
+cudaError_t launch_fill_u8(uint8_t* out, int n, uint8_t v, cudaStream_t st);
+cudaError_t launch_row_nonzero(const float* y, int N, const int* rows, const int* count, uint8_t* flag_pos,
+                               int max_rows, int num_sms, cudaStream_t st);
+cudaError_t launch_compact(const int* list_in, const int* count_in, const uint8_t* flag_pos, int* list_out,
+                           int* count_out, int max_n, cudaStream_t st);
+cudaError_t launch_downsample(const float* y, int N, const int* rows, const int* count, int s, int n_seg,
+                              double* F, cudaStream_t st);
+cudaError_t launch_prune(const double* F, const int* count, int s, int n_seg, float eta, float eps,
+                         const int* rows, int* cent, int* n_cent, int* s_eff, int* col_idx, cudaStream_t st);
+cudaError_t launch_map_residual(const float* y, int N, const int* rows, const int* count, const int* cent,
+                                const int* n_cent, int* M, int* cslot, uint8_t* ne_row, uint8_t* flag_pos,
+                                float* yhat, float* cbuf, int max_rows, int num_sms, cudaStream_t st);
+cudaError_t launch_recover(int N, int R, int plain, const float* yfinal, const uint8_t* live_row, const int* M,
+                           const int* cslot, const uint8_t* ne_row, const float* cbuf, float* y_out,
+                           uint8_t* cat, int num_sms, cudaStream_t st);
+cudaError_t launch_mark_rows(const int* rows, const int* count, uint8_t* flag_row, int max_rows, cudaStream_t st);
+
+}  // namespace snicit

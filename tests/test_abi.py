@@ -1,0 +1,98 @@
+"""The C-ABI library (no GPU needed): it loads, exports every symbol include/snicit.h declares, and
+its host-side argument validation reports bad input with the documented status codes."""
+import ctypes
+import os
+import re
+
+import numpy as np
+import pytest
+
+import paper_conf_icpp_jiangh0h23_b200 as pkg
+from paper_conf_icpp_jiangh0h23_b200 import _lib
+from paper_conf_icpp_jiangh0h23_b200 import build as pkg_build
+
+ROOT = os.path.dirname(os.path.dirname(os.path.abspath(__file__)))
+
+
+@pytest.fixture(scope="module")
+def lib():
+    pkg_build.build()
+    return _lib.load_library()
+
+
+def header_functions():
+    src = open(os.path.join(ROOT, "include", "snicit.h")).read()
+    src = re.sub(r"/\*.*?\*/", "", src, flags=re.S)
+    return sorted(set(re.findall(r"\b(snicit_[a-z_]+)\s*\(", src)))
+
+
+def test_header_symbols_exported(lib):
+    names = header_functions()
+    assert "snicit_infer" in names and "snicit_load_network" in names and "snicit_categories" in names
+    for n in names:
+        assert hasattr(lib, n), f"{n} declared in include/snicit.h but not exported"
+    assert sorted(_lib.EXPORTED) == names
+
+
+def test_abi_version_and_defaults(lib):
+    assert lib.snicit_abi_version() == 1
+    o = _lib.default_options()
+    # SDGC defaults, P:1038 / P:1138
+    assert o.n_segments == 16 and abs(o.eta - 0.03) < 1e-7 and abs(o.eps - 0.03) < 1e-7
+    assert o.prune_eps == 0.0 and o.drop_dead_rows == 1 and o.kernel == 0 and o.ne_interval == 64
+
+
+def _load(lib, N, L, ptr, idx, val, bias, ymax=32.0, fmt=0):
+    h = ctypes.c_void_p()
+    ptr = np.ascontiguousarray(ptr, np.int64)
+    idx = np.ascontiguousarray(idx, np.int32)
+    val = np.ascontiguousarray(val, np.float32)
+    bias = np.ascontiguousarray(bias, np.float32)
+    st = lib.snicit_load_network(N, L, fmt, ptr.ctypes.data, idx.ctypes.data, val.ctypes.data, bias.ctypes.data,
+                                 ymax, 0, ctypes.byref(h))
+    if st == 0:
+        lib.snicit_free_network(h)
+    return st
+
+
+def test_validation_codes(lib):
+    N = 8
+    ptr = np.arange(N + 1) * 2
+    idx = np.array([(j + d) % N for j in range(N) for d in (0, 1)])
+    val = np.full(2 * N, 0.5)
+    bias = np.zeros(N)
+    bad = idx.copy()
+    bad[3] = N  # out of range
+    assert _load(lib, N, 1, ptr, bad, val, bias) == -2
+    dup = idx.copy()
+    dup[1] = dup[0]  # duplicate input in column 0
+    assert _load(lib, N, 1, ptr, dup, val, bias) == -2
+    nonmono = ptr.copy()
+    nonmono[2], nonmono[3] = nonmono[3], nonmono[2]
+    assert _load(lib, N, 1, nonmono, idx, val, bias) == -2
+    nan = val.copy()
+    nan[0] = np.nan
+    assert _load(lib, N, 1, ptr, idx, nan, bias) == -1
+    assert _load(lib, N, 1, ptr, idx, val, bias, ymax=-1.0) == -1
+    assert _load(lib, 6, 1, np.arange(7) * 0, idx[:0], val[:0], np.zeros(6)) == -6  # N % 4 != 0
+    # a valid network: without a GPU the library reports E_CUDA (never a CPU fallback)
+    st = _load(lib, N, 1, ptr, idx, val, bias)
+    try:
+        import torch
+        has_gpu = torch.cuda.is_available()
+    except Exception:
+        has_gpu = False
+    assert st == (0 if has_gpu else -4)
+    assert lib.snicit_last_error() is not None
+
+
+def test_null_handle_errors(lib):
+    n = ctypes.c_int64(0)
+    assert lib.snicit_categories(None, None, ctypes.byref(n), 0) == -1
+    assert lib.snicit_infer(None, None, 0, 0, 0, 0, 1, None, None, 0) == -1
+    lib.snicit_free_network(None)  # no-op
+
+
+def test_package_exports():
+    assert callable(pkg.SnicitNetwork) and callable(pkg.shard_rows)
+    assert pkg.shard_rows(10, 3, 0) == (0, 4) and pkg.shard_rows(10, 3, 2) == (7, 10)

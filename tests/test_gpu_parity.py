@@ -1,0 +1,226 @@
+"""GPU parity: the CUDA path (through the C ABI) against the CPU oracle on identical seeded inputs.
+
+Bars (north_star / DESIGN.md): category set bit-exact; fp32 activations within 1e-4 abs or 1e-5 rel
+of the plain oracle; the uncompressed path and every step that follows the oracle's evaluation
+order are bit-exact (compared with ==, so +0 == -0, reading R19).
+"""
+import numpy as np
+import pytest
+
+torch = pytest.importorskip("torch")
+
+import oracle  # noqa: E402
+from paper_conf_icpp_jiangh0h23_b200 import KERNEL_CIRC, KERNEL_ELL, SnicitNetwork  # noqa: E402
+from workload import sdgc  # noqa: E402
+from workload.sdgc import Network  # noqa: E402
+
+pytestmark = pytest.mark.gpu
+
+ATOL, RTOL = 1e-4, 1e-5
+
+
+@pytest.fixture(scope="module", autouse=True)
+def _need_gpu():
+    if not torch.cuda.is_available():
+        pytest.skip("no CUDA device")
+    from paper_conf_icpp_jiangh0h23_b200 import build
+    build.build()
+
+
+def run_gpu(net, Y0, t, s=32, device_io=True, **opt):
+    with SnicitNetwork.from_network(net) as g:
+        g.set_stream(torch.cuda.current_stream())
+        if device_io:
+            y0 = torch.from_numpy(np.ascontiguousarray(Y0)).cuda()
+            out = torch.empty_like(y0)
+            g.infer(y0, t=t, s=s, y_out=out, **opt)
+            cats = g.categories()
+            Y = out.cpu().numpy()
+        else:
+            out = np.empty_like(Y0)
+            g.infer(np.ascontiguousarray(Y0), t=t, s=s, y_out=out, **opt)
+            cats = g.categories()
+            Y = out
+        st = g.stats()
+        clus = g.debug_clustering(n_segments=opt.get("n_segments", 16), s=s) if t < net.L else None
+    return Y, cats, st, clus
+
+
+def ragged_net(N, L, seed, ymax=32.0):
+    rs = np.random.RandomState(seed)
+    ptr, idx, val = [], [], []
+    off = 0
+    for l in range(L):
+        p = [off]
+        for j in range(N):
+            kk = rs.choice(N, size=rs.randint(0, 40), replace=False)
+            idx.extend(kk.tolist())
+            val.extend(rs.uniform(-0.2, 0.4, size=len(kk)).tolist())
+            off += len(kk)
+            p.append(off)
+        ptr.extend(p)
+    bias = rs.uniform(-0.3, 0.2, size=L * N)
+    return Network(N=N, L=L, ptr=np.array(ptr, np.int64), idx=np.array(idx, np.int32), val=np.array(val, np.float32),
+                   bias=bias.astype(np.float32), ymax=ymax, mode="ragged")
+
+
+# ------------------------------------------------------------------------------ single layer, bit-exact
+
+@pytest.mark.parametrize("N,mode,rows", [(1024, "radix", 333), (4096, "radix", 97), (16384, "radix", 9),
+                                         (1024, "perm", 130), (4096, "random", 41)])
+def test_layer_kernels_bit_exact(N, mode, rows):
+    net = sdgc.gen_network(N, 4, mode)
+    Y0 = sdgc.gen_inputs(N, rows) * np.float32(7.5)  # non-binary values exercise rounding
+    Y0[::5] = np.random.RandomState(0).uniform(0, 32, size=Y0[::5].shape).astype(np.float32)
+    with SnicitNetwork.from_network(net) as g:
+        yin = torch.from_numpy(Y0).cuda()
+        for l in range(net.L):
+            ref = oracle.layers_f32(net, Y0, l, l + 1)
+            kernels = [KERNEL_ELL] + ([KERNEL_CIRC] if g.layer_is_circulant(l) else [])
+            assert g.layer_is_circulant(l) == (mode == "radix")
+            for k in kernels:
+                out = torch.full_like(yin, float("nan"))
+                g.debug_layer(l, yin, out, kernel=k)
+                assert np.array_equal(out.cpu().numpy(), ref), f"layer {l} kernel {k}"
+
+
+def test_layer_ell_ragged_and_values():
+    net = ragged_net(64, 3, 1, ymax=4.0)
+    Y0 = np.random.RandomState(2).uniform(0, 3, size=(50, 64)).astype(np.float32)
+    with SnicitNetwork.from_network(net) as g:
+        yin = torch.from_numpy(Y0).cuda()
+        for l in range(3):
+            out = torch.empty_like(yin)
+            g.debug_layer(l, yin, out)
+            assert np.array_equal(out.cpu().numpy(), oracle.layers_f32(net, Y0, l, l + 1))
+
+
+# ------------------------------------------------------------------------------ whole path
+
+@pytest.mark.parametrize("mode", ["radix", "perm"])
+def test_uncompressed_path_bit_exact_c1(mode):
+    net = sdgc.gen_network(1024, 120, mode)
+    Y0 = sdgc.gen_inputs(1024, 2000)
+    ref = oracle.layers_f32(net, Y0)
+    Y, cats, st, _ = run_gpu(net, Y0, t=net.L)
+    assert np.array_equal(Y, ref)
+    assert np.array_equal(cats, oracle.categories(ref))
+    assert st["n_categories"] == len(cats)
+
+
+@pytest.mark.parametrize("t", [0, 2, 5, 10, 30])
+def test_snicit_c1_vs_oracle(t):
+    """C1 (SDGC 1024 x 120, B = 2000): the GPU SNICIT path equals the oracle's SNICIT pipeline
+    bit-exactly (same clustering, same evaluation order) and the plain result within tolerance."""
+    net = sdgc.gen_network(1024, 120, "radix")
+    Y0 = sdgc.gen_inputs(1024, 2000)
+    plain = oracle.layers_f32(net, Y0)
+    ref = oracle.snicit(net, Y0, t=t, s=32, n=16)
+    Y, cats, st, clus = run_gpu(net, Y0, t=t)
+    assert np.array_equal(cats, oracle.categories(plain))
+    assert np.array_equal(cats, ref["categories"])
+    np.testing.assert_allclose(Y, plain, atol=ATOL, rtol=RTOL)
+    assert np.array_equal(Y, ref["Y"])
+    # step-level: sampled F, centroids, mapper, ne at t, live rows at t
+    assert np.array_equal(clus["live_t"], ref["live_t"])
+    assert np.array_equal(clus["F"], ref["F"])
+    assert np.array_equal(clus["cent"], ref["cent"])
+    assert np.array_equal(clus["M"], ref["M"])
+    assert st["n_centroids"] == len(ref["cent"]) >= 1
+    assert Y.min() >= 0 and Y.max() <= 32
+
+
+def test_snicit_ell_forced_equals_auto():
+    net = sdgc.gen_network(1024, 40, "radix")
+    Y0 = sdgc.gen_inputs(1024, 700)
+    a = run_gpu(net, Y0, t=4)
+    b = run_gpu(net, Y0, t=4, kernel=KERNEL_ELL)
+    assert np.array_equal(a[0], b[0]) and np.array_equal(a[1], b[1])
+    assert a[2]["circ_layers"] == 40 and b[2]["circ_layers"] == 0
+
+
+def test_snicit_perm_4096_small_t():
+    net = sdgc.gen_network(4096, 24, "perm")
+    Y0 = sdgc.gen_inputs(4096, 300)
+    plain = oracle.layers_f32(net, Y0)
+    ref = oracle.snicit(net, Y0, t=3)
+    Y, cats, st, clus = run_gpu(net, Y0, t=3)
+    assert np.array_equal(cats, oracle.categories(plain))
+    assert np.array_equal(Y, ref["Y"])
+    np.testing.assert_allclose(Y, plain, atol=ATOL, rtol=RTOL)
+    assert st["residual_at_t"] > 0  # residual kernels exercised
+
+
+def test_medium_net_config5():
+    """Config 5 stand-in: YMAX 1, per-neuron values and biases (some > 0: no dead-row drop), no
+    downsampling (n = N), s = 128."""
+    net = sdgc.gen_medium_network(256, 18)
+    Y0 = sdgc.gen_medium_inputs(256, 3000)
+    plain = oracle.layers_f32(net, Y0)
+    t = sdgc.medium_t(18)
+    ref = oracle.snicit(net, Y0, t=t, s=128, n=0)
+    Y, cats, st, clus = run_gpu(net, Y0, t=t, s=128, n_segments=0)
+    assert np.array_equal(cats, oracle.categories(plain))
+    np.testing.assert_allclose(Y, plain, atol=ATOL, rtol=RTOL)
+    assert np.array_equal(Y, ref["Y"])
+    assert np.array_equal(clus["cent"], ref["cent"])
+
+
+def test_host_buffers_path():
+    net = sdgc.gen_network(1024, 30, "radix")
+    Y0 = sdgc.gen_inputs(1024, 333)
+    ref = oracle.snicit(net, Y0, t=7)
+    Y, cats, _, _ = run_gpu(net, Y0, t=7, device_io=False)
+    assert np.array_equal(Y, ref["Y"]) and np.array_equal(cats, ref["categories"])
+
+
+@pytest.mark.parametrize("B", [0, 1, 5, 33])
+def test_edge_batches(B):
+    net = sdgc.gen_network(1024, 16, "radix")
+    Y0 = sdgc.gen_inputs(1024, max(B, 1))[:B]
+    ref = oracle.snicit(net, Y0, t=3) if B else None
+    Y, cats, st, _ = run_gpu(net, Y0, t=3)
+    if B:
+        assert np.array_equal(Y, ref["Y"]) and np.array_equal(cats, ref["categories"])
+    else:
+        assert len(cats) == 0
+
+
+def test_s_one_and_no_dead_drop():
+    net = sdgc.gen_network(1024, 20, "radix")
+    Y0 = sdgc.gen_inputs(1024, 400)
+    plain = oracle.layers_f32(net, Y0)
+    for kw in (dict(s=1), dict(s=32, drop_dead_rows=0), dict(s=64, n_segments=0)):
+        s = kw.pop("s")
+        Y, cats, _, _ = run_gpu(net, Y0, t=5, s=s, **kw)
+        assert np.array_equal(cats, oracle.categories(plain))
+        np.testing.assert_allclose(Y, plain, atol=ATOL, rtol=RTOL)
+
+
+def test_near_zero_pruning_runs():
+    """prune_eps > 0 is the paper's approximate relaxation: outside exact parity; the
+    outputs must stay in range and close to the exact result for a tiny eps."""
+    net = sdgc.gen_network(1024, 30, "radix")
+    Y0 = sdgc.gen_inputs(1024, 500)
+    Y, cats, _, _ = run_gpu(net, Y0, t=4, prune_eps=1e-6)
+    assert Y.min() >= -1e-6 and Y.max() <= 32
+
+
+def test_full_size_c2_sampled_rows():
+    """C2 at full size (SDGC 4096 x 480, B = 60000, t = 30) in bench.py's configuration: sampled rows
+    against the plain oracle row by row, and category membership of the sampled rows."""
+    net = sdgc.gen_network(4096, 480, "radix")
+    B = 60000
+    Y0 = sdgc.gen_inputs(4096, B)
+    Y, cats, st, _ = run_gpu(net, Y0, t=30)
+    rs = np.random.RandomState(0)
+    sample = np.unique(np.concatenate([rs.choice(B, 40, replace=False), [0, 1, B - 1]]))
+    ref = oracle.layers_f32(net, Y0[sample])
+    np.testing.assert_allclose(Y[sample], ref, atol=ATOL, rtol=RTOL)
+    catset = set(cats.tolist())
+    for i, r in enumerate(sample):
+        assert (r in catset) == bool((ref[i] != 0).any())
+    # properties at any size: ranges, categories = non-zero rows of the returned activations
+    assert Y.min() >= 0 and Y.max() <= 32
+    assert np.array_equal(cats, np.nonzero((Y != 0).any(1))[0])
+    assert st["n_categories"] == len(cats)
