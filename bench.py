@@ -161,6 +161,23 @@ def measured_peaks():
     return 6650.0, "fallback (B200_PROFILING.md: 6.65 TB/s)"
 
 
+def oracle_sample_time(oracle, net, Y, cores, seconds, probe_only=False):
+    """Rows of Y the oracle processes in ~`seconds` on all host cores (calibrated on `cores` rows run
+    with all threads), and the measured time for that many rows."""
+    k = max(1, min(len(Y), cores))
+    t0 = time.perf_counter()
+    oracle.layers_f32(net, Y[:k])
+    t_probe = max(time.perf_counter() - t0, 1e-6)
+    rows = int(max(k, min(len(Y), k * seconds / t_probe)))
+    if probe_only:
+        return rows, None
+    if rows == k:
+        return k, t_probe
+    t0 = time.perf_counter()
+    oracle.layers_f32(net, Y[:rows])
+    return rows, time.perf_counter() - t0
+
+
 # ------------------------------------------------------------------ reference arm (CPU oracle)
 def run_reference(args):
     rank = int(os.environ.get("RANK", "0"))
@@ -172,16 +189,12 @@ def run_reference(args):
     net = make_network(args, c)
     nnz = net.nnz
     cores = os.cpu_count() or 1
-    # size the per-step sample to ~cpu_seconds of the oracle on all cores (1 calibration row)
-    probe = make_inputs(args, c, 1, 0)
-    t0 = time.perf_counter()
-    oracle.layers_f32(net, probe, nthreads=1)
-    per_row = max(time.perf_counter() - t0, 1e-6)
-    rows = int(max(cores, min(c["B"], args.cpu_seconds * cores / per_row / max(args.steps, 1))))
-    rows = max(1, min(rows, c["B"]))
+    # size the per-step sample to ~cpu_seconds / steps of the oracle on all cores
+    probe = make_inputs(args, c, cores, 0)
+    rows, _ = oracle_sample_time(oracle, net, probe, cores, args.cpu_seconds / max(args.steps, 1), probe_only=True)
     Y = make_inputs(args, c, rows, 0)
-    for _ in range(max(args.warmup, 0) if rows * per_row / cores < 2 else 1):
-        oracle.layers_f32(net, Y[: max(1, rows // 8)])
+    if args.warmup > 0:
+        oracle.layers_f32(net, Y[: max(1, min(rows, cores))])
     times = []
     for _ in range(args.steps):
         t0 = time.perf_counter()
@@ -351,13 +364,7 @@ def run_snicit(args):
     if rank == 0 and world == 1 and not args.no_cpu_baseline:
         import oracle
         cores = os.cpu_count() or 1
-        t0 = time.perf_counter()
-        oracle.layers_f32(net, Yh[:1], nthreads=1)
-        per_row = max(time.perf_counter() - t0, 1e-6)
-        rows = int(max(cores, min(B_local, args.cpu_seconds * cores / per_row)))
-        t0 = time.perf_counter()
-        oracle.layers_f32(net, Yh[:rows])
-        T = time.perf_counter() - t0
+        rows, T = oracle_sample_time(oracle, net, Yh, cores, args.cpu_seconds)
         cpu = {"value": rows * nnz / T, "unit": UNIT, "cores": cores, "kind": "oracle",
                "sample": f"{rows} of {B_local} rows, plain Eq. 1 oracle over all {net.L} layers ({T:.1f} s)",
                "cpu": cpu_info()}

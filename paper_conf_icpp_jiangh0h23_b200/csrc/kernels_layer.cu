@@ -22,9 +22,43 @@
 //    global memory (L1/L2).
 #include <cuda_runtime.h>
 
+#include <map>
+#include <mutex>
+#include <utility>
+
 #include "snicit_internal.cuh"
 
 namespace snicit {
+
+// Blocks per SM of a kernel at a given dynamic shared-memory size, cached per (device, kernel, smem)
+// so a launch costs no host-side attribute/occupancy queries after the first (the post-convergence
+// loop launches ~2 kernels per layer for up to 1890 layers).
+cudaError_t blocks_per_sm(const void* kern, int threads, size_t smem, int* out) {
+    static std::mutex mu;
+    static std::map<std::pair<std::pair<int, const void*>, size_t>, int> cache;
+    int dev = 0;
+    cudaError_t e = cudaGetDevice(&dev);
+    if (e != cudaSuccess) return e;
+    const auto key = std::make_pair(std::make_pair(dev, kern), smem);
+    {
+        std::lock_guard<std::mutex> g(mu);
+        auto it = cache.find(key);
+        if (it != cache.end()) {
+            *out = it->second;
+            return cudaSuccess;
+        }
+    }
+    e = cudaFuncSetAttribute(kern, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)smem);
+    if (e != cudaSuccess) return e;
+    int per_sm = 1;
+    e = cudaOccupancyMaxActiveBlocksPerMultiprocessor(&per_sm, kern, threads, smem);
+    if (e != cudaSuccess) return e;
+    if (per_sm < 1) per_sm = 1;
+    std::lock_guard<std::mutex> g(mu);
+    cache[key] = per_sm;
+    *out = per_sm;
+    return cudaSuccess;
+}
 
 constexpr int kCircThreads = 256;
 constexpr int kEllThreads = 512;
@@ -159,12 +193,9 @@ static cudaError_t launch_circ_t(const LayerArgs& a, int max_rows, int num_sms, 
     while (RT > 1 && (size_t)RT * a.N * 8 > 96 * 1024) --RT;
     const size_t smem = (size_t)RT * a.N * 8 + 16 + 12 * (size_t)RT + 16;
     auto kern = layer_circ_kernel<MODE, M, UNIF>;
-    cudaError_t e = cudaFuncSetAttribute(kern, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)smem);
-    if (e != cudaSuccess) return e;
     int per_sm = 1;
-    e = cudaOccupancyMaxActiveBlocksPerMultiprocessor(&per_sm, kern, kCircThreads, smem);
+    cudaError_t e = blocks_per_sm((const void*)kern, kCircThreads, smem, &per_sm);
     if (e != cudaSuccess) return e;
-    if (per_sm < 1) per_sm = 1;
     const int tiles = (max_rows + RT - 1) / RT;
     int grid = num_sms * per_sm;
     if (grid > tiles) grid = tiles;
@@ -290,12 +321,9 @@ static cudaError_t launch_ell_t(const LayerArgs& a, int max_rows, int num_sms, c
     SNICIT_PICK(false, true, true)
     SNICIT_PICK(false, false, true)
 #undef SNICIT_PICK
-    cudaError_t e = cudaFuncSetAttribute(kern, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)smem);
-    if (e != cudaSuccess) return e;
     int per_sm = 1;
-    e = cudaOccupancyMaxActiveBlocksPerMultiprocessor(&per_sm, kern, kEllThreads, smem);
+    cudaError_t e = blocks_per_sm((const void*)kern, kEllThreads, smem, &per_sm);
     if (e != cudaSuccess) return e;
-    if (per_sm < 1) per_sm = 1;
     const int tiles = (max_rows + RT - 1) / RT;
     int grid = num_sms * per_sm;
     if (grid > tiles) grid = tiles;
