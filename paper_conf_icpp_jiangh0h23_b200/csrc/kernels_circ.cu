@@ -1,0 +1,317 @@
+// kernels_circ.cu -- the fused layer kernel for shift-invariant (circulant) layers, sm_100a.
+//
+// A layer is circulant when output column j reads inputs (j + n*nu) mod N, n = 0..K-1 (K = 32),
+// with per-n weights -- the RadiX-Net-like SDGC layers "sums of cyclic permutations".
+// Writing j = a*nu + c (Q = N/nu), output (a, c) reads (a + n mod Q, c): every residue class c is
+// an independent circular sliding window of length K over Q values.  A thread loads a window of
+// WIN inputs of one class into registers and produces M outputs from it, so each staged input
+// element is read from shared memory WIN/M times instead of K times, and the FMA chain of every
+// output is evaluated exactly in the stored order n = 0..K-1 (R12: acc = fmaf(y, w_n, acc)).
+//
+// Stride classes (template CLS):
+//   NU1  nu == 1: lanes walk chunk starts 17 apart (odd -> conflict-free LDS); the staged row gets a
+//        64-float circular halo (a second TMA copy of the row head) so windows never wrap.
+//   Q32  Q == 32: one thread owns a whole residue class (32 loads, 32 outputs, all rotations at
+//        compile time); lanes walk consecutive residues.
+//   GEN  other nu: M = 16 outputs per thread, lanes walk consecutive residues; windows that wrap
+//        (warp-uniform) take a masked path.
+//
+// Pipeline per CTA (persistent over row tiles): TMA bulk loads of tile i+1 are in flight while tile
+// i is computed; outputs are staged in shared memory and stored with TMA bulk stores (coalesced for
+// every nu), double-buffered when shared memory allows.  Epilogues: see LayerMode.
+#include <cuda_runtime.h>
+
+#include "snicit_internal.cuh"
+
+namespace snicit {
+
+constexpr int kCircThreads = 256;
+constexpr int kK = 32;      // taps per column (SDGC: 32 connections per neuron)
+constexpr int kHalo = 64;   // floats appended to each staged row for NU1 (>= M + K - 2 = 47)
+
+enum CircClass : int { CLS_NU1 = 0, CLS_Q32 = 1, CLS_GEN = 2 };
+template <int CLS>
+struct CircCfg;
+template <>
+struct CircCfg<CLS_NU1> {
+    static constexpr int M = 17, WIN = M + kK - 1;
+};
+template <>
+struct CircCfg<CLS_Q32> {
+    static constexpr int M = 32, WIN = 32;
+};
+template <>
+struct CircCfg<CLS_GEN> {
+    static constexpr int M = 16, WIN = M + kK - 1;
+};
+
+__host__ __device__ constexpr int circ_stride(int N, int cls) { return N + (cls == CLS_NU1 ? kHalo : 0); }
+__host__ __device__ constexpr size_t circ_smem(int N, int cls, int RT, int nbuf_out) {
+    return sizeof(float) * ((size_t)2 * RT * circ_stride(N, cls) + (size_t)nbuf_out * RT * N) + 2 * sizeof(uint64_t) +
+           3 * 2 * sizeof(int) * (size_t)RT;
+}
+
+template <int MODE, int CLS, bool UNIF, bool UBIAS, int NUCT>
+__global__ void __launch_bounds__(kCircThreads, MODE == MODE_PLAIN ? 3 : 2) layer_circ_kernel(LayerArgs a, int RT, int nbuf_out) {
+    constexpr int M = CircCfg<CLS>::M;
+    constexpr int WIN = CircCfg<CLS>::WIN;
+    extern __shared__ __align__(128) unsigned char smem[];
+    const int N = a.N;
+    const int nu = NUCT ? NUCT : a.nu;
+    const int Q = N / nu;
+    const int stride = circ_stride(N, CLS);
+    float* s_in = reinterpret_cast<float*>(smem);
+    float* s_out = s_in + (size_t)2 * RT * stride;
+    uint64_t* bars = reinterpret_cast<uint64_t*>(s_out + (size_t)nbuf_out * RT * N);
+    int* s_row = reinterpret_cast<int*>(bars + 2);
+    int* s_slot = s_row + 2 * RT;
+    int* s_flag = s_slot + 2 * RT;
+
+    const int chunks = (CLS == CLS_Q32) ? 1 : (Q + M - 1) / M;
+    const int ipr = nu * chunks;  // work items per row
+    const int count = *a.count;
+    const int ntiles = (count + RT - 1) / RT;
+    if ((int)blockIdx.x >= ntiles) return;
+
+    float w[UNIF ? 1 : kK];
+    if constexpr (!UNIF) {
+#pragma unroll
+        for (int n = 0; n < kK; ++n) w[n] = __ldg(a.wtab + n);
+    }
+    const float w0 = a.w0;
+    const float b0 = UBIAS ? __ldg(a.bias) : 0.0f;
+
+    if (threadIdx.x == 0) {
+        mbar_init(&bars[0], 1);
+        mbar_init(&bars[1], 1);
+        fence_proxy_async_smem();
+    }
+    __syncthreads();
+
+    // thread 0: stage the rows of `tile` into input buffer b (TMA bulk copies, one mbarrier)
+    auto issue = [&](int tile, int b) {
+        const int r0 = tile * RT;
+        const int nr = min(RT, count - r0);
+        const uint32_t bytes = (uint32_t)nr * (uint32_t)(N * 4 + (CLS == CLS_NU1 ? kHalo * 4 : 0));
+        mbar_arrive_expect_tx(&bars[b], bytes);
+        for (int i = 0; i < nr; ++i) {
+            const int row = a.rows[r0 + i];
+            s_row[b * RT + i] = row;
+            if constexpr (MODE == MODE_RESIDUAL) s_slot[b * RT + i] = a.cslot[row];
+            const float* g = a.yin + (size_t)row * N;
+            float* d = s_in + (size_t)(b * RT + i) * stride;
+            bulk_g2s(d, g, N * 4, &bars[b]);
+            if constexpr (CLS == CLS_NU1) bulk_g2s(d + N, g, kHalo * 4, &bars[b]);  // circular halo
+        }
+    };
+    if (threadIdx.x == 0) issue(blockIdx.x, 0);
+
+    int it = 0;
+    for (int tile = blockIdx.x; tile < ntiles; tile += gridDim.x, ++it) {
+        const int b = it & 1;
+        const int ob = (nbuf_out == 2) ? b : 0;
+        if (threadIdx.x == 0) {
+            const int next = tile + gridDim.x;
+            if (next < ntiles) issue(next, b ^ 1);  // overlaps this tile's compute
+            if (nbuf_out == 2)
+                bulk_wait_read1();  // the store that last used s_out[ob] has read it
+            else
+                bulk_wait_read0();
+        }
+        if ((int)threadIdx.x < RT) s_flag[b * RT + threadIdx.x] = 0;
+        mbar_wait(&bars[b], (uint32_t)((it >> 1) & 1));
+        __syncthreads();
+
+        const int r0 = tile * RT;
+        const int nr = min(RT, count - r0);
+        const float* in_b = s_in + (size_t)b * RT * stride;
+        float* out_b = s_out + (size_t)ob * RT * N;
+        for (int item = threadIdx.x; item < nr * ipr; item += blockDim.x) {
+            const int rr = item / ipr;
+            const int rem = item - rr * ipr;
+            const int row = s_row[b * RT + rr];
+            const int slot = (MODE == MODE_RESIDUAL) ? s_slot[b * RT + rr] : 0;
+            float mx = 0.0f;
+            if constexpr (CLS == CLS_NU1) {
+                const int a0 = rem * M;
+                const float* src = in_b + (size_t)rr * stride + a0;
+                float R[WIN];
+#pragma unroll
+                for (int i = 0; i < WIN; ++i) R[i] = src[i];
+                float* dst = out_b + (size_t)rr * N + a0;
+                if (a0 + M <= N) {  // all but the last chunk of a row: no guards, chains interleave
+#pragma unroll
+                    for (int m = 0; m < M; ++m) {
+                        float acc = 0.0f;
+#pragma unroll
+                        for (int n = 0; n < kK; ++n) acc = fmaf(R[m + n], UNIF ? w0 : w[n], acc);
+                        const float bq = UBIAS ? b0 : __ldg(a.bias + a0 + m);
+                        const float v = epilogue<MODE>(a, acc, bq, a0 + m, row, slot);
+                        dst[m] = v;
+                        mx = fmaxf(mx, fabsf(v));
+                    }
+                } else {
+#pragma unroll
+                    for (int m = 0; m < M; ++m) {
+                        if (a0 + m < N) {
+                            float acc = 0.0f;
+#pragma unroll
+                            for (int n = 0; n < kK; ++n) acc = fmaf(R[m + n], UNIF ? w0 : w[n], acc);
+                            const float bq = UBIAS ? b0 : __ldg(a.bias + a0 + m);
+                            const float v = epilogue<MODE>(a, acc, bq, a0 + m, row, slot);
+                            dst[m] = v;
+                            mx = fmaxf(mx, fabsf(v));
+                        }
+                    }
+                }
+            } else if constexpr (CLS == CLS_Q32) {
+                const int c = rem;
+                const float* src = in_b + (size_t)rr * stride + c;
+                float R[32];
+#pragma unroll
+                for (int j = 0; j < 32; ++j) R[j] = src[j * nu];
+                float* dst = out_b + (size_t)rr * N + c;
+#pragma unroll
+                for (int m = 0; m < 32; ++m) {
+                    float acc = 0.0f;
+#pragma unroll
+                    for (int n = 0; n < kK; ++n) acc = fmaf(R[(m + n) & 31], UNIF ? w0 : w[n], acc);
+                    const int q = m * nu + c;
+                    const float bq = UBIAS ? b0 : __ldg(a.bias + q);
+                    const float v = epilogue<MODE>(a, acc, bq, q, row, slot);
+                    dst[m * nu] = v;
+                    mx = fmaxf(mx, fabsf(v));
+                }
+            } else {  // CLS_GEN
+                const int c = rem % nu;
+                const int a0 = (rem / nu) * M;
+                const float* src = in_b + (size_t)rr * stride + c;
+                float R[WIN];
+                if (a0 + WIN <= Q) {  // warp-uniform: lanes share a0
+#pragma unroll
+                    for (int i = 0; i < WIN; ++i) R[i] = src[(a0 + i) * nu];
+                } else {
+#pragma unroll
+                    for (int i = 0; i < WIN; ++i) {
+                        int ai = a0 + i;  // < 3Q since Q >= K and M < K
+                        ai = ai >= Q ? ai - Q : ai;
+                        ai = ai >= Q ? ai - Q : ai;
+                        R[i] = src[ai * nu];
+                    }
+                }
+                float* dst = out_b + (size_t)rr * N + c + (size_t)a0 * nu;
+                const int mlim = min(M, Q - a0);  // == M unless Q % M != 0
+#pragma unroll
+                for (int m = 0; m < M; ++m) {
+                    if (m < mlim) {
+                        float acc = 0.0f;
+#pragma unroll
+                        for (int n = 0; n < kK; ++n) acc = fmaf(R[m + n], UNIF ? w0 : w[n], acc);
+                        const int q = (a0 + m) * nu + c;
+                        const float bq = UBIAS ? b0 : __ldg(a.bias + q);
+                        const float v = epilogue<MODE>(a, acc, bq, q, row, slot);
+                        dst[m * nu] = v;
+                        mx = fmaxf(mx, fabsf(v));
+                    }
+                }
+            }
+            if (mx != 0.0f) s_flag[b * RT + rr] = 1;
+        }
+        fence_proxy_async_smem();  // this thread's s_out writes -> visible to the TMA engine
+        __syncthreads();
+        if (threadIdx.x == 0) {
+            for (int i = 0; i < nr; ++i) {
+                const int row = s_row[b * RT + i];
+                bulk_s2g(a.yout + (size_t)row * N, out_b + (size_t)i * N, N * 4);
+                const uint8_t f = s_flag[b * RT + i] ? 1 : 0;
+                if (a.flag_pos) a.flag_pos[r0 + i] = f;
+                if (a.flag_row) a.flag_row[row] = f;
+            }
+            bulk_commit();
+        }
+    }
+    if (threadIdx.x == 0) bulk_wait0();
+}
+
+static int circ_class(int N, int nu) {
+    if (nu == 1) return CLS_NU1;
+    if (N / nu == 32) return CLS_Q32;
+    return CLS_GEN;
+}
+
+bool circ_supported(int N, int K, int nu) {
+    if (K != kK || nu <= 0 || N % nu != 0 || N % 4 != 0) return false;
+    if ((long long)K * nu > N) return false;  // distinct inputs -> Q >= K
+    const int cls = circ_class(N, nu);
+    if (cls == CLS_NU1 && N < kHalo) return false;
+    return circ_smem(N, cls, 1, 1) <= 220 * 1024;
+}
+
+struct CircPlan {
+    int RT, nbuf_out;
+    size_t smem;
+};
+
+static CircPlan circ_plan(int N, int nu) {
+    const int cls = circ_class(N, nu);
+    const int Q = N / nu;
+    const int M = cls == CLS_NU1 ? CircCfg<CLS_NU1>::M : (cls == CLS_Q32 ? 32 : CircCfg<CLS_GEN>::M);
+    const int ipr = nu * (cls == CLS_Q32 ? 1 : (Q + M - 1) / M);
+    int RT = kCircThreads / ipr;
+    if (RT < 1) RT = 1;
+    if (RT > 16) RT = 16;
+    while (RT > 1 && circ_smem(N, cls, RT, 2) > 116 * 1024) --RT;
+    CircPlan p{RT, 2, circ_smem(N, cls, RT, 2)};
+    if (p.smem > 220 * 1024) {
+        p.nbuf_out = 1;
+        p.smem = circ_smem(N, cls, RT, 1);
+    }
+    return p;
+}
+
+template <int MODE, int CLS, bool UNIF, bool UBIAS, int NUCT>
+static cudaError_t launch_circ_t(const LayerArgs& a, int max_rows, int num_sms, cudaStream_t st) {
+    const CircPlan p = circ_plan(a.N, a.nu);
+    auto kern = layer_circ_kernel<MODE, CLS, UNIF, UBIAS, NUCT>;
+    int per_sm = 1;
+    cudaError_t e = blocks_per_sm((const void*)kern, kCircThreads, p.smem, &per_sm);
+    if (e != cudaSuccess) return e;
+    const int tiles = (max_rows + p.RT - 1) / p.RT;
+    int grid = num_sms * per_sm;
+    if (grid > tiles) grid = tiles;
+    if (grid < 1) grid = 1;
+    kern<<<grid, kCircThreads, p.smem, st>>>(a, p.RT, p.nbuf_out);
+    return cudaGetLastError();
+}
+
+template <int MODE, int CLS, int NUCT>
+static cudaError_t launch_circ_wb(const LayerArgs& a, int max_rows, int num_sms, cudaStream_t st) {
+    const bool unif = a.wtab == nullptr;
+    const bool ub = a.uniform_bias != 0;
+    if (unif && ub) return launch_circ_t<MODE, CLS, true, true, NUCT>(a, max_rows, num_sms, st);
+    if (unif) return launch_circ_t<MODE, CLS, true, false, NUCT>(a, max_rows, num_sms, st);
+    if (ub) return launch_circ_t<MODE, CLS, false, true, NUCT>(a, max_rows, num_sms, st);
+    return launch_circ_t<MODE, CLS, false, false, NUCT>(a, max_rows, num_sms, st);
+}
+
+template <int MODE>
+static cudaError_t launch_circ_m(const LayerArgs& a, int max_rows, int num_sms, cudaStream_t st) {
+    switch (circ_class(a.N, a.nu)) {
+        case CLS_NU1: return launch_circ_wb<MODE, CLS_NU1, 0>(a, max_rows, num_sms, st);
+        case CLS_Q32: return launch_circ_wb<MODE, CLS_Q32, 0>(a, max_rows, num_sms, st);
+        default:
+            if (a.nu == 32) return launch_circ_wb<MODE, CLS_GEN, 32>(a, max_rows, num_sms, st);
+            return launch_circ_wb<MODE, CLS_GEN, 0>(a, max_rows, num_sms, st);
+    }
+}
+
+cudaError_t launch_layer_circ(const LayerArgs& a, int mode, int max_rows, int num_sms, cudaStream_t st) {
+    if (max_rows <= 0) return cudaSuccess;
+    switch (mode) {
+        case MODE_PLAIN: return launch_circ_m<MODE_PLAIN>(a, max_rows, num_sms, st);
+        case MODE_CENTROID: return launch_circ_m<MODE_CENTROID>(a, max_rows, num_sms, st);
+        default: return launch_circ_m<MODE_RESIDUAL>(a, max_rows, num_sms, st);
+    }
+}
+
+}  // namespace snicit

@@ -9,13 +9,7 @@
 //             Alg. 3 line 9); optional near-zero pruning
 // plus the per-row "any non-zero" flag consumed by row compaction (ne_rec, Alg. 3 lines 10-13).
 //
-// Two kernels:
-//  * layer_circ_kernel: layers whose column j reads (j + n*nu) mod N, n = 0..K-1, with per-n
-//    weights (shift-invariant RadiX-like layers).  Rows are staged in shared memory
-//    with TMA bulk copies; each thread keeps a register window of M + K - 1 inputs of one residue
-//    class and produces M outputs (sliding window), so shared-memory traffic is (M+K-1)/(M*K) of
-//    a plain gather and the kernel is bound by HBM / FMA issue instead of LDS bandwidth.  Outputs
-//    are staged in shared memory and written back with TMA bulk stores (coalesced for any nu).
+// This file: layer_ell_kernel (the circulant fast path is in kernels_circ.cu)
 //  * layer_ell_kernel: general CSC stored as n-major ELL (uint16 or int32 indices); a tile of RT
 //    rows in shared memory (TMA), one thread per output column, RT accumulators in registers so
 //    each index/value load is reused RT times.  N too large for shared memory: rows gathered from
@@ -60,169 +54,7 @@ cudaError_t blocks_per_sm(const void* kern, int threads, size_t smem, int* out) 
     return cudaSuccess;
 }
 
-constexpr int kCircThreads = 256;
 constexpr int kEllThreads = 512;
-constexpr int kCircK = 32;  // taps per column of the circulant fast path (SDGC: 32)
-
-template <int MODE>
-__device__ __forceinline__ float epilogue(const LayerArgs& a, float acc, int q, int row, int slot) {
-    const float b = __ldg(a.bias + q);
-    if constexpr (MODE == MODE_RESIDUAL) {
-        const float ac = __ldg(a.a_c + (size_t)slot * a.N + q);
-        float v = sigma((ac + acc) + b, a.ymax) - sigma(ac + b, a.ymax);
-        if (a.prune_eps > 0.0f && fabsf(v) <= a.prune_eps) v = 0.0f;
-        return v;
-    } else {
-        if constexpr (MODE == MODE_CENTROID) a.a_out[(size_t)row * a.N + q] = acc;
-        return sigma(acc + b, a.ymax);
-    }
-}
-
-// ------------------------------------------------------------------------------ circulant
-template <int MODE, int M, bool UNIF>
-__global__ void __launch_bounds__(kCircThreads, 2) layer_circ_kernel(LayerArgs a, int RT) {
-    constexpr int K = kCircK;
-    extern __shared__ __align__(128) unsigned char smem[];
-    const int N = a.N;
-    float* s_in = reinterpret_cast<float*>(smem);
-    float* s_out = s_in + (size_t)RT * N;
-    uint64_t* bar = reinterpret_cast<uint64_t*>(s_out + (size_t)RT * N);
-    int* s_flag = reinterpret_cast<int*>(bar + 1);
-    int* s_row = s_flag + RT;
-    int* s_slot = s_row + RT;
-
-    const int nu = a.nu;
-    const int Q = N / nu;
-    const int chunks = (Q + M - 1) / M;
-    const int ipr = nu * chunks;  // work items per row
-    const int count = *a.count;
-    const int ntiles = (count + RT - 1) / RT;
-
-    float w[UNIF ? 1 : K];
-    if constexpr (!UNIF) {
-#pragma unroll
-        for (int n = 0; n < K; ++n) w[n] = __ldg(a.wtab + n);
-    }
-    if (threadIdx.x == 0) {
-        mbar_init(bar, 1);
-        fence_proxy_async_smem();
-    }
-    __syncthreads();
-    uint32_t parity = 0;
-    for (int tile = blockIdx.x; tile < ntiles; tile += gridDim.x) {
-        const int r0 = tile * RT;
-        const int nr = min(RT, count - r0);
-        if (threadIdx.x < nr) {
-            const int row = a.rows[r0 + threadIdx.x];
-            s_row[threadIdx.x] = row;
-            s_flag[threadIdx.x] = 0;
-            if constexpr (MODE == MODE_RESIDUAL) s_slot[threadIdx.x] = a.cslot[row];
-        }
-        __syncthreads();
-        if (threadIdx.x == 0) {
-            mbar_arrive_expect_tx(bar, (uint32_t)(nr * N * 4));
-            for (int i = 0; i < nr; ++i) bulk_g2s(s_in + (size_t)i * N, a.yin + (size_t)s_row[i] * N, N * 4, bar);
-        }
-        mbar_wait(bar, parity);
-        parity ^= 1u;
-
-        for (int it = threadIdx.x; it < nr * ipr; it += blockDim.x) {
-            const int rr = it / ipr;
-            const int rem = it - rr * ipr;
-            const int c = rem % nu;
-            const int a0 = (rem / nu) * M;
-            const float* src = s_in + (size_t)rr * N + c;
-            float R[M + K - 1];
-#pragma unroll
-            for (int i = 0; i < M + K - 1; ++i) {
-                int ai = a0 + i;  // a0 + i < 3Q because Q >= K and M < K
-                ai -= (ai >= Q) ? Q : 0;
-                ai -= (ai >= Q) ? Q : 0;
-                R[i] = src[ai * nu];
-            }
-            const int row = s_row[rr];
-            const int slot = (MODE == MODE_RESIDUAL) ? s_slot[rr] : 0;
-            float* dst = s_out + (size_t)rr * N + c;
-            bool any = false;
-#pragma unroll
-            for (int m = 0; m < M; ++m) {
-                float acc = 0.0f;
-#pragma unroll
-                for (int n = 0; n < K; ++n) acc = fmaf(R[m + n], UNIF ? a.w0 : w[n], acc);
-                const int am = a0 + m;
-                if (am < Q) {
-                    const float v = epilogue<MODE>(a, acc, am * nu + c, row, slot);
-                    dst[am * nu] = v;
-                    any |= (v != 0.0f);
-                }
-            }
-            if (any) s_flag[rr] = 1;
-        }
-        fence_proxy_async_smem();  // make this thread's s_out writes visible to the TMA engine
-        __syncthreads();
-        if (threadIdx.x == 0) {
-            for (int i = 0; i < nr; ++i) bulk_s2g(a.yout + (size_t)s_row[i] * N, s_out + (size_t)i * N, N * 4);
-            bulk_commit();
-        }
-        if (threadIdx.x < nr) {
-            const uint8_t f = s_flag[threadIdx.x] ? 1 : 0;
-            if (a.flag_pos) a.flag_pos[r0 + threadIdx.x] = f;
-            if (a.flag_row) a.flag_row[s_row[threadIdx.x]] = f;
-        }
-        if (threadIdx.x == 0) bulk_wait_read0();  // s_out reusable
-        __syncthreads();
-    }
-    if (threadIdx.x == 0) bulk_wait0();
-}
-
-bool circ_supported(int N, int K, int nu) {
-    if (K != kCircK || nu <= 0 || N % nu != 0) return false;
-    if (!(nu == 1 || nu % 32 == 0)) return false;
-    if ((long long)K * nu > N) return false;
-    if ((size_t)N * 8 + 64 > 200 * 1024) return false;  // in + out row in shared memory
-    if (N % 4 != 0) return false;
-    return true;
-}
-
-template <int MODE, int M, bool UNIF>
-static cudaError_t launch_circ_t(const LayerArgs& a, int max_rows, int num_sms, cudaStream_t st) {
-    const int Q = a.N / a.nu;
-    const int ipr = a.nu * ((Q + M - 1) / M);
-    int RT = kCircThreads / ipr;
-    if (RT < 1) RT = 1;
-    while (RT > 1 && (size_t)RT * a.N * 8 > 96 * 1024) --RT;
-    const size_t smem = (size_t)RT * a.N * 8 + 16 + 12 * (size_t)RT + 16;
-    auto kern = layer_circ_kernel<MODE, M, UNIF>;
-    int per_sm = 1;
-    cudaError_t e = blocks_per_sm((const void*)kern, kCircThreads, smem, &per_sm);
-    if (e != cudaSuccess) return e;
-    const int tiles = (max_rows + RT - 1) / RT;
-    int grid = num_sms * per_sm;
-    if (grid > tiles) grid = tiles;
-    if (grid < 1) grid = 1;
-    kern<<<grid, kCircThreads, smem, st>>>(a, RT);
-    return cudaGetLastError();
-}
-
-template <int MODE>
-static cudaError_t launch_circ_m(const LayerArgs& a, int max_rows, int num_sms, cudaStream_t st) {
-    const bool unif = (a.wtab == nullptr);
-    // nu == 1: lanes walk chunk starts 17 apart (odd) -> conflict-free shared-memory windows;
-    // nu >= 32: lanes walk consecutive residues -> conflict-free with any M.
-    if (a.nu == 1) return unif ? launch_circ_t<MODE, 17, true>(a, max_rows, num_sms, st)
-                               : launch_circ_t<MODE, 17, false>(a, max_rows, num_sms, st);
-    return unif ? launch_circ_t<MODE, 16, true>(a, max_rows, num_sms, st)
-                : launch_circ_t<MODE, 16, false>(a, max_rows, num_sms, st);
-}
-
-cudaError_t launch_layer_circ(const LayerArgs& a, int mode, int max_rows, int num_sms, cudaStream_t st) {
-    if (max_rows <= 0) return cudaSuccess;
-    switch (mode) {
-        case MODE_PLAIN: return launch_circ_m<MODE_PLAIN>(a, max_rows, num_sms, st);
-        case MODE_CENTROID: return launch_circ_m<MODE_CENTROID>(a, max_rows, num_sms, st);
-        default: return launch_circ_m<MODE_RESIDUAL>(a, max_rows, num_sms, st);
-    }
-}
 
 // ------------------------------------------------------------------------------ ELL (general)
 template <int MODE, int RT, bool IDX16, bool UNIF, bool RAGGED, bool SMEM>
@@ -284,7 +116,7 @@ __global__ void __launch_bounds__(kEllThreads, 1) layer_ell_kernel(LayerArgs a) 
             for (int r = 0; r < RT; ++r) {
                 if (r < nr) {
                     const int row = s_row[r];
-                    const float v = epilogue<MODE>(a, acc[r], j, row, MODE == MODE_RESIDUAL ? s_slot[r] : 0);
+                    const float v = epilogue<MODE>(a, acc[r], __ldg(a.bias + j), j, row, MODE == MODE_RESIDUAL ? s_slot[r] : 0);
                     a.yout[(size_t)row * N + j] = v;
                     if (v != 0.0f) anyr |= 1 << r;
                 }

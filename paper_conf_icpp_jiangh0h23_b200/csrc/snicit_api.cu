@@ -295,6 +295,13 @@ snicit_status snicit_load_network(int32_t N, int32_t L, snicit_format fmt, const
             if (ragged) lay_len[l][j] = (uint8_t)cidx[j].size();
         }
     }
+    // uniform bias per layer
+    for (int l = 0; l < L; ++l) {
+        bool ub = true;
+        const float* b = bias + (int64_t)l * N;
+        for (int j = 1; j < N && ub; ++j) ub = b[j] == b[0] && std::signbit(b[j]) == std::signbit(b[0]);
+        net->plan[l].ubias = ub;
+    }
     // dead_ok
     net->dead_ok.assign(L + 1, 1);
     for (int l = L - 1; l >= 0; --l) {
@@ -397,6 +404,7 @@ static LayerArgs layer_args(snicit_network* net, int l, bool force_ell) {
     a.val = pl.uniform ? nullptr : net->val_d.p + pl.ell_off;
     a.len = pl.ragged ? net->len_d.p + (size_t)l * net->N : nullptr;
     a.w0 = pl.w0;
+    a.uniform_bias = pl.ubias ? 1 : 0;
     if (pl.kind == 1 && !force_ell) {
         a.nu = pl.nu;
         a.wtab = pl.uniform ? nullptr : net->wtab_d.p + pl.w_off;

@@ -54,6 +54,7 @@ __device__ __forceinline__ void bulk_s2g(void* gdst, const void* ssrc, uint32_t 
 }
 __device__ __forceinline__ void bulk_commit() { asm volatile("cp.async.bulk.commit_group;" ::: "memory"); }
 __device__ __forceinline__ void bulk_wait_read0() { asm volatile("cp.async.bulk.wait_group.read 0;" ::: "memory"); }
+__device__ __forceinline__ void bulk_wait_read1() { asm volatile("cp.async.bulk.wait_group.read 1;" ::: "memory"); }
 __device__ __forceinline__ void bulk_wait0() { asm volatile("cp.async.bulk.wait_group 0;" ::: "memory"); }
 
 // sigma(x) = min(max(x, 0), ymax): Table 2
@@ -87,6 +88,7 @@ struct LayerArgs {
     const float* val;       // nullable when uniform
     const uint8_t* len;     // nullable: per-column length (ragged); NULL = all K
     float w0;               // uniform value
+    int uniform_bias;       // 1: bias[j] == bias[0] for all j of this layer
     // circulant: column j reads (j + n*nu) mod N, n = 0..K-1, weight w[n] (or w0)
     int nu;
     const float* wtab;      // K per-n weights (device), nullable when uniform
@@ -98,12 +100,30 @@ struct LayerPlan {
     int nu;         // CIRC
     bool uniform;   // all values equal (w0)
     bool ragged;    // column lengths differ
+    bool ubias;     // bias[j] identical for all j (SDGC: a constant per benchmark, Table 1)
     float w0;
     size_t ell_off; // element offset of this layer in the ELL arrays
     size_t w_off;   // offset in the per-n weight table
 };
 
-// launchers (kernels_layer.cu); return cudaError_t of the launch
+// Epilogue of one output q of one row (acc = the fma chain, b = bias[q]).
+template <int MODE>
+__device__ __forceinline__ float epilogue(const LayerArgs& a, float acc, float b, int q, int row, int slot) {
+    if constexpr (MODE == MODE_RESIDUAL) {
+        const float ac = __ldg(a.a_c + (size_t)slot * a.N + q);
+        float v = sigma((ac + acc) + b, a.ymax) - sigma(ac + b, a.ymax);
+        if (a.prune_eps > 0.0f && fabsf(v) <= a.prune_eps) v = 0.0f;
+        return v;
+    } else {
+        if constexpr (MODE == MODE_CENTROID) a.a_out[(size_t)row * a.N + q] = acc;
+        return sigma(acc + b, a.ymax);
+    }
+}
+
+// cached blocks-per-SM (sets the dynamic shared-memory attribute on first use)
+cudaError_t blocks_per_sm(const void* kern, int threads, size_t smem, int* out);
+
+// launchers (kernels_circ.cu / kernels_layer.cu); return cudaError_t of the launch
 cudaError_t launch_layer_ell(const LayerArgs& a, int mode, int max_rows, int num_sms, cudaStream_t st);
 cudaError_t launch_layer_circ(const LayerArgs& a, int mode, int max_rows, int num_sms, cudaStream_t st);
 bool circ_supported(int N, int K, int nu);
