@@ -16,9 +16,10 @@
 //   GEN  other nu: M = 16 outputs per thread, lanes walk consecutive residues; windows that wrap
 //        (warp-uniform) take a masked path.
 //
-// Pipeline per CTA (persistent over row tiles): TMA bulk loads of tile i+1 are in flight while tile
-// i is computed; outputs are staged in shared memory and stored with TMA bulk stores (coalesced for
-// every nu), double-buffered when shared memory allows.  Epilogues: see LayerMode.
+// Pipeline per CTA (persistent over row tiles, warp-specialised): a producer warp stages tile i+1
+// with TMA bulk loads while 8 consumer warps compute tile i; outputs are staged in shared memory
+// (double-buffered) and written back by the producer with TMA bulk stores (coalesced for every nu).
+// Producer and consumers synchronise only through mbarriers.  Epilogues: see LayerMode.
 #include <cuda_runtime.h>
 
 #include "snicit_internal.cuh"
@@ -46,13 +47,24 @@ struct CircCfg<CLS_GEN> {
 };
 
 __host__ __device__ constexpr int circ_stride(int N, int cls) { return N + (cls == CLS_NU1 ? kHalo : 0); }
-__host__ __device__ constexpr size_t circ_smem(int N, int cls, int RT, int nbuf_out) {
-    return sizeof(float) * ((size_t)2 * RT * circ_stride(N, cls) + (size_t)nbuf_out * RT * N) + 2 * sizeof(uint64_t) +
+
+// Shared-memory layout (per CTA): in[2][RT][stride] | out[2][RT][N] | 8 mbarriers | row/slot/flag [2][RT]
+__host__ __device__ constexpr size_t circ_smem2(int N, int cls, int RT) {
+    return sizeof(float) * ((size_t)2 * RT * circ_stride(N, cls) + (size_t)2 * RT * N) + 8 * sizeof(uint64_t) +
            3 * 2 * sizeof(int) * (size_t)RT;
 }
 
+// Warp-specialised: warps 0..7 compute (kCircThreads consumer threads), warp 8 lane 0 is the
+// producer/storer.  mbarriers per buffer b in {0,1}:
+//   in_full[b]   producer arrive.expect_tx + TMA bytes    -> consumers may read in[b]
+//   in_empty[b]  one arrive per consumer warp              -> producer may reload in[b]
+//   out_full[b]  one arrive per consumer warp (after proxy fence) -> producer may TMA-store out[b]
+//   out_empty[b] producer arrive once the store has read out[b]  -> consumers may write out[b]
+// Buffer b serves tiles it = b, b+2, ...; its k-th use waits on parity k & 1 ("empty" barriers
+// start released: waiting on the opposite parity of a fresh barrier returns immediately).
 template <int MODE, int CLS, bool UNIF, bool UBIAS, int NUCT>
-__global__ void __launch_bounds__(kCircThreads, MODE == MODE_PLAIN ? 3 : 2) layer_circ_kernel(LayerArgs a, int RT, int nbuf_out) {
+__global__ void __launch_bounds__(kCircThreads + 32, (MODE == MODE_PLAIN && UNIF) ? 3 : 2)
+    layer_circ_kernel(LayerArgs a, int RT) {
     constexpr int M = CircCfg<CLS>::M;
     constexpr int WIN = CircCfg<CLS>::WIN;
     extern __shared__ __align__(128) unsigned char smem[];
@@ -62,17 +74,86 @@ __global__ void __launch_bounds__(kCircThreads, MODE == MODE_PLAIN ? 3 : 2) laye
     const int stride = circ_stride(N, CLS);
     float* s_in = reinterpret_cast<float*>(smem);
     float* s_out = s_in + (size_t)2 * RT * stride;
-    uint64_t* bars = reinterpret_cast<uint64_t*>(s_out + (size_t)nbuf_out * RT * N);
-    int* s_row = reinterpret_cast<int*>(bars + 2);
+    uint64_t* bars = reinterpret_cast<uint64_t*>(s_out + (size_t)2 * RT * N);
+    uint64_t* in_full = bars;
+    uint64_t* in_empty = bars + 2;
+    uint64_t* out_full = bars + 4;
+    uint64_t* out_empty = bars + 6;
+    int* s_row = reinterpret_cast<int*>(bars + 8);
     int* s_slot = s_row + 2 * RT;
     int* s_flag = s_slot + 2 * RT;
+    constexpr int kConsumerWarps = kCircThreads / 32;
 
     const int chunks = (CLS == CLS_Q32) ? 1 : (Q + M - 1) / M;
     const int ipr = nu * chunks;  // work items per row
     const int count = *a.count;
     const int ntiles = (count + RT - 1) / RT;
     if ((int)blockIdx.x >= ntiles) return;
+    const int my_tiles = (ntiles - (int)blockIdx.x + (int)gridDim.x - 1) / (int)gridDim.x;
 
+    if (threadIdx.x == 0) {
+        for (int b = 0; b < 2; ++b) {
+            mbar_init(&in_full[b], 1);
+            mbar_init(&in_empty[b], kConsumerWarps);
+            mbar_init(&out_full[b], kConsumerWarps);
+            mbar_init(&out_empty[b], 1);
+        }
+        fence_proxy_async_smem();
+    }
+    __syncthreads();
+
+    if (threadIdx.x >= kCircThreads) {
+        // ------------------------------------------------------------ producer / storer
+        if (threadIdx.x != kCircThreads) return;
+        auto load = [&](int j) {
+            const int b = j & 1;
+            const int tile = (int)blockIdx.x + j * (int)gridDim.x;
+            mbar_wait(&in_empty[b], (uint32_t)(((j >> 1) & 1) ^ 1));  // tile j-2 released in[b]
+            const int r0 = tile * RT;
+            const int nr = min(RT, count - r0);
+            const uint32_t bytes = (uint32_t)nr * (uint32_t)(N * 4 + (CLS == CLS_NU1 ? kHalo * 4 : 0));
+            for (int i = 0; i < nr; ++i) {
+                const int row = a.rows[r0 + i];
+                s_row[b * RT + i] = row;
+                s_flag[b * RT + i] = 0;
+                if constexpr (MODE == MODE_RESIDUAL) s_slot[b * RT + i] = a.cslot[row];
+            }
+            mbar_arrive_expect_tx(&in_full[b], bytes);
+            for (int i = 0; i < nr; ++i) {
+                const float* g = a.yin + (size_t)s_row[b * RT + i] * N;
+                float* d = s_in + (size_t)(b * RT + i) * stride;
+                bulk_g2s(d, g, N * 4, &in_full[b]);
+                if constexpr (CLS == CLS_NU1) bulk_g2s(d + N, g, kHalo * 4, &in_full[b]);  // circular halo
+            }
+        };
+        auto store = [&](int j) {
+            const int b = j & 1;
+            const int tile = (int)blockIdx.x + j * (int)gridDim.x;
+            mbar_wait(&out_full[b], (uint32_t)((j >> 1) & 1));
+            const int r0 = tile * RT;
+            const int nr = min(RT, count - r0);
+            const float* ob = s_out + (size_t)b * RT * N;
+            for (int i = 0; i < nr; ++i) {
+                const int row = s_row[b * RT + i];
+                bulk_s2g(a.yout + (size_t)row * N, ob + (size_t)i * N, N * 4);
+                const uint8_t f = s_flag[b * RT + i] ? 1 : 0;
+                if (a.flag_pos) a.flag_pos[r0 + i] = f;
+                if (a.flag_row) a.flag_row[row] = f;
+            }
+            bulk_commit();
+            bulk_wait_read0();  // the TMA engine has read out[b]
+            mbar_arrive(&out_empty[b]);
+        };
+        for (int j = 0; j < my_tiles; ++j) {
+            load(j);
+            if (j >= 1) store(j - 1);
+        }
+        store(my_tiles - 1);
+        bulk_wait0();
+        return;
+    }
+
+    // ---------------------------------------------------------------- consumers (compute)
     float w[UNIF ? 1 : kK];
     if constexpr (!UNIF) {
 #pragma unroll
@@ -80,53 +161,17 @@ __global__ void __launch_bounds__(kCircThreads, MODE == MODE_PLAIN ? 3 : 2) laye
     }
     const float w0 = a.w0;
     const float b0 = UBIAS ? __ldg(a.bias) : 0.0f;
-
-    if (threadIdx.x == 0) {
-        mbar_init(&bars[0], 1);
-        mbar_init(&bars[1], 1);
-        fence_proxy_async_smem();
-    }
-    __syncthreads();
-
-    // thread 0: stage the rows of `tile` into input buffer b (TMA bulk copies, one mbarrier)
-    auto issue = [&](int tile, int b) {
-        const int r0 = tile * RT;
-        const int nr = min(RT, count - r0);
-        const uint32_t bytes = (uint32_t)nr * (uint32_t)(N * 4 + (CLS == CLS_NU1 ? kHalo * 4 : 0));
-        mbar_arrive_expect_tx(&bars[b], bytes);
-        for (int i = 0; i < nr; ++i) {
-            const int row = a.rows[r0 + i];
-            s_row[b * RT + i] = row;
-            if constexpr (MODE == MODE_RESIDUAL) s_slot[b * RT + i] = a.cslot[row];
-            const float* g = a.yin + (size_t)row * N;
-            float* d = s_in + (size_t)(b * RT + i) * stride;
-            bulk_g2s(d, g, N * 4, &bars[b]);
-            if constexpr (CLS == CLS_NU1) bulk_g2s(d + N, g, kHalo * 4, &bars[b]);  // circular halo
-        }
-    };
-    if (threadIdx.x == 0) issue(blockIdx.x, 0);
-
-    int it = 0;
-    for (int tile = blockIdx.x; tile < ntiles; tile += gridDim.x, ++it) {
-        const int b = it & 1;
-        const int ob = (nbuf_out == 2) ? b : 0;
-        if (threadIdx.x == 0) {
-            const int next = tile + gridDim.x;
-            if (next < ntiles) issue(next, b ^ 1);  // overlaps this tile's compute
-            if (nbuf_out == 2)
-                bulk_wait_read1();  // the store that last used s_out[ob] has read it
-            else
-                bulk_wait_read0();
-        }
-        if ((int)threadIdx.x < RT) s_flag[b * RT + threadIdx.x] = 0;
-        mbar_wait(&bars[b], (uint32_t)((it >> 1) & 1));
-        __syncthreads();
-
-        const int r0 = tile * RT;
-        const int nr = min(RT, count - r0);
+    const int lane = threadIdx.x & 31;
+    for (int j = 0; j < my_tiles; ++j) {
+        const int b = j & 1;
+        const uint32_t ph = (uint32_t)((j >> 1) & 1);
+        const int tile = (int)blockIdx.x + j * (int)gridDim.x;
+        const int nr = min(RT, count - tile * RT);
+        mbar_wait(&in_full[b], ph);
+        mbar_wait(&out_empty[b], ph ^ 1u);
         const float* in_b = s_in + (size_t)b * RT * stride;
-        float* out_b = s_out + (size_t)ob * RT * N;
-        for (int item = threadIdx.x; item < nr * ipr; item += blockDim.x) {
+        float* out_b = s_out + (size_t)b * RT * N;
+        for (int item = threadIdx.x; item < nr * ipr; item += kCircThreads) {
             const int rr = item / ipr;
             const int rem = item - rr * ipr;
             const int row = s_row[b * RT + rr];
@@ -169,7 +214,7 @@ __global__ void __launch_bounds__(kCircThreads, MODE == MODE_PLAIN ? 3 : 2) laye
                 const float* src = in_b + (size_t)rr * stride + c;
                 float R[32];
 #pragma unroll
-                for (int j = 0; j < 32; ++j) R[j] = src[j * nu];
+                for (int jj = 0; jj < 32; ++jj) R[jj] = src[jj * nu];
                 float* dst = out_b + (size_t)rr * N + c;
 #pragma unroll
                 for (int m = 0; m < 32; ++m) {
@@ -217,20 +262,13 @@ __global__ void __launch_bounds__(kCircThreads, MODE == MODE_PLAIN ? 3 : 2) laye
             }
             if (mx != 0.0f) s_flag[b * RT + rr] = 1;
         }
-        fence_proxy_async_smem();  // this thread's s_out writes -> visible to the TMA engine
-        __syncthreads();
-        if (threadIdx.x == 0) {
-            for (int i = 0; i < nr; ++i) {
-                const int row = s_row[b * RT + i];
-                bulk_s2g(a.yout + (size_t)row * N, out_b + (size_t)i * N, N * 4);
-                const uint8_t f = s_flag[b * RT + i] ? 1 : 0;
-                if (a.flag_pos) a.flag_pos[r0 + i] = f;
-                if (a.flag_row) a.flag_row[row] = f;
-            }
-            bulk_commit();
+        fence_proxy_async_smem();  // this thread's out[b] writes -> visible to the TMA engine
+        __syncwarp();
+        if (lane == 0) {
+            mbar_arrive(&in_empty[b]);
+            mbar_arrive(&out_full[b]);
         }
     }
-    if (threadIdx.x == 0) bulk_wait0();
 }
 
 static int circ_class(int N, int nu) {
@@ -244,11 +282,11 @@ bool circ_supported(int N, int K, int nu) {
     if ((long long)K * nu > N) return false;  // distinct inputs -> Q >= K
     const int cls = circ_class(N, nu);
     if (cls == CLS_NU1 && N < kHalo) return false;
-    return circ_smem(N, cls, 1, 1) <= 220 * 1024;
+    return circ_smem2(N, cls, 1) <= 220 * 1024;  // N <= ~13.7K (N = 16384 uses the ELL kernel)
 }
 
 struct CircPlan {
-    int RT, nbuf_out;
+    int RT;
     size_t smem;
 };
 
@@ -260,13 +298,8 @@ static CircPlan circ_plan(int N, int nu) {
     int RT = kCircThreads / ipr;
     if (RT < 1) RT = 1;
     if (RT > 16) RT = 16;
-    while (RT > 1 && circ_smem(N, cls, RT, 2) > 116 * 1024) --RT;
-    CircPlan p{RT, 2, circ_smem(N, cls, RT, 2)};
-    if (p.smem > 220 * 1024) {
-        p.nbuf_out = 1;
-        p.smem = circ_smem(N, cls, RT, 1);
-    }
-    return p;
+    while (RT > 1 && circ_smem2(N, cls, RT) > 116 * 1024) --RT;
+    return CircPlan{RT, circ_smem2(N, cls, RT)};
 }
 
 template <int MODE, int CLS, bool UNIF, bool UBIAS, int NUCT>
@@ -274,13 +307,13 @@ static cudaError_t launch_circ_t(const LayerArgs& a, int max_rows, int num_sms, 
     const CircPlan p = circ_plan(a.N, a.nu);
     auto kern = layer_circ_kernel<MODE, CLS, UNIF, UBIAS, NUCT>;
     int per_sm = 1;
-    cudaError_t e = blocks_per_sm((const void*)kern, kCircThreads, p.smem, &per_sm);
+    cudaError_t e = blocks_per_sm((const void*)kern, kCircThreads + 32, p.smem, &per_sm);
     if (e != cudaSuccess) return e;
     const int tiles = (max_rows + p.RT - 1) / p.RT;
     int grid = num_sms * per_sm;
     if (grid > tiles) grid = tiles;
     if (grid < 1) grid = 1;
-    kern<<<grid, kCircThreads, p.smem, st>>>(a, p.RT, p.nbuf_out);
+    kern<<<grid, kCircThreads + 32, p.smem, st>>>(a, p.RT);
     return cudaGetLastError();
 }
 
