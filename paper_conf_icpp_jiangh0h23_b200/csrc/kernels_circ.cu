@@ -48,23 +48,26 @@ struct CircCfg<CLS_GEN> {
 
 __host__ __device__ constexpr int circ_stride(int N, int cls) { return N + (cls == CLS_NU1 ? kHalo : 0); }
 
-// Shared-memory layout (per CTA): in[2][RT][stride] | out[2][RT][N] | 8 mbarriers | row/slot/flag [2][RT]
-__host__ __device__ constexpr size_t circ_smem2(int N, int cls, int RT) {
-    return sizeof(float) * ((size_t)2 * RT * circ_stride(N, cls) + (size_t)2 * RT * N) + 8 * sizeof(uint64_t) +
-           3 * 2 * sizeof(int) * (size_t)RT;
+constexpr int kMaxStages = 8;
+// Shared-memory layout (per CTA): in[S][RT][stride] | out[2][RT][N] | mbarriers (2S + 4) |
+// row/slot/flag [S][RT]   (flags are per input stage: the producer stores tile j before reusing stage j % S)
+__host__ __device__ constexpr size_t circ_smem2(int N, int cls, int RT, int S) {
+    return sizeof(float) * ((size_t)S * RT * circ_stride(N, cls) + (size_t)2 * RT * N) +
+           (2 * (size_t)S + 4) * sizeof(uint64_t) + 3 * (size_t)S * sizeof(int) * (size_t)RT;
 }
 
 // Warp-specialised: warps 0..7 compute (kCircThreads consumer threads), warp 8 lane 0 is the
-// producer/storer.  mbarriers per buffer b in {0,1}:
-//   in_full[b]   producer arrive.expect_tx + TMA bytes    -> consumers may read in[b]
-//   in_empty[b]  one arrive per consumer warp              -> producer may reload in[b]
-//   out_full[b]  one arrive per consumer warp (after proxy fence) -> producer may TMA-store out[b]
-//   out_empty[b] producer arrive once the store has read out[b]  -> consumers may write out[b]
-// Buffer b serves tiles it = b, b+2, ...; its k-th use waits on parity k & 1 ("empty" barriers
-// start released: waiting on the opposite parity of a fresh barrier returns immediately).
+// producer/storer.  mbarriers:
+//   in_full[s]   (S input stages) producer arrive.expect_tx + TMA bytes -> consumers may read in[s]
+//   in_empty[s]  one arrive per consumer warp                          -> producer may reload in[s]
+//   out_full[b]  (2 output buffers) one arrive per consumer warp after the proxy fence
+//                                                                       -> producer may TMA-store out[b]
+//   out_empty[b] producer arrive once the store has read out[b]        -> consumers may write out[b]
+// Tile j (of this CTA) uses input stage j % S (k-th use: parity k & 1) and output buffer j & 1.
+// "empty" barriers start released (waiting on the opposite parity of a fresh barrier returns at
+// once).  The producer keeps up to S - 1 tiles of loads in flight ahead of the consumers.
 template <int MODE, int CLS, bool UNIF, bool UBIAS, int NUCT>
-__global__ void __launch_bounds__(kCircThreads + 32, (MODE == MODE_PLAIN && UNIF) ? 3 : 2)
-    layer_circ_kernel(LayerArgs a, int RT) {
+__global__ void __launch_bounds__(kCircThreads + 32, 2) layer_circ_kernel(LayerArgs a, int RT, int S) {
     constexpr int M = CircCfg<CLS>::M;
     constexpr int WIN = CircCfg<CLS>::WIN;
     extern __shared__ __align__(128) unsigned char smem[];
@@ -73,15 +76,15 @@ __global__ void __launch_bounds__(kCircThreads + 32, (MODE == MODE_PLAIN && UNIF
     const int Q = N / nu;
     const int stride = circ_stride(N, CLS);
     float* s_in = reinterpret_cast<float*>(smem);
-    float* s_out = s_in + (size_t)2 * RT * stride;
+    float* s_out = s_in + (size_t)S * RT * stride;
     uint64_t* bars = reinterpret_cast<uint64_t*>(s_out + (size_t)2 * RT * N);
     uint64_t* in_full = bars;
-    uint64_t* in_empty = bars + 2;
-    uint64_t* out_full = bars + 4;
-    uint64_t* out_empty = bars + 6;
-    int* s_row = reinterpret_cast<int*>(bars + 8);
-    int* s_slot = s_row + 2 * RT;
-    int* s_flag = s_slot + 2 * RT;
+    uint64_t* in_empty = bars + S;
+    uint64_t* out_full = bars + 2 * S;
+    uint64_t* out_empty = bars + 2 * S + 2;
+    int* s_row = reinterpret_cast<int*>(bars + 2 * S + 4);
+    int* s_slot = s_row + S * RT;
+    int* s_flag = s_slot + S * RT;
     constexpr int kConsumerWarps = kCircThreads / 32;
 
     const int chunks = (CLS == CLS_Q32) ? 1 : (Q + M - 1) / M;
@@ -92,9 +95,11 @@ __global__ void __launch_bounds__(kCircThreads + 32, (MODE == MODE_PLAIN && UNIF
     const int my_tiles = (ntiles - (int)blockIdx.x + (int)gridDim.x - 1) / (int)gridDim.x;
 
     if (threadIdx.x == 0) {
-        for (int b = 0; b < 2; ++b) {
+        for (int b = 0; b < S; ++b) {
             mbar_init(&in_full[b], 1);
             mbar_init(&in_empty[b], kConsumerWarps);
+        }
+        for (int b = 0; b < 2; ++b) {
             mbar_init(&out_full[b], kConsumerWarps);
             mbar_init(&out_empty[b], 1);
         }
@@ -106,9 +111,9 @@ __global__ void __launch_bounds__(kCircThreads + 32, (MODE == MODE_PLAIN && UNIF
         // ------------------------------------------------------------ producer / storer
         if (threadIdx.x != kCircThreads) return;
         auto load = [&](int j) {
-            const int b = j & 1;
+            const int b = j % S;
             const int tile = (int)blockIdx.x + j * (int)gridDim.x;
-            mbar_wait(&in_empty[b], (uint32_t)(((j >> 1) & 1) ^ 1));  // tile j-2 released in[b]
+            mbar_wait(&in_empty[b], (uint32_t)(((j / S) & 1) ^ 1));  // tile j-S released in[b]
             const int r0 = tile * RT;
             const int nr = min(RT, count - r0);
             const uint32_t bytes = (uint32_t)nr * (uint32_t)(N * 4 + (CLS == CLS_NU1 ? kHalo * 4 : 0));
@@ -127,16 +132,17 @@ __global__ void __launch_bounds__(kCircThreads + 32, (MODE == MODE_PLAIN && UNIF
             }
         };
         auto store = [&](int j) {
-            const int b = j & 1;
+            const int b = j & 1;      // output buffer
+            const int sb = j % S;     // input stage (row ids, flags)
             const int tile = (int)blockIdx.x + j * (int)gridDim.x;
             mbar_wait(&out_full[b], (uint32_t)((j >> 1) & 1));
             const int r0 = tile * RT;
             const int nr = min(RT, count - r0);
             const float* ob = s_out + (size_t)b * RT * N;
             for (int i = 0; i < nr; ++i) {
-                const int row = s_row[b * RT + i];
+                const int row = s_row[sb * RT + i];
                 bulk_s2g(a.yout + (size_t)row * N, ob + (size_t)i * N, N * 4);
-                const uint8_t f = s_flag[b * RT + i] ? 1 : 0;
+                const uint8_t f = s_flag[sb * RT + i] ? 1 : 0;
                 if (a.flag_pos) a.flag_pos[r0 + i] = f;
                 if (a.flag_row) a.flag_row[row] = f;
             }
@@ -144,11 +150,12 @@ __global__ void __launch_bounds__(kCircThreads + 32, (MODE == MODE_PLAIN && UNIF
             bulk_wait_read0();  // the TMA engine has read out[b]
             mbar_arrive(&out_empty[b]);
         };
-        for (int j = 0; j < my_tiles; ++j) {
-            load(j);
-            if (j >= 1) store(j - 1);
+        // loads run up to S - 1 tiles ahead; store(j) needs tile j computed.  load(j) waits for
+        // tile j - S to be consumed, which precedes tile j - S + 1, so no cycle can form.
+        for (int j = 0; j < my_tiles + S - 1; ++j) {
+            if (j < my_tiles) load(j);
+            if (j >= S - 1) store(j - (S - 1));
         }
-        store(my_tiles - 1);
         bulk_wait0();
         return;
     }
@@ -163,19 +170,19 @@ __global__ void __launch_bounds__(kCircThreads + 32, (MODE == MODE_PLAIN && UNIF
     const float b0 = UBIAS ? __ldg(a.bias) : 0.0f;
     const int lane = threadIdx.x & 31;
     for (int j = 0; j < my_tiles; ++j) {
-        const int b = j & 1;
-        const uint32_t ph = (uint32_t)((j >> 1) & 1);
+        const int sb = j % S;  // input stage
+        const int b = j & 1;   // output buffer
         const int tile = (int)blockIdx.x + j * (int)gridDim.x;
         const int nr = min(RT, count - tile * RT);
-        mbar_wait(&in_full[b], ph);
-        mbar_wait(&out_empty[b], ph ^ 1u);
-        const float* in_b = s_in + (size_t)b * RT * stride;
+        mbar_wait(&in_full[sb], (uint32_t)((j / S) & 1));
+        mbar_wait(&out_empty[b], (uint32_t)(((j >> 1) & 1) ^ 1));
+        const float* in_b = s_in + (size_t)sb * RT * stride;
         float* out_b = s_out + (size_t)b * RT * N;
         for (int item = threadIdx.x; item < nr * ipr; item += kCircThreads) {
             const int rr = item / ipr;
             const int rem = item - rr * ipr;
-            const int row = s_row[b * RT + rr];
-            const int slot = (MODE == MODE_RESIDUAL) ? s_slot[b * RT + rr] : 0;
+            const int row = s_row[sb * RT + rr];
+            const int slot = (MODE == MODE_RESIDUAL) ? s_slot[sb * RT + rr] : 0;
             float mx = 0.0f;
             if constexpr (CLS == CLS_NU1) {
                 const int a0 = rem * M;
@@ -260,12 +267,12 @@ __global__ void __launch_bounds__(kCircThreads + 32, (MODE == MODE_PLAIN && UNIF
                     }
                 }
             }
-            if (mx != 0.0f) s_flag[b * RT + rr] = 1;
+            if (mx != 0.0f) s_flag[sb * RT + rr] = 1;
         }
         fence_proxy_async_smem();  // this thread's out[b] writes -> visible to the TMA engine
         __syncwarp();
         if (lane == 0) {
-            mbar_arrive(&in_empty[b]);
+            mbar_arrive(&in_empty[sb]);
             mbar_arrive(&out_full[b]);
         }
     }
@@ -282,11 +289,11 @@ bool circ_supported(int N, int K, int nu) {
     if ((long long)K * nu > N) return false;  // distinct inputs -> Q >= K
     const int cls = circ_class(N, nu);
     if (cls == CLS_NU1 && N < kHalo) return false;
-    return circ_smem2(N, cls, 1) <= 220 * 1024;  // N <= ~13.7K (N = 16384 uses the ELL kernel)
+    return circ_smem2(N, cls, 1, 2) <= 220 * 1024;  // N <= ~13.7K (larger N: the ELL kernel)
 }
 
 struct CircPlan {
-    int RT;
+    int RT, S;
     size_t smem;
 };
 
@@ -298,8 +305,12 @@ static CircPlan circ_plan(int N, int nu) {
     int RT = kCircThreads / ipr;
     if (RT < 1) RT = 1;
     if (RT > 16) RT = 16;
-    while (RT > 1 && circ_smem2(N, cls, RT) > 116 * 1024) --RT;
-    return CircPlan{RT, circ_smem2(N, cls, RT)};
+    // two CTAs per SM (~113 KB each): as many input stages as fit (bytes in flight hide HBM latency)
+    const size_t budget = 113 * 1024;
+    while (RT > 1 && circ_smem2(N, cls, RT, 3) > budget) --RT;
+    int S = 2;
+    while (S < kMaxStages && circ_smem2(N, cls, RT, S + 1) <= budget) ++S;
+    return CircPlan{RT, S, circ_smem2(N, cls, RT, S)};
 }
 
 template <int MODE, int CLS, bool UNIF, bool UBIAS, int NUCT>
@@ -313,7 +324,7 @@ static cudaError_t launch_circ_t(const LayerArgs& a, int max_rows, int num_sms, 
     int grid = num_sms * per_sm;
     if (grid > tiles) grid = tiles;
     if (grid < 1) grid = 1;
-    kern<<<grid, kCircThreads + 32, p.smem, st>>>(a, p.RT);
+    kern<<<grid, kCircThreads + 32, p.smem, st>>>(a, p.RT, p.S);
     return cudaGetLastError();
 }
 

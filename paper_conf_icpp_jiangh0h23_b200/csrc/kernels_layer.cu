@@ -30,6 +30,7 @@ namespace snicit {
 cudaError_t blocks_per_sm(const void* kern, int threads, size_t smem, int* out) {
     static std::mutex mu;
     static std::map<std::pair<std::pair<int, const void*>, size_t>, int> cache;
+    static std::map<std::pair<int, const void*>, size_t> attr;  // max dynamic smem set per kernel
     int dev = 0;
     cudaError_t e = cudaGetDevice(&dev);
     if (e != cudaSuccess) return e;
@@ -41,9 +42,15 @@ cudaError_t blocks_per_sm(const void* kern, int threads, size_t smem, int* out) 
             *out = it->second;
             return cudaSuccess;
         }
+        // the attribute is a per-kernel maximum: only ever raise it (a kernel launched with several
+        // shared-memory sizes must keep the largest one allowed)
+        size_t& cur = attr[key.first];
+        if (smem > cur) {
+            e = cudaFuncSetAttribute(kern, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)smem);
+            if (e != cudaSuccess) return e;
+            cur = smem;
+        }
     }
-    e = cudaFuncSetAttribute(kern, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)smem);
-    if (e != cudaSuccess) return e;
     int per_sm = 1;
     e = cudaOccupancyMaxActiveBlocksPerMultiprocessor(&per_sm, kern, threads, smem);
     if (e != cudaSuccess) return e;
