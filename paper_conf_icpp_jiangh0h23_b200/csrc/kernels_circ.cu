@@ -67,7 +67,8 @@ __host__ __device__ constexpr size_t circ_smem2(int N, int cls, int RT, int S) {
 // "empty" barriers start released (waiting on the opposite parity of a fresh barrier returns at
 // once).  The producer keeps up to S - 1 tiles of loads in flight ahead of the consumers.
 template <int MODE, int CLS, bool UNIF, bool UBIAS, int NUCT>
-__global__ void __launch_bounds__(kCircThreads + 32, 2) layer_circ_kernel(LayerArgs a, int RT, int S) {
+__global__ void __launch_bounds__(kCircThreads + 32, (MODE == MODE_PLAIN && UNIF) ? 3 : 2)
+    layer_circ_kernel(LayerArgs a, int RT, int S) {
     constexpr int M = CircCfg<CLS>::M;
     constexpr int WIN = CircCfg<CLS>::WIN;
     extern __shared__ __align__(128) unsigned char smem[];
@@ -91,8 +92,11 @@ __global__ void __launch_bounds__(kCircThreads + 32, 2) layer_circ_kernel(LayerA
     const int ipr = nu * chunks;  // work items per row
     const int count = *a.count;
     const int ntiles = (count + RT - 1) / RT;
-    if ((int)blockIdx.x >= ntiles) return;
-    const int my_tiles = (ntiles - (int)blockIdx.x + (int)gridDim.x - 1) / (int)gridDim.x;
+    // contiguous tile range per CTA: its row ids are contiguous in the list (prefetchable)
+    const int tpc = (ntiles + (int)gridDim.x - 1) / (int)gridDim.x;
+    const int t_begin = (int)blockIdx.x * tpc;
+    const int my_tiles = min(ntiles, t_begin + tpc) - t_begin;
+    if (my_tiles <= 0) return;
 
     if (threadIdx.x == 0) {
         for (int b = 0; b < S; ++b) {
@@ -108,47 +112,70 @@ __global__ void __launch_bounds__(kCircThreads + 32, 2) layer_circ_kernel(LayerA
     __syncthreads();
 
     if (threadIdx.x >= kCircThreads) {
-        // ------------------------------------------------------------ producer / storer
-        if (threadIdx.x != kCircThreads) return;
+        // ------------------------------------------------------------ producer / storer warp
+        const int lane = threadIdx.x & 31;
+        const int row_base = t_begin * RT;                        // first list position of this CTA
+        const int my_rows = min(count, (t_begin + my_tiles) * RT) - row_base;
+        // register windows of row ids (and centroid slots): lane l holds local position w0 + l (cur)
+        // and w0 + 32 + l (nxt); the global loads of a window are issued 32 positions ahead of use
+        int w0 = 0;
+        int cur = lane < my_rows ? a.rows[row_base + lane] : 0;
+        int nxt = 32 + lane < my_rows ? a.rows[row_base + 32 + lane] : 0;
+        int scur = 0;
+        if constexpr (MODE == MODE_RESIDUAL) scur = lane < my_rows ? a.cslot[cur] : 0;
+        auto advance_to = [&](int p) {  // warp-uniform, p non-decreasing
+            while (p >= w0 + 32) {
+                cur = nxt;
+                w0 += 32;
+                nxt = (w0 + 32 + lane < my_rows) ? a.rows[row_base + w0 + 32 + lane] : 0;
+                if constexpr (MODE == MODE_RESIDUAL) scur = (w0 + lane < my_rows) ? a.cslot[cur] : 0;
+            }
+        };
         auto load = [&](int j) {
             const int b = j % S;
-            const int tile = (int)blockIdx.x + j * (int)gridDim.x;
-            mbar_wait(&in_empty[b], (uint32_t)(((j / S) & 1) ^ 1));  // tile j-S released in[b]
-            const int r0 = tile * RT;
+            const int r0 = (t_begin + j) * RT;
             const int nr = min(RT, count - r0);
+            if (lane == 0) mbar_wait(&in_empty[b], (uint32_t)(((j / S) & 1) ^ 1));  // tile j-S released in[b]
+            __syncwarp();
             const uint32_t bytes = (uint32_t)nr * (uint32_t)(N * 4 + (CLS == CLS_NU1 ? kHalo * 4 : 0));
+            if (lane == 0) mbar_arrive_expect_tx(&in_full[b], bytes);
             for (int i = 0; i < nr; ++i) {
-                const int row = a.rows[r0 + i];
-                s_row[b * RT + i] = row;
-                s_flag[b * RT + i] = 0;
-                if constexpr (MODE == MODE_RESIDUAL) s_slot[b * RT + i] = a.cslot[row];
-            }
-            mbar_arrive_expect_tx(&in_full[b], bytes);
-            for (int i = 0; i < nr; ++i) {
-                const float* g = a.yin + (size_t)s_row[b * RT + i] * N;
-                float* d = s_in + (size_t)(b * RT + i) * stride;
-                bulk_g2s(d, g, N * 4, &in_full[b]);
-                if constexpr (CLS == CLS_NU1) bulk_g2s(d + N, g, kHalo * 4, &in_full[b]);  // circular halo
+                const int p = r0 + i - row_base;
+                advance_to(p);
+                const int row = __shfl_sync(0xffffffffu, cur, p - w0);
+                int slot = 0;
+                if constexpr (MODE == MODE_RESIDUAL) slot = __shfl_sync(0xffffffffu, scur, p - w0);
+                if (lane == 0) {
+                    s_row[b * RT + i] = row;
+                    s_flag[b * RT + i] = 0;
+                    if constexpr (MODE == MODE_RESIDUAL) s_slot[b * RT + i] = slot;
+                    const float* g = a.yin + (size_t)row * N;
+                    float* d = s_in + (size_t)(b * RT + i) * stride;
+                    bulk_g2s(d, g, N * 4, &in_full[b]);
+                    if constexpr (CLS == CLS_NU1) bulk_g2s(d + N, g, kHalo * 4, &in_full[b]);  // circular halo
+                }
             }
         };
         auto store = [&](int j) {
-            const int b = j & 1;      // output buffer
-            const int sb = j % S;     // input stage (row ids, flags)
-            const int tile = (int)blockIdx.x + j * (int)gridDim.x;
-            mbar_wait(&out_full[b], (uint32_t)((j >> 1) & 1));
-            const int r0 = tile * RT;
-            const int nr = min(RT, count - r0);
-            const float* ob = s_out + (size_t)b * RT * N;
-            for (int i = 0; i < nr; ++i) {
-                const int row = s_row[sb * RT + i];
-                bulk_s2g(a.yout + (size_t)row * N, ob + (size_t)i * N, N * 4);
-                const uint8_t f = s_flag[sb * RT + i] ? 1 : 0;
-                if (a.flag_pos) a.flag_pos[r0 + i] = f;
-                if (a.flag_row) a.flag_row[row] = f;
+            if (lane == 0) {
+                const int b = j & 1;   // output buffer
+                const int sb = j % S;  // input stage (row ids, flags)
+                const int r0 = (t_begin + j) * RT;
+                const int nr = min(RT, count - r0);
+                mbar_wait(&out_full[b], (uint32_t)((j >> 1) & 1));
+                const float* ob = s_out + (size_t)b * RT * N;
+                for (int i = 0; i < nr; ++i) {
+                    const int row = s_row[sb * RT + i];
+                    bulk_s2g(a.yout + (size_t)row * N, ob + (size_t)i * N, N * 4);
+                    const uint8_t f = s_flag[sb * RT + i] ? 1 : 0;
+                    if (a.flag_pos) a.flag_pos[r0 + i] = f;
+                    if (a.flag_row) a.flag_row[row] = f;
+                }
+                bulk_commit();
+                bulk_wait_read0();  // the TMA engine has read out[b]
+                mbar_arrive(&out_empty[b]);
             }
-            bulk_commit();
-            bulk_wait_read0();  // the TMA engine has read out[b]
-            mbar_arrive(&out_empty[b]);
+            __syncwarp();
         };
         // loads run up to S - 1 tiles ahead; store(j) needs tile j computed.  load(j) waits for
         // tile j - S to be consumed, which precedes tile j - S + 1, so no cycle can form.
@@ -156,7 +183,7 @@ __global__ void __launch_bounds__(kCircThreads + 32, 2) layer_circ_kernel(LayerA
             if (j < my_tiles) load(j);
             if (j >= S - 1) store(j - (S - 1));
         }
-        bulk_wait0();
+        if (lane == 0) bulk_wait0();
         return;
     }
 
@@ -172,8 +199,7 @@ __global__ void __launch_bounds__(kCircThreads + 32, 2) layer_circ_kernel(LayerA
     for (int j = 0; j < my_tiles; ++j) {
         const int sb = j % S;  // input stage
         const int b = j & 1;   // output buffer
-        const int tile = (int)blockIdx.x + j * (int)gridDim.x;
-        const int nr = min(RT, count - tile * RT);
+        const int nr = min(RT, count - (t_begin + j) * RT);
         mbar_wait(&in_full[sb], (uint32_t)((j / S) & 1));
         mbar_wait(&out_empty[b], (uint32_t)(((j >> 1) & 1) ^ 1));
         const float* in_b = s_in + (size_t)sb * RT * stride;
@@ -305,8 +331,8 @@ static CircPlan circ_plan(int N, int nu) {
     int RT = kCircThreads / ipr;
     if (RT < 1) RT = 1;
     if (RT > 16) RT = 16;
-    // two CTAs per SM (~113 KB each): as many input stages as fit (bytes in flight hide HBM latency)
-    const size_t budget = 113 * 1024;
+    // three CTAs per SM (~75 KB each): as many input stages as fit (bytes in flight hide HBM latency)
+    const size_t budget = 75 * 1024;
     while (RT > 1 && circ_smem2(N, cls, RT, 3) > budget) --RT;
     int S = 2;
     while (S < kMaxStages && circ_smem2(N, cls, RT, S + 1) <= budget) ++S;
