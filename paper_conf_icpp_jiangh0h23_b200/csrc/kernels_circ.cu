@@ -16,10 +16,10 @@
 //   GEN  other nu: M = 16 outputs per thread, lanes walk consecutive residues; windows that wrap
 //        (warp-uniform) take a masked path.
 //
-// Pipeline per CTA (persistent over row tiles, warp-specialised): a producer warp stages tile i+1
-// with TMA bulk loads while 8 consumer warps compute tile i; outputs are staged in shared memory
-// (double-buffered) and written back by the producer with TMA bulk stores (coalesced for every nu).
-// Producer and consumers synchronise only through mbarriers.  Epilogues: see LayerMode.
+// Pipeline per CTA (persistent over a contiguous range of row tiles, warp-specialised): a producer
+// warp keeps S - 1 tiles of TMA bulk loads in flight while 8 consumer warps compute; the outputs
+// overwrite the tile's stage in shared memory and the producer writes them back with TMA bulk stores
+// (coalesced for every nu).  Producer and consumers synchronise only through mbarriers.
 #include <cuda_runtime.h>
 
 #include "snicit_internal.cuh"
@@ -49,23 +49,23 @@ struct CircCfg<CLS_GEN> {
 __host__ __device__ constexpr int circ_stride(int N, int cls) { return N + (cls == CLS_NU1 ? kHalo : 0); }
 
 constexpr int kMaxStages = 8;
-// Shared-memory layout (per CTA): in[S][RT][stride] | out[2][RT][N] | mbarriers (2S + 4) |
-// row/slot/flag [S][RT]   (flags are per input stage: the producer stores tile j before reusing stage j % S)
+// Shared-memory layout (per CTA): stage[S][RT][stride] | mbarriers (2S) | row/slot/flag [S][RT]
 __host__ __device__ constexpr size_t circ_smem2(int N, int cls, int RT, int S) {
-    return sizeof(float) * ((size_t)S * RT * circ_stride(N, cls) + (size_t)2 * RT * N) +
-           (2 * (size_t)S + 4) * sizeof(uint64_t) + 3 * (size_t)S * sizeof(int) * (size_t)RT;
+    return sizeof(float) * (size_t)S * RT * circ_stride(N, cls) + 2 * (size_t)S * sizeof(uint64_t) +
+           3 * (size_t)S * sizeof(int) * (size_t)RT;
 }
 
-// Warp-specialised: warps 0..7 compute (kCircThreads consumer threads), warp 8 lane 0 is the
-// producer/storer.  mbarriers:
-//   in_full[s]   (S input stages) producer arrive.expect_tx + TMA bytes -> consumers may read in[s]
-//   in_empty[s]  one arrive per consumer warp                          -> producer may reload in[s]
-//   out_full[b]  (2 output buffers) one arrive per consumer warp after the proxy fence
-//                                                                       -> producer may TMA-store out[b]
-//   out_empty[b] producer arrive once the store has read out[b]        -> consumers may write out[b]
-// Tile j (of this CTA) uses input stage j % S (k-th use: parity k & 1) and output buffer j & 1.
-// "empty" barriers start released (waiting on the opposite parity of a fresh barrier returns at
-// once).  The producer keeps up to S - 1 tiles of loads in flight ahead of the consumers.
+__device__ __forceinline__ void consumer_bar() { asm volatile("bar.sync 1, %0;" ::"n"(kCircThreads) : "memory"); }
+
+// Warp-specialised, in-place: warps 0..7 compute (one work item per thread per tile), warp 8 is the
+// producer/storer.  Tile j of this CTA lives in stage j % S (k-th use: parity k & 1):
+//   in_full[s]   producer arrive.expect_tx + TMA load bytes  -> consumers may read stage s
+//   out_full[s]  one arrive per consumer warp (after the outputs were written into stage s and
+//                proxy-fenced)                                -> producer TMA-stores stage s; once the
+//                store has read it (bulk wait_group.read) the producer reloads the stage.
+// Consumers keep their M outputs in registers, meet at a consumer-only named barrier (every read of
+// the stage is done), then overwrite the stage with the outputs, so no separate output buffers are
+// needed and more stages (bytes in flight) fit.  The producer keeps S - 1 tiles of loads ahead.
 template <int MODE, int CLS, bool UNIF, bool UBIAS, int NUCT>
 __global__ void __launch_bounds__(kCircThreads + 32, (MODE == MODE_PLAIN && UNIF) ? 3 : 2)
     layer_circ_kernel(LayerArgs a, int RT, int S) {
@@ -76,20 +76,17 @@ __global__ void __launch_bounds__(kCircThreads + 32, (MODE == MODE_PLAIN && UNIF
     const int nu = NUCT ? NUCT : a.nu;
     const int Q = N / nu;
     const int stride = circ_stride(N, CLS);
-    float* s_in = reinterpret_cast<float*>(smem);
-    float* s_out = s_in + (size_t)S * RT * stride;
-    uint64_t* bars = reinterpret_cast<uint64_t*>(s_out + (size_t)2 * RT * N);
+    float* s_st = reinterpret_cast<float*>(smem);
+    uint64_t* bars = reinterpret_cast<uint64_t*>(s_st + (size_t)S * RT * stride);
     uint64_t* in_full = bars;
-    uint64_t* in_empty = bars + S;
-    uint64_t* out_full = bars + 2 * S;
-    uint64_t* out_empty = bars + 2 * S + 2;
-    int* s_row = reinterpret_cast<int*>(bars + 2 * S + 4);
+    uint64_t* out_full = bars + S;
+    int* s_row = reinterpret_cast<int*>(bars + 2 * S);
     int* s_slot = s_row + S * RT;
     int* s_flag = s_slot + S * RT;
     constexpr int kConsumerWarps = kCircThreads / 32;
 
     const int chunks = (CLS == CLS_Q32) ? 1 : (Q + M - 1) / M;
-    const int ipr = nu * chunks;  // work items per row
+    const int ipr = nu * chunks;  // work items per row (RT * ipr <= kCircThreads by the plan)
     const int count = *a.count;
     const int ntiles = (count + RT - 1) / RT;
     // contiguous tile range per CTA: its row ids are contiguous in the list (prefetchable)
@@ -101,11 +98,7 @@ __global__ void __launch_bounds__(kCircThreads + 32, (MODE == MODE_PLAIN && UNIF
     if (threadIdx.x == 0) {
         for (int b = 0; b < S; ++b) {
             mbar_init(&in_full[b], 1);
-            mbar_init(&in_empty[b], kConsumerWarps);
-        }
-        for (int b = 0; b < 2; ++b) {
             mbar_init(&out_full[b], kConsumerWarps);
-            mbar_init(&out_empty[b], 1);
         }
         fence_proxy_async_smem();
     }
@@ -114,7 +107,7 @@ __global__ void __launch_bounds__(kCircThreads + 32, (MODE == MODE_PLAIN && UNIF
     if (threadIdx.x >= kCircThreads) {
         // ------------------------------------------------------------ producer / storer warp
         const int lane = threadIdx.x & 31;
-        const int row_base = t_begin * RT;                        // first list position of this CTA
+        const int row_base = t_begin * RT;  // first list position of this CTA
         const int my_rows = min(count, (t_begin + my_tiles) * RT) - row_base;
         // register windows of row ids (and centroid slots): lane l holds local position w0 + l (cur)
         // and w0 + 32 + l (nxt); the global loads of a window are issued 32 positions ahead of use
@@ -131,12 +124,10 @@ __global__ void __launch_bounds__(kCircThreads + 32, (MODE == MODE_PLAIN && UNIF
                 if constexpr (MODE == MODE_RESIDUAL) scur = (w0 + lane < my_rows) ? a.cslot[cur] : 0;
             }
         };
-        auto load = [&](int j) {
+        auto load = [&](int j) {  // stage j % S is free (its previous tile was stored and read)
             const int b = j % S;
             const int r0 = (t_begin + j) * RT;
             const int nr = min(RT, count - r0);
-            if (lane == 0) mbar_wait(&in_empty[b], (uint32_t)(((j / S) & 1) ^ 1));  // tile j-S released in[b]
-            __syncwarp();
             const uint32_t bytes = (uint32_t)nr * (uint32_t)(N * 4 + (CLS == CLS_NU1 ? kHalo * 4 : 0));
             if (lane == 0) mbar_arrive_expect_tx(&in_full[b], bytes);
             for (int i = 0; i < nr; ++i) {
@@ -150,7 +141,7 @@ __global__ void __launch_bounds__(kCircThreads + 32, (MODE == MODE_PLAIN && UNIF
                     s_flag[b * RT + i] = 0;
                     if constexpr (MODE == MODE_RESIDUAL) s_slot[b * RT + i] = slot;
                     const float* g = a.yin + (size_t)row * N;
-                    float* d = s_in + (size_t)(b * RT + i) * stride;
+                    float* d = s_st + (size_t)(b * RT + i) * stride;
                     bulk_g2s(d, g, N * 4, &in_full[b]);
                     if constexpr (CLS == CLS_NU1) bulk_g2s(d + N, g, kHalo * 4, &in_full[b]);  // circular halo
                 }
@@ -158,31 +149,27 @@ __global__ void __launch_bounds__(kCircThreads + 32, (MODE == MODE_PLAIN && UNIF
         };
         auto store = [&](int j) {
             if (lane == 0) {
-                const int b = j & 1;   // output buffer
-                const int sb = j % S;  // input stage (row ids, flags)
+                const int b = j % S;
                 const int r0 = (t_begin + j) * RT;
                 const int nr = min(RT, count - r0);
-                mbar_wait(&out_full[b], (uint32_t)((j >> 1) & 1));
-                const float* ob = s_out + (size_t)b * RT * N;
+                mbar_wait(&out_full[b], (uint32_t)((j / S) & 1));
                 for (int i = 0; i < nr; ++i) {
-                    const int row = s_row[sb * RT + i];
-                    bulk_s2g(a.yout + (size_t)row * N, ob + (size_t)i * N, N * 4);
-                    const uint8_t f = s_flag[sb * RT + i] ? 1 : 0;
+                    const int row = s_row[b * RT + i];
+                    bulk_s2g(a.yout + (size_t)row * N, s_st + (size_t)(b * RT + i) * stride, N * 4);
+                    const uint8_t f = s_flag[b * RT + i] ? 1 : 0;
                     if (a.flag_pos) a.flag_pos[r0 + i] = f;
                     if (a.flag_row) a.flag_row[row] = f;
                 }
                 bulk_commit();
-                bulk_wait_read0();  // the TMA engine has read out[b]
-                mbar_arrive(&out_empty[b]);
+                bulk_wait_read0();  // the TMA engine has read the stage: it may be reloaded
             }
             __syncwarp();
         };
-        // loads run up to S - 1 tiles ahead; store(j) needs tile j computed.  load(j) waits for
-        // tile j - S to be consumed, which precedes tile j - S + 1, so no cycle can form.
-        for (int j = 0; j < my_tiles + S - 1; ++j) {
-            if (j < my_tiles) load(j);
-            if (j >= S - 1) store(j - (S - 1));
+        for (int j = 0; j < my_tiles; ++j) {
+            if (j >= S) store(j - S);
+            load(j);
         }
+        for (int j = max(0, my_tiles - S); j < my_tiles; ++j) store(j);
         if (lane == 0) bulk_wait0();
         return;
     }
@@ -196,59 +183,48 @@ __global__ void __launch_bounds__(kCircThreads + 32, (MODE == MODE_PLAIN && UNIF
     const float w0 = a.w0;
     const float b0 = UBIAS ? __ldg(a.bias) : 0.0f;
     const int lane = threadIdx.x & 31;
+    const int item = threadIdx.x;
     for (int j = 0; j < my_tiles; ++j) {
-        const int sb = j % S;  // input stage
-        const int b = j & 1;   // output buffer
+        const int sb = j % S;
         const int nr = min(RT, count - (t_begin + j) * RT);
         mbar_wait(&in_full[sb], (uint32_t)((j / S) & 1));
-        mbar_wait(&out_empty[b], (uint32_t)(((j >> 1) & 1) ^ 1));
-        const float* in_b = s_in + (size_t)sb * RT * stride;
-        float* out_b = s_out + (size_t)b * RT * N;
-        for (int item = threadIdx.x; item < nr * ipr; item += kCircThreads) {
-            const int rr = item / ipr;
+        float* st = s_st + (size_t)sb * RT * stride;
+        float v[M];
+        int rr = 0, obase = 0, ostep = 1, mlim = 0;
+        float mx = 0.0f;
+        if (item < nr * ipr) {
+            rr = item / ipr;
             const int rem = item - rr * ipr;
             const int row = s_row[sb * RT + rr];
             const int slot = (MODE == MODE_RESIDUAL) ? s_slot[sb * RT + rr] : 0;
-            float mx = 0.0f;
+            const float* src0 = st + (size_t)rr * stride;
             if constexpr (CLS == CLS_NU1) {
                 const int a0 = rem * M;
-                const float* src = in_b + (size_t)rr * stride + a0;
+                const float* src = src0 + a0;
                 float R[WIN];
 #pragma unroll
                 for (int i = 0; i < WIN; ++i) R[i] = src[i];
-                float* dst = out_b + (size_t)rr * N + a0;
-                if (a0 + M <= N) {  // all but the last chunk of a row: no guards, chains interleave
+                obase = a0;
+                ostep = 1;
+                mlim = min(M, N - a0);
 #pragma unroll
-                    for (int m = 0; m < M; ++m) {
-                        float acc = 0.0f;
+                for (int m = 0; m < M; ++m) {
+                    float acc = 0.0f;
 #pragma unroll
-                        for (int n = 0; n < kK; ++n) acc = fmaf(R[m + n], UNIF ? w0 : w[n], acc);
-                        const float bq = UBIAS ? b0 : __ldg(a.bias + a0 + m);
-                        const float v = epilogue<MODE>(a, acc, bq, a0 + m, row, slot);
-                        dst[m] = v;
-                        mx = fmaxf(mx, fabsf(v));
-                    }
-                } else {
-#pragma unroll
-                    for (int m = 0; m < M; ++m) {
-                        if (a0 + m < N) {
-                            float acc = 0.0f;
-#pragma unroll
-                            for (int n = 0; n < kK; ++n) acc = fmaf(R[m + n], UNIF ? w0 : w[n], acc);
-                            const float bq = UBIAS ? b0 : __ldg(a.bias + a0 + m);
-                            const float v = epilogue<MODE>(a, acc, bq, a0 + m, row, slot);
-                            dst[m] = v;
-                            mx = fmaxf(mx, fabsf(v));
-                        }
-                    }
+                    for (int n = 0; n < kK; ++n) acc = fmaf(R[m + n], UNIF ? w0 : w[n], acc);
+                    const int q = min(a0 + m, N - 1);  // tail outputs (m >= mlim) are discarded
+                    const float bq = UBIAS ? b0 : __ldg(a.bias + q);
+                    v[m] = epilogue<MODE>(a, acc, bq, q, row, slot);
                 }
             } else if constexpr (CLS == CLS_Q32) {
                 const int c = rem;
-                const float* src = in_b + (size_t)rr * stride + c;
+                const float* src = src0 + c;
                 float R[32];
 #pragma unroll
                 for (int jj = 0; jj < 32; ++jj) R[jj] = src[jj * nu];
-                float* dst = out_b + (size_t)rr * N + c;
+                obase = c;
+                ostep = nu;
+                mlim = 32;
 #pragma unroll
                 for (int m = 0; m < 32; ++m) {
                     float acc = 0.0f;
@@ -256,14 +232,12 @@ __global__ void __launch_bounds__(kCircThreads + 32, (MODE == MODE_PLAIN && UNIF
                     for (int n = 0; n < kK; ++n) acc = fmaf(R[(m + n) & 31], UNIF ? w0 : w[n], acc);
                     const int q = m * nu + c;
                     const float bq = UBIAS ? b0 : __ldg(a.bias + q);
-                    const float v = epilogue<MODE>(a, acc, bq, q, row, slot);
-                    dst[m * nu] = v;
-                    mx = fmaxf(mx, fabsf(v));
+                    v[m] = epilogue<MODE>(a, acc, bq, q, row, slot);
                 }
             } else {  // CLS_GEN
                 const int c = rem % nu;
                 const int a0 = (rem / nu) * M;
-                const float* src = in_b + (size_t)rr * stride + c;
+                const float* src = src0 + c;
                 float R[WIN];
                 if (a0 + WIN <= Q) {  // warp-uniform: lanes share a0
 #pragma unroll
@@ -277,30 +251,42 @@ __global__ void __launch_bounds__(kCircThreads + 32, (MODE == MODE_PLAIN && UNIF
                         R[i] = src[ai * nu];
                     }
                 }
-                float* dst = out_b + (size_t)rr * N + c + (size_t)a0 * nu;
-                const int mlim = min(M, Q - a0);  // == M unless Q % M != 0
+                obase = a0 * nu + c;
+                ostep = nu;
+                mlim = min(M, Q - a0);
 #pragma unroll
                 for (int m = 0; m < M; ++m) {
-                    if (m < mlim) {
-                        float acc = 0.0f;
+                    float acc = 0.0f;
 #pragma unroll
-                        for (int n = 0; n < kK; ++n) acc = fmaf(R[m + n], UNIF ? w0 : w[n], acc);
-                        const int q = (a0 + m) * nu + c;
-                        const float bq = UBIAS ? b0 : __ldg(a.bias + q);
-                        const float v = epilogue<MODE>(a, acc, bq, q, row, slot);
-                        dst[m * nu] = v;
-                        mx = fmaxf(mx, fabsf(v));
-                    }
+                    for (int n = 0; n < kK; ++n) acc = fmaf(R[m + n], UNIF ? w0 : w[n], acc);
+                    const int q = min(a0 + m, Q - 1) * nu + c;  // tail outputs are discarded
+                    const float bq = UBIAS ? b0 : __ldg(a.bias + q);
+                    v[m] = epilogue<MODE>(a, acc, bq, q, row, slot);
                 }
+            }
+        }
+        consumer_bar();  // every read of this stage is done: overwrite it with the outputs
+        if (item < nr * ipr) {
+            float* dst = st + (size_t)rr * stride + obase;
+            if (mlim == M) {
+#pragma unroll
+                for (int m = 0; m < M; ++m) {
+                    dst[m * ostep] = v[m];
+                    mx = fmaxf(mx, fabsf(v[m]));
+                }
+            } else {
+#pragma unroll
+                for (int m = 0; m < M; ++m)
+                    if (m < mlim) {
+                        dst[m * ostep] = v[m];
+                        mx = fmaxf(mx, fabsf(v[m]));
+                    }
             }
             if (mx != 0.0f) s_flag[sb * RT + rr] = 1;
         }
-        fence_proxy_async_smem();  // this thread's out[b] writes -> visible to the TMA engine
+        fence_proxy_async_smem();  // this thread's writes -> visible to the TMA engine
         __syncwarp();
-        if (lane == 0) {
-            mbar_arrive(&in_empty[sb]);
-            mbar_arrive(&out_full[b]);
-        }
+        if (lane == 0) mbar_arrive(&out_full[sb]);
     }
 }
 
@@ -315,7 +301,11 @@ bool circ_supported(int N, int K, int nu) {
     if ((long long)K * nu > N) return false;  // distinct inputs -> Q >= K
     const int cls = circ_class(N, nu);
     if (cls == CLS_NU1 && N < kHalo) return false;
-    return circ_smem2(N, cls, 1, 2) <= 220 * 1024;  // N <= ~13.7K (larger N: the ELL kernel)
+    const int Q = N / nu;
+    const int M = cls == CLS_NU1 ? CircCfg<CLS_NU1>::M : (cls == CLS_Q32 ? 32 : CircCfg<CLS_GEN>::M);
+    const int ipr = nu * (cls == CLS_Q32 ? 1 : (Q + M - 1) / M);
+    if (ipr > kCircThreads) return false;  // one item per consumer thread (larger N: the ELL kernel)
+    return circ_smem2(N, cls, 1, 2) <= 220 * 1024;
 }
 
 struct CircPlan {
@@ -331,7 +321,7 @@ static CircPlan circ_plan(int N, int nu) {
     int RT = kCircThreads / ipr;
     if (RT < 1) RT = 1;
     if (RT > 16) RT = 16;
-    // three CTAs per SM (~75 KB each): as many input stages as fit (bytes in flight hide HBM latency)
+    // three CTAs per SM (~75 KB each): as many stages as fit (bytes in flight hide HBM latency)
     const size_t budget = 75 * 1024;
     while (RT > 1 && circ_smem2(N, cls, RT, 3) > budget) --RT;
     int S = 2;
