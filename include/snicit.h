@@ -68,10 +68,15 @@ typedef struct {
     int32_t timing;         /* 1 = record per-phase CUDA-event times for snicit_stats;
                                2 = also one event pair around every pre-convergence layer kernel
                                (snicit_layer_profile) */
-    int32_t ne_interval;    /* host reads the active-residual count every this many post layers
-                               (P:966-970 uses 200) and stops launching residual work at 0;
-                               0 = default (64) */
-    int32_t reserved[4];
+    int32_t ne_interval;    /* per-layer post mode: host reads the active-residual count every this
+                               many post layers (P:966-970 uses 200) and stops launching residual
+                               work at 0; 0 = default (64) */
+    int32_t post_mode;      /* 0 = fused: centroid rows and each residue row carried through all
+                               post-convergence layers in shared memory (2 launches; rows leave when
+                               their residue becomes empty); 1 = per layer: centroid layer + residue
+                               layer + ne_idx row compaction for every layer.  Results are
+                               identical.  N > 24576 always uses the per-layer mode. */
+    int32_t reserved[3];
 } snicit_options;
 
 /* Per-run statistics of the last snicit_infer (times in ms, valid when options.timing). */

@@ -29,7 +29,8 @@ EXPORTED = ["snicit_default_options", "snicit_load_network", "snicit_set_stream"
 class Options(ctypes.Structure):
     _fields_ = [("n_segments", ctypes.c_int32), ("eta", ctypes.c_float), ("eps", ctypes.c_float),
                 ("prune_eps", ctypes.c_float), ("drop_dead_rows", ctypes.c_int32), ("kernel", ctypes.c_int32),
-                ("timing", ctypes.c_int32), ("ne_interval", ctypes.c_int32), ("reserved", ctypes.c_int32 * 4)]
+                ("timing", ctypes.c_int32), ("ne_interval", ctypes.c_int32), ("post_mode", ctypes.c_int32),
+                ("reserved", ctypes.c_int32 * 3)]
 
 
 class Stats(ctypes.Structure):

@@ -295,6 +295,7 @@ static int circ_class(int N, int nu) {
     if (N / nu == 32) return CLS_Q32;
     return CLS_GEN;
 }
+int circ_class_of(int N, int nu) { return circ_class(N, nu); }
 
 bool circ_supported(int N, int K, int nu) {
     if (K != kK || nu <= 0 || N % nu != 0 || N % 4 != 0) return false;

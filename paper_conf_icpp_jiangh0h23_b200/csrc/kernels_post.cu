@@ -1,0 +1,267 @@
+// kernels_post.cu -- fused (multi-layer) post-convergence update, sm_100a.
+//
+// Eq. 5 (Alg. 3) for layers i = t..L-1 in two launches instead of ~3 per layer:
+//
+//  * centroid_traj_kernel: a centroid row evolves by Eq. 1 alone ("If a column in Yhat(i) is a
+//    centroid, then we do not have to consider any errors"), independently of every
+//    residue row.  One CTA per centroid keeps its row in shared memory for all L - t layers and
+//    records the pre-activation a_c of every layer (needed by Eq. 5's second case).
+//  * residual_traj_kernel: every residue row r is independent given a_c of its centroid M(r).  A CTA
+//    takes a row from the non-empty list (ne_idx), keeps it in shared memory and applies
+//    Yhat'_r = sigma((a_c + W.Yhat_r) + b) - sigma(a_c + b) layer after layer; the moment the row
+//    becomes all-zero it leaves (ne_rec false, Alg. 3 lines 12-13).  A zero residue stays zero
+//    (sigma((a_c + 0) + b) - sigma(a_c + b) == 0 exactly, reading R16), so this per-row early exit
+//    returns exactly what per-layer ne_idx compaction returns.
+//
+// Per-layer arithmetic is identical to kernels_circ.cu / kernels_layer.cu (the stored-order fma
+// chain, reading R12), so results are bit-identical to the per-layer path.
+#include <cuda_runtime.h>
+
+#include "snicit_internal.cuh"
+
+namespace snicit {
+
+constexpr int kPostThreads = 256;
+constexpr int kPK = 32;
+constexpr int kPHalo = 64;  // circular halo of each staged row (nu == 1 windows, M + K - 1 = 48)
+
+enum { PCLS_NU1 = 0, PCLS_Q32 = 1, PCLS_GEN = 2 };  // == CircClass of kernels_circ.cu
+
+int post_fused_max_n() { return 24576; }  // 2 rows (+ halo) of shared memory per CTA
+
+template <int MODE>
+__device__ __forceinline__ float post_epi(float acc, float b, const float* ac, int q, float ymax, float prune_eps) {
+    if constexpr (MODE == MODE_RESIDUAL) {
+        const float c = __ldg(ac + q);
+        float v = sigma((c + acc) + b, ymax) - sigma(c + b, ymax);
+        if (prune_eps > 0.0f && fabsf(v) <= prune_eps) v = 0.0f;
+        return v;
+    } else {
+        return sigma(acc + b, ymax);
+    }
+}
+
+// One layer of one row by the whole CTA: in (N + halo floats) -> out.  Returns this thread's
+// "some output != 0".  CENTROID mode also stores acc into aout (if non-NULL).
+template <int MODE, bool UNIF>
+__device__ bool post_row_circ(const PostLayer& Ld, int N, float ymax, float prune_eps, const float* __restrict__ in,
+                              float* __restrict__ out, const float* __restrict__ ac, float* __restrict__ aout) {
+    float w[UNIF ? 1 : kPK];
+    if constexpr (!UNIF) {
+#pragma unroll
+        for (int n = 0; n < kPK; ++n) w[n] = __ldg(Ld.wtab + n);
+    }
+    const float w0 = Ld.w0;
+    const int nu = Ld.nu, Q = N / nu;
+    bool any = false;
+    auto emit = [&](float acc, int q) {
+        const float b = Ld.ubias ? Ld.b0 : __ldg(Ld.bias + q);
+        if constexpr (MODE == MODE_CENTROID) {
+            if (aout) aout[q] = acc;
+        }
+        const float v = post_epi<MODE>(acc, b, ac, q, ymax, prune_eps);
+        out[q] = v;
+        any |= (v != 0.0f);
+    };
+    if (Ld.cls == PCLS_NU1) {
+        constexpr int M = 17, WIN = M + kPK - 1;
+        const int items = (N + M - 1) / M;
+        for (int it = threadIdx.x; it < items; it += blockDim.x) {
+            const int a0 = it * M;
+            float R[WIN];
+#pragma unroll
+            for (int i = 0; i < WIN; ++i) R[i] = in[a0 + i];  // halo: in[N + i] == in[i]
+#pragma unroll
+            for (int m = 0; m < M; ++m) {
+                if (a0 + m < N) {
+                    float acc = 0.0f;
+#pragma unroll
+                    for (int n = 0; n < kPK; ++n) acc = fmaf(R[m + n], UNIF ? w0 : w[n], acc);
+                    emit(acc, a0 + m);
+                }
+            }
+        }
+    } else if (Ld.cls == PCLS_Q32) {
+        for (int c = threadIdx.x; c < nu; c += blockDim.x) {
+            float R[32];
+#pragma unroll
+            for (int j = 0; j < 32; ++j) R[j] = in[j * nu + c];
+#pragma unroll
+            for (int m = 0; m < 32; ++m) {
+                float acc = 0.0f;
+#pragma unroll
+                for (int n = 0; n < kPK; ++n) acc = fmaf(R[(m + n) & 31], UNIF ? w0 : w[n], acc);
+                emit(acc, m * nu + c);
+            }
+        }
+    } else {
+        constexpr int M = 16, WIN = M + kPK - 1;
+        const int items = nu * ((Q + M - 1) / M);
+        for (int it = threadIdx.x; it < items; it += blockDim.x) {
+            const int c = it % nu;
+            const int a0 = (it / nu) * M;
+            float R[WIN];
+#pragma unroll
+            for (int i = 0; i < WIN; ++i) {
+                int ai = a0 + i;  // < 3Q since Q >= K
+                ai = ai >= Q ? ai - Q : ai;
+                ai = ai >= Q ? ai - Q : ai;
+                R[i] = in[ai * nu + c];
+            }
+#pragma unroll
+            for (int m = 0; m < M; ++m) {
+                if (a0 + m < Q) {
+                    float acc = 0.0f;
+#pragma unroll
+                    for (int n = 0; n < kPK; ++n) acc = fmaf(R[m + n], UNIF ? w0 : w[n], acc);
+                    emit(acc, (a0 + m) * nu + c);
+                }
+            }
+        }
+    }
+    return any;
+}
+
+template <int MODE>
+__device__ bool post_row_ell(const PostLayer& Ld, int N, float ymax, float prune_eps, const float* __restrict__ in,
+                             float* __restrict__ out, const float* __restrict__ ac, float* __restrict__ aout) {
+    bool any = false;
+    for (int j = threadIdx.x; j < N; j += blockDim.x) {
+        const int len = Ld.len ? (int)Ld.len[j] : Ld.K;
+        float acc = 0.0f;
+        for (int n = 0; n < len; ++n) {
+            const size_t e = (size_t)n * N + j;
+            const int k = Ld.idx16 ? (int)__ldg(Ld.idx16 + e) : __ldg(Ld.idx32 + e);
+            const float w = Ld.uniform_w ? Ld.w0 : __ldg(Ld.val + e);
+            acc = fmaf(in[k], w, acc);
+        }
+        const float b = Ld.ubias ? Ld.b0 : __ldg(Ld.bias + j);
+        if constexpr (MODE == MODE_CENTROID) {
+            if (aout) aout[j] = acc;
+        }
+        const float v = post_epi<MODE>(acc, b, ac, j, ymax, prune_eps);
+        out[j] = v;
+        any |= (v != 0.0f);
+    }
+    return any;
+}
+
+template <int MODE>
+__device__ __forceinline__ bool post_row_layer(const PostLayer& Ld, int N, float ymax, float prune_eps,
+                                               const float* in, float* out, const float* ac, float* aout,
+                                               int force_ell) {
+    if (Ld.kind == 1 && !force_ell) {
+        if (Ld.uniform_w) return post_row_circ<MODE, true>(Ld, N, ymax, prune_eps, in, out, ac, aout);
+        return post_row_circ<MODE, false>(Ld, N, ymax, prune_eps, in, out, ac, aout);
+    }
+    return post_row_ell<MODE>(Ld, N, ymax, prune_eps, in, out, ac, aout);
+}
+
+__device__ __forceinline__ void stage_row(float* dst, const float* __restrict__ src, int N) {
+    const float4* s4 = reinterpret_cast<const float4*>(src);
+    float4* d4 = reinterpret_cast<float4*>(dst);
+    for (int k = threadIdx.x; k < (N >> 2); k += blockDim.x) d4[k] = s4[k];
+}
+__device__ __forceinline__ void unstage_row(float* dst, const float* src, int N) {
+    const float4* s4 = reinterpret_cast<const float4*>(src);
+    float4* d4 = reinterpret_cast<float4*>(dst);
+    for (int k = threadIdx.x; k < (N >> 2); k += blockDim.x) d4[k] = s4[k];
+}
+__device__ __forceinline__ void fill_halo(float* row, int N) {
+    const int h = min(kPHalo, N);
+    for (int i = threadIdx.x; i < h; i += blockDim.x) row[N + i] = row[i];
+}
+
+__global__ void __launch_bounds__(kPostThreads) centroid_traj_kernel(PostArgs a) {
+    extern __shared__ __align__(128) float sm[];
+    const int C = *a.n_cent;
+    const int c = blockIdx.x;
+    if (c >= C) return;
+    const int N = a.N;
+    const int stride = N + kPHalo;
+    float* cur = sm;
+    float* nxt = sm + stride;
+    stage_row(cur, a.cbuf + (size_t)c * N, N);
+    __syncthreads();
+    fill_halo(cur, N);
+    __syncthreads();
+    for (int l = a.t; l < a.L; ++l) {
+        const PostLayer Ld = a.layers[l];
+        float* aout = a.a_all ? a.a_all + ((size_t)(l - a.t) * a.s + c) * N : nullptr;
+        post_row_layer<MODE_CENTROID>(Ld, N, a.ymax, 0.0f, cur, nxt, nullptr, aout, a.force_ell);
+        __syncthreads();
+        fill_halo(nxt, N);
+        __syncthreads();
+        float* tmp = cur;
+        cur = nxt;
+        nxt = tmp;
+    }
+    unstage_row(a.cbuf + (size_t)c * N, cur, N);
+}
+
+__global__ void __launch_bounds__(kPostThreads) residual_traj_kernel(PostArgs a) {
+    extern __shared__ __align__(128) float sm[];
+    __shared__ int s_p;
+    const int N = a.N;
+    const int stride = N + kPHalo;
+    const int n = *a.rcount;
+    for (;;) {
+        if (threadIdx.x == 0) s_p = atomicAdd(a.work_counter, 1);
+        __syncthreads();
+        const int p = s_p;
+        if (p >= n) break;
+        const int row = a.rlist[p];
+        const int slot = a.cslot[row];
+        float* cur = sm;
+        float* nxt = sm + stride;
+        stage_row(cur, a.yhat + (size_t)row * N, N);
+        __syncthreads();
+        fill_halo(cur, N);
+        __syncthreads();
+        bool alive = true;
+        for (int l = a.t; l < a.L; ++l) {
+            const PostLayer Ld = a.layers[l];
+            const float* ac = a.a_all + ((size_t)(l - a.t) * a.s + slot) * N;
+            const bool any = post_row_layer<MODE_RESIDUAL>(Ld, N, a.ymax, a.prune_eps, cur, nxt, ac, nullptr, a.force_ell);
+            if (!__syncthreads_or(any)) {  // the residue became empty: it stays empty (R16)
+                alive = false;
+                break;
+            }
+            fill_halo(nxt, N);
+            __syncthreads();
+            float* tmp = cur;
+            cur = nxt;
+            nxt = tmp;
+        }
+        if (alive) unstage_row(a.yhat + (size_t)row * N, cur, N);
+        if (threadIdx.x == 0) {
+            a.ne_row[row] = alive ? 1 : 0;
+            if (alive && a.alive_count) atomicAdd(a.alive_count, 1);
+        }
+        __syncthreads();  // s_p and the row buffers are reused
+    }
+}
+
+cudaError_t launch_centroid_traj(const PostArgs& a, int C_max, cudaStream_t st) {
+    if (C_max <= 0) return cudaSuccess;
+    const size_t smem = sizeof(float) * 2 * (size_t)(a.N + kPHalo);
+    int per_sm = 1;
+    cudaError_t e = blocks_per_sm((const void*)centroid_traj_kernel, kPostThreads, smem, &per_sm);
+    if (e != cudaSuccess) return e;
+    centroid_traj_kernel<<<C_max, kPostThreads, smem, st>>>(a);
+    return cudaGetLastError();
+}
+
+cudaError_t launch_residual_traj(const PostArgs& a, int max_rows, int num_sms, cudaStream_t st) {
+    if (max_rows <= 0) return cudaSuccess;
+    const size_t smem = sizeof(float) * 2 * (size_t)(a.N + kPHalo);
+    int per_sm = 1;
+    cudaError_t e = blocks_per_sm((const void*)residual_traj_kernel, kPostThreads, smem, &per_sm);
+    if (e != cudaSuccess) return e;
+    int grid = num_sms * per_sm;
+    if (grid > max_rows) grid = max_rows;
+    residual_traj_kernel<<<grid, kPostThreads, smem, st>>>(a);
+    return cudaGetLastError();
+}
+
+}  // namespace snicit

@@ -59,7 +59,9 @@ struct DevBuf {
 };
 
 // device counters (one int each)
-enum Counter { CNT_LIVE0 = 0, CNT_LIVE1, CNT_RES0, CNT_RES1, CNT_NCENT, CNT_SEFF, CNT_ALL, CNT_NCAT, CNT_N };
+enum Counter {
+    CNT_LIVE0 = 0, CNT_LIVE1, CNT_RES0, CNT_RES1, CNT_NCENT, CNT_SEFF, CNT_ALL, CNT_NCAT, CNT_WORK, CNT_ALIVE, CNT_N
+};
 
 }  // namespace
 
@@ -79,6 +81,8 @@ struct snicit_network {
     DevBuf<uint8_t> len_d;
     DevBuf<float> wtab_d;
     DevBuf<float> bias_d;
+    DevBuf<PostLayer> post_layers_d;  // per-layer descriptors for the fused post-convergence kernels
+    DevBuf<float> a_all;              // [(L - t)][s][N] centroid pre-activations (fused post mode)
     // workspace
     int64_t cap_rows = 0;
     int cap_s = 0, cap_n = 0;
@@ -96,6 +100,8 @@ struct snicit_network {
     int last_s = 0, last_n = 0;
     bool last_converted = false;
     int live_counter = 0;  // which CNT_LIVE* holds the live count at t
+    int res_final_counter = -1;  // counter holding the non-empty residue rows after the last layer
+    bool last_fused = false;
     bool last_kernel_circ = false;
     snicit_stats_t stats{};
     cudaEvent_t ev[6] = {nullptr, nullptr, nullptr, nullptr, nullptr, nullptr};
@@ -117,6 +123,7 @@ void snicit_default_options(snicit_options* opt) {
     opt->kernel = SNICIT_KERNEL_AUTO;
     opt->timing = 0;
     opt->ne_interval = 64;
+    opt->post_mode = 0;
 }
 
 const char* snicit_last_error(void) { return g_last_error.c_str(); }
@@ -147,6 +154,8 @@ void snicit_free_network(snicit_network* net) {
     for (auto& e : net->lev)
         if (e) cudaEventDestroy(e);
     net->hist.release();
+    net->post_layers_d.release();
+    net->a_all.release();
     delete net;
 }
 
@@ -365,6 +374,29 @@ snicit_status snicit_load_network(int32_t N, int32_t L, snicit_format fmt, const
     }
     if (e == cudaSuccess) e = up(net->wtab_d, wtab.data(), wtab.size());
     if (e == cudaSuccess) e = up(net->bias_d, bias, (size_t)L * N);
+    if (e == cudaSuccess) {
+        std::vector<PostLayer> pls(L);
+        for (int l = 0; l < L; ++l) {
+            const LayerPlan& pl = net->plan[l];
+            PostLayer& d = pls[l];
+            memset(&d, 0, sizeof(d));
+            d.kind = pl.kind;
+            d.cls = pl.kind == 1 ? circ_class_of(N, pl.nu) : 0;
+            d.nu = pl.nu;
+            d.K = pl.K;
+            d.uniform_w = pl.uniform ? 1 : 0;
+            d.ubias = pl.ubias ? 1 : 0;
+            d.w0 = pl.w0;
+            d.b0 = bias[(int64_t)l * N];
+            d.bias = net->bias_d.p + (size_t)l * N;
+            d.wtab = (pl.kind == 1 && !pl.uniform) ? net->wtab_d.p + pl.w_off : nullptr;
+            d.idx16 = net->idx16 ? net->idx16_d.p + pl.ell_off : nullptr;
+            d.idx32 = net->idx16 ? nullptr : net->idx32_d.p + pl.ell_off;
+            d.val = pl.uniform ? nullptr : net->val_d.p + pl.ell_off;
+            d.len = pl.ragged ? net->len_d.p + (size_t)l * N : nullptr;
+        }
+        e = up(net->post_layers_d, pls.data(), pls.size());
+    }
     if (e == cudaSuccess) e = net->counters.ensure(CNT_N);
     if (e == cudaSuccess) e = cudaMallocHost(&net->h_counters, sizeof(int) * CNT_N);
     for (int i = 0; i < 6 && e == cudaSuccess; ++i) e = cudaEventCreate(&net->ev[i]);
@@ -472,6 +504,7 @@ snicit_status snicit_infer(snicit_network* net, const float* y0, int64_t batch, 
     if (!(opt.eps >= 0.0f) || std::isnan(opt.eta) || !(opt.prune_eps >= 0.0f))
         return fail(SNICIT_E_INVALID_ARG, "bad eta/eps/prune_eps");
     if (opt.kernel < 0 || opt.kernel > 2) return fail(SNICIT_E_INVALID_ARG, "bad kernel option");
+    if (opt.post_mode < 0 || opt.post_mode > 1) return fail(SNICIT_E_INVALID_ARG, "bad post_mode");
     const int N = net->N, L = net->L;
     if (opt.kernel == SNICIT_KERNEL_CIRC)
         for (int l = 0; l < L; ++l)
@@ -607,7 +640,42 @@ snicit_status snicit_infer(snicit_network* net, const float* y0, int64_t batch, 
         stats.residual_at_t = res_host;
         float* yh_cur = yhat;
         float* yh_nxt = yhat_other;
-        for (int l = tt; l < L; ++l) {
+        const bool fused = opt.post_mode == 0 && N <= post_fused_max_n();
+        net->last_fused = fused;
+        if (fused) {
+            // centroid trajectories (+ a_c per layer when residue rows exist), then residue rows
+            PostArgs pa{};
+            pa.N = N;
+            pa.L = L;
+            pa.t = tt;
+            pa.ymax = net->ymax;
+            pa.prune_eps = opt.prune_eps;
+            pa.layers = net->post_layers_d.p;
+            pa.cbuf = net->cbuf0.p;
+            pa.n_cent = cnt + CNT_NCENT;
+            pa.s = s;
+            if (res_host > 0) {
+                CUDA_TRY(net->a_all.ensure((size_t)(L - tt) * (size_t)s * N));
+                pa.a_all = net->a_all.p;
+            }
+            pa.rlist = rlist;
+            pa.rcount = rcnt;
+            pa.work_counter = cnt + CNT_WORK;
+            pa.yhat = yhat;
+            pa.cslot = net->cslot.p;
+            pa.ne_row = net->ne_row.p;
+            pa.alive_count = cnt + CNT_ALIVE;
+            CUDA_TRY(cudaMemsetAsync(cnt + CNT_WORK, 0, 2 * sizeof(int), st));
+            pa.force_ell = opt.kernel == SNICIT_KERNEL_ELL ? 1 : 0;
+            CUDA_TRY(launch_centroid_traj(pa, s, st));
+            ++launches;
+            for (int l = tt; l < L; ++l) circ_layers += use_circ(net, l, opt.kernel);
+            if (res_host > 0) {
+                CUDA_TRY(launch_residual_traj(pa, res_host, net->num_sms, st));
+                ++launches;
+            }
+        }
+        for (int l = tt; l < L && !fused; ++l) {
             // centroids: Eq. 5 first case, keep a_c
             LayerArgs a = layer_args(net, l, opt.kernel == SNICIT_KERNEL_ELL);
             a.yin = c_cur;
@@ -644,12 +712,9 @@ snicit_status snicit_infer(snicit_network* net, const float* y0, int64_t batch, 
             std::swap(c_cur, c_nxt);
         }
         if (opt.timing) CUDA_TRY(cudaEventRecord(net->ev[3], st));
-        {
-            int rf = 0;
-            const int which = (rcnt == cnt + CNT_RES0) ? CNT_RES0 : CNT_RES1;
-            if (res_host > 0) CUDA_TRY(read_counter(net, which, &rf));
-            stats.residual_final = res_host > 0 ? rf : 0;
-        }
+        net->res_final_counter = -1;
+        if (res_host > 0) net->res_final_counter = fused ? CNT_ALIVE : ((rcnt == cnt + CNT_RES0) ? CNT_RES0 : CNT_RES1);
+        stats.residual_final = 0;
         yfinal = yh_cur;
         cfinal = c_cur;
         // ---- a6: recovery (Eq. 6)
@@ -733,6 +798,10 @@ snicit_status snicit_stats(snicit_network* net, snicit_stats_t* out) {
     net->stats.live_at_t = v;
     CUDA_TRY(read_counter(net, CNT_NCAT, &v));
     net->stats.n_categories = v;
+    if (net->last_converted && net->res_final_counter >= 0) {
+        CUDA_TRY(read_counter(net, net->res_final_counter, &v));
+        net->stats.residual_final = v;
+    }
     if (net->last_converted) {
         CUDA_TRY(read_counter(net, CNT_NCENT, &v));
         net->stats.n_centroids = v;

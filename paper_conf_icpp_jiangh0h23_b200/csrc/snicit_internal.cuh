@@ -132,6 +132,47 @@ cudaError_t launch_layer_circ(const LayerArgs& a, int mode, int max_rows, int nu
 bool circ_supported(int N, int K, int nu);
 bool ell_smem_ok(int N);
 
+// ------------------------------------------------------------------ fused post-convergence (kernels_post.cu)
+// Per-layer descriptor, resident in device memory, read by the multi-layer kernels.
+struct PostLayer {
+    int kind;       // 0 = ELL, 1 = circulant
+    int cls;        // circulant stride class (kernels_circ.cu)
+    int nu, K;
+    int uniform_w;  // 1: all weights == w0
+    int ubias;      // 1: all biases == b0
+    float w0, b0;
+    const float* bias;  // [N]
+    const float* wtab;  // [K] per-n weights (circulant, !uniform_w)
+    const uint16_t* idx16;
+    const int32_t* idx32;
+    const float* val;   // ELL values (n-major) or NULL when uniform
+    const uint8_t* len; // ragged column lengths or NULL
+};
+
+struct PostArgs {
+    int N, L, t;
+    float ymax, prune_eps;
+    int force_ell;            // 1: evaluate every layer with the general (ELL) gather
+    const PostLayer* layers;  // device array [L]
+    // centroid trajectory: rows cbuf[0..C) hold Yhat_c(t) on entry and Yhat_c(L) on exit
+    float* cbuf;
+    const int* n_cent;
+    float* a_all;  // [(L - t)][s][N] pre-activations a_c per post layer, or NULL
+    int s;
+    // residual rows: rlist[0..*rcount) rows of yhat (Yhat_r(t) on entry, Yhat_r(L) on exit if alive)
+    const int* rlist;
+    const int* rcount;
+    int* work_counter;  // zero on entry
+    float* yhat;
+    const int* cslot;
+    uint8_t* ne_row;     // set to the row's final ne (0 once its residue became empty)
+    int* alive_count;    // += 1 per row still non-empty at L (may be NULL)
+};
+int post_fused_max_n();
+cudaError_t launch_centroid_traj(const PostArgs& a, int C_max, cudaStream_t st);
+cudaError_t launch_residual_traj(const PostArgs& a, int max_rows, int num_sms, cudaStream_t st);
+int circ_class_of(int N, int nu);
+
 // kernels_convert.cu
 cudaError_t launch_iota(int* out, int n, int* count_out, cudaStream_t st);
 cudaError_t launch_fill_i32(int* out, int n, int v, cudaStream_t st);

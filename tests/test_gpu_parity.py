@@ -225,3 +225,20 @@ def test_full_size_c2_sampled_rows():
     assert Y.min() >= 0 and Y.max() <= 32
     assert np.array_equal(cats, np.nonzero((Y != 0).any(1))[0])
     assert st["n_categories"] == len(cats)
+
+
+@pytest.mark.parametrize("mode,N,L,B,t", [("radix", 1024, 60, 1500, 2), ("radix", 1024, 60, 1500, 6),
+                                          ("perm", 4096, 20, 300, 3), ("radix", 4096, 40, 400, 4)])
+def test_post_modes_identical(mode, N, L, B, t):
+    """Fused multi-layer post-convergence kernels (default) == per-layer Eq. 5 + ne_idx compaction
+     == the oracle's SNICIT pipeline, bit for bit, with residue rows present."""
+    net = sdgc.gen_network(N, L, mode)
+    Y0 = sdgc.gen_inputs(N, B)
+    ref = oracle.snicit(net, Y0, t=t)
+    a = run_gpu(net, Y0, t=t, post_mode=0)
+    b = run_gpu(net, Y0, t=t, post_mode=1)
+    assert a[2]["residual_at_t"] > 0
+    for Y, cats, st, _ in (a, b):
+        assert np.array_equal(Y, ref["Y"])
+        assert np.array_equal(cats, ref["categories"])
+    assert a[2]["residual_final"] == b[2]["residual_final"] == int((ref["ne"] & (ref["M"] >= 0)).sum())
