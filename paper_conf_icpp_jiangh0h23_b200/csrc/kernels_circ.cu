@@ -66,7 +66,10 @@ __device__ __forceinline__ void consumer_bar() { asm volatile("bar.sync 1, %0;" 
 // Consumers keep their M outputs in registers, meet at a consumer-only named barrier (every read of
 // the stage is done), then overwrite the stage with the outputs, so no separate output buffers are
 // needed and more stages (bytes in flight) fit.  The producer keeps S - 1 tiles of loads ahead.
-template <int MODE, int CLS, bool UNIF, bool UBIAS, int NUCT>
+// PAIR (PLAIN mode): each consumer thread runs its work item on two rows of the tile at once, the
+// two rows' window elements sharing a register pair, so every FMA of the chain is one FFMA2 issue
+// for two outputs (per-lane rounding identical to fmaf).
+template <int MODE, int CLS, bool UNIF, bool UBIAS, int NUCT, bool PAIR>
 __global__ void __launch_bounds__(kCircThreads + 32, (MODE == MODE_PLAIN && UNIF) ? 3 : 2)
     layer_circ_kernel(LayerArgs a, int RT, int S) {
     constexpr int M = CircCfg<CLS>::M;
@@ -86,7 +89,8 @@ __global__ void __launch_bounds__(kCircThreads + 32, (MODE == MODE_PLAIN && UNIF
     constexpr int kConsumerWarps = kCircThreads / 32;
 
     const int chunks = (CLS == CLS_Q32) ? 1 : (Q + M - 1) / M;
-    const int ipr = nu * chunks;  // work items per row (RT * ipr <= kCircThreads by the plan)
+    const int ipr = nu * chunks;  // work items per row (RT / (1 + PAIR) * ipr <= kCircThreads by the plan)
+    constexpr int RPI = PAIR ? 2 : 1;  // rows per work item
     const int count = *a.count;
     const int ntiles = (count + RT - 1) / RT;
     // contiguous tile range per CTA: its row ids are contiguous in the list (prefetchable)
@@ -189,6 +193,107 @@ __global__ void __launch_bounds__(kCircThreads + 32, (MODE == MODE_PLAIN && UNIF
         const int nr = min(RT, count - (t_begin + j) * RT);
         mbar_wait(&in_full[sb], (uint32_t)((j / S) & 1));
         float* st = s_st + (size_t)sb * RT * stride;
+        const int n_items = ((nr + RPI - 1) / RPI) * ipr;
+        if constexpr (PAIR) {
+            // ---------------- two rows per item (rows rr, rr + 1 of the tile), FFMA2 chains
+            float v0[M], v1[M];
+            int rr = 0, obase = 0, ostep = 1, mlim = 0;
+            if (item < n_items) {
+                rr = (item / ipr) * 2;
+                const int rem = item - (item / ipr) * ipr;
+                const float* r0 = st + (size_t)rr * stride;
+                const float* r1 = r0 + stride;  // rr + 1 may be past nr: in-bounds garbage, never stored
+                const unsigned long long W2 = f2_pack(w0, w0);
+                auto finish = [&](unsigned long long acc, int q, float& o0, float& o1) {
+                    const float bq = UBIAS ? b0 : __ldg(a.bias + q);
+                    float z0, z1;
+                    f2_unpack(f2_add(acc, f2_pack(bq, bq)), z0, z1);
+                    o0 = sigma(z0, a.ymax);
+                    o1 = sigma(z1, a.ymax);
+                };
+                if constexpr (CLS == CLS_NU1) {
+                    const int a0 = rem * M;
+                    unsigned long long R[WIN];
+#pragma unroll
+                    for (int i = 0; i < WIN; ++i) R[i] = f2_pack(r0[a0 + i], r1[a0 + i]);
+                    obase = a0;
+                    ostep = 1;
+                    mlim = min(M, N - a0);
+#pragma unroll
+                    for (int m = 0; m < M; ++m) {
+                        unsigned long long acc = 0ull;
+#pragma unroll
+                        for (int n = 0; n < kK; ++n) acc = f2_fma(R[m + n], UNIF ? W2 : f2_pack(w[n], w[n]), acc);
+                        finish(acc, min(a0 + m, N - 1), v0[m], v1[m]);
+                    }
+                } else if constexpr (CLS == CLS_Q32) {
+                    const int c = rem;
+                    unsigned long long R[32];
+#pragma unroll
+                    for (int jj = 0; jj < 32; ++jj) R[jj] = f2_pack(r0[jj * nu + c], r1[jj * nu + c]);
+                    obase = c;
+                    ostep = nu;
+                    mlim = 32;
+#pragma unroll
+                    for (int m = 0; m < 32; ++m) {
+                        unsigned long long acc = 0ull;
+#pragma unroll
+                        for (int n = 0; n < kK; ++n)
+                            acc = f2_fma(R[(m + n) & 31], UNIF ? W2 : f2_pack(w[n], w[n]), acc);
+                        finish(acc, m * nu + c, v0[m], v1[m]);
+                    }
+                } else {  // CLS_GEN
+                    const int c = rem % nu;
+                    const int a0 = (rem / nu) * M;
+                    unsigned long long R[WIN];
+                    if (a0 + WIN <= Q) {
+#pragma unroll
+                        for (int i = 0; i < WIN; ++i) R[i] = f2_pack(r0[(a0 + i) * nu + c], r1[(a0 + i) * nu + c]);
+                    } else {
+#pragma unroll
+                        for (int i = 0; i < WIN; ++i) {
+                            int ai = a0 + i;
+                            ai = ai >= Q ? ai - Q : ai;
+                            ai = ai >= Q ? ai - Q : ai;
+                            R[i] = f2_pack(r0[ai * nu + c], r1[ai * nu + c]);
+                        }
+                    }
+                    obase = a0 * nu + c;
+                    ostep = nu;
+                    mlim = min(M, Q - a0);
+#pragma unroll
+                    for (int m = 0; m < M; ++m) {
+                        unsigned long long acc = 0ull;
+#pragma unroll
+                        for (int n = 0; n < kK; ++n) acc = f2_fma(R[m + n], UNIF ? W2 : f2_pack(w[n], w[n]), acc);
+                        finish(acc, min(a0 + m, Q - 1) * nu + c, v0[m], v1[m]);
+                    }
+                }
+            }
+            consumer_bar();  // every read of this stage is done: overwrite it with the outputs
+            if (item < n_items) {
+                float mx0 = 0.0f, mx1 = 0.0f;
+                float* d0 = st + (size_t)rr * stride + obase;
+                float* d1 = d0 + stride;
+                const bool second = rr + 1 < nr;
+#pragma unroll
+                for (int m = 0; m < M; ++m)
+                    if (mlim == M || m < mlim) {
+                        d0[m * ostep] = v0[m];
+                        mx0 = fmaxf(mx0, fabsf(v0[m]));
+                        if (second) {
+                            d1[m * ostep] = v1[m];
+                            mx1 = fmaxf(mx1, fabsf(v1[m]));
+                        }
+                    }
+                if (mx0 != 0.0f) s_flag[sb * RT + rr] = 1;
+                if (second && mx1 != 0.0f) s_flag[sb * RT + rr + 1] = 1;
+            }
+            fence_proxy_async_smem();
+            __syncwarp();
+            if (lane == 0) mbar_arrive(&out_full[sb]);
+            continue;
+        }
         float v[M];
         int rr = 0, obase = 0, ostep = 1, mlim = 0;
         float mx = 0.0f;
@@ -314,17 +419,18 @@ struct CircPlan {
     size_t smem;
 };
 
-static CircPlan circ_plan(int N, int nu) {
+static CircPlan circ_plan(int N, int nu, bool pair) {
     const int cls = circ_class(N, nu);
     const int Q = N / nu;
     const int M = cls == CLS_NU1 ? CircCfg<CLS_NU1>::M : (cls == CLS_Q32 ? 32 : CircCfg<CLS_GEN>::M);
     const int ipr = nu * (cls == CLS_Q32 ? 1 : (Q + M - 1) / M);
-    int RT = kCircThreads / ipr;
-    if (RT < 1) RT = 1;
+    const int rpi = pair ? 2 : 1;
+    int RT = (kCircThreads / ipr) * rpi;
+    if (RT < rpi) RT = rpi;
     if (RT > 16) RT = 16;
     // three CTAs per SM (~75 KB each): as many stages as fit (bytes in flight hide HBM latency)
     const size_t budget = 75 * 1024;
-    while (RT > 1 && circ_smem2(N, cls, RT, 3) > budget) --RT;
+    while (RT > rpi && circ_smem2(N, cls, RT, 3) > budget) RT -= rpi;
     int S = 2;
     while (S < kMaxStages && circ_smem2(N, cls, RT, S + 1) <= budget) ++S;
     return CircPlan{RT, S, circ_smem2(N, cls, RT, S)};
@@ -332,8 +438,10 @@ static CircPlan circ_plan(int N, int nu) {
 
 template <int MODE, int CLS, bool UNIF, bool UBIAS, int NUCT>
 static cudaError_t launch_circ_t(const LayerArgs& a, int max_rows, int num_sms, cudaStream_t st) {
-    const CircPlan p = circ_plan(a.N, a.nu);
-    auto kern = layer_circ_kernel<MODE, CLS, UNIF, UBIAS, NUCT>;
+    // paired rows where the register budget allows it without spills (nu == 1: the window streams)
+    constexpr bool PAIR = MODE == MODE_PLAIN && UNIF && CLS == CLS_NU1;
+    const CircPlan p = circ_plan(a.N, a.nu, PAIR);
+    auto kern = layer_circ_kernel<MODE, CLS, UNIF, UBIAS, NUCT, PAIR>;
     int per_sm = 1;
     cudaError_t e = blocks_per_sm((const void*)kern, kCircThreads + 32, p.smem, &per_sm);
     if (e != cudaSuccess) return e;
