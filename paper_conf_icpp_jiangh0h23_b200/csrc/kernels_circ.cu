@@ -46,12 +46,18 @@ struct CircCfg<CLS_GEN> {
     static constexpr int M = 16, WIN = M + kK - 1;
 };
 
-__host__ __device__ constexpr int circ_stride(int N, int cls) { return N + (cls == CLS_NU1 ? kHalo : 0); }
+// Circular halo appended to each staged row (a second TMA copy of the row head) so sliding windows
+// never wrap: nu == 1 -> 64 floats; general class -> WIN - 1 = 46 whole a-rows (46 * nu floats) when
+// that is at most the row itself (Q >= 46); Q == 32 class -> none (rotations are compile-time).
+__host__ __device__ constexpr int circ_halo(int N, int cls, int nu) {
+    return cls == CLS_NU1 ? kHalo : (cls == CLS_GEN && 46 * nu <= N && nu % 2 == 0 ? 46 * nu : 0);
+}
+__host__ __device__ constexpr int circ_stride(int N, int cls, int nu) { return N + circ_halo(N, cls, nu); }
 
 constexpr int kMaxStages = 8;
 // Shared-memory layout (per CTA): stage[S][RT][stride] | mbarriers (2S) | row/slot/flag [S][RT]
-__host__ __device__ constexpr size_t circ_smem2(int N, int cls, int RT, int S) {
-    return sizeof(float) * (size_t)S * RT * circ_stride(N, cls) + 2 * (size_t)S * sizeof(uint64_t) +
+__host__ __device__ constexpr size_t circ_smem2(int N, int cls, int nu, int RT, int S) {
+    return sizeof(float) * (size_t)S * RT * circ_stride(N, cls, nu) + 2 * (size_t)S * sizeof(uint64_t) +
            3 * (size_t)S * sizeof(int) * (size_t)RT;
 }
 
@@ -78,7 +84,8 @@ __global__ void __launch_bounds__(kCircThreads + 32, (MODE == MODE_PLAIN && UNIF
     const int N = a.N;
     const int nu = NUCT ? NUCT : a.nu;
     const int Q = N / nu;
-    const int stride = circ_stride(N, CLS);
+    const int halo = circ_halo(N, CLS, nu);
+    const int stride = N + halo;
     float* s_st = reinterpret_cast<float*>(smem);
     uint64_t* bars = reinterpret_cast<uint64_t*>(s_st + (size_t)S * RT * stride);
     uint64_t* in_full = bars;
@@ -132,7 +139,7 @@ __global__ void __launch_bounds__(kCircThreads + 32, (MODE == MODE_PLAIN && UNIF
             const int b = j % S;
             const int r0 = (t_begin + j) * RT;
             const int nr = min(RT, count - r0);
-            const uint32_t bytes = (uint32_t)nr * (uint32_t)(N * 4 + (CLS == CLS_NU1 ? kHalo * 4 : 0));
+            const uint32_t bytes = (uint32_t)nr * (uint32_t)((N + halo) * 4);
             if (lane == 0) mbar_arrive_expect_tx(&in_full[b], bytes);
             for (int i = 0; i < nr; ++i) {
                 const int p = r0 + i - row_base;
@@ -147,7 +154,7 @@ __global__ void __launch_bounds__(kCircThreads + 32, (MODE == MODE_PLAIN && UNIF
                     const float* g = a.yin + (size_t)row * N;
                     float* d = s_st + (size_t)(b * RT + i) * stride;
                     bulk_g2s(d, g, N * 4, &in_full[b]);
-                    if constexpr (CLS == CLS_NU1) bulk_g2s(d + N, g, kHalo * 4, &in_full[b]);  // circular halo
+                    if (halo) bulk_g2s(d + N, g, halo * 4, &in_full[b]);  // circular halo
                 }
             }
         };
@@ -246,7 +253,7 @@ __global__ void __launch_bounds__(kCircThreads + 32, (MODE == MODE_PLAIN && UNIF
                     const int c = rem % nu;
                     const int a0 = (rem / nu) * M;
                     unsigned long long R[WIN];
-                    if (a0 + WIN <= Q) {
+                    if (halo || a0 + WIN <= Q) {
 #pragma unroll
                         for (int i = 0; i < WIN; ++i) R[i] = f2_pack(r0[(a0 + i) * nu + c], r1[(a0 + i) * nu + c]);
                     } else {
@@ -344,7 +351,7 @@ __global__ void __launch_bounds__(kCircThreads + 32, (MODE == MODE_PLAIN && UNIF
                 const int a0 = (rem / nu) * M;
                 const float* src = src0 + c;
                 float R[WIN];
-                if (a0 + WIN <= Q) {  // warp-uniform: lanes share a0
+                if (halo || a0 + WIN <= Q) {  // halo staged, or no wrap (warp-uniform: lanes share a0)
 #pragma unroll
                     for (int i = 0; i < WIN; ++i) R[i] = src[(a0 + i) * nu];
                 } else {
@@ -411,7 +418,7 @@ bool circ_supported(int N, int K, int nu) {
     const int M = cls == CLS_NU1 ? CircCfg<CLS_NU1>::M : (cls == CLS_Q32 ? 32 : CircCfg<CLS_GEN>::M);
     const int ipr = nu * (cls == CLS_Q32 ? 1 : (Q + M - 1) / M);
     if (ipr > kCircThreads) return false;  // one item per consumer thread (larger N: the ELL kernel)
-    return circ_smem2(N, cls, 1, 2) <= 220 * 1024;
+    return circ_smem2(N, cls, nu, 1, 2) <= 220 * 1024;
 }
 
 struct CircPlan {
@@ -430,10 +437,10 @@ static CircPlan circ_plan(int N, int nu, bool pair) {
     if (RT > 16) RT = 16;
     // three CTAs per SM (~75 KB each): as many stages as fit (bytes in flight hide HBM latency)
     const size_t budget = 75 * 1024;
-    while (RT > rpi && circ_smem2(N, cls, RT, 3) > budget) RT -= rpi;
+    while (RT > rpi && circ_smem2(N, cls, nu, RT, 3) > budget) RT -= rpi;
     int S = 2;
-    while (S < kMaxStages && circ_smem2(N, cls, RT, S + 1) <= budget) ++S;
-    return CircPlan{RT, S, circ_smem2(N, cls, RT, S)};
+    while (S < kMaxStages && circ_smem2(N, cls, nu, RT, S + 1) <= budget) ++S;
+    return CircPlan{RT, S, circ_smem2(N, cls, nu, RT, S)};
 }
 
 template <int MODE, int CLS, bool UNIF, bool UBIAS, int NUCT>
@@ -467,7 +474,11 @@ template <int MODE>
 static cudaError_t launch_circ_m(const LayerArgs& a, int max_rows, int num_sms, cudaStream_t st) {
     switch (circ_class(a.N, a.nu)) {
         case CLS_NU1: return launch_circ_wb<MODE, CLS_NU1, 0>(a, max_rows, num_sms, st);
-        case CLS_Q32: return launch_circ_wb<MODE, CLS_Q32, 0>(a, max_rows, num_sms, st);
+        case CLS_Q32:  // compile-time nu for the SDGC strides: immediate shared-memory offsets
+            if (a.nu == 32) return launch_circ_wb<MODE, CLS_Q32, 32>(a, max_rows, num_sms, st);
+            if (a.nu == 128) return launch_circ_wb<MODE, CLS_Q32, 128>(a, max_rows, num_sms, st);
+            if (a.nu == 512) return launch_circ_wb<MODE, CLS_Q32, 512>(a, max_rows, num_sms, st);
+            return launch_circ_wb<MODE, CLS_Q32, 0>(a, max_rows, num_sms, st);
         default:
             if (a.nu == 32) return launch_circ_wb<MODE, CLS_GEN, 32>(a, max_rows, num_sms, st);
             return launch_circ_wb<MODE, CLS_GEN, 0>(a, max_rows, num_sms, st);
