@@ -55,10 +55,11 @@ __host__ __device__ constexpr int circ_halo(int N, int cls, int nu) {
 __host__ __device__ constexpr int circ_stride(int N, int cls, int nu) { return N + circ_halo(N, cls, nu); }
 
 constexpr int kMaxStages = 8;
-// Shared-memory layout (per CTA): stage[S][RT][stride] | mbarriers (2S) | row/slot/flag [S][RT]
+constexpr int kSurvCap = 256;  // per-CTA buffer of surviving row ids (fused dead-row compaction)
+// Shared-memory layout (per CTA): stage[S][RT][stride] | mbarriers (2S) | row/slot/flag [S][RT] | surv[256]
 __host__ __device__ constexpr size_t circ_smem2(int N, int cls, int nu, int RT, int S) {
     return sizeof(float) * (size_t)S * RT * circ_stride(N, cls, nu) + 2 * (size_t)S * sizeof(uint64_t) +
-           3 * (size_t)S * sizeof(int) * (size_t)RT;
+           3 * (size_t)S * sizeof(int) * (size_t)RT + sizeof(int) * kSurvCap;
 }
 
 __device__ __forceinline__ void consumer_bar() { asm volatile("bar.sync 1, %0;" ::"n"(kCircThreads) : "memory"); }
@@ -93,6 +94,7 @@ __global__ void __launch_bounds__(kCircThreads + 32, (MODE == MODE_PLAIN && UNIF
     int* s_row = reinterpret_cast<int*>(bars + 2 * S);
     int* s_slot = s_row + S * RT;
     int* s_flag = s_slot + S * RT;
+    int* s_surv = s_flag + S * RT;
     constexpr int kConsumerWarps = kCircThreads / 32;
 
     const int chunks = (CLS == CLS_Q32) ? 1 : (Q + M - 1) / M;
@@ -118,6 +120,8 @@ __global__ void __launch_bounds__(kCircThreads + 32, (MODE == MODE_PLAIN && UNIF
     if (threadIdx.x >= kCircThreads) {
         // ------------------------------------------------------------ producer / storer warp
         const int lane = threadIdx.x & 31;
+        if (blockIdx.x == 0 && lane == 0 && a.zero_count) *a.zero_count = 0;  // next layer's append counter
+        int nsurv = 0;  // lane 0: surviving rows buffered in s_surv
         const int row_base = t_begin * RT;  // first list position of this CTA
         const int my_rows = min(count, (t_begin + my_tiles) * RT) - row_base;
         // register windows of row ids (and centroid slots): lane l holds local position w0 + l (cur)
@@ -170,17 +174,36 @@ __global__ void __launch_bounds__(kCircThreads + 32, (MODE == MODE_PLAIN && UNIF
                     const uint8_t f = s_flag[b * RT + i] ? 1 : 0;
                     if (a.flag_pos) a.flag_pos[r0 + i] = f;
                     if (a.flag_row) a.flag_row[row] = f;
+                    if (a.app_list && f) s_surv[nsurv++] = row;
                 }
                 bulk_commit();
                 bulk_wait_read0();  // the TMA engine has read the stage: it may be reloaded
             }
             __syncwarp();
         };
+        // append the buffered survivors to the next active list: one atomic per batch (warp-wide copy)
+        auto flush = [&](bool force) {
+            const int n = __shfl_sync(0xffffffffu, nsurv, 0);
+            if (n == 0 || (!force && n <= kSurvCap - RT)) return;
+            int pos = 0;
+            if (lane == 0) pos = atomicAdd(a.app_count, n);
+            pos = __shfl_sync(0xffffffffu, pos, 0);
+            for (int i = lane; i < n; i += 32) a.app_list[pos + i] = s_surv[i];
+            __syncwarp();
+            nsurv = 0;
+        };
         for (int j = 0; j < my_tiles; ++j) {
-            if (j >= S) store(j - S);
+            if (j >= S) {
+                store(j - S);
+                if (a.app_list) flush(false);
+            }
             load(j);
         }
-        for (int j = max(0, my_tiles - S); j < my_tiles; ++j) store(j);
+        for (int j = max(0, my_tiles - S); j < my_tiles; ++j) {
+            store(j);
+            if (a.app_list) flush(false);
+        }
+        if (a.app_list) flush(true);
         if (lane == 0) bulk_wait0();
         return;
     }

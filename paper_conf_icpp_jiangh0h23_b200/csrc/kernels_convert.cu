@@ -8,6 +8,7 @@
 //                       Alg. 2
 //  recover_kernel       final results recovery (Eq. 6) + category flags (R13)
 #include <cuda_runtime.h>
+#include <string.h>
 
 #include "snicit_internal.cuh"
 
@@ -81,53 +82,111 @@ cudaError_t launch_row_nonzero(const float* y, int N, const int* rows, const int
 }
 
 // ------------------------------------------------------------------------------ compaction
-// Order-preserving stream compaction of list_in by flag_pos (indexed by list position), one CTA:
-// each thread owns a contiguous segment, counts its survivors, block-wide exclusive scan (warp
-// shuffles + one shared-memory pass), then scatters.  ne_idx "sorted indices of ne_rec == true"
-// is thereby rebuilt on device every layer instead of by the paper's serial host loop
-// -- result-neutral by reading R16.
-constexpr int kCompactThreads = 1024;
-__global__ void __launch_bounds__(kCompactThreads) compact_kernel(const int* __restrict__ list_in,
-                                                                  const int* count_in,
-                                                                  const uint8_t* __restrict__ flag_pos,
-                                                                  int* __restrict__ list_out, int* count_out) {
-    __shared__ int warp_sums[32];
-    const int n = *count_in;
-    const int per = (n + kCompactThreads - 1) / kCompactThreads;
-    const int beg = min(n, (int)threadIdx.x * per);
-    const int end = min(n, beg + per);
+// Order-preserving stream compaction (ne_idx "sorted indices of ne_rec == true", rebuilt
+// on device instead of the paper's serial host loop):
+//   out = [list_in[i] for i < *count_in if flag_pos[i]]      (list_in NULL: the identity)
+// Two launches over chunks of kChunk positions: per-chunk counts, then each chunk sums the counts
+// before it (<= a few hundred), scans its own flags (16 per thread, 16-byte loads) and scatters.
+constexpr int kCompactThreads = 256;
+constexpr int kChunk = kCompactThreads * 16;
+
+__device__ __forceinline__ int popc_bytes(uint4 v) {
+    // number of non-zero bytes among 16
     int c = 0;
-    for (int i = beg; i < end; ++i) c += flag_pos[i] ? 1 : 0;
+    const uint32_t w[4] = {v.x, v.y, v.z, v.w};
+#pragma unroll
+    for (int i = 0; i < 4; ++i) {
+        const uint32_t x = w[i];
+        const uint32_t nz = ((x & 0x7f7f7f7fu) + 0x7f7f7f7fu | x) & 0x80808080u;  // high bit per non-zero byte
+        c += __popc(nz);
+    }
+    return c;
+}
+
+__device__ __forceinline__ uint4 load_flags16(const uint8_t* f, int base, int n) {
+    if (base + 16 <= n && (reinterpret_cast<uintptr_t>(f + base) & 15) == 0)
+        return *reinterpret_cast<const uint4*>(f + base);
+    uint8_t b[16];
+#pragma unroll
+    for (int i = 0; i < 16; ++i) b[i] = (base + i < n) ? f[base + i] : 0;
+    uint4 v;
+    memcpy(&v, b, 16);
+    return v;
+}
+
+__global__ void __launch_bounds__(kCompactThreads) compact_count_kernel(const int* count_in,
+                                                                        const uint8_t* __restrict__ flag_pos,
+                                                                        int* block_counts) {
+    const int n = *count_in;
+    const int base = blockIdx.x * kChunk + threadIdx.x * 16;
+    int c = base < n ? popc_bytes(load_flags16(flag_pos, base, n)) : 0;
+#pragma unroll
+    for (int o = 16; o > 0; o >>= 1) c += __shfl_down_sync(0xffffffffu, c, o);
+    __shared__ int ws[kCompactThreads / 32];
+    if ((threadIdx.x & 31) == 0) ws[threadIdx.x >> 5] = c;
+    __syncthreads();
+    if (threadIdx.x == 0) {
+        int t = 0;
+        for (int w = 0; w < kCompactThreads / 32; ++w) t += ws[w];
+        block_counts[blockIdx.x] = t;
+    }
+}
+
+__global__ void __launch_bounds__(kCompactThreads) compact_scatter_kernel(const int* __restrict__ list_in,
+                                                                          const int* count_in,
+                                                                          const uint8_t* __restrict__ flag_pos,
+                                                                          const int* block_counts,
+                                                                          int* __restrict__ list_out,
+                                                                          int* count_out) {
+    const int n = *count_in;
+    const int nblk = (n + kChunk - 1) / kChunk;
+    __shared__ int s_prefix, s_ws[kCompactThreads / 32];
+    if ((int)blockIdx.x >= max(nblk, 1)) return;
+    if (threadIdx.x < 32) {  // exclusive prefix of the chunks before this one
+        int p = 0;
+        for (int b = threadIdx.x; b < (int)blockIdx.x; b += 32) p += block_counts[b];
+#pragma unroll
+        for (int o = 16; o > 0; o >>= 1) p += __shfl_down_sync(0xffffffffu, p, o);
+        if (threadIdx.x == 0) s_prefix = p;
+    }
+    const int base = blockIdx.x * kChunk + threadIdx.x * 16;
+    const uint4 v = base < n ? load_flags16(flag_pos, base, n) : make_uint4(0, 0, 0, 0);
+    const int c = popc_bytes(v);
     const int lane = threadIdx.x & 31, wid = threadIdx.x >> 5;
     int incl = c;
 #pragma unroll
     for (int o = 1; o < 32; o <<= 1) {
-        const int v = __shfl_up_sync(0xffffffffu, incl, o);
-        if (lane >= o) incl += v;
+        const int t = __shfl_up_sync(0xffffffffu, incl, o);
+        if (lane >= o) incl += t;
     }
-    if (lane == 31) warp_sums[wid] = incl;
+    if (lane == 31) s_ws[wid] = incl;
     __syncthreads();
-    if (wid == 0) {
-        int ws = warp_sums[lane];
-        int wi = ws;
+    int woff = 0, total = 0;
+    for (int w = 0; w < kCompactThreads / 32; ++w) {
+        const int t = s_ws[w];
+        if (w < wid) woff += t;
+        total += t;
+    }
+    int pos = s_prefix + woff + incl - c;
+    uint8_t bytes[16];
+    memcpy(bytes, &v, 16);
 #pragma unroll
-        for (int o = 1; o < 32; o <<= 1) {
-            const int v = __shfl_up_sync(0xffffffffu, wi, o);
-            if (lane >= o) wi += v;
-        }
-        warp_sums[lane] = wi - ws;  // exclusive warp offsets
-        if (lane == 31) *count_out = wi;
-    }
-    __syncthreads();
-    int pos = warp_sums[wid] + incl - c;
-    for (int i = beg; i < end; ++i)
-        if (flag_pos[i]) list_out[pos++] = list_in[i];
+    for (int i = 0; i < 16; ++i)
+        if (bytes[i]) list_out[pos++] = list_in ? list_in[base + i] : base + i;
+    if ((int)blockIdx.x == max(nblk, 1) - 1 && threadIdx.x == 0) *count_out = s_prefix + total;
 }
+
 cudaError_t launch_compact(const int* list_in, const int* count_in, const uint8_t* flag_pos, int* list_out,
-                           int* count_out, int /*max_n*/, cudaStream_t st) {
-    compact_kernel<<<1, kCompactThreads, 0, st>>>(list_in, count_in, flag_pos, list_out, count_out);
+                           int* count_out, int max_n, int* scratch, cudaStream_t st) {
+    const int nblk = max(1, (max_n + kChunk - 1) / kChunk);
+    compact_count_kernel<<<nblk, kCompactThreads, 0, st>>>(count_in, flag_pos, scratch);
+    cudaError_t e = cudaGetLastError();
+    if (e != cudaSuccess) return e;
+    compact_scatter_kernel<<<nblk, kCompactThreads, 0, st>>>(list_in, count_in, flag_pos, scratch, list_out,
+                                                              count_out);
     return cudaGetLastError();
 }
+int compact_scratch_ints(int max_n) { return max(1, (max_n + kChunk - 1) / kChunk); }
 
 // ------------------------------------------------------------------------------ conversion
 // Sum downsampling: block (g, q) sums segment g of sampled row q ("first s columns", of

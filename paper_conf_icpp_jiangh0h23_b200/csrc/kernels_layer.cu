@@ -64,6 +64,21 @@ cudaError_t blocks_per_sm(const void* kern, int threads, size_t smem, int* out) 
 constexpr int kEllThreads = 512;
 
 // ------------------------------------------------------------------------------ ELL (general)
+constexpr int kEllSurvCap = 256;
+// block-wide: append the buffered surviving rows to the next active list (one atomic per batch)
+__device__ __forceinline__ void ell_flush(const LayerArgs& a, const int* s_surv, int* s_nsurv, int* s_pos) {
+    __syncthreads();
+    const int n = *s_nsurv;
+    if (n > 0) {
+        if (threadIdx.x == 0) *s_pos = atomicAdd(a.app_count, n);
+        __syncthreads();
+        const int pos = *s_pos;
+        for (int i = threadIdx.x; i < n; i += blockDim.x) a.app_list[pos + i] = s_surv[i];
+    }
+    __syncthreads();
+    if (threadIdx.x == 0) *s_nsurv = 0;
+    __syncthreads();
+}
 template <int MODE, int RT, bool IDX16, bool UNIF, bool RAGGED, bool SMEM>
 __global__ void __launch_bounds__(kEllThreads, 1) layer_ell_kernel(LayerArgs a) {
     extern __shared__ __align__(128) unsigned char smem[];
@@ -73,7 +88,11 @@ __global__ void __launch_bounds__(kEllThreads, 1) layer_ell_kernel(LayerArgs a) 
     int* s_flag = reinterpret_cast<int*>(bar + 1);
     int* s_row = s_flag + RT;
     int* s_slot = s_row + RT;
+    int* s_surv = s_slot + RT;  // kEllSurvCap surviving row ids (fused dead-row compaction)
+    __shared__ int s_nsurv, s_pos;
 
+    if (blockIdx.x == 0 && threadIdx.x == 0 && a.zero_count) *a.zero_count = 0;
+    if (threadIdx.x == 0) s_nsurv = 0;
     const int count = *a.count;
     const int ntiles = (count + RT - 1) / RT;
     if (SMEM && threadIdx.x == 0) {
@@ -138,15 +157,21 @@ __global__ void __launch_bounds__(kEllThreads, 1) layer_ell_kernel(LayerArgs a) 
             if (a.flag_pos) a.flag_pos[r0 + threadIdx.x] = f;
             if (a.flag_row) a.flag_row[s_row[threadIdx.x]] = f;
         }
+        if (a.app_list && threadIdx.x == 0) {
+            for (int i = 0; i < nr; ++i)
+                if (s_flag[i]) s_surv[s_nsurv++] = s_row[i];
+        }
         __syncthreads();
+        if (a.app_list && s_nsurv > kEllSurvCap - RT) ell_flush(a, s_surv, &s_nsurv, &s_pos);
     }
+    if (a.app_list) ell_flush(a, s_surv, &s_nsurv, &s_pos);
 }
 
 bool ell_smem_ok(int N) { return (size_t)N * 4 * 2 <= 200 * 1024 && N % 4 == 0; }
 
 template <int MODE, int RT, bool SMEM>
 static cudaError_t launch_ell_t(const LayerArgs& a, int max_rows, int num_sms, cudaStream_t st) {
-    const size_t smem = (SMEM ? (size_t)RT * a.N * 4 : 0) + 16 + 12 * RT + 16;
+    const size_t smem = (SMEM ? (size_t)RT * a.N * 4 : 0) + 16 + 12 * RT + 16 + 4 * kEllSurvCap;
     const bool i16 = a.idx16 != nullptr, unif = a.val == nullptr, rag = a.len != nullptr;
     void (*kern)(LayerArgs) = nullptr;
 #define SNICIT_PICK(I, U, G) \

@@ -60,7 +60,8 @@ struct DevBuf {
 
 // device counters (one int each)
 enum Counter {
-    CNT_LIVE0 = 0, CNT_LIVE1, CNT_RES0, CNT_RES1, CNT_NCENT, CNT_SEFF, CNT_ALL, CNT_NCAT, CNT_WORK, CNT_ALIVE, CNT_N
+    CNT_LIVE0 = 0, CNT_LIVE1, CNT_LIVE2, CNT_ORD, CNT_RES0, CNT_RES1, CNT_NCENT, CNT_SEFF, CNT_ALL, CNT_NCAT,
+    CNT_WORK, CNT_ALIVE, CNT_N
 };
 
 }  // namespace
@@ -90,6 +91,7 @@ struct snicit_network {
     DevBuf<int> list0, list1, res0, res1, M, cslot, catlist, cent, col_idx, iota_s;
     DevBuf<uint8_t> flag_pos, live_row, ne_row, cat, ne_t;
     DevBuf<float> cbuf0, cbuf1, ac;
+    DevBuf<int> cscratch;  // per-chunk counts of the ordered compaction
     DevBuf<double> F;
     DevBuf<int> counters;
     int* h_counters = nullptr;  // pinned mirror
@@ -146,6 +148,7 @@ void snicit_free_network(snicit_network* net) {
     for (auto* b : {&net->flag_pos, &net->live_row, &net->ne_row, &net->cat, &net->ne_t}) b->release();
     net->cbuf0.release();
     net->cbuf1.release();
+    net->cscratch.release();
     net->ac.release();
     net->F.release();
     if (net->h_counters) cudaFreeHost(net->h_counters);
@@ -471,6 +474,7 @@ static cudaError_t ensure_workspace(snicit_network* net, int64_t R, int s, int n
     if ((e = net->col_idx.ensure(ss)) != cudaSuccess) return e;
     if ((e = net->iota_s.ensure(ss)) != cudaSuccess) return e;
     if ((e = net->F.ensure((size_t)std::max(n, 1) * ss)) != cudaSuccess) return e;
+    if ((e = net->cscratch.ensure((size_t)compact_scratch_ints((int)rows))) != cudaSuccess) return e;
     return cudaSuccess;
 }
 
@@ -537,20 +541,24 @@ snicit_status snicit_infer(snicit_network* net, const float* y0, int64_t batch, 
         nxt_i = 1;
     }
     int* cnt = net->counters.p;
-    int* list_cur = net->list0.p;
-    int* list_nxt = net->list1.p;
-    int* cnt_cur = cnt + CNT_LIVE0;
-    int* cnt_nxt = cnt + CNT_LIVE1;
-    CUDA_TRY(launch_iota(list_cur, R, cnt_cur, st));
-    ++launches;
+    int* scratch = net->cscratch.p;
+    int* lists[2] = {net->list0.p, net->list1.p};
+    int li = 0;                                         // lists[li] is the active-row list
+    const int live_ctr[3] = {CNT_LIVE0, CNT_LIVE1, CNT_LIVE2};
+    int ci = 0;                                         // cnt + live_ctr[ci] is its length
+    CUDA_TRY(launch_iota(lists[0], R, cnt + CNT_LIVE0, st));
+    CUDA_TRY(cudaMemsetAsync(cnt + CNT_LIVE1, 0, sizeof(int), st));
+    launches += 1;
     const bool drop = opt.drop_dead_rows != 0;
     // zero input rows are dead only when the conversion happens at t = 0 (otherwise layer 0 drops them)
     if (drop && net->dead_ok[0] && tt == 0 && R > 0) {
-        CUDA_TRY(launch_row_nonzero(cur, N, list_cur, cnt_cur, net->flag_pos.p, R, net->num_sms, st));
-        CUDA_TRY(launch_compact(list_cur, cnt_cur, net->flag_pos.p, list_nxt, cnt_nxt, R, st));
-        launches += 2;
-        std::swap(list_cur, list_nxt);
-        std::swap(cnt_cur, cnt_nxt);
+        CUDA_TRY(launch_row_nonzero(cur, N, lists[li], cnt + live_ctr[ci], net->flag_pos.p, R, net->num_sms, st));
+        CUDA_TRY(launch_compact(lists[li], cnt + live_ctr[ci], net->flag_pos.p, lists[li ^ 1],
+                                cnt + live_ctr[(ci + 1) % 3], R, scratch, st));
+        launches += 3;
+        CUDA_TRY(cudaMemsetAsync(cnt + live_ctr[(ci + 2) % 3], 0, sizeof(int), st));
+        li ^= 1;
+        ci = (ci + 1) % 3;
     }
     // ---- a1: pre-convergence layers, Eq. 1 for i = 0..t-1
     const bool prof = opt.timing >= 2;
@@ -566,17 +574,24 @@ snicit_status snicit_infer(snicit_network* net, const float* y0, int64_t batch, 
         net->prof_layers = 0;
     }
     for (int l = 0; l < tt; ++l) {
+        // exact dead-row compaction (R23) fused into the layer: rows with a non-zero output are
+        // appended (unordered) to the other list; the append counter of the NEXT dropping layer is
+        // zeroed by this one (rotating counters), so no extra launch is needed
         const bool drop_now = drop && net->dead_ok[l + 1];
         if (prof) {
-            CUDA_TRY(cudaMemcpyAsync(net->hist.p + l, cnt_cur, sizeof(int), cudaMemcpyDeviceToDevice, st));
+            CUDA_TRY(cudaMemcpyAsync(net->hist.p + l, cnt + live_ctr[ci], sizeof(int), cudaMemcpyDeviceToDevice, st));
             CUDA_TRY(cudaEventRecord(net->lev[2 * l], st));
         }
         LayerArgs a = layer_args(net, l, opt.kernel == SNICIT_KERNEL_ELL);
         a.yin = cur;
         a.yout = bufs[nxt_i];
-        a.rows = list_cur;
-        a.count = cnt_cur;
-        a.flag_pos = drop_now ? net->flag_pos.p : nullptr;
+        a.rows = lists[li];
+        a.count = cnt + live_ctr[ci];
+        if (drop_now) {
+            a.app_list = lists[li ^ 1];
+            a.app_count = cnt + live_ctr[(ci + 1) % 3];
+            a.zero_count = cnt + live_ctr[(ci + 2) % 3];
+        }
         CUDA_TRY(run_layer(net, l, opt.kernel, MODE_PLAIN, a, R));
         if (prof) CUDA_TRY(cudaEventRecord(net->lev[2 * l + 1], st));
         ++launches;
@@ -585,17 +600,19 @@ snicit_status snicit_infer(snicit_network* net, const float* y0, int64_t batch, 
         cur = bufs[nxt_i];
         nxt_i ^= 1;
         if (drop_now) {
-            CUDA_TRY(launch_compact(list_cur, cnt_cur, net->flag_pos.p, list_nxt, cnt_nxt, R, st));
-            ++launches;
-            std::swap(list_cur, list_nxt);
-            std::swap(cnt_cur, cnt_nxt);
+            li ^= 1;
+            ci = (ci + 1) % 3;
         }
     }
+    int* list_cur = lists[li];
+    int* cnt_cur = cnt + live_ctr[ci];
+    int* list_nxt = lists[li ^ 1];
     if (opt.timing) CUDA_TRY(cudaEventRecord(net->ev[1], st));
-    // live flags at t (for recovery of the plain path and the debug hook)
+    // live flags at t (recovery of the plain path, ordered live list, debug hook)
     CUDA_TRY(launch_fill_u8(net->live_row.p, R, 0, st));
     CUDA_TRY(launch_mark_rows(list_cur, cnt_cur, net->live_row.p, R, st));
-    launches += 2;
+    CUDA_TRY(launch_fill_i32(cnt + CNT_ALL, 1, R, st));
+    launches += 3;
 
     float* y_dst = y_out_on_device ? y_out : nullptr;
     const float* yfinal = cur;
@@ -612,6 +629,11 @@ snicit_status snicit_infer(snicit_network* net, const float* y0, int64_t batch, 
                                 net->cat.p, net->num_sms, st));
         ++launches;
     } else {
+        // ordered live list: "the first s columns" are the first s live rows by id (R14)
+        CUDA_TRY(launch_compact(nullptr, cnt + CNT_ALL, net->live_row.p, list_nxt, cnt + CNT_ORD, R, scratch, st));
+        launches += 2;
+        list_cur = list_nxt;
+        cnt_cur = cnt + CNT_ORD;
         // ---- a2/a3: sampling + sum downsampling + Alg. 1 pruning -> y*
         CUDA_TRY(launch_downsample(cur, N, list_cur, cnt_cur, s, n_seg, net->F.p, st));
         CUDA_TRY(launch_prune(net->F.p, cnt_cur, s, n_seg, opt.eta, opt.eps, list_cur, net->cent.p, cnt + CNT_NCENT,
@@ -627,7 +649,7 @@ snicit_status snicit_infer(snicit_network* net, const float* y0, int64_t batch, 
         int* rlist_nxt = net->res1.p;
         int* rcnt = cnt + CNT_RES0;
         int* rcnt_nxt = cnt + CNT_RES1;
-        CUDA_TRY(launch_compact(list_cur, cnt_cur, net->flag_pos.p, rlist, rcnt, R, st));
+        CUDA_TRY(launch_compact(list_cur, cnt_cur, net->flag_pos.p, rlist, rcnt, R, scratch, st));
         CUDA_TRY(launch_iota(net->iota_s.p, s, nullptr, st));
         CUDA_TRY(cudaMemcpyAsync(net->ne_t.p, net->ne_row.p, (size_t)R, cudaMemcpyDeviceToDevice, st));
         launches += 7;
@@ -699,7 +721,7 @@ snicit_status snicit_infer(snicit_network* net, const float* y0, int64_t batch, 
                 b.flag_row = net->ne_row.p;
                 b.prune_eps = opt.prune_eps;
                 CUDA_TRY(run_layer(net, l, opt.kernel, MODE_RESIDUAL, b, R));
-                CUDA_TRY(launch_compact(rlist, rcnt, net->flag_pos.p, rlist_nxt, rcnt_nxt, R, st));
+                CUDA_TRY(launch_compact(rlist, rcnt, net->flag_pos.p, rlist_nxt, rcnt_nxt, R, scratch, st));
                 launches += 2;
                 std::swap(rlist, rlist_nxt);
                 std::swap(rcnt, rcnt_nxt);
@@ -723,10 +745,8 @@ snicit_status snicit_infer(snicit_network* net, const float* y0, int64_t batch, 
                                 net->cat.p, net->num_sms, st));
         ++launches;
     }
-    // categories: ordered compaction of cat flags over all rows
-    CUDA_TRY(launch_iota(net->list1.p == list_cur ? net->list0.p : net->list1.p, R, cnt + CNT_ALL, st));
-    CUDA_TRY(launch_compact(net->list1.p == list_cur ? net->list0.p : net->list1.p, cnt + CNT_ALL, net->cat.p,
-                            net->catlist.p, cnt + CNT_NCAT, R, st));
+    // categories: ordered compaction of the cat flags over all rows (R13)
+    CUDA_TRY(launch_compact(nullptr, cnt + CNT_ALL, net->cat.p, net->catlist.p, cnt + CNT_NCAT, R, scratch, st));
     launches += 2;
     if (opt.timing) CUDA_TRY(cudaEventRecord(net->ev[4], st));
     if (!y_out_on_device && y_out && R > 0)
@@ -745,7 +765,7 @@ snicit_status snicit_infer(snicit_network* net, const float* y0, int64_t batch, 
         net->stats.t_pre_ms = net->stats.t_convert_ms = net->stats.t_post_ms = net->stats.t_recover_ms = -1.0;
         net->stats.t_total_ms = -1.0;
     }
-    net->live_counter = (cnt_cur == cnt + CNT_LIVE0) ? CNT_LIVE0 : CNT_LIVE1;
+    net->live_counter = live_ctr[ci];
     if (opt.timing) {
         CUDA_TRY(cudaEventSynchronize(net->ev[5]));
         float ms;

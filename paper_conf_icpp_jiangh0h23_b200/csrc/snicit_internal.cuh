@@ -104,6 +104,9 @@ struct LayerArgs {
     float ymax;
     uint8_t* flag_pos;      // nullable: any-non-zero of the row, indexed by list position
     uint8_t* flag_row;      // nullable: same, indexed by row id
+    int* app_list;          // nullable: rows with a non-zero output are appended here (unordered)
+    int* app_count;         //   ... at atomicAdd(app_count, n) (zero on entry)
+    int* zero_count;        // nullable: set to 0 by the kernel (rotating append counters)
     float* a_out;           // CENTROID: a_c [row][N]
     const float* a_c;       // RESIDUAL: a_c [slot][N]
     const int* cslot;       // RESIDUAL: centroid slot of each row id
@@ -204,7 +207,8 @@ cudaError_t launch_fill_u8(uint8_t* out, int n, uint8_t v, cudaStream_t st);
 cudaError_t launch_row_nonzero(const float* y, int N, const int* rows, const int* count, uint8_t* flag_pos,
                                int max_rows, int num_sms, cudaStream_t st);
 cudaError_t launch_compact(const int* list_in, const int* count_in, const uint8_t* flag_pos, int* list_out,
-                           int* count_out, int max_n, cudaStream_t st);
+                           int* count_out, int max_n, int* scratch, cudaStream_t st);
+int compact_scratch_ints(int max_n);
 cudaError_t launch_downsample(const float* y, int N, const int* rows, const int* count, int s, int n_seg,
                               double* F, cudaStream_t st);
 cudaError_t launch_prune(const double* F, const int* count, int s, int n_seg, float eta, float eps,
