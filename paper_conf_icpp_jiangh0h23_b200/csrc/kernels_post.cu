@@ -43,7 +43,10 @@ __device__ __forceinline__ float post_epi(float acc, float b, const float* ac, i
 
 // One layer of one row by the whole CTA: in (N + halo floats) -> out.  Returns this thread's
 // "some output != 0".  CENTROID mode also stores acc into aout (if non-NULL).
-template <int MODE, bool UNIF>
+// MNU1 / MGEN: outputs per work item of the nu == 1 / general classes; QG: threads per residue class
+// of the Q == 32 class (32 / QG outputs each).  Small values -> more, shorter items (latency-bound
+// centroid trajectory on one SM); large -> fewer shared-memory loads per FMA (throughput).
+template <int MODE, bool UNIF, int MNU1, int MGEN, int QG>
 __device__ bool post_row_circ(const PostLayer& Ld, int N, float ymax, float prune_eps, const float* __restrict__ in,
                               float* __restrict__ out, const float* __restrict__ ac, float* __restrict__ aout) {
     float w[UNIF ? 1 : kPK];
@@ -64,7 +67,7 @@ __device__ bool post_row_circ(const PostLayer& Ld, int N, float ymax, float prun
         any |= (v != 0.0f);
     };
     if (Ld.cls == PCLS_NU1) {
-        constexpr int M = 17, WIN = M + kPK - 1;
+        constexpr int M = MNU1, WIN = M + kPK - 1;
         const int items = (N + M - 1) / M;
         for (int it = threadIdx.x; it < items; it += blockDim.x) {
             const int a0 = it * M;
@@ -82,12 +85,16 @@ __device__ bool post_row_circ(const PostLayer& Ld, int N, float ymax, float prun
             }
         }
     } else if (Ld.cls == PCLS_Q32) {
-        for (int c = threadIdx.x; c < nu; c += blockDim.x) {
+        constexpr int OG = 32 / QG;  // outputs per item
+        for (int it = threadIdx.x; it < nu * QG; it += blockDim.x) {
+            const int c = it % nu;
+            const int g = it / nu;  // output group: a = g*OG .. g*OG + OG - 1
             float R[32];
 #pragma unroll
             for (int j = 0; j < 32; ++j) R[j] = in[j * nu + c];
 #pragma unroll
-            for (int m = 0; m < 32; ++m) {
+            for (int mm = 0; mm < OG; ++mm) {
+                const int m = g * OG + mm;
                 float acc = 0.0f;
 #pragma unroll
                 for (int n = 0; n < kPK; ++n) acc = fmaf(R[(m + n) & 31], UNIF ? w0 : w[n], acc);
@@ -95,7 +102,7 @@ __device__ bool post_row_circ(const PostLayer& Ld, int N, float ymax, float prun
             }
         }
     } else {
-        constexpr int M = 16, WIN = M + kPK - 1;
+        constexpr int M = MGEN, WIN = M + kPK - 1;
         const int items = nu * ((Q + M - 1) / M);
         for (int it = threadIdx.x; it < items; it += blockDim.x) {
             const int c = it % nu;
@@ -146,13 +153,14 @@ __device__ bool post_row_ell(const PostLayer& Ld, int N, float ymax, float prune
     return any;
 }
 
-template <int MODE>
+template <int MODE, int MNU1, int MGEN, int QG>
 __device__ __forceinline__ bool post_row_layer(const PostLayer& Ld, int N, float ymax, float prune_eps,
                                                const float* in, float* out, const float* ac, float* aout,
                                                int force_ell) {
     if (Ld.kind == 1 && !force_ell) {
-        if (Ld.uniform_w) return post_row_circ<MODE, true>(Ld, N, ymax, prune_eps, in, out, ac, aout);
-        return post_row_circ<MODE, false>(Ld, N, ymax, prune_eps, in, out, ac, aout);
+        if (Ld.uniform_w)
+            return post_row_circ<MODE, true, MNU1, MGEN, QG>(Ld, N, ymax, prune_eps, in, out, ac, aout);
+        return post_row_circ<MODE, false, MNU1, MGEN, QG>(Ld, N, ymax, prune_eps, in, out, ac, aout);
     }
     return post_row_ell<MODE>(Ld, N, ymax, prune_eps, in, out, ac, aout);
 }
@@ -172,7 +180,11 @@ __device__ __forceinline__ void fill_halo(float* row, int N) {
     for (int i = threadIdx.x; i < h; i += blockDim.x) row[N + i] = row[i];
 }
 
-__global__ void __launch_bounds__(kPostThreads) centroid_traj_kernel(PostArgs a) {
+constexpr int kCentThreads = 1024;
+// One CTA (1024 threads) per centroid row; items of 4 outputs (nu == 1, general) or 4 per residue
+// class (Q == 32) so the whole SM works on every layer; the next layer's descriptor is loaded while
+// the current layer computes (it is on the serial critical path otherwise).
+__global__ void __launch_bounds__(kCentThreads) centroid_traj_kernel(PostArgs a) {
     extern __shared__ __align__(128) float sm[];
     const int C = *a.n_cent;
     const int c = blockIdx.x;
@@ -185,16 +197,18 @@ __global__ void __launch_bounds__(kPostThreads) centroid_traj_kernel(PostArgs a)
     __syncthreads();
     fill_halo(cur, N);
     __syncthreads();
+    PostLayer Ld = a.layers[a.t];
     for (int l = a.t; l < a.L; ++l) {
-        const PostLayer Ld = a.layers[l];
+        const PostLayer Lnext = a.layers[min(l + 1, a.L - 1)];  // prefetch
         float* aout = a.a_all ? a.a_all + ((size_t)(l - a.t) * a.s + c) * N : nullptr;
-        post_row_layer<MODE_CENTROID>(Ld, N, a.ymax, 0.0f, cur, nxt, nullptr, aout, a.force_ell);
+        post_row_layer<MODE_CENTROID, 4, 4, 8>(Ld, N, a.ymax, 0.0f, cur, nxt, nullptr, aout, a.force_ell);
         __syncthreads();
         fill_halo(nxt, N);
         __syncthreads();
         float* tmp = cur;
         cur = nxt;
         nxt = tmp;
+        Ld = Lnext;
     }
     unstage_row(a.cbuf + (size_t)c * N, cur, N);
 }
@@ -222,7 +236,8 @@ __global__ void __launch_bounds__(kPostThreads) residual_traj_kernel(PostArgs a)
         for (int l = a.t; l < a.L; ++l) {
             const PostLayer Ld = a.layers[l];
             const float* ac = a.a_all + ((size_t)(l - a.t) * a.s + slot) * N;
-            const bool any = post_row_layer<MODE_RESIDUAL>(Ld, N, a.ymax, a.prune_eps, cur, nxt, ac, nullptr, a.force_ell);
+            const bool any =
+                post_row_layer<MODE_RESIDUAL, 17, 16, 1>(Ld, N, a.ymax, a.prune_eps, cur, nxt, ac, nullptr, a.force_ell);
             if (!__syncthreads_or(any)) {  // the residue became empty: it stays empty (R16)
                 alive = false;
                 break;
@@ -246,9 +261,9 @@ cudaError_t launch_centroid_traj(const PostArgs& a, int C_max, cudaStream_t st) 
     if (C_max <= 0) return cudaSuccess;
     const size_t smem = sizeof(float) * 2 * (size_t)(a.N + kPHalo);
     int per_sm = 1;
-    cudaError_t e = blocks_per_sm((const void*)centroid_traj_kernel, kPostThreads, smem, &per_sm);
+    cudaError_t e = blocks_per_sm((const void*)centroid_traj_kernel, kCentThreads, smem, &per_sm);
     if (e != cudaSuccess) return e;
-    centroid_traj_kernel<<<C_max, kPostThreads, smem, st>>>(a);
+    centroid_traj_kernel<<<C_max, kCentThreads, smem, st>>>(a);
     return cudaGetLastError();
 }
 
