@@ -49,16 +49,23 @@ __device__ __forceinline__ float post_epi(float acc, float b, const float* ac, i
 template <int MODE, bool UNIF, int MNU1, int MGEN, int QG>
 __device__ bool post_row_circ(const PostLayer& Ld, int N, float ymax, float prune_eps, const float* __restrict__ in,
                               float* __restrict__ out, const float* __restrict__ ac, float* __restrict__ aout) {
+    // descriptor fields in registers (the descriptor itself may live in local memory and would be
+    // re-read after every shared-memory store otherwise)
+    const float* __restrict__ wtab = Ld.wtab;
+    const float* __restrict__ bias = Ld.bias;
+    const float w0 = Ld.w0;
+    const float b0 = Ld.b0;
+    const bool ubias = Ld.ubias != 0;
+    const int cls = Ld.cls;
+    const int nu = Ld.nu, Q = N / nu;
     float w[UNIF ? 1 : kPK];
     if constexpr (!UNIF) {
 #pragma unroll
-        for (int n = 0; n < kPK; ++n) w[n] = __ldg(Ld.wtab + n);
+        for (int n = 0; n < kPK; ++n) w[n] = __ldg(wtab + n);
     }
-    const float w0 = Ld.w0;
-    const int nu = Ld.nu, Q = N / nu;
     bool any = false;
     auto emit = [&](float acc, int q) {
-        const float b = Ld.ubias ? Ld.b0 : __ldg(Ld.bias + q);
+        const float b = ubias ? b0 : __ldg(bias + q);
         if constexpr (MODE == MODE_CENTROID) {
             if (aout) aout[q] = acc;
         }
@@ -66,7 +73,7 @@ __device__ bool post_row_circ(const PostLayer& Ld, int N, float ymax, float prun
         out[q] = v;
         any |= (v != 0.0f);
     };
-    if (Ld.cls == PCLS_NU1) {
+    if (cls == PCLS_NU1) {
         constexpr int M = MNU1, WIN = M + kPK - 1;
         const int items = (N + M - 1) / M;
         for (int it = threadIdx.x; it < items; it += blockDim.x) {
@@ -84,7 +91,7 @@ __device__ bool post_row_circ(const PostLayer& Ld, int N, float ymax, float prun
                 }
             }
         }
-    } else if (Ld.cls == PCLS_Q32) {
+    } else if (cls == PCLS_Q32) {
         constexpr int OG = 32 / QG;  // outputs per item
         for (int it = threadIdx.x; it < nu * QG; it += blockDim.x) {
             const int c = it % nu;
@@ -132,17 +139,25 @@ __device__ bool post_row_circ(const PostLayer& Ld, int N, float ymax, float prun
 template <int MODE>
 __device__ bool post_row_ell(const PostLayer& Ld, int N, float ymax, float prune_eps, const float* __restrict__ in,
                              float* __restrict__ out, const float* __restrict__ ac, float* __restrict__ aout) {
+    const uint8_t* __restrict__ lens = Ld.len;
+    const uint16_t* __restrict__ i16 = Ld.idx16;
+    const int32_t* __restrict__ i32 = Ld.idx32;
+    const float* __restrict__ val = Ld.val;
+    const float* __restrict__ bias = Ld.bias;
+    const int K = Ld.K;
+    const bool unif = Ld.uniform_w != 0, ubias = Ld.ubias != 0;
+    const float w0 = Ld.w0, b0 = Ld.b0;
     bool any = false;
     for (int j = threadIdx.x; j < N; j += blockDim.x) {
-        const int len = Ld.len ? (int)Ld.len[j] : Ld.K;
+        const int len = lens ? (int)lens[j] : K;
         float acc = 0.0f;
         for (int n = 0; n < len; ++n) {
             const size_t e = (size_t)n * N + j;
-            const int k = Ld.idx16 ? (int)__ldg(Ld.idx16 + e) : __ldg(Ld.idx32 + e);
-            const float w = Ld.uniform_w ? Ld.w0 : __ldg(Ld.val + e);
+            const int k = i16 ? (int)__ldg(i16 + e) : __ldg(i32 + e);
+            const float w = unif ? w0 : __ldg(val + e);
             acc = fmaf(in[k], w, acc);
         }
-        const float b = Ld.ubias ? Ld.b0 : __ldg(Ld.bias + j);
+        const float b = ubias ? b0 : __ldg(bias + j);
         if constexpr (MODE == MODE_CENTROID) {
             if (aout) aout[j] = acc;
         }
