@@ -41,27 +41,55 @@ __device__ __forceinline__ float post_epi(float acc, float b, const float* ac, i
     }
 }
 
-// One layer of one row by the whole CTA: in (N + halo floats) -> out.  Returns this thread's
-// "some output != 0".  CENTROID mode also stores acc into aout (if non-NULL).
+// The descriptor of one layer, held in registers (fields read once per layer).
+struct PL {
+    int kind, cls, nu, K, unif, ubias;
+    float w0, b0;
+    const float* bias;
+    const float* wtab;
+    const uint16_t* idx16;
+    const int32_t* idx32;
+    const float* val;
+    const uint8_t* len;
+};
+__device__ __forceinline__ PL load_pl(const PostLayer* __restrict__ p) {
+    PL r;
+    r.kind = p->kind;
+    r.cls = p->cls;
+    r.nu = p->nu;
+    r.K = p->K;
+    r.unif = p->uniform_w;
+    r.ubias = p->ubias;
+    r.w0 = p->w0;
+    r.b0 = p->b0;
+    r.bias = p->bias;
+    r.wtab = p->wtab;
+    r.idx16 = p->idx16;
+    r.idx32 = p->idx32;
+    r.val = p->val;
+    r.len = p->len;
+    return r;
+}
+
+// One layer of one row by the whole CTA: in -> out (shared memory).  `dup` != 0: in[N .. 2N) holds a
+// copy of in[0 .. N) (windows of every stride class read without wrap-around); else only a 64-float
+// halo is present (nu == 1 windows) and the general class wraps explicitly.  Returns this thread's
+// "some output != 0"; CENTROID mode also stores acc into aout (if non-NULL).
 // MNU1 / MGEN: outputs per work item of the nu == 1 / general classes; QG: threads per residue class
 // of the Q == 32 class (32 / QG outputs each).  Small values -> more, shorter items (latency-bound
 // centroid trajectory on one SM); large -> fewer shared-memory loads per FMA (throughput).
 template <int MODE, bool UNIF, int MNU1, int MGEN, int QG>
-__device__ bool post_row_circ(const PostLayer& Ld, int N, float ymax, float prune_eps, const float* __restrict__ in,
-                              float* __restrict__ out, const float* __restrict__ ac, float* __restrict__ aout) {
-    // descriptor fields in registers (the descriptor itself may live in local memory and would be
-    // re-read after every shared-memory store otherwise)
-    const float* __restrict__ wtab = Ld.wtab;
-    const float* __restrict__ bias = Ld.bias;
-    const float w0 = Ld.w0;
-    const float b0 = Ld.b0;
+__device__ __forceinline__ bool post_row_circ(const PL& Ld, int N, int dup, float ymax, float prune_eps,
+                                              const float* __restrict__ in, float* __restrict__ out,
+                                              const float* __restrict__ ac, float* __restrict__ aout) {
+    const float w0 = Ld.w0, b0 = Ld.b0;
     const bool ubias = Ld.ubias != 0;
-    const int cls = Ld.cls;
+    const float* __restrict__ bias = Ld.bias;
     const int nu = Ld.nu, Q = N / nu;
     float w[UNIF ? 1 : kPK];
     if constexpr (!UNIF) {
 #pragma unroll
-        for (int n = 0; n < kPK; ++n) w[n] = __ldg(wtab + n);
+        for (int n = 0; n < kPK; ++n) w[n] = __ldg(Ld.wtab + n);
     }
     bool any = false;
     auto emit = [&](float acc, int q) {
@@ -73,17 +101,18 @@ __device__ bool post_row_circ(const PostLayer& Ld, int N, float ymax, float prun
         out[q] = v;
         any |= (v != 0.0f);
     };
-    if (cls == PCLS_NU1) {
+    if (Ld.cls == PCLS_NU1) {
         constexpr int M = MNU1, WIN = M + kPK - 1;
         const int items = (N + M - 1) / M;
+        const bool exact = N % M == 0;
         for (int it = threadIdx.x; it < items; it += blockDim.x) {
             const int a0 = it * M;
             float R[WIN];
 #pragma unroll
-            for (int i = 0; i < WIN; ++i) R[i] = in[a0 + i];  // halo: in[N + i] == in[i]
+            for (int i = 0; i < WIN; ++i) R[i] = in[a0 + i];  // halo / copy: in[N + i] == in[i]
 #pragma unroll
             for (int m = 0; m < M; ++m) {
-                if (a0 + m < N) {
+                if (exact || a0 + m < N) {
                     float acc = 0.0f;
 #pragma unroll
                     for (int n = 0; n < kPK; ++n) acc = fmaf(R[m + n], UNIF ? w0 : w[n], acc);
@@ -91,40 +120,48 @@ __device__ bool post_row_circ(const PostLayer& Ld, int N, float ymax, float prun
                 }
             }
         }
-    } else if (cls == PCLS_Q32) {
+    } else if (Ld.cls == PCLS_Q32) {
         constexpr int OG = 32 / QG;  // outputs per item
         for (int it = threadIdx.x; it < nu * QG; it += blockDim.x) {
             const int c = it % nu;
-            const int g = it / nu;  // output group: a = g*OG .. g*OG + OG - 1
-            float R[32];
+            const int g0 = (it / nu) * OG;  // output group: a = g0 .. g0 + OG - 1
+            const float* src = in + c;
+            float R[32];  // rotated so that every index below is a compile-time constant
 #pragma unroll
-            for (int j = 0; j < 32; ++j) R[j] = in[j * nu + c];
+            for (int j = 0; j < 32; ++j) R[j] = src[((g0 + j) & 31) * nu];
 #pragma unroll
             for (int mm = 0; mm < OG; ++mm) {
-                const int m = g * OG + mm;
                 float acc = 0.0f;
 #pragma unroll
-                for (int n = 0; n < kPK; ++n) acc = fmaf(R[(m + n) & 31], UNIF ? w0 : w[n], acc);
-                emit(acc, m * nu + c);
+                for (int n = 0; n < kPK; ++n) acc = fmaf(R[(mm + n) & 31], UNIF ? w0 : w[n], acc);
+                emit(acc, (g0 + mm) * nu + c);
             }
         }
     } else {
         constexpr int M = MGEN, WIN = M + kPK - 1;
         const int items = nu * ((Q + M - 1) / M);
+        const bool exact = Q % M == 0;
         for (int it = threadIdx.x; it < items; it += blockDim.x) {
             const int c = it % nu;
             const int a0 = (it / nu) * M;
+            const float* src = in + c;
             float R[WIN];
+            if (dup || a0 + WIN <= Q) {
+                const float* p = src + (size_t)a0 * nu;
 #pragma unroll
-            for (int i = 0; i < WIN; ++i) {
-                int ai = a0 + i;  // < 3Q since Q >= K
-                ai = ai >= Q ? ai - Q : ai;
-                ai = ai >= Q ? ai - Q : ai;
-                R[i] = in[ai * nu + c];
+                for (int i = 0; i < WIN; ++i) R[i] = p[i * nu];
+            } else {
+#pragma unroll
+                for (int i = 0; i < WIN; ++i) {
+                    int ai = a0 + i;  // < 3Q since Q >= K
+                    ai = ai >= Q ? ai - Q : ai;
+                    ai = ai >= Q ? ai - Q : ai;
+                    R[i] = src[ai * nu];
+                }
             }
 #pragma unroll
             for (int m = 0; m < M; ++m) {
-                if (a0 + m < Q) {
+                if (exact || a0 + m < Q) {
                     float acc = 0.0f;
 #pragma unroll
                     for (int n = 0; n < kPK; ++n) acc = fmaf(R[m + n], UNIF ? w0 : w[n], acc);
@@ -137,15 +174,16 @@ __device__ bool post_row_circ(const PostLayer& Ld, int N, float ymax, float prun
 }
 
 template <int MODE>
-__device__ bool post_row_ell(const PostLayer& Ld, int N, float ymax, float prune_eps, const float* __restrict__ in,
-                             float* __restrict__ out, const float* __restrict__ ac, float* __restrict__ aout) {
+__device__ __forceinline__ bool post_row_ell(const PL& Ld, int N, float ymax, float prune_eps,
+                                             const float* __restrict__ in, float* __restrict__ out,
+                                             const float* __restrict__ ac, float* __restrict__ aout) {
     const uint8_t* __restrict__ lens = Ld.len;
     const uint16_t* __restrict__ i16 = Ld.idx16;
     const int32_t* __restrict__ i32 = Ld.idx32;
     const float* __restrict__ val = Ld.val;
     const float* __restrict__ bias = Ld.bias;
     const int K = Ld.K;
-    const bool unif = Ld.uniform_w != 0, ubias = Ld.ubias != 0;
+    const bool unif = Ld.unif != 0, ubias = Ld.ubias != 0;
     const float w0 = Ld.w0, b0 = Ld.b0;
     bool any = false;
     for (int j = threadIdx.x; j < N; j += blockDim.x) {
@@ -169,13 +207,13 @@ __device__ bool post_row_ell(const PostLayer& Ld, int N, float ymax, float prune
 }
 
 template <int MODE, int MNU1, int MGEN, int QG>
-__device__ __forceinline__ bool post_row_layer(const PostLayer& Ld, int N, float ymax, float prune_eps,
+__device__ __forceinline__ bool post_row_layer(const PL& Ld, int N, int dup, float ymax, float prune_eps,
                                                const float* in, float* out, const float* ac, float* aout,
                                                int force_ell) {
     if (Ld.kind == 1 && !force_ell) {
-        if (Ld.uniform_w)
-            return post_row_circ<MODE, true, MNU1, MGEN, QG>(Ld, N, ymax, prune_eps, in, out, ac, aout);
-        return post_row_circ<MODE, false, MNU1, MGEN, QG>(Ld, N, ymax, prune_eps, in, out, ac, aout);
+        if (Ld.unif)
+            return post_row_circ<MODE, true, MNU1, MGEN, QG>(Ld, N, dup, ymax, prune_eps, in, out, ac, aout);
+        return post_row_circ<MODE, false, MNU1, MGEN, QG>(Ld, N, dup, ymax, prune_eps, in, out, ac, aout);
     }
     return post_row_ell<MODE>(Ld, N, ymax, prune_eps, in, out, ac, aout);
 }
@@ -190,10 +228,18 @@ __device__ __forceinline__ void unstage_row(float* dst, const float* src, int N)
     float4* d4 = reinterpret_cast<float4*>(dst);
     for (int k = threadIdx.x; k < (N >> 2); k += blockDim.x) d4[k] = s4[k];
 }
-__device__ __forceinline__ void fill_halo(float* row, int N) {
-    const int h = min(kPHalo, N);
-    for (int i = threadIdx.x; i < h; i += blockDim.x) row[N + i] = row[i];
+// row[N .. N + h) = row[0 .. h): h = N (full copy, `dup`) or the 64-float halo
+__device__ __forceinline__ void fill_halo(float* row, int N, int h) {
+    if ((h & 3) == 0 && (N & 3) == 0) {
+        const float4* s4 = reinterpret_cast<const float4*>(row);
+        float4* d4 = reinterpret_cast<float4*>(row + N);
+        for (int i = threadIdx.x; i < (h >> 2); i += blockDim.x) d4[i] = s4[i];
+    } else {
+        for (int i = threadIdx.x; i < h; i += blockDim.x) row[N + i] = row[i];
+    }
 }
+// staged row stride and halo: a full copy when two of them fit the shared-memory budget
+__host__ __device__ inline int post_halo(int N) { return (size_t)N * 16 <= 200 * 1024 ? N : min(kPHalo, N); }
 
 constexpr int kCentThreads = 1024;
 // One CTA (1024 threads) per centroid row; items of 4 outputs (nu == 1, general) or 4 per residue
@@ -205,20 +251,21 @@ __global__ void __launch_bounds__(kCentThreads) centroid_traj_kernel(PostArgs a)
     const int c = blockIdx.x;
     if (c >= C) return;
     const int N = a.N;
-    const int stride = N + kPHalo;
+    const int h = post_halo(N);
+    const int dup = h == N;
     float* cur = sm;
-    float* nxt = sm + stride;
+    float* nxt = sm + N + h;
     stage_row(cur, a.cbuf + (size_t)c * N, N);
     __syncthreads();
-    fill_halo(cur, N);
+    fill_halo(cur, N, h);
     __syncthreads();
-    PostLayer Ld = a.layers[a.t];
+    PL Ld = load_pl(a.layers + a.t);
     for (int l = a.t; l < a.L; ++l) {
-        const PostLayer Lnext = a.layers[min(l + 1, a.L - 1)];  // prefetch
+        const PL Lnext = load_pl(a.layers + min(l + 1, a.L - 1));  // prefetch (serial critical path)
         float* aout = a.a_all ? a.a_all + ((size_t)(l - a.t) * a.s + c) * N : nullptr;
-        post_row_layer<MODE_CENTROID, 4, 4, 8>(Ld, N, a.ymax, 0.0f, cur, nxt, nullptr, aout, a.force_ell);
+        post_row_layer<MODE_CENTROID, 4, 4, 8>(Ld, N, dup, a.ymax, 0.0f, cur, nxt, nullptr, aout, a.force_ell);
         __syncthreads();
-        fill_halo(nxt, N);
+        fill_halo(nxt, N, h);
         __syncthreads();
         float* tmp = cur;
         cur = nxt;
@@ -228,11 +275,12 @@ __global__ void __launch_bounds__(kCentThreads) centroid_traj_kernel(PostArgs a)
     unstage_row(a.cbuf + (size_t)c * N, cur, N);
 }
 
-__global__ void __launch_bounds__(kPostThreads) residual_traj_kernel(PostArgs a) {
+__global__ void __launch_bounds__(kPostThreads, 2) residual_traj_kernel(PostArgs a) {
     extern __shared__ __align__(128) float sm[];
     __shared__ int s_p;
     const int N = a.N;
-    const int stride = N + kPHalo;
+    const int h = post_halo(N);
+    const int dup = h == N;
     const int n = *a.rcount;
     for (;;) {
         if (threadIdx.x == 0) s_p = atomicAdd(a.work_counter, 1);
@@ -242,26 +290,28 @@ __global__ void __launch_bounds__(kPostThreads) residual_traj_kernel(PostArgs a)
         const int row = a.rlist[p];
         const int slot = a.cslot[row];
         float* cur = sm;
-        float* nxt = sm + stride;
+        float* nxt = sm + N + h;
         stage_row(cur, a.yhat + (size_t)row * N, N);
         __syncthreads();
-        fill_halo(cur, N);
+        fill_halo(cur, N, h);
         __syncthreads();
         bool alive = true;
+        PL Ld = load_pl(a.layers + a.t);
         for (int l = a.t; l < a.L; ++l) {
-            const PostLayer Ld = a.layers[l];
+            const PL Lnext = load_pl(a.layers + min(l + 1, a.L - 1));
             const float* ac = a.a_all + ((size_t)(l - a.t) * a.s + slot) * N;
-            const bool any =
-                post_row_layer<MODE_RESIDUAL, 17, 16, 1>(Ld, N, a.ymax, a.prune_eps, cur, nxt, ac, nullptr, a.force_ell);
+            const bool any = post_row_layer<MODE_RESIDUAL, 17, 16, 1>(Ld, N, dup, a.ymax, a.prune_eps, cur, nxt, ac,
+                                                                      nullptr, a.force_ell);
             if (!__syncthreads_or(any)) {  // the residue became empty: it stays empty (R16)
                 alive = false;
                 break;
             }
-            fill_halo(nxt, N);
+            fill_halo(nxt, N, h);
             __syncthreads();
             float* tmp = cur;
             cur = nxt;
             nxt = tmp;
+            Ld = Lnext;
         }
         if (alive) unstage_row(a.yhat + (size_t)row * N, cur, N);
         if (threadIdx.x == 0) {
@@ -274,7 +324,7 @@ __global__ void __launch_bounds__(kPostThreads) residual_traj_kernel(PostArgs a)
 
 cudaError_t launch_centroid_traj(const PostArgs& a, int C_max, cudaStream_t st) {
     if (C_max <= 0) return cudaSuccess;
-    const size_t smem = sizeof(float) * 2 * (size_t)(a.N + kPHalo);
+    const size_t smem = sizeof(float) * 2 * (size_t)(a.N + post_halo(a.N));
     int per_sm = 1;
     cudaError_t e = blocks_per_sm((const void*)centroid_traj_kernel, kCentThreads, smem, &per_sm);
     if (e != cudaSuccess) return e;
@@ -284,7 +334,7 @@ cudaError_t launch_centroid_traj(const PostArgs& a, int C_max, cudaStream_t st) 
 
 cudaError_t launch_residual_traj(const PostArgs& a, int max_rows, int num_sms, cudaStream_t st) {
     if (max_rows <= 0) return cudaSuccess;
-    const size_t smem = sizeof(float) * 2 * (size_t)(a.N + kPHalo);
+    const size_t smem = sizeof(float) * 2 * (size_t)(a.N + post_halo(a.N));
     int per_sm = 1;
     cudaError_t e = blocks_per_sm((const void*)residual_traj_kernel, kPostThreads, smem, &per_sm);
     if (e != cudaSuccess) return e;
