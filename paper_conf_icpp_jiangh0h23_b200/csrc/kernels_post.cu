@@ -242,7 +242,8 @@ __device__ __forceinline__ void fill_halo(float* row, int N, int h) {
 __host__ __device__ inline int post_halo(int N) { return (size_t)N * 16 <= 200 * 1024 ? N : min(kPHalo, N); }
 
 constexpr int kCentThreads = 1024;
-// One CTA (1024 threads) per centroid row; items of 4 outputs (nu == 1, general) or 4 per residue
+// One CTA (1024 threads) per centroid row; items of 5 outputs (nu == 1: odd -> conflict-free LDS),
+// 4 (general class) or 4 per residue
 // class (Q == 32) so the whole SM works on every layer; the next layer's descriptor is loaded while
 // the current layer computes (it is on the serial critical path otherwise).
 __global__ void __launch_bounds__(kCentThreads) centroid_traj_kernel(PostArgs a) {
@@ -263,7 +264,7 @@ __global__ void __launch_bounds__(kCentThreads) centroid_traj_kernel(PostArgs a)
     for (int l = a.t; l < a.L; ++l) {
         const PL Lnext = load_pl(a.layers + min(l + 1, a.L - 1));  // prefetch (serial critical path)
         float* aout = a.a_all ? a.a_all + ((size_t)(l - a.t) * a.s + c) * N : nullptr;
-        post_row_layer<MODE_CENTROID, 4, 4, 8>(Ld, N, dup, a.ymax, 0.0f, cur, nxt, nullptr, aout, a.force_ell);
+        post_row_layer<MODE_CENTROID, 5, 4, 8>(Ld, N, dup, a.ymax, 0.0f, cur, nxt, nullptr, aout, a.force_ell);
         __syncthreads();
         fill_halo(nxt, N, h);
         __syncthreads();
