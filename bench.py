@@ -229,11 +229,18 @@ def run_snicit(args):
     rank = int(os.environ.get("RANK", "0"))
     local = int(os.environ.get("LOCAL_RANK", "0"))
     distributed = world > 1
-    if distributed:
-        torch.cuda.set_device(local)
-        dist.init_process_group("nccl", device_id=torch.device("cuda", local))
-    dev = torch.device("cuda", local)
+    # SNICIT_DIST_BACKEND=gloo: test hook for boxes with fewer GPUs than ranks (ranks share devices,
+    # collectives run on host tensors); the production path is NCCL, one rank per GPU
+    backend = os.environ.get("SNICIT_DIST_BACKEND", "nccl")
+    ndev = torch.cuda.device_count()
+    dev = torch.device("cuda", local % max(ndev, 1))
     torch.cuda.set_device(dev)
+    coll_dev = dev if backend == "nccl" else torch.device("cpu")
+    if distributed:
+        if backend == "nccl":
+            dist.init_process_group("nccl", device_id=dev)
+        else:
+            dist.init_process_group(backend)
 
     c, snic = config_params(args)
     if args.scaling == "weak":
@@ -258,7 +265,7 @@ def run_snicit(args):
         g.infer(y0, t=t, s=s, options=opt, y_out=y_out, row_offset=row0)
         if distributed:
             with torch.cuda.stream(stream):
-                ids = torch.from_numpy(g.categories()).to(dev)
+                ids = torch.from_numpy(g.categories()).to(coll_dev)
                 allgather_categories(ids)
         else:
             g.num_categories()  # category set present (count read synchronises the stream)
@@ -277,7 +284,7 @@ def run_snicit(args):
             dist.barrier()
         ms = e0.elapsed_time(e1) / k
         if distributed:
-            tt = torch.tensor([ms], device=dev)
+            tt = torch.tensor([ms], device=coll_dev)
             dist.all_reduce(tt, op=dist.ReduceOp.MAX)
             ms = float(tt.item())
         return ms
@@ -339,7 +346,7 @@ def run_snicit(args):
             cats = g.categories()
             if distributed:
                 with torch.cuda.stream(stream):
-                    allgather_categories(torch.from_numpy(cats).to(dev))
+                    allgather_categories(torch.from_numpy(cats).to(coll_dev))
             return cats
         step_e2e()
         if distributed:
@@ -352,7 +359,7 @@ def run_snicit(args):
         torch.cuda.synchronize(dev)
         ms_e = (time.perf_counter() - t0) * 1e3 / k
         if distributed:
-            tt = torch.tensor([ms_e], device=dev)
+            tt = torch.tensor([ms_e], device=coll_dev)
             dist.all_reduce(tt, op=dist.ReduceOp.MAX)
             ms_e = float(tt.item())
         e2e = {"value": B_global * nnz / (ms_e * 1e-3), "unit": UNIT, "ms_per_step": ms_e,

@@ -1,0 +1,25 @@
+"""Small SNICIT runs for compute-sanitizer (memcheck / racecheck / synccheck / initcheck):
+    compute-sanitizer --tool memcheck python scripts/sanitize.py"""
+import os
+import sys
+
+sys.path.insert(0, os.path.dirname(os.path.dirname(os.path.abspath(__file__))))
+import numpy as np  # noqa: E402
+import torch  # noqa: E402
+
+from paper_conf_icpp_jiangh0h23_b200 import KERNEL_ELL, SnicitNetwork  # noqa: E402
+from workload import sdgc  # noqa: E402
+
+for mode, N, L, B, t, kw in (("radix", 1024, 24, 300, 3, {}), ("radix", 4096, 12, 64, 2, {}),
+                             ("perm", 1024, 10, 100, 2, {}), ("radix", 1024, 12, 200, 2, dict(post_mode=1)),
+                             ("radix", 1024, 12, 100, 3, dict(kernel=KERNEL_ELL))):
+    net = sdgc.gen_network(N, L, mode)
+    Y0 = torch.from_numpy(sdgc.gen_inputs(N, B)).cuda()
+    out = torch.empty_like(Y0)
+    with SnicitNetwork.from_network(net) as g:
+        g.set_stream(torch.cuda.current_stream())
+        g.infer(Y0, t=t, s=32, y_out=out, **kw)
+        cats = g.categories()
+        torch.cuda.synchronize()
+    print(mode, N, L, B, t, kw, "categories", len(cats), "sum", float(out.sum()))
+print("sanitize run done")
