@@ -253,7 +253,7 @@ def run_snicit(args):
     nnz = net.nnz
     kern = {"auto": KERNEL_AUTO, "ell": KERNEL_ELL, "circ": KERNEL_CIRC}[args.kernel]
     Yh = make_inputs(args, c, B_local, row0)
-    g = SnicitNetwork.from_network(net, device=local)
+    g = SnicitNetwork.from_network(net, device=dev.index)
     stream = torch.cuda.Stream(device=dev)
     g.set_stream(stream)
     y0 = torch.from_numpy(Yh).to(dev)

@@ -64,6 +64,19 @@ __host__ __device__ constexpr size_t circ_smem2(int N, int cls, int nu, int RT, 
 
 __device__ __forceinline__ void consumer_bar() { asm volatile("bar.sync 1, %0;" ::"n"(kCircThreads) : "memory"); }
 
+// Warp-aggregated row flags: lane 0 sets flag[r] for every row r that some lane reported non-zero, so
+// the only writer of a flag is the lane that then arrives on the mbarrier (release) -- the producer's
+// acquire sees it without relying on cross-lane ordering.  `nz`/`r` per lane; warp-uniform loop.
+__device__ __forceinline__ void warp_flag_rows(int* flags, bool nz, int r) {
+    unsigned m = __ballot_sync(0xffffffffu, nz);
+    while (m) {
+        const int src = __ffs(m) - 1;
+        const int rs = __shfl_sync(0xffffffffu, r, src);
+        m &= ~__ballot_sync(0xffffffffu, r == rs);
+        if ((threadIdx.x & 31) == 0) flags[rs] = 1;
+    }
+}
+
 // Warp-specialised, in-place: warps 0..7 compute (one work item per thread per tile), warp 8 is the
 // producer/storer.  Tile j of this CTA lives in stage j % S (k-th use: parity k & 1):
 //   in_full[s]   producer arrive.expect_tx + TMA load bytes  -> consumers may read stage s
@@ -301,11 +314,11 @@ __global__ void __launch_bounds__(kCircThreads + 32, (MODE == MODE_PLAIN && UNIF
                 }
             }
             consumer_bar();  // every read of this stage is done: overwrite it with the outputs
+            float mx0 = 0.0f, mx1 = 0.0f;
+            const bool second = rr + 1 < nr;
             if (item < n_items) {
-                float mx0 = 0.0f, mx1 = 0.0f;
                 float* d0 = st + (size_t)rr * stride + obase;
                 float* d1 = d0 + stride;
-                const bool second = rr + 1 < nr;
 #pragma unroll
                 for (int m = 0; m < M; ++m)
                     if (mlim == M || m < mlim) {
@@ -316,9 +329,9 @@ __global__ void __launch_bounds__(kCircThreads + 32, (MODE == MODE_PLAIN && UNIF
                             mx1 = fmaxf(mx1, fabsf(v1[m]));
                         }
                     }
-                if (mx0 != 0.0f) s_flag[sb * RT + rr] = 1;
-                if (second && mx1 != 0.0f) s_flag[sb * RT + rr + 1] = 1;
             }
+            warp_flag_rows(s_flag + sb * RT, mx0 != 0.0f, rr);
+            warp_flag_rows(s_flag + sb * RT, second && mx1 != 0.0f, rr + 1);
             fence_proxy_async_smem();
             __syncwarp();
             if (lane == 0) mbar_arrive(&out_full[sb]);
@@ -417,8 +430,8 @@ __global__ void __launch_bounds__(kCircThreads + 32, (MODE == MODE_PLAIN && UNIF
                         mx = fmaxf(mx, fabsf(v[m]));
                     }
             }
-            if (mx != 0.0f) s_flag[sb * RT + rr] = 1;
         }
+        warp_flag_rows(s_flag + sb * RT, mx != 0.0f, rr);
         fence_proxy_async_smem();  // this thread's writes -> visible to the TMA engine
         __syncwarp();
         if (lane == 0) mbar_arrive(&out_full[sb]);
