@@ -134,10 +134,11 @@ __global__ void __launch_bounds__(kCompactThreads) compact_count_kernel(const in
 
 __global__ void __launch_bounds__(kCompactThreads) compact_scatter_kernel(const int* __restrict__ list_in,
                                                                           const int* count_in,
-                                                                          const uint8_t* __restrict__ flag_pos,
+                                                                          uint8_t* __restrict__ flag_pos,
                                                                           const int* block_counts,
                                                                           int* __restrict__ list_out,
-                                                                          int* count_out) {
+                                                                          int* count_out, int clear,
+                                                                          uint8_t* __restrict__ row_flags) {
     const int n = *count_in;
     const int nblk = (n + kChunk - 1) / kChunk;
     __shared__ int s_prefix, s_ws[kCompactThreads / 32];
@@ -171,19 +172,25 @@ __global__ void __launch_bounds__(kCompactThreads) compact_scatter_kernel(const 
     uint8_t bytes[16];
     memcpy(bytes, &v, 16);
 #pragma unroll
-    for (int i = 0; i < 16; ++i)
-        if (bytes[i]) list_out[pos++] = list_in ? list_in[base + i] : base + i;
+    for (int i = 0; i < 16; ++i) {
+        if (base + i >= n) break;
+        const int id = list_in ? list_in[base + i] : base + i;
+        if (bytes[i]) list_out[pos++] = id;
+        if (row_flags) row_flags[id] = bytes[i] ? 1 : 0;  // e.g. ne_rec of residue rows (Alg. 3 l.13)
+        if (clear) flag_pos[base + i] = 0;                 // flags OR-ed by several CTAs start at 0
+    }
     if ((int)blockIdx.x == max(nblk, 1) - 1 && threadIdx.x == 0) *count_out = s_prefix + total;
 }
 
 cudaError_t launch_compact(const int* list_in, const int* count_in, const uint8_t* flag_pos, int* list_out,
-                           int* count_out, int max_n, int* scratch, cudaStream_t st) {
+                           int* count_out, int max_n, int* scratch, cudaStream_t st, int clear,
+                           uint8_t* row_flags) {
     const int nblk = max(1, (max_n + kChunk - 1) / kChunk);
     compact_count_kernel<<<nblk, kCompactThreads, 0, st>>>(count_in, flag_pos, scratch);
     cudaError_t e = cudaGetLastError();
     if (e != cudaSuccess) return e;
-    compact_scatter_kernel<<<nblk, kCompactThreads, 0, st>>>(list_in, count_in, flag_pos, scratch, list_out,
-                                                              count_out);
+    compact_scatter_kernel<<<nblk, kCompactThreads, 0, st>>>(list_in, count_in, const_cast<uint8_t*>(flag_pos),
+                                                              scratch, list_out, count_out, clear, row_flags);
     return cudaGetLastError();
 }
 int compact_scratch_ints(int max_n) { return max(1, (max_n + kChunk - 1) / kChunk); }

@@ -92,6 +92,7 @@ struct snicit_network {
     DevBuf<uint8_t> flag_pos, live_row, ne_row, cat, ne_t;
     DevBuf<float> cbuf0, cbuf1, ac;
     DevBuf<int> cscratch;  // per-chunk counts of the ordered compaction
+    DevBuf<uint8_t> segflag;  // row flags OR-ed by segmented layers (kept zero by the clearing compaction)
     DevBuf<double> F;
     DevBuf<int> counters;
     int* h_counters = nullptr;  // pinned mirror
@@ -149,6 +150,7 @@ void snicit_free_network(snicit_network* net) {
     net->cbuf0.release();
     net->cbuf1.release();
     net->cscratch.release();
+    net->segflag.release();
     net->ac.release();
     net->F.release();
     if (net->h_counters) cudaFreeHost(net->h_counters);
@@ -279,7 +281,7 @@ snicit_status snicit_load_network(int32_t N, int32_t L, snicit_format fmt, const
         pl.nu = 0;
         if (!ragged && K >= 2) {
             const int nu = (int)(((int64_t)cidx[0][1] - cidx[0][0] + N) % N);
-            bool circ = cidx[0][0] == 0 && circ_supported(N, K, nu);
+            bool circ = cidx[0][0] == 0 && (circ_supported(N, K, nu) || circ_seg_supported(N, K, nu));
             for (int j = 0; j < N && circ; ++j)
                 for (int n = 0; n < K; ++n) {
                     if (cidx[j][n] != (int32_t)(((int64_t)j + (int64_t)n * nu) % N) || cval[j][n] != cval[0][n] ||
@@ -289,7 +291,7 @@ snicit_status snicit_load_network(int32_t N, int32_t L, snicit_format fmt, const
                     }
                 }
             if (circ) {
-                pl.kind = 1;
+                pl.kind = circ_supported(N, K, nu) ? 1 : 2;  // whole rows staged, or segmented rows
                 pl.nu = nu;
                 pl.w_off = wtab.size();
                 for (int n = 0; n < K; ++n) wtab.push_back(cval[0][n]);
@@ -383,8 +385,8 @@ snicit_status snicit_load_network(int32_t N, int32_t L, snicit_format fmt, const
             const LayerPlan& pl = net->plan[l];
             PostLayer& d = pls[l];
             memset(&d, 0, sizeof(d));
-            d.kind = pl.kind;
-            d.cls = pl.kind == 1 ? circ_class_of(N, pl.nu) : 0;
+            d.kind = pl.kind != 0 ? 1 : 0;
+            d.cls = pl.kind != 0 ? circ_class_of(N, pl.nu) : 0;
             d.nu = pl.nu;
             d.K = pl.K;
             d.uniform_w = pl.uniform ? 1 : 0;
@@ -392,7 +394,7 @@ snicit_status snicit_load_network(int32_t N, int32_t L, snicit_format fmt, const
             d.w0 = pl.w0;
             d.b0 = bias[(int64_t)l * N];
             d.bias = net->bias_d.p + (size_t)l * N;
-            d.wtab = (pl.kind == 1 && !pl.uniform) ? net->wtab_d.p + pl.w_off : nullptr;
+            d.wtab = (pl.kind != 0 && !pl.uniform) ? net->wtab_d.p + pl.w_off : nullptr;
             d.idx16 = net->idx16 ? net->idx16_d.p + pl.ell_off : nullptr;
             d.idx32 = net->idx16 ? nullptr : net->idx32_d.p + pl.ell_off;
             d.val = pl.uniform ? nullptr : net->val_d.p + pl.ell_off;
@@ -419,7 +421,7 @@ snicit_status snicit_set_stream(snicit_network* net, void* s) {
 
 int32_t snicit_layer_is_circulant(const snicit_network* net, int32_t l) {
     if (!net || l < 0 || l >= net->L) return -1;
-    return net->plan[l].kind == 1 ? 1 : 0;
+    return net->plan[l].kind != 0 ? 1 : 0;
 }
 
 }  // extern "C"
@@ -440,7 +442,7 @@ static LayerArgs layer_args(snicit_network* net, int l, bool force_ell) {
     a.len = pl.ragged ? net->len_d.p + (size_t)l * net->N : nullptr;
     a.w0 = pl.w0;
     a.uniform_bias = pl.ubias ? 1 : 0;
-    if (pl.kind == 1 && !force_ell) {
+    if (pl.kind != 0 && !force_ell) {
         a.nu = pl.nu;
         a.wtab = pl.uniform ? nullptr : net->wtab_d.p + pl.w_off;
     }
@@ -449,10 +451,16 @@ static LayerArgs layer_args(snicit_network* net, int l, bool force_ell) {
 
 static bool use_circ(const snicit_network* net, int l, int kernel_opt) {
     if (kernel_opt == SNICIT_KERNEL_ELL) return false;
-    return net->plan[l].kind == 1;
+    return net->plan[l].kind != 0;
+}
+// segmented circulant layers: a row spans several CTAs, so row flags are OR-ed into `segflag` and
+// compacted by a separate (ordered, clearing) compaction instead of the fused append
+static bool use_seg(const snicit_network* net, int l, int kernel_opt) {
+    return use_circ(net, l, kernel_opt) && net->plan[l].kind == 2;
 }
 
 static cudaError_t run_layer(snicit_network* net, int l, int kernel_opt, int mode, LayerArgs a, int max_rows) {
+    if (use_seg(net, l, kernel_opt)) return launch_layer_circ_seg(a, mode, max_rows, net->num_sms, net->stream);
     if (use_circ(net, l, kernel_opt)) return launch_layer_circ(a, mode, max_rows, net->num_sms, net->stream);
     return launch_layer_ell(a, mode, max_rows, net->num_sms, net->stream);
 }
@@ -475,6 +483,10 @@ static cudaError_t ensure_workspace(snicit_network* net, int64_t R, int s, int n
     if ((e = net->iota_s.ensure(ss)) != cudaSuccess) return e;
     if ((e = net->F.ensure((size_t)std::max(n, 1) * ss)) != cudaSuccess) return e;
     if ((e = net->cscratch.ensure((size_t)compact_scratch_ints((int)rows))) != cudaSuccess) return e;
+    if (net->segflag.n < rows) {
+        if ((e = net->segflag.ensure(rows)) != cudaSuccess) return e;
+        if ((e = cudaMemset(net->segflag.p, 0, rows)) != cudaSuccess) return e;
+    }
     return cudaSuccess;
 }
 
@@ -512,7 +524,7 @@ snicit_status snicit_infer(snicit_network* net, const float* y0, int64_t batch, 
     const int N = net->N, L = net->L;
     if (opt.kernel == SNICIT_KERNEL_CIRC)
         for (int l = 0; l < L; ++l)
-            if (net->plan[l].kind != 1)
+            if (net->plan[l].kind == 0)
                 return fail(SNICIT_E_UNSUPPORTED, "layer " + std::to_string(l) + " is not circulant");
     const int R = (int)batch;
     const int tt = std::min(t, L);
@@ -587,14 +599,22 @@ snicit_status snicit_infer(snicit_network* net, const float* y0, int64_t batch, 
         a.yout = bufs[nxt_i];
         a.rows = lists[li];
         a.count = cnt + live_ctr[ci];
-        if (drop_now) {
+        const bool seg = use_seg(net, l, opt.kernel);
+        if (drop_now && !seg) {
             a.app_list = lists[li ^ 1];
             a.app_count = cnt + live_ctr[(ci + 1) % 3];
             a.zero_count = cnt + live_ctr[(ci + 2) % 3];
         }
+        if (drop_now && seg) a.flag_pos = net->segflag.p;
         CUDA_TRY(run_layer(net, l, opt.kernel, MODE_PLAIN, a, R));
         if (prof) CUDA_TRY(cudaEventRecord(net->lev[2 * l + 1], st));
         ++launches;
+        if (drop_now && seg) {
+            CUDA_TRY(launch_compact(lists[li], cnt + live_ctr[ci], net->segflag.p, lists[li ^ 1],
+                                    cnt + live_ctr[(ci + 1) % 3], R, scratch, st, 1));
+            CUDA_TRY(cudaMemsetAsync(cnt + live_ctr[(ci + 2) % 3], 0, sizeof(int), st));
+            launches += 2;
+        }
         circ_layers += use_circ(net, l, opt.kernel);
         net->last_kernel_circ = use_circ(net, l, opt.kernel);
         cur = bufs[nxt_i];
@@ -717,11 +737,18 @@ snicit_status snicit_infer(snicit_network* net, const float* y0, int64_t batch, 
                 b.count = rcnt;
                 b.a_c = net->ac.p;
                 b.cslot = net->cslot.p;
-                b.flag_pos = net->flag_pos.p;
-                b.flag_row = net->ne_row.p;
                 b.prune_eps = opt.prune_eps;
-                CUDA_TRY(run_layer(net, l, opt.kernel, MODE_RESIDUAL, b, R));
-                CUDA_TRY(launch_compact(rlist, rcnt, net->flag_pos.p, rlist_nxt, rcnt_nxt, R, scratch, st));
+                if (use_seg(net, l, opt.kernel)) {  // flags OR-ed across segments; ne_rec set by the compaction
+                    b.flag_pos = net->segflag.p;
+                    CUDA_TRY(run_layer(net, l, opt.kernel, MODE_RESIDUAL, b, R));
+                    CUDA_TRY(launch_compact(rlist, rcnt, net->segflag.p, rlist_nxt, rcnt_nxt, R, scratch, st, 1,
+                                            net->ne_row.p));
+                } else {
+                    b.flag_pos = net->flag_pos.p;
+                    b.flag_row = net->ne_row.p;
+                    CUDA_TRY(run_layer(net, l, opt.kernel, MODE_RESIDUAL, b, R));
+                    CUDA_TRY(launch_compact(rlist, rcnt, net->flag_pos.p, rlist_nxt, rcnt_nxt, R, scratch, st));
+                }
                 launches += 2;
                 std::swap(rlist, rlist_nxt);
                 std::swap(rcnt, rcnt_nxt);
@@ -850,7 +877,7 @@ snicit_status snicit_layer_profile(snicit_network* net, int32_t max, double* ms,
             const LayerPlan& pl = net->plan[l];
             // algorithmic bytes: rows read + written, weights, bias
             double wb;
-            if (pl.kind == 1 && net->last_kernel_circ)
+            if (pl.kind != 0 && net->last_kernel_circ)
                 wb = 4.0 * pl.K;
             else
                 wb = (double)pl.K * net->N * ((net->idx16 ? 2.0 : 4.0) + (pl.uniform ? 0.0 : 4.0));
@@ -893,7 +920,7 @@ snicit_status snicit_debug_layer(snicit_network* net, int32_t layer, const float
     if (!net || !yin || !yout) return fail(SNICIT_E_INVALID_ARG, "NULL argument");
     if (layer < 0 || layer >= net->L) return fail(SNICIT_E_INVALID_ARG, "bad layer");
     if (rows < 0 || rows > 0x7fffffffLL) return fail(SNICIT_E_INVALID_ARG, "bad rows");
-    if (kernel == SNICIT_KERNEL_CIRC && net->plan[layer].kind != 1)
+    if (kernel == SNICIT_KERNEL_CIRC && net->plan[layer].kind == 0)
         return fail(SNICIT_E_UNSUPPORTED, "layer is not circulant");
     CUDA_TRY(cudaSetDevice(net->device));
     CUDA_TRY(ensure_workspace(net, rows, 1, 1));

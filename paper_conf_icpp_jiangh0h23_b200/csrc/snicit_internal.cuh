@@ -125,7 +125,7 @@ struct LayerArgs {
 };
 
 struct LayerPlan {
-    int kind;       // 0 = ELL, 1 = CIRC
+    int kind;       // 0 = ELL, 1 = CIRC (whole rows staged), 2 = CIRC segmented (large rows)
     int K;
     int nu;         // CIRC
     bool uniform;   // all values equal (w0)
@@ -157,6 +157,9 @@ cudaError_t blocks_per_sm(const void* kern, int threads, size_t smem, int* out);
 cudaError_t launch_layer_ell(const LayerArgs& a, int mode, int max_rows, int num_sms, cudaStream_t st);
 cudaError_t launch_layer_circ(const LayerArgs& a, int mode, int max_rows, int num_sms, cudaStream_t st);
 bool circ_supported(int N, int K, int nu);
+// segmented circulant kernel (rows too large for kernels_circ.cu), kernels_circ_seg.cu
+cudaError_t launch_layer_circ_seg(const LayerArgs& a, int mode, int max_rows, int num_sms, cudaStream_t st);
+bool circ_seg_supported(int N, int K, int nu);
 bool ell_smem_ok(int N);
 
 // ------------------------------------------------------------------ fused post-convergence (kernels_post.cu)
@@ -206,8 +209,11 @@ cudaError_t launch_fill_i32(int* out, int n, int v, cudaStream_t st);
 cudaError_t launch_fill_u8(uint8_t* out, int n, uint8_t v, cudaStream_t st);
 cudaError_t launch_row_nonzero(const float* y, int N, const int* rows, const int* count, uint8_t* flag_pos,
                                int max_rows, int num_sms, cudaStream_t st);
+// clear != 0: flag_pos[0 .. *count_in) is zeroed after it is read; row_flags (nullable):
+// row_flags[list_in[i]] = flag_pos[i] for every position i
 cudaError_t launch_compact(const int* list_in, const int* count_in, const uint8_t* flag_pos, int* list_out,
-                           int* count_out, int max_n, int* scratch, cudaStream_t st);
+                           int* count_out, int max_n, int* scratch, cudaStream_t st, int clear = 0,
+                           uint8_t* row_flags = nullptr);
 int compact_scratch_ints(int max_n);
 cudaError_t launch_downsample(const float* y, int N, const int* rows, const int* count, int s, int n_seg,
                               double* F, cudaStream_t st);

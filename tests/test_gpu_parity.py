@@ -67,7 +67,7 @@ def ragged_net(N, L, seed, ymax=32.0):
 # ------------------------------------------------------------------------------ single layer, bit-exact
 
 @pytest.mark.parametrize("N,mode,rows", [(1024, "radix", 333), (4096, "radix", 97), (16384, "radix", 9),
-                                         (1024, "perm", 130), (4096, "random", 41)])
+                                         (65536, "radix", 3), (1024, "perm", 130), (4096, "random", 41)])
 def test_layer_kernels_bit_exact(N, mode, rows):
     net = sdgc.gen_network(N, 4, mode)
     Y0 = sdgc.gen_inputs(N, rows) * np.float32(7.5)  # non-binary values exercise rounding
@@ -77,8 +77,7 @@ def test_layer_kernels_bit_exact(N, mode, rows):
         for l in range(net.L):
             ref = oracle.layers_f32(net, Y0, l, l + 1)
             kernels = [KERNEL_ELL] + ([KERNEL_CIRC] if g.layer_is_circulant(l) else [])
-            if N <= 8192:
-                assert g.layer_is_circulant(l) == (mode == "radix")
+            assert g.layer_is_circulant(l) == (mode == "radix")  # N >= 16384: segmented circulant kernel
             for k in kernels:
                 out = torch.full_like(yin, float("nan"))
                 g.debug_layer(l, yin, out, kernel=k)
@@ -242,3 +241,21 @@ def test_post_modes_identical(mode, N, L, B, t):
         assert np.array_equal(Y, ref["Y"])
         assert np.array_equal(cats, ref["categories"])
     assert a[2]["residual_final"] == b[2]["residual_final"] == int((ref["ne"] & (ref["M"] >= 0)).sum())
+
+
+@pytest.mark.parametrize("N,L,B,t", [(16384, 12, 60, 3), (65536, 8, 12, 2)])
+def test_large_rows_segmented(N, L, B, t):
+    """C3/C4-sized rows (16384 / 65536 neurons): segmented circulant kernel (A- and C-segments),
+    per-layer post mode for N > 24576, both post modes for 16384; against the oracle."""
+    net = sdgc.gen_network(N, L, "radix")
+    Y0 = sdgc.gen_inputs(N, B)
+    plain = oracle.layers_f32(net, Y0)
+    ref = oracle.snicit(net, Y0, t=t)
+    for pm in ((0, 1) if N <= 24576 else (1,)):
+        Y, cats, st, clus = run_gpu(net, Y0, t=t, post_mode=pm)
+        assert np.array_equal(cats, oracle.categories(plain))
+        assert np.array_equal(Y, ref["Y"])
+        np.testing.assert_allclose(Y, plain, atol=ATOL, rtol=RTOL)
+        assert st["circ_layers"] > 0
+    Yu, catsu, _, _ = run_gpu(net, Y0, t=L)  # uncompressed path, bit-exact
+    assert np.array_equal(Yu, plain) and np.array_equal(catsu, oracle.categories(plain))
