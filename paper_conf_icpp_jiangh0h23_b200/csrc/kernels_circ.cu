@@ -362,7 +362,7 @@ __global__ void __launch_bounds__(kCircThreads + 32, (MODE == MODE_PLAIN && UNIF
                     for (int n = 0; n < kK; ++n) acc = fmaf(R[m + n], UNIF ? w0 : w[n], acc);
                     const int q = min(a0 + m, N - 1);  // tail outputs (m >= mlim) are discarded
                     const float bq = UBIAS ? b0 : __ldg(a.bias + q);
-                    v[m] = epilogue<MODE>(a, acc, bq, q, row, slot);
+                    v[m] = epilogue<MODE>(a, acc, bq, q, row, slot, a0 + m < N);
                 }
             } else if constexpr (CLS == CLS_Q32) {
                 const int c = rem;
@@ -409,7 +409,7 @@ __global__ void __launch_bounds__(kCircThreads + 32, (MODE == MODE_PLAIN && UNIF
                     for (int n = 0; n < kK; ++n) acc = fmaf(R[m + n], UNIF ? w0 : w[n], acc);
                     const int q = min(a0 + m, Q - 1) * nu + c;  // tail outputs are discarded
                     const float bq = UBIAS ? b0 : __ldg(a.bias + q);
-                    v[m] = epilogue<MODE>(a, acc, bq, q, row, slot);
+                    v[m] = epilogue<MODE>(a, acc, bq, q, row, slot, a0 + m < Q);
                 }
             }
         }

@@ -225,9 +225,9 @@ __global__ void __launch_bounds__(kSegThreads + 32, 2) layer_circ_seg_kernel(Lay
         float v[32];
         int n_out = 0, ob = 0, os = 1;
         bool have = false;
-        auto fin = [&](float acc, int q, int m) {
+        auto fin = [&](float acc, int q, int m, bool valid) {
             const float bq = UBIAS ? b0 : __ldg(a.bias + q);
-            v[m] = epilogue<MODE>(a, acc, bq, q, row, slot);
+            v[m] = epilogue<MODE>(a, acc, bq, q, row, slot, valid);
         };
         if (g.cls == 0) {  // nu == 1, A-segment: outputs a in [lo + 17 it, ...)
             constexpr int M = 17, WIN = M + kSK - 1;
@@ -246,7 +246,7 @@ __global__ void __launch_bounds__(kSegThreads + 32, 2) layer_circ_seg_kernel(Lay
                     float acc = 0.0f;
 #pragma unroll
                     for (int k = 0; k < kSK; ++k) acc = fmaf(R[m + k], UNIF ? w0 : w[k], acc);
-                    fin(acc, lo + min(a0 + m, n - 1), m);
+                    fin(acc, lo + min(a0 + m, n - 1), m, a0 + m < n);
                 }
             }
         } else if (g.cls == 1) {  // Q == 32, C-segment: one residue per thread, all 32 a
@@ -264,7 +264,7 @@ __global__ void __launch_bounds__(kSegThreads + 32, 2) layer_circ_seg_kernel(Lay
                     float acc = 0.0f;
 #pragma unroll
                     for (int k = 0; k < kSK; ++k) acc = fmaf(R[(m + k) & 31], UNIF ? w0 : w[k], acc);
-                    fin(acc, m * nu + lo + item, m);
+                    fin(acc, m * nu + lo + item, m, true);
                 }
             }
         } else {  // general stride, M = 16
@@ -301,7 +301,7 @@ __global__ void __launch_bounds__(kSegThreads + 32, 2) layer_circ_seg_kernel(Lay
 #pragma unroll
                     for (int k = 0; k < kSK; ++k) acc = fmaf(R[m + k], UNIF ? w0 : w[k], acc);
                     const int am = lo_a + min(a0 + m, na - 1);
-                    fin(acc, am * nu + lo_c + c, m);
+                    fin(acc, am * nu + lo_c + c, m, a0 + m < na);
                 }
             }
         }

@@ -136,16 +136,20 @@ struct LayerPlan {
     size_t w_off;   // offset in the per-n weight table
 };
 
-// Epilogue of one output q of one row (acc = the fma chain, b = bias[q]).
+// Epilogue of one output q of one row (acc = the fma chain, b = bias[q]).  `valid` == false marks a
+// discarded tail output (computed unguarded for speed, q clamped): it must not store anything.
 template <int MODE>
-__device__ __forceinline__ float epilogue(const LayerArgs& a, float acc, float b, int q, int row, int slot) {
+__device__ __forceinline__ float epilogue(const LayerArgs& a, float acc, float b, int q, int row, int slot,
+                                          bool valid = true) {
     if constexpr (MODE == MODE_RESIDUAL) {
         const float ac = __ldg(a.a_c + (size_t)slot * a.N + q);
         float v = sigma((ac + acc) + b, a.ymax) - sigma(ac + b, a.ymax);
         if (a.prune_eps > 0.0f && fabsf(v) <= a.prune_eps) v = 0.0f;
         return v;
     } else {
-        if constexpr (MODE == MODE_CENTROID) a.a_out[(size_t)row * a.N + q] = acc;
+        if constexpr (MODE == MODE_CENTROID) {
+            if (valid) a.a_out[(size_t)row * a.N + q] = acc;
+        }
         return sigma(acc + b, a.ymax);
     }
 }

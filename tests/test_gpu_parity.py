@@ -259,3 +259,17 @@ def test_large_rows_segmented(N, L, B, t):
         assert st["circ_layers"] > 0
     Yu, catsu, _, _ = run_gpu(net, Y0, t=L)  # uncompressed path, bit-exact
     assert np.array_equal(Yu, plain) and np.array_equal(catsu, oracle.categories(plain))
+
+
+@pytest.mark.parametrize("N,L", [(1024, 10), (4096, 9)])
+def test_post_modes_unsaturated_centroids(N, L):
+    """Per-layer post mode with centroids far from saturation (random real-valued inputs), so the
+    centroid pre-activations a_c differ per column: regression for the a_c of a row's tail outputs."""
+    net = sdgc.gen_network(N, L, "radix")
+    rs = np.random.RandomState(5)
+    Y0 = (sdgc.gen_inputs(N, 200) * rs.uniform(0.2, 1.5, size=(200, N))).astype(np.float32)
+    ref = oracle.snicit(net, Y0, t=2, n=0, eta=0.0, eps=0.01, s=8)
+    for pm in (0, 1):
+        Y, cats, st, _ = run_gpu(net, Y0, t=2, s=8, n_segments=0, eta=0.0, eps=0.01, post_mode=pm)
+        assert st["residual_at_t"] > 0
+        assert np.array_equal(Y, ref["Y"]) and np.array_equal(cats, ref["categories"])
