@@ -50,6 +50,9 @@ def parse():
     p.add_argument("--t", type=int, default=None)
     p.add_argument("--s", type=int, default=None)
     p.add_argument("--kernel", default="auto", choices=["auto", "ell", "circ"])
+    p.add_argument("--load", default="auto", choices=["auto", "csc", "compact"],
+                   help="network ABI: explicit CSC (snicit_load_network) or compact circulant form; auto = "
+                        "compact for radix nets with N >= 16384 (C3/C4 CSC is 8-32 GB)")
     p.add_argument("--scaling", default="weak", choices=["weak", "strong"])
     p.add_argument("--batch", type=int, default=None, help="override rows per rank (weak) / global (strong)")
     p.add_argument("--no-e2e", action="store_true")
@@ -74,10 +77,24 @@ def config_params(args):
     return c, snic
 
 
+def use_compact(args, c):
+    if args.config == "C5" or args.mode != "radix":
+        return False
+    return args.load == "compact" or (args.load == "auto" and c["N"] >= 16384)
+
+
 def make_network(args, c):
     if args.config == "C5":
         return sdgc.gen_medium_network(c["N"], c["L"])
+    if use_compact(args, c):
+        return sdgc.gen_circulant(c["N"], c["L"])
     return sdgc.gen_network(c["N"], c["L"], args.mode)
+
+
+def oracle_layers(oracle, net, Y, nthreads=0):
+    if isinstance(net, sdgc.CirculantNetwork):
+        return oracle.layers_circulant_f32(net, Y, nthreads=nthreads)
+    return oracle.layers_f32(net, Y, nthreads=nthreads)
 
 
 def make_inputs(args, c, B, row0):
@@ -166,7 +183,7 @@ def oracle_sample_time(oracle, net, Y, cores, seconds, probe_only=False):
     with all threads), and the measured time for that many rows."""
     k = max(1, min(len(Y), cores))
     t0 = time.perf_counter()
-    oracle.layers_f32(net, Y[:k])
+    oracle_layers(oracle, net, Y[:k])
     t_probe = max(time.perf_counter() - t0, 1e-6)
     rows = int(max(k, min(len(Y), k * seconds / t_probe)))
     if probe_only:
@@ -174,7 +191,7 @@ def oracle_sample_time(oracle, net, Y, cores, seconds, probe_only=False):
     if rows == k:
         return k, t_probe
     t0 = time.perf_counter()
-    oracle.layers_f32(net, Y[:rows])
+    oracle_layers(oracle, net, Y[:rows])
     return rows, time.perf_counter() - t0
 
 
@@ -194,11 +211,11 @@ def run_reference(args):
     rows, _ = oracle_sample_time(oracle, net, probe, cores, args.cpu_seconds / max(args.steps, 1), probe_only=True)
     Y = make_inputs(args, c, rows, 0)
     if args.warmup > 0:
-        oracle.layers_f32(net, Y[: max(1, min(rows, cores))])
+        oracle_layers(oracle, net, Y[: max(1, min(rows, cores))])
     times = []
     for _ in range(args.steps):
         t0 = time.perf_counter()
-        oracle.layers_f32(net, Y)
+        oracle_layers(oracle, net, Y)
         times.append(time.perf_counter() - t0)
     T = float(np.mean(times))
     value = rows * nnz / T
@@ -253,7 +270,10 @@ def run_snicit(args):
     nnz = net.nnz
     kern = {"auto": KERNEL_AUTO, "ell": KERNEL_ELL, "circ": KERNEL_CIRC}[args.kernel]
     Yh = make_inputs(args, c, B_local, row0)
-    g = SnicitNetwork.from_network(net, device=dev.index)
+    if isinstance(net, sdgc.CirculantNetwork):
+        g = SnicitNetwork.circulant(net.N, net.L, net.nu, net.w, net.bias, net.ymax, device=dev.index)
+    else:
+        g = SnicitNetwork.from_network(net, device=dev.index)
     stream = torch.cuda.Stream(device=dev)
     g.set_stream(stream)
     y0 = torch.from_numpy(Yh).to(dev)
@@ -384,6 +404,7 @@ def run_snicit(args):
             "config": {"workload": f"{args.config}: {c['desc']}", "neurons": c["N"], "layers": c["L"],
                        "batch_per_rank": B_local, "global_batch": B_global, "connections": nnz, "w_mode": args.mode,
                        "t": t, "s": s, "n": snic["n"], "eta": 0.03, "eps": 0.03, "kernel": args.kernel,
+                       "network_abi": "compact circulant" if isinstance(net, sdgc.CirculantNetwork) else "CSC",
                        "l2": "inputs larger than L2 (no flush)", "parallelism": f"dp{world} (row shards)"},
             "roofline": roof, "cpu_baseline": cpu, "e2e": e2e, "clocks": clk,
             "gpu_launches": int(launches_per_step * args.steps),

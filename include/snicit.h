@@ -110,6 +110,18 @@ snicit_status snicit_load_network(int32_t n_neurons, int32_t n_layers, snicit_fo
                                   const float* bias, float ymax, int32_t cuda_device,
                                   snicit_network** out);
 
+/* Load a network given in the compact form of shift-invariant ("circulant") layers: column j of
+ * layer l reads inputs (j + n*nu[l]) mod N, n = 0..K-1, in that order, with weight w[l*K + n] --
+ * the RadiX-Net layers of SDGC, "sums of cyclic permutations".  Equivalent to
+ * snicit_load_network with the explicit CSC (same plans, same results; tested) without the
+ * L*N*K index arrays (C4: 32 GB).  Requirements: N % nu[l] == 0, K*nu[l] <= N (distinct inputs),
+ * K == 32 (the circulant kernels' tap count) -> else SNICIT_E_BAD_SPARSE / SNICIT_E_UNSUPPORTED.
+ * nu: L int32; w: L*K fp32; bias: L*N fp32 (host pointers, copied).  The general ELL kernel is
+ * unavailable for such a handle (options.kernel = SNICIT_KERNEL_ELL -> SNICIT_E_UNSUPPORTED). */
+snicit_status snicit_load_network_circulant(int32_t n_neurons, int32_t n_layers, const int32_t* nu,
+                                            int32_t K, const float* w, const float* bias, float ymax,
+                                            int32_t cuda_device, snicit_network** out);
+
 /* All work of this handle is issued on `cuda_stream` (a cudaStream_t, e.g.
  * torch.cuda.current_stream().cuda_stream); NULL = the legacy default stream. */
 snicit_status snicit_set_stream(snicit_network* net, void* cuda_stream);

@@ -45,6 +45,7 @@ def lib():
         L.oracle_version.restype = i32
         L.oracle_layers_f32.argtypes = [i32, P, P, P, P, f32, i32, i32, i64, P, P, i32]
         L.oracle_layers_f64.argtypes = [i32, P, P, P, P, f32, i32, i32, i64, P, P, i32]
+        L.oracle_layers_circulant_f32.argtypes = [i32, i32, P, P, P, f32, i32, i32, i64, P, P, i32]
         L.oracle_sum_downsample.argtypes = [i32, i32, i32, P, P]
         L.oracle_prune.argtypes = [i32, i32, P, f32, f32, P]
         L.oracle_prune.restype = i32
@@ -86,6 +87,19 @@ def layers_f64(net, Y: np.ndarray, l0: int = 0, l1: Optional[int] = None, nthrea
     ptr, idx, val, bias = _net_arrays(net)
     lib().oracle_layers_f64(net.N, _p(ptr), _p(idx), _p(val), _p(bias), net.ymax, l0, l1,
                             Y.shape[0], _p(Y), _p(out), nthreads)
+    return out
+
+
+def layers_circulant_f32(cnet, Y: np.ndarray, l0: int = 0, l1: Optional[int] = None, nthreads: int = 0) -> np.ndarray:
+    """Plain Eq. (1) in fp32 for a network in compact circulant form (workload.sdgc.CirculantNetwork)."""
+    l1 = cnet.L if l1 is None else l1
+    Y = np.ascontiguousarray(Y, dtype=np.float32)
+    out = np.empty_like(Y)
+    nu = np.ascontiguousarray(cnet.nu, dtype=np.int32)
+    w = np.ascontiguousarray(cnet.w, dtype=np.float32)
+    b = np.ascontiguousarray(cnet.bias, dtype=np.float32)
+    lib().oracle_layers_circulant_f32(cnet.N, w.shape[1], _p(nu), _p(w), _p(b), cnet.ymax, l0, l1, Y.shape[0],
+                                      _p(Y), _p(out), nthreads)
     return out
 
 

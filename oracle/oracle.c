@@ -98,6 +98,38 @@ void oracle_layers_f64(int32_t N, const int64_t* ptr, const int32_t* idx, const 
     }
 }
 
+__attribute__((target_clones("fma", "default")))
+static void row_layer_circ_f32(int32_t N, int32_t K, int32_t nu, const float* w, const float* b, float ymax,
+                               const float* y, float* y_next) {
+    for (int32_t j = 0; j < N; ++j) {
+        float acc = 0.0f;
+        for (int32_t n = 0; n < K; ++n) acc = fmaf(y[(int32_t)(((int64_t)j + (int64_t)n * nu) % N)], w[n], acc);
+        y_next[j] = sigma_f32(acc + b[j], ymax);
+    }
+}
+
+void oracle_layers_circulant_f32(int32_t N, int32_t K, const int32_t* nu, const float* w, const float* bias,
+                                 float ymax, int32_t l0, int32_t l1, int64_t B, const float* Yin, float* Yout,
+                                 int32_t nthreads) {
+    set_threads(nthreads);
+#pragma omp parallel
+    {
+        float* a = (float*)malloc(sizeof(float) * (size_t)N);
+        float* c = (float*)malloc(sizeof(float) * (size_t)N);
+#pragma omp for schedule(dynamic, 4)
+        for (int64_t r = 0; r < B; ++r) {
+            memcpy(a, Yin + r * N, sizeof(float) * (size_t)N);
+            for (int32_t l = l0; l < l1; ++l) {
+                row_layer_circ_f32(N, K, nu[l], w + (int64_t)l * K, bias + (int64_t)l * N, ymax, a, c);
+                float* tmp = a; a = c; c = tmp;
+            }
+            memcpy(Yout + r * N, a, sizeof(float) * (size_t)N);
+        }
+        free(a);
+        free(c);
+    }
+}
+
 /* Sum downsampling: "divides the original column into n segments, each containing N/n elements
  * ... For each segment, we run a simple sum reduction". */
 void oracle_sum_downsample(int32_t N, int32_t n, int32_t s, const float* rows, double* F) {

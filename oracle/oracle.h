@@ -38,6 +38,14 @@ void oracle_layers_f64(int32_t N, const int64_t* ptr, const int32_t* idx, const 
                        const float* bias, float ymax, int32_t l0, int32_t l1,
                        int64_t B, const double* Yin, double* Yout, int32_t nthreads);
 
+/* Eq. (1) for networks given in the compact circulant form (column j of layer l reads
+ * (j + n*nu[l]) mod N, n = 0..K-1, weight w[l*K + n]): the same definition with the
+ * index computed instead of stored; fp32, the same fma order as oracle_layers_f32 on the expanded
+ * CSC (pinned against it in tests). */
+void oracle_layers_circulant_f32(int32_t N, int32_t K, const int32_t* nu, const float* w, const float* bias,
+                                 float ymax, int32_t l0, int32_t l1, int64_t B, const float* Yin, float* Yout,
+                                 int32_t nthreads);
+
 /* ---- Sum downsampling, Sec. 3.2.1, Fig. 3a PAPER.md:587-596.
  * rows: s x N (the sampled rows).  F: n x s row-major, F[g*s+q] = sum of rows[q][k] over
  * segment g, segments of floor(N/n) elements, last segment takes the remainder (R15).

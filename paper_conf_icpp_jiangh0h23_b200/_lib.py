@@ -23,7 +23,7 @@ KERNEL_AUTO, KERNEL_ELL, KERNEL_CIRC = 0, 1, 2
 EXPORTED = ["snicit_default_options", "snicit_load_network", "snicit_set_stream", "snicit_infer",
             "snicit_categories", "snicit_stats", "snicit_debug_clustering", "snicit_debug_layer",
             "snicit_layer_is_circulant", "snicit_free_network", "snicit_last_error", "snicit_abi_version",
-            "snicit_layer_profile"]
+            "snicit_layer_profile", "snicit_load_network_circulant"]
 
 
 class Options(ctypes.Structure):
@@ -65,6 +65,8 @@ def load_library(path: str = LIB_PATH):
     L.snicit_default_options.restype = None
     L.snicit_load_network.argtypes = [i32, i32, i32, P, P, P, P, f32, i32, ctypes.POINTER(P)]
     L.snicit_load_network.restype = i32
+    L.snicit_load_network_circulant.argtypes = [i32, i32, P, i32, P, P, f32, i32, ctypes.POINTER(P)]
+    L.snicit_load_network_circulant.restype = i32
     L.snicit_set_stream.argtypes = [P, P]
     L.snicit_set_stream.restype = i32
     L.snicit_infer.argtypes = [P, P, i64, i32, i64, i32, i32, ctypes.POINTER(Options), P, i32]

@@ -43,6 +43,27 @@ class SnicitNetwork:
         self._stream = None
 
     @classmethod
+    def circulant(cls, N: int, L: int, nu, w, bias, ymax: float, device: int = 0):
+        """Compact shift-invariant form (snicit_load_network_circulant): column j of layer l reads
+        (j + n*nu[l]) mod N with weight w[l, n], n = 0..K-1."""
+        self = cls.__new__(cls)
+        self._lib = load_library()
+        self.N, self.L, self.ymax, self.device = int(N), int(L), float(ymax), int(device)
+        nu = np.ascontiguousarray(nu, dtype=np.int32)
+        w = np.ascontiguousarray(w, dtype=np.float32).reshape(L, -1)
+        bias = np.ascontiguousarray(bias, dtype=np.float32)
+        if nu.size != L or bias.size != L * N:
+            raise ValueError("nu must have L entries and bias L*N")
+        h = ctypes.c_void_p()
+        check(self._lib.snicit_load_network_circulant(self.N, self.L, nu.ctypes.data, int(w.shape[1]),
+                                                      w.ctypes.data, bias.ctypes.data, self.ymax, self.device,
+                                                      ctypes.byref(h)), "snicit_load_network_circulant")
+        self._h = h
+        self._last_batch = 0
+        self._stream = None
+        return self
+
+    @classmethod
     def from_network(cls, net, device: int = 0):
         """From a workload.sdgc.Network-like object (N, L, ptr, idx, val, bias, ymax)."""
         return cls(net.N, net.L, net.ptr, net.idx, net.val, net.bias, net.ymax, device=device)

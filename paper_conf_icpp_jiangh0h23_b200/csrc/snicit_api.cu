@@ -75,6 +75,7 @@ struct snicit_network {
     std::vector<LayerPlan> plan;
     std::vector<uint8_t> dead_ok;  // dead_ok[l]: all biases of layers >= l are <= 0 (R23)
     bool idx16 = true;
+    bool has_ell = true;  // ELL copies exist (CSC loads); compact circulant loads have none
     // weights
     DevBuf<uint16_t> idx16_d;
     DevBuf<int32_t> idx32_d;
@@ -112,6 +113,87 @@ struct snicit_network {
     DevBuf<int> hist;              // active rows at the start of each pre-convergence layer
     int prof_layers = 0;
 };
+
+
+// ---------------------------------------------------------------------------------------- load helpers
+static snicit_status net_device_init(snicit_network* net, int cuda_device) {
+    int ndev = 0;
+    if (cudaGetDeviceCount(&ndev) != cudaSuccess || ndev < 1) return fail(SNICIT_E_CUDA, "no CUDA device");
+    if (cuda_device < 0 || cuda_device >= ndev) return fail(SNICIT_E_INVALID_ARG, "bad cuda_device");
+    cudaDeviceProp prop;
+    cudaError_t pe = cudaGetDeviceProperties(&prop, cuda_device);
+    if (pe != cudaSuccess) return fail(SNICIT_E_CUDA, cudaGetErrorString(pe));
+    if (prop.major != 10)
+        return fail(SNICIT_E_CUDA, "libsnicit is built for sm_100a (B200); device is sm_" +
+                                       std::to_string(prop.major) + std::to_string(prop.minor));
+    net->num_sms = prop.multiProcessorCount;
+    net->device = cuda_device;
+    cudaSetDevice(cuda_device);
+    return SNICIT_OK;
+}
+
+// per-layer uniform-bias flag (SDGC: a constant per benchmark, Table 1) and dead_ok[l]: every bias
+// of layers >= l is <= 0, so an all-zero row stays zero (R23)
+static void net_bias_flags(snicit_network* net, const float* bias) {
+    const int N = net->N, L = net->L;
+    for (int l = 0; l < L; ++l) {
+        bool ub = true;
+        const float* b = bias + (int64_t)l * N;
+        for (int j = 1; j < N && ub; ++j) ub = b[j] == b[0] && std::signbit(b[j]) == std::signbit(b[0]);
+        net->plan[l].ubias = ub;
+    }
+    net->dead_ok.assign(L + 1, 1);
+    for (int l = L - 1; l >= 0; --l) {
+        bool ok = net->dead_ok[l + 1];
+        for (int j = 0; j < N; ++j)
+            if (bias[(int64_t)l * N + j] > 0.0f) ok = false;
+        net->dead_ok[l] = ok ? 1 : 0;
+    }
+}
+
+template <typename B, typename T>
+static cudaError_t upload(B& buf, const T* host, size_t count) {
+    cudaError_t e = buf.ensure(count);
+    if (e != cudaSuccess) return e;
+    if (count) return cudaMemcpy(buf.p, host, count * sizeof(T), cudaMemcpyHostToDevice);
+    return cudaSuccess;
+}
+
+// weight table, bias, fused-post layer descriptors, counters, events (after the ELL arrays, if any)
+static cudaError_t net_upload_common(snicit_network* net, const float* bias, const std::vector<float>& wtab) {
+    const int N = net->N, L = net->L;
+    cudaError_t e = upload(net->wtab_d, wtab.data(), wtab.size());
+    if (e == cudaSuccess) e = upload(net->bias_d, bias, (size_t)L * N);
+    if (e == cudaSuccess) {
+        std::vector<PostLayer> pls(L);
+        for (int l = 0; l < L; ++l) {
+            const LayerPlan& pl = net->plan[l];
+            PostLayer& d = pls[l];
+            memset(&d, 0, sizeof(d));
+            d.kind = pl.kind != 0 ? 1 : 0;
+            d.cls = pl.kind != 0 ? circ_class_of(N, pl.nu) : 0;
+            d.nu = pl.nu;
+            d.K = pl.K;
+            d.uniform_w = pl.uniform ? 1 : 0;
+            d.ubias = pl.ubias ? 1 : 0;
+            d.w0 = pl.w0;
+            d.b0 = bias[(int64_t)l * N];
+            d.bias = net->bias_d.p + (size_t)l * N;
+            d.wtab = (pl.kind != 0 && !pl.uniform) ? net->wtab_d.p + pl.w_off : nullptr;
+            if (net->has_ell) {
+                d.idx16 = net->idx16 ? net->idx16_d.p + pl.ell_off : nullptr;
+                d.idx32 = net->idx16 ? nullptr : net->idx32_d.p + pl.ell_off;
+                d.val = pl.uniform ? nullptr : net->val_d.p + pl.ell_off;
+                d.len = pl.ragged ? net->len_d.p + (size_t)l * N : nullptr;
+            }
+        }
+        e = upload(net->post_layers_d, pls.data(), pls.size());
+    }
+    if (e == cudaSuccess) e = net->counters.ensure(CNT_N);
+    if (e == cudaSuccess) e = cudaMallocHost(&net->h_counters, sizeof(int) * CNT_N);
+    for (int i = 0; i < 6 && e == cudaSuccess; ++i) e = cudaEventCreate(&net->ev[i]);
+    return e;
+}
 
 extern "C" {
 
@@ -309,42 +391,15 @@ snicit_status snicit_load_network(int32_t N, int32_t L, snicit_format fmt, const
             if (ragged) lay_len[l][j] = (uint8_t)cidx[j].size();
         }
     }
-    // uniform bias per layer
-    for (int l = 0; l < L; ++l) {
-        bool ub = true;
-        const float* b = bias + (int64_t)l * N;
-        for (int j = 1; j < N && ub; ++j) ub = b[j] == b[0] && std::signbit(b[j]) == std::signbit(b[0]);
-        net->plan[l].ubias = ub;
-    }
-    // dead_ok
-    net->dead_ok.assign(L + 1, 1);
-    for (int l = L - 1; l >= 0; --l) {
-        bool ok = net->dead_ok[l + 1];
-        for (int j = 0; j < N; ++j)
-            if (bias[(int64_t)l * N + j] > 0.0f) ok = false;
-        net->dead_ok[l] = ok ? 1 : 0;
-    }
+    net_bias_flags(net, bias);
     // ---- device (validation above needs no GPU, so bad input is reported on any host)
     {
-        int ndev = 0;
-        if (cudaGetDeviceCount(&ndev) != cudaSuccess || ndev < 1) {
+        const snicit_status ds = net_device_init(net, cuda_device);
+        if (ds != SNICIT_OK) {
+            const std::string msg = g_last_error;
             snicit_free_network(net);
-            return fail(SNICIT_E_CUDA, "no CUDA device");
+            return fail(ds, msg);
         }
-        if (cuda_device < 0 || cuda_device >= ndev) {
-            snicit_free_network(net);
-            return fail(SNICIT_E_INVALID_ARG, "bad cuda_device");
-        }
-        cudaDeviceProp prop;
-        cudaError_t pe = cudaGetDeviceProperties(&prop, cuda_device);
-        if (pe != cudaSuccess || prop.major != 10) {
-            snicit_free_network(net);
-            return fail(SNICIT_E_CUDA, pe != cudaSuccess ? std::string(cudaGetErrorString(pe))
-                                                         : "libsnicit is built for sm_100a (B200); device is sm_" +
-                                                               std::to_string(prop.major) + std::to_string(prop.minor));
-        }
-        net->num_sms = prop.multiProcessorCount;
-        cudaSetDevice(cuda_device);
     }
     // ---- upload
     auto up = [&](auto& buf, const auto* host, size_t count) -> cudaError_t {
@@ -377,34 +432,68 @@ snicit_status snicit_load_network(int32_t N, int32_t L, snicit_format fmt, const
             e = up(net->len_d, alll.data(), alll.size());
         }
     }
-    if (e == cudaSuccess) e = up(net->wtab_d, wtab.data(), wtab.size());
-    if (e == cudaSuccess) e = up(net->bias_d, bias, (size_t)L * N);
-    if (e == cudaSuccess) {
-        std::vector<PostLayer> pls(L);
-        for (int l = 0; l < L; ++l) {
-            const LayerPlan& pl = net->plan[l];
-            PostLayer& d = pls[l];
-            memset(&d, 0, sizeof(d));
-            d.kind = pl.kind != 0 ? 1 : 0;
-            d.cls = pl.kind != 0 ? circ_class_of(N, pl.nu) : 0;
-            d.nu = pl.nu;
-            d.K = pl.K;
-            d.uniform_w = pl.uniform ? 1 : 0;
-            d.ubias = pl.ubias ? 1 : 0;
-            d.w0 = pl.w0;
-            d.b0 = bias[(int64_t)l * N];
-            d.bias = net->bias_d.p + (size_t)l * N;
-            d.wtab = (pl.kind != 0 && !pl.uniform) ? net->wtab_d.p + pl.w_off : nullptr;
-            d.idx16 = net->idx16 ? net->idx16_d.p + pl.ell_off : nullptr;
-            d.idx32 = net->idx16 ? nullptr : net->idx32_d.p + pl.ell_off;
-            d.val = pl.uniform ? nullptr : net->val_d.p + pl.ell_off;
-            d.len = pl.ragged ? net->len_d.p + (size_t)l * N : nullptr;
-        }
-        e = up(net->post_layers_d, pls.data(), pls.size());
+    if (e == cudaSuccess) e = net_upload_common(net, bias, wtab);
+    if (e != cudaSuccess) {
+        snicit_free_network(net);
+        return fail(e == cudaErrorMemoryAllocation ? SNICIT_E_OOM : SNICIT_E_CUDA, cudaGetErrorString(e));
     }
-    if (e == cudaSuccess) e = net->counters.ensure(CNT_N);
-    if (e == cudaSuccess) e = cudaMallocHost(&net->h_counters, sizeof(int) * CNT_N);
-    for (int i = 0; i < 6 && e == cudaSuccess; ++i) e = cudaEventCreate(&net->ev[i]);
+    *out = net;
+    return SNICIT_OK;
+}
+
+snicit_status snicit_load_network_circulant(int32_t N, int32_t L, const int32_t* nu, int32_t K, const float* w,
+                                            const float* bias, float ymax, int32_t cuda_device,
+                                            snicit_network** out) {
+    if (!out) return fail(SNICIT_E_INVALID_ARG, "out is NULL");
+    *out = nullptr;
+    if (N < 1 || L < 1 || K < 1) return fail(SNICIT_E_INVALID_ARG, "n_neurons, n_layers, K must be >= 1");
+    if (!nu || !w || !bias) return fail(SNICIT_E_INVALID_ARG, "nu/w/bias NULL");
+    if (!(ymax > 0.0f) || std::isnan(ymax)) return fail(SNICIT_E_INVALID_ARG, "ymax must be > 0");
+    if (N % 4 != 0) return fail(SNICIT_E_UNSUPPORTED, "n_neurons must be a multiple of 4 (16-byte rows)");
+    for (int64_t i = 0; i < (int64_t)L * K; ++i)
+        if (!std::isfinite(w[i])) return fail(SNICIT_E_INVALID_ARG, "non-finite weight");
+    for (int64_t i = 0; i < (int64_t)L * N; ++i)
+        if (!std::isfinite(bias[i])) return fail(SNICIT_E_INVALID_ARG, "non-finite bias");
+    auto* net = new snicit_network();
+    net->N = N;
+    net->L = L;
+    net->ymax = ymax;
+    net->idx16 = N <= 65536;
+    net->has_ell = false;
+    net->plan.resize(L);
+    std::vector<float> wtab;
+    for (int l = 0; l < L; ++l) {
+        const int v = nu[l];
+        if (v < 1 || v > N || N % v != 0 || (int64_t)K * v > N) {
+            snicit_free_network(net);
+            return fail(SNICIT_E_BAD_SPARSE, "layer " + std::to_string(l) + ": stride must divide N with K*nu <= N");
+        }
+        if (!(circ_supported(N, K, v) || circ_seg_supported(N, K, v))) {
+            snicit_free_network(net);
+            return fail(SNICIT_E_UNSUPPORTED, "layer " + std::to_string(l) + ": no circulant kernel for (N, K, nu)");
+        }
+        LayerPlan& pl = net->plan[l];
+        pl.kind = circ_supported(N, K, v) ? 1 : 2;
+        pl.nu = v;
+        pl.K = K;
+        pl.ragged = false;
+        const float* wl = w + (int64_t)l * K;
+        bool uniform = true;
+        for (int n = 1; n < K; ++n) uniform &= wl[n] == wl[0] && std::signbit(wl[n]) == std::signbit(wl[0]);
+        pl.uniform = uniform;
+        pl.w0 = wl[0];
+        pl.w_off = wtab.size();
+        for (int n = 0; n < K; ++n) wtab.push_back(wl[n]);
+        pl.ell_off = 0;
+    }
+    net_bias_flags(net, bias);
+    snicit_status ds = net_device_init(net, cuda_device);
+    if (ds != SNICIT_OK) {
+        const std::string msg = g_last_error;
+        snicit_free_network(net);
+        return fail(ds, msg);
+    }
+    cudaError_t e = net_upload_common(net, bias, wtab);
     if (e != cudaSuccess) {
         snicit_free_network(net);
         return fail(e == cudaErrorMemoryAllocation ? SNICIT_E_OOM : SNICIT_E_CUDA, cudaGetErrorString(e));
@@ -434,12 +523,14 @@ static LayerArgs layer_args(snicit_network* net, int l, bool force_ell) {
     a.bias = net->bias_d.p + (size_t)l * net->N;
     a.ymax = net->ymax;
     a.K = pl.K;
-    if (net->idx16)
-        a.idx16 = net->idx16_d.p + pl.ell_off;
-    else
-        a.idx32 = net->idx32_d.p + pl.ell_off;
-    a.val = pl.uniform ? nullptr : net->val_d.p + pl.ell_off;
-    a.len = pl.ragged ? net->len_d.p + (size_t)l * net->N : nullptr;
+    if (net->has_ell) {
+        if (net->idx16)
+            a.idx16 = net->idx16_d.p + pl.ell_off;
+        else
+            a.idx32 = net->idx32_d.p + pl.ell_off;
+        a.val = pl.uniform ? nullptr : net->val_d.p + pl.ell_off;
+        a.len = pl.ragged ? net->len_d.p + (size_t)l * net->N : nullptr;
+    }
     a.w0 = pl.w0;
     a.uniform_bias = pl.ubias ? 1 : 0;
     if (pl.kind != 0 && !force_ell) {
@@ -521,6 +612,8 @@ snicit_status snicit_infer(snicit_network* net, const float* y0, int64_t batch, 
         return fail(SNICIT_E_INVALID_ARG, "bad eta/eps/prune_eps");
     if (opt.kernel < 0 || opt.kernel > 2) return fail(SNICIT_E_INVALID_ARG, "bad kernel option");
     if (opt.post_mode < 0 || opt.post_mode > 1) return fail(SNICIT_E_INVALID_ARG, "bad post_mode");
+    if (opt.kernel == SNICIT_KERNEL_ELL && !net->has_ell)
+        return fail(SNICIT_E_UNSUPPORTED, "network loaded in compact circulant form has no ELL copy");
     const int N = net->N, L = net->L;
     if (opt.kernel == SNICIT_KERNEL_CIRC)
         for (int l = 0; l < L; ++l)
@@ -920,6 +1013,8 @@ snicit_status snicit_debug_layer(snicit_network* net, int32_t layer, const float
     if (!net || !yin || !yout) return fail(SNICIT_E_INVALID_ARG, "NULL argument");
     if (layer < 0 || layer >= net->L) return fail(SNICIT_E_INVALID_ARG, "bad layer");
     if (rows < 0 || rows > 0x7fffffffLL) return fail(SNICIT_E_INVALID_ARG, "bad rows");
+    if (kernel == SNICIT_KERNEL_ELL && !net->has_ell)
+        return fail(SNICIT_E_UNSUPPORTED, "network loaded in compact circulant form has no ELL copy");
     if (kernel == SNICIT_KERNEL_CIRC && net->plan[layer].kind == 0)
         return fail(SNICIT_E_UNSUPPORTED, "layer is not circulant");
     CUDA_TRY(cudaSetDevice(net->device));

@@ -273,3 +273,23 @@ def test_post_modes_unsaturated_centroids(N, L):
         Y, cats, st, _ = run_gpu(net, Y0, t=2, s=8, n_segments=0, eta=0.0, eps=0.01, post_mode=pm)
         assert st["residual_at_t"] > 0
         assert np.array_equal(Y, ref["Y"]) and np.array_equal(cats, ref["categories"])
+
+
+@pytest.mark.parametrize("N,L,B,t", [(1024, 30, 500, 4), (16384, 9, 40, 3)])
+def test_compact_circulant_loader_equals_csc(N, L, B, t):
+    """snicit_load_network_circulant (compact RadiX form) == snicit_load_network (explicit CSC)."""
+    c = sdgc.gen_circulant(N, L)
+    net = c.to_network()
+    Y0 = sdgc.gen_inputs(N, B)
+    ref = run_gpu(net, Y0, t=t)
+    with SnicitNetwork.circulant(N, L, c.nu, c.w, c.bias, c.ymax) as g:
+        g.set_stream(torch.cuda.current_stream())
+        y0 = torch.from_numpy(Y0).cuda()
+        out = torch.empty_like(y0)
+        g.infer(y0, t=t, s=32, y_out=out)
+        cats = g.categories()
+        Y = out.cpu().numpy()
+        with pytest.raises(Exception):
+            g.infer(y0, t=t, s=32, kernel=KERNEL_ELL)  # no ELL copy in compact form
+    assert np.array_equal(Y, ref[0]) and np.array_equal(cats, ref[1])
+    assert np.array_equal(cats, oracle.categories(oracle.layers_circulant_f32(c, Y0)))

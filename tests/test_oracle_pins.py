@@ -373,3 +373,16 @@ def test_medium_net_snicit_vs_plain():
     assert np.array_equal(res["categories"], oracle.categories(plain))
     np.testing.assert_allclose(res["Y"], plain, atol=1e-4, rtol=1e-5)
     assert plain.max() <= 1.0
+
+
+def test_circulant_form_equals_csc():
+    """The compact circulant network is the radix CSC network, and the oracle's circulant-form layer
+    loop equals its CSC layer loop bit for bit (same definition, same fma order)."""
+    for N, L in ((1024, 6), (4096, 4)):
+        c = sdgc.gen_circulant(N, L)
+        net = sdgc.gen_network(N, L, "radix")
+        e = c.to_network()
+        assert np.array_equal(e.ptr, net.ptr) and np.array_equal(e.idx, net.idx) and np.array_equal(e.val, net.val)
+        assert c.nnz == net.nnz
+        Y0 = sdgc.gen_inputs(N, 7) * np.float32(3.3)
+        assert np.array_equal(oracle.layers_circulant_f32(c, Y0), oracle.layers_f32(net, Y0))

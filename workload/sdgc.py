@@ -142,6 +142,44 @@ def gen_network(N: int, L: int, mode: str = "radix", seed: int = BASE_SEED, K: i
     return _assemble(N, L, cols, vals, b, ymax, mode, strides)
 
 
+@dataclasses.dataclass
+class CirculantNetwork:
+    """Compact form of a radix network: column j of layer l reads (j + n*nu[l]) mod N, n = 0..K-1, in
+    that order, with weight w[l, n] (exactly what gen_network(mode="radix") stores as CSC)."""
+
+    N: int
+    L: int
+    nu: np.ndarray    # int32 [L]
+    w: np.ndarray     # float32 [L, K]
+    bias: np.ndarray  # float32 [L*N]
+    ymax: float
+
+    @property
+    def nnz(self) -> int:
+        return int(self.L) * int(self.N) * int(self.w.shape[1])
+
+    def to_network(self) -> Network:
+        K = self.w.shape[1]
+        cols, vals = [], []
+        for l in range(self.L):
+            j = np.arange(self.N, dtype=np.int64)[:, None]
+            cols.append((j + np.arange(K, dtype=np.int64)[None, :] * int(self.nu[l])) % self.N)
+            vals.append(np.broadcast_to(self.w[l][None, :], (self.N, K)).astype(np.float32))
+        return _assemble(self.N, self.L, cols, vals, self.bias, self.ymax, "radix",
+                         radix_strides(self.N))
+
+
+def gen_circulant(N: int, L: int, K: int = SDGC_K, bias: Optional[float] = None, weight: float = SDGC_WEIGHT,
+                  ymax: float = SDGC_YMAX) -> CirculantNetwork:
+    """The radix network of gen_network(N, L, "radix") in compact form (no L*N*K index arrays)."""
+    if bias is None:
+        bias = SDGC_BIAS.get(N, -0.3)
+    strides = radix_strides(N)
+    nu = np.array([strides[l % len(strides)] for l in range(L)], dtype=np.int32)
+    w = np.full((L, K), weight, dtype=np.float32)
+    return CirculantNetwork(N=N, L=L, nu=nu, w=w, bias=np.full(L * N, bias, dtype=np.float32), ymax=float(ymax))
+
+
 def gen_medium_network(N: int = 256, L: int = 18, K: int = 26, seed: int = BASE_SEED) -> Network:
     """Config 5 stand-in: pruned MNIST/CIFAR-shaped sparse MLP, random init.
 
