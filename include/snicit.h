@@ -76,7 +76,11 @@ typedef struct {
                                their residue becomes empty); 1 = per layer: centroid layer + residue
                                layer + ne_idx row compaction for every layer.  Results are
                                identical.  N > 24576 always uses the per-layer mode. */
-    int32_t reserved[3];
+    int32_t post_cluster;   /* fused mode: 1 = each centroid row carried by a thread-block cluster of
+                               8 CTAs exchanging layer outputs through distributed shared memory
+                               (when every post layer is circulant and partition-compatible); 0 = one
+                               CTA per centroid.  Results identical. */
+    int32_t reserved[2];
 } snicit_options;
 
 /* Per-run statistics of the last snicit_infer (times in ms, valid when options.timing). */
@@ -95,7 +99,7 @@ typedef struct {
 } snicit_stats_t;
 
 /* Fill *opt with the paper's SDGC defaults (n = 16, eta = eps = 0.03, prune_eps = 0,
- * drop_dead_rows = 1, kernel = AUTO, timing = 0, ne_interval = 64). */
+ * drop_dead_rows = 1, kernel = AUTO, timing = 0, ne_interval = 64, post_mode = 0, post_cluster = 1). */
 void snicit_default_options(snicit_options* opt);
 
 /* Load a network (one-time; untimed in the benchmark).  All pointers are HOST pointers and

@@ -30,7 +30,7 @@ class Options(ctypes.Structure):
     _fields_ = [("n_segments", ctypes.c_int32), ("eta", ctypes.c_float), ("eps", ctypes.c_float),
                 ("prune_eps", ctypes.c_float), ("drop_dead_rows", ctypes.c_int32), ("kernel", ctypes.c_int32),
                 ("timing", ctypes.c_int32), ("ne_interval", ctypes.c_int32), ("post_mode", ctypes.c_int32),
-                ("reserved", ctypes.c_int32 * 3)]
+                ("post_cluster", ctypes.c_int32), ("reserved", ctypes.c_int32 * 2)]
 
 
 class Stats(ctypes.Structure):

@@ -15,9 +15,12 @@
 //
 // Per-layer arithmetic is identical to kernels_circ.cu / kernels_layer.cu (the stored-order fma
 // chain, reading R12), so results are bit-identical to the per-layer path.
+#include <cooperative_groups.h>
 #include <cuda_runtime.h>
 
 #include "snicit_internal.cuh"
+
+namespace cg = cooperative_groups;
 
 namespace snicit {
 
@@ -321,6 +324,192 @@ __global__ void __launch_bounds__(kPostThreads, 2) residual_traj_kernel(PostArgs
         }
         __syncthreads();  // s_p and the row buffers are reused
     }
+}
+
+// ------------------------------------------------------------------------------ cluster version
+// The centroid trajectory is a serial chain of L - t layers; one SM per centroid leaves it bound by
+// a single SM's issue rate.  Here a thread-block cluster of kCL CTAs carries one centroid row: every
+// layer, CTA r computes 1/kCL of the outputs and keeps them in its shared memory; the next layer's
+// input window of each CTA is gathered from its peers' shared memory (distributed shared memory,
+// ld through cluster-mapped addresses), and one cluster barrier per layer orders the exchange.
+// Output ownership per layer: index partition (CTA r owns outputs [r*S, (r+1)*S), S = N/kCL) for
+// nu == 1 and general strides, residue partition (CTA r owns residues [r*nu/kCL, (r+1)*nu/kCL) at
+// all 32 a) for Q == 32 layers, so every CTA's input window is a small, mostly local set.
+constexpr int kCL = 8;
+constexpr int kClThreads = 512;
+constexpr int kClMaxWin = 16384;  // floats of the gathered input window
+
+__device__ __forceinline__ int cl_owner(int k, int part, int nu, int S, int& off) {
+    if (part == 0) {
+        const int o = k / S;
+        off = k - o * S;
+        return o;
+    }
+    const int a = k / nu, c = k - a * nu;
+    const int cs = nu / kCL;
+    const int o = c / cs;
+    off = a * cs + (c - o * cs);
+    return o;
+}
+
+__global__ void __cluster_dims__(kCL, 1, 1) __launch_bounds__(kClThreads) centroid_cluster_kernel(PostArgs a) {
+    extern __shared__ __align__(128) float sm[];
+    cg::cluster_group cl = cg::this_cluster();
+    const int r = (int)cl.block_rank();
+    const int cid = blockIdx.x / kCL;
+    const int C = *a.n_cent;
+    if (cid >= C) return;  // uniform over the cluster
+    const int N = a.N, S = N / kCL;
+    float* slice[2] = {sm, sm + S};
+    float* win = sm + 2 * S;
+    for (int i = threadIdx.x; i < S; i += blockDim.x) slice[0][i] = a.cbuf[(size_t)cid * N + r * S + i];
+    int prev_part = 0, prev_nu = 1, cur = 0;
+    cl.sync();
+    PL Ld = load_pl(a.layers + a.t);
+    for (int l = a.t; l < a.L; ++l) {
+        const PL Lnext = load_pl(a.layers + min(l + 1, a.L - 1));
+        const int nu = Ld.nu, Q = N / nu, cls = Ld.cls;
+        const int part = cls == PCLS_Q32 ? 1 : 0;
+        const float w0 = Ld.w0, b0 = Ld.b0;
+        const bool ubias = Ld.ubias != 0, unif = Ld.unif != 0;
+        const float* __restrict__ bias = Ld.bias;
+        float wr[kPK];
+#pragma unroll
+        for (int n = 0; n < kPK; ++n) wr[n] = unif ? w0 : __ldg(Ld.wtab + n);
+        float* aout = a.a_all ? a.a_all + ((size_t)(l - a.t) * a.s + cid) * N : nullptr;
+        // ---- gather this CTA's input window from the peers' slices (previous layer's outputs)
+        const float* src = slice[cur];
+        auto fetch = [&](int k) -> float {
+            int off;
+            const int o = cl_owner(k, prev_part, prev_nu, S, off);
+            const float* p = cl.map_shared_rank(src, o);
+            return p[off];
+        };
+        int wlen, q0 = 0, a_s = 0, c0 = 0, cs = 0;
+        if (cls == PCLS_NU1) {
+            q0 = r * S;
+            wlen = S + kPK;
+            for (int i = threadIdx.x; i < wlen; i += blockDim.x) win[i] = fetch((q0 + i) % N);
+        } else if (cls == PCLS_GEN) {
+            a_s = r * (S / nu);
+            wlen = (S / nu + kPK) * nu;
+            for (int i = threadIdx.x; i < wlen; i += blockDim.x) {
+                const int aa = i / nu, c = i - aa * nu;
+                win[i] = fetch(((a_s + aa) % Q) * nu + c);
+            }
+        } else {
+            cs = nu / kCL;
+            c0 = r * cs;
+            wlen = 32 * cs;
+            for (int i = threadIdx.x; i < wlen; i += blockDim.x) {
+                const int aa = i / cs, cc = i - aa * cs;
+                win[i] = fetch(aa * nu + c0 + cc);
+            }
+        }
+        __syncthreads();
+        // ---- compute this CTA's outputs (stored-order fma chains, R12) into its next slice
+        float* out = slice[cur ^ 1];
+        auto emit = [&](float acc, int q, int so) {
+            const float b = ubias ? b0 : __ldg(bias + q);
+            if (aout) aout[q] = acc;
+            out[so] = sigma(acc + b, a.ymax);
+        };
+        if (cls == PCLS_NU1) {
+            constexpr int M = 5, WIN = M + kPK - 1;  // odd M: conflict-free window loads
+            for (int it = threadIdx.x; it * M < S; it += blockDim.x) {
+                const int a0 = it * M;
+                float R[WIN];
+#pragma unroll
+                for (int i = 0; i < WIN; ++i) R[i] = win[a0 + i];
+#pragma unroll
+                for (int m = 0; m < M; ++m) {
+                    if (a0 + m < S) {
+                        float acc = 0.0f;
+#pragma unroll
+                        for (int n = 0; n < kPK; ++n) acc = fmaf(R[m + n], wr[n], acc);
+                        emit(acc, q0 + a0 + m, a0 + m);
+                    }
+                }
+            }
+        } else if (cls == PCLS_GEN) {
+            constexpr int M = 4, WIN = M + kPK - 1;
+            const int na = S / nu;
+            for (int it = threadIdx.x; it < nu * ((na + M - 1) / M); it += blockDim.x) {
+                const int c = it % nu, al = (it / nu) * M;
+                float R[WIN];
+#pragma unroll
+                for (int i = 0; i < WIN; ++i) R[i] = win[(al + i) * nu + c];
+#pragma unroll
+                for (int m = 0; m < M; ++m) {
+                    if (al + m < na) {
+                        float acc = 0.0f;
+#pragma unroll
+                        for (int n = 0; n < kPK; ++n) acc = fmaf(R[m + n], wr[n], acc);
+                        emit(acc, (a_s + al + m) * nu + c, (al + m) * nu + c);
+                    }
+                }
+            }
+        } else {
+            constexpr int OG = 4;
+            for (int it = threadIdx.x; it < cs * (32 / OG); it += blockDim.x) {
+                const int cc = it % cs, g0 = (it / cs) * OG;
+                float R[32];
+#pragma unroll
+                for (int j = 0; j < 32; ++j) R[j] = win[((g0 + j) & 31) * cs + cc];
+#pragma unroll
+                for (int mm = 0; mm < OG; ++mm) {
+                    float acc = 0.0f;
+#pragma unroll
+                    for (int n = 0; n < kPK; ++n) acc = fmaf(R[(mm + n) & 31], wr[n], acc);
+                    emit(acc, (g0 + mm) * nu + c0 + cc, (g0 + mm) * cs + cc);
+                }
+            }
+        }
+        cl.sync();  // outputs of this layer visible cluster-wide; nobody still reads slice[cur]
+        cur ^= 1;
+        prev_part = part;
+        prev_nu = nu;
+        Ld = Lnext;
+    }
+    // ---- the final centroid row back to global memory
+    for (int i = threadIdx.x; i < S; i += blockDim.x) {
+        int k;
+        if (prev_part == 0) {
+            k = r * S + i;
+        } else {
+            const int csz = prev_nu / kCL;
+            const int aa = i / csz, cc = i - aa * csz;
+            k = aa * prev_nu + r * csz + cc;
+        }
+        a.cbuf[(size_t)cid * N + k] = slice[cur][i];
+    }
+}
+
+// host: can the cluster kernel carry layers [t, L)?  (every layer circulant, partition-compatible)
+bool centroid_cluster_ok(int N, const int* nu, const int* cls, int t, int L) {
+    if (N % (kCL * 4) != 0) return false;
+    const int S = N / kCL;
+    for (int l = t; l < L; ++l) {
+        if (cls[l] < 0) return false;  // not circulant (or ELL forced)
+        if (cls[l] == PCLS_NU1) {
+            if (S + kPK > kClMaxWin) return false;
+        } else if (cls[l] == PCLS_Q32) {
+            if (nu[l] % kCL != 0) return false;
+        } else {
+            if (S % nu[l] != 0 || (size_t)(S / nu[l] + kPK) * nu[l] > kClMaxWin) return false;
+        }
+    }
+    return true;
+}
+
+cudaError_t launch_centroid_cluster(const PostArgs& a, int C_max, int win_max, cudaStream_t st) {
+    if (C_max <= 0) return cudaSuccess;
+    const size_t smem = sizeof(float) * (2 * (size_t)(a.N / kCL) + (size_t)win_max);
+    int per_sm = 1;
+    cudaError_t e = blocks_per_sm((const void*)centroid_cluster_kernel, kClThreads, smem, &per_sm);
+    if (e != cudaSuccess) return e;
+    centroid_cluster_kernel<<<C_max * kCL, kClThreads, smem, st>>>(a);
+    return cudaGetLastError();
 }
 
 cudaError_t launch_centroid_traj(const PostArgs& a, int C_max, cudaStream_t st) {

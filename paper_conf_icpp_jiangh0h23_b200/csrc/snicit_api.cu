@@ -106,6 +106,7 @@ struct snicit_network {
     int live_counter = 0;  // which CNT_LIVE* holds the live count at t
     int res_final_counter = -1;  // counter holding the non-empty residue rows after the last layer
     bool last_fused = false;
+    bool last_cluster = false;
     bool last_kernel_circ = false;
     snicit_stats_t stats{};
     cudaEvent_t ev[6] = {nullptr, nullptr, nullptr, nullptr, nullptr, nullptr};
@@ -209,6 +210,7 @@ void snicit_default_options(snicit_options* opt) {
     opt->timing = 0;
     opt->ne_interval = 64;
     opt->post_mode = 0;
+    opt->post_cluster = 1;
 }
 
 const char* snicit_last_error(void) { return g_last_error.c_str(); }
@@ -802,7 +804,24 @@ snicit_status snicit_infer(snicit_network* net, const float* y0, int64_t batch, 
             pa.alive_count = cnt + CNT_ALIVE;
             CUDA_TRY(cudaMemsetAsync(cnt + CNT_WORK, 0, 2 * sizeof(int), st));
             pa.force_ell = opt.kernel == SNICIT_KERNEL_ELL ? 1 : 0;
-            CUDA_TRY(launch_centroid_traj(pa, s, st));
+            // cluster (DSMEM) trajectory when every post layer is circulant and partition-compatible
+            std::vector<int> nus(L, 0), clss(L, -1);
+            int win_max = 0;
+            for (int l = 0; l < L; ++l) {
+                if (use_circ(net, l, opt.kernel)) {
+                    nus[l] = net->plan[l].nu;
+                    clss[l] = circ_class_of(N, nus[l]);
+                    const int S8 = N / 8;
+                    const int w = clss[l] == 0 ? S8 + 32 : (clss[l] == 1 ? S8 : (S8 / nus[l] + 32) * nus[l]);
+                    if (l >= tt) win_max = std::max(win_max, w);
+                }
+            }
+            const bool use_cluster = opt.post_cluster != 0 && centroid_cluster_ok(N, nus.data(), clss.data(), tt, L);
+            net->last_cluster = use_cluster;
+            if (use_cluster)
+                CUDA_TRY(launch_centroid_cluster(pa, s, win_max, st));
+            else
+                CUDA_TRY(launch_centroid_traj(pa, s, st));
             ++launches;
             for (int l = tt; l < L; ++l) circ_layers += use_circ(net, l, opt.kernel);
             if (res_host > 0) {

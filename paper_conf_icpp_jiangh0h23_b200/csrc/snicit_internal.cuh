@@ -204,6 +204,9 @@ struct PostArgs {
 };
 int post_fused_max_n();
 cudaError_t launch_centroid_traj(const PostArgs& a, int C_max, cudaStream_t st);
+// cluster (DSMEM) centroid trajectory: cls[l] = circulant stride class of layer l or -1
+bool centroid_cluster_ok(int N, const int* nu, const int* cls, int t, int L);
+cudaError_t launch_centroid_cluster(const PostArgs& a, int C_max, int win_max, cudaStream_t st);
 cudaError_t launch_residual_traj(const PostArgs& a, int max_rows, int num_sms, cudaStream_t st);
 int circ_class_of(int N, int nu);
 

@@ -293,3 +293,17 @@ def test_compact_circulant_loader_equals_csc(N, L, B, t):
             g.infer(y0, t=t, s=32, kernel=KERNEL_ELL)  # no ELL copy in compact form
     assert np.array_equal(Y, ref[0]) and np.array_equal(cats, ref[1])
     assert np.array_equal(cats, oracle.categories(oracle.layers_circulant_f32(c, Y0)))
+
+
+@pytest.mark.parametrize("N,L,B,t", [(1024, 40, 800, 3), (4096, 24, 300, 3), (16384, 10, 40, 3)])
+def test_cluster_centroid_trajectory(N, L, B, t):
+    """Fused post mode: the 8-CTA cluster (DSMEM) centroid trajectory == one CTA per centroid == the
+    oracle pipeline, with residue rows present (they consume the cluster kernel's a_c)."""
+    net = sdgc.gen_network(N, L, "radix")
+    Y0 = sdgc.gen_inputs(N, B)
+    ref = oracle.snicit(net, Y0, t=t)
+    a = run_gpu(net, Y0, t=t, post_cluster=1)
+    b = run_gpu(net, Y0, t=t, post_cluster=0)
+    assert a[2]["residual_at_t"] > 0
+    for Y, cats, _, _ in (a, b):
+        assert np.array_equal(Y, ref["Y"]) and np.array_equal(cats, ref["categories"])
