@@ -339,71 +339,79 @@ constexpr int kCL = 8;
 constexpr int kClThreads = 512;
 constexpr int kClMaxWin = 16384;  // floats of the gathered input window
 
-__device__ __forceinline__ int cl_owner(int k, int part, int nu, int S, int& off) {
-    if (part == 0) {
-        const int o = k / S;
-        off = k - o * S;
-        return o;
-    }
-    const int a = k / nu, c = k - a * nu;
-    const int cs = nu / kCL;
-    const int o = c / cs;
-    off = a * cs + (c - o * cs);
-    return o;
-}
+__device__ __forceinline__ int ilog2(int x) { return 31 - __clz(x); }
 
 __global__ void __cluster_dims__(kCL, 1, 1) __launch_bounds__(kClThreads) centroid_cluster_kernel(PostArgs a) {
     extern __shared__ __align__(128) float sm[];
+    __shared__ float* s_rbase[2][kCL];  // peers' slice buffers (cluster-mapped generic pointers)
     cg::cluster_group cl = cg::this_cluster();
     const int r = (int)cl.block_rank();
     const int cid = blockIdx.x / kCL;
     const int C = *a.n_cent;
     if (cid >= C) return;  // uniform over the cluster
-    const int N = a.N, S = N / kCL;
+    const int N = a.N, S = N / kCL;  // powers of two (centroid_cluster_ok)
+    const int shS = ilog2(S);
     float* slice[2] = {sm, sm + S};
     float* win = sm + 2 * S;
+    if (threadIdx.x < 2 * kCL) {
+        const int bsel = threadIdx.x / kCL, o = threadIdx.x % kCL;
+        s_rbase[bsel][o] = cl.map_shared_rank(slice[bsel], o);
+    }
     for (int i = threadIdx.x; i < S; i += blockDim.x) slice[0][i] = a.cbuf[(size_t)cid * N + r * S + i];
     int prev_part = 0, prev_nu = 1, cur = 0;
     cl.sync();
     PL Ld = load_pl(a.layers + a.t);
     for (int l = a.t; l < a.L; ++l) {
         const PL Lnext = load_pl(a.layers + min(l + 1, a.L - 1));
-        const int nu = Ld.nu, Q = N / nu, cls = Ld.cls;
+        const int nu = Ld.nu, cls = Ld.cls;
+        const int shnu = ilog2(nu), Q = N >> shnu;
         const int part = cls == PCLS_Q32 ? 1 : 0;
         const float w0 = Ld.w0, b0 = Ld.b0;
         const bool ubias = Ld.ubias != 0, unif = Ld.unif != 0;
         const float* __restrict__ bias = Ld.bias;
         float wr[kPK];
+        if (unif) {
 #pragma unroll
-        for (int n = 0; n < kPK; ++n) wr[n] = unif ? w0 : __ldg(Ld.wtab + n);
+            for (int n = 0; n < kPK; ++n) wr[n] = w0;
+        } else {
+#pragma unroll
+            for (int n = 0; n < kPK; ++n) wr[n] = __ldg(Ld.wtab + n);
+        }
         float* aout = a.a_all ? a.a_all + ((size_t)(l - a.t) * a.s + cid) * N : nullptr;
         // ---- gather this CTA's input window from the peers' slices (previous layer's outputs)
-        const float* src = slice[cur];
-        auto fetch = [&](int k) -> float {
-            int off;
-            const int o = cl_owner(k, prev_part, prev_nu, S, off);
-            const float* p = cl.map_shared_rank(src, o);
-            return p[off];
+        float* const* rb = s_rbase[cur];
+        const int shnp = ilog2(prev_nu);
+        const int shcp = prev_part ? shnp - 3 : 0;  // log2(prev_nu / kCL)
+        auto fetch = [&](int k) -> float {           // element k of the previous layer's row
+            int o, off;
+            if (prev_part == 0) {
+                o = k >> shS;
+                off = k & (S - 1);
+            } else {
+                const int aa = k >> shnp, c = k & (prev_nu - 1);
+                o = c >> shcp;
+                off = (aa << shcp) | (c & ((1 << shcp) - 1));
+            }
+            return rb[o][off];
         };
-        int wlen, q0 = 0, a_s = 0, c0 = 0, cs = 0;
+        int q0 = 0, a_s = 0, c0 = 0, cs = 0, shcs = 0;
         if (cls == PCLS_NU1) {
             q0 = r * S;
-            wlen = S + kPK;
-            for (int i = threadIdx.x; i < wlen; i += blockDim.x) win[i] = fetch((q0 + i) % N);
+            for (int i = threadIdx.x; i < S + kPK; i += blockDim.x) win[i] = fetch((q0 + i) & (N - 1));
         } else if (cls == PCLS_GEN) {
-            a_s = r * (S / nu);
-            wlen = (S / nu + kPK) * nu;
+            a_s = r * (S >> shnu);
+            const int wlen = ((S >> shnu) + kPK) << shnu;
             for (int i = threadIdx.x; i < wlen; i += blockDim.x) {
-                const int aa = i / nu, c = i - aa * nu;
-                win[i] = fetch(((a_s + aa) % Q) * nu + c);
+                const int aa = i >> shnu, c = i & (nu - 1);
+                win[i] = fetch((((a_s + aa) & (Q - 1)) << shnu) | c);
             }
         } else {
-            cs = nu / kCL;
+            shcs = shnu - 3;
+            cs = nu >> 3;
             c0 = r * cs;
-            wlen = 32 * cs;
-            for (int i = threadIdx.x; i < wlen; i += blockDim.x) {
-                const int aa = i / cs, cc = i - aa * cs;
-                win[i] = fetch(aa * nu + c0 + cc);
+            for (int i = threadIdx.x; i < (32 << shcs); i += blockDim.x) {
+                const int aa = i >> shcs, cc = i & (cs - 1);
+                win[i] = fetch((aa << shnu) + c0 + cc);
             }
         }
         __syncthreads();
@@ -433,35 +441,35 @@ __global__ void __cluster_dims__(kCL, 1, 1) __launch_bounds__(kClThreads) centro
             }
         } else if (cls == PCLS_GEN) {
             constexpr int M = 4, WIN = M + kPK - 1;
-            const int na = S / nu;
+            const int na = S >> shnu;
             for (int it = threadIdx.x; it < nu * ((na + M - 1) / M); it += blockDim.x) {
-                const int c = it % nu, al = (it / nu) * M;
+                const int c = it & (nu - 1), al = (it >> shnu) * M;
                 float R[WIN];
 #pragma unroll
-                for (int i = 0; i < WIN; ++i) R[i] = win[(al + i) * nu + c];
+                for (int i = 0; i < WIN; ++i) R[i] = win[((al + i) << shnu) + c];
 #pragma unroll
                 for (int m = 0; m < M; ++m) {
                     if (al + m < na) {
                         float acc = 0.0f;
 #pragma unroll
                         for (int n = 0; n < kPK; ++n) acc = fmaf(R[m + n], wr[n], acc);
-                        emit(acc, (a_s + al + m) * nu + c, (al + m) * nu + c);
+                        emit(acc, ((a_s + al + m) << shnu) + c, ((al + m) << shnu) + c);
                     }
                 }
             }
         } else {
             constexpr int OG = 4;
             for (int it = threadIdx.x; it < cs * (32 / OG); it += blockDim.x) {
-                const int cc = it % cs, g0 = (it / cs) * OG;
+                const int cc = it & (cs - 1), g0 = (it >> shcs) * OG;
                 float R[32];
 #pragma unroll
-                for (int j = 0; j < 32; ++j) R[j] = win[((g0 + j) & 31) * cs + cc];
+                for (int j = 0; j < 32; ++j) R[j] = win[(((g0 + j) & 31) << shcs) + cc];
 #pragma unroll
                 for (int mm = 0; mm < OG; ++mm) {
                     float acc = 0.0f;
 #pragma unroll
                     for (int n = 0; n < kPK; ++n) acc = fmaf(R[(mm + n) & 31], wr[n], acc);
-                    emit(acc, (g0 + mm) * nu + c0 + cc, (g0 + mm) * cs + cc);
+                    emit(acc, ((g0 + mm) << shnu) + c0 + cc, ((g0 + mm) << shcs) + cc);
                 }
             }
         }
@@ -486,11 +494,12 @@ __global__ void __cluster_dims__(kCL, 1, 1) __launch_bounds__(kClThreads) centro
 }
 
 // host: can the cluster kernel carry layers [t, L)?  (every layer circulant, partition-compatible)
+static bool pow2(int x) { return x > 0 && (x & (x - 1)) == 0; }
 bool centroid_cluster_ok(int N, const int* nu, const int* cls, int t, int L) {
-    if (N % (kCL * 4) != 0) return false;
+    if (!pow2(N) || N < kCL * 64) return false;  // shift/mask index arithmetic
     const int S = N / kCL;
     for (int l = t; l < L; ++l) {
-        if (cls[l] < 0) return false;  // not circulant (or ELL forced)
+        if (cls[l] < 0 || !pow2(nu[l])) return false;  // not circulant (or ELL forced)
         if (cls[l] == PCLS_NU1) {
             if (S + kPK > kClMaxWin) return false;
         } else if (cls[l] == PCLS_Q32) {
