@@ -397,7 +397,8 @@ __global__ void __cluster_dims__(kCL, 1, 1) __launch_bounds__(kClThreads) centro
         int q0 = 0, a_s = 0, c0 = 0, cs = 0, shcs = 0;
         if (cls == PCLS_NU1) {
             q0 = r * S;
-            for (int i = threadIdx.x; i < S + kPK; i += blockDim.x) win[i] = fetch((q0 + i) & (N - 1));
+            // S + 40 >= the last item's window end (a0 + M + 31 with a0 < S, M = 5)
+            for (int i = threadIdx.x; i < S + 40; i += blockDim.x) win[i] = fetch((q0 + i) & (N - 1));
         } else if (cls == PCLS_GEN) {
             a_s = r * (S >> shnu);
             const int wlen = ((S >> shnu) + kPK) << shnu;
@@ -501,7 +502,7 @@ bool centroid_cluster_ok(int N, const int* nu, const int* cls, int t, int L) {
     for (int l = t; l < L; ++l) {
         if (cls[l] < 0 || !pow2(nu[l])) return false;  // not circulant (or ELL forced)
         if (cls[l] == PCLS_NU1) {
-            if (S + kPK > kClMaxWin) return false;
+            if (S + 40 > kClMaxWin) return false;
         } else if (cls[l] == PCLS_Q32) {
             if (nu[l] % kCL != 0) return false;
         } else {

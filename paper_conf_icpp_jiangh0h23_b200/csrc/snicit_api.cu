@@ -812,7 +812,7 @@ snicit_status snicit_infer(snicit_network* net, const float* y0, int64_t batch, 
                     nus[l] = net->plan[l].nu;
                     clss[l] = circ_class_of(N, nus[l]);
                     const int S8 = N / 8;
-                    const int w = clss[l] == 0 ? S8 + 32 : (clss[l] == 1 ? S8 : (S8 / nus[l] + 32) * nus[l]);
+                    const int w = clss[l] == 0 ? S8 + 40 : (clss[l] == 1 ? S8 : (S8 / nus[l] + 32) * nus[l]);
                     if (l >= tt) win_max = std::max(win_max, w);
                 }
             }
