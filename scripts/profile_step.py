@@ -25,9 +25,13 @@ p.add_argument("--batch", type=int, default=None)
 a = p.parse_args()
 c = sdgc.CONFIGS[a.config]
 B = a.batch or c["B"]
-net = sdgc.gen_network(c["N"], c["L"], a.mode)
 Y0 = sdgc.gen_inputs(c["N"], B)
-g = SnicitNetwork.from_network(net)
+if a.mode == "radix" and c["N"] >= 16384:  # compact circulant ABI (the CSC would be 8-32 GB)
+    cn = sdgc.gen_circulant(c["N"], c["L"])
+    g = SnicitNetwork.circulant(cn.N, cn.L, cn.nu, cn.w, cn.bias, cn.ymax)
+else:
+    net = sdgc.gen_network(c["N"], c["L"], a.mode)
+    g = SnicitNetwork.from_network(net)
 st = torch.cuda.Stream()
 g.set_stream(st)
 y0 = torch.from_numpy(Y0).cuda()
