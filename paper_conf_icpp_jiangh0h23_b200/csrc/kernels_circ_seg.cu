@@ -1,20 +1,25 @@
 // kernels_circ_seg.cu -- circulant layer kernel for large rows (N >= ~8K: C3 = 16384, C4 = 65536).
 //
 // Same arithmetic as kernels_circ.cu (the stored-order fma chain of every output, reading R12), but a
-// row no longer has to fit in shared memory: a tile is (row, segment) of about 4K outputs.
+// row no longer has to fit in shared memory: the row is cut into segments of about 4K outputs.
 //   A-segment (nu == 1, or a general stride whose staged window is small): outputs a in [a_s, a_e)
-//     (all residues c); the stage holds a-rows [a_s, a_e + 31) mod Q, i.e. the contiguous float range
-//     [a_s*nu, (a_e + 31)*nu) mod N (one or two TMA bulk copies), so windows never wrap.
+//     (all residues c); the window holds a-rows [a_s, a_e + 32) mod Q, i.e. the contiguous float range
+//     [a_s*nu, (a_e + 32)*nu) mod N (one or two TMA bulk copies), so windows never wrap.
 //   C-segment (Q == 32, or a general stride with small Q): outputs for residues c in [c_s, c_s + C_T)
-//     and every a; the stage holds a-rows 0 .. Q + 31 (the first 31 repeated for Q > 32 windows)
+//     and every a; the window holds a-rows 0 .. Q + 31 (the first 31 repeated for Q > 32 windows)
 //     of C_T contiguous floats each: one bulk copy per a-row, issued by all producer lanes.
-// The stage element (a_local, c_local) lives at a_local * P + c_local (P = nu for A-segments, C_T
-// for C-segments), outputs are written back in place and TMA-stored (one copy for A-segments, one per
-// a-row for C-segments).  A row's any-non-zero flag is OR-ed into flag_pos[list position] from every
-// segment (plain stores of 1; the ordered compaction that reads it also clears it).
+// A window element (a_local, c_local) lives at a_local * P + c_local (P = nu for A-segments, C_T for
+// C-segments); outputs are written back in place and TMA-stored (one copy for A-segments, one per
+// a-row for C-segments).
 //
-// Pipeline: as kernels_circ.cu -- one producer warp (S stages, row ids via the tile index) and 8
-// consumer warps (one work item per thread), mbarrier full/empty handshakes, no CTA-wide barriers.
+// Tiles.  PAIR (PLAIN mode): a tile is (row, segment pair {s, s + half}); both windows share the
+// stage and every consumer thread runs the same work item on both, the two windows' elements sharing
+// a register pair, so each FMA of the chain is one FFMA2 for two outputs (per-lane rounding identical
+// to fmaf).  Otherwise a tile is (row, segment).  A row's any-non-zero flag is OR-ed into
+// flag_pos[list position] (plain stores of 1; the ordered compaction that reads it also clears it).
+//
+// Pipeline: one producer warp (S stages) and 8 consumer warps (one work item per thread), mbarrier
+// full/empty handshakes, no CTA-wide barriers (as kernels_circ.cu).
 #include <cuda_runtime.h>
 
 #include "snicit_internal.cuh"
@@ -27,73 +32,77 @@ constexpr int kSegMaxStages = 6;
 
 struct SegGeom {
     int cseg;      // 0: A-segment, 1: C-segment
-    int cls;       // 0: nu == 1 (M = 17), 1: Q == 32 (whole class), 2: general (M = 16)
+    int cls;       // 0: nu == 1, 1: Q == 32 (whole class), 2: general
+    int pair;      // 1: a tile holds two segments of one row (FFMA2)
     int nseg;      // segments per row
+    int tpr;       // tiles per row (nseg, or ceil(nseg / 2) when paired)
     int A_T;       // A: a-rows of outputs per segment
     int C_T;       // C: residues per segment
-    int P;         // stage pitch (floats per staged a-row)
-    int rows_st;   // staged a-rows per segment
-    int stage;     // floats per stage (16-byte multiple)
-    int items;     // work items per (full) segment
+    int P;         // window pitch (floats per staged a-row)
+    int rows_st;   // staged a-rows per window
+    int sw;        // floats per window (16-byte multiple)
 };
 
-__host__ __device__ inline int seg_M(int cls) { return cls == 0 ? 17 : (cls == 1 ? 32 : 16); }
+// outputs per work item: nu == 1: 17 (odd -> conflict-free); general: 16 (8 paired); Q == 32: 32
+// (16 paired) outputs of one residue class per item
+__host__ __device__ constexpr int seg_M(int cls, int pair) {
+    return cls == 0 ? 17 : (cls == 1 ? (pair ? 16 : 32) : (pair ? 8 : 16));
+}
 
-static SegGeom seg_geom(int N, int nu) {
+static SegGeom seg_geom(int N, int nu, int pair) {
     SegGeom g{};
     const int Q = N / nu;
     g.cls = nu == 1 ? 0 : (Q == 32 ? 1 : 2);
-    const int M = seg_M(g.cls);
+    g.pair = pair;
+    const int M = seg_M(g.cls, pair);
     if (g.cls == 0) {  // A-segments of 256 items x 17 outputs
         g.cseg = 0;
         g.A_T = 256 * M;
         g.P = 1;
         g.rows_st = g.A_T + kSK;  // + 31-row halo, rounded so every copy is a 16-byte multiple
-        g.items = 256;
-    } else if (g.cls == 2 && (size_t)(256 / nu * M + kSK - 1) * nu <= 8192 && nu <= 256) {
-        g.cseg = 0;  // general stride, A-segments: nu residues x (A_T / 16) chunks = 256 items
+    } else if (g.cls == 2 && nu <= 256 && (size_t)(256 / nu * M + kSK) * nu <= 8192) {
+        g.cseg = 0;  // general stride, A-segments: nu residues x (A_T / M) chunks = 256 items
         g.A_T = (256 / nu) * M;
         g.P = nu;
         g.rows_st = g.A_T + kSK;
-        g.items = 256;
     } else {
-        g.cseg = 1;  // C-segments: C_T residues; Q32: one item per residue, general: Q/16 per residue
-        const int per_c = g.cls == 1 ? 1 : (Q + M - 1) / M;
+        g.cseg = 1;  // C-segments: C_T residues x (items per residue)
+        const int per_c = g.cls == 1 ? 32 / M : (Q + M - 1) / M;
         g.C_T = 256 / per_c;
         if (g.C_T > nu) g.C_T = nu;
         g.C_T &= ~3;  // 16-byte rows
         if (g.C_T < 4) g.C_T = 4;
         g.P = g.C_T;
         g.rows_st = g.cls == 1 ? 32 : Q + kSK - 1;
-        g.items = g.C_T * per_c;
     }
-    if (g.cseg == 0) {
-        const int Aall = Q;
-        g.nseg = (Aall + g.A_T - 1) / g.A_T;
-    } else {
-        g.nseg = (nu + g.C_T - 1) / g.C_T;
-    }
-    g.stage = ((g.rows_st * g.P) + 3) & ~3;
+    g.nseg = g.cseg == 0 ? (Q + g.A_T - 1) / g.A_T : (nu + g.C_T - 1) / g.C_T;
+    g.tpr = pair ? (g.nseg + 1) / 2 : g.nseg;
+    g.sw = ((g.rows_st * g.P) + 3) & ~3;
     return g;
 }
 
 bool circ_seg_supported(int N, int K, int nu) {
     if (K != kSK || nu <= 0 || N % nu != 0 || N % 4 != 0) return false;
     if ((long long)K * nu > N) return false;
-    const SegGeom g = seg_geom(N, nu);
-    if (g.cseg == 1 && (nu % 4 != 0 || g.C_T < 4)) return false;
-    if (g.cseg == 0 && g.cls == 2 && (nu % 4 != 0)) return false;
-    return (size_t)g.stage * 4 * 2 <= 200 * 1024;
+    for (int pair = 0; pair < 2; ++pair) {
+        const SegGeom g = seg_geom(N, nu, pair);
+        if (g.cseg == 1 && (nu % 4 != 0 || g.C_T < 4)) return false;
+        if (g.cseg == 0 && g.cls == 2 && (nu % 4 != 0)) return false;
+        if ((size_t)g.sw * 4 * (pair ? 2 : 1) * 2 > 200 * 1024) return false;
+    }
+    return true;
 }
 
-template <int MODE, bool UNIF, bool UBIAS>
+template <int MODE, bool UNIF, bool UBIAS, bool PAIR>
 __global__ void __launch_bounds__(kSegThreads + 32, 2) layer_circ_seg_kernel(LayerArgs a, SegGeom g, int S) {
+    constexpr int NW = PAIR ? 2 : 1;  // windows per tile
     extern __shared__ __align__(128) unsigned char smem[];
     const int N = a.N;
     const int nu = a.nu;
     const int Q = N / nu;
+    const int tstage = NW * g.sw;
     float* s_st = reinterpret_cast<float*>(smem);
-    uint64_t* bars = reinterpret_cast<uint64_t*>(s_st + (size_t)S * g.stage);
+    uint64_t* bars = reinterpret_cast<uint64_t*>(s_st + (size_t)S * tstage);
     uint64_t* in_full = bars;
     uint64_t* out_full = bars + S;
     int* s_row = reinterpret_cast<int*>(bars + 2 * S);  // [S]
@@ -102,7 +111,7 @@ __global__ void __launch_bounds__(kSegThreads + 32, 2) layer_circ_seg_kernel(Lay
     constexpr int kConsumerWarps = kSegThreads / 32;
 
     const int count = *a.count;
-    const long long ntiles = (long long)count * g.nseg;
+    const long long ntiles = (long long)count * g.tpr;
     const long long tpc = (ntiles + gridDim.x - 1) / gridDim.x;
     const long long t_begin = (long long)blockIdx.x * tpc;
     const int my_tiles = (int)max(0LL, min(ntiles, t_begin + tpc) - t_begin);
@@ -116,76 +125,92 @@ __global__ void __launch_bounds__(kSegThreads + 32, 2) layer_circ_seg_kernel(Lay
     }
     __syncthreads();
 
+    // segment geometry: [lo, lo + n) a-rows (A) or residues (C); segment id >= nseg: absent (n = 0)
+    auto seg_range = [&](int seg, int& lo, int& n) {
+        if (seg >= g.nseg) {
+            lo = 0;
+            n = 0;
+        } else if (g.cseg == 0) {
+            lo = seg * g.A_T;
+            n = min(g.A_T, Q - lo);
+        } else {
+            lo = seg * g.C_T;
+            n = min(g.C_T, nu - lo);
+        }
+    };
+    auto win_bytes = [&](int n) -> uint32_t {
+        if (n == 0) return 0u;
+        return g.cseg == 0 ? (uint32_t)((n + kSK) * nu * 4) : (uint32_t)g.rows_st * (uint32_t)n * 4;
+    };
+
     if (threadIdx.x >= kSegThreads) {
         // ------------------------------------------------------------ producer / storer warp
         const int lane = threadIdx.x & 31;
-        auto seg_range = [&](int seg, int& lo, int& n) {  // a-range (A) or residue range (C)
-            if (g.cseg == 0) {
-                lo = seg * g.A_T;
-                n = min(g.A_T, Q - lo);
-            } else {
-                lo = seg * g.C_T;
-                n = min(g.C_T, nu - lo);
-            }
-        };
-        auto load = [&](int j) {
-            const int b = j % S;
-            const long long tile = t_begin + j;
-            const int pos = (int)(tile / g.nseg), seg = (int)(tile % g.nseg);
-            const int row = a.rows[pos];
+        auto load_window = [&](const float* gr, int seg, float* st, uint64_t* bar) {
             int lo, n;
             seg_range(seg, lo, n);
-            const float* gr = a.yin + (size_t)row * N;
-            float* st = s_st + (size_t)b * g.stage;
-            uint32_t bytes;
+            if (n == 0) return;
             if (g.cseg == 0) {
-                const long long f0 = (long long)lo * nu;
-                const long long f1 = (long long)(lo + n + kSK) * nu;  // exclusive, may pass N (wraps)
-                bytes = (uint32_t)((f1 - f0) * 4);
                 if (lane == 0) {
-                    s_row[b] = row;
-                    s_flag[b] = 0;
-                    if constexpr (MODE == MODE_RESIDUAL) s_slot[b] = a.cslot[row];
-                    mbar_arrive_expect_tx(&in_full[b], bytes);
+                    const long long f0 = (long long)lo * nu;
+                    const long long f1 = (long long)(lo + n + kSK) * nu;  // exclusive, may pass N (wraps)
                     const long long e0 = min(f1, (long long)N);
-                    bulk_g2s(st, gr + f0, (uint32_t)((e0 - f0) * 4), &in_full[b]);
+                    bulk_g2s(st, gr + f0, (uint32_t)((e0 - f0) * 4), bar);
                     long long done = e0 - f0;
                     while (f0 + done < f1) {  // wrap: continue from the row head
                         const long long len = min(f1 - f0 - done, (long long)N);
-                        bulk_g2s(st + done, gr, (uint32_t)(len * 4), &in_full[b]);
+                        bulk_g2s(st + done, gr, (uint32_t)(len * 4), bar);
                         done += len;
                     }
                 }
             } else {
-                bytes = (uint32_t)g.rows_st * (uint32_t)n * 4;
-                if (lane == 0) {
-                    s_row[b] = row;
-                    s_flag[b] = 0;
-                    if constexpr (MODE == MODE_RESIDUAL) s_slot[b] = a.cslot[row];
-                    mbar_arrive_expect_tx(&in_full[b], bytes);
-                }
-                __syncwarp();
                 for (int r = lane; r < g.rows_st; r += 32)
-                    bulk_g2s(st + (size_t)r * g.P, gr + (size_t)(r % Q) * nu + lo, (uint32_t)n * 4, &in_full[b]);
+                    bulk_g2s(st + (size_t)r * g.P, gr + (size_t)(r % Q) * nu + lo, (uint32_t)n * 4, bar);
             }
-            __syncwarp();
         };
-        auto store = [&](int j) {
-            const int b = j % S;
-            const long long tile = t_begin + j;
-            const int pos = (int)(tile / g.nseg), seg = (int)(tile % g.nseg);
+        auto store_window = [&](float* gr, int seg, const float* st) {
             int lo, n;
             seg_range(seg, lo, n);
-            if (lane == 0) mbar_wait(&out_full[b], (uint32_t)((j / S) & 1));
-            __syncwarp();
-            const int row = s_row[b];
-            float* gr = a.yout + (size_t)row * N;
-            const float* st = s_st + (size_t)b * g.stage;
+            if (n == 0) return;
             if (g.cseg == 0) {
                 if (lane == 0) bulk_s2g(gr + (size_t)lo * nu, st, (uint32_t)n * nu * 4);
             } else {
                 for (int r = lane; r < Q; r += 32) bulk_s2g(gr + (size_t)r * nu + lo, st + (size_t)r * g.P, (uint32_t)n * 4);
             }
+        };
+        auto load = [&](int j) {
+            const int b = j % S;
+            const long long tile = t_begin + j;
+            const int pos = (int)(tile / g.tpr), tp = (int)(tile % g.tpr);
+            const int row = a.rows[pos];
+            const int sa = tp, sb = PAIR ? tp + g.tpr : g.nseg;
+            int lo, na, nb;
+            seg_range(sa, lo, na);
+            seg_range(sb, lo, nb);
+            const float* gr = a.yin + (size_t)row * N;
+            float* st = s_st + (size_t)b * tstage;
+            if (lane == 0) {
+                s_row[b] = row;
+                s_flag[b] = 0;
+                if constexpr (MODE == MODE_RESIDUAL) s_slot[b] = a.cslot[row];
+                mbar_arrive_expect_tx(&in_full[b], win_bytes(na) + (PAIR ? win_bytes(nb) : 0u));
+            }
+            __syncwarp();
+            load_window(gr, sa, st, &in_full[b]);
+            if constexpr (PAIR) load_window(gr, sb, st + g.sw, &in_full[b]);
+            __syncwarp();
+        };
+        auto store = [&](int j) {
+            const int b = j % S;
+            const long long tile = t_begin + j;
+            const int pos = (int)(tile / g.tpr), tp = (int)(tile % g.tpr);
+            if (lane == 0) mbar_wait(&out_full[b], (uint32_t)((j / S) & 1));
+            __syncwarp();
+            const int row = s_row[b];
+            float* gr = a.yout + (size_t)row * N;
+            const float* st = s_st + (size_t)b * tstage;
+            store_window(gr, tp, st);
+            if constexpr (PAIR) store_window(gr, tp + g.tpr, st + g.sw);
             if (lane == 0 && s_flag[b]) {
                 if (a.flag_pos) a.flag_pos[pos] = 1;
                 if (a.flag_row) a.flag_row[row] = 1;
@@ -204,6 +229,9 @@ __global__ void __launch_bounds__(kSegThreads + 32, 2) layer_circ_seg_kernel(Lay
     }
 
     // ---------------------------------------------------------------- consumers
+    constexpr int MG = seg_M(2, PAIR);  // general class
+    constexpr int OQ = seg_M(1, PAIR);  // Q == 32 class
+    constexpr int VM = 32;              // max outputs per item
     float w[UNIF ? 1 : kSK];
     if constexpr (!UNIF) {
 #pragma unroll
@@ -211,109 +239,170 @@ __global__ void __launch_bounds__(kSegThreads + 32, 2) layer_circ_seg_kernel(Lay
     }
     const float w0 = a.w0;
     const float b0 = UBIAS ? __ldg(a.bias) : 0.0f;
+    const unsigned long long W2 = f2_pack(w0, w0);
     const int lane = threadIdx.x & 31;
     const int item = threadIdx.x;
     const int P = g.P;
     for (int j = 0; j < my_tiles; ++j) {
         const int b = j % S;
         const long long tile = t_begin + j;
-        const int seg = (int)(tile % g.nseg);
+        const int tp = (int)(tile % g.tpr);
         mbar_wait(&in_full[b], (uint32_t)((j / S) & 1));
-        float* st = s_st + (size_t)b * g.stage;
+        float* stA = s_st + (size_t)b * tstage;
+        float* stB = stA + g.sw;  // PAIR only
         const int row = s_row[b];
         const int slot = (MODE == MODE_RESIDUAL) ? s_slot[b] : 0;
-        float v[32];
-        int n_out = 0, ob = 0, os = 1;
-        bool have = false;
-        auto fin = [&](float acc, int q, int m, bool valid) {
+        int loA, nA, loB = 0, nB = 0;
+        seg_range(tp, loA, nA);
+        if constexpr (PAIR) seg_range(tp + g.tpr, loB, nB);
+        float v0[VM], v1[PAIR ? VM : 1];
+        int nv0 = 0, nv1 = 0, ob = 0, os = 1;
+        // one output of the single window: global index q, validity (no side effects if invalid)
+        auto fin1 = [&](float acc, int q, int m, bool valid) {
             const float bq = UBIAS ? b0 : __ldg(a.bias + q);
-            v[m] = epilogue<MODE>(a, acc, bq, q, row, slot, valid);
+            v0[m] = epilogue<MODE>(a, acc, bq, q, row, slot, valid);
         };
-        if (g.cls == 0) {  // nu == 1, A-segment: outputs a in [lo + 17 it, ...)
+        // one output of each of the two windows (PLAIN only): FADD2 + clamp
+        auto fin2 = [&](unsigned long long acc, int qa, int qb, int m) {
+            float z0, z1;
+            const float ba = UBIAS ? b0 : __ldg(a.bias + qa), bb = UBIAS ? b0 : __ldg(a.bias + qb);
+            f2_unpack(f2_add(acc, f2_pack(ba, bb)), z0, z1);
+            v0[m] = sigma(z0, a.ymax);
+            if constexpr (PAIR) v1[m] = sigma(z1, a.ymax);
+        };
+        if (g.cls == 0) {  // nu == 1, A-segment: outputs a in [lo + 17 item, ...)
             constexpr int M = 17, WIN = M + kSK - 1;
-            const int lo = seg * g.A_T, n = min(g.A_T, Q - lo);
             const int a0 = item * M;
-            if (a0 < n) {
-                have = true;
-                float R[WIN];
-#pragma unroll
-                for (int i = 0; i < WIN; ++i) R[i] = st[a0 + i];
-                n_out = min(M, n - a0);
+            if (a0 < max(nA, nB)) {
+                nv0 = max(0, min(M, nA - a0));
+                nv1 = max(0, min(M, nB - a0));
                 ob = a0;
                 os = 1;
+                if constexpr (PAIR) {
+                    unsigned long long R[WIN];
 #pragma unroll
-                for (int m = 0; m < M; ++m) {
-                    float acc = 0.0f;
+                    for (int i = 0; i < WIN; ++i) R[i] = f2_pack(stA[a0 + i], stB[a0 + i]);
 #pragma unroll
-                    for (int k = 0; k < kSK; ++k) acc = fmaf(R[m + k], UNIF ? w0 : w[k], acc);
-                    fin(acc, lo + min(a0 + m, n - 1), m, a0 + m < n);
+                    for (int m = 0; m < M; ++m) {
+                        unsigned long long acc = 0ull;
+#pragma unroll
+                        for (int k = 0; k < kSK; ++k) acc = f2_fma(R[m + k], W2, acc);
+                        fin2(acc, loA + min(a0 + m, max(nA, 1) - 1), loB + min(a0 + m, max(nB, 1) - 1), m);
+                    }
+                } else {
+                    float R[WIN];
+#pragma unroll
+                    for (int i = 0; i < WIN; ++i) R[i] = stA[a0 + i];
+#pragma unroll
+                    for (int m = 0; m < M; ++m) {
+                        float acc = 0.0f;
+#pragma unroll
+                        for (int k = 0; k < kSK; ++k) acc = fmaf(R[m + k], UNIF ? w0 : w[k], acc);
+                        fin1(acc, loA + min(a0 + m, nA - 1), m, a0 + m < nA);
+                    }
                 }
             }
-        } else if (g.cls == 1) {  // Q == 32, C-segment: one residue per thread, all 32 a
-            const int lo = seg * g.C_T, n = min(g.C_T, nu - lo);
-            if (item < n) {
-                have = true;
-                float R[32];
-#pragma unroll
-                for (int jj = 0; jj < 32; ++jj) R[jj] = st[jj * P + item];
-                n_out = 32;
-                ob = item;
+        } else if (g.cls == 1) {  // Q == 32, C-segment: OQ outputs of one residue class per item
+            const int cc = item % g.C_T, g0 = (item / g.C_T) * OQ;
+            if (g0 < 32 && cc < max(nA, nB)) {
+                nv0 = cc < nA ? OQ : 0;
+                nv1 = cc < nB ? OQ : 0;
+                ob = g0 * P + cc;
                 os = P;
+                if constexpr (PAIR) {
+                    unsigned long long R[32];
 #pragma unroll
-                for (int m = 0; m < 32; ++m) {
-                    float acc = 0.0f;
+                    for (int jj = 0; jj < 32; ++jj) {
+                        const int ro = ((g0 + jj) & 31) * P + cc;  // rotated: compile-time indices below
+                        R[jj] = f2_pack(stA[ro], stB[ro]);
+                    }
 #pragma unroll
-                    for (int k = 0; k < kSK; ++k) acc = fmaf(R[(m + k) & 31], UNIF ? w0 : w[k], acc);
-                    fin(acc, m * nu + lo + item, m, true);
+                    for (int m = 0; m < OQ; ++m) {
+                        unsigned long long acc = 0ull;
+#pragma unroll
+                        for (int k = 0; k < kSK; ++k) acc = f2_fma(R[(m + k) & 31], W2, acc);
+                        fin2(acc, (g0 + m) * nu + loA + min(cc, max(nA, 1) - 1),
+                             (g0 + m) * nu + loB + min(cc, max(nB, 1) - 1), m);
+                    }
+                } else {
+                    float R[32];
+#pragma unroll
+                    for (int jj = 0; jj < 32; ++jj) R[jj] = stA[((g0 + jj) & 31) * P + cc];
+#pragma unroll
+                    for (int m = 0; m < OQ; ++m) {
+                        float acc = 0.0f;
+#pragma unroll
+                        for (int k = 0; k < kSK; ++k) acc = fmaf(R[(m + k) & 31], UNIF ? w0 : w[k], acc);
+                        fin1(acc, (g0 + m) * nu + loA + min(cc, nA - 1), m, cc < nA);
+                    }
                 }
             }
-        } else {  // general stride, M = 16
-            constexpr int M = 16, WIN = M + kSK - 1;
-            int c, a0, lo_a, lo_c, na;
-            bool valid;
+        } else {  // general stride
+            constexpr int M = MG, WIN = M + kSK - 1;
+            int c, a0;
+            bool active;
             if (g.cseg == 0) {
-                lo_a = seg * g.A_T;
-                lo_c = 0;
-                na = min(g.A_T, Q - lo_a);
                 c = item % nu;
                 a0 = (item / nu) * M;
-                valid = a0 < na;
+                active = a0 < max(nA, nB);
+                nv0 = max(0, min(M, nA - a0));
+                nv1 = max(0, min(M, nB - a0));
             } else {
-                lo_a = 0;
-                lo_c = seg * g.C_T;
-                na = Q;
-                const int nc = min(g.C_T, nu - lo_c);
                 c = item % g.C_T;
                 a0 = (item / g.C_T) * M;
-                valid = c < nc && a0 < Q;
+                active = a0 < Q && c < max(nA, nB);
+                nv0 = c < nA ? min(M, Q - a0) : 0;
+                nv1 = c < nB ? min(M, Q - a0) : 0;
             }
-            if (valid) {
-                have = true;
-                float R[WIN];
-#pragma unroll
-                for (int i = 0; i < WIN; ++i) R[i] = st[(a0 + i) * P + c];
-                n_out = min(M, na - a0);
+            if (active) {
                 ob = a0 * P + c;
                 os = P;
+                // global index of output m of a window (segment lo, n), clamped for discarded outputs
+                auto gq = [&](int lo, int n, int m) -> int {
+                    if (g.cseg == 0) return (lo + min(a0 + m, max(n, 1) - 1)) * nu + c;
+                    return min(a0 + m, Q - 1) * nu + lo + min(c, max(n, 1) - 1);
+                };
+                if constexpr (PAIR) {
+                    unsigned long long R[WIN];
 #pragma unroll
-                for (int m = 0; m < M; ++m) {
-                    float acc = 0.0f;
+                    for (int i = 0; i < WIN; ++i) R[i] = f2_pack(stA[(a0 + i) * P + c], stB[(a0 + i) * P + c]);
 #pragma unroll
-                    for (int k = 0; k < kSK; ++k) acc = fmaf(R[m + k], UNIF ? w0 : w[k], acc);
-                    const int am = lo_a + min(a0 + m, na - 1);
-                    fin(acc, am * nu + lo_c + c, m, a0 + m < na);
+                    for (int m = 0; m < M; ++m) {
+                        unsigned long long acc = 0ull;
+#pragma unroll
+                        for (int k = 0; k < kSK; ++k) acc = f2_fma(R[m + k], W2, acc);
+                        fin2(acc, gq(loA, nA, m), gq(loB, nB, m), m);
+                    }
+                } else {
+                    float R[WIN];
+#pragma unroll
+                    for (int i = 0; i < WIN; ++i) R[i] = stA[(a0 + i) * P + c];
+#pragma unroll
+                    for (int m = 0; m < M; ++m) {
+                        float acc = 0.0f;
+#pragma unroll
+                        for (int k = 0; k < kSK; ++k) acc = fmaf(R[m + k], UNIF ? w0 : w[k], acc);
+                        fin1(acc, gq(loA, nA, m), m, m < nv0);
+                    }
                 }
+            } else {
+                nv0 = nv1 = 0;
             }
         }
         asm volatile("bar.sync 2, %0;" ::"n"(kSegThreads) : "memory");  // all stage reads done
         float mx = 0.0f;
-        if (have) {
 #pragma unroll
-            for (int m = 0; m < 32; ++m)
-                if (m < n_out) {
-                    st[ob + m * os] = v[m];
-                    mx = fmaxf(mx, fabsf(v[m]));
+        for (int m = 0; m < VM; ++m) {
+            if (m < nv0) {
+                stA[ob + m * os] = v0[m];
+                mx = fmaxf(mx, fabsf(v0[m]));
+            }
+            if constexpr (PAIR) {
+                if (m < nv1) {
+                    stB[ob + m * os] = v1[m];
+                    mx = fmaxf(mx, fabsf(v1[m]));
                 }
+            }
         }
         const unsigned any = __ballot_sync(0xffffffffu, mx != 0.0f);
         if (lane == 0 && any) s_flag[b] = 1;
@@ -325,15 +414,17 @@ __global__ void __launch_bounds__(kSegThreads + 32, 2) layer_circ_seg_kernel(Lay
 
 template <int MODE, bool UNIF, bool UBIAS>
 static cudaError_t launch_seg_t(const LayerArgs& a, int max_rows, int num_sms, cudaStream_t st) {
-    const SegGeom g = seg_geom(a.N, a.nu);
+    constexpr bool PAIR = MODE == MODE_PLAIN && UNIF;
+    const SegGeom g = seg_geom(a.N, a.nu, PAIR ? 1 : 0);
+    const size_t tstage = (size_t)(PAIR ? 2 : 1) * g.sw * 4;
     int S = kSegMaxStages;
-    while (S > 2 && (size_t)S * g.stage * 4 + 64 * S > 110 * 1024) --S;
-    const size_t smem = (size_t)S * g.stage * 4 + 2 * S * sizeof(uint64_t) + 3 * S * sizeof(int);
-    auto kern = layer_circ_seg_kernel<MODE, UNIF, UBIAS>;
+    while (S > 2 && (size_t)S * tstage + 64 * S > 110 * 1024) --S;
+    const size_t smem = (size_t)S * tstage + 2 * S * sizeof(uint64_t) + 3 * S * sizeof(int);
+    auto kern = layer_circ_seg_kernel<MODE, UNIF, UBIAS, PAIR>;
     int per_sm = 1;
     cudaError_t e = blocks_per_sm((const void*)kern, kSegThreads + 32, smem, &per_sm);
     if (e != cudaSuccess) return e;
-    long long tiles = (long long)max_rows * g.nseg;
+    long long tiles = (long long)max_rows * g.tpr;
     int grid = num_sms * per_sm;
     if (grid > tiles) grid = (int)tiles;
     if (grid < 1) grid = 1;
