@@ -412,9 +412,8 @@ __global__ void __launch_bounds__(kSegThreads + 32, 2) layer_circ_seg_kernel(Lay
     }
 }
 
-template <int MODE, bool UNIF, bool UBIAS>
+template <int MODE, bool UNIF, bool UBIAS, bool PAIR>
 static cudaError_t launch_seg_t(const LayerArgs& a, int max_rows, int num_sms, cudaStream_t st) {
-    constexpr bool PAIR = MODE == MODE_PLAIN && UNIF;
     const SegGeom g = seg_geom(a.N, a.nu, PAIR ? 1 : 0);
     const size_t tstage = (size_t)(PAIR ? 2 : 1) * g.sw * 4;
     int S = kSegMaxStages;
@@ -435,10 +434,15 @@ static cudaError_t launch_seg_t(const LayerArgs& a, int max_rows, int num_sms, c
 template <int MODE>
 static cudaError_t launch_seg_m(const LayerArgs& a, int max_rows, int num_sms, cudaStream_t st) {
     const bool unif = a.wtab == nullptr, ub = a.uniform_bias != 0;
-    if (unif && ub) return launch_seg_t<MODE, true, true>(a, max_rows, num_sms, st);
-    if (unif) return launch_seg_t<MODE, true, false>(a, max_rows, num_sms, st);
-    if (ub) return launch_seg_t<MODE, false, true>(a, max_rows, num_sms, st);
-    return launch_seg_t<MODE, false, false>(a, max_rows, num_sms, st);
+    // paired segments (FFMA2) for nu == 1 PLAIN layers: measured faster there; for the strided classes
+    // the paired windows halve the copy granularity and the kernel becomes copy-issue-bound
+    const bool pair = MODE == MODE_PLAIN && unif && a.nu == 1;
+    if (pair && ub) return launch_seg_t<MODE, true, true, MODE == MODE_PLAIN>(a, max_rows, num_sms, st);
+    if (pair) return launch_seg_t<MODE, true, false, MODE == MODE_PLAIN>(a, max_rows, num_sms, st);
+    if (unif && ub) return launch_seg_t<MODE, true, true, false>(a, max_rows, num_sms, st);
+    if (unif) return launch_seg_t<MODE, true, false, false>(a, max_rows, num_sms, st);
+    if (ub) return launch_seg_t<MODE, false, true, false>(a, max_rows, num_sms, st);
+    return launch_seg_t<MODE, false, false, false>(a, max_rows, num_sms, st);
 }
 
 cudaError_t launch_layer_circ_seg(const LayerArgs& a, int mode, int max_rows, int num_sms, cudaStream_t st) {
