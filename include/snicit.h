@@ -53,7 +53,9 @@ typedef enum {
 typedef enum {
     SNICIT_KERNEL_AUTO = 0, /* shift-invariant layers use the circulant kernel, others ELL */
     SNICIT_KERNEL_ELL = 1,  /* force the general gather kernel on every layer */
-    SNICIT_KERNEL_CIRC = 2  /* require the circulant kernel (error if a layer is not eligible) */
+    SNICIT_KERNEL_CIRC = 2, /* require the circulant kernel (error if a layer is not eligible) */
+    SNICIT_KERNEL_CIRC_SMEM = 3 /* as CIRC, but strided layers use the shared-memory staged kernels
+                                   instead of the column-streaming kernel (A/B and parity tests) */
 } snicit_kernel;
 
 /* SNICIT parameters (s = 32, t = 30, n = 16, eps = eta = 0.03 for SDGC;
@@ -179,7 +181,7 @@ snicit_status snicit_debug_clustering(snicit_network* net, int32_t* cent, int32_
                                       uint8_t* live_t);
 
 /* One plain layer (Eq. 1) of the loaded network on `rows` device rows: yout = sigma(yin . W(l) + b(l)).
- * kernel: SNICIT_KERNEL_ELL or SNICIT_KERNEL_CIRC (error if not eligible) or AUTO.
+ * kernel: SNICIT_KERNEL_ELL, SNICIT_KERNEL_CIRC / SNICIT_KERNEL_CIRC_SMEM (error if not eligible) or AUTO.
  * yin, yout: device pointers, rows*N fp32, must not alias. */
 snicit_status snicit_debug_layer(snicit_network* net, int32_t layer, const float* yin,
                                  float* yout, int64_t rows, int32_t kernel);

@@ -18,7 +18,7 @@ SNICIT_OK = 0
 STATUS_NAMES = {0: "OK", -1: "E_INVALID_ARG", -2: "E_BAD_SPARSE", -3: "E_OOM", -4: "E_CUDA", -5: "E_STATE",
                 -6: "E_UNSUPPORTED"}
 CSC, CSR = 0, 1
-KERNEL_AUTO, KERNEL_ELL, KERNEL_CIRC = 0, 1, 2
+KERNEL_AUTO, KERNEL_ELL, KERNEL_CIRC, KERNEL_CIRC_SMEM = 0, 1, 2, 3
 
 EXPORTED = ["snicit_default_options", "snicit_load_network", "snicit_set_stream", "snicit_infer",
             "snicit_categories", "snicit_stats", "snicit_debug_clustering", "snicit_debug_layer",

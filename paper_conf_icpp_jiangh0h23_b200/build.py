@@ -7,7 +7,7 @@ import subprocess
 HERE = os.path.dirname(os.path.abspath(__file__))
 CSRC = os.path.join(HERE, "csrc")
 OUT = os.path.join(HERE, "lib", "libsnicit.so")
-SOURCES = ["snicit_api.cu", "kernels_layer.cu", "kernels_circ.cu", "kernels_circ_seg.cu", "kernels_post.cu", "kernels_convert.cu"]
+SOURCES = ["snicit_api.cu", "kernels_layer.cu", "kernels_circ.cu", "kernels_circ_seg.cu", "kernels_circ_col.cu", "kernels_post.cu", "kernels_convert.cu"]
 HEADERS = ["snicit_internal.cuh", os.path.join("..", "..", "include", "snicit.h")]
 NVCC_FLAGS = ["-gencode", "arch=compute_100a,code=sm_100a", "-O3", "-lineinfo", "-std=c++17",
               "-Xcompiler", "-fPIC", "-shared"]
@@ -21,13 +21,29 @@ def nvcc_path() -> str:
 
 
 def build(force: bool = False, verbose: bool = False) -> str:
-    deps = [os.path.join(CSRC, s) for s in SOURCES + HEADERS]
-    if not force and os.path.exists(OUT) and os.path.getmtime(OUT) >= max(os.path.getmtime(d) for d in deps):
+    """Compile each .cu to an object in parallel (only those older than their sources/headers unless
+    `force`), then link libsnicit.so."""
+    from concurrent.futures import ThreadPoolExecutor
+
+    hdr_t = max(os.path.getmtime(os.path.join(CSRC, h)) for h in HEADERS)
+    objdir = os.path.join(HERE, "lib", "obj")
+    os.makedirs(objdir, exist_ok=True)
+    objs = [os.path.join(objdir, s[:-3] + ".o") for s in SOURCES]
+    stale = [i for i, (s, o) in enumerate(zip(SOURCES, objs))
+             if force or not os.path.exists(o) or os.path.getmtime(o) < max(hdr_t, os.path.getmtime(os.path.join(CSRC, s)))]
+    if not stale and os.path.exists(OUT) and os.path.getmtime(OUT) >= max(os.path.getmtime(o) for o in objs):
         return OUT
-    os.makedirs(os.path.dirname(OUT), exist_ok=True)
+    flags = [f for f in NVCC_FLAGS if f != "-shared"]
+
+    def compile_one(i: int) -> None:
+        cmd = [nvcc_path()] + flags + (["-Xptxas", "-v"] if verbose else []) + ["-c", SOURCES[i], "-o", objs[i] + ".tmp"]
+        subprocess.check_call(cmd, cwd=CSRC)
+        os.replace(objs[i] + ".tmp", objs[i])
+
+    with ThreadPoolExecutor(max_workers=max(1, min(len(stale), os.cpu_count() or 1))) as ex:
+        list(ex.map(compile_one, stale))
     tmp = OUT + ".tmp"
-    cmd = [nvcc_path()] + NVCC_FLAGS + (["-Xptxas", "-v"] if verbose else []) + ["-o", tmp] + SOURCES
-    subprocess.check_call(cmd, cwd=CSRC)
+    subprocess.check_call([nvcc_path(), "-gencode", "arch=compute_100a,code=sm_100a", "-shared", "-o", tmp] + objs, cwd=CSRC)
     os.replace(tmp, OUT)
     return OUT
 

@@ -82,6 +82,7 @@ struct snicit_network {
     DevBuf<float> val_d;
     DevBuf<uint8_t> len_d;
     DevBuf<float> wtab_d;
+    std::vector<float> wtab_h;  // host copy (weights passed as kernel parameters)
     DevBuf<float> bias_d;
     DevBuf<PostLayer> post_layers_d;  // per-layer descriptors for the fused post-convergence kernels
     DevBuf<float> a_all;              // [(L - t)][s][N] centroid pre-activations (fused post mode)
@@ -163,6 +164,7 @@ static cudaError_t upload(B& buf, const T* host, size_t count) {
 // weight table, bias, fused-post layer descriptors, counters, events (after the ELL arrays, if any)
 static cudaError_t net_upload_common(snicit_network* net, const float* bias, const std::vector<float>& wtab) {
     const int N = net->N, L = net->L;
+    net->wtab_h = wtab;
     cudaError_t e = upload(net->wtab_d, wtab.data(), wtab.size());
     if (e == cudaSuccess) e = upload(net->bias_d, bias, (size_t)L * N);
     if (e == cudaSuccess) {
@@ -376,6 +378,7 @@ snicit_status snicit_load_network(int32_t N, int32_t L, snicit_format fmt, const
                 }
             if (circ) {
                 pl.kind = circ_supported(N, K, nu) ? 1 : 2;  // whole rows staged, or segmented rows
+                pl.col = circ_col_supported(N, K, nu);
                 pl.nu = nu;
                 pl.w_off = wtab.size();
                 for (int n = 0; n < K; ++n) wtab.push_back(cval[0][n]);
@@ -476,6 +479,7 @@ snicit_status snicit_load_network_circulant(int32_t N, int32_t L, const int32_t*
         }
         LayerPlan& pl = net->plan[l];
         pl.kind = circ_supported(N, K, v) ? 1 : 2;
+        pl.col = circ_col_supported(N, K, v);
         pl.nu = v;
         pl.K = K;
         pl.ragged = false;
@@ -538,6 +542,7 @@ static LayerArgs layer_args(snicit_network* net, int l, bool force_ell) {
     if (pl.kind != 0 && !force_ell) {
         a.nu = pl.nu;
         a.wtab = pl.uniform ? nullptr : net->wtab_d.p + pl.w_off;
+        a.wtab_host = pl.uniform ? nullptr : net->wtab_h.data() + pl.w_off;
     }
     return a;
 }
@@ -551,8 +556,15 @@ static bool use_circ(const snicit_network* net, int l, int kernel_opt) {
 static bool use_seg(const snicit_network* net, int l, int kernel_opt) {
     return use_circ(net, l, kernel_opt) && net->plan[l].kind == 2;
 }
+// strided circulant layers in PLAIN mode: the column-streaming kernel (rows from global memory, row
+// flags OR-ed like the segmented kernel) unless SNICIT_KERNEL_CIRC_SMEM asks for the staged kernels
+static bool use_col(const snicit_network* net, int l, int kernel_opt) {
+    return use_circ(net, l, kernel_opt) && kernel_opt != SNICIT_KERNEL_CIRC_SMEM && net->plan[l].col;
+}
 
 static cudaError_t run_layer(snicit_network* net, int l, int kernel_opt, int mode, LayerArgs a, int max_rows) {
+    if (mode == MODE_PLAIN && use_col(net, l, kernel_opt))
+        return launch_layer_circ_col(a, max_rows, net->num_sms, net->stream);
     if (use_seg(net, l, kernel_opt)) return launch_layer_circ_seg(a, mode, max_rows, net->num_sms, net->stream);
     if (use_circ(net, l, kernel_opt)) return launch_layer_circ(a, mode, max_rows, net->num_sms, net->stream);
     return launch_layer_ell(a, mode, max_rows, net->num_sms, net->stream);
@@ -612,12 +624,12 @@ snicit_status snicit_infer(snicit_network* net, const float* y0, int64_t batch, 
     if (opt.n_segments < 0 || opt.n_segments > net->N) return fail(SNICIT_E_INVALID_ARG, "n_segments out of range");
     if (!(opt.eps >= 0.0f) || std::isnan(opt.eta) || !(opt.prune_eps >= 0.0f))
         return fail(SNICIT_E_INVALID_ARG, "bad eta/eps/prune_eps");
-    if (opt.kernel < 0 || opt.kernel > 2) return fail(SNICIT_E_INVALID_ARG, "bad kernel option");
+    if (opt.kernel < 0 || opt.kernel > SNICIT_KERNEL_CIRC_SMEM) return fail(SNICIT_E_INVALID_ARG, "bad kernel option");
     if (opt.post_mode < 0 || opt.post_mode > 1) return fail(SNICIT_E_INVALID_ARG, "bad post_mode");
     if (opt.kernel == SNICIT_KERNEL_ELL && !net->has_ell)
         return fail(SNICIT_E_UNSUPPORTED, "network loaded in compact circulant form has no ELL copy");
     const int N = net->N, L = net->L;
-    if (opt.kernel == SNICIT_KERNEL_CIRC)
+    if (opt.kernel == SNICIT_KERNEL_CIRC || opt.kernel == SNICIT_KERNEL_CIRC_SMEM)
         for (int l = 0; l < L; ++l)
             if (net->plan[l].kind == 0)
                 return fail(SNICIT_E_UNSUPPORTED, "layer " + std::to_string(l) + " is not circulant");
@@ -694,7 +706,7 @@ snicit_status snicit_infer(snicit_network* net, const float* y0, int64_t batch, 
         a.yout = bufs[nxt_i];
         a.rows = lists[li];
         a.count = cnt + live_ctr[ci];
-        const bool seg = use_seg(net, l, opt.kernel);
+        const bool seg = use_seg(net, l, opt.kernel) || use_col(net, l, opt.kernel);  // OR-ed row flags
         if (drop_now && !seg) {
             a.app_list = lists[li ^ 1];
             a.app_count = cnt + live_ctr[(ci + 1) % 3];
@@ -1034,7 +1046,8 @@ snicit_status snicit_debug_layer(snicit_network* net, int32_t layer, const float
     if (rows < 0 || rows > 0x7fffffffLL) return fail(SNICIT_E_INVALID_ARG, "bad rows");
     if (kernel == SNICIT_KERNEL_ELL && !net->has_ell)
         return fail(SNICIT_E_UNSUPPORTED, "network loaded in compact circulant form has no ELL copy");
-    if (kernel == SNICIT_KERNEL_CIRC && net->plan[layer].kind == 0)
+    if (kernel < 0 || kernel > SNICIT_KERNEL_CIRC_SMEM) return fail(SNICIT_E_INVALID_ARG, "bad kernel");
+    if ((kernel == SNICIT_KERNEL_CIRC || kernel == SNICIT_KERNEL_CIRC_SMEM) && net->plan[layer].kind == 0)
         return fail(SNICIT_E_UNSUPPORTED, "layer is not circulant");
     CUDA_TRY(cudaSetDevice(net->device));
     CUDA_TRY(ensure_workspace(net, rows, 1, 1));

@@ -122,6 +122,7 @@ struct LayerArgs {
     // circulant: column j reads (j + n*nu) mod N, n = 0..K-1, weight w[n] (or w0)
     int nu;
     const float* wtab;      // K per-n weights (device), nullable when uniform
+    const float* wtab_host; // the same K weights in host memory (kernels taking them as parameters)
 };
 
 struct LayerPlan {
@@ -131,6 +132,7 @@ struct LayerPlan {
     bool uniform;   // all values equal (w0)
     bool ragged;    // column lengths differ
     bool ubias;     // bias[j] identical for all j (SDGC: a constant per benchmark, Table 1)
+    bool col;       // CIRC, strided: PLAIN layers may use the column-streaming kernel
     float w0;
     size_t ell_off; // element offset of this layer in the ELL arrays
     size_t w_off;   // offset in the per-n weight table
@@ -164,6 +166,9 @@ bool circ_supported(int N, int K, int nu);
 // segmented circulant kernel (rows too large for kernels_circ.cu), kernels_circ_seg.cu
 cudaError_t launch_layer_circ_seg(const LayerArgs& a, int mode, int max_rows, int num_sms, cudaStream_t st);
 bool circ_seg_supported(int N, int K, int nu);
+// column-streaming circulant kernel for strided layers (PLAIN mode), kernels_circ_col.cu
+cudaError_t launch_layer_circ_col(const LayerArgs& a, int max_rows, int num_sms, cudaStream_t st);
+bool circ_col_supported(int N, int K, int nu);
 bool ell_smem_ok(int N);
 
 // ------------------------------------------------------------------ fused post-convergence (kernels_post.cu)

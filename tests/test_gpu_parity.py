@@ -10,7 +10,7 @@ import pytest
 torch = pytest.importorskip("torch")
 
 import oracle  # noqa: E402
-from paper_conf_icpp_jiangh0h23_b200 import KERNEL_CIRC, KERNEL_ELL, SnicitNetwork  # noqa: E402
+from paper_conf_icpp_jiangh0h23_b200 import KERNEL_CIRC, KERNEL_CIRC_SMEM, KERNEL_ELL, SnicitNetwork  # noqa: E402
 from workload import sdgc  # noqa: E402
 from workload.sdgc import Network  # noqa: E402
 
@@ -76,12 +76,40 @@ def test_layer_kernels_bit_exact(N, mode, rows):
         yin = torch.from_numpy(Y0).cuda()
         for l in range(net.L):
             ref = oracle.layers_f32(net, Y0, l, l + 1)
-            kernels = [KERNEL_ELL] + ([KERNEL_CIRC] if g.layer_is_circulant(l) else [])
+            kernels = [KERNEL_ELL] + ([KERNEL_CIRC, KERNEL_CIRC_SMEM] if g.layer_is_circulant(l) else [])
             assert g.layer_is_circulant(l) == (mode == "radix")  # N >= 16384: segmented circulant kernel
             for k in kernels:
                 out = torch.full_like(yin, float("nan"))
                 g.debug_layer(l, yin, out, kernel=k)
                 assert np.array_equal(out.cpu().numpy(), ref), f"layer {l} kernel {k}"
+
+
+@pytest.mark.parametrize("N,nus,rows", [(2048, (32, 64), 37), (3072, (32, 96), 29), (8192, (64, 256, 128), 11),
+                                         (16384, (32, 512), 5), (65536, (1024, 2048, 32), 2)])
+@pytest.mark.parametrize("uniform", [True, False])
+def test_column_stream_kernel_bit_exact(N, nus, rows, uniform):
+    """Column-streaming kernel (strided layers, Q = N/nu in {32, 64, 96, 128, 512, 2048}: whole-column
+    and ring paths, odd chunk counts) vs the oracle's Eq. 1, per-n weights and per-neuron bias too."""
+    rs = np.random.RandomState(N + len(nus))
+    L = len(nus)
+    if uniform:
+        w = np.full((L, 32), 1.0 / 16.0, np.float32)
+        bias = np.full(L * N, -0.35, np.float32)
+    else:
+        w = rs.uniform(-0.1, 0.2, size=(L, 32)).astype(np.float32)
+        bias = rs.uniform(-0.4, 0.1, size=L * N).astype(np.float32)
+    cn = sdgc.CirculantNetwork(N=N, L=L, nu=np.array(nus, np.int32), w=w, bias=bias, ymax=32.0)
+    net = cn.to_network()
+    Y0 = rs.uniform(0, 32, size=(rows, N)).astype(np.float32)
+    Y0[1::3] = 0.0  # all-zero rows (row flags)
+    with SnicitNetwork.circulant(cn.N, cn.L, cn.nu, cn.w, cn.bias, cn.ymax) as g:
+        yin = torch.from_numpy(Y0).cuda()
+        for l in range(L):
+            ref = oracle.layers_f32(net, Y0, l, l + 1)
+            for k in (KERNEL_CIRC, KERNEL_CIRC_SMEM):
+                out = torch.full_like(yin, float("nan"))
+                g.debug_layer(l, yin, out, kernel=k)
+                assert np.array_equal(out.cpu().numpy(), ref), f"layer {l} nu {nus[l]} kernel {k}"
 
 
 def test_layer_ell_ragged_and_values():
@@ -259,6 +287,8 @@ def test_large_rows_segmented(N, L, B, t):
         assert st["circ_layers"] > 0
     Yu, catsu, _, _ = run_gpu(net, Y0, t=L)  # uncompressed path, bit-exact
     assert np.array_equal(Yu, plain) and np.array_equal(catsu, oracle.categories(plain))
+    Ys, catss, _, _ = run_gpu(net, Y0, t=t, kernel=KERNEL_CIRC_SMEM)  # staged kernels for strided layers
+    assert np.array_equal(catss, oracle.categories(plain)) and np.array_equal(Ys, ref["Y"])
 
 
 @pytest.mark.parametrize("N,L", [(1024, 10), (4096, 9)])
