@@ -169,6 +169,18 @@ class ClockSampler:
         return {"sm_mhz": float(np.median(sm)), "sm_max_mhz": mx, "reasons": sorted(reasons), "samples": len(sm)}
 
 
+def committed_traffic(config: str):
+    """Mean DRAM bytes per a1 layer-kernel launch from the latest committed ncu capture of this config
+    (profiles/rNN_traffic_<config>.json, written by scripts/traffic.py), or (None, None)."""
+    import glob
+    files = sorted(glob.glob(os.path.join(os.path.dirname(os.path.abspath(__file__)), "profiles",
+                                          f"r*_traffic_{config}.json")))
+    if not files:
+        return None, None
+    d = json.load(open(files[-1]))
+    return float(d["mean_dram_bytes_per_launch"]), f"{os.path.basename(files[-1])} ({d['launches']} launches)"
+
+
 def measured_peaks():
     p = os.path.join(ROOT, "MEASURED_PEAKS.json")
     if os.path.exists(p):
@@ -337,12 +349,26 @@ def run_snicit(args):
         avg_ms = float(pm.mean())
         avg_bytes = float(pb.mean())
         achieved = avg_bytes / (avg_ms * 1e-3) / 1e9
+        traffic, traffic_src = committed_traffic(args.config) if args.t is None and args.mode == "radix" else (None, None)
         roof = {"bound": "hbm", "achieved": achieved, "peak": peak, "unit": "GB/s", "frac": achieved / peak,
-                "traffic": None, "kernel": "layer_circ_kernel" if st["circ_layers"] else "layer_ell_kernel",
+                "traffic": traffic, "traffic_unit": "bytes per launch (ncu dram read + write)",
+                "traffic_source": traffic_src,
+                "kernel": ("a1 layer kernels: layer_circ_kernel / layer_circ_seg_kernel (nu = 1), "
+                           "layer_circ_col_kernel (strided)") if st["circ_layers"] else "layer_ell_kernel",
                 "peak_source": peak_src, "launches": int(len(pm)), "avg_launch_ms": avg_ms,
                 "avg_algorithmic_bytes": avg_bytes,
                 "share_of_step": float(pm.sum() / ms) if ms > 0 else None,
                 "layer0_frac": float(pb[0] / (pm[0] * 1e-3) / 1e9 / peak)}
+        if args.mode == "radix":  # per stride class (layer l has stride nu_l; DESIGN.md §7 kernels)
+            strides = sdgc.radix_strides(c["N"])
+            by = {}
+            for l in range(len(pm)):
+                e = by.setdefault(f"nu={strides[l % len(strides)]}", [0, 0.0, 0.0])
+                e[0] += 1
+                e[1] += float(pm[l])
+                e[2] += float(pb[l])
+            roof["by_stride"] = {k: {"launches": n, "ms": round(ms_, 4),
+                                     "frac": round(b_ / (ms_ * 1e-3) / 1e9 / peak, 4)} for k, (n, ms_, b_) in by.items()}
 
     # ---- uncompressed GPU baseline (t >= L, same kernels)
     unc = None

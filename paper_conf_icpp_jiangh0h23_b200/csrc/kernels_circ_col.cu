@@ -53,14 +53,46 @@ __global__ void __launch_bounds__(kColThreads, 2) layer_circ_col_kernel(LayerArg
     const float b0 = UBIAS ? __ldg(a.bias) : 0.0f;
     const float ymax = a.ymax;
 
+    if (blockIdx.x == 0 && threadIdx.x == 0 && a.zero_count) *a.zero_count = 0;  // next append counter
+
     // unit u = (list position, column group): offset of column c of the row
     auto unit_base = [&](long long u, int& pos, int& c) -> size_t {
         pos = (int)(u / G);
         c = (int)(u - (long long)pos * G) * 32 + lane;
         return (size_t)__ldg(a.rows + pos) * (size_t)N + (size_t)c;
     };
+    // fused dead-row compaction (R23): rows with a non-zero output go to app_list (unordered, R24).
+    // A row spans G warps: each counts in at row_ctr[pos] (+1, +65536 if it saw a non-zero) and the
+    // last one decides, appends and clears the counter.  Appends are buffered one row per lane and
+    // flushed with one atomic per 32 rows.
+    int abuf = 0, nbuf = 0;
+    auto flush = [&]() {
+        int p0 = 0;
+        if (lane == 0 && nbuf) p0 = atomicAdd(a.app_count, nbuf);
+        p0 = __shfl_sync(0xffffffffu, p0, 0);
+        if (lane < nbuf) a.app_list[p0 + lane] = abuf;
+        nbuf = 0;
+    };
     auto flag = [&](int pos, size_t base, float mx) {
-        if (__any_sync(0xffffffffu, mx != 0.0f) && lane == 0) {
+        const bool nz = __any_sync(0xffffffffu, mx != 0.0f);
+        if (a.app_list) {
+            int app = 0;
+            if (lane == 0) {
+                if (G == 1) {
+                    app = nz;
+                } else {
+                    const int old = atomicAdd(a.row_ctr + pos, 1 + (nz ? 65536 : 0));
+                    if ((old & 0xffff) == G - 1) {
+                        app = nz || (old >> 16) != 0;
+                        a.row_ctr[pos] = 0;
+                    }
+                }
+            }
+            if (__shfl_sync(0xffffffffu, app, 0)) {
+                if (lane == nbuf) abuf = (int)(base / (size_t)N);
+                if (++nbuf == 32) flush();
+            }
+        } else if (nz && lane == 0) {
             if (a.flag_pos) a.flag_pos[pos] = 1;
             if (a.flag_row) a.flag_row[base / (size_t)N] = 1;
         }
@@ -162,6 +194,7 @@ __global__ void __launch_bounds__(kColThreads, 2) layer_circ_col_kernel(LayerArg
             flag(pos, base, mx);
         }
     }
+    if (a.app_list) flush();
 }
 
 template <bool UNIF, bool UBIAS, bool Q32, int NUCT>

@@ -95,6 +95,7 @@ struct snicit_network {
     DevBuf<float> cbuf0, cbuf1, ac;
     DevBuf<int> cscratch;  // per-chunk counts of the ordered compaction
     DevBuf<uint8_t> segflag;  // row flags OR-ed by segmented layers (kept zero by the clearing compaction)
+    DevBuf<int> rowctr;       // per-position warp counters of the column-streaming kernel (self-clearing)
     DevBuf<double> F;
     DevBuf<int> counters;
     int* h_counters = nullptr;  // pinned mirror
@@ -237,6 +238,7 @@ void snicit_free_network(snicit_network* net) {
     net->cbuf1.release();
     net->cscratch.release();
     net->segflag.release();
+    net->rowctr.release();
     net->ac.release();
     net->F.release();
     if (net->h_counters) cudaFreeHost(net->h_counters);
@@ -592,6 +594,10 @@ static cudaError_t ensure_workspace(snicit_network* net, int64_t R, int s, int n
         if ((e = net->segflag.ensure(rows)) != cudaSuccess) return e;
         if ((e = cudaMemset(net->segflag.p, 0, rows)) != cudaSuccess) return e;
     }
+    if (net->rowctr.n < rows) {
+        if ((e = net->rowctr.ensure(rows)) != cudaSuccess) return e;
+        if ((e = cudaMemset(net->rowctr.p, 0, rows * sizeof(int))) != cudaSuccess) return e;
+    }
     return cudaSuccess;
 }
 
@@ -706,7 +712,9 @@ snicit_status snicit_infer(snicit_network* net, const float* y0, int64_t batch, 
         a.yout = bufs[nxt_i];
         a.rows = lists[li];
         a.count = cnt + live_ctr[ci];
-        const bool seg = use_seg(net, l, opt.kernel) || use_col(net, l, opt.kernel);  // OR-ed row flags
+        // segmented layers: row flags OR-ed across CTAs + a compaction launch; the others append
+        const bool seg = use_seg(net, l, opt.kernel) && !use_col(net, l, opt.kernel);
+        a.row_ctr = net->rowctr.p;                     // column-streaming kernel: last warp of a row appends
         if (drop_now && !seg) {
             a.app_list = lists[li ^ 1];
             a.app_count = cnt + live_ctr[(ci + 1) % 3];

@@ -107,6 +107,8 @@ struct LayerArgs {
     int* app_list;          // nullable: rows with a non-zero output are appended here (unordered)
     int* app_count;         //   ... at atomicAdd(app_count, n) (zero on entry)
     int* zero_count;        // nullable: set to 0 by the kernel (rotating append counters)
+    int* row_ctr;           // column-streaming kernel with app_list: per list position, zero on entry
+                            //   and on exit (warps of a row count in; the last one appends the row)
     float* a_out;           // CENTROID: a_c [row][N]
     const float* a_c;       // RESIDUAL: a_c [slot][N]
     const int* cslot;       // RESIDUAL: centroid slot of each row id

@@ -1,5 +1,5 @@
 """Write a markdown summary of one round's measurements for profiles/:
-    python scripts/profile_summary.py <bench.json> <launches.csv> <full.ncu-rep> > profiles/rNN_summary.md
+    python scripts/profile_summary.py <bench.json> <launches.csv> <full.raw.csv | full.ncu-rep> > profiles/rNN_summary.md
 Launch shares come from the ncu launch list (cold-cache, serialised: compare SHARES, not absolutes)."""
 import collections
 import csv
@@ -45,7 +45,8 @@ for k, (n, us) in sorted(agg.items(), key=lambda x: -x[1][1]):
     print(f"| `{k}` | {n} | {us:.1f} | {100 * us / tot:.1f}% |")
 print(f"\nTotal {sum(v[0] for v in agg.values())} launches, {tot:.1f} us serialised.\n")
 
-out = subprocess.run(["ncu", "-i", rep, "--page", "raw", "--csv"], capture_output=True, text=True).stdout
+out = open(rep).read() if rep.endswith(".csv") else \
+    subprocess.run(["ncu", "-i", rep, "--page", "raw", "--csv"], capture_output=True, text=True).stdout
 rr = list(csv.reader(io.StringIO(out)))
 hh = rr[0]
 want = ["Kernel Name", "gpu__time_duration.sum", "dram__bytes_read.sum", "dram__bytes_write.sum",
