@@ -381,36 +381,59 @@ def run_snicit(args):
         unc = {"value": B_global * nnz / (ms_u * 1e-3), "unit": UNIT, "ms_per_step": ms_u,
                "speedup_snicit": ms_u / ms}
 
-    # ---- e2e through the C ABI with host (pinned) buffers
-    e2e = None
+    # ---- e2e through the C ABI with host (pinned) buffers.  Headline: the SDGC inputs are binary, so
+    # Y0 is uploaded as the packed bitmap of snicit_infer_packed (H2D inside the call) and the step's
+    # result is the category set (D2H).  Also reported: fp32 rows in and Y(L) out (e2e_fp32_io).
+    e2e = e2e_fp32 = None
     if not args.no_e2e:
+        from paper_conf_icpp_jiangh0h23_b200 import pack_rows
+        bits_pin = torch.from_numpy(pack_rows(Yh).view(np.int32)).pin_memory()
         yh_pin = torch.from_numpy(Yh).pin_memory()
         yo_pin = torch.empty_like(yh_pin).pin_memory()
 
-        def step_e2e():
+        def step_packed():
+            g.infer_packed(bits_pin.numpy(), t=t, s=s, options=opt, row_offset=row0)
+            cats = g.categories()
+            if distributed:
+                with torch.cuda.stream(stream):
+                    allgather_categories(torch.from_numpy(cats).to(coll_dev))
+            return cats
+
+        def step_fp32():
             g.infer(yh_pin.numpy(), t=t, s=s, options=opt, y_out=yo_pin.numpy(), row_offset=row0)
             cats = g.categories()
             if distributed:
                 with torch.cuda.stream(stream):
                     allgather_categories(torch.from_numpy(cats).to(coll_dev))
             return cats
-        step_e2e()
-        if distributed:
-            dist.barrier()
-        torch.cuda.synchronize(dev)
-        k = max(1, min(args.steps, 3))
-        t0 = time.perf_counter()
-        for _ in range(k):
-            cats = step_e2e()
-        torch.cuda.synchronize(dev)
-        ms_e = (time.perf_counter() - t0) * 1e3 / k
-        if distributed:
-            tt = torch.tensor([ms_e], device=coll_dev)
-            dist.all_reduce(tt, op=dist.ReduceOp.MAX)
-            ms_e = float(tt.item())
+
+        def wall(fn):
+            fn()
+            if distributed:
+                dist.barrier()
+            torch.cuda.synchronize(dev)
+            k = max(1, min(args.steps, 3))
+            t0 = time.perf_counter()
+            for _ in range(k):
+                cats = fn()
+            torch.cuda.synchronize(dev)
+            ms_e = (time.perf_counter() - t0) * 1e3 / k
+            if distributed:
+                tt = torch.tensor([ms_e], device=coll_dev)
+                dist.all_reduce(tt, op=dist.ReduceOp.MAX)
+                ms_e = float(tt.item())
+            return ms_e, cats
+
+        ms_e, cats = wall(step_packed)
         e2e = {"value": B_global * nnz / (ms_e * 1e-3), "unit": UNIT, "ms_per_step": ms_e,
-               "h2d_bytes_per_step": int(Yh.nbytes) * world, "d2h_bytes_per_step": (int(Yh.nbytes) + 8 * len(cats)) * world,
+               "h2d_bytes_per_step": int(bits_pin.numel() * 4) * world, "d2h_bytes_per_step": (4 + 8 * len(cats)) * world,
+               "api": "snicit_infer_packed (Y0 as packed binary bitmap) + snicit_categories",
                "timer": "host wall clock around K synchronous C-ABI calls"}
+        ms_f, cats = wall(step_fp32)
+        e2e_fp32 = {"value": B_global * nnz / (ms_f * 1e-3), "unit": UNIT, "ms_per_step": ms_f,
+                    "h2d_bytes_per_step": int(Yh.nbytes) * world, "d2h_bytes_per_step": (int(Yh.nbytes) + 8 * len(cats)) * world,
+                    "api": "snicit_infer (fp32 Y0 in, fp32 Y(L) out) + snicit_categories",
+                    "timer": "host wall clock around K synchronous C-ABI calls"}
 
     # ---- CPU oracle baseline (rank 0, N = 1 only), bounded sample
     cpu = None
@@ -432,7 +455,7 @@ def run_snicit(args):
                        "t": t, "s": s, "n": snic["n"], "eta": 0.03, "eps": 0.03, "kernel": args.kernel,
                        "network_abi": "compact circulant" if isinstance(net, sdgc.CirculantNetwork) else "CSC",
                        "l2": "inputs larger than L2 (no flush)", "parallelism": f"dp{world} (row shards)"},
-            "roofline": roof, "cpu_baseline": cpu, "e2e": e2e, "clocks": clk,
+            "roofline": roof, "cpu_baseline": cpu, "e2e": e2e, "e2e_fp32_io": e2e_fp32, "clocks": clk,
             "gpu_launches": int(launches_per_step * args.steps),
             "uncompressed": unc, "phases_ms": phases,
             "dynamics": {k: st[k] for k in ("live_at_t", "n_centroids", "n_sampled", "residual_at_t",

@@ -150,6 +150,19 @@ snicit_status snicit_infer(snicit_network* net, const float* y0, int64_t batch,
                            int32_t centroid_count, const snicit_options* opt, float* y_out,
                            int32_t y_out_on_device);
 
+/* snicit_infer for binary inputs given as a packed bitmap (the SDGC inputs are binary images,
+ * P:297-302; 32x fewer bytes to upload than fp32 rows).  Row r of Y0 is
+ *   Y0[r][j] = (y0_bits[r*W + j/32] >> (j % 32)) & 1 ? one_value : 0.0f,   W = ceil(N/32) words,
+ * i.e. bit j%32 (LSB first) of 32-bit word j/32; bits of the last word beyond N are ignored.
+ * y0_bits: batch*W uint32, device pointer if bits_on_device else host (copied to the device
+ * inside the call).  one_value: finite.  The rows are unpacked on the device into the handle's
+ * workspace and the inference proceeds exactly as snicit_infer on the equivalent fp32 Y0 (same
+ * results, tested).  All other arguments as snicit_infer. */
+snicit_status snicit_infer_packed(snicit_network* net, const uint32_t* y0_bits, int64_t batch,
+                                  int32_t bits_on_device, float one_value, int64_t row_offset,
+                                  int32_t threshold_layer, int32_t centroid_count,
+                                  const snicit_options* opt, float* y_out, int32_t y_out_on_device);
+
 /* Category ids of the last infer, ascending, as int64 global row ids (library-owned until
  * the next infer/free; copied out here).  Two-call pattern: rows == NULL -> *count = total.
  * Otherwise *count is the capacity of rows on entry and the number written on return

@@ -5,5 +5,5 @@ thin Python binding (``api.SnicitNetwork``) plus row sharding / the category all
 (``parallel``).  No CPU fallback: the library must be built (``build.build()``).
 """
 from ._lib import KERNEL_AUTO, KERNEL_CIRC, KERNEL_CIRC_SMEM, KERNEL_ELL, Options, SnicitError, default_options, load_library  # noqa: F401
-from .api import SnicitNetwork  # noqa: F401
+from .api import SnicitNetwork, pack_rows  # noqa: F401
 from .parallel import allgather_categories, shard_rows  # noqa: F401

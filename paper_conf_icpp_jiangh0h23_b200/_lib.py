@@ -23,7 +23,7 @@ KERNEL_AUTO, KERNEL_ELL, KERNEL_CIRC, KERNEL_CIRC_SMEM = 0, 1, 2, 3
 EXPORTED = ["snicit_default_options", "snicit_load_network", "snicit_set_stream", "snicit_infer",
             "snicit_categories", "snicit_stats", "snicit_debug_clustering", "snicit_debug_layer",
             "snicit_layer_is_circulant", "snicit_free_network", "snicit_last_error", "snicit_abi_version",
-            "snicit_layer_profile", "snicit_load_network_circulant"]
+            "snicit_layer_profile", "snicit_load_network_circulant", "snicit_infer_packed"]
 
 
 class Options(ctypes.Structure):
@@ -71,6 +71,8 @@ def load_library(path: str = LIB_PATH):
     L.snicit_set_stream.restype = i32
     L.snicit_infer.argtypes = [P, P, i64, i32, i64, i32, i32, ctypes.POINTER(Options), P, i32]
     L.snicit_infer.restype = i32
+    L.snicit_infer_packed.argtypes = [P, P, i64, i32, f32, i64, i32, i32, ctypes.POINTER(Options), P, i32]
+    L.snicit_infer_packed.restype = i32
     L.snicit_categories.argtypes = [P, P, ctypes.POINTER(i64), i32]
     L.snicit_categories.restype = i32
     L.snicit_stats.argtypes = [P, ctypes.POINTER(Stats)]

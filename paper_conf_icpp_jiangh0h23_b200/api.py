@@ -17,6 +17,22 @@ def _is_cuda_tensor(x) -> bool:
     return hasattr(x, "is_cuda") and bool(x.is_cuda)
 
 
+def pack_rows(Y: np.ndarray, one: float = 1.0) -> np.ndarray:
+    """Binary B x N rows (every value 0 or `one`) -> the packed bitmap of snicit_infer_packed:
+    B x ceil(N/32) uint32, bit j % 32 (LSB first) of word j / 32 set where Y[r, j] == one.
+    Layout marshalling only (no SNICIT arithmetic)."""
+    Y = np.asarray(Y)
+    nz = Y != 0
+    if not np.all(Y[nz] == np.float32(one)):
+        raise ValueError("pack_rows: rows must be binary (0 or `one`)")
+    B, N = Y.shape
+    W = (N + 31) // 32
+    padded = np.zeros((B, W * 32), dtype=bool)
+    padded[:, :N] = nz
+    by = np.packbits(padded.reshape(B, W * 4, 8), axis=2, bitorder="little").reshape(B, W * 4)
+    return np.ascontiguousarray(by).view("<u4").reshape(B, W)
+
+
 class SnicitNetwork:
     """Owns one `snicit_network*` (device copy of W, b + workspace) on `device`.
 
@@ -128,6 +144,37 @@ class SnicitNetwork:
         st = self._lib.snicit_infer(self._h, y0p, B, y0_dev, int(row_offset), int(t), int(s), ctypes.byref(options),
                                     yop, yo_dev)
         check(st, "snicit_infer")
+        self._last_batch = B
+        return y_out
+
+    def infer_packed(self, bits, t: int, s: int = 32, options: Optional[Options] = None, y_out=None,
+                     row_offset: int = 0, one: float = 1.0, **opt_kw):
+        """snicit_infer_packed: binary inputs as the packed bitmap of `pack_rows` (B x ceil(N/32)
+        uint32: numpy array, CPU tensor or CUDA tensor of int32/uint32).  Same results as infer()."""
+        if options is None:
+            options = default_options(**opt_kw)
+        elif opt_kw:
+            raise ValueError("pass either options or keyword options")
+        W = (self.N + 31) // 32
+        if _is_cuda_tensor(bits):
+            assert bits.element_size() == 4 and bits.is_contiguous()
+            B, dev, bp = int(bits.shape[0]), 1, bits.data_ptr()
+        else:
+            arr = bits.numpy() if hasattr(bits, "numpy") else bits
+            if not (isinstance(arr, np.ndarray) and arr.dtype.itemsize == 4 and arr.flags.c_contiguous):
+                raise ValueError("host bits must be a C-contiguous 32-bit array")
+            B, dev, bp = int(arr.shape[0]), 0, arr.ctypes.data
+        if B and int(bits.shape[1]) != W:
+            raise ValueError(f"bits must be B x {W}")
+        if y_out is None:
+            yo_dev, yop = 0, None
+        elif _is_cuda_tensor(y_out):
+            yo_dev, yop = 1, y_out.data_ptr()
+        else:
+            ya = y_out.numpy() if hasattr(y_out, "numpy") else y_out
+            yo_dev, yop = 0, ya.ctypes.data
+        check(self._lib.snicit_infer_packed(self._h, bp, B, dev, float(one), int(row_offset), int(t), int(s),
+                                            ctypes.byref(options), yop, yo_dev), "snicit_infer_packed")
         self._last_batch = B
         return y_out
 

@@ -442,4 +442,33 @@ cudaError_t launch_recover(int N, int R, int plain, const float* yfinal, const u
     return cudaGetLastError();
 }
 
+// ------------------------------------------------------------------ packed binary input (snicit_infer_packed)
+// One thread per 4 consecutive outputs of a row: coalesced float4 stores; the 8 threads sharing a
+// 32-bit word read it from L1.  N % 4 == 0 (load-time requirement), W = ceil(N / 32) words per row.
+__global__ void unpack_bits_kernel(const uint32_t* __restrict__ bits, long long quads, int N, int W, float one,
+                                   float* __restrict__ y) {
+    const int qpr = N >> 2;
+    for (long long q = (long long)blockIdx.x * blockDim.x + threadIdx.x; q < quads;
+         q += (long long)gridDim.x * blockDim.x) {
+        const long long r = q / qpr;
+        const int j = (int)(q - r * qpr) << 2;
+        const uint32_t w = __ldg(bits + r * W + (j >> 5)) >> (j & 31);
+        float4 v;
+        v.x = (w & 1u) ? one : 0.0f;
+        v.y = (w & 2u) ? one : 0.0f;
+        v.z = (w & 4u) ? one : 0.0f;
+        v.w = (w & 8u) ? one : 0.0f;
+        reinterpret_cast<float4*>(y + r * N)[j >> 2] = v;
+    }
+}
+
+cudaError_t launch_unpack_bits(const uint32_t* bits, int R, int N, float one, float* y, int num_sms, cudaStream_t st) {
+    const long long quads = (long long)R * (N / 4);
+    if (quads <= 0) return cudaSuccess;
+    long long grid = (quads + 255) / 256;
+    if (grid > (long long)num_sms * 16) grid = (long long)num_sms * 16;
+    unpack_bits_kernel<<<(int)grid, 256, 0, st>>>(bits, quads, N, (N + 31) / 32, one, y);
+    return cudaGetLastError();
+}
+
 }  // namespace snicit

@@ -96,6 +96,7 @@ struct snicit_network {
     DevBuf<int> cscratch;  // per-chunk counts of the ordered compaction
     DevBuf<uint8_t> segflag;  // row flags OR-ed by segmented layers (kept zero by the clearing compaction)
     DevBuf<int> rowctr;       // per-position warp counters of the column-streaming kernel (self-clearing)
+    DevBuf<uint32_t> bits;    // packed binary input rows (snicit_infer_packed, host bits)
     DevBuf<double> F;
     DevBuf<int> counters;
     int* h_counters = nullptr;  // pinned mirror
@@ -239,6 +240,7 @@ void snicit_free_network(snicit_network* net) {
     net->cscratch.release();
     net->segflag.release();
     net->rowctr.release();
+    net->bits.release();
     net->ac.release();
     net->F.release();
     if (net->h_counters) cudaFreeHost(net->h_counters);
@@ -613,12 +615,15 @@ static cudaError_t read_counter(snicit_network* net, int which, int* outv) {
 
 extern "C" {
 
-snicit_status snicit_infer(snicit_network* net, const float* y0, int64_t batch, int32_t y0_on_device,
-                           int64_t row_offset, int32_t t, int32_t s, const snicit_options* opt_in, float* y_out,
-                           int32_t y_out_on_device) {
+// y0_mode: 0 = y0 is a device pointer, 1 = host pointer, 2 = the input rows are already in net->Ya
+// (snicit_infer_packed unpacked them there)
+static snicit_status infer_core(snicit_network* net, const float* y0, int64_t batch, int32_t y0_mode,
+                                int64_t row_offset, int32_t t, int32_t s, const snicit_options* opt_in, float* y_out,
+                                int32_t y_out_on_device) {
+    const int32_t y0_on_device = y0_mode == 0;
     if (!net) return fail(SNICIT_E_INVALID_ARG, "net NULL");
     if (batch < 0 || batch > 0x7fffffffLL) return fail(SNICIT_E_INVALID_ARG, "batch out of range");
-    if (batch > 0 && !y0) return fail(SNICIT_E_INVALID_ARG, "y0 NULL");
+    if (batch > 0 && !y0 && y0_mode != 2) return fail(SNICIT_E_INVALID_ARG, "y0 NULL");
     if (t < 0) return fail(SNICIT_E_INVALID_ARG, "threshold_layer < 0");
     if (s < 1) return fail(SNICIT_E_INVALID_ARG, "centroid_count < 1");
     if (row_offset < 0) return fail(SNICIT_E_INVALID_ARG, "row_offset < 0");
@@ -646,7 +651,7 @@ snicit_status snicit_infer(snicit_network* net, const float* y0, int64_t batch, 
     CUDA_TRY(cudaSetDevice(net->device));
     CUDA_TRY(ensure_workspace(net, R, s, n_seg));
     cudaStream_t st = net->stream;
-    int64_t launches = 0;
+    int64_t launches = y0_mode == 2 ? 1 : 0;  // + the unpack kernel of snicit_infer_packed
     int circ_layers = 0;
     net->have_result = false;
     snicit_stats_t stats{};
@@ -661,7 +666,8 @@ snicit_status snicit_infer(snicit_network* net, const float* y0, int64_t batch, 
     if (y0_on_device) {
         cur = y0;
     } else {
-        CUDA_TRY(cudaMemcpyAsync(net->Ya.p, y0, sizeof(float) * (size_t)R * N, cudaMemcpyHostToDevice, st));
+        if (y0_mode == 1)
+            CUDA_TRY(cudaMemcpyAsync(net->Ya.p, y0, sizeof(float) * (size_t)R * N, cudaMemcpyHostToDevice, st));
         cur = net->Ya.p;
         nxt_i = 1;
     }
@@ -940,6 +946,37 @@ snicit_status snicit_infer(snicit_network* net, const float* y0, int64_t batch, 
         net->stats.t_total_ms = ms;
     }
     return SNICIT_OK;
+}
+
+snicit_status snicit_infer(snicit_network* net, const float* y0, int64_t batch, int32_t y0_on_device,
+                           int64_t row_offset, int32_t t, int32_t s, const snicit_options* opt, float* y_out,
+                           int32_t y_out_on_device) {
+    return infer_core(net, y0, batch, y0_on_device ? 0 : 1, row_offset, t, s, opt, y_out, y_out_on_device);
+}
+
+snicit_status snicit_infer_packed(snicit_network* net, const uint32_t* y0_bits, int64_t batch, int32_t bits_on_device,
+                                  float one_value, int64_t row_offset, int32_t t, int32_t s,
+                                  const snicit_options* opt, float* y_out, int32_t y_out_on_device) {
+    if (!net) return fail(SNICIT_E_INVALID_ARG, "net NULL");
+    if (batch < 0 || batch > 0x7fffffffLL) return fail(SNICIT_E_INVALID_ARG, "batch out of range");
+    if (batch > 0 && !y0_bits) return fail(SNICIT_E_INVALID_ARG, "y0_bits NULL");
+    if (!std::isfinite(one_value)) return fail(SNICIT_E_INVALID_ARG, "one_value not finite");
+    if (t < 0 || s < 1) return fail(SNICIT_E_INVALID_ARG, "threshold_layer < 0 or centroid_count < 1");
+    const int N = net->N;
+    const int R = (int)batch;
+    const size_t W = ((size_t)N + 31) / 32;
+    CUDA_TRY(cudaSetDevice(net->device));
+    const int n_seg = (opt && opt->n_segments > 0 && opt->n_segments <= N) ? opt->n_segments : N;
+    CUDA_TRY(ensure_workspace(net, R, s, n_seg));
+    const uint32_t* bits = y0_bits;
+    if (!bits_on_device && R > 0) {
+        CUDA_TRY(net->bits.ensure((size_t)R * W));
+        CUDA_TRY(cudaMemcpyAsync(net->bits.p, y0_bits, sizeof(uint32_t) * (size_t)R * W, cudaMemcpyHostToDevice,
+                                 net->stream));
+        bits = net->bits.p;
+    }
+    if (R > 0) CUDA_TRY(launch_unpack_bits(bits, R, N, one_value, net->Ya.p, net->num_sms, net->stream));
+    return infer_core(net, nullptr, batch, 2, row_offset, t, s, opt, y_out, y_out_on_device);
 }
 
 snicit_status snicit_categories(snicit_network* net, int64_t* rows, int64_t* count, int32_t rows_on_device) {

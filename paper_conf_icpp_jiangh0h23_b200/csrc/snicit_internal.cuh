@@ -239,6 +239,8 @@ cudaError_t launch_map_residual(const float* y, int N, const int* rows, const in
 cudaError_t launch_recover(int N, int R, int plain, const float* yfinal, const uint8_t* live_row, const int* M,
                            const int* cslot, const uint8_t* ne_row, const float* cbuf, float* y_out,
                            uint8_t* cat, int num_sms, cudaStream_t st);
+// packed binary rows -> fp32 rows: y[r][j] = bit j of row r ? one : 0 (snicit_infer_packed)
+cudaError_t launch_unpack_bits(const uint32_t* bits, int R, int N, float one, float* y, int num_sms, cudaStream_t st);
 cudaError_t launch_mark_rows(const int* rows, const int* count, uint8_t* flag_row, int max_rows, cudaStream_t st);
 
 }  // namespace snicit

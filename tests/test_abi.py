@@ -90,6 +90,7 @@ def test_null_handle_errors(lib):
     n = ctypes.c_int64(0)
     assert lib.snicit_categories(None, None, ctypes.byref(n), 0) == -1
     assert lib.snicit_infer(None, None, 0, 0, 0, 0, 1, None, None, 0) == -1
+    assert lib.snicit_infer_packed(None, None, 0, 0, 1.0, 0, 0, 1, None, None, 0) == -1
     lib.snicit_free_network(None)  # no-op
 
 

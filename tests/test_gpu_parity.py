@@ -112,6 +112,27 @@ def test_column_stream_kernel_bit_exact(N, nus, rows, uniform):
                 assert np.array_equal(out.cpu().numpy(), ref), f"layer {l} nu {nus[l]} kernel {k}"
 
 
+@pytest.mark.parametrize("N,L,B,t,dev", [(1024, 40, 700, 4, True), (1024, 40, 700, 40, False),
+                                         (4096, 20, 300, 3, True), (16384, 6, 20, 2, False)])
+def test_packed_inputs_equal_fp32(N, L, B, t, dev):
+    """snicit_infer_packed (binary rows as a bitmap, unpacked on the device) == snicit_infer on the
+    equivalent fp32 rows, bit for bit, and == the oracle's categories."""
+    from paper_conf_icpp_jiangh0h23_b200 import pack_rows
+    net = sdgc.gen_network(N, L, "radix")
+    Y0 = sdgc.gen_inputs(N, B)
+    bits = pack_rows(Y0)
+    plain = oracle.layers_f32(net, Y0)
+    Y, cats, _, _ = run_gpu(net, Y0, t=t)
+    with SnicitNetwork.from_network(net) as g:
+        g.set_stream(torch.cuda.current_stream())
+        out = torch.empty((B, N), dtype=torch.float32, device="cuda")
+        g.infer_packed(torch.from_numpy(bits.view(np.int32)).cuda() if dev else bits, t=t, s=32, y_out=out)
+        cp = g.categories()
+        Yp = out.cpu().numpy()
+    assert np.array_equal(Yp, Y) and np.array_equal(cp, cats)
+    assert np.array_equal(cp, oracle.categories(plain))
+
+
 def test_layer_ell_ragged_and_values():
     net = ragged_net(64, 3, 1, ymax=4.0)
     Y0 = np.random.RandomState(2).uniform(0, 3, size=(50, 64)).astype(np.float32)

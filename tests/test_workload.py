@@ -1,5 +1,6 @@
 """The seeded generators: determinism, chunk independence, shapes and the SDGC constants."""
 import numpy as np
+import pytest
 
 from workload import rng, sdgc
 
@@ -46,3 +47,19 @@ def test_medium_network_shape():
     assert np.all(np.diff(net.ptr[:257]) == 26)
     assert (net.bias > 0).any() and (net.bias < 0).any()
     assert sdgc.medium_t(18) == 8 and sdgc.medium_t(12) == 6
+
+
+def test_pack_rows_layout():
+    """snicit_infer_packed's bitmap (include/snicit.h): bit j % 32, LSB first, of word j / 32; ragged N."""
+    from paper_conf_icpp_jiangh0h23_b200 import pack_rows
+    rs = np.random.RandomState(5)
+    for N in (4, 36, 64, 100, 1024):
+        Y = (rs.uniform(size=(7, N)) < 0.3).astype(np.float32) * np.float32(2.5)
+        bits = pack_rows(Y, one=2.5)
+        W = (N + 31) // 32
+        assert bits.shape == (7, W) and bits.dtype == np.uint32
+        for r in range(7):
+            for j in range(N):
+                assert ((int(bits[r, j // 32]) >> (j % 32)) & 1) == (Y[r, j] != 0)
+    with pytest.raises(ValueError):
+        pack_rows(np.array([[0.0, 0.5, 1.0, 1.0]], np.float32))
