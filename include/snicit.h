@@ -82,7 +82,12 @@ typedef struct {
                                8 CTAs exchanging layer outputs through distributed shared memory
                                (when every post layer is circulant and partition-compatible); 0 = one
                                CTA per centroid.  Results identical. */
-    int32_t reserved[2];
+    int32_t post_const;     /* 1 = a centroid row that is constant at t (all elements bitwise equal)
+                               is carried through the post layers by one scalar fma chain per layer
+                               when every post layer is circulant with uniform weights and bias
+                               (such a layer maps a constant row to a constant row; bit-identical
+                               results); 0 = always the full-row evaluation */
+    int32_t reserved[1];
 } snicit_options;
 
 /* Per-run statistics of the last snicit_infer (times in ms, valid when options.timing). */
@@ -98,10 +103,12 @@ typedef struct {
     int32_t threshold_layer;  /* t used (min(t, L)) */
     int32_t circ_layers;      /* layers run by the circulant kernel */
     int64_t kernel_launches;  /* kernels launched by this infer */
+    int32_t const_centroids;  /* centroids carried through the post layers as constant rows
+                                 (options.post_const) */
 } snicit_stats_t;
 
 /* Fill *opt with the paper's SDGC defaults (n = 16, eta = eps = 0.03, prune_eps = 0,
- * drop_dead_rows = 1, kernel = AUTO, timing = 0, ne_interval = 64, post_mode = 0, post_cluster = 1). */
+ * drop_dead_rows = 1, kernel = AUTO, timing = 0, ne_interval = 64, post_mode = 0, post_cluster = 1, post_const = 1). */
 void snicit_default_options(snicit_options* opt);
 
 /* Load a network (one-time; untimed in the benchmark).  All pointers are HOST pointers and

@@ -30,7 +30,8 @@ class Options(ctypes.Structure):
     _fields_ = [("n_segments", ctypes.c_int32), ("eta", ctypes.c_float), ("eps", ctypes.c_float),
                 ("prune_eps", ctypes.c_float), ("drop_dead_rows", ctypes.c_int32), ("kernel", ctypes.c_int32),
                 ("timing", ctypes.c_int32), ("ne_interval", ctypes.c_int32), ("post_mode", ctypes.c_int32),
-                ("post_cluster", ctypes.c_int32), ("reserved", ctypes.c_int32 * 2)]
+                ("post_cluster", ctypes.c_int32), ("post_const", ctypes.c_int32),
+                ("reserved", ctypes.c_int32 * 1)]
 
 
 class Stats(ctypes.Structure):
@@ -39,7 +40,8 @@ class Stats(ctypes.Structure):
                 ("live_at_t", ctypes.c_int64), ("residual_at_t", ctypes.c_int64),
                 ("residual_final", ctypes.c_int64), ("n_categories", ctypes.c_int64),
                 ("n_centroids", ctypes.c_int32), ("n_sampled", ctypes.c_int32), ("threshold_layer", ctypes.c_int32),
-                ("circ_layers", ctypes.c_int32), ("kernel_launches", ctypes.c_int64)]
+                ("circ_layers", ctypes.c_int32), ("kernel_launches", ctypes.c_int64),
+                ("const_centroids", ctypes.c_int32)]
 
     def as_dict(self):
         return {k: getattr(self, k) for k, _ in self._fields_}

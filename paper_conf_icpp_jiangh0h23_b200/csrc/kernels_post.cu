@@ -253,7 +253,7 @@ __global__ void __launch_bounds__(kCentThreads) centroid_traj_kernel(PostArgs a)
     extern __shared__ __align__(128) float sm[];
     const int C = *a.n_cent;
     const int c = blockIdx.x;
-    if (c >= C) return;
+    if (c >= C || (a.cdone && a.cdone[c])) return;
     const int N = a.N;
     const int h = post_halo(N);
     const int dup = h == N;
@@ -348,7 +348,7 @@ __global__ void __cluster_dims__(kCL, 1, 1) __launch_bounds__(kClThreads) centro
     const int r = (int)cl.block_rank();
     const int cid = blockIdx.x / kCL;
     const int C = *a.n_cent;
-    if (cid >= C) return;  // uniform over the cluster
+    if (cid >= C || (a.cdone && a.cdone[cid])) return;  // uniform over the cluster
     const int N = a.N, S = N / kCL;  // powers of two (centroid_cluster_ok)
     const int shS = ilog2(S);
     float* slice[2] = {sm, sm + S};
@@ -510,6 +510,90 @@ bool centroid_cluster_ok(int N, const int* nu, const int* cls, int t, int L) {
         }
     }
     return true;
+}
+
+// ------------------------------------------------------------------ constant centroid rows
+// A circulant layer with uniform bias maps a constant row (every element bitwise equal to v) to a
+// constant row: every output j evaluates the same stored-order chain acc = fma(v, w_n, acc),
+// n = 0..K-1, then sigma(acc + b) -- the chain of Eq. 1 / Eq. 5 (first case) with all inputs equal
+// (R12).  So a centroid that is constant at t is carried through the post layers (all circulant,
+// uniform weights and bias; checked by the caller) by one scalar chain per layer, bit-identical to
+// the full-row evaluation (tested against the oracle and the general kernels).  Each CTA checks one
+// centroid row (bitwise AND == OR), preloads the layers' (w0, b0) into shared memory, runs the scalar
+// trajectory in one thread, then writes the final row (and a_c of every layer when residues need it).
+__global__ void __launch_bounds__(256) centroid_const_kernel(PostArgs a, float* cout, int* cdone, int* ndone) {
+    extern __shared__ float2 s_wb[];  // [L - t] (w0, b0); then acc per layer (a_all)
+    __shared__ unsigned s_and[8], s_or[8];
+    __shared__ float s_v;
+    const int c = blockIdx.x;
+    if (c >= *a.n_cent) return;
+    const int N = a.N, nl = a.L - a.t;
+    const float* row = a.cbuf + (size_t)c * N;
+    unsigned an = 0xffffffffu, o = 0u;
+    for (int j = threadIdx.x; j < N; j += blockDim.x) {
+        const unsigned u = __float_as_uint(row[j]);
+        an &= u;
+        o |= u;
+    }
+    for (int d = 16; d; d >>= 1) {
+        an &= __shfl_xor_sync(0xffffffffu, an, d);
+        o |= __shfl_xor_sync(0xffffffffu, o, d);
+    }
+    if ((threadIdx.x & 31) == 0) {
+        s_and[threadIdx.x >> 5] = an;
+        s_or[threadIdx.x >> 5] = o;
+    }
+    for (int l = threadIdx.x; l < nl; l += blockDim.x) {
+        const PostLayer* p = a.layers + a.t + l;
+        s_wb[l] = make_float2(p->w0, p->b0);
+    }
+    __syncthreads();
+    an = s_and[0];
+    o = s_or[0];
+    for (int w = 1; w < (int)(blockDim.x >> 5); ++w) {
+        an &= s_and[w];
+        o |= s_or[w];
+    }
+    if (an != o) {  // not constant: the general trajectory kernels carry it
+        if (threadIdx.x == 0) cdone[c] = 0;
+        return;
+    }
+    float* s_acc = reinterpret_cast<float*>(s_wb + nl);
+    if (threadIdx.x == 0) {
+        float v = __uint_as_float(an);
+        for (int l = 0; l < nl; ++l) {
+            const float2 wb = s_wb[l];
+            float acc = 0.0f;
+#pragma unroll
+            for (int n = 0; n < kPK; ++n) acc = fmaf(v, wb.x, acc);
+            s_acc[l] = acc;
+            v = sigma(acc + wb.y, a.ymax);
+        }
+        s_v = v;
+    }
+    __syncthreads();
+    if (a.a_all)
+        for (int l = 0; l < nl; ++l) {
+            float* dst = a.a_all + ((size_t)l * a.s + c) * N;
+            const float acc = s_acc[l];
+            for (int j = threadIdx.x; j < N; j += blockDim.x) dst[j] = acc;
+        }
+    const float v = s_v;
+    for (int j = threadIdx.x; j < N; j += blockDim.x) cout[(size_t)c * N + j] = v;
+    if (threadIdx.x == 0) {
+        cdone[c] = 1;
+        atomicAdd(ndone, 1);
+    }
+}
+
+cudaError_t launch_centroid_const(const PostArgs& a, float* cout, int* cdone, int* ndone, int C_max, cudaStream_t st) {
+    if (C_max <= 0) return cudaSuccess;
+    const size_t smem = (size_t)(a.L - a.t) * (sizeof(float2) + sizeof(float));
+    int per_sm = 1;
+    cudaError_t e = blocks_per_sm((const void*)centroid_const_kernel, 256, smem, &per_sm);
+    if (e != cudaSuccess) return e;
+    centroid_const_kernel<<<C_max, 256, smem, st>>>(a, cout, cdone, ndone);
+    return cudaGetLastError();
 }
 
 cudaError_t launch_centroid_cluster(const PostArgs& a, int C_max, int win_max, cudaStream_t st) {

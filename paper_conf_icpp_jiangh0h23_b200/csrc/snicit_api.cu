@@ -61,7 +61,7 @@ struct DevBuf {
 // device counters (one int each)
 enum Counter {
     CNT_LIVE0 = 0, CNT_LIVE1, CNT_LIVE2, CNT_ORD, CNT_RES0, CNT_RES1, CNT_NCENT, CNT_SEFF, CNT_ALL, CNT_NCAT,
-    CNT_WORK, CNT_ALIVE, CNT_N
+    CNT_WORK, CNT_ALIVE, CNT_CDONE, CNT_N
 };
 
 }  // namespace
@@ -97,6 +97,7 @@ struct snicit_network {
     DevBuf<uint8_t> segflag;  // row flags OR-ed by segmented layers (kept zero by the clearing compaction)
     DevBuf<int> rowctr;       // per-position warp counters of the column-streaming kernel (self-clearing)
     DevBuf<uint32_t> bits;    // packed binary input rows (snicit_infer_packed, host bits)
+    DevBuf<int> cdone;        // per centroid: carried to L by the constant-row kernel
     DevBuf<double> F;
     DevBuf<int> counters;
     int* h_counters = nullptr;  // pinned mirror
@@ -109,6 +110,7 @@ struct snicit_network {
     int live_counter = 0;  // which CNT_LIVE* holds the live count at t
     int res_final_counter = -1;  // counter holding the non-empty residue rows after the last layer
     bool last_fused = false;
+    bool last_const = false;  // the constant-row centroid kernel ran in the last infer
     bool last_cluster = false;
     bool last_kernel_circ = false;
     snicit_stats_t stats{};
@@ -215,6 +217,7 @@ void snicit_default_options(snicit_options* opt) {
     opt->ne_interval = 64;
     opt->post_mode = 0;
     opt->post_cluster = 1;
+    opt->post_const = 1;
 }
 
 const char* snicit_last_error(void) { return g_last_error.c_str(); }
@@ -241,6 +244,7 @@ void snicit_free_network(snicit_network* net) {
     net->segflag.release();
     net->rowctr.release();
     net->bits.release();
+    net->cdone.release();
     net->ac.release();
     net->F.release();
     if (net->h_counters) cudaFreeHost(net->h_counters);
@@ -760,6 +764,7 @@ static snicit_status infer_core(snicit_network* net, const float* y0, int64_t ba
     const float* cfinal = net->cbuf0.p;
     const bool converted = tt < L;
     net->last_converted = converted;
+    net->last_const = false;
     if (!converted) {
         if (opt.timing) {
             CUDA_TRY(cudaEventRecord(net->ev[2], st));
@@ -805,6 +810,46 @@ static snicit_status infer_core(snicit_network* net, const float* y0, int64_t ba
         float* yh_nxt = yhat_other;
         const bool fused = opt.post_mode == 0 && N <= post_fused_max_n();
         net->last_fused = fused;
+        // constant centroid rows (centroid_const_kernel): every post layer circulant with uniform
+        // weights and bias.  Fused mode: in place, the trajectory kernels skip the carried rows.
+        // Per-layer mode (no residues): into cbuf1; the layer loop is skipped when all were carried.
+        bool const_ok = opt.post_const != 0 && opt.kernel != SNICIT_KERNEL_ELL;
+        for (int l = tt; l < L && const_ok; ++l)
+            const_ok = use_circ(net, l, opt.kernel) && net->plan[l].uniform && net->plan[l].ubias;
+        int* cdone = nullptr;
+        bool all_const = false;
+        if (const_ok && (fused || res_host == 0)) {
+            CUDA_TRY(net->cdone.ensure((size_t)s));
+            cdone = net->cdone.p;
+            CUDA_TRY(cudaMemsetAsync(cnt + CNT_CDONE, 0, sizeof(int), st));
+            PostArgs pc{};
+            pc.N = N;
+            pc.L = L;
+            pc.t = tt;
+            pc.ymax = net->ymax;
+            pc.layers = net->post_layers_d.p;
+            pc.cbuf = net->cbuf0.p;
+            pc.n_cent = cnt + CNT_NCENT;
+            pc.s = s;
+            if (fused && res_host > 0) {
+                CUDA_TRY(net->a_all.ensure((size_t)(L - tt) * (size_t)s * N));
+                pc.a_all = net->a_all.p;
+            }
+            CUDA_TRY(launch_centroid_const(pc, fused ? net->cbuf0.p : net->cbuf1.p, cdone, cnt + CNT_CDONE, s, st));
+            ++launches;
+            if (!fused) {
+                int nd = 0, nc = 0;
+                CUDA_TRY(read_counter(net, CNT_CDONE, &nd));
+                CUDA_TRY(read_counter(net, CNT_NCENT, &nc));
+                all_const = nd == nc;
+                if (all_const) {
+                    c_cur = net->cbuf1.p;
+                    c_nxt = net->cbuf0.p;
+                    for (int l = tt; l < L; ++l) circ_layers += use_circ(net, l, opt.kernel);
+                }
+            }
+        }
+        net->last_const = cdone != nullptr;
         if (fused) {
             // centroid trajectories (+ a_c per layer when residue rows exist), then residue rows
             PostArgs pa{};
@@ -828,6 +873,7 @@ static snicit_status infer_core(snicit_network* net, const float* y0, int64_t ba
             pa.cslot = net->cslot.p;
             pa.ne_row = net->ne_row.p;
             pa.alive_count = cnt + CNT_ALIVE;
+            pa.cdone = cdone;
             CUDA_TRY(cudaMemsetAsync(cnt + CNT_WORK, 0, 2 * sizeof(int), st));
             pa.force_ell = opt.kernel == SNICIT_KERNEL_ELL ? 1 : 0;
             // cluster (DSMEM) trajectory when every post layer is circulant and partition-compatible
@@ -855,7 +901,7 @@ static snicit_status infer_core(snicit_network* net, const float* y0, int64_t ba
                 ++launches;
             }
         }
-        for (int l = tt; l < L && !fused; ++l) {
+        for (int l = tt; l < L && !fused && !all_const; ++l) {
             // centroids: Eq. 5 first case, keep a_c
             LayerArgs a = layer_args(net, l, opt.kernel == SNICIT_KERNEL_ELL);
             a.yin = c_cur;
@@ -1023,6 +1069,11 @@ snicit_status snicit_stats(snicit_network* net, snicit_stats_t* out) {
         net->stats.n_centroids = v;
         CUDA_TRY(read_counter(net, CNT_SEFF, &v));
         net->stats.n_sampled = v;
+    }
+    net->stats.const_centroids = 0;
+    if (net->last_converted && net->last_const) {
+        CUDA_TRY(read_counter(net, CNT_CDONE, &v));
+        net->stats.const_centroids = v;
     }
     *out = net->stats;
     return SNICIT_OK;

@@ -208,6 +208,7 @@ struct PostArgs {
     const int* cslot;
     uint8_t* ne_row;     // set to the row's final ne (0 once its residue became empty)
     int* alive_count;    // += 1 per row still non-empty at L (may be NULL)
+    const int* cdone;    // nullable: centroid c already carried to L by centroid_const_kernel (skip it)
 };
 int post_fused_max_n();
 cudaError_t launch_centroid_traj(const PostArgs& a, int C_max, cudaStream_t st);
@@ -215,6 +216,10 @@ cudaError_t launch_centroid_traj(const PostArgs& a, int C_max, cudaStream_t st);
 bool centroid_cluster_ok(int N, const int* nu, const int* cls, int t, int L);
 cudaError_t launch_centroid_cluster(const PostArgs& a, int C_max, int win_max, cudaStream_t st);
 cudaError_t launch_residual_traj(const PostArgs& a, int max_rows, int num_sms, cudaStream_t st);
+// constant centroid rows through layers t..L-1 that are all circulant with uniform weights and bias:
+// one scalar chain per layer (exact, see kernels_post.cu); cout[c] = row at L, a.a_all filled if set,
+// cdone[c] = 1 and ++*ndone for constant rows, cdone[c] = 0 otherwise
+cudaError_t launch_centroid_const(const PostArgs& a, float* cout, int* cdone, int* ndone, int C_max, cudaStream_t st);
 int circ_class_of(int N, int nu);
 
 // kernels_convert.cu

@@ -133,6 +133,25 @@ def test_packed_inputs_equal_fp32(N, L, B, t, dev):
     assert np.array_equal(cp, oracle.categories(plain))
 
 
+@pytest.mark.parametrize("N,L,B,t,pm", [(1024, 60, 1500, 30, 0), (1024, 60, 1500, 30, 1), (1024, 60, 1500, 12, 0),
+                                        (1024, 60, 1500, 6, 0), (4096, 40, 400, 25, 0), (4096, 40, 400, 25, 1)])
+def test_constant_centroid_rows(N, L, B, t, pm):
+    """post_const (constant centroid rows carried by one scalar chain per circulant layer) is
+    bit-identical to the full-row evaluation and to the oracle's SNICIT reference, fused and
+    per-layer post modes, with and without residue rows."""
+    net = sdgc.gen_network(N, L, "radix")
+    Y0 = sdgc.gen_inputs(N, B)
+    ref = oracle.snicit(net, Y0, t=t)
+    plain = oracle.layers_f32(net, Y0)
+    Ya, ca, sa, _ = run_gpu(net, Y0, t=t, post_mode=pm, post_const=1)
+    Yb, cb, sb, _ = run_gpu(net, Y0, t=t, post_mode=pm, post_const=0)
+    assert sb["const_centroids"] == 0
+    assert np.array_equal(Ya, Yb) and np.array_equal(ca, cb)
+    assert np.array_equal(Ya, ref["Y"]) and np.array_equal(ca, oracle.categories(plain))
+    if t >= 25:  # the synthetic rows have collapsed to the all-YMAX row (DESIGN.md section 5)
+        assert sa["const_centroids"] >= 1
+
+
 def test_layer_ell_ragged_and_values():
     net = ragged_net(64, 3, 1, ymax=4.0)
     Y0 = np.random.RandomState(2).uniform(0, 3, size=(50, 64)).astype(np.float32)
