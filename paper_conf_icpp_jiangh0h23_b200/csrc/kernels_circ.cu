@@ -317,18 +317,31 @@ __global__ void __launch_bounds__(kCircThreads + 32, (MODE == MODE_PLAIN && UNIF
             float mx0 = 0.0f, mx1 = 0.0f;
             const bool second = rr + 1 < nr;
             if (item < n_items) {
+                static_assert(CLS == CLS_NU1, "PAIR: nu == 1 (ostep 1, outputs a0 .. a0 + M - 1)");
+                // unguarded stores: tail outputs (m >= mlim) land in the row's halo and the second row
+                // of an odd tail in the tile's unused row slot -- neither is ever TMA-stored
                 float* d0 = st + (size_t)rr * stride + obase;
                 float* d1 = d0 + stride;
 #pragma unroll
-                for (int m = 0; m < M; ++m)
-                    if (mlim == M || m < mlim) {
-                        d0[m * ostep] = v0[m];
-                        mx0 = fmaxf(mx0, fabsf(v0[m]));
-                        if (second) {
-                            d1[m * ostep] = v1[m];
-                            mx1 = fmaxf(mx1, fabsf(v1[m]));
-                        }
+                for (int m = 0; m < M; ++m) {
+                    d0[m] = v0[m];
+                    d1[m] = v1[m];
+                }
+                if (mlim == M) {  // outputs are >= 0 (sigma), so max == max |.|
+#pragma unroll
+                    for (int m = 0; m < M; ++m) {
+                        mx0 = fmaxf(mx0, v0[m]);
+                        mx1 = fmaxf(mx1, v1[m]);
                     }
+                } else {
+#pragma unroll
+                    for (int m = 0; m < M; ++m)
+                        if (m < mlim) {
+                            mx0 = fmaxf(mx0, v0[m]);
+                            mx1 = fmaxf(mx1, v1[m]);
+                        }
+                }
+                if (!second) mx1 = 0.0f;
             }
             warp_flag_rows(s_flag + sb * RT, mx0 != 0.0f, rr);
             warp_flag_rows(s_flag + sb * RT, second && mx1 != 0.0f, rr + 1);
