@@ -391,16 +391,39 @@ __global__ void __launch_bounds__(kSegThreads + 32, 2) layer_circ_seg_kernel(Lay
         }
         asm volatile("bar.sync 2, %0;" ::"n"(kSegThreads) : "memory");  // all stage reads done
         float mx = 0.0f;
+        if (PAIR && g.cls == 0) {
+            // nu == 1, two windows: unguarded stores (outputs past a window's segment land in the
+            // window's halo, an absent second window's buffer is never stored); max of the valid ones
+            constexpr int M = 17;
+            if (nv0 > 0 || nv1 > 0) {
 #pragma unroll
-        for (int m = 0; m < VM; ++m) {
-            if (m < nv0) {
-                stA[ob + m * os] = v0[m];
-                mx = fmaxf(mx, fabsf(v0[m]));
+                for (int m = 0; m < M; ++m) {
+                    stA[ob + m] = v0[m];
+                    stB[ob + m] = v1[PAIR ? m : 0];
+                }
+                if (nv0 == M && nv1 == M) {
+#pragma unroll
+                    for (int m = 0; m < M; ++m) mx = fmaxf(mx, fmaxf(v0[m], v1[PAIR ? m : 0]));
+                } else {
+#pragma unroll
+                    for (int m = 0; m < M; ++m) {
+                        if (m < nv0) mx = fmaxf(mx, fabsf(v0[m]));
+                        if (m < nv1) mx = fmaxf(mx, fabsf(v1[PAIR ? m : 0]));
+                    }
+                }
             }
-            if constexpr (PAIR) {
-                if (m < nv1) {
-                    stB[ob + m * os] = v1[m];
-                    mx = fmaxf(mx, fabsf(v1[m]));
+        } else {
+#pragma unroll
+            for (int m = 0; m < VM; ++m) {
+                if (m < nv0) {
+                    stA[ob + m * os] = v0[m];
+                    mx = fmaxf(mx, fabsf(v0[m]));
+                }
+                if constexpr (PAIR) {
+                    if (m < nv1) {
+                        stB[ob + m * os] = v1[m];
+                        mx = fmaxf(mx, fabsf(v1[m]));
+                    }
                 }
             }
         }
