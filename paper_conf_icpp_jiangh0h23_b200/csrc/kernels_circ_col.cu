@@ -44,11 +44,12 @@ __global__ void __launch_bounds__(kColThreads, 2) layer_circ_col_kernel(LayerArg
     const int N = a.N;
     const int nu = NUCT ? NUCT : a.nu;
     const int Q = N / nu;
-    const int G = nu >> 5;  // 32-column groups per row
-    const long long units = (long long)(*a.count) * G;
+    const unsigned G = (unsigned)nu >> 5;  // 32-column groups per row (compile-time with NUCT)
+    // 32-bit unit indices (the launcher checks rows * G < 2^31): u / G is a shift for the SDGC strides
+    const unsigned units = (unsigned)(*a.count) * G;
     const int lane = threadIdx.x & 31;
-    const long long warp0 = ((long long)blockIdx.x * kColThreads + threadIdx.x) >> 5;
-    const long long nwarps = ((long long)gridDim.x * kColThreads) >> 5;
+    const unsigned warp0 = (blockIdx.x * kColThreads + threadIdx.x) >> 5;
+    const unsigned nwarps = (gridDim.x * kColThreads) >> 5;
     const float w0 = a.w0;
     const float b0 = UBIAS ? __ldg(a.bias) : 0.0f;
     const float ymax = a.ymax;
@@ -56,9 +57,9 @@ __global__ void __launch_bounds__(kColThreads, 2) layer_circ_col_kernel(LayerArg
     if (blockIdx.x == 0 && threadIdx.x == 0 && a.zero_count) *a.zero_count = 0;  // next append counter
 
     // unit u = (list position, column group): offset of column c of the row
-    auto unit_base = [&](long long u, int& pos, int& c) -> size_t {
+    auto unit_base = [&](unsigned u, int& pos, int& c) -> size_t {
         pos = (int)(u / G);
-        c = (int)(u - (long long)pos * G) * 32 + lane;
+        c = (int)(u - (unsigned)pos * G) * 32 + lane;
         return (size_t)__ldg(a.rows + pos) * (size_t)N + (size_t)c;
     };
     // fused dead-row compaction (R23): rows with a non-zero output go to app_list (unordered, R24).
@@ -126,7 +127,7 @@ __global__ void __launch_bounds__(kColThreads, 2) layer_circ_col_kernel(LayerArg
             flag(pos, base, mx);
         };
         float RA[32], RB[32];
-        long long u = warp0;
+        unsigned u = warp0;
         int posA = 0, cA = 0, posB = 0, cB = 0;
         size_t bA = 0, bB = 0;
         if (u < units) {
@@ -134,14 +135,14 @@ __global__ void __launch_bounds__(kColThreads, 2) layer_circ_col_kernel(LayerArg
             load(RA, bA);
         }
         while (u < units) {
-            const long long u2 = u + nwarps;
+            const unsigned u2 = u + nwarps;
             if (u2 < units) {
                 bB = unit_base(u2, posB, cB);
                 load(RB, bB);
             }
             compute(RA, bA, cA, posA);
             if (u2 >= units) break;
-            const long long u3 = u2 + nwarps;
+            const unsigned u3 = u2 + nwarps;
             if (u3 < units) {
                 bA = unit_base(u3, posA, cA);
                 load(RA, bA);
@@ -174,7 +175,7 @@ __global__ void __launch_bounds__(kColThreads, 2) layer_circ_col_kernel(LayerArg
         auto nld = [&](int x) -> int { return min(32, max(0, Q + 31 - x)); };
         using I0 = std::integral_constant<int, 0>;
         using I32 = std::integral_constant<int, 32>;
-        for (long long u = warp0; u < units; u += nwarps) {
+        for (unsigned u = warp0; u < units; u += nwarps) {
             int pos, c;
             const size_t base = unit_base(u, pos, c);
             const float* src = a.yin + base;
@@ -204,6 +205,7 @@ static cudaError_t launch_col_t(const LayerArgs& a, int max_rows, int num_sms, c
     cudaError_t e = blocks_per_sm((const void*)kern, kColThreads, 0, &per_sm);
     if (e != cudaSuccess) return e;
     const long long units = (long long)max_rows * (a.nu / 32);
+    if (units + (long long)num_sms * 64 >= (1LL << 31)) return cudaErrorInvalidValue;  // 32-bit unit ids
     long long grid = (long long)num_sms * per_sm;
     const long long need = (units + kColThreads / 32 - 1) / (kColThreads / 32);
     if (grid > need) grid = need;
