@@ -58,6 +58,10 @@ def parse():
     p.add_argument("--no-e2e", action="store_true")
     p.add_argument("--no-cpu-baseline", action="store_true")
     p.add_argument("--no-uncompressed", action="store_true")
+    p.add_argument("--pre-fused", type=int, default=1, choices=[0, 1, 2],
+                   help="options.pre_fused: 1 = row-resident pre phase (default), 2 = without the constant-row "
+                        "shortcut, 0 = one launch per layer")
+    p.add_argument("--no-variants", action="store_true", help="skip the pre_fused = 2 / 0 roofline variants")
     p.add_argument("--cpu-seconds", type=float, default=15.0, help="target CPU work of the oracle sample")
     return p.parse_args()
 
@@ -181,6 +185,14 @@ def committed_traffic(config: str):
     return float(d["mean_dram_bytes_per_launch"]), f"{os.path.basename(files[-1])} ({d['launches']} launches)"
 
 
+# FP32 FMA pipe of a B200: 148 SMs x 128 FMA lanes/clk x 2 flop x 1965 MHz (B200_PROFILING.md: 148 SMs,
+# clocks.max.sm 1965 MHz; 128 FP32 lanes per SM: scripts/ubench_ffma.cu measured 127.9 FMA/clk/SM =
+# 37.1 TFMA/s for FFMA and FFMA2 alike)
+FMA_PEAK_TFLOPS = 148 * 128 * 2 * 1965e6 / 1e12
+FMA_PEAK_SRC = ("derived: 148 SMs x 128 FP32 FMA/clk x 2 flop x 1965 MHz = 74.45 TFLOP/s (DESIGN.md §7; "
+                "scripts/ubench_ffma.cu measured 74.2)")
+
+
 def measured_peaks():
     p = os.path.join(ROOT, "MEASURED_PEAKS.json")
     if os.path.exists(p):
@@ -290,7 +302,7 @@ def run_snicit(args):
     g.set_stream(stream)
     y0 = torch.from_numpy(Yh).to(dev)
     y_out = torch.empty_like(y0)
-    opt = default_options(kernel=kern, n_segments=snic["n"])
+    opt = default_options(kernel=kern, n_segments=snic["n"], pre_fused=args.pre_fused)
     t, s = snic["t"], snic["s"]
 
     def step():
@@ -330,45 +342,87 @@ def run_snicit(args):
     launches_per_step = g.stats()["kernel_launches"]
     value = B_global * nnz / (ms * 1e-3)
 
-    # ---- roofline of the dominant kernel (the pre-convergence layer kernel), live CUDA events
-    opt_prof = default_options(kernel=kern, n_segments=snic["n"], timing=2)
-    prof_ms, prof_bytes, prof_rows = [], [], []
-    for _ in range(max(1, min(args.steps, 3))):
-        g.infer(y0, t=t, s=s, options=opt_prof, y_out=y_out, row_offset=row0)
-        pr = g.layer_profile()
-        prof_ms.append(pr["ms"])
-        prof_bytes.append(pr["bytes"])
-        prof_rows.append(pr["rows"])
-    st = g.stats()
+    # ---- roofline of the dominant kernel (the pre-convergence a1 kernel), live CUDA events
+    def profile_pre(pre_fused):
+        o = default_options(kernel=kern, n_segments=snic["n"], timing=2, pre_fused=pre_fused)
+        g.infer(y0, t=t, s=s, options=o, y_out=y_out, row_offset=row0)  # first launches of these kernels
+        pms, pbs = [], []
+        for _ in range(max(1, min(args.steps, 3))):
+            g.infer(y0, t=t, s=s, options=o, y_out=y_out, row_offset=row0)
+            pr = g.layer_profile()
+            pms.append(pr["ms"])
+            pbs.append(pr["bytes"])
+        st_ = g.stats()
+        pm_ = np.mean(np.stack(pms), axis=0) if pms and len(pms[0]) else np.zeros(0)
+        pb_ = pbs[0] if pbs else np.zeros(0)
+        return st_, pm_, pb_
+
+    st, pm, pb = profile_pre(args.pre_fused)
     phases = {k: st[k] for k in ("t_pre_ms", "t_convert_ms", "t_post_ms", "t_recover_ms", "t_total_ms")}
-    pm = np.mean(np.stack(prof_ms), axis=0) if prof_ms and len(prof_ms[0]) else np.zeros(0)
-    pb = prof_bytes[0] if prof_bytes else np.zeros(0)
     peak, peak_src = measured_peaks()
-    roof = None
-    if len(pm):
-        avg_ms = float(pm.mean())
-        avg_bytes = float(pb.mean())
+    tag = args.config if args.t is None and args.mode == "radix" else None
+
+    def hbm_roof(pm_, pb_, st_):
+        """HBM roofline of the per-layer a1 kernels (8 B per live row-element per layer)."""
+        avg_ms = float(pm_.mean())
+        avg_bytes = float(pb_.mean())
         achieved = avg_bytes / (avg_ms * 1e-3) / 1e9
-        traffic, traffic_src = committed_traffic(args.config) if args.t is None and args.mode == "radix" else (None, None)
-        roof = {"bound": "hbm", "achieved": achieved, "peak": peak, "unit": "GB/s", "frac": achieved / peak,
-                "traffic": traffic, "traffic_unit": "bytes per launch (ncu dram read + write)",
-                "traffic_source": traffic_src,
-                "kernel": ("a1 layer kernels: layer_circ_kernel / layer_circ_seg_kernel (nu = 1), "
-                           "layer_circ_col_kernel (strided)") if st["circ_layers"] else "layer_ell_kernel",
-                "peak_source": peak_src, "launches": int(len(pm)), "avg_launch_ms": avg_ms,
-                "avg_algorithmic_bytes": avg_bytes,
-                "share_of_step": float(pm.sum() / ms) if ms > 0 else None,
-                "layer0_frac": float(pb[0] / (pm[0] * 1e-3) / 1e9 / peak)}
+        traffic, traffic_src = committed_traffic(tag) if tag else (None, None)
+        r = {"bound": "hbm", "achieved": achieved, "peak": peak, "unit": "GB/s", "frac": achieved / peak,
+             "traffic": traffic, "traffic_unit": "bytes per launch (ncu dram read + write)",
+             "traffic_source": traffic_src,
+             "kernel": ("a1 layer kernels: layer_circ_kernel / layer_circ_seg_kernel (nu = 1), "
+                        "layer_circ_col_kernel (strided)") if st_["circ_layers"] else "layer_ell_kernel",
+             "peak_source": peak_src, "launches": int(len(pm_)), "avg_launch_ms": avg_ms,
+             "avg_algorithmic_bytes": avg_bytes,
+             "layer0_frac": float(pb_[0] / (pm_[0] * 1e-3) / 1e9 / peak)}
         if args.mode == "radix":  # per stride class (layer l has stride nu_l; DESIGN.md §7 kernels)
             strides = sdgc.radix_strides(c["N"])
             by = {}
-            for l in range(len(pm)):
+            for l in range(len(pm_)):
                 e = by.setdefault(f"nu={strides[l % len(strides)]}", [0, 0.0, 0.0])
                 e[0] += 1
-                e[1] += float(pm[l])
-                e[2] += float(pb[l])
-            roof["by_stride"] = {k: {"launches": n, "ms": round(ms_, 4),
-                                     "frac": round(b_ / (ms_ * 1e-3) / 1e9 / peak, 4)} for k, (n, ms_, b_) in by.items()}
+                e[1] += float(pm_[l])
+                e[2] += float(pb_[l])
+            r["by_stride"] = {k: {"launches": n, "ms": round(ms_, 4),
+                                  "frac": round(b_ / (ms_ * 1e-3) / 1e9 / peak, 4)} for k, (n, ms_, b_) in by.items()}
+        return r
+
+    def alu_roof(pm_, pb_, st_):
+        """FP32 FMA-pipe roofline of the row-resident kernel: algorithmic flops = 2 x 32 x N per full
+        row-layer evaluation (constant rows carried by a scalar chain are not counted)."""
+        kms = float(pm_.sum())
+        flops = 2.0 * 32 * c["N"] * float(st_["pre_full_rows"])
+        achieved = flops / (kms * 1e-3) / 1e12
+        hbm_gbs = float(pb_.sum()) / (kms * 1e-3) / 1e9
+        traffic, traffic_src = committed_traffic(tag + "_fused") if tag else (None, None)
+        return {"bound": "alu", "achieved": achieved, "peak": FMA_PEAK_TFLOPS, "unit": "TFLOP/s",
+                "frac": achieved / FMA_PEAK_TFLOPS, "traffic": traffic,
+                "traffic_unit": "bytes per launch (ncu dram read + write)", "traffic_source": traffic_src,
+                "kernel": "pre_fused_kernel (row-resident a1: layers 0..t-1 of a row in shared memory, FFMA2 chains)",
+                "peak_source": FMA_PEAK_SRC, "launches": int(len(pm_)), "avg_launch_ms": kms,
+                "algorithmic_flops": flops, "full_row_layers": int(st_["pre_full_rows"]),
+                "const_rows": int(st_["pre_const_rows"]),
+                "hbm": {"algorithmic_bytes": float(pb_.sum()), "achieved_gbs": hbm_gbs, "frac": hbm_gbs / peak}}
+
+    roof = None
+    if len(pm):
+        roof = alu_roof(pm, pb, st) if st["pre_fused"] else hbm_roof(pm, pb, st)
+        roof["share_of_step"] = float(pm.sum() / ms) if ms > 0 else None
+        if st["pre_fused"] and not args.no_variants:
+            # the same kernel with every live row evaluated in full (no constant-row shortcut), and the
+            # per-layer kernels (one launch per layer, HBM-bound) on the same inputs
+            st2, pm2, pb2 = profile_pre(2)
+            if st2["pre_fused"] and len(pm2):
+                r2 = alu_roof(pm2, pb2, st2)
+                roof["no_const_skip"] = {k: r2[k] for k in ("achieved", "frac", "avg_launch_ms", "full_row_layers")}
+            st0, pm0, pb0 = profile_pre(0)
+            if len(pm0):
+                r0 = hbm_roof(pm0, pb0, st0)
+                roof["per_layer_kernels"] = {k: r0[k] for k in ("bound", "achieved", "peak", "unit", "frac", "traffic",
+                                                                "traffic_source", "launches", "avg_launch_ms",
+                                                                "by_stride") if k in r0}
+                roof["per_layer_kernels"]["ms_total"] = float(pm0.sum())
 
     # ---- uncompressed GPU baseline (t >= L, same kernels)
     unc = None
@@ -379,7 +433,16 @@ def run_snicit(args):
         step_unc()
         ms_u = timed(step_unc, max(1, min(args.steps, 3)))
         unc = {"value": B_global * nnz / (ms_u * 1e-3), "unit": UNIT, "ms_per_step": ms_u,
-               "speedup_snicit": ms_u / ms}
+               "speedup_snicit": ms_u / ms, "pre_fused": args.pre_fused}
+        if args.pre_fused and not args.no_variants:  # plain layer-by-layer launches (no row residency)
+            opt0 = default_options(kernel=kern, n_segments=snic["n"], pre_fused=0)
+
+            def step_unc0():
+                g.infer(y0, t=net.L, s=s, options=opt0, y_out=y_out, row_offset=row0)
+                g.num_categories()
+            step_unc0()
+            ms_u0 = timed(step_unc0, max(1, min(args.steps, 3)))
+            unc["per_layer_kernels"] = {"value": B_global * nnz / (ms_u0 * 1e-3), "ms_per_step": ms_u0}
 
     # ---- e2e through the C ABI with host (pinned) buffers.  Headline: the SDGC inputs are binary, so
     # Y0 is uploaded as the packed bitmap of snicit_infer_packed (H2D inside the call) and the step's
@@ -453,6 +516,7 @@ def run_snicit(args):
             "config": {"workload": f"{args.config}: {c['desc']}", "neurons": c["N"], "layers": c["L"],
                        "batch_per_rank": B_local, "global_batch": B_global, "connections": nnz, "w_mode": args.mode,
                        "t": t, "s": s, "n": snic["n"], "eta": 0.03, "eps": 0.03, "kernel": args.kernel,
+                       "pre_fused": args.pre_fused,
                        "network_abi": "compact circulant" if isinstance(net, sdgc.CirculantNetwork) else "CSC",
                        "l2": "inputs larger than L2 (no flush)", "parallelism": f"dp{world} (row shards)"},
             "roofline": roof, "cpu_baseline": cpu, "e2e": e2e, "e2e_fp32_io": e2e_fp32, "clocks": clk,

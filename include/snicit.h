@@ -30,7 +30,7 @@
 extern "C" {
 #endif
 
-#define SNICIT_ABI_VERSION 1
+#define SNICIT_ABI_VERSION 2
 
 typedef struct snicit_network snicit_network; /* opaque: owns device copies of W, b + workspace */
 
@@ -87,7 +87,15 @@ typedef struct {
                                when every post layer is circulant with uniform weights and bias
                                (such a layer maps a constant row to a constant row; bit-identical
                                results); 0 = always the full-row evaluation */
-    int32_t reserved[1];
+    int32_t pre_fused;      /* pre-convergence layers 0..t-1 (Eq. 1): 1 = row-resident fused kernel -- a
+                               CTA keeps one row in shared memory for all t layers (Y0 read and Y(t)
+                               written once) and carries a row that became constant (all elements
+                               equal) by one scalar fma chain per layer (R26, exact); 2 = the same kernel
+                               without the constant-row shortcut (every live row evaluated in full);
+                               0 = one kernel launch per layer.  Used when every layer < t is circulant
+                               with 32 taps, uniform weight and uniform bias, and N/32 is one of
+                               32..512 (N = 1024..16384); otherwise the per-layer kernels run.
+                               Results are bit-identical in every mode (tested). */
 } snicit_options;
 
 /* Per-run statistics of the last snicit_infer (times in ms, valid when options.timing). */
@@ -105,10 +113,14 @@ typedef struct {
     int64_t kernel_launches;  /* kernels launched by this infer */
     int32_t const_centroids;  /* centroids carried through the post layers as constant rows
                                  (options.post_const) */
+    int32_t pre_fused;        /* the pre-convergence layers ran in the row-resident fused kernel */
+    int32_t pre_const_rows;   /* fused: rows that became constant before t (carried by a scalar) */
+    int64_t pre_full_rows;    /* fused: full-row layer evaluations (row x layer, 32*N fma each) */
 } snicit_stats_t;
 
 /* Fill *opt with the paper's SDGC defaults (n = 16, eta = eps = 0.03, prune_eps = 0,
- * drop_dead_rows = 1, kernel = AUTO, timing = 0, ne_interval = 64, post_mode = 0, post_cluster = 1, post_const = 1). */
+ * drop_dead_rows = 1, kernel = AUTO, timing = 0, ne_interval = 64, post_mode = 0, post_cluster = 1, post_const = 1,
+ * pre_fused = 1). */
 void snicit_default_options(snicit_options* opt);
 
 /* Load a network (one-time; untimed in the benchmark).  All pointers are HOST pointers and

@@ -31,7 +31,7 @@ class Options(ctypes.Structure):
                 ("prune_eps", ctypes.c_float), ("drop_dead_rows", ctypes.c_int32), ("kernel", ctypes.c_int32),
                 ("timing", ctypes.c_int32), ("ne_interval", ctypes.c_int32), ("post_mode", ctypes.c_int32),
                 ("post_cluster", ctypes.c_int32), ("post_const", ctypes.c_int32),
-                ("reserved", ctypes.c_int32 * 1)]
+                ("pre_fused", ctypes.c_int32)]
 
 
 class Stats(ctypes.Structure):
@@ -41,7 +41,8 @@ class Stats(ctypes.Structure):
                 ("residual_final", ctypes.c_int64), ("n_categories", ctypes.c_int64),
                 ("n_centroids", ctypes.c_int32), ("n_sampled", ctypes.c_int32), ("threshold_layer", ctypes.c_int32),
                 ("circ_layers", ctypes.c_int32), ("kernel_launches", ctypes.c_int64),
-                ("const_centroids", ctypes.c_int32)]
+                ("const_centroids", ctypes.c_int32), ("pre_fused", ctypes.c_int32),
+                ("pre_const_rows", ctypes.c_int32), ("pre_full_rows", ctypes.c_int64)]
 
     def as_dict(self):
         return {k: getattr(self, k) for k, _ in self._fields_}

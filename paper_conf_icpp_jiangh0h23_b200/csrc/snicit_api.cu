@@ -61,7 +61,7 @@ struct DevBuf {
 // device counters (one int each)
 enum Counter {
     CNT_LIVE0 = 0, CNT_LIVE1, CNT_LIVE2, CNT_ORD, CNT_RES0, CNT_RES1, CNT_NCENT, CNT_SEFF, CNT_ALL, CNT_NCAT,
-    CNT_WORK, CNT_ALIVE, CNT_CDONE, CNT_N
+    CNT_WORK, CNT_ALIVE, CNT_CDONE, CNT_PFWORK, CNT_PFCONST, CNT_N
 };
 
 }  // namespace
@@ -85,6 +85,10 @@ struct snicit_network {
     std::vector<float> wtab_h;  // host copy (weights passed as kernel parameters)
     DevBuf<float> bias_d;
     DevBuf<PostLayer> post_layers_d;  // per-layer descriptors for the fused post-convergence kernels
+    DevBuf<PreFusedLayer> pf_layers_d;  // per-layer descriptors of the row-resident pre-convergence kernel
+    std::vector<PreFusedLayer> pf_layers_h;
+    std::vector<uint8_t> pf_elig;       // layer l can run in the row-resident kernel
+    DevBuf<unsigned long long> pf_full; // full-row layer evaluations of the last fused pre phase
     DevBuf<float> a_all;              // [(L - t)][s][N] centroid pre-activations (fused post mode)
     // workspace
     int64_t cap_rows = 0;
@@ -113,6 +117,7 @@ struct snicit_network {
     bool last_const = false;  // the constant-row centroid kernel ran in the last infer
     bool last_cluster = false;
     bool last_kernel_circ = false;
+    bool last_pre_fused = false;
     snicit_stats_t stats{};
     cudaEvent_t ev[6] = {nullptr, nullptr, nullptr, nullptr, nullptr, nullptr};
     std::vector<cudaEvent_t> lev;  // 2 per pre-convergence layer (timing == 2)
@@ -196,6 +201,39 @@ static cudaError_t net_upload_common(snicit_network* net, const float* bias, con
         }
         e = upload(net->post_layers_d, pls.data(), pls.size());
     }
+    if (e == cudaSuccess) {
+        // row-resident pre-convergence kernel (kernels_pre_fused.cu): circulant, 32 taps, uniform weight
+        // and bias; stride classes nu == 1, Q == 32, or nu >= 32 with Q >= 64 and Q % 32 == 0
+        net->pf_layers_h.assign(L, PreFusedLayer{});
+        net->pf_elig.assign(L, 0);
+        for (int l = 0; l < L; ++l) {
+            const LayerPlan& pl = net->plan[l];
+            PreFusedLayer& d = net->pf_layers_h[l];
+            d.nu = pl.nu;
+            d.w0 = pl.w0;
+            d.b0 = bias[(int64_t)l * N];
+            d.dead_next = net->dead_ok[l + 1];
+            {  // constant row YMAX through this layer: the kernel's chain (acc = fma(v, w0, acc) x 32, + b0)
+                float acc = 0.0f;
+                for (int n = 0; n < 32; ++n) acc = std::fma(net->ymax, pl.w0, acc);
+                const float z = acc + d.b0;
+                d.ymax_fixed = std::fmin(std::fmax(z, 0.0f), net->ymax) == net->ymax ? 1 : 0;
+            }
+            d.cls = -1;
+            if (pl.kind != 0 && pl.K == 32 && pl.uniform && pl.ubias && pl.nu >= 1 && N % pl.nu == 0) {
+                const int Q = N / pl.nu;
+                if (pl.nu == 1)
+                    d.cls = PF_NU1;
+                else if (Q == 32)
+                    d.cls = PF_Q32;
+                else if (pl.nu >= 32 && Q >= 64 && Q % 32 == 0)
+                    d.cls = PF_STR;
+            }
+            net->pf_elig[l] = d.cls >= 0 ? 1 : 0;
+        }
+        e = upload(net->pf_layers_d, net->pf_layers_h.data(), net->pf_layers_h.size());
+    }
+    if (e == cudaSuccess) e = net->pf_full.ensure(1);
     if (e == cudaSuccess) e = net->counters.ensure(CNT_N);
     if (e == cudaSuccess) e = cudaMallocHost(&net->h_counters, sizeof(int) * CNT_N);
     for (int i = 0; i < 6 && e == cudaSuccess; ++i) e = cudaEventCreate(&net->ev[i]);
@@ -218,6 +256,7 @@ void snicit_default_options(snicit_options* opt) {
     opt->post_mode = 0;
     opt->post_cluster = 1;
     opt->post_const = 1;
+    opt->pre_fused = 1;
 }
 
 const char* snicit_last_error(void) { return g_last_error.c_str(); }
@@ -254,6 +293,8 @@ void snicit_free_network(snicit_network* net) {
         if (e) cudaEventDestroy(e);
     net->hist.release();
     net->post_layers_d.release();
+    net->pf_layers_d.release();
+    net->pf_full.release();
     net->a_all.release();
     delete net;
 }
@@ -641,6 +682,7 @@ static snicit_status infer_core(snicit_network* net, const float* y0, int64_t ba
         return fail(SNICIT_E_INVALID_ARG, "bad eta/eps/prune_eps");
     if (opt.kernel < 0 || opt.kernel > SNICIT_KERNEL_CIRC_SMEM) return fail(SNICIT_E_INVALID_ARG, "bad kernel option");
     if (opt.post_mode < 0 || opt.post_mode > 1) return fail(SNICIT_E_INVALID_ARG, "bad post_mode");
+    if (opt.pre_fused < 0 || opt.pre_fused > 2) return fail(SNICIT_E_INVALID_ARG, "bad pre_fused");
     if (opt.kernel == SNICIT_KERNEL_ELL && !net->has_ell)
         return fail(SNICIT_E_UNSUPPORTED, "network loaded in compact circulant form has no ELL copy");
     const int N = net->N, L = net->L;
@@ -708,7 +750,61 @@ static snicit_status infer_core(snicit_network* net, const float* y0, int64_t ba
     } else {
         net->prof_layers = 0;
     }
-    for (int l = 0; l < tt; ++l) {
+    // row-resident fused pre phase (kernels_pre_fused.cu): one launch for layers 0..t-1
+    bool pf = opt.pre_fused != 0 && tt > 0 && R > 0 && opt.kernel == SNICIT_KERNEL_AUTO && pre_fused_threads(N) > 0;
+    for (int l = 0; l < tt && pf; ++l) pf = net->pf_elig[l] != 0;
+    int pf_gen = 0;
+    int pf_H = 64;  // circular halo: nu == 1 windows need 48 floats, STR windows 31*nu
+    if (pf) {
+        for (int l = 0; l < tt; ++l)
+            if (net->pf_layers_h[l].cls == PF_STR) {
+                pf_H = std::max(pf_H, 31 * net->pf_layers_h[l].nu);
+                if (net->pf_layers_h[l].nu != 32) pf_gen = 1;
+            }
+        pf_H = (pf_H + 31) / 32 * 32;
+        if (pf_H > N || pre_fused_smem(N, pf_H) > (size_t)227 * 1024) pf = false;
+    }
+    net->last_pre_fused = pf;
+    stats.pre_fused = pf ? 1 : 0;
+    if (pf) {
+        if (prof) {
+            CUDA_TRY(cudaMemcpyAsync(net->hist.p, cnt + live_ctr[ci], sizeof(int), cudaMemcpyDeviceToDevice, st));
+            CUDA_TRY(cudaEventRecord(net->lev[0], st));
+            net->prof_layers = 1;
+        }
+        CUDA_TRY(cudaMemsetAsync(cnt + CNT_PFWORK, 0, 2 * sizeof(int), st));
+        CUDA_TRY(cudaMemsetAsync(net->pf_full.p, 0, sizeof(unsigned long long), st));
+        PreFusedArgs pa{};
+        pa.N = N;
+        pa.t = tt;
+        pa.H = pf_H;
+        pa.ymax = net->ymax;
+        pa.drop = drop ? 1 : 0;
+        pa.const_skip = opt.pre_fused == 1 ? 1 : 0;
+        pa.gen_str = pf_gen;
+        pa.yin = cur;
+        pa.yout = bufs[nxt_i];
+        pa.rows = lists[li];
+        pa.count = cnt + live_ctr[ci];
+        pa.app_list = drop ? lists[li ^ 1] : nullptr;
+        pa.app_count = cnt + live_ctr[(ci + 1) % 3];
+        pa.work = cnt + CNT_PFWORK;
+        pa.layers = net->pf_layers_d.p;
+        pa.full_rl = net->pf_full.p;
+        pa.n_const = cnt + CNT_PFCONST;
+        CUDA_TRY(launch_pre_fused(pa, net->num_sms, st));
+        if (prof) CUDA_TRY(cudaEventRecord(net->lev[1], st));
+        ++launches;
+        circ_layers += tt;
+        net->last_kernel_circ = true;
+        cur = bufs[nxt_i];
+        nxt_i ^= 1;
+        if (drop) {
+            li ^= 1;
+            ci = (ci + 1) % 3;
+        }
+    }
+    for (int l = 0; l < tt && !pf; ++l) {
         // exact dead-row compaction (R23) fused into the layer: rows with a non-zero output are
         // appended (unordered) to the other list; the append counter of the NEXT dropping layer is
         // zeroed by this one (rotating counters), so no extra launch is needed
@@ -1075,6 +1171,15 @@ snicit_status snicit_stats(snicit_network* net, snicit_stats_t* out) {
         CUDA_TRY(read_counter(net, CNT_CDONE, &v));
         net->stats.const_centroids = v;
     }
+    net->stats.pre_const_rows = 0;
+    net->stats.pre_full_rows = 0;
+    if (net->last_pre_fused) {
+        CUDA_TRY(read_counter(net, CNT_PFCONST, &v));
+        net->stats.pre_const_rows = v;
+        unsigned long long f = 0;
+        CUDA_TRY(cudaMemcpy(&f, net->pf_full.p, sizeof(f), cudaMemcpyDeviceToHost));
+        net->stats.pre_full_rows = (int64_t)f;
+    }
     *out = net->stats;
     return SNICIT_OK;
 }
@@ -1093,7 +1198,12 @@ snicit_status snicit_layer_profile(snicit_network* net, int32_t max, double* ms,
         CUDA_TRY(cudaEventElapsedTime(&t, net->lev[2 * l], net->lev[2 * l + 1]));
         if (ms) ms[l] = t;
         if (rows) rows[l] = h[l];
-        if (bytes) {
+        if (bytes && net->last_pre_fused) {
+            // row-resident kernel: every input row read once, every row alive at t written once
+            int live = 0;
+            CUDA_TRY(read_counter(net, net->live_counter, &live));
+            bytes[l] = 4.0 * net->N * ((double)h[l] + live) + sizeof(PreFusedLayer) * (double)net->last_t;
+        } else if (bytes) {
             const LayerPlan& pl = net->plan[l];
             // algorithmic bytes: rows read + written, weights, bias
             double wb;

@@ -222,6 +222,39 @@ cudaError_t launch_residual_traj(const PostArgs& a, int max_rows, int num_sms, c
 cudaError_t launch_centroid_const(const PostArgs& a, float* cout, int* cdone, int* ndone, int C_max, cudaStream_t st);
 int circ_class_of(int N, int nu);
 
+// ------------------------------------------------------------------ row-resident pre-convergence (kernels_pre_fused.cu)
+enum PfClass : int { PF_NU1 = 0, PF_STR = 1, PF_Q32 = 2 };
+struct PreFusedLayer {
+    int nu;
+    int cls;        // PfClass
+    float w0, b0;   // uniform weight / bias of the layer
+    int dead_next;  // dead_ok[l + 1]: an all-zero row after this layer stays zero (R23)
+    int ymax_fixed; // the constant row YMAX maps to YMAX (sigma(chain(YMAX) + b0) == YMAX, evaluated on
+                    // the host with the kernel's fma order)
+    int pad[2];
+};
+struct PreFusedArgs {
+    int N, t, H;     // H: circular halo (floats) of every staged row, >= 64 and >= 31*nu of STR layers
+    float ymax;
+    int drop;        // drop dead rows (R23)
+    int const_skip;  // carry constant rows by one scalar chain per layer (R26)
+    int gen_str;     // some layer < t is STR with nu != 32 (runtime-stride body needed)
+    const float* yin;
+    float* yout;
+    const int* rows;   // input list [*count]
+    const int* count;
+    int* app_list;     // rows alive at t, appended unordered (nullable)
+    int* app_count;    //   zero on entry
+    int* work;         // row scheduler, zero on entry
+    const PreFusedLayer* layers;  // device [t]
+    unsigned long long* full_rl;  // nullable: += full (non-constant) row-layer evaluations
+    int* n_const;                 // nullable: += rows that became constant
+};
+// 0 if N is not supported (T = N/32 threads must be 32..512)
+int pre_fused_threads(int N);
+size_t pre_fused_smem(int N, int H);
+cudaError_t launch_pre_fused(const PreFusedArgs& a, int num_sms, cudaStream_t st);
+
 // kernels_convert.cu
 cudaError_t launch_iota(int* out, int n, int* count_out, cudaStream_t st);
 cudaError_t launch_fill_i32(int* out, int n, int v, cudaStream_t st);

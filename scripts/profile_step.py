@@ -22,6 +22,7 @@ p.add_argument("--mode", default="radix")
 p.add_argument("--kernel", default="auto")
 p.add_argument("--steps", type=int, default=1)
 p.add_argument("--batch", type=int, default=None)
+p.add_argument("--pre-fused", type=int, default=1)
 a = p.parse_args()
 c = sdgc.CONFIGS[a.config]
 B = a.batch or c["B"]
@@ -36,7 +37,7 @@ st = torch.cuda.Stream()
 g.set_stream(st)
 y0 = torch.from_numpy(Y0).cuda()
 out = torch.empty_like(y0)
-opt = default_options(kernel={"auto": KERNEL_AUTO, "ell": KERNEL_ELL, "circ": KERNEL_CIRC}[a.kernel])
+opt = default_options(kernel={"auto": KERNEL_AUTO, "ell": KERNEL_ELL, "circ": KERNEL_CIRC}[a.kernel], pre_fused=a.pre_fused)
 for _ in range(2):
     g.infer(y0, t=a.t, s=a.s, options=opt, y_out=out)
     g.num_categories()

@@ -377,3 +377,82 @@ def test_cluster_centroid_trajectory(N, L, B, t):
     assert a[2]["residual_at_t"] > 0
     for Y, cats, _, _ in (a, b):
         assert np.array_equal(Y, ref["Y"]) and np.array_equal(cats, ref["categories"])
+
+
+# ------------------------------------------------------------------------------ row-resident pre phase
+
+def _pf_inputs(N, B, seed):
+    """Binary MNIST-like rows plus the degenerate rows the fused kernel branches on: all-zero rows,
+    constant rows (0 < v < 32 and v = 32), rows that die after a few layers, random-valued rows."""
+    rs = np.random.RandomState(seed)
+    if int(np.sqrt(N)) ** 2 == N:
+        Y0 = sdgc.gen_inputs(N, B)
+    else:  # non-square N: binary rows at the SDGC-like density
+        Y0 = (rs.uniform(size=(B, N)) < 0.25).astype(np.float32)
+    Y0[1::7] = 0.0
+    Y0[2::7] = np.float32(32.0)
+    Y0[3::7] = np.float32(0.375)
+    Y0[4::7] *= np.float32(0.02)  # sparse small values: dead after a few layers
+    Y0[5::7] = rs.uniform(0, 32, size=Y0[5::7].shape).astype(np.float32)
+    return Y0
+
+
+@pytest.mark.parametrize("N,nus,B", [(1024, (1, 32), 301), (2048, (1, 32, 64), 97), (4096, (1, 32, 128), 150),
+                                     (8192, (1, 64, 256, 32), 41), (16384, (1, 32, 512), 23)])
+@pytest.mark.parametrize("drop", [1, 0])
+def test_pre_fused_bit_exact(N, nus, B, drop):
+    """Row-resident pre-convergence kernel (every stride class: nu = 1, Q = 32, STR with compile-time
+    nu = 32 and runtime nu = 64) with and without the constant-row shortcut (R26) == the per-layer
+    kernels == the oracle's Eq. 1, bit for bit, on the uncompressed path (t = L: every layer runs in the
+    pre phase) and in the full SNICIT pipeline."""
+    L = 3 * len(nus) + 1
+    nu = np.array([nus[l % len(nus)] for l in range(L)], np.int32)
+    w = np.full((L, 32), 1.0 / 16.0, np.float32)
+    bias = np.repeat(np.array([-0.3 - 0.01 * (l % 3) for l in range(L)], np.float32), N)
+    cn = sdgc.CirculantNetwork(N=N, L=L, nu=nu, w=w, bias=bias, ymax=32.0)
+    net = cn.to_network()
+    Y0 = _pf_inputs(N, B, N + B)
+    plain = oracle.layers_f32(net, Y0)
+    res = {}
+    for pf in (1, 2, 0):
+        Y, cats, st, _ = run_gpu(net, Y0, t=L, drop_dead_rows=drop, pre_fused=pf)
+        assert st["pre_fused"] == (1 if pf else 0)
+        res[pf] = (Y, cats, st)
+        assert np.array_equal(Y, plain), f"pre_fused={pf}"
+        assert np.array_equal(cats, oracle.categories(plain))
+    assert res[1][2]["pre_const_rows"] > 0 and res[2][2]["pre_const_rows"] == 0
+    assert res[1][2]["pre_full_rows"] < res[2][2]["pre_full_rows"]
+    assert res[1][2]["live_at_t"] == res[0][2]["live_at_t"] == res[2][2]["live_at_t"]
+    # SNICIT pipeline with conversion at t = L // 2: fused pre phase == per-layer pre phase
+    Ya, ca, sa, cla = run_gpu(net, Y0, t=L // 2, drop_dead_rows=drop, pre_fused=1)
+    Yb, cb, sb, clb = run_gpu(net, Y0, t=L // 2, drop_dead_rows=drop, pre_fused=0)
+    assert np.array_equal(Ya, Yb) and np.array_equal(ca, cb)
+    assert np.array_equal(ca, oracle.categories(plain))
+    assert np.allclose(Ya, plain, atol=ATOL, rtol=RTOL)
+
+
+def test_pre_fused_positive_bias_and_fallbacks():
+    """A positive bias (no dead-row dropping after it, R23) runs fused and stays exact; per-n weights,
+    per-neuron bias or an unsupported N fall back to the per-layer kernels (stats.pre_fused == 0)."""
+    N, L, B = 4096, 7, 80
+    nu = np.array([1, 32, 128, 1, 32, 128, 1], np.int32)
+    w = np.full((L, 32), 1.0 / 16.0, np.float32)
+    bias = np.full(L * N, -0.35, np.float32)
+    bias[4 * N:5 * N] = 0.05
+    cn = sdgc.CirculantNetwork(N=N, L=L, nu=nu, w=w, bias=bias, ymax=32.0)
+    net = cn.to_network()
+    Y0 = _pf_inputs(N, B, 7)
+    plain = oracle.layers_f32(net, Y0)
+    Y, cats, st, _ = run_gpu(net, Y0, t=L)
+    assert st["pre_fused"] == 1 and np.array_equal(Y, plain)
+    # per-n weights -> per-layer kernels
+    w2 = w.copy()
+    w2[2, 5] = np.float32(0.07)
+    cn2 = sdgc.CirculantNetwork(N=N, L=L, nu=nu, w=w2, bias=bias, ymax=32.0)
+    net2 = cn2.to_network()
+    Y2, _, st2, _ = run_gpu(net2, Y0, t=L)
+    assert st2["pre_fused"] == 0 and np.array_equal(Y2, oracle.layers_f32(net2, Y0))
+    # but a prefix of eligible layers before t still runs fused
+    Y3, _, st3, _ = run_gpu(net2, Y0, t=2)
+    assert st3["pre_fused"] == 1
+    assert np.array_equal(oracle.categories(oracle.layers_f32(net2, Y0)), run_gpu(net2, Y0, t=2)[1])
