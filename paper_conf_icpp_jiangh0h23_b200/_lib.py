@@ -56,10 +56,12 @@ _lib = None
 
 
 def load_library(path: str = LIB_PATH):
-    """Load libsnicit.so and declare the C signatures (raises if the library was not built)."""
+    """Load libsnicit.so and declare the C signatures (raises if the library was not built).
+    SNICIT_LIB overrides the path (A/B builds in experiments)."""
     global _lib
     if _lib is not None:
         return _lib
+    path = os.environ.get("SNICIT_LIB", path)
     if not os.path.exists(path):
         raise SnicitError(f"{path} not found: run __graft_entry__.build() (nvcc, sm_100a)")
     L = ctypes.CDLL(path)

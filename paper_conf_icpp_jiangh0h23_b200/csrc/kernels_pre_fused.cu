@@ -17,17 +17,22 @@
 //        (c, a0 + Q/2), i.e. base offsets b and b + N/2.
 //   Q32  nu == N/32: a thread owns residue class c (T == nu) -- 32 inputs, the two items are
 //        a0 = 0 and a0 = 16 and every rotation is compile-time.
-// Windows never wrap: every buffer carries a circular halo (a copy of the row head, H floats,
-// H >= 64 and >= 31*nu of every STR layer); each layer writes outputs q < H twice.
+// Windows never wrap: every buffer carries a circular halo (a copy of the row head, H floats: 64 for
+// NU1, and 31*nu of STR layers); each layer writes outputs q < H twice.
 //
 // Constant rows (R26, exact): a circulant layer with uniform weight and bias maps a row whose elements
 // are all equal to v to the constant row sigma(chain(v) + b0) -- every output evaluates the same
 // stored-order chain on the same values (the R25 argument of the post phase).  After each layer the
-// CTA tests "all outputs equal" (one __syncthreads_and); a constant row is then carried by one scalar
-// chain per remaining layer and written with plain vector stores.  An all-zero row is dead (R23) when
+// CTA tests "all outputs equal"; a constant row is then carried by one scalar
+// chain per remaining layer and written with plain vector stores.  The test costs no extra barrier:
+// warps vote on their outputs and publish (vote, value) before the layer's barrier.  An all-zero row is dead (R23) when
 // every later bias is <= 0: it leaves without a write.  Survivors are appended (unordered, R24) to the
 // active list at t.  Rows are scheduled dynamically (one atomic per row).
 #include <cuda_runtime.h>
+
+#include <algorithm>
+#include <cstdlib>
+#include <cstring>
 
 #include "snicit_internal.cuh"
 
@@ -41,22 +46,26 @@ constexpr int kPfW = kPfM + 31;
 typedef unsigned long long u64;
 
 // ---------------------------------------------------------------------------- layer bodies
+// Unguarded stores: the last item's outputs past N (q = N .. 17*n1 - 1 < N + 17) are computed from the
+// halo, i.e. they ARE the circular outputs q - N, and land in the output halo where they belong; a
+// thread without a second item recomputes the last item (identical values, benign duplicate stores).
+// The head outputs q < H are also written to the halo (H >= 96 > 47 + 17).
 template <int T>
 __device__ __forceinline__ void pf_body_nu1(const float* __restrict__ in, float* __restrict__ out, float w0, float b0,
                                             float ymax, int H, float& mn, float& mx) {
     constexpr int N = 32 * T;
     constexpr int n1 = (N + kPfM1 - 1) / kPfM1;
     const int i1 = threadIdx.x;
-    const bool has2 = i1 + T < n1;
-    const int i2 = has2 ? i1 + T : n1 - 1;
+    const int i2 = min(i1 + T, n1 - 1);
     const float* s1 = in + kPfM1 * i1;
     const float* s2 = in + kPfM1 * i2;
     u64 R[kPfW1];
 #pragma unroll
     for (int i = 0; i < kPfW1; ++i) R[i] = f2_pack(s1[i], s2[i]);
     const u64 W2 = f2_pack(w0, w0), B2 = f2_pack(b0, b0);
-    const bool full1 = kPfM1 * i1 + kPfM1 <= N;
-    const bool full2 = has2 && kPfM1 * i2 + kPfM1 <= N;
+    float o1s[kPfM1];
+    float* d1 = out + kPfM1 * i1;
+    float* d2 = out + kPfM1 * i2;
 #pragma unroll
     for (int m = 0; m < kPfM1; ++m) {
         u64 acc = 0ull;
@@ -65,35 +74,42 @@ __device__ __forceinline__ void pf_body_nu1(const float* __restrict__ in, float*
         float z1, z2;
         f2_unpack(f2_add(acc, B2), z1, z2);
         const float o1 = sigma(z1, ymax), o2 = sigma(z2, ymax);
-        const int q1 = kPfM1 * i1 + m, q2 = kPfM1 * i2 + m;
-        if (full1 || q1 < N) {
-            out[q1] = o1;
-            if (q1 < H) out[N + q1] = o1;
-            mn = fminf(mn, o1);
-            mx = fmaxf(mx, o1);
-        }
-        if (full2 || (has2 && q2 < N)) {
-            out[q2] = o2;
-            if (q2 < H) out[N + q2] = o2;
-            mn = fminf(mn, o2);
-            mx = fmaxf(mx, o2);
-        }
+        d1[m] = o1;
+        d2[m] = o2;
+        o1s[m] = o1;
+        mn = fminf(mn, fminf(o1, o2));
+        mx = fmaxf(mx, fmaxf(o1, o2));
+    }
+    if (kPfM1 * i1 < H) {  // head outputs -> halo (item 2 never: 17*T > 31*nu_max for every STR layer)
+#pragma unroll
+        for (int m = 0; m < kPfM1; ++m)
+            if (kPfM1 * i1 + m < H) out[N + kPfM1 * i1 + m] = o1s[m];
     }
 }
 
-// NU > 0: compile-time stride; NU == 0: runtime nu
-template <int T, int NU>
+// NU > 0: compile-time stride; NU == 0: runtime nu.  Item 1 (a0 <= Q/2 - 16) never wraps for Q >= 64;
+// item 2 (a-rows a0 + Q/2 + i) wraps: HALO -> the buffers carry H >= 31*nu floats of circular halo;
+// otherwise its a-row index is taken mod Q (Q a power of two: a mask), which keeps the smem small.
+template <int T, int NU, bool HALO>
 __device__ __forceinline__ void pf_body_str(const float* __restrict__ in, float* __restrict__ out, int nu_rt, float w0,
                                             float b0, float ymax, int H, float& mn, float& mx) {
     constexpr int N = 32 * T;
     const int nu = NU ? NU : nu_rt;
+    const int Q = N / nu;
     const int c = (int)threadIdx.x % nu;
     const int a0 = ((int)threadIdx.x / nu) * kPfM;
     const int base = a0 * nu + c;
     const float* s = in + base;
     u64 R[kPfW];
+    if constexpr (HALO) {
 #pragma unroll
-    for (int i = 0; i < kPfW; ++i) R[i] = f2_pack(s[i * nu], s[i * nu + N / 2]);
+        for (int i = 0; i < kPfW; ++i) R[i] = f2_pack(s[i * nu], s[i * nu + N / 2]);
+    } else {
+        const float* sc = in + c;
+        const int k2 = a0 + Q / 2;
+#pragma unroll
+        for (int i = 0; i < kPfW; ++i) R[i] = f2_pack(s[i * nu], sc[((k2 + i) & (Q - 1)) * nu]);
+    }
     const u64 W2 = f2_pack(w0, w0), B2 = f2_pack(b0, b0);
 #pragma unroll
     for (int m = 0; m < kPfM; ++m) {
@@ -107,7 +123,7 @@ __device__ __forceinline__ void pf_body_str(const float* __restrict__ in, float*
         out[q1] = o1;
         out[q2] = o2;
         if (q1 < H) out[N + q1] = o1;
-        if (q2 < H) out[N + q2] = o2;
+        if (HALO && q2 < H) out[N + q2] = o2;
         mn = fminf(mn, fminf(o1, o2));
         mx = fmaxf(mx, fmaxf(o1, o2));
     }
@@ -144,15 +160,36 @@ __device__ __forceinline__ void pf_body_q32(const float* __restrict__ in, float*
     }
 }
 
+// STR wrap handling: a 31*nu halo, or (kPfStrHalo = false) the a-row index mod Q
+template <int T>
+constexpr bool kPfStrHalo = true;  // measured: the masked form (H = 64, 6 CTAs/SM at N = 4096) is slower
+bool pre_fused_str_halo(int N) { return kPfStrHalo<128> || N < 0; }
+
 template <int T>
 struct PfCfg {
     static constexpr int kMinBlocks = T <= 32 ? 16 : (T <= 64 ? 8 : (T <= 128 ? 4 : (T <= 256 ? 2 : 1)));
 };
 
 // ---------------------------------------------------------------------------- the kernel
-// GENSTR: the network has STR layers with nu != 32 (runtime-stride body compiled in)
-template <int T, bool GENSTR>
-__global__ void __launch_bounds__(T, PfCfg<T>::kMinBlocks) pre_fused_kernel(PreFusedArgs a) {
+// Layer descriptors travel in the kernel's parameter space (constant bank).  When every layer has the
+// same weight it is read at a constant offset, so the FFMA2 weight operand is a uniform register
+// (fewer register-file reads than a per-thread copy: measured +5% on the Q32 / STR bodies).
+struct PfLayerParam {
+    float w0, b0;
+    int nu;
+    int flags;  // cls | dead_next << 4 | ymax_fixed << 5
+};
+struct PreFusedParams {
+    PreFusedArgs a;
+    PfLayerParam L[kPfMaxLayers];
+};
+static_assert(sizeof(PreFusedParams) <= 32764, "kernel parameter space");
+
+// GENSTR: the network has STR layers with nu != 32 (runtime-stride body compiled in); WUNI: every
+// layer < t has the same weight
+template <int T, bool GENSTR, bool WUNI>
+__global__ void __launch_bounds__(T, PfCfg<T>::kMinBlocks) pre_fused_kernel(const __grid_constant__ PreFusedParams p) {
+    const PreFusedArgs& a = p.a;
     constexpr int N = 32 * T;
     extern __shared__ __align__(128) unsigned char smem[];
     const int H = a.H;
@@ -161,6 +198,9 @@ __global__ void __launch_bounds__(T, PfCfg<T>::kMinBlocks) pre_fused_kernel(PreF
     float* buf1 = buf0 + S;
     uint64_t* bar = reinterpret_cast<uint64_t*>(buf1 + S);
     int* s_pos = reinterpret_cast<int*>(bar + 1);
+    constexpr int kWarps = T / 32;
+    float* s_rep = reinterpret_cast<float*>(s_pos + 4);  // [2][kWarps] per-warp reference value
+    int* s_ok = reinterpret_cast<int*>(s_rep + 2 * kWarps);  // [2][kWarps] per-warp "all equal" vote
     const int tid = threadIdx.x;
     const int count = *a.count;
     if (tid == 0) {
@@ -189,23 +229,39 @@ __global__ void __launch_bounds__(T, PfCfg<T>::kMinBlocks) pre_fused_kernel(PreF
         bool cst = false, dead = false;
         float v = 0.0f;
         int full = 0;
-        PreFusedLayer d = a.layers[0];
         for (int l = 0; l < a.t; ++l) {
+            // WUNI: one weight for every layer, read at a constant offset -> a uniform register operand
+            const float w0 = WUNI ? p.L[0].w0 : p.L[l].w0, b0 = p.L[l].b0;
+            const int fl = p.L[l].flags;
+            const bool dead_next = (fl >> 4) & 1;
             if (!cst) {
-                // next layer's descriptor, loaded while this layer computes
-                const PreFusedLayer dn = a.layers[min(l + 1, a.t - 1)];
                 float mn = __int_as_float(0x7f800000), mx = -__int_as_float(0x7f800000);
-                if (d.cls == PF_NU1)
-                    pf_body_nu1<T>(in, out, d.w0, d.b0, a.ymax, H, mn, mx);
-                else if (d.cls == PF_Q32)
-                    pf_body_q32<T>(in, out, d.w0, d.b0, a.ymax, H, mn, mx);
-                else if (GENSTR && d.nu != 32)
-                    pf_body_str<T, 0>(in, out, d.nu, d.w0, d.b0, a.ymax, H, mn, mx);
+                const int cls = fl & 15;
+                if (cls == PF_NU1)
+                    pf_body_nu1<T>(in, out, w0, b0, a.ymax, H, mn, mx);
+                else if (cls == PF_Q32)
+                    pf_body_q32<T>(in, out, w0, b0, a.ymax, H, mn, mx);
+                else if (GENSTR && p.L[l].nu != 32)
+                    pf_body_str<T, 0, kPfStrHalo<T>>(in, out, p.L[l].nu, w0, b0, a.ymax, H, mn, mx);
                 else
-                    pf_body_str<T, 32>(in, out, 32, d.w0, d.b0, a.ymax, H, mn, mx);
-                __syncthreads();  // outputs written
-                const float o0 = out[0];
-                const bool all_eq = __syncthreads_and(mn >= o0 && mx <= o0) != 0;
+                    pf_body_str<T, 32, kPfStrHalo<T>>(in, out, 32, w0, b0, a.ymax, H, mn, mx);
+                // "all outputs equal" in one barrier: a warp votes against its lane 0's minimum and
+                // publishes (vote, value) before the barrier; after it every thread combines the warps'
+                // entries (slots double-buffered by layer parity, so no second barrier is needed)
+                {
+                    const float ref = __shfl_sync(0xffffffffu, mn, 0);
+                    const bool ok = __all_sync(0xffffffffu, mn >= ref && mx <= ref);
+                    if ((tid & 31) == 0) {
+                        s_rep[(l & 1) * kWarps + (tid >> 5)] = ref;
+                        s_ok[(l & 1) * kWarps + (tid >> 5)] = ok ? 1 : 0;
+                    }
+                }
+                __syncthreads();  // outputs and votes written
+                bool all_eq = true;
+                const float o0 = s_rep[(l & 1) * kWarps];
+#pragma unroll
+                for (int w = 0; w < kWarps; ++w)
+                    all_eq = all_eq && s_ok[(l & 1) * kWarps + w] && s_rep[(l & 1) * kWarps + w] == o0;
                 ++full;
                 float* tmp = in;
                 in = out;
@@ -213,25 +269,23 @@ __global__ void __launch_bounds__(T, PfCfg<T>::kMinBlocks) pre_fused_kernel(PreF
                 if (all_eq) {
                     v = o0;
                     if (a.const_skip) cst = true;
-                    if (v == 0.0f && a.drop && d.dead_next) {
+                    if (v == 0.0f && a.drop && dead_next) {
                         dead = true;
                         break;
                     }
                 }
-                d = dn;
             } else {
                 // constant row (R26): v' = sigma(chain(v) + b0).  chain(+-0) = +0 exactly, and the host
                 // evaluated chain(YMAX) with the same fma order (ymax_fixed)
-                d = a.layers[l];
                 if (v == 0.0f) {
-                    v = sigma(0.0f + d.b0, a.ymax);
-                } else if (!(v == a.ymax && d.ymax_fixed)) {
+                    v = sigma(0.0f + b0, a.ymax);
+                } else if (!(v == a.ymax && ((fl >> 5) & 1))) {
                     float acc = 0.0f;
 #pragma unroll
-                    for (int n = 0; n < 32; ++n) acc = fmaf(v, d.w0, acc);
-                    v = sigma(acc + d.b0, a.ymax);
+                    for (int n = 0; n < 32; ++n) acc = fmaf(v, w0, acc);
+                    v = sigma(acc + b0, a.ymax);
                 }
-                if (v == 0.0f && a.drop && d.dead_next) {
+                if (v == 0.0f && a.drop && dead_next) {
                     dead = true;
                     break;
                 }
@@ -272,30 +326,49 @@ int pre_fused_threads(int N) {
     return (T == 32 || T == 64 || T == 128 || T == 256 || T == 512) ? T : 0;
 }
 
-size_t pre_fused_smem(int N, int H) { return sizeof(float) * 2 * (size_t)(N + H) + 2 * sizeof(uint64_t); }
+size_t pre_fused_smem(int N, int H) {
+    return sizeof(float) * 2 * (size_t)(N + H) + sizeof(uint64_t) + 4 * sizeof(int) + 4 * sizeof(int) * (N / 32 / 32);
+}
 
-template <int T, bool GENSTR>
-static cudaError_t launch_tg(const PreFusedArgs& a, int num_sms, cudaStream_t st) {
-    const size_t smem = pre_fused_smem(a.N, a.H);
+template <int T, bool GENSTR, bool WUNI>
+static cudaError_t launch_tg(const PreFusedParams& p, int num_sms, cudaStream_t st) {
+    const size_t smem = pre_fused_smem(p.a.N, p.a.H);
     int bps = 0;
-    cudaError_t e = blocks_per_sm((const void*)pre_fused_kernel<T, GENSTR>, T, smem, &bps);
+    cudaError_t e = blocks_per_sm((const void*)pre_fused_kernel<T, GENSTR, WUNI>, T, smem, &bps);
     if (e != cudaSuccess) return e;
     if (bps < 1) return cudaErrorInvalidConfiguration;
-    pre_fused_kernel<T, GENSTR><<<num_sms * bps, T, smem, st>>>(a);
+    static const int bps_env = [] {  // experiment hook: cap the CTAs per SM
+        const char* v = getenv("SNICIT_PF_BPS");
+        return v ? atoi(v) : 0;
+    }();
+    if (bps_env > 0) bps = std::min(bps, bps_env);
+    pre_fused_kernel<T, GENSTR, WUNI><<<num_sms * bps, T, smem, st>>>(p);
     return cudaGetLastError();
 }
 template <int T>
-static cudaError_t launch_t(const PreFusedArgs& a, int num_sms, cudaStream_t st) {
-    return a.gen_str ? launch_tg<T, true>(a, num_sms, st) : launch_tg<T, false>(a, num_sms, st);
+static cudaError_t launch_t(const PreFusedParams& p, bool wuni, int num_sms, cudaStream_t st) {
+    if (p.a.gen_str) return wuni ? launch_tg<T, true, true>(p, num_sms, st) : launch_tg<T, true, false>(p, num_sms, st);
+    return wuni ? launch_tg<T, false, true>(p, num_sms, st) : launch_tg<T, false, false>(p, num_sms, st);
 }
 
-cudaError_t launch_pre_fused(const PreFusedArgs& a, int num_sms, cudaStream_t st) {
+cudaError_t launch_pre_fused(const PreFusedArgs& a, const PreFusedLayer* layers, int num_sms, cudaStream_t st) {
+    if (a.t < 1 || a.t > kPfMaxLayers) return cudaErrorInvalidValue;
+    static thread_local PreFusedParams p;  // 32 KB: not on the stack
+    p.a = a;
+    for (int l = 0; l < a.t; ++l) {
+        p.L[l].w0 = layers[l].w0;
+        p.L[l].b0 = layers[l].b0;
+        p.L[l].nu = layers[l].nu;
+        p.L[l].flags = (layers[l].cls & 15) | (layers[l].dead_next ? 16 : 0) | (layers[l].ymax_fixed ? 32 : 0);
+    }
+    bool wuni = true;
+    for (int l = 1; l < a.t; ++l) wuni = wuni && memcmp(&p.L[l].w0, &p.L[0].w0, sizeof(float)) == 0;
     switch (pre_fused_threads(a.N)) {
-        case 32: return launch_t<32>(a, num_sms, st);
-        case 64: return launch_t<64>(a, num_sms, st);
-        case 128: return launch_t<128>(a, num_sms, st);
-        case 256: return launch_t<256>(a, num_sms, st);
-        case 512: return launch_t<512>(a, num_sms, st);
+        case 32: return launch_t<32>(p, wuni, num_sms, st);
+        case 64: return launch_t<64>(p, wuni, num_sms, st);
+        case 128: return launch_t<128>(p, wuni, num_sms, st);
+        case 256: return launch_t<256>(p, wuni, num_sms, st);
+        case 512: return launch_t<512>(p, wuni, num_sms, st);
         default: return cudaErrorInvalidValue;
     }
 }

@@ -751,14 +751,15 @@ static snicit_status infer_core(snicit_network* net, const float* y0, int64_t ba
         net->prof_layers = 0;
     }
     // row-resident fused pre phase (kernels_pre_fused.cu): one launch for layers 0..t-1
-    bool pf = opt.pre_fused != 0 && tt > 0 && R > 0 && opt.kernel == SNICIT_KERNEL_AUTO && pre_fused_threads(N) > 0;
+    bool pf = opt.pre_fused != 0 && tt > 0 && tt <= kPfMaxLayers && R > 0 && opt.kernel == SNICIT_KERNEL_AUTO &&
+              pre_fused_threads(N) > 0;
     for (int l = 0; l < tt && pf; ++l) pf = net->pf_elig[l] != 0;
     int pf_gen = 0;
-    int pf_H = 64;  // circular halo: nu == 1 windows need 48 floats, STR windows 31*nu
+    int pf_H = 96;  // circular halo: nu == 1 windows read 47 past an item, head items write 68; STR 31*nu
     if (pf) {
         for (int l = 0; l < tt; ++l)
             if (net->pf_layers_h[l].cls == PF_STR) {
-                pf_H = std::max(pf_H, 31 * net->pf_layers_h[l].nu);
+                if (pre_fused_str_halo(N)) pf_H = std::max(pf_H, 31 * net->pf_layers_h[l].nu);
                 if (net->pf_layers_h[l].nu != 32) pf_gen = 1;
             }
         pf_H = (pf_H + 31) / 32 * 32;
@@ -789,10 +790,9 @@ static snicit_status infer_core(snicit_network* net, const float* y0, int64_t ba
         pa.app_list = drop ? lists[li ^ 1] : nullptr;
         pa.app_count = cnt + live_ctr[(ci + 1) % 3];
         pa.work = cnt + CNT_PFWORK;
-        pa.layers = net->pf_layers_d.p;
         pa.full_rl = net->pf_full.p;
         pa.n_const = cnt + CNT_PFCONST;
-        CUDA_TRY(launch_pre_fused(pa, net->num_sms, st));
+        CUDA_TRY(launch_pre_fused(pa, net->pf_layers_h.data(), net->num_sms, st));
         if (prof) CUDA_TRY(cudaEventRecord(net->lev[1], st));
         ++launches;
         circ_layers += tt;

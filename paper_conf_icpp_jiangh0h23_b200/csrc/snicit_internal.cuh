@@ -246,14 +246,16 @@ struct PreFusedArgs {
     int* app_list;     // rows alive at t, appended unordered (nullable)
     int* app_count;    //   zero on entry
     int* work;         // row scheduler, zero on entry
-    const PreFusedLayer* layers;  // device [t]
     unsigned long long* full_rl;  // nullable: += full (non-constant) row-layer evaluations
     int* n_const;                 // nullable: += rows that became constant
 };
 // 0 if N is not supported (T = N/32 threads must be 32..512)
 int pre_fused_threads(int N);
 size_t pre_fused_smem(int N, int H);
-cudaError_t launch_pre_fused(const PreFusedArgs& a, int num_sms, cudaStream_t st);
+bool pre_fused_str_halo(int N);  // STR layers need H >= 31*nu
+constexpr int kPfMaxLayers = 2000;  // t limit of the row-resident kernel (descriptors in parameter space)
+// layers: host descriptors of layers 0..t-1
+cudaError_t launch_pre_fused(const PreFusedArgs& a, const PreFusedLayer* layers, int num_sms, cudaStream_t st);
 
 // kernels_convert.cu
 cudaError_t launch_iota(int* out, int n, int* count_out, cudaStream_t st);
