@@ -561,11 +561,24 @@ __global__ void __launch_bounds__(256) centroid_const_kernel(PostArgs a, float* 
     float* s_acc = reinterpret_cast<float*>(s_wb + nl);
     if (threadIdx.x == 0) {
         float v = __uint_as_float(an);
+        // the chain is a pure function of (v, w0): reuse the previous layer's value when both repeat
+        // (SDGC: one weight for every layer and a fixed point v = YMAX -> one chain for all layers)
+        float pv = 0.0f, pw = 0.0f, pacc = 0.0f;
+        bool have = false;
         for (int l = 0; l < nl; ++l) {
             const float2 wb = s_wb[l];
-            float acc = 0.0f;
+            float acc;
+            if (have && __float_as_uint(v) == __float_as_uint(pv) && __float_as_uint(wb.x) == __float_as_uint(pw)) {
+                acc = pacc;
+            } else {
+                acc = 0.0f;
 #pragma unroll
-            for (int n = 0; n < kPK; ++n) acc = fmaf(v, wb.x, acc);
+                for (int n = 0; n < kPK; ++n) acc = fmaf(v, wb.x, acc);
+                pv = v;
+                pw = wb.x;
+                pacc = acc;
+                have = true;
+            }
             s_acc[l] = acc;
             v = sigma(acc + wb.y, a.ymax);
         }

@@ -165,6 +165,11 @@ template <int T>
 constexpr bool kPfStrHalo = true;  // measured: the masked form (H = 64, 6 CTAs/SM at N = 4096) is slower
 bool pre_fused_str_halo(int N) { return kPfStrHalo<128> || N < 0; }
 
+// row buffers: two (ping-pong) and, when one CTA fills the SM anyway (N = 16384), a third that receives
+// the next row while this one computes (otherwise the next row is only prefetched into L2)
+template <int T>
+constexpr int kPfBufs = T >= 512 ? 3 : 2;
+
 template <int T>
 struct PfCfg {
     static constexpr int kMinBlocks = T <= 32 ? 16 : (T <= 64 ? 8 : (T <= 128 ? 4 : (T <= 256 ? 2 : 1)));
@@ -194,38 +199,55 @@ __global__ void __launch_bounds__(T, PfCfg<T>::kMinBlocks) pre_fused_kernel(cons
     extern __shared__ __align__(128) unsigned char smem[];
     const int H = a.H;
     const int S = N + H;  // buffer stride (floats): row + circular halo
-    float* buf0 = reinterpret_cast<float*>(smem);
-    float* buf1 = buf0 + S;
-    uint64_t* bar = reinterpret_cast<uint64_t*>(buf1 + S);
-    int* s_pos = reinterpret_cast<int*>(bar + 1);
+    constexpr int NB = kPfBufs<T>;
+    float* const buf = reinterpret_cast<float*>(smem);  // NB buffers of S floats
+    uint64_t* bar = reinterpret_cast<uint64_t*>(buf + NB * S);  // [2] row loads, alternating per row
+    int* s_pos = reinterpret_cast<int*>(bar + 2);               // [0] first row, [2 + (k & 1)] next row
     constexpr int kWarps = T / 32;
     float* s_rep = reinterpret_cast<float*>(s_pos + 4);  // [2][kWarps] per-warp reference value
     int* s_ok = reinterpret_cast<int*>(s_rep + 2 * kWarps);  // [2][kWarps] per-warp "all equal" vote
     const int tid = threadIdx.x;
     const int count = *a.count;
     if (tid == 0) {
-        mbar_init(bar, 1);
+        mbar_init(&bar[0], 1);
+        mbar_init(&bar[1], 1);
         fence_proxy_async_smem();
-        *s_pos = atomicAdd(a.work, 1);
+        s_pos[0] = atomicAdd(a.work, 1);
     }
     __syncthreads();
-    int pos = *s_pos;
-    uint32_t phase = 0;
-    while (pos < count) {
+    int pos = s_pos[0];
+    // one row (and its circular halo: a second copy of the row head) -> buffer `dst`, completion on `b`
+    auto issue_load = [&](int p_, float* dst, uint64_t* b) {
+        const float* g = a.yin + (size_t)__ldg(a.rows + p_) * N;
+        mbar_arrive_expect_tx(b, (uint32_t)(S * 4));
+        bulk_g2s(dst, g, N * 4, b);
+        bulk_g2s(dst + N, g, H * 4, b);
+    };
+    int i_in = 0, i_out = 1, i_pf = 2;  // buffer roles (NB == 3: i_pf receives the next row)
+    uint32_t ph = 0;                    // phase bit of bar[0], bar[1]
+    if (NB == 3 && tid == 0 && pos < count) issue_load(pos, buf, &bar[0]);
+    for (int k = 0; pos < count; ++k) {
         const int row = __ldg(a.rows + pos);
-        const float* g = a.yin + (size_t)row * N;
-        __syncthreads();  // every thread has read s_pos
         if (tid == 0) {
-            bulk_wait_read0();  // the previous row's TMA store has finished reading its buffer
-            mbar_arrive_expect_tx(bar, (uint32_t)(S * 4));
-            bulk_g2s(buf0, g, N * 4, bar);
-            bulk_g2s(buf0 + N, g, H * 4, bar);  // circular halo: a second copy of the row head
-            *s_pos = atomicAdd(a.work, 1);      // next row (read after the end-of-row barrier)
+            if (NB == 2) {
+                bulk_wait_read0();  // the previous row's TMA store has finished reading its buffer
+                issue_load(pos, buf, &bar[k & 1]);
+            }
+            const int np = atomicAdd(a.work, 1);  // next row (read after the end-of-row barrier)
+            s_pos[2 + (k & 1)] = np;
+            if (np < count) {
+                if (NB == 3) {  // load it now, behind this row's compute
+                    bulk_wait_read0();
+                    issue_load(np, buf + i_pf * S, &bar[(k + 1) & 1]);
+                } else if (a.l2_prefetch) {  // pull it into L2 so its load at the next row start is short
+                    bulk_prefetch_l2(a.yin + (size_t)__ldg(a.rows + np) * N, N * 4);
+                }
+            }
         }
-        mbar_wait(bar, phase);
-        phase ^= 1u;
-        float* in = buf0;
-        float* out = buf1;
+        mbar_wait(&bar[k & 1], (ph >> (k & 1)) & 1u);
+        ph ^= 1u << (k & 1);
+        float* in = buf + i_in * S;
+        float* out = buf + i_out * S;
         bool cst = false, dead = false;
         float v = 0.0f;
         int full = 0;
@@ -266,6 +288,9 @@ __global__ void __launch_bounds__(T, PfCfg<T>::kMinBlocks) pre_fused_kernel(cons
                 float* tmp = in;
                 in = out;
                 out = tmp;
+                const int ti = i_in;
+                i_in = i_out;
+                i_out = ti;
                 if (all_eq) {
                     v = o0;
                     if (a.const_skip) cst = true;
@@ -315,7 +340,15 @@ __global__ void __launch_bounds__(T, PfCfg<T>::kMinBlocks) pre_fused_kernel(cons
             if (a.n_const && cst) atomicAdd(a.n_const, 1);
         }
         __syncthreads();  // buffers free, next position visible
-        pos = *s_pos;
+        pos = s_pos[2 + (k & 1)];
+        if (NB == 3) {  // the prefetched row becomes the input; the result buffer (store pending) the target
+            const int ti = i_in;
+            i_in = i_pf;
+            i_pf = ti;
+        } else {
+            i_in = 0;
+            i_out = 1;
+        }
     }
     if (tid == 0) bulk_wait0();
 }
@@ -327,7 +360,8 @@ int pre_fused_threads(int N) {
 }
 
 size_t pre_fused_smem(int N, int H) {
-    return sizeof(float) * 2 * (size_t)(N + H) + sizeof(uint64_t) + 4 * sizeof(int) + 4 * sizeof(int) * (N / 32 / 32);
+    const int nb = N / 32 >= 512 ? 3 : 2;  // kPfBufs
+    return sizeof(float) * nb * (size_t)(N + H) + 2 * sizeof(uint64_t) + 4 * sizeof(int) + 4 * sizeof(int) * (N / 32 / 32);
 }
 
 template <int T, bool GENSTR, bool WUNI>
@@ -355,6 +389,11 @@ cudaError_t launch_pre_fused(const PreFusedArgs& a, const PreFusedLayer* layers,
     if (a.t < 1 || a.t > kPfMaxLayers) return cudaErrorInvalidValue;
     static thread_local PreFusedParams p;  // 32 KB: not on the stack
     p.a = a;
+    static const int l2pf = [] {  // experiment hook (default on)
+        const char* v = getenv("SNICIT_PF_L2PF");
+        return v ? atoi(v) : 1;
+    }();
+    p.a.l2_prefetch = l2pf;
     for (int l = 0; l < a.t; ++l) {
         p.L[l].w0 = layers[l].w0;
         p.L[l].b0 = layers[l].b0;

@@ -57,6 +57,10 @@ __device__ __forceinline__ void bulk_s2g(void* gdst, const void* ssrc, uint32_t 
                  "r"(bytes)
                  : "memory");
 }
+// L2 prefetch of a global range (TMA engine, no completion tracking)
+__device__ __forceinline__ void bulk_prefetch_l2(const void* gsrc, uint32_t bytes) {
+    asm volatile("cp.async.bulk.prefetch.L2.global [%0], %1;" ::"l"(gsrc), "r"(bytes) : "memory");
+}
 __device__ __forceinline__ void bulk_commit() { asm volatile("cp.async.bulk.commit_group;" ::: "memory"); }
 __device__ __forceinline__ void bulk_wait_read0() { asm volatile("cp.async.bulk.wait_group.read 0;" ::: "memory"); }
 __device__ __forceinline__ void bulk_wait_read1() { asm volatile("cp.async.bulk.wait_group.read 1;" ::: "memory"); }
@@ -239,6 +243,7 @@ struct PreFusedArgs {
     int drop;        // drop dead rows (R23)
     int const_skip;  // carry constant rows by one scalar chain per layer (R26)
     int gen_str;     // some layer < t is STR with nu != 32 (runtime-stride body needed)
+    int l2_prefetch; // two-buffer configurations: prefetch the next row into L2
     const float* yin;
     float* yout;
     const int* rows;   // input list [*count]

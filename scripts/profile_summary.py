@@ -15,9 +15,20 @@ print(f"* metric: {b['metric']}; value **{b['value']:.4g} {b['unit']}**, {b['ms_
       f"({b['config']['workload']}, t={b['config']['t']}, s={b['config']['s']})")
 r = b.get("roofline") or {}
 if r:
-    print(f"* dominant kernel `{r['kernel']}`: achieved {r['achieved']:.0f} GB/s of {r['peak']:.0f} GB/s "
-          f"({r['peak_source']}) = **{100 * r['frac']:.1f}%**, {r['launches']} launches, "
+    print(f"* dominant kernel `{r['kernel']}` ({r['bound']}-bound): achieved {r['achieved']:.1f} {r['unit']} of "
+          f"{r['peak']:.1f} {r['unit']} ({r['peak_source']}) = **{100 * r['frac']:.1f}%**, {r['launches']} launches, "
           f"{100 * (r.get('share_of_step') or 0):.1f}% of the step (CUDA events, live)")
+    if r.get("hbm"):
+        print(f"  * its HBM traffic: {r['hbm']['achieved_gbs']:.0f} GB/s algorithmic ({100 * r['hbm']['frac']:.1f}% of HBM); "
+              f"ncu DRAM bytes per launch {r.get('traffic')} ({r.get('traffic_source')})")
+    if r.get("no_const_skip"):
+        q = r["no_const_skip"]
+        print(f"  * without the constant-row shortcut (pre_fused = 2): {q['avg_launch_ms']:.3f} ms, "
+              f"{q['full_row_layers']} full row-layers, **{100 * q['frac']:.1f}%** of the FMA peak")
+    if r.get("per_layer_kernels"):
+        q = r["per_layer_kernels"]
+        print(f"  * one launch per layer (pre_fused = 0): {q['ms_total']:.3f} ms over {q['launches']} launches, "
+              f"{q['achieved']:.0f} GB/s = **{100 * q['frac']:.1f}%** of HBM; by stride {q.get('by_stride')}")
 for k in ("uncompressed", "e2e", "cpu_baseline"):
     if b.get(k):
         print(f"* {k}: {b[k]['value']:.4g} {b[k]['unit']}" + (f" ({b[k].get('sample')}, {b[k].get('cores')} cores)" if k == "cpu_baseline" else ""))
