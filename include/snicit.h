@@ -173,10 +173,15 @@ snicit_status snicit_infer(snicit_network* net, const float* y0, int64_t batch,
  * P:297-302; 32x fewer bytes to upload than fp32 rows).  Row r of Y0 is
  *   Y0[r][j] = (y0_bits[r*W + j/32] >> (j % 32)) & 1 ? one_value : 0.0f,   W = ceil(N/32) words,
  * i.e. bit j%32 (LSB first) of 32-bit word j/32; bits of the last word beyond N are ignored.
- * y0_bits: batch*W uint32, device pointer if bits_on_device else host (copied to the device
- * inside the call).  one_value: finite.  The rows are unpacked on the device into the handle's
- * workspace and the inference proceeds exactly as snicit_infer on the equivalent fp32 Y0 (same
- * results, tested).  All other arguments as snicit_infer. */
+ * y0_bits: batch*W uint32, device pointer if bits_on_device else host.  one_value: finite.
+ * When the row-resident pre-convergence kernel applies (options.pre_fused, N % 128 == 0) it reads
+ * each row's bits itself and expands them in shared memory (no fp32 Y0 in HBM); host bits are then
+ * uploaded in chunks of 2048 rows by the copy engine on a side stream WHILE the kernel runs (it
+ * waits per chunk on a ready flag), so the upload overlaps the compute (pinned host memory gives
+ * the asynchronous copies; pageable memory works but the copies block the host).  Otherwise the
+ * rows are copied, then unpacked by
+ * a kernel into the handle's workspace.  Either way the inference proceeds exactly as snicit_infer
+ * on the equivalent fp32 Y0 (same results, tested).  All other arguments as snicit_infer. */
 snicit_status snicit_infer_packed(snicit_network* net, const uint32_t* y0_bits, int64_t batch,
                                   int32_t bits_on_device, float one_value, int64_t row_offset,
                                   int32_t threshold_layer, int32_t centroid_count,

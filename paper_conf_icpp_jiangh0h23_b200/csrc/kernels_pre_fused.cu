@@ -217,35 +217,60 @@ __global__ void __launch_bounds__(T, PfCfg<T>::kMinBlocks) pre_fused_kernel(cons
     __syncthreads();
     int pos = s_pos[0];
     // one row (and its circular halo: a second copy of the row head) -> buffer `dst`, completion on `b`
-    auto issue_load = [&](int p_, float* dst, uint64_t* b) {
-        const float* g = a.yin + (size_t)__ldg(a.rows + p_) * N;
-        mbar_arrive_expect_tx(b, (uint32_t)(S * 4));
-        bulk_g2s(dst, g, N * 4, b);
-        bulk_g2s(dst + N, g, H * 4, b);
+    uint32_t* s_bits = reinterpret_cast<uint32_t*>(s_ok + 2 * kWarps);  // [2][N/32] packed rows (a.ybits)
+    auto issue_load = [&](int p_, float* dst, uint64_t* b, int slot) {
+        const size_t r_ = (size_t)__ldg(a.rows + p_);
+        if (a.ybits) {  // packed binary row: N/8 bytes
+            if (a.ready) {  // streamed upload: wait until the copy engine has delivered this row's chunk
+                const int* f = a.ready + r_ / a.ready_rows;
+                while (ld_acquire_gpu(f) == 0) __nanosleep(256);
+                fence_proxy_async_global();
+            }
+            mbar_arrive_expect_tx(b, (uint32_t)(N / 8));
+            bulk_g2s(s_bits + slot * (N / 32), a.ybits + r_ * (N / 32), N / 8, b);
+        } else {
+            const float* g = a.yin + r_ * N;
+            mbar_arrive_expect_tx(b, (uint32_t)(S * 4));
+            bulk_g2s(dst, g, N * 4, b);
+            bulk_g2s(dst + N, g, H * 4, b);
+        }
     };
     int i_in = 0, i_out = 1, i_pf = 2;  // buffer roles (NB == 3: i_pf receives the next row)
     uint32_t ph = 0;                    // phase bit of bar[0], bar[1]
-    if (NB == 3 && tid == 0 && pos < count) issue_load(pos, buf, &bar[0]);
+    if (NB == 3 && tid == 0 && pos < count) issue_load(pos, buf, &bar[0], 0);
     for (int k = 0; pos < count; ++k) {
         const int row = __ldg(a.rows + pos);
         if (tid == 0) {
             if (NB == 2) {
                 bulk_wait_read0();  // the previous row's TMA store has finished reading its buffer
-                issue_load(pos, buf, &bar[k & 1]);
+                issue_load(pos, buf, &bar[k & 1], k & 1);
             }
             const int np = atomicAdd(a.work, 1);  // next row (read after the end-of-row barrier)
             s_pos[2 + (k & 1)] = np;
             if (np < count) {
                 if (NB == 3) {  // load it now, behind this row's compute
                     bulk_wait_read0();
-                    issue_load(np, buf + i_pf * S, &bar[(k + 1) & 1]);
-                } else if (a.l2_prefetch) {  // pull it into L2 so its load at the next row start is short
+                    issue_load(np, buf + i_pf * S, &bar[(k + 1) & 1], (k + 1) & 1);
+                } else if (a.l2_prefetch && !a.ybits) {  // pull it into L2: its load at the next row start is short
                     bulk_prefetch_l2(a.yin + (size_t)__ldg(a.rows + np) * N, N * 4);
                 }
             }
         }
         mbar_wait(&bar[k & 1], (ph >> (k & 1)) & 1u);
         ph ^= 1u << (k & 1);
+        if (a.ybits) {  // expand the bits (value a.one, as snicit_infer_packed's unpack) + the halo copy
+            float* dst = buf + i_in * S;
+            const uint32_t* sb = s_bits + (k & 1) * (N / 32);
+            const int wq = tid >> 5, lane = tid & 31;
+#pragma unroll 4
+            for (int j = 0; j < 32; ++j) {  // warp wq: words 32 wq .. 32 wq + 31, lane = bit (conflict-free)
+                const int wi = wq * 32 + j;
+                const float val = ((sb[wi] >> lane) & 1u) ? a.one : 0.0f;
+                dst[wi * 32 + lane] = val;
+                if (wi * 32 < H) dst[N + wi * 32 + lane] = val;
+            }
+            __syncthreads();
+        }
         float* in = buf + i_in * S;
         float* out = buf + i_out * S;
         bool cst = false, dead = false;
@@ -361,7 +386,8 @@ int pre_fused_threads(int N) {
 
 size_t pre_fused_smem(int N, int H) {
     const int nb = N / 32 >= 512 ? 3 : 2;  // kPfBufs
-    return sizeof(float) * nb * (size_t)(N + H) + 2 * sizeof(uint64_t) + 4 * sizeof(int) + 4 * sizeof(int) * (N / 32 / 32);
+    return sizeof(float) * nb * (size_t)(N + H) + 2 * sizeof(uint64_t) + 4 * sizeof(int) + 4 * sizeof(int) * (N / 32 / 32) +
+           2 * sizeof(uint32_t) * (size_t)(N / 32);  // packed-row slots
 }
 
 template <int T, bool GENSTR, bool WUNI>

@@ -101,6 +101,10 @@ struct snicit_network {
     DevBuf<uint8_t> segflag;  // row flags OR-ed by segmented layers (kept zero by the clearing compaction)
     DevBuf<int> rowctr;       // per-position warp counters of the column-streaming kernel (self-clearing)
     DevBuf<uint32_t> bits;    // packed binary input rows (snicit_infer_packed, host bits)
+    DevBuf<int> bits_ready;   // per chunk of uploaded rows: set by the copy engine after the chunk
+    cudaStream_t copy_stream = nullptr;  // non-blocking upload stream (overlaps the row-resident kernel)
+    cudaEvent_t cev[2] = {nullptr, nullptr};
+    int* h_ones = nullptr;    // pinned source of the ready flags
     DevBuf<int> cdone;        // per centroid: carried to L by the constant-row kernel
     DevBuf<double> F;
     DevBuf<int> counters;
@@ -287,6 +291,11 @@ void snicit_free_network(snicit_network* net) {
     net->ac.release();
     net->F.release();
     if (net->h_counters) cudaFreeHost(net->h_counters);
+    if (net->h_ones) cudaFreeHost(net->h_ones);
+    for (auto& e : net->cev)
+        if (e) cudaEventDestroy(e);
+    if (net->copy_stream) cudaStreamDestroy(net->copy_stream);
+    net->bits_ready.release();
     for (auto& e : net->ev)
         if (e) cudaEventDestroy(e);
     for (auto& e : net->lev)
@@ -660,15 +669,40 @@ static cudaError_t read_counter(snicit_network* net, int which, int* outv) {
 
 extern "C" {
 
-// y0_mode: 0 = y0 is a device pointer, 1 = host pointer, 2 = the input rows are already in net->Ya
+// Row-resident pre phase applicable?  (kernels_pre_fused.cu: circulant layers < t with 32 taps,
+// uniform weight and bias, N / 32 in 32..512, t <= kPfMaxLayers, smem fits); *H = circular halo
+static bool pf_plan(const snicit_network* net, int tt, const snicit_options& opt, int R, int* H, int* gen) {
+    const int N = net->N;
+    bool pf = opt.pre_fused != 0 && tt > 0 && tt <= kPfMaxLayers && R > 0 && opt.kernel == SNICIT_KERNEL_AUTO &&
+              pre_fused_threads(N) > 0;
+    for (int l = 0; l < tt && pf; ++l) pf = net->pf_elig[l] != 0;
+    int h = 96, g = 0;  // nu == 1 windows read 47 past an item, head items write 68; STR 31*nu
+    if (pf) {
+        for (int l = 0; l < tt; ++l)
+            if (net->pf_layers_h[l].cls == PF_STR) {
+                if (pre_fused_str_halo(N)) h = std::max(h, 31 * net->pf_layers_h[l].nu);
+                if (net->pf_layers_h[l].nu != 32) g = 1;
+            }
+        h = (h + 31) / 32 * 32;
+        if (h > N || pre_fused_smem(N, h) > (size_t)227 * 1024) pf = false;
+    }
+    *H = h;
+    *gen = g;
+    return pf;
+}
+
+// y0_mode: 0 = y0 is a device pointer, 1 = host pointer, 2 = the input rows are already in net->Ya,
+// 3 = packed binary rows `bits` (device-accessible, possibly host-mapped) read by the row-resident
+// kernel (the caller checked pf_plan)
 // (snicit_infer_packed unpacked them there)
 static snicit_status infer_core(snicit_network* net, const float* y0, int64_t batch, int32_t y0_mode,
                                 int64_t row_offset, int32_t t, int32_t s, const snicit_options* opt_in, float* y_out,
-                                int32_t y_out_on_device) {
+                                int32_t y_out_on_device, const uint32_t* bits = nullptr, float one = 1.0f,
+                                const int* bits_ready = nullptr, int ready_rows = 0) {
     const int32_t y0_on_device = y0_mode == 0;
     if (!net) return fail(SNICIT_E_INVALID_ARG, "net NULL");
     if (batch < 0 || batch > 0x7fffffffLL) return fail(SNICIT_E_INVALID_ARG, "batch out of range");
-    if (batch > 0 && !y0 && y0_mode != 2) return fail(SNICIT_E_INVALID_ARG, "y0 NULL");
+    if (batch > 0 && !y0 && y0_mode < 2) return fail(SNICIT_E_INVALID_ARG, "y0 NULL");
     if (t < 0) return fail(SNICIT_E_INVALID_ARG, "threshold_layer < 0");
     if (s < 1) return fail(SNICIT_E_INVALID_ARG, "centroid_count < 1");
     if (row_offset < 0) return fail(SNICIT_E_INVALID_ARG, "row_offset < 0");
@@ -697,7 +731,7 @@ static snicit_status infer_core(snicit_network* net, const float* y0, int64_t ba
     CUDA_TRY(cudaSetDevice(net->device));
     CUDA_TRY(ensure_workspace(net, R, s, n_seg));
     cudaStream_t st = net->stream;
-    int64_t launches = y0_mode == 2 ? 1 : 0;  // + the unpack kernel of snicit_infer_packed
+    int64_t launches = y0_mode == 2 ? 1 : 0;  // + the unpack kernel of snicit_infer_packed (mode 2)
     int circ_layers = 0;
     net->have_result = false;
     snicit_stats_t stats{};
@@ -711,6 +745,8 @@ static snicit_status infer_core(snicit_network* net, const float* y0, int64_t ba
     int nxt_i = 0;
     if (y0_on_device) {
         cur = y0;
+    } else if (y0_mode == 3) {
+        cur = nullptr;  // the row-resident kernel reads the packed rows itself
     } else {
         if (y0_mode == 1)
             CUDA_TRY(cudaMemcpyAsync(net->Ya.p, y0, sizeof(float) * (size_t)R * N, cudaMemcpyHostToDevice, st));
@@ -751,20 +787,9 @@ static snicit_status infer_core(snicit_network* net, const float* y0, int64_t ba
         net->prof_layers = 0;
     }
     // row-resident fused pre phase (kernels_pre_fused.cu): one launch for layers 0..t-1
-    bool pf = opt.pre_fused != 0 && tt > 0 && tt <= kPfMaxLayers && R > 0 && opt.kernel == SNICIT_KERNEL_AUTO &&
-              pre_fused_threads(N) > 0;
-    for (int l = 0; l < tt && pf; ++l) pf = net->pf_elig[l] != 0;
-    int pf_gen = 0;
-    int pf_H = 96;  // circular halo: nu == 1 windows read 47 past an item, head items write 68; STR 31*nu
-    if (pf) {
-        for (int l = 0; l < tt; ++l)
-            if (net->pf_layers_h[l].cls == PF_STR) {
-                if (pre_fused_str_halo(N)) pf_H = std::max(pf_H, 31 * net->pf_layers_h[l].nu);
-                if (net->pf_layers_h[l].nu != 32) pf_gen = 1;
-            }
-        pf_H = (pf_H + 31) / 32 * 32;
-        if (pf_H > N || pre_fused_smem(N, pf_H) > (size_t)227 * 1024) pf = false;
-    }
+    int pf_H = 96, pf_gen = 0;
+    const bool pf = pf_plan(net, tt, opt, R, &pf_H, &pf_gen);
+    if (y0_mode == 3 && !pf && R > 0) return fail(SNICIT_E_STATE, "packed rows without the row-resident kernel");
     net->last_pre_fused = pf;
     stats.pre_fused = pf ? 1 : 0;
     if (pf) {
@@ -784,6 +809,10 @@ static snicit_status infer_core(snicit_network* net, const float* y0, int64_t ba
         pa.const_skip = opt.pre_fused == 1 ? 1 : 0;
         pa.gen_str = pf_gen;
         pa.yin = cur;
+        pa.ybits = y0_mode == 3 ? bits : nullptr;
+        pa.one = one;
+        pa.ready = y0_mode == 3 ? bits_ready : nullptr;
+        pa.ready_rows = ready_rows;
         pa.yout = bufs[nxt_i];
         pa.rows = lists[li];
         pa.count = cnt + live_ctr[ci];
@@ -1111,14 +1140,64 @@ snicit_status snicit_infer_packed(snicit_network* net, const uint32_t* y0_bits, 
     const int n_seg = (opt && opt->n_segments > 0 && opt->n_segments <= N) ? opt->n_segments : N;
     CUDA_TRY(ensure_workspace(net, R, s, n_seg));
     const uint32_t* bits = y0_bits;
+    snicit_options o;
+    if (opt)
+        o = *opt;
+    else
+        snicit_default_options(&o);
+    int H = 0, gen = 0;
+    const bool direct = N % 128 == 0 && pf_plan(net, std::min(t, net->L), o, R, &H, &gen);
+    const int* ready = nullptr;
+    int ready_rows = 0;
+    bool streamed = false;
     if (!bits_on_device && R > 0) {
         CUDA_TRY(net->bits.ensure((size_t)R * W));
-        CUDA_TRY(cudaMemcpyAsync(net->bits.p, y0_bits, sizeof(uint32_t) * (size_t)R * W, cudaMemcpyHostToDevice,
-                                 net->stream));
+        if (direct) {
+            // streamed upload: the copy engine delivers chunks of rows on a side stream while the
+            // row-resident kernel runs; each chunk is followed by its ready flag (the kernel polls it
+            // before loading a row of the chunk), so the upload overlaps the compute
+            constexpr int kChunk = 2048;
+            const int nch = (R + kChunk - 1) / kChunk;
+            if (!net->copy_stream) CUDA_TRY(cudaStreamCreateWithFlags(&net->copy_stream, cudaStreamNonBlocking));
+            for (auto& e : net->cev)
+                if (!e) CUDA_TRY(cudaEventCreateWithFlags(&e, cudaEventDisableTiming));
+            if (!net->h_ones) {
+                CUDA_TRY(cudaMallocHost(&net->h_ones, sizeof(int)));
+                *net->h_ones = 1;
+            }
+            CUDA_TRY(net->bits_ready.ensure((size_t)nch));
+            CUDA_TRY(cudaMemsetAsync(net->bits_ready.p, 0, sizeof(int) * nch, net->stream));
+            CUDA_TRY(cudaEventRecord(net->cev[0], net->stream));
+            CUDA_TRY(cudaStreamWaitEvent(net->copy_stream, net->cev[0], 0));
+            for (int c = 0; c < nch; ++c) {
+                const size_t r0 = (size_t)c * kChunk, nr = std::min<size_t>(kChunk, R - r0);
+                CUDA_TRY(cudaMemcpyAsync(net->bits.p + r0 * W, y0_bits + r0 * W, sizeof(uint32_t) * nr * W,
+                                         cudaMemcpyHostToDevice, net->copy_stream));
+                CUDA_TRY(cudaMemcpyAsync(net->bits_ready.p + c, net->h_ones, sizeof(int), cudaMemcpyHostToDevice,
+                                         net->copy_stream));
+            }
+            CUDA_TRY(cudaEventRecord(net->cev[1], net->copy_stream));
+            ready = net->bits_ready.p;
+            ready_rows = kChunk;
+            streamed = true;
+        } else {
+            CUDA_TRY(cudaMemcpyAsync(net->bits.p, y0_bits, sizeof(uint32_t) * (size_t)R * W, cudaMemcpyHostToDevice,
+                                     net->stream));
+        }
         bits = net->bits.p;
     }
-    if (R > 0) CUDA_TRY(launch_unpack_bits(bits, R, N, one_value, net->Ya.p, net->num_sms, net->stream));
-    return infer_core(net, nullptr, batch, 2, row_offset, t, s, opt, y_out, y_out_on_device);
+    snicit_status stt;
+    if (direct) {
+        // the row-resident kernel expands each row's bits in shared memory (no fp32 Y0 in HBM)
+        stt = infer_core(net, nullptr, batch, 3, row_offset, t, s, opt, y_out, y_out_on_device, bits, one_value, ready,
+                         ready_rows);
+    } else {
+        if (R > 0) CUDA_TRY(launch_unpack_bits(bits, R, N, one_value, net->Ya.p, net->num_sms, net->stream));
+        stt = infer_core(net, nullptr, batch, 2, row_offset, t, s, opt, y_out, y_out_on_device);
+    }
+    // later work on the handle's stream (and the next upload) is ordered after this upload
+    if (streamed) CUDA_TRY(cudaStreamWaitEvent(net->stream, net->cev[1], 0));
+    return stt;
 }
 
 snicit_status snicit_categories(snicit_network* net, int64_t* rows, int64_t* count, int32_t rows_on_device) {

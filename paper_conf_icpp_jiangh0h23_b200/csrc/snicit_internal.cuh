@@ -57,6 +57,14 @@ __device__ __forceinline__ void bulk_s2g(void* gdst, const void* ssrc, uint32_t 
                  "r"(bytes)
                  : "memory");
 }
+// acquire load of a flag written by another agent (copy engine / other kernel), gpu scope
+__device__ __forceinline__ int ld_acquire_gpu(const int* p) {
+    int v;
+    asm volatile("ld.acquire.gpu.global.b32 %0, [%1];" : "=r"(v) : "l"(p) : "memory");
+    return v;
+}
+// order generic-proxy observations before later async-proxy (TMA) global accesses
+__device__ __forceinline__ void fence_proxy_async_global() { asm volatile("fence.proxy.async.global;" ::: "memory"); }
 // L2 prefetch of a global range (TMA engine, no completion tracking)
 __device__ __forceinline__ void bulk_prefetch_l2(const void* gsrc, uint32_t bytes) {
     asm volatile("cp.async.bulk.prefetch.L2.global [%0], %1;" ::"l"(gsrc), "r"(bytes) : "memory");
@@ -245,6 +253,10 @@ struct PreFusedArgs {
     int gen_str;     // some layer < t is STR with nu != 32 (runtime-stride body needed)
     int l2_prefetch; // two-buffer configurations: prefetch the next row into L2
     const float* yin;
+    const uint32_t* ybits;  // non-null: input rows as packed bits (N/32 words per row, LSB first), value `one`
+    float one;
+    const int* ready;       // nullable: ready[r / ready_rows] != 0 once rows of that chunk are in ybits
+    int ready_rows;         //   (uploaded by the copy engine while the kernel runs)
     float* yout;
     const int* rows;   // input list [*count]
     const int* count;

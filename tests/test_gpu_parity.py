@@ -113,10 +113,14 @@ def test_column_stream_kernel_bit_exact(N, nus, rows, uniform):
 
 
 @pytest.mark.parametrize("N,L,B,t,dev", [(1024, 40, 700, 4, True), (1024, 40, 700, 40, False),
-                                         (4096, 20, 300, 3, True), (16384, 6, 20, 2, False)])
+                                         (4096, 20, 300, 3, True), (16384, 6, 20, 2, False),
+                                         (4096, 20, 300, 6, "pinned"), (16384, 6, 20, 3, "pinned"),
+                                         (1024, 40, 700, 0, "pinned")])
 def test_packed_inputs_equal_fp32(N, L, B, t, dev):
-    """snicit_infer_packed (binary rows as a bitmap, unpacked on the device) == snicit_infer on the
-    equivalent fp32 rows, bit for bit, and == the oracle's categories."""
+    """snicit_infer_packed (binary rows as a bitmap: expanded inside the row-resident kernel, or
+    unpacked by a kernel when that path does not apply, e.g. t = 0) == snicit_infer on the equivalent
+    fp32 rows, bit for bit, and == the oracle's categories.  Bits from device memory, pageable host
+    memory (staged copy) and pinned host memory (read by the kernel over PCIe, zero-copy)."""
     from paper_conf_icpp_jiangh0h23_b200 import pack_rows
     net = sdgc.gen_network(N, L, "radix")
     Y0 = sdgc.gen_inputs(N, B)
@@ -126,7 +130,13 @@ def test_packed_inputs_equal_fp32(N, L, B, t, dev):
     with SnicitNetwork.from_network(net) as g:
         g.set_stream(torch.cuda.current_stream())
         out = torch.empty((B, N), dtype=torch.float32, device="cuda")
-        g.infer_packed(torch.from_numpy(bits.view(np.int32)).cuda() if dev else bits, t=t, s=32, y_out=out)
+        if dev == "pinned":
+            src = torch.from_numpy(bits.view(np.int32)).pin_memory().numpy()
+        elif dev:
+            src = torch.from_numpy(bits.view(np.int32)).cuda()
+        else:
+            src = bits
+        g.infer_packed(src, t=t, s=32, y_out=out)
         cp = g.categories()
         Yp = out.cpu().numpy()
     assert np.array_equal(Yp, Y) and np.array_equal(cp, cats)
