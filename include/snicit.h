@@ -30,7 +30,7 @@
 extern "C" {
 #endif
 
-#define SNICIT_ABI_VERSION 2
+#define SNICIT_ABI_VERSION 3
 
 typedef struct snicit_network snicit_network; /* opaque: owns device copies of W, b + workspace */
 
@@ -96,6 +96,11 @@ typedef struct {
                                with 32 taps, uniform weight and uniform bias, and N/32 is one of
                                32..512 (N = 1024..16384); otherwise the per-layer kernels run.
                                Results are bit-identical in every mode (tested). */
+    int32_t pre_const;      /* per-layer pre-convergence path (pre_fused = 0 or not applicable): 1 = a row
+                               whose outputs are all equal leaves the active list and is carried by one
+                               scalar fma chain per layer, written once at t (R26, exact; column-streaming
+                               and segmented layer kernels, every layer < t circulant with uniform weight
+                               and bias); 0 = every live row through every layer */
 } snicit_options;
 
 /* Per-run statistics of the last snicit_infer (times in ms, valid when options.timing). */
@@ -120,7 +125,7 @@ typedef struct {
 
 /* Fill *opt with the paper's SDGC defaults (n = 16, eta = eps = 0.03, prune_eps = 0,
  * drop_dead_rows = 1, kernel = AUTO, timing = 0, ne_interval = 64, post_mode = 0, post_cluster = 1, post_const = 1,
- * pre_fused = 1). */
+ * pre_fused = 1, pre_const = 1). */
 void snicit_default_options(snicit_options* opt);
 
 /* Load a network (one-time; untimed in the benchmark).  All pointers are HOST pointers and

@@ -74,7 +74,53 @@ __global__ void __launch_bounds__(kColThreads, 2) layer_circ_col_kernel(LayerArg
         if (lane < nbuf) a.app_list[p0 + lane] = abuf;
         nbuf = 0;
     };
-    auto flag = [&](int pos, size_t base, float mx) {
+    // constant-row mode (a.cmin, R26): rows whose outputs are all equal leave the list for the
+    // constant list (row, value, layer); the warps of a row combine (min, max) at cmin/cmax[pos]
+    auto push_const = [&](int row, float v) {
+        const int p = atomicAdd(a.ccount, 1);
+        a.clist[p] = row;
+        a.cval[p] = v;
+        a.clayer[p] = a.layer;
+    };
+    auto flag = [&](int pos, size_t base, float mx, float mn) {
+        if (a.cmin) {
+#pragma unroll
+            for (int d = 16; d; d >>= 1) {
+                mx = fmaxf(mx, __shfl_xor_sync(0xffffffffu, mx, d));
+                mn = fminf(mn, __shfl_xor_sync(0xffffffffu, mn, d));
+            }
+            int app = 0;
+            if (lane == 0) {
+                unsigned umn = __float_as_uint(mn + 0.0f), umx = __float_as_uint(mx + 0.0f);  // -0 -> +0
+                bool last = true;
+                if (G > 1) {
+                    atomicMin(a.cmin + pos, umn);
+                    atomicMax(a.cmax + pos, umx);
+                    __threadfence();
+                    last = (atomicAdd(a.row_ctr + pos, 1) & 0xffff) == G - 1;
+                    if (last) {
+                        __threadfence();
+                        umn = atomicExch(a.cmin + pos, 0xffffffffu);
+                        umx = atomicExch(a.cmax + pos, 0u);
+                        a.row_ctr[pos] = 0;
+                    }
+                }
+                if (last) {
+                    const int row = (int)(base / (size_t)N);
+                    if (umn == umx) {
+                        const float v = __uint_as_float(umn);
+                        if (!(v == 0.0f && a.dead_drop)) push_const(row, v);
+                    } else {
+                        app = 1;
+                    }
+                }
+            }
+            if (__shfl_sync(0xffffffffu, app, 0)) {
+                if (lane == nbuf) abuf = (int)(base / (size_t)N);
+                if (++nbuf == 32) flush();
+            }
+            return;
+        }
         const bool nz = __any_sync(0xffffffffu, mx != 0.0f);
         if (a.app_list) {
             int app = 0;
@@ -98,12 +144,13 @@ __global__ void __launch_bounds__(kColThreads, 2) layer_circ_col_kernel(LayerArg
             if (a.flag_row) a.flag_row[base / (size_t)N] = 1;
         }
     };
-    // output epilogue: Eq. 1 bias + sigma (Table 2), store, running max for the row flag
-    auto emit = [&](float acc, float* dst, const float* bsrc, float& mx) {
+    // output epilogue: Eq. 1 bias + sigma (Table 2), store, running max / min for the row flags
+    auto emit = [&](float acc, float* dst, const float* bsrc, float& mx, float& mn) {
         const float bq = UBIAS ? b0 : __ldg(bsrc);
         const float v = sigma(acc + bq, ymax);
         *dst = v;
         mx = fmaxf(mx, v);
+        mn = fminf(mn, v);
     };
 
     if constexpr (Q32) {
@@ -116,15 +163,15 @@ __global__ void __launch_bounds__(kColThreads, 2) layer_circ_col_kernel(LayerArg
         auto compute = [&](const float (&R)[32], size_t base, int c, int pos) {
             float* dst = a.yout + base;
             const float* bsrc = a.bias + c;
-            float mx = 0.0f;
+            float mx = 0.0f, mn = ymax;
 #pragma unroll
             for (int m = 0; m < 32; ++m) {
                 float acc = 0.0f;
 #pragma unroll
                 for (int n = 0; n < kColK; ++n) acc = fmaf(R[(m + n) & 31], UNIF ? w0 : cw.w[n], acc);
-                emit(acc, dst + m * nu, bsrc + m * nu, mx);
+                emit(acc, dst + m * nu, bsrc + m * nu, mx, mn);
             }
-            flag(pos, base, mx);
+            flag(pos, base, mx, mn);
         };
         float RA[32], RB[32];
         unsigned u = warp0;
@@ -158,14 +205,14 @@ __global__ void __launch_bounds__(kColThreads, 2) layer_circ_col_kernel(LayerArg
         // input a0 + 64 + m.  One loop body (two chunks) serves every step, tail included: the code
         // stays small enough for the instruction cache (fully unrolled tails thrashed it).
         float R[64];
-        auto chunk = [&](auto sb_tag, const float* ld, int nload, float* st, const float* bs, float& mx) {
+        auto chunk = [&](auto sb_tag, const float* ld, int nload, float* st, const float* bs, float& mx, float& mn) {
             constexpr int SB = decltype(sb_tag)::value;
 #pragma unroll
             for (int m = 0; m < 32; ++m) {
                 float acc = 0.0f;
 #pragma unroll
                 for (int n = 0; n < kColK; ++n) acc = fmaf(R[(SB + m + n) & 63], UNIF ? w0 : cw.w[n], acc);
-                emit(acc, st + m * nu, bs + m * nu, mx);
+                emit(acc, st + m * nu, bs + m * nu, mx, mn);
                 if (m < nload) R[SB + m] = ld[m * nu];
             }
         };
@@ -183,16 +230,16 @@ __global__ void __launch_bounds__(kColThreads, 2) layer_circ_col_kernel(LayerArg
             const float* bsrc = a.bias + c;
 #pragma unroll
             for (int i = 0; i < 64; ++i) R[i] = src[i * nu];  // inputs 0..63 (Q >= 64)
-            float mx = 0.0f;
+            float mx = 0.0f, mn = ymax;
             for (int a0 = 0; a0 < Q; a0 += 64) {
                 const size_t o0 = (size_t)a0 * nu;
-                chunk(I0(), src + blk(a0 + 64), nld(a0 + 64), dst + o0, bsrc + o0, mx);
+                chunk(I0(), src + blk(a0 + 64), nld(a0 + 64), dst + o0, bsrc + o0, mx, mn);
                 if (a0 + 32 < Q) {
                     const size_t o1 = o0 + 32 * (size_t)nu;
-                    chunk(I32(), src + blk(a0 + 96), nld(a0 + 96), dst + o1, bsrc + o1, mx);
+                    chunk(I32(), src + blk(a0 + 96), nld(a0 + 96), dst + o1, bsrc + o1, mx, mn);
                 }
             }
-            flag(pos, base, mx);
+            flag(pos, base, mx, mn);
         }
     }
     if (a.app_list) flush();

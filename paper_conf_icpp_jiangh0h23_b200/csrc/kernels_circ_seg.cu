@@ -108,6 +108,8 @@ __global__ void __launch_bounds__(kSegThreads + 32, 2) layer_circ_seg_kernel(Lay
     int* s_row = reinterpret_cast<int*>(bars + 2 * S);  // [S]
     int* s_slot = s_row + S;
     int* s_flag = s_slot + S;
+    unsigned* s_cmin = reinterpret_cast<unsigned*>(s_flag + S);  // [S] constant-row mode: min / max bits
+    unsigned* s_cmax = s_cmin + S;
     constexpr int kConsumerWarps = kSegThreads / 32;
 
     const int count = *a.count;
@@ -192,6 +194,8 @@ __global__ void __launch_bounds__(kSegThreads + 32, 2) layer_circ_seg_kernel(Lay
             if (lane == 0) {
                 s_row[b] = row;
                 s_flag[b] = 0;
+                s_cmin[b] = 0xffffffffu;
+                s_cmax[b] = 0u;
                 if constexpr (MODE == MODE_RESIDUAL) s_slot[b] = a.cslot[row];
                 mbar_arrive_expect_tx(&in_full[b], win_bytes(na) + (PAIR ? win_bytes(nb) : 0u));
             }
@@ -214,6 +218,10 @@ __global__ void __launch_bounds__(kSegThreads + 32, 2) layer_circ_seg_kernel(Lay
             if (lane == 0 && s_flag[b]) {
                 if (a.flag_pos) a.flag_pos[pos] = 1;
                 if (a.flag_row) a.flag_row[row] = 1;
+            }
+            if (lane == 0 && a.cmin) {  // constant-row mode: this tile's (min, max) into the row's
+                atomicMin(a.cmin + pos, s_cmin[b]);
+                atomicMax(a.cmax + pos, s_cmax[b]);
             }
             bulk_commit();
             bulk_wait_read0();  // this lane's stores have read the stage
@@ -390,7 +398,7 @@ __global__ void __launch_bounds__(kSegThreads + 32, 2) layer_circ_seg_kernel(Lay
             }
         }
         asm volatile("bar.sync 2, %0;" ::"n"(kSegThreads) : "memory");  // all stage reads done
-        float mx = 0.0f;
+        float mx = 0.0f, mn = a.ymax;
         if (PAIR && g.cls == 0) {
             // nu == 1, two windows: unguarded stores (outputs past a window's segment land in the
             // window's halo, an absent second window's buffer is never stored); max of the valid ones
@@ -404,11 +412,21 @@ __global__ void __launch_bounds__(kSegThreads + 32, 2) layer_circ_seg_kernel(Lay
                 if (nv0 == M && nv1 == M) {
 #pragma unroll
                     for (int m = 0; m < M; ++m) mx = fmaxf(mx, fmaxf(v0[m], v1[PAIR ? m : 0]));
+                    if (a.cmin) {
+#pragma unroll
+                        for (int m = 0; m < M; ++m) mn = fminf(mn, fminf(v0[m], v1[PAIR ? m : 0]));
+                    }
                 } else {
 #pragma unroll
                     for (int m = 0; m < M; ++m) {
-                        if (m < nv0) mx = fmaxf(mx, fabsf(v0[m]));
-                        if (m < nv1) mx = fmaxf(mx, fabsf(v1[PAIR ? m : 0]));
+                        if (m < nv0) {
+                            mx = fmaxf(mx, fabsf(v0[m]));
+                            mn = fminf(mn, v0[m]);
+                        }
+                        if (m < nv1) {
+                            mx = fmaxf(mx, fabsf(v1[PAIR ? m : 0]));
+                            mn = fminf(mn, v1[PAIR ? m : 0]);
+                        }
                     }
                 }
             }
@@ -418,17 +436,30 @@ __global__ void __launch_bounds__(kSegThreads + 32, 2) layer_circ_seg_kernel(Lay
                 if (m < nv0) {
                     stA[ob + m * os] = v0[m];
                     mx = fmaxf(mx, fabsf(v0[m]));
+                    mn = fminf(mn, v0[m]);
                 }
                 if constexpr (PAIR) {
                     if (m < nv1) {
                         stB[ob + m * os] = v1[m];
                         mx = fmaxf(mx, fabsf(v1[m]));
+                        mn = fminf(mn, v1[m]);
                     }
                 }
             }
         }
         const unsigned any = __ballot_sync(0xffffffffu, mx != 0.0f);
         if (lane == 0 && any) s_flag[b] = 1;
+        if (MODE == MODE_PLAIN && a.cmin) {  // constant-row mode: the tile's output range (bits, -0 -> +0)
+#pragma unroll
+            for (int d = 16; d; d >>= 1) {
+                mx = fmaxf(mx, __shfl_xor_sync(0xffffffffu, mx, d));
+                mn = fminf(mn, __shfl_xor_sync(0xffffffffu, mn, d));
+            }
+            if (lane == 0) {
+                atomicMin(&s_cmin[b], __float_as_uint(mn + 0.0f));
+                atomicMax(&s_cmax[b], __float_as_uint(mx + 0.0f));
+            }
+        }
         fence_proxy_async_smem();
         __syncwarp();
         if (lane == 0) mbar_arrive(&out_full[b]);
@@ -441,7 +472,7 @@ static cudaError_t launch_seg_t(const LayerArgs& a, int max_rows, int num_sms, c
     const size_t tstage = (size_t)(PAIR ? 2 : 1) * g.sw * 4;
     int S = kSegMaxStages;
     while (S > 2 && (size_t)S * tstage + 64 * S > 110 * 1024) --S;
-    const size_t smem = (size_t)S * tstage + 2 * S * sizeof(uint64_t) + 3 * S * sizeof(int);
+    const size_t smem = (size_t)S * tstage + 2 * S * sizeof(uint64_t) + 5 * S * sizeof(int);
     auto kern = layer_circ_seg_kernel<MODE, UNIF, UBIAS, PAIR>;
     int per_sm = 1;
     cudaError_t e = blocks_per_sm((const void*)kern, kSegThreads + 32, smem, &per_sm);

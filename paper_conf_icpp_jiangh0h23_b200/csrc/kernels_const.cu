@@ -1,0 +1,118 @@
+// kernels_const.cu -- constant rows in the per-layer pre-convergence path (reading R26), sm_100a.
+//
+// A circulant layer with uniform weight and bias maps a row whose elements are all equal to v to the
+// constant row sigma(chain(v) + b0) (every output evaluates the same stored-order fma chain on the
+// same values, R12).  In constant-row mode the column-streaming and segmented layer kernels report
+// each row's output range (min, max); a row with min == max leaves the active list for a constant
+// list (row, value, layer), so later layers neither read nor write it.  At t, const_finish carries
+// each constant row through the remaining layers with one scalar chain per layer and writes it once.
+// Exact: results are bit-identical to the full evaluation (tested).
+#include <cuda_runtime.h>
+
+#include "snicit_internal.cuh"
+
+namespace snicit {
+
+// After a segmented layer: per list position, the row's (min, max) output bits (restored to the
+// initial 0xffffffff / 0) decide constant -> constant list (or dead), else -> next active list
+// (unordered, R24; warp-aggregated appends).
+__global__ void const_split_kernel(const int* list_in, const int* count_in, unsigned* cmin, unsigned* cmax,
+                                   int* list_out, int* count_out, int* clist, float* cval, int* clayer, int* ccount,
+                                   int layer, int dead_drop) {
+    const int n = *count_in;
+    const int lane = threadIdx.x & 31;
+    for (int i0 = blockIdx.x * blockDim.x; i0 < n; i0 += gridDim.x * blockDim.x) {
+        const int i = i0 + threadIdx.x;
+        bool keep = false, cst = false;
+        int row = 0;
+        float v = 0.0f;
+        if (i < n) {
+            row = list_in[i];
+            const unsigned umn = cmin[i], umx = cmax[i];
+            cmin[i] = 0xffffffffu;
+            cmax[i] = 0u;
+            if (umn == umx) {
+                v = __uint_as_float(umn);
+                cst = !(v == 0.0f && dead_drop);
+            } else {
+                keep = true;
+            }
+        }
+        const unsigned mk = __ballot_sync(0xffffffffu, keep);
+        int base = 0;
+        if (lane == 0 && mk) base = atomicAdd(count_out, __popc(mk));
+        base = __shfl_sync(0xffffffffu, base, 0);
+        if (keep) list_out[base + __popc(mk & ((1u << lane) - 1u))] = row;
+        if (cst) {
+            const int p = atomicAdd(ccount, 1);
+            clist[p] = row;
+            cval[p] = v;
+            clayer[p] = layer;
+        }
+    }
+}
+
+cudaError_t launch_const_split(const int* list_in, const int* count_in, unsigned* cmin, unsigned* cmax, int* list_out,
+                               int* count_out, int* clist, float* cval, int* clayer, int* ccount, int layer,
+                               int dead_drop, int max_rows, cudaStream_t st) {
+    int grid = max_rows > 0 ? (max_rows + 255) / 256 : 1;
+    if (grid > 2048) grid = 2048;
+    const_split_kernel<<<grid, 256, 0, st>>>(list_in, count_in, cmin, cmax, list_out, count_out, clist, cval, clayer,
+                                             ccount, layer, dead_drop);
+    return cudaGetLastError();
+}
+
+// At t: each constant row (value v after layer clayer) through layers clayer + 1 .. t - 1 by one scalar
+// chain per layer (chain(+-0) = +0; chain(YMAX) precomputed on the host, ymax_fixed); dead rows (R23)
+// vanish, the others are written (N values) and appended to the live list.
+__global__ void __launch_bounds__(256) const_finish_kernel(const int* clist, const float* cval, const int* clayer,
+                                                           const int* ccount, const PreFusedLayer* layers, int t,
+                                                           float ymax, int drop, int N, float* y, int* live,
+                                                           int* live_count) {
+    __shared__ float s_v;
+    __shared__ int s_alive;
+    const int n = *ccount;
+    for (int e = blockIdx.x; e < n; e += gridDim.x) {
+        if (threadIdx.x == 0) {
+            float v = cval[e];
+            bool alive = true;
+            for (int l = clayer[e] + 1; l < t; ++l) {
+                const PreFusedLayer d = layers[l];
+                if (v == 0.0f) {
+                    v = sigma(0.0f + d.b0, ymax);
+                } else if (!(v == ymax && d.ymax_fixed)) {
+                    float acc = 0.0f;
+#pragma unroll
+                    for (int k = 0; k < 32; ++k) acc = fmaf(v, d.w0, acc);
+                    v = sigma(acc + d.b0, ymax);
+                }
+                if (v == 0.0f && drop && d.dead_next) {
+                    alive = false;
+                    break;
+                }
+            }
+            s_v = v;
+            s_alive = alive;
+            if (alive) live[atomicAdd(live_count, 1)] = clist[e];
+        }
+        __syncthreads();
+        if (s_alive) {
+            float4* dst = reinterpret_cast<float4*>(y + (size_t)clist[e] * N);
+            const float v = s_v;
+            const float4 v4 = make_float4(v, v, v, v);
+            for (int j = threadIdx.x; j < N / 4; j += blockDim.x) dst[j] = v4;
+            for (int j = (N / 4) * 4 + threadIdx.x; j < N; j += blockDim.x) y[(size_t)clist[e] * N + j] = v;
+        }
+        __syncthreads();
+    }
+}
+
+cudaError_t launch_const_finish(const int* clist, const float* cval, const int* clayer, const int* ccount,
+                                const PreFusedLayer* layers, int t, float ymax, int drop, int N, float* y, int* live,
+                                int* live_count, int num_sms, cudaStream_t st) {
+    const_finish_kernel<<<num_sms * 8, 256, 0, st>>>(clist, cval, clayer, ccount, layers, t, ymax, drop, N, y, live,
+                                                     live_count);
+    return cudaGetLastError();
+}
+
+}  // namespace snicit

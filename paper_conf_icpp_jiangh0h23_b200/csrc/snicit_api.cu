@@ -61,7 +61,7 @@ struct DevBuf {
 // device counters (one int each)
 enum Counter {
     CNT_LIVE0 = 0, CNT_LIVE1, CNT_LIVE2, CNT_ORD, CNT_RES0, CNT_RES1, CNT_NCENT, CNT_SEFF, CNT_ALL, CNT_NCAT,
-    CNT_WORK, CNT_ALIVE, CNT_CDONE, CNT_PFWORK, CNT_PFCONST, CNT_N
+    CNT_WORK, CNT_ALIVE, CNT_CDONE, CNT_PFWORK, CNT_PFCONST, CNT_CCOUNT, CNT_N
 };
 
 }  // namespace
@@ -100,6 +100,10 @@ struct snicit_network {
     DevBuf<int> cscratch;  // per-chunk counts of the ordered compaction
     DevBuf<uint8_t> segflag;  // row flags OR-ed by segmented layers (kept zero by the clearing compaction)
     DevBuf<int> rowctr;       // per-position warp counters of the column-streaming kernel (self-clearing)
+    DevBuf<unsigned> cmin, cmax;  // constant-row mode: per position output range bits (self-restoring)
+    DevBuf<int> clist, clayer;    // constant rows of the per-layer pre phase (R26)
+    DevBuf<float> cval;
+    bool last_pre_const = false;
     DevBuf<uint32_t> bits;    // packed binary input rows (snicit_infer_packed, host bits)
     DevBuf<int> bits_ready;   // per chunk of uploaded rows: set by the copy engine after the chunk
     cudaStream_t copy_stream = nullptr;  // non-blocking upload stream (overlaps the row-resident kernel)
@@ -261,6 +265,7 @@ void snicit_default_options(snicit_options* opt) {
     opt->post_cluster = 1;
     opt->post_const = 1;
     opt->pre_fused = 1;
+    opt->pre_const = 1;
 }
 
 const char* snicit_last_error(void) { return g_last_error.c_str(); }
@@ -304,6 +309,11 @@ void snicit_free_network(snicit_network* net) {
     net->post_layers_d.release();
     net->pf_layers_d.release();
     net->pf_full.release();
+    net->cmin.release();
+    net->cmax.release();
+    net->clist.release();
+    net->clayer.release();
+    net->cval.release();
     net->a_all.release();
     delete net;
 }
@@ -650,6 +660,17 @@ static cudaError_t ensure_workspace(snicit_network* net, int64_t R, int s, int n
         if ((e = net->segflag.ensure(rows)) != cudaSuccess) return e;
         if ((e = cudaMemset(net->segflag.p, 0, rows)) != cudaSuccess) return e;
     }
+    if (net->cmin.n < rows) {
+        if ((e = net->cmin.ensure(rows)) != cudaSuccess) return e;
+        if ((e = cudaMemset(net->cmin.p, 0xff, rows * sizeof(unsigned))) != cudaSuccess) return e;
+    }
+    if (net->cmax.n < rows) {
+        if ((e = net->cmax.ensure(rows)) != cudaSuccess) return e;
+        if ((e = cudaMemset(net->cmax.p, 0, rows * sizeof(unsigned))) != cudaSuccess) return e;
+    }
+    for (auto* b : {&net->clist, &net->clayer})
+        if ((e = b->ensure(rows)) != cudaSuccess) return e;
+    if ((e = net->cval.ensure(rows)) != cudaSuccess) return e;
     if (net->rowctr.n < rows) {
         if ((e = net->rowctr.ensure(rows)) != cudaSuccess) return e;
         if ((e = cudaMemset(net->rowctr.p, 0, rows * sizeof(int))) != cudaSuccess) return e;
@@ -717,6 +738,7 @@ static snicit_status infer_core(snicit_network* net, const float* y0, int64_t ba
     if (opt.kernel < 0 || opt.kernel > SNICIT_KERNEL_CIRC_SMEM) return fail(SNICIT_E_INVALID_ARG, "bad kernel option");
     if (opt.post_mode < 0 || opt.post_mode > 1) return fail(SNICIT_E_INVALID_ARG, "bad post_mode");
     if (opt.pre_fused < 0 || opt.pre_fused > 2) return fail(SNICIT_E_INVALID_ARG, "bad pre_fused");
+    if (opt.pre_const < 0 || opt.pre_const > 1) return fail(SNICIT_E_INVALID_ARG, "bad pre_const");
     if (opt.kernel == SNICIT_KERNEL_ELL && !net->has_ell)
         return fail(SNICIT_E_UNSUPPORTED, "network loaded in compact circulant form has no ELL copy");
     const int N = net->N, L = net->L;
@@ -833,11 +855,20 @@ static snicit_status infer_core(snicit_network* net, const float* y0, int64_t ba
             ci = (ci + 1) % 3;
         }
     }
+    // constant-row mode of the per-layer path (R26, kernels_const.cu): every layer < t circulant with
+    // uniform weight and bias and run by the column-streaming or segmented kernel
+    bool pcst = !pf && opt.pre_const != 0 && tt > 0 && R > 0 && opt.kernel == SNICIT_KERNEL_AUTO;
+    for (int l = 0; l < tt && pcst; ++l)
+        pcst = net->pf_elig[l] != 0 && (use_col(net, l, opt.kernel) || use_seg(net, l, opt.kernel));
+    net->last_pre_const = pcst;
+    if (pcst) CUDA_TRY(cudaMemsetAsync(cnt + CNT_CCOUNT, 0, sizeof(int), st));
     for (int l = 0; l < tt && !pf; ++l) {
         // exact dead-row compaction (R23) fused into the layer: rows with a non-zero output are
         // appended (unordered) to the other list; the append counter of the NEXT dropping layer is
-        // zeroed by this one (rotating counters), so no extra launch is needed
-        const bool drop_now = drop && net->dead_ok[l + 1];
+        // zeroed by this one (rotating counters), so no extra launch is needed.  Constant-row mode:
+        // the list changes at every layer (constant rows leave it)
+        const bool dead_now = drop && net->dead_ok[l + 1];
+        const bool drop_now = dead_now || pcst;
         if (prof) {
             CUDA_TRY(cudaMemcpyAsync(net->hist.p + l, cnt + live_ctr[ci], sizeof(int), cudaMemcpyDeviceToDevice, st));
             CUDA_TRY(cudaEventRecord(net->lev[2 * l], st));
@@ -855,11 +886,27 @@ static snicit_status infer_core(snicit_network* net, const float* y0, int64_t ba
             a.app_count = cnt + live_ctr[(ci + 1) % 3];
             a.zero_count = cnt + live_ctr[(ci + 2) % 3];
         }
-        if (drop_now && seg) a.flag_pos = net->segflag.p;
+        if (drop_now && seg && !pcst) a.flag_pos = net->segflag.p;
+        if (pcst) {
+            a.cmin = net->cmin.p;
+            a.cmax = net->cmax.p;
+            a.clist = net->clist.p;
+            a.cval = net->cval.p;
+            a.clayer = net->clayer.p;
+            a.ccount = cnt + CNT_CCOUNT;
+            a.layer = l;
+            a.dead_drop = dead_now ? 1 : 0;
+        }
         CUDA_TRY(run_layer(net, l, opt.kernel, MODE_PLAIN, a, R));
         if (prof) CUDA_TRY(cudaEventRecord(net->lev[2 * l + 1], st));
         ++launches;
-        if (drop_now && seg) {
+        if (pcst && seg) {
+            CUDA_TRY(launch_const_split(lists[li], cnt + live_ctr[ci], net->cmin.p, net->cmax.p, lists[li ^ 1],
+                                        cnt + live_ctr[(ci + 1) % 3], net->clist.p, net->cval.p, net->clayer.p,
+                                        cnt + CNT_CCOUNT, l, dead_now ? 1 : 0, R, st));
+            CUDA_TRY(cudaMemsetAsync(cnt + live_ctr[(ci + 2) % 3], 0, sizeof(int), st));
+            launches += 1;
+        } else if (drop_now && seg) {
             CUDA_TRY(launch_compact(lists[li], cnt + live_ctr[ci], net->segflag.p, lists[li ^ 1],
                                     cnt + live_ctr[(ci + 1) % 3], R, scratch, st, 1));
             CUDA_TRY(cudaMemsetAsync(cnt + live_ctr[(ci + 2) % 3], 0, sizeof(int), st));
@@ -873,6 +920,12 @@ static snicit_status infer_core(snicit_network* net, const float* y0, int64_t ba
             li ^= 1;
             ci = (ci + 1) % 3;
         }
+    }
+    if (pcst) {  // constant rows through the remaining layers (scalar chains), written once, relisted
+        CUDA_TRY(launch_const_finish(net->clist.p, net->cval.p, net->clayer.p, cnt + CNT_CCOUNT, net->pf_layers_d.p, tt,
+                                     net->ymax, drop ? 1 : 0, N, bufs[nxt_i ^ 1], lists[li], cnt + live_ctr[ci],
+                                     net->num_sms, st));
+        ++launches;
     }
     int* list_cur = lists[li];
     int* cnt_cur = cnt + live_ctr[ci];
@@ -1252,6 +1305,10 @@ snicit_status snicit_stats(snicit_network* net, snicit_stats_t* out) {
     }
     net->stats.pre_const_rows = 0;
     net->stats.pre_full_rows = 0;
+    if (net->last_pre_const) {
+        CUDA_TRY(read_counter(net, CNT_CCOUNT, &v));
+        net->stats.pre_const_rows = v;
+    }
     if (net->last_pre_fused) {
         CUDA_TRY(read_counter(net, CNT_PFCONST, &v));
         net->stats.pre_const_rows = v;

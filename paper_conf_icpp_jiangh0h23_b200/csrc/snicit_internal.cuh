@@ -137,6 +137,15 @@ struct LayerArgs {
     int nu;
     const float* wtab;      // K per-n weights (device), nullable when uniform
     const float* wtab_host; // the same K weights in host memory (kernels taking them as parameters)
+    // constant-row mode of the pre-convergence per-layer path (R26; column and segmented kernels)
+    unsigned* cmin;         // nullable: per list position, min / max output bits (init 0xffffffff / 0,
+    unsigned* cmax;         //   restored by the consumer)
+    int* clist;             // rows that became constant: row id, value, layer (append at *ccount)
+    float* cval;
+    int* clayer;
+    int* ccount;
+    int layer;              // index of this layer
+    int dead_drop;          // an all-zero row after this layer is dead (drop && dead_ok[l + 1])
 };
 
 struct LayerPlan {
@@ -273,6 +282,14 @@ bool pre_fused_str_halo(int N);  // STR layers need H >= 31*nu
 constexpr int kPfMaxLayers = 2000;  // t limit of the row-resident kernel (descriptors in parameter space)
 // layers: host descriptors of layers 0..t-1
 cudaError_t launch_pre_fused(const PreFusedArgs& a, const PreFusedLayer* layers, int num_sms, cudaStream_t st);
+
+// kernels_const.cu: constant rows in the per-layer pre-convergence path (R26)
+cudaError_t launch_const_split(const int* list_in, const int* count_in, unsigned* cmin, unsigned* cmax, int* list_out,
+                               int* count_out, int* clist, float* cval, int* clayer, int* ccount, int layer,
+                               int dead_drop, int max_rows, cudaStream_t st);
+cudaError_t launch_const_finish(const int* clist, const float* cval, const int* clayer, const int* ccount,
+                                const PreFusedLayer* layers, int t, float ymax, int drop, int N, float* y, int* live,
+                                int* live_count, int num_sms, cudaStream_t st);
 
 // kernels_convert.cu
 cudaError_t launch_iota(int* out, int n, int* count_out, cudaStream_t st);
