@@ -82,41 +82,29 @@ __global__ void __launch_bounds__(kColThreads, 2) layer_circ_col_kernel(LayerArg
         a.cval[p] = v;
         a.clayer[p] = a.layer;
     };
-    auto flag = [&](int pos, size_t base, float mx, float mn) {
-        if (a.cmin) {
+    // Constant-row mode walks the units row-major per warp (all G column groups of a row in one warp,
+    // see nextu), so a row's output range is combined in registers and decided by that warp alone.
+    const bool rowmajor = a.cmin != nullptr;
+    float rmx = 0.0f, rmn = ymax;  // running range of the current row (constant-row mode)
+    auto flag = [&](int pos, size_t base, float mx, float mn, bool last) {
+        if (rowmajor) {
+            rmx = fmaxf(rmx, mx);
+            rmn = fminf(rmn, mn);
+            if (!last) return;
 #pragma unroll
             for (int d = 16; d; d >>= 1) {
-                mx = fmaxf(mx, __shfl_xor_sync(0xffffffffu, mx, d));
-                mn = fminf(mn, __shfl_xor_sync(0xffffffffu, mn, d));
+                rmx = fmaxf(rmx, __shfl_xor_sync(0xffffffffu, rmx, d));
+                rmn = fminf(rmn, __shfl_xor_sync(0xffffffffu, rmn, d));
             }
-            int app = 0;
-            if (lane == 0) {
-                unsigned umn = __float_as_uint(mn + 0.0f), umx = __float_as_uint(mx + 0.0f);  // -0 -> +0
-                bool last = true;
-                if (G > 1) {
-                    atomicMin(a.cmin + pos, umn);
-                    atomicMax(a.cmax + pos, umx);
-                    __threadfence();
-                    last = (atomicAdd(a.row_ctr + pos, 1) & 0xffff) == G - 1;
-                    if (last) {
-                        __threadfence();
-                        umn = atomicExch(a.cmin + pos, 0xffffffffu);
-                        umx = atomicExch(a.cmax + pos, 0u);
-                        a.row_ctr[pos] = 0;
-                    }
-                }
-                if (last) {
-                    const int row = (int)(base / (size_t)N);
-                    if (umn == umx) {
-                        const float v = __uint_as_float(umn);
-                        if (!(v == 0.0f && a.dead_drop)) push_const(row, v);
-                    } else {
-                        app = 1;
-                    }
-                }
-            }
-            if (__shfl_sync(0xffffffffu, app, 0)) {
-                if (lane == nbuf) abuf = (int)(base / (size_t)N);
+            const unsigned umn = __float_as_uint(rmn + 0.0f), umx = __float_as_uint(rmx + 0.0f);  // -0 -> +0
+            rmx = 0.0f;
+            rmn = ymax;
+            const int row = (int)(base / (size_t)N);
+            if (umn == umx) {
+                const float v = __uint_as_float(umn);
+                if (lane == 0 && !(v == 0.0f && a.dead_drop)) push_const(row, v);
+            } else {
+                if (lane == nbuf) abuf = row;
                 if (++nbuf == 32) flush();
             }
             return;
@@ -153,6 +141,15 @@ __global__ void __launch_bounds__(kColThreads, 2) layer_circ_col_kernel(LayerArg
         mn = fminf(mn, v);
     };
 
+    // unit order: round-robin over warps, or (constant-row mode) row-major: warp w takes rows w,
+    // w + nwarps, ... and within a row its G column groups in order
+    const unsigned u_first = rowmajor ? warp0 * G : warp0;
+    auto nextu = [&](unsigned u) -> unsigned {
+        if (!rowmajor) return u + nwarps;
+        return (u % G == G - 1) ? (u / G + nwarps) * G : u + 1;
+    };
+    auto is_last = [&](unsigned u) -> bool { return u % G == G - 1; };
+
     if constexpr (Q32) {
         // ---------------------------------------------------------------- Q == 32: whole column
         auto load = [&](float (&R)[32], size_t base) {
@@ -160,7 +157,7 @@ __global__ void __launch_bounds__(kColThreads, 2) layer_circ_col_kernel(LayerArg
 #pragma unroll
             for (int i = 0; i < 32; ++i) R[i] = src[i * nu];
         };
-        auto compute = [&](const float (&R)[32], size_t base, int c, int pos) {
+        auto compute = [&](const float (&R)[32], size_t base, int c, int pos, bool last) {
             float* dst = a.yout + base;
             const float* bsrc = a.bias + c;
             float mx = 0.0f, mn = ymax;
@@ -171,10 +168,10 @@ __global__ void __launch_bounds__(kColThreads, 2) layer_circ_col_kernel(LayerArg
                 for (int n = 0; n < kColK; ++n) acc = fmaf(R[(m + n) & 31], UNIF ? w0 : cw.w[n], acc);
                 emit(acc, dst + m * nu, bsrc + m * nu, mx, mn);
             }
-            flag(pos, base, mx, mn);
+            flag(pos, base, mx, mn, last);
         };
         float RA[32], RB[32];
-        unsigned u = warp0;
+        unsigned u = u_first;
         int posA = 0, cA = 0, posB = 0, cB = 0;
         size_t bA = 0, bB = 0;
         if (u < units) {
@@ -182,19 +179,19 @@ __global__ void __launch_bounds__(kColThreads, 2) layer_circ_col_kernel(LayerArg
             load(RA, bA);
         }
         while (u < units) {
-            const unsigned u2 = u + nwarps;
+            const unsigned u2 = nextu(u);
             if (u2 < units) {
                 bB = unit_base(u2, posB, cB);
                 load(RB, bB);
             }
-            compute(RA, bA, cA, posA);
+            compute(RA, bA, cA, posA, is_last(u));
             if (u2 >= units) break;
-            const unsigned u3 = u2 + nwarps;
+            const unsigned u3 = nextu(u2);
             if (u3 < units) {
                 bA = unit_base(u3, posA, cA);
                 load(RA, bA);
             }
-            compute(RB, bB, cB, posB);
+            compute(RB, bB, cB, posB, is_last(u2));
             u = u3;
         }
     } else {
@@ -222,7 +219,7 @@ __global__ void __launch_bounds__(kColThreads, 2) layer_circ_col_kernel(LayerArg
         auto nld = [&](int x) -> int { return min(32, max(0, Q + 31 - x)); };
         using I0 = std::integral_constant<int, 0>;
         using I32 = std::integral_constant<int, 32>;
-        for (unsigned u = warp0; u < units; u += nwarps) {
+        for (unsigned u = u_first; u < units; u = nextu(u)) {
             int pos, c;
             const size_t base = unit_base(u, pos, c);
             const float* src = a.yin + base;
@@ -239,7 +236,7 @@ __global__ void __launch_bounds__(kColThreads, 2) layer_circ_col_kernel(LayerArg
                     chunk(I32(), src + blk(a0 + 96), nld(a0 + 96), dst + o1, bsrc + o1, mx, mn);
                 }
             }
-            flag(pos, base, mx, mn);
+            flag(pos, base, mx, mn, is_last(u));
         }
     }
     if (a.app_list) flush();
@@ -257,6 +254,8 @@ static cudaError_t launch_col_t(const LayerArgs& a, int max_rows, int num_sms, c
     const long long need = (units + kColThreads / 32 - 1) / (kColThreads / 32);
     if (grid > need) grid = need;
     if (grid < 1) grid = 1;
+    // row-major unit walk (constant-row mode) steps past the last unit by up to nwarps * G
+    if (units + grid * (kColThreads / 32) * (long long)(a.nu / 32) >= (1LL << 31)) return cudaErrorInvalidValue;
     ColW cw{};
     if (!UNIF)
         for (int n = 0; n < kColK; ++n) cw.w[n] = a.wtab_host[n];
