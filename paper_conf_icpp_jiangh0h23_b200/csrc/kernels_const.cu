@@ -68,7 +68,7 @@ cudaError_t launch_const_split(const int* list_in, const int* count_in, unsigned
 __global__ void __launch_bounds__(256) const_finish_kernel(const int* clist, const float* cval, const int* clayer,
                                                            const int* ccount, const PreFusedLayer* layers, int t,
                                                            float ymax, int drop, int N, float* y, int* live,
-                                                           int* live_count) {
+                                                           int* live_count, uint8_t* rconst, float* rval) {
     __shared__ float s_v;
     __shared__ int s_alive;
     const int n = *ccount;
@@ -93,7 +93,13 @@ __global__ void __launch_bounds__(256) const_finish_kernel(const int* clist, con
             }
             s_v = v;
             s_alive = alive;
-            if (alive) live[atomicAdd(live_count, 1)] = clist[e];
+            if (alive) {
+                live[atomicAdd(live_count, 1)] = clist[e];
+                if (rconst) {
+                    rconst[clist[e]] = 1;
+                    rval[clist[e]] = v;
+                }
+            }
         }
         __syncthreads();
         if (s_alive) {
@@ -109,9 +115,9 @@ __global__ void __launch_bounds__(256) const_finish_kernel(const int* clist, con
 
 cudaError_t launch_const_finish(const int* clist, const float* cval, const int* clayer, const int* ccount,
                                 const PreFusedLayer* layers, int t, float ymax, int drop, int N, float* y, int* live,
-                                int* live_count, int num_sms, cudaStream_t st) {
+                                int* live_count, int num_sms, cudaStream_t st, uint8_t* rconst, float* rval) {
     const_finish_kernel<<<num_sms * 8, 256, 0, st>>>(clist, cval, clayer, ccount, layers, t, ymax, drop, N, y, live,
-                                                     live_count);
+                                                     live_count, rconst, rval);
     return cudaGetLastError();
 }
 

@@ -291,7 +291,9 @@ __global__ void __launch_bounds__(kMapThreads) map_residual_kernel(const float* 
                                                                    const int* cent, const int* n_cent, int* M,
                                                                    int* cslot, uint8_t* ne_row, uint8_t* flag_pos,
                                                                    float* __restrict__ yhat,
-                                                                   float* __restrict__ cbuf) {
+                                                                   float* __restrict__ cbuf,
+                                                                   const uint8_t* __restrict__ rconst,
+                                                                   const float* __restrict__ rval) {
     __shared__ int red[kMapThreads / 32];
     __shared__ int s_best, s_slot;
     const int n = *count;
@@ -319,6 +321,24 @@ __global__ void __launch_bounds__(kMapThreads) map_residual_kernel(const float* 
             }
             __syncthreads();
             continue;
+        }
+        if (rconst && rconst[r]) {
+            // constant row (R26, flags from the pre phase): its L0 distance to a centroid that is the
+            // same constant is 0 and to any other centroid > 0, so the first such centroid is Alg. 2's
+            // argmin (strict <) -- empty residue, nothing to read or write
+            int hit = -1;
+            const float v = rval[r];
+            for (int c = 0; c < C && hit < 0; ++c)
+                if (rconst[cent[c]] && rval[cent[c]] == v) hit = c;
+            if (hit >= 0) {
+                if (threadIdx.x == 0) {
+                    M[r] = cent[hit];
+                    cslot[r] = hit;
+                    ne_row[r] = 0;
+                    flag_pos[p] = 0;
+                }
+                continue;  // uniform across the CTA: no barrier needed
+            }
         }
         int best_dist = N + 1, best = 0;  // Alg. 2 line 3 (tracked by thread 0)
         for (int c = 0; c < C; ++c) {
@@ -365,12 +385,13 @@ __global__ void __launch_bounds__(kMapThreads) map_residual_kernel(const float* 
 }
 cudaError_t launch_map_residual(const float* y, int N, const int* rows, const int* count, const int* cent,
                                 const int* n_cent, int* M, int* cslot, uint8_t* ne_row, uint8_t* flag_pos,
-                                float* yhat, float* cbuf, int max_rows, int num_sms, cudaStream_t st) {
+                                float* yhat, float* cbuf, int max_rows, int num_sms, cudaStream_t st,
+                                const uint8_t* rconst, const float* rval) {
     int grid = num_sms * 8;
     if (grid > max_rows) grid = max_rows;
     if (grid < 1) grid = 1;
     map_residual_kernel<<<grid, kMapThreads, 0, st>>>(y, N, rows, count, cent, n_cent, M, cslot, ne_row, flag_pos,
-                                                      yhat, cbuf);
+                                                      yhat, cbuf, rconst, rval);
     return cudaGetLastError();
 }
 

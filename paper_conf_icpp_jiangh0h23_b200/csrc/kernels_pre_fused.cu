@@ -359,6 +359,10 @@ __global__ void __launch_bounds__(T, PfCfg<T>::kMinBlocks) pre_fused_kernel(cons
                 const int p = atomicAdd(a.app_count, 1);
                 a.app_list[p] = row;
             }
+            if (tid == 0 && a.rconst && cst) {  // constant at t: conversion needs no read of the row
+                a.rconst[row] = 1;
+                a.rval[row] = v;
+            }
         }
         if (tid == 0) {
             if (a.full_rl) atomicAdd(a.full_rl, (unsigned long long)full);

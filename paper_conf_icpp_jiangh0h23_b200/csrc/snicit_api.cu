@@ -103,6 +103,8 @@ struct snicit_network {
     DevBuf<unsigned> cmin, cmax;  // constant-row mode: per position output range bits (self-restoring)
     DevBuf<int> clist, clayer;    // constant rows of the per-layer pre phase (R26)
     DevBuf<float> cval;
+    DevBuf<uint8_t> rconst;   // rows constant at t (R26): flag + value, set by the pre phase
+    DevBuf<float> rval;
     bool last_pre_const = false;
     DevBuf<uint32_t> bits;    // packed binary input rows (snicit_infer_packed, host bits)
     DevBuf<int> bits_ready;   // per chunk of uploaded rows: set by the copy engine after the chunk
@@ -314,6 +316,8 @@ void snicit_free_network(snicit_network* net) {
     net->clist.release();
     net->clayer.release();
     net->cval.release();
+    net->rconst.release();
+    net->rval.release();
     net->a_all.release();
     delete net;
 }
@@ -671,6 +675,8 @@ static cudaError_t ensure_workspace(snicit_network* net, int64_t R, int s, int n
     for (auto* b : {&net->clist, &net->clayer})
         if ((e = b->ensure(rows)) != cudaSuccess) return e;
     if ((e = net->cval.ensure(rows)) != cudaSuccess) return e;
+    if ((e = net->rconst.ensure(rows)) != cudaSuccess) return e;
+    if ((e = net->rval.ensure(rows)) != cudaSuccess) return e;
     if (net->rowctr.n < rows) {
         if ((e = net->rowctr.ensure(rows)) != cudaSuccess) return e;
         if ((e = cudaMemset(net->rowctr.p, 0, rows * sizeof(int))) != cudaSuccess) return e;
@@ -814,6 +820,7 @@ static snicit_status infer_core(snicit_network* net, const float* y0, int64_t ba
     if (y0_mode == 3 && !pf && R > 0) return fail(SNICIT_E_STATE, "packed rows without the row-resident kernel");
     net->last_pre_fused = pf;
     stats.pre_fused = pf ? 1 : 0;
+    if (R > 0) CUDA_TRY(cudaMemsetAsync(net->rconst.p, 0, (size_t)R, st));  // rows constant at t (R26)
     if (pf) {
         if (prof) {
             CUDA_TRY(cudaMemcpyAsync(net->hist.p, cnt + live_ctr[ci], sizeof(int), cudaMemcpyDeviceToDevice, st));
@@ -842,6 +849,8 @@ static snicit_status infer_core(snicit_network* net, const float* y0, int64_t ba
         pa.app_count = cnt + live_ctr[(ci + 1) % 3];
         pa.work = cnt + CNT_PFWORK;
         pa.full_rl = net->pf_full.p;
+        pa.rconst = net->rconst.p;
+        pa.rval = net->rval.p;
         pa.n_const = cnt + CNT_PFCONST;
         CUDA_TRY(launch_pre_fused(pa, net->pf_layers_h.data(), net->num_sms, st));
         if (prof) CUDA_TRY(cudaEventRecord(net->lev[1], st));
@@ -924,7 +933,7 @@ static snicit_status infer_core(snicit_network* net, const float* y0, int64_t ba
     if (pcst) {  // constant rows through the remaining layers (scalar chains), written once, relisted
         CUDA_TRY(launch_const_finish(net->clist.p, net->cval.p, net->clayer.p, cnt + CNT_CCOUNT, net->pf_layers_d.p, tt,
                                      net->ymax, drop ? 1 : 0, N, bufs[nxt_i ^ 1], lists[li], cnt + live_ctr[ci],
-                                     net->num_sms, st));
+                                     net->num_sms, st, net->rconst.p, net->rval.p));
         ++launches;
     }
     int* list_cur = lists[li];
@@ -968,7 +977,8 @@ static snicit_status infer_core(snicit_network* net, const float* y0, int64_t ba
         float* yhat = bufs[nxt_i];
         float* yhat_other = bufs[nxt_i ^ 1];
         CUDA_TRY(launch_map_residual(cur, N, list_cur, cnt_cur, net->cent.p, cnt + CNT_NCENT, net->M.p, net->cslot.p,
-                                     net->ne_row.p, net->flag_pos.p, yhat, net->cbuf0.p, R, net->num_sms, st));
+                                     net->ne_row.p, net->flag_pos.p, yhat, net->cbuf0.p, R, net->num_sms, st,
+                                     net->rconst.p, net->rval.p));
         int* rlist = net->res0.p;
         int* rlist_nxt = net->res1.p;
         int* rcnt = cnt + CNT_RES0;

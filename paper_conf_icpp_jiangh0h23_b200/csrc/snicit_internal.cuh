@@ -272,6 +272,8 @@ struct PreFusedArgs {
     int* app_list;     // rows alive at t, appended unordered (nullable)
     int* app_count;    //   zero on entry
     int* work;         // row scheduler, zero on entry
+    uint8_t* rconst;              // nullable: rconst[row] = 1, rval[row] = v for rows constant at t (R26)
+    float* rval;
     unsigned long long* full_rl;  // nullable: += full (non-constant) row-layer evaluations
     int* n_const;                 // nullable: += rows that became constant
 };
@@ -289,7 +291,8 @@ cudaError_t launch_const_split(const int* list_in, const int* count_in, unsigned
                                int dead_drop, int max_rows, cudaStream_t st);
 cudaError_t launch_const_finish(const int* clist, const float* cval, const int* clayer, const int* ccount,
                                 const PreFusedLayer* layers, int t, float ymax, int drop, int N, float* y, int* live,
-                                int* live_count, int num_sms, cudaStream_t st);
+                                int* live_count, int num_sms, cudaStream_t st, uint8_t* rconst = nullptr,
+                                float* rval = nullptr);
 
 // kernels_convert.cu
 cudaError_t launch_iota(int* out, int n, int* count_out, cudaStream_t st);
@@ -309,7 +312,8 @@ cudaError_t launch_prune(const double* F, const int* count, int s, int n_seg, fl
                          const int* rows, int* cent, int* n_cent, int* s_eff, int* col_idx, cudaStream_t st);
 cudaError_t launch_map_residual(const float* y, int N, const int* rows, const int* count, const int* cent,
                                 const int* n_cent, int* M, int* cslot, uint8_t* ne_row, uint8_t* flag_pos,
-                                float* yhat, float* cbuf, int max_rows, int num_sms, cudaStream_t st);
+                                float* yhat, float* cbuf, int max_rows, int num_sms, cudaStream_t st,
+                                const uint8_t* rconst = nullptr, const float* rval = nullptr);
 cudaError_t launch_recover(int N, int R, int plain, const float* yfinal, const uint8_t* live_row, const int* M,
                            const int* cslot, const uint8_t* ne_row, const float* cbuf, float* y_out,
                            uint8_t* cat, int num_sms, cudaStream_t st);
