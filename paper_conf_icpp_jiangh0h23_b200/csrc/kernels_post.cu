@@ -299,9 +299,12 @@ __global__ void __launch_bounds__(kPostThreads, 2) residual_traj_kernel(PostArgs
         __syncthreads();
         fill_halo(cur, N, h);
         __syncthreads();
-        bool alive = true;
+        bool alive = true, cst = false;
+        float vr = 0.0f;
+        const int cfrom = a.cfrom ? a.cfrom[slot] : a.L - a.t;
         PL Ld = load_pl(a.layers + a.t);
-        for (int l = a.t; l < a.L; ++l) {
+        int l = a.t;
+        for (; l < a.L; ++l) {
             const PL Lnext = load_pl(a.layers + min(l + 1, a.L - 1));
             const float* ac = a.a_all + ((size_t)(l - a.t) * a.s + slot) * N;
             const bool any = post_row_layer<MODE_RESIDUAL, 17, 16, 1>(Ld, N, dup, a.ymax, a.prune_eps, cur, nxt, ac,
@@ -310,6 +313,20 @@ __global__ void __launch_bounds__(kPostThreads, 2) residual_traj_kernel(PostArgs
                 alive = false;
                 break;
             }
+            if (a.scalar_ok && l + 1 < a.L && l + 1 - a.t >= cfrom) {
+                // the centroid row is constant from here on (its a_c rows are): if this residue row is
+                // constant too, Eq. 5 maps it to a constant row every layer -- carry it by a scalar
+                // (R25/R26 argument; bit-identical)
+                const float v0 = nxt[0];
+                bool eq = true;
+                for (int k = threadIdx.x; k < N; k += blockDim.x) eq = eq && nxt[k] == v0;
+                if (__syncthreads_and(eq)) {
+                    cst = true;
+                    vr = v0;
+                    ++l;
+                    break;
+                }
+            }
             fill_halo(nxt, N, h);
             __syncthreads();
             float* tmp = cur;
@@ -317,13 +334,62 @@ __global__ void __launch_bounds__(kPostThreads, 2) residual_traj_kernel(PostArgs
             nxt = tmp;
             Ld = Lnext;
         }
-        if (alive) unstage_row(a.yhat + (size_t)row * N, cur, N);
+        if (cst) {  // layers l .. L-1: every thread evaluates the same scalar chain
+            for (; l < a.L; ++l) {
+                const PostLayer* pl = a.layers + l;
+                const float w0 = pl->w0, b0 = pl->b0;
+                const float acv = __ldg(a.a_all + ((size_t)(l - a.t) * a.s + slot) * N);
+                float acc = 0.0f;
+#pragma unroll
+                for (int n2 = 0; n2 < kPK; ++n2) acc = fmaf(vr, w0, acc);
+                float v = sigma((acv + acc) + b0, a.ymax) - sigma(acv + b0, a.ymax);
+                if (a.prune_eps > 0.0f && fabsf(v) <= a.prune_eps) v = 0.0f;
+                vr = v;
+                if (v == 0.0f) {
+                    alive = false;
+                    break;
+                }
+            }
+            if (alive) {
+                float4* d4 = reinterpret_cast<float4*>(a.yhat + (size_t)row * N);
+                const float4 v4 = make_float4(vr, vr, vr, vr);
+                for (int k = threadIdx.x; k < (N >> 2); k += blockDim.x) d4[k] = v4;
+            }
+        } else if (alive) {
+            unstage_row(a.yhat + (size_t)row * N, cur, N);
+        }
         if (threadIdx.x == 0) {
             a.ne_row[row] = alive ? 1 : 0;
             if (alive && a.alive_count) atomicAdd(a.alive_count, 1);
         }
         __syncthreads();  // s_p and the row buffers are reused
     }
+}
+
+// cfrom[c] = first post layer index (l - t) whose centroid pre-activation row a_c is constant (then
+// every later one is: a constant input row stays constant, R25), or L - t; scans layers in order
+__global__ void __launch_bounds__(256) acconst_kernel(PostArgs a) {
+    const int c = blockIdx.x;
+    if (c >= *a.n_cent) return;
+    const int N = a.N, nl = a.L - a.t;
+    int l2 = 0;
+    if (a.cdone && a.cdone[c]) {
+        l2 = 0;  // constant at t (centroid_const_kernel)
+    } else {
+        for (; l2 < nl; ++l2) {
+            const float* row = a.a_all + ((size_t)l2 * a.s + c) * N;
+            const float v0 = __ldg(row);
+            bool eq = true;
+            for (int k = threadIdx.x; k < N; k += blockDim.x) eq = eq && __ldg(row + k) == v0;
+            if (__syncthreads_and(eq)) break;
+        }
+    }
+    if (threadIdx.x == 0) a.cfrom[c] = l2;
+}
+cudaError_t launch_acconst(const PostArgs& a, int C_max, cudaStream_t st) {
+    if (C_max <= 0) return cudaSuccess;
+    acconst_kernel<<<C_max, 256, 0, st>>>(a);
+    return cudaGetLastError();
 }
 
 // ------------------------------------------------------------------------------ cluster version

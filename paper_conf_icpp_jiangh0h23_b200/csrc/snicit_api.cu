@@ -103,6 +103,7 @@ struct snicit_network {
     DevBuf<unsigned> cmin, cmax;  // constant-row mode: per position output range bits (self-restoring)
     DevBuf<int> clist, clayer;    // constant rows of the per-layer pre phase (R26)
     DevBuf<float> cval;
+    DevBuf<int> cfrom;        // per centroid: first post layer with a constant a_c row (residual_traj)
     DevBuf<uint8_t> rconst;   // rows constant at t (R26): flag + value, set by the pre phase
     DevBuf<float> rval;
     bool last_pre_const = false;
@@ -317,6 +318,7 @@ void snicit_free_network(snicit_network* net) {
     net->clayer.release();
     net->cval.release();
     net->rconst.release();
+    net->cfrom.release();
     net->rval.release();
     net->a_all.release();
     delete net;
@@ -1085,6 +1087,15 @@ static snicit_status infer_core(snicit_network* net, const float* y0, int64_t ba
             ++launches;
             for (int l = tt; l < L; ++l) circ_layers += use_circ(net, l, opt.kernel);
             if (res_host > 0) {
+                bool sok = opt.post_const != 0 && opt.kernel == SNICIT_KERNEL_AUTO;
+                for (int l = tt; l < L && sok; ++l) sok = net->pf_elig[l] != 0;
+                if (sok) {  // constant residue rows over constant centroids leave as scalars
+                    CUDA_TRY(net->cfrom.ensure((size_t)s));
+                    pa.cfrom = net->cfrom.p;
+                    pa.scalar_ok = 1;
+                    CUDA_TRY(launch_acconst(pa, s, st));
+                    ++launches;
+                }
                 CUDA_TRY(launch_residual_traj(pa, res_host, net->num_sms, st));
                 ++launches;
             }

@@ -230,7 +230,11 @@ struct PostArgs {
     uint8_t* ne_row;     // set to the row's final ne (0 once its residue became empty)
     int* alive_count;    // += 1 per row still non-empty at L (may be NULL)
     const int* cdone;    // nullable: centroid c already carried to L by centroid_const_kernel (skip it)
+    int* cfrom;          // nullable: per centroid, first post layer (l - t) with a constant a_c row
+    int scalar_ok;       // every post layer circulant with uniform weight and bias: constant residue rows
+                         //   over constant centroids are carried by a scalar (residual_traj_kernel)
 };
+cudaError_t launch_acconst(const PostArgs& a, int C_max, cudaStream_t st);
 int post_fused_max_n();
 cudaError_t launch_centroid_traj(const PostArgs& a, int C_max, cudaStream_t st);
 // cluster (DSMEM) centroid trajectory: cls[l] = circulant stride class of layer l or -1
