@@ -404,7 +404,8 @@ __global__ void __launch_bounds__(kRecThreads) recover_kernel(int N, int R, int 
                                                               const uint8_t* live_row, const int* M,
                                                               const int* cslot, const uint8_t* ne_row,
                                                               const float* __restrict__ cbuf,
-                                                              float* __restrict__ y_out, uint8_t* cat) {
+                                                              float* __restrict__ y_out, uint8_t* cat,
+                                                              int dead_zeroed) {
     const int N4 = N >> 2;
     for (int r = blockIdx.x; r < R; r += gridDim.x) {
         int mode;  // 0 zero, 1 copy a, 2 a + c, 3 0 + c
@@ -430,6 +431,10 @@ __global__ void __launch_bounds__(kRecThreads) recover_kernel(int N, int R, int 
                 }
             }
         }
+        if (mode == 0 && dead_zeroed) {  // dead row: y_out already zeroed by the pre phase
+            if (threadIdx.x == 0) cat[r] = 0;
+            continue;  // uniform across the CTA
+        }
         int any = 0;
         float4* o4 = y_out ? reinterpret_cast<float4*>(y_out + (size_t)r * N) : nullptr;
         for (int k = threadIdx.x; k < N4; k += blockDim.x) {
@@ -454,12 +459,12 @@ __global__ void __launch_bounds__(kRecThreads) recover_kernel(int N, int R, int 
 }
 cudaError_t launch_recover(int N, int R, int plain, const float* yfinal, const uint8_t* live_row, const int* M,
                            const int* cslot, const uint8_t* ne_row, const float* cbuf, float* y_out,
-                           uint8_t* cat, int num_sms, cudaStream_t st) {
+                           uint8_t* cat, int num_sms, cudaStream_t st, int dead_zeroed) {
     if (R <= 0) return cudaSuccess;
     int grid = num_sms * 8;
     if (grid > R) grid = R;
     recover_kernel<<<grid, kRecThreads, 0, st>>>(N, R, plain, yfinal, live_row, M, cslot, ne_row, cbuf, y_out,
-                                                 cat);
+                                                 cat, dead_zeroed);
     return cudaGetLastError();
 }
 

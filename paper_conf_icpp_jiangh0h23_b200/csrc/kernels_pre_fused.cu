@@ -341,6 +341,11 @@ __global__ void __launch_bounds__(T, PfCfg<T>::kMinBlocks) pre_fused_kernel(cons
                 }
             }
         }
+        if (dead && a.ydead) {  // final activations of a dead row: zeros, written now (the SMs' HBM is idle)
+            float4* dz = reinterpret_cast<float4*>(a.ydead + (size_t)row * N);
+#pragma unroll
+            for (int i = 0; i < N / 4 / T; ++i) dz[i * T + tid] = make_float4(0.f, 0.f, 0.f, 0.f);
+        }
         if (!dead) {
             float* gout = a.yout + (size_t)row * N;
             if (cst) {

@@ -821,6 +821,7 @@ static snicit_status infer_core(snicit_network* net, const float* y0, int64_t ba
     const bool pf = pf_plan(net, tt, opt, R, &pf_H, &pf_gen);
     if (y0_mode == 3 && !pf && R > 0) return fail(SNICIT_E_STATE, "packed rows without the row-resident kernel");
     net->last_pre_fused = pf;
+    const int dead_zeroed = (pf && y_out_on_device && y_out && drop) ? 1 : 0;  // y_out rows of dead rows
     stats.pre_fused = pf ? 1 : 0;
     if (R > 0) CUDA_TRY(cudaMemsetAsync(net->rconst.p, 0, (size_t)R, st));  // rows constant at t (R26)
     if (pf) {
@@ -851,6 +852,7 @@ static snicit_status infer_core(snicit_network* net, const float* y0, int64_t ba
         pa.app_count = cnt + live_ctr[(ci + 1) % 3];
         pa.work = cnt + CNT_PFWORK;
         pa.full_rl = net->pf_full.p;
+        pa.ydead = (y_out_on_device && y_out && drop) ? y_out : nullptr;
         pa.rconst = net->rconst.p;
         pa.rval = net->rval.p;
         pa.n_const = cnt + CNT_PFCONST;
@@ -961,7 +963,7 @@ static snicit_status infer_core(snicit_network* net, const float* y0, int64_t ba
         }
         if (!y_out_on_device && y_out) y_dst = bufs[nxt_i];
         CUDA_TRY(launch_recover(N, R, 1, yfinal, net->live_row.p, nullptr, nullptr, nullptr, nullptr, y_dst,
-                                net->cat.p, net->num_sms, st));
+                                net->cat.p, net->num_sms, st, y_dst == y_out ? dead_zeroed : 0));
         ++launches;
     } else {
         // ordered live list: "the first s columns" are the first s live rows by id (R14)
@@ -1152,7 +1154,7 @@ static snicit_status infer_core(snicit_network* net, const float* y0, int64_t ba
         // ---- a6: recovery (Eq. 6)
         if (!y_out_on_device && y_out) y_dst = yh_nxt;  // free buffer
         CUDA_TRY(launch_recover(N, R, 0, yfinal, nullptr, net->M.p, net->cslot.p, net->ne_row.p, cfinal, y_dst,
-                                net->cat.p, net->num_sms, st));
+                                net->cat.p, net->num_sms, st, y_dst == y_out ? dead_zeroed : 0));
         ++launches;
     }
     // categories: ordered compaction of the cat flags over all rows (R13)

@@ -276,6 +276,7 @@ struct PreFusedArgs {
     int* app_list;     // rows alive at t, appended unordered (nullable)
     int* app_count;    //   zero on entry
     int* work;         // row scheduler, zero on entry
+    float* ydead;                 // nullable: rows found dead (R23) get N zeros here (the caller's y_out)
     uint8_t* rconst;              // nullable: rconst[row] = 1, rval[row] = v for rows constant at t (R26)
     float* rval;
     unsigned long long* full_rl;  // nullable: += full (non-constant) row-layer evaluations
@@ -320,7 +321,7 @@ cudaError_t launch_map_residual(const float* y, int N, const int* rows, const in
                                 const uint8_t* rconst = nullptr, const float* rval = nullptr);
 cudaError_t launch_recover(int N, int R, int plain, const float* yfinal, const uint8_t* live_row, const int* M,
                            const int* cslot, const uint8_t* ne_row, const float* cbuf, float* y_out,
-                           uint8_t* cat, int num_sms, cudaStream_t st);
+                           uint8_t* cat, int num_sms, cudaStream_t st, int dead_zeroed = 0);
 // packed binary rows -> fp32 rows: y[r][j] = bit j of row r ? one : 0 (snicit_infer_packed)
 cudaError_t launch_unpack_bits(const uint32_t* bits, int R, int N, float one, float* y, int num_sms, cudaStream_t st);
 cudaError_t launch_mark_rows(const int* rows, const int* count, uint8_t* flag_row, int max_rows, cudaStream_t st);
