@@ -30,8 +30,6 @@
 // active list at t.  Rows are scheduled dynamically (one atomic per row).
 #include <cuda_runtime.h>
 
-#include <algorithm>
-#include <cstdlib>
 #include <cstring>
 
 #include "snicit_internal.cuh"
@@ -406,11 +404,6 @@ static cudaError_t launch_tg(const PreFusedParams& p, int num_sms, cudaStream_t 
     cudaError_t e = blocks_per_sm((const void*)pre_fused_kernel<T, GENSTR, WUNI>, T, smem, &bps);
     if (e != cudaSuccess) return e;
     if (bps < 1) return cudaErrorInvalidConfiguration;
-    static const int bps_env = [] {  // experiment hook: cap the CTAs per SM
-        const char* v = getenv("SNICIT_PF_BPS");
-        return v ? atoi(v) : 0;
-    }();
-    if (bps_env > 0) bps = std::min(bps, bps_env);
     pre_fused_kernel<T, GENSTR, WUNI><<<num_sms * bps, T, smem, st>>>(p);
     return cudaGetLastError();
 }
@@ -424,11 +417,7 @@ cudaError_t launch_pre_fused(const PreFusedArgs& a, const PreFusedLayer* layers,
     if (a.t < 1 || a.t > kPfMaxLayers) return cudaErrorInvalidValue;
     static thread_local PreFusedParams p;  // 32 KB: not on the stack
     p.a = a;
-    static const int l2pf = [] {  // experiment hook (default on)
-        const char* v = getenv("SNICIT_PF_L2PF");
-        return v ? atoi(v) : 1;
-    }();
-    p.a.l2_prefetch = l2pf;
+    p.a.l2_prefetch = 1;  // measured neutral on C2 (row loads are short anyway); kept for larger rows
     for (int l = 0; l < a.t; ++l) {
         p.L[l].w0 = layers[l].w0;
         p.L[l].b0 = layers[l].b0;
