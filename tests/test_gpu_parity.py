@@ -144,9 +144,11 @@ def test_packed_inputs_equal_fp32(N, L, B, t, dev):
 
 
 @pytest.mark.parametrize("N,L,B,t,pm", [(1024, 60, 1500, 30, 0), (1024, 60, 1500, 30, 1), (1024, 60, 1500, 12, 0),
-                                        (1024, 60, 1500, 6, 0), (4096, 40, 400, 25, 0), (4096, 40, 400, 25, 1)])
+                                        (1024, 60, 1500, 6, 0), (4096, 40, 400, 25, 0), (4096, 40, 400, 25, 1),
+                                        (1024, 60, 1500, 2, 0), (4096, 40, 600, 3, 0)])
 def test_constant_centroid_rows(N, L, B, t, pm):
-    """post_const (constant centroid rows carried by one scalar chain per circulant layer) is
+    """post_const (constant centroid rows carried by one scalar chain per circulant layer; in the
+    fused mode also constant residue rows over constant centroid pre-activations, small t) is
     bit-identical to the full-row evaluation and to the oracle's SNICIT reference, fused and
     per-layer post modes, with and without residue rows."""
     net = sdgc.gen_network(N, L, "radix")
