@@ -4,6 +4,8 @@
   B-sweep   (Fig. 9 analog, P:1248-1351 / P:1399-1408): C2 edges/s vs batch size B (t = 30)
   prune_eps (approximate relaxation, P:883-888 / P:1469-1472): residue-heavy C2 (small t) with
             near-zero residual pruning: time, surviving residues, category flips and max |dY| vs exact
+  fig6      (Fig. 6 analog): post-convergence time per layer (fused and per-layer post
+            modes) vs the uncompressed per-layer kernels' time per layer on the same layers
   C5        (conventional-DNN path): medium sparse MLP 256 x 18, B = 60000, ELL kernel
 
     python scripts/sweeps.py [--quick]
@@ -68,6 +70,22 @@ def main():
              phases={k: st[k] for k in ("t_pre_ms", "t_convert_ms", "t_post_ms", "t_recover_ms")},
              live_at_t=st["live_at_t"], centroids=st["n_centroids"], residual_at_t=st["residual_at_t"],
              residual_final=st["residual_final"])
+
+    # ---- Fig. 6 analog: post-convergence time per layer vs uncompressed time per layer
+    opt_u = default_options(timing=2, pre_fused=0)  # one launch per layer: per-layer CUDA-event times
+    g.infer(y0, t=L, s=32, options=opt_u, y_out=out)
+    g.infer(y0, t=L, s=32, options=opt_u, y_out=out)
+    unc_ms = np.asarray(g.layer_profile(L)["ms"])
+    for t in ([30] if args.quick else [10, 20, 30]):
+        for pm in (0, 1):
+            opt = default_options(timing=1, post_mode=pm)
+            ms = timed(g, y0, out, t, 32, opt)
+            st = g.stats()
+            emit(study="fig6", config="C2", t=t, post_mode=pm, post_ms=st["t_post_ms"],
+                 post_ms_per_layer=st["t_post_ms"] / (L - t),
+                 uncompressed_ms_per_layer_same_layers=float(unc_ms[t:].mean()),
+                 ratio=float(unc_ms[t:].mean()) / (st["t_post_ms"] / (L - t)),
+                 residual_at_t=st["residual_at_t"], centroids=st["n_centroids"])
 
     # ---- B sweep (t = 30)
     for b in ([10000, 60000] if args.quick else [2000, 5000, 10000, 20000, 30000, 60000]):
