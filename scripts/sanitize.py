@@ -22,4 +22,27 @@ for mode, N, L, B, t, kw in (("radix", 1024, 24, 300, 3, {}), ("radix", 4096, 12
         cats = g.categories()
         torch.cuda.synchronize()
     print(mode, N, L, B, t, kw, "categories", len(cats), "sum", float(out.sum()))
+# row-resident pre phase at N = 16384 (three row buffers), per-layer constant-row mode (segmented +
+# column kernels, kernels_const.cu), packed rows streamed from pinned host memory (ready flags)
+from paper_conf_icpp_jiangh0h23_b200 import pack_rows  # noqa: E402
+for N, L, B, t, kw in ((16384, 7, 12, 3, {}), (16384, 7, 12, 7, dict(pre_fused=0)), (65536, 5, 4, 3, {})):
+    net = sdgc.gen_network(N, L, "radix")
+    Y0 = torch.from_numpy(sdgc.gen_inputs(N, B)).cuda()
+    out = torch.empty_like(Y0)
+    with SnicitNetwork.from_network(net) as g:
+        g.set_stream(torch.cuda.current_stream())
+        g.infer(Y0, t=t, s=32, y_out=out, **kw)
+        cats = g.categories()
+        torch.cuda.synchronize()
+    print("radix", N, L, B, t, kw, "categories", len(cats), "sum", float(out.sum()))
+net = sdgc.gen_network(4096, 12, "radix")
+Yh = sdgc.gen_inputs(4096, 5000)
+bits = torch.from_numpy(pack_rows(Yh).view(np.int32)).pin_memory()
+out = torch.empty((5000, 4096), dtype=torch.float32, device="cuda")
+with SnicitNetwork.from_network(net) as g:
+    g.set_stream(torch.cuda.current_stream())
+    g.infer_packed(bits.numpy(), t=4, s=32, y_out=out)
+    cats = g.categories()
+    torch.cuda.synchronize()
+print("packed streamed 4096 12 5000 4 categories", len(cats), "sum", float(out.sum()))
 print("sanitize run done")
