@@ -61,7 +61,7 @@ def load_library(path: str = LIB_PATH):
     global _lib
     if _lib is not None:
         return _lib
-    path = os.environ.get("SNICIT_LIB", path)
+    path = os.environ.get("SNICIT_LIB") or path
     if not os.path.exists(path):
         raise SnicitError(f"{path} not found: run __graft_entry__.build() (nvcc, sm_100a)")
     L = ctypes.CDLL(path)

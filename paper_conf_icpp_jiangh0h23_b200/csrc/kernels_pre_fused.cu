@@ -10,8 +10,8 @@
 // RadiX layers): T = N/32 threads, each evaluating two work items at once with packed
 // fma.rn.f32x2 (FFMA2: per-lane RN fmas, bit-identical to fmaf, R17) -- two items of the SAME row and
 // layer, so the pair never diverges.  Stride classes:
-//   NU1  nu == 1: item i = outputs [17i, 17i + 17) (odd stride between lanes: conflict-free LDS),
-//        window of 48 inputs; items i and i + T form the pair.
+//   NU1  nu == 1: N = 17T + 15T: thread i owns outputs [17i, 17i + 17) and [17T + 15i, 17T + 15i + 15)
+//        (odd lane strides: conflict-free LDS; exact tiling), paired for 15 outputs.
 //   STR  nu >= 32 with Q = N/nu >= 64: item (c, a0) = outputs (a0 + m)*nu + c, m < 16, window of 47
 //        inputs of residue class c; lanes on consecutive c (conflict-free); the pair is (c, a0) and
 //        (c, a0 + Q/2), i.e. base offsets b and b + N/2.
@@ -37,35 +37,36 @@
 namespace snicit {
 
 constexpr int kPfM1 = 17;  // NU1 outputs per item
-constexpr int kPfW1 = kPfM1 + 31;
 constexpr int kPfM = 16;   // STR / Q32 outputs per item
 constexpr int kPfW = kPfM + 31;
 
 typedef unsigned long long u64;
 
 // ---------------------------------------------------------------------------- layer bodies
-// Unguarded stores: the last item's outputs past N (q = N .. 17*n1 - 1 < N + 17) are computed from the
-// halo, i.e. they ARE the circular outputs q - N, and land in the output halo where they belong; a
-// thread without a second item recomputes the last item (identical values, benign duplicate stores).
-// The head outputs q < H are also written to the halo (H >= 96 > 47 + 17).
+// nu == 1: N = 32T = 17T + 15T, so thread i owns item 1 = outputs [17i, 17i + 17) and item 2 =
+// [17T + 15i, 17T + 15i + 15): both lane strides odd (conflict-free LDS), the row tiled exactly (no
+// idle lanes, no outputs past N).  Outputs 0..14 of both items are FFMA2 pairs; item 1's outputs 15,
+// 16 are scalar chains on the low halves (half the FMA-pipe cycles of a half-used pair).  Windows read
+// up to N + 30 (halo); the head outputs q < H are also written to the halo.
 template <int T>
 __device__ __forceinline__ void pf_body_nu1(const float* __restrict__ in, float* __restrict__ out, float w0, float b0,
                                             float ymax, int H, float& mn, float& mx) {
     constexpr int N = 32 * T;
-    constexpr int n1 = (N + kPfM1 - 1) / kPfM1;
+    constexpr int M2 = 15;           // item 2 outputs
+    constexpr int W2N = M2 + 31;     // paired window (46)
     const int i1 = threadIdx.x;
-    const int i2 = min(i1 + T, n1 - 1);
     const float* s1 = in + kPfM1 * i1;
-    const float* s2 = in + kPfM1 * i2;
-    u64 R[kPfW1];
+    const float* s2 = in + kPfM1 * T + M2 * i1;
+    u64 R[W2N];
 #pragma unroll
-    for (int i = 0; i < kPfW1; ++i) R[i] = f2_pack(s1[i], s2[i]);
+    for (int i = 0; i < W2N; ++i) R[i] = f2_pack(s1[i], s2[i]);
+    const float e46 = s1[W2N], e47 = s1[W2N + 1];  // item 1's window tail
     const u64 W2 = f2_pack(w0, w0), B2 = f2_pack(b0, b0);
     float o1s[kPfM1];
     float* d1 = out + kPfM1 * i1;
-    float* d2 = out + kPfM1 * i2;
+    float* d2 = out + kPfM1 * T + M2 * i1;
 #pragma unroll
-    for (int m = 0; m < kPfM1; ++m) {
+    for (int m = 0; m < M2; ++m) {
         u64 acc = 0ull;
 #pragma unroll
         for (int n = 0; n < 32; ++n) acc = f2_fma(R[m + n], W2, acc);
@@ -78,7 +79,27 @@ __device__ __forceinline__ void pf_body_nu1(const float* __restrict__ in, float*
         mn = fminf(mn, fminf(o1, o2));
         mx = fmaxf(mx, fmaxf(o1, o2));
     }
-    if (kPfM1 * i1 < H) {  // head outputs -> halo (item 2 never: 17*T > 31*nu_max for every STR layer)
+#pragma unroll
+    for (int m = M2; m < kPfM1; ++m) {  // item 1 only: scalar chains on the low halves
+        float acc = 0.0f;
+#pragma unroll
+        for (int n = 0; n < 32; ++n) {
+            float x;
+            if (m + n < W2N) {
+                float hi;
+                f2_unpack(R[m + n], x, hi);
+            } else {
+                x = (m + n == W2N) ? e46 : e47;
+            }
+            acc = fmaf(x, w0, acc);
+        }
+        const float o1 = sigma(acc + b0, ymax);
+        d1[m] = o1;
+        o1s[m] = o1;
+        mn = fminf(mn, o1);
+        mx = fmaxf(mx, o1);
+    }
+    if (kPfM1 * i1 < H) {  // head outputs -> halo (item 2 starts at 17T > H)
 #pragma unroll
         for (int m = 0; m < kPfM1; ++m)
             if (kPfM1 * i1 + m < H) out[N + kPfM1 * i1 + m] = o1s[m];
