@@ -38,6 +38,7 @@ namespace snicit {
 
 constexpr int kPfM1 = 17;  // NU1 outputs per item
 constexpr int kPfM = 16;   // STR / Q32 outputs per item
+constexpr int kPfSurv = 32;  // survivor batch per CTA
 constexpr int kPfW = kPfM + 31;
 
 typedef unsigned long long u64;
@@ -237,6 +238,17 @@ __global__ void __launch_bounds__(T, PfCfg<T>::kMinBlocks) pre_fused_kernel(cons
     int pos = s_pos[0];
     // one row (and its circular halo: a second copy of the row head) -> buffer `dst`, completion on `b`
     uint32_t* s_bits = reinterpret_cast<uint32_t*>(s_ok + 2 * kWarps);  // [2][N/32] packed rows (a.ybits)
+    int* s_surv = reinterpret_cast<int*>(s_bits + 2 * (N / 32));       // [kPfSurv] rows alive at t, batched
+    int nsurv = 0;                                                     // (tid 0) entries in s_surv
+    // one atomic per kPfSurv survivors (an atomic whose result is waited on stalls the whole CTA at the
+    // next barrier; per row that was ~1 us)
+    auto flush_surv = [&](bool force) {
+        if (tid == 0 && nsurv > 0 && (force || nsurv == kPfSurv)) {
+            const int p0 = atomicAdd(a.app_count, nsurv);
+            for (int i = 0; i < nsurv; ++i) a.app_list[p0 + i] = s_surv[i];
+            nsurv = 0;
+        }
+    };
     auto issue_load = [&](int p_, float* dst, uint64_t* b, int slot) {
         const size_t r_ = (size_t)__ldg(a.rows + p_);
         if (a.ybits) {  // packed binary row: N/8 bytes
@@ -257,6 +269,7 @@ __global__ void __launch_bounds__(T, PfCfg<T>::kMinBlocks) pre_fused_kernel(cons
     int i_in = 0, i_out = 1, i_pf = 2;  // buffer roles (NB == 3: i_pf receives the next row)
     uint32_t ph = 0;                    // phase bit of bar[0], bar[1]
     if (NB == 3 && tid == 0 && pos < count) issue_load(pos, buf, &bar[0], 0);
+    int np = 0;  // tid 0: the next row's list position
     for (int k = 0; pos < count; ++k) {
         const int row = __ldg(a.rows + pos);
         if (tid == 0) {
@@ -264,14 +277,12 @@ __global__ void __launch_bounds__(T, PfCfg<T>::kMinBlocks) pre_fused_kernel(cons
                 bulk_wait_read0();  // the previous row's TMA store has finished reading its buffer
                 issue_load(pos, buf, &bar[k & 1], k & 1);
             }
-            const int np = atomicAdd(a.work, 1);  // next row (read after the end-of-row barrier)
-            s_pos[2 + (k & 1)] = np;
-            if (np < count) {
-                if (NB == 3) {  // load it now, behind this row's compute
+            np = atomicAdd(a.work, 1);  // next row (NB == 2: consumed at the row end, latency hidden)
+            if (NB == 3) {
+                s_pos[2 + (k & 1)] = np;
+                if (np < count) {  // load it now, behind this row's compute
                     bulk_wait_read0();
                     issue_load(np, buf + i_pf * S, &bar[(k + 1) & 1], (k + 1) & 1);
-                } else if (a.l2_prefetch && !a.ybits) {  // pull it into L2: its load at the next row start is short
-                    bulk_prefetch_l2(a.yin + (size_t)__ldg(a.rows + np) * N, N * 4);
                 }
             }
         }
@@ -380,8 +391,8 @@ __global__ void __launch_bounds__(T, PfCfg<T>::kMinBlocks) pre_fused_kernel(cons
                 }
             }
             if (tid == 0 && a.app_list) {
-                const int p = atomicAdd(a.app_count, 1);
-                a.app_list[p] = row;
+                s_surv[nsurv++] = row;
+                flush_surv(false);
             }
             if (tid == 0 && a.rconst && cst) {  // constant at t: conversion needs no read of the row
                 a.rconst[row] = 1;
@@ -391,6 +402,11 @@ __global__ void __launch_bounds__(T, PfCfg<T>::kMinBlocks) pre_fused_kernel(cons
         if (tid == 0) {
             if (a.full_rl) atomicAdd(a.full_rl, (unsigned long long)full);
             if (a.n_const && cst) atomicAdd(a.n_const, 1);
+        }
+        if (NB == 2 && tid == 0) {
+            s_pos[2 + (k & 1)] = np;
+            if (np < count && a.l2_prefetch && !a.ybits)  // pull it into L2: its load is short
+                bulk_prefetch_l2(a.yin + (size_t)__ldg(a.rows + np) * N, N * 4);
         }
         __syncthreads();  // buffers free, next position visible
         pos = s_pos[2 + (k & 1)];
@@ -403,6 +419,7 @@ __global__ void __launch_bounds__(T, PfCfg<T>::kMinBlocks) pre_fused_kernel(cons
             i_out = 1;
         }
     }
+    if (a.app_list) flush_surv(true);
     if (tid == 0) bulk_wait0();
 }
 
@@ -415,7 +432,7 @@ int pre_fused_threads(int N) {
 size_t pre_fused_smem(int N, int H) {
     const int nb = N / 32 >= 512 ? 3 : 2;  // kPfBufs
     return sizeof(float) * nb * (size_t)(N + H) + 2 * sizeof(uint64_t) + 4 * sizeof(int) + 4 * sizeof(int) * (N / 32 / 32) +
-           2 * sizeof(uint32_t) * (size_t)(N / 32);  // packed-row slots
+           2 * sizeof(uint32_t) * (size_t)(N / 32) + sizeof(int) * kPfSurv;  // packed-row slots, survivors
 }
 
 template <int T, bool GENSTR, bool WUNI>
