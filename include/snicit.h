@@ -207,7 +207,9 @@ snicit_status snicit_stats(snicit_network* net, snicit_stats_t* out);
 /* Per-launch profile of the pre-convergence layer kernels of the last infer run with
  * options.timing == 2: for layer i < *n (n = min(t, max)): ms[i] = CUDA-event duration of the
  * layer kernel launch (on the handle's stream), rows[i] = active rows it processed, bytes[i] =
- * algorithmic HBM bytes of the launch (8*rows*N + W bytes + 4*N).
+ * algorithmic HBM bytes of the launch (8*rows*N + W bytes + 4*N; the
+ * row-resident kernel: one launch, 4*N per input row + 4*N per row alive at t (+ 4*N per dead row
+ * when it wrote the dead rows' zeros into a device y_out)).
  * Host pointers; any may be NULL.  Synchronises the stream. */
 snicit_status snicit_layer_profile(snicit_network* net, int32_t max, double* ms, int64_t* rows, double* bytes,
                                    int32_t* n);

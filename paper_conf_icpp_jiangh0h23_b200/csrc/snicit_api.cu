@@ -129,6 +129,7 @@ struct snicit_network {
     bool last_cluster = false;
     bool last_kernel_circ = false;
     bool last_pre_fused = false;
+    bool last_dead_zeroed = false;  // the row-resident kernel wrote dead rows' zeros into y_out
     snicit_stats_t stats{};
     cudaEvent_t ev[6] = {nullptr, nullptr, nullptr, nullptr, nullptr, nullptr};
     std::vector<cudaEvent_t> lev;  // 2 per pre-convergence layer (timing == 2)
@@ -822,6 +823,7 @@ static snicit_status infer_core(snicit_network* net, const float* y0, int64_t ba
     if (y0_mode == 3 && !pf && R > 0) return fail(SNICIT_E_STATE, "packed rows without the row-resident kernel");
     net->last_pre_fused = pf;
     const int dead_zeroed = (pf && y_out_on_device && y_out && drop) ? 1 : 0;  // y_out rows of dead rows
+    net->last_dead_zeroed = dead_zeroed != 0;
     stats.pre_fused = pf ? 1 : 0;
     if (R > 0) CUDA_TRY(cudaMemsetAsync(net->rconst.p, 0, (size_t)R, st));  // rows constant at t (R26)
     if (pf) {
@@ -1361,7 +1363,9 @@ snicit_status snicit_layer_profile(snicit_network* net, int32_t max, double* ms,
             // row-resident kernel: every input row read once, every row alive at t written once
             int live = 0;
             CUDA_TRY(read_counter(net, net->live_counter, &live));
-            bytes[l] = 4.0 * net->N * ((double)h[l] + live) + sizeof(PreFusedLayer) * (double)net->last_t;
+            // (+ the zeros of the rows found dead, written into y_out when it is on the device)
+            const double dead = net->last_dead_zeroed ? (double)h[l] - live : 0.0;
+            bytes[l] = 4.0 * net->N * ((double)h[l] + live + dead) + sizeof(PreFusedLayer) * (double)net->last_t;
         } else if (bytes) {
             const LayerPlan& pl = net->plan[l];
             // algorithmic bytes: rows read + written, weights, bias
