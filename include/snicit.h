@@ -181,7 +181,8 @@ snicit_status snicit_infer(snicit_network* net, const float* y0, int64_t batch,
  * y0_bits: batch*W uint32, device pointer if bits_on_device else host.  one_value: finite.
  * When the row-resident pre-convergence kernel applies (options.pre_fused, N % 128 == 0) it reads
  * each row's bits itself and expands them in shared memory (no fp32 Y0 in HBM); host bits are then
- * uploaded in chunks of 2048 rows by the copy engine on a side stream WHILE the kernel runs (it
+ * uploaded in geometrically growing chunks (512, 1024, 2048, ... rows) by the copy engine on a side
+ * stream WHILE the kernel runs (it
  * waits per chunk on a ready flag), so the upload overlaps the compute (pinned host memory gives
  * the asynchronous copies; pageable memory works but the copies block the host).  Otherwise the
  * rows are copied, then unpacked by

@@ -1234,8 +1234,11 @@ snicit_status snicit_infer_packed(snicit_network* net, const uint32_t* y0_bits, 
             // streamed upload: the copy engine delivers chunks of rows on a side stream while the
             // row-resident kernel runs; each chunk is followed by its ready flag (the kernel polls it
             // before loading a row of the chunk), so the upload overlaps the compute
-            constexpr int kChunk = 2048;
-            const int nch = (R + kChunk - 1) / kChunk;
+            // geometric chunks: chunk c = rows [b (2^c - 1), b (2^(c+1) - 1)), b = kChunk0 -- the first
+            // rows arrive within microseconds and the whole batch takes a handful of API calls
+            constexpr int kChunk0 = 512;
+            int nch = 0;
+            while ((long long)kChunk0 * ((1LL << nch) - 1) < R) ++nch;
             if (!net->copy_stream) CUDA_TRY(cudaStreamCreateWithFlags(&net->copy_stream, cudaStreamNonBlocking));
             for (auto& e : net->cev)
                 if (!e) CUDA_TRY(cudaEventCreateWithFlags(&e, cudaEventDisableTiming));
@@ -1243,12 +1246,13 @@ snicit_status snicit_infer_packed(snicit_network* net, const uint32_t* y0_bits, 
                 CUDA_TRY(cudaMallocHost(&net->h_ones, sizeof(int)));
                 *net->h_ones = 1;
             }
-            CUDA_TRY(net->bits_ready.ensure((size_t)nch));
-            CUDA_TRY(cudaMemsetAsync(net->bits_ready.p, 0, sizeof(int) * nch, net->stream));
+            CUDA_TRY(net->bits_ready.ensure((size_t)std::max(nch, 1)));
+            CUDA_TRY(cudaMemsetAsync(net->bits_ready.p, 0, sizeof(int) * std::max(nch, 1), net->stream));
             CUDA_TRY(cudaEventRecord(net->cev[0], net->stream));
             CUDA_TRY(cudaStreamWaitEvent(net->copy_stream, net->cev[0], 0));
             for (int c = 0; c < nch; ++c) {
-                const size_t r0 = (size_t)c * kChunk, nr = std::min<size_t>(kChunk, R - r0);
+                const size_t r0 = (size_t)kChunk0 * ((1ull << c) - 1);
+                const size_t nr = std::min<size_t>((size_t)kChunk0 << c, R - r0);
                 CUDA_TRY(cudaMemcpyAsync(net->bits.p + r0 * W, y0_bits + r0 * W, sizeof(uint32_t) * nr * W,
                                          cudaMemcpyHostToDevice, net->copy_stream));
                 CUDA_TRY(cudaMemcpyAsync(net->bits_ready.p + c, net->h_ones, sizeof(int), cudaMemcpyHostToDevice,
@@ -1256,7 +1260,7 @@ snicit_status snicit_infer_packed(snicit_network* net, const uint32_t* y0_bits, 
             }
             CUDA_TRY(cudaEventRecord(net->cev[1], net->copy_stream));
             ready = net->bits_ready.p;
-            ready_rows = kChunk;
+            ready_rows = kChunk0;
             streamed = true;
         } else {
             CUDA_TRY(cudaMemcpyAsync(net->bits.p, y0_bits, sizeof(uint32_t) * (size_t)R * W, cudaMemcpyHostToDevice,

@@ -268,8 +268,8 @@ struct PreFusedArgs {
     const float* yin;
     const uint32_t* ybits;  // non-null: input rows as packed bits (N/32 words per row, LSB first), value `one`
     float one;
-    const int* ready;       // nullable: ready[r / ready_rows] != 0 once rows of that chunk are in ybits
-    int ready_rows;         //   (uploaded by the copy engine while the kernel runs)
+    const int* ready;       // nullable: ready[c] != 0 once chunk c (rows [b (2^c - 1), b (2^(c+1) - 1)),
+    int ready_rows;         //   b = ready_rows) is in ybits (uploaded by the copy engine while the kernel runs)
     float* yout;
     const int* rows;   // input list [*count]
     const int* count;
