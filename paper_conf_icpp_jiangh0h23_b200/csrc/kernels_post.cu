@@ -254,6 +254,7 @@ __global__ void __launch_bounds__(kCentThreads) centroid_traj_kernel(PostArgs a)
     const int C = *a.n_cent;
     const int c = blockIdx.x;
     if (c >= C || (a.cdone && a.cdone[c])) return;
+    const bool want_a = a.a_all && (!a.rcount || *a.rcount > 0);  // a_c rows only for residue rows
     const int N = a.N;
     const int h = post_halo(N);
     const int dup = h == N;
@@ -266,7 +267,7 @@ __global__ void __launch_bounds__(kCentThreads) centroid_traj_kernel(PostArgs a)
     PL Ld = load_pl(a.layers + a.t);
     for (int l = a.t; l < a.L; ++l) {
         const PL Lnext = load_pl(a.layers + min(l + 1, a.L - 1));  // prefetch (serial critical path)
-        float* aout = a.a_all ? a.a_all + ((size_t)(l - a.t) * a.s + c) * N : nullptr;
+        float* aout = want_a ? a.a_all + ((size_t)(l - a.t) * a.s + c) * N : nullptr;
         post_row_layer<MODE_CENTROID, 5, 4, 8>(Ld, N, dup, a.ymax, 0.0f, cur, nxt, nullptr, aout, a.force_ell);
         __syncthreads();
         fill_halo(nxt, N, h);
@@ -370,7 +371,7 @@ __global__ void __launch_bounds__(kPostThreads, 2) residual_traj_kernel(PostArgs
 // every later one is: a constant input row stays constant, R25), or L - t; scans layers in order
 __global__ void __launch_bounds__(256) acconst_kernel(PostArgs a) {
     const int c = blockIdx.x;
-    if (c >= *a.n_cent) return;
+    if (c >= *a.n_cent || (a.rcount && *a.rcount == 0)) return;
     const int N = a.N, nl = a.L - a.t;
     int l2 = 0;
     if (a.cdone && a.cdone[c]) {
@@ -415,6 +416,7 @@ __global__ void __cluster_dims__(kCL, 1, 1) __launch_bounds__(kClThreads) centro
     const int cid = blockIdx.x / kCL;
     const int C = *a.n_cent;
     if (cid >= C || (a.cdone && a.cdone[cid])) return;  // uniform over the cluster
+    const bool want_a = a.a_all && (!a.rcount || *a.rcount > 0);  // a_c rows only for residue rows
     const int N = a.N, S = N / kCL;  // powers of two (centroid_cluster_ok)
     const int shS = ilog2(S);
     float* slice[2] = {sm, sm + S};
@@ -443,7 +445,7 @@ __global__ void __cluster_dims__(kCL, 1, 1) __launch_bounds__(kClThreads) centro
 #pragma unroll
             for (int n = 0; n < kPK; ++n) wr[n] = __ldg(Ld.wtab + n);
         }
-        float* aout = a.a_all ? a.a_all + ((size_t)(l - a.t) * a.s + cid) * N : nullptr;
+        float* aout = want_a ? a.a_all + ((size_t)(l - a.t) * a.s + cid) * N : nullptr;
         // ---- gather this CTA's input window from the peers' slices (previous layer's outputs)
         float* const* rb = s_rbase[cur];
         const int shnp = ilog2(prev_nu);
@@ -651,7 +653,7 @@ __global__ void __launch_bounds__(256) centroid_const_kernel(PostArgs a, float* 
         s_v = v;
     }
     __syncthreads();
-    if (a.a_all)
+    if (a.a_all && (!a.rcount || *a.rcount > 0))  // a_c rows only when residue rows need them
         for (int l = 0; l < nl; ++l) {
             float* dst = a.a_all + ((size_t)l * a.s + c) * N;
             const float acc = s_acc[l];

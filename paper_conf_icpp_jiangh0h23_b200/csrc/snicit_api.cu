@@ -130,6 +130,7 @@ struct snicit_network {
     bool last_kernel_circ = false;
     bool last_pre_fused = false;
     bool last_dead_zeroed = false;  // the row-resident kernel wrote dead rows' zeros into y_out
+    bool res_at_t_lazy = false;     // residual_at_t is read from CNT_RES0 by snicit_stats
     snicit_stats_t stats{};
     cudaEvent_t ev[6] = {nullptr, nullptr, nullptr, nullptr, nullptr, nullptr};
     std::vector<cudaEvent_t> lev;  // 2 per pre-convergence layer (timing == 2)
@@ -997,12 +998,16 @@ static snicit_status infer_core(snicit_network* net, const float* y0, int64_t ba
         // ---- a5: post-convergence layers, Eq. 5 for i = t..L-1
         float* c_cur = net->cbuf0.p;
         float* c_nxt = net->cbuf1.p;
-        int res_host = 1;
-        CUDA_TRY(read_counter(net, CNT_RES0, &res_host));
-        stats.residual_at_t = res_host;
         float* yh_cur = yhat;
         float* yh_nxt = yhat_other;
         const bool fused = opt.post_mode == 0 && N <= post_fused_max_n();
+        // fused mode: no host read of the residue count (the kernels read it on the device and the
+        // a_c rows are written only when residue rows exist), so the stream is never stalled here;
+        // res_host = 1 means "maybe"
+        int res_host = 1;
+        if (!fused) CUDA_TRY(read_counter(net, CNT_RES0, &res_host));
+        if (!fused) stats.residual_at_t = res_host;
+        net->res_at_t_lazy = fused;  // fused: CNT_RES0 still holds it when snicit_stats reads it
         net->last_fused = fused;
         // constant centroid rows (centroid_const_kernel): every post layer circulant with uniform
         // weights and bias.  Fused mode: in place, the trajectory kernels skip the carried rows.
@@ -1028,6 +1033,7 @@ static snicit_status infer_core(snicit_network* net, const float* y0, int64_t ba
             if (fused && res_host > 0) {
                 CUDA_TRY(net->a_all.ensure((size_t)(L - tt) * (size_t)s * N));
                 pc.a_all = net->a_all.p;
+                pc.rcount = rcnt;
             }
             CUDA_TRY(launch_centroid_const(pc, fused ? net->cbuf0.p : net->cbuf1.p, cdone, cnt + CNT_CDONE, s, st));
             ++launches;
@@ -1100,7 +1106,7 @@ static snicit_status infer_core(snicit_network* net, const float* y0, int64_t ba
                     CUDA_TRY(launch_acconst(pa, s, st));
                     ++launches;
                 }
-                CUDA_TRY(launch_residual_traj(pa, res_host, net->num_sms, st));
+                CUDA_TRY(launch_residual_traj(pa, R, net->num_sms, st));
                 ++launches;
             }
         }
@@ -1320,6 +1326,10 @@ snicit_status snicit_stats(snicit_network* net, snicit_stats_t* out) {
     if (net->last_converted && net->res_final_counter >= 0) {
         CUDA_TRY(read_counter(net, net->res_final_counter, &v));
         net->stats.residual_final = v;
+    }
+    if (net->last_converted && net->res_at_t_lazy) {
+        CUDA_TRY(read_counter(net, CNT_RES0, &v));
+        net->stats.residual_at_t = v;
     }
     if (net->last_converted) {
         CUDA_TRY(read_counter(net, CNT_NCENT, &v));
