@@ -409,6 +409,15 @@ def run_snicit(args):
     if len(pm):
         roof = alu_roof(pm, pb, st) if st["pre_fused"] else hbm_roof(pm, pb, st)
         roof["share_of_step"] = float(pm.sum() / ms) if ms > 0 else None
+        if st["pre_fused"] and ms > 0:
+            # whole step: the step's algorithmic flops (the row-resident pre phase: post
+            # layers of constant centroids are scalars) and bytes (pre phase + the live rows' final
+            # activations written by the recovery) over the measured step time
+            step_flops = roof["algorithmic_flops"]
+            step_bytes = roof["hbm"]["algorithmic_bytes"] + 4.0 * c["N"] * st["live_at_t"]
+            roof["whole_step"] = {"alu_frac": step_flops / (ms * 1e-3) / 1e12 / FMA_PEAK_TFLOPS,
+                                  "hbm_frac": step_bytes / (ms * 1e-3) / 1e9 / peak,
+                                  "algorithmic_flops": step_flops, "algorithmic_bytes": step_bytes}
         if st["pre_fused"] and not args.no_variants:
             # the same kernel with every live row evaluated in full (no constant-row shortcut), and the
             # per-layer kernels (one launch per layer, HBM-bound) on the same inputs
