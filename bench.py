@@ -202,14 +202,21 @@ def measured_peaks():
     return 6650.0, "fallback (B200_PROFILING.md: 6.65 TB/s)"
 
 
-def oracle_sample_time(oracle, net, Y, cores, seconds, probe_only=False):
+def oracle_sample_time(oracle, net, Y, cores, seconds, probe_only=False, max_rows=None):
     """Rows of Y the oracle processes in ~`seconds` on all host cores (calibrated on `cores` rows run
-    with all threads), and the measured time for that many rows."""
+    with all threads; at most `max_rows`, default len(Y)), and the measured time for that many rows."""
+    cap = len(Y) if max_rows is None else max_rows
+    # probe sizes double until one takes >= seconds / 2 (small probes are dominated by per-call and
+    # thread start-up cost, which would under-size the sample)
     k = max(1, min(len(Y), cores))
-    t0 = time.perf_counter()
-    oracle_layers(oracle, net, Y[:k])
-    t_probe = max(time.perf_counter() - t0, 1e-6)
-    rows = int(max(k, min(len(Y), k * seconds / t_probe)))
+    while True:
+        t0 = time.perf_counter()
+        oracle_layers(oracle, net, Y[:k])
+        t_probe = max(time.perf_counter() - t0, 1e-6)
+        if t_probe >= seconds / 2 or k >= len(Y):
+            break
+        k = min(len(Y), 2 * k)
+    rows = int(max(k, min(cap, k * seconds / t_probe)))
     if probe_only:
         return rows, None
     if rows == k:
@@ -231,8 +238,9 @@ def run_reference(args):
     nnz = net.nnz
     cores = os.cpu_count() or 1
     # size the per-step sample to ~cpu_seconds / steps of the oracle on all cores
-    probe = make_inputs(args, c, cores, 0)
-    rows, _ = oracle_sample_time(oracle, net, probe, cores, args.cpu_seconds / max(args.steps, 1), probe_only=True)
+    probe = make_inputs(args, c, min(c["B"], 64 * cores), 0)
+    rows, _ = oracle_sample_time(oracle, net, probe, cores, args.cpu_seconds / max(args.steps, 1), probe_only=True,
+                                 max_rows=c["B"])
     Y = make_inputs(args, c, rows, 0)
     if args.warmup > 0:
         oracle_layers(oracle, net, Y[: max(1, min(rows, cores))])
