@@ -30,7 +30,7 @@
 extern "C" {
 #endif
 
-#define SNICIT_ABI_VERSION 3
+#define SNICIT_ABI_VERSION 4
 
 typedef struct snicit_network snicit_network; /* opaque: owns device copies of W, b + workspace */
 
@@ -166,9 +166,13 @@ snicit_status snicit_set_stream(snicit_network* net, void* cuda_stream);
  *  opt:             NULL = snicit_default_options.
  *  y_out:           batch*N fp32, caller-owned; device pointer if y_out_on_device else host;
  *                   NULL = do not materialise Y(L) (categories are still computed).
- * Synchronous w.r.t. the host only when a host pointer is involved or opt->ne_interval
- * triggers a count read; otherwise work is queued on the handle's stream.
- * Call snicit_categories afterwards (it synchronises the stream). */
+ * Alignment: device y0 / y_out must be 16-byte aligned (TMA bulk copies and float4 accesses);
+ * otherwise SNICIT_E_INVALID_ARG.
+ * Host synchronisation: when y0 or y_out is a HOST pointer the call returns only after the stream
+ * has finished with it (y_out filled, y0 consumed).  With device pointers only, the work is queued
+ * on the handle's stream and the call returns immediately (per-layer post mode may read a device
+ * counter every opt->ne_interval layers).  snicit_categories synchronises the stream.
+ * The caller's current CUDA device is restored on return (every entry point). */
 snicit_status snicit_infer(snicit_network* net, const float* y0, int64_t batch,
                            int32_t y0_on_device, int64_t row_offset, int32_t threshold_layer,
                            int32_t centroid_count, const snicit_options* opt, float* y_out,
@@ -187,7 +191,9 @@ snicit_status snicit_infer(snicit_network* net, const float* y0, int64_t batch,
  * the asynchronous copies; pageable memory works but the copies block the host).  Otherwise the
  * rows are copied, then unpacked by
  * a kernel into the handle's workspace.  Either way the inference proceeds exactly as snicit_infer
- * on the equivalent fp32 Y0 (same results, tested).  All other arguments as snicit_infer. */
+ * on the equivalent fp32 Y0 (same results, tested).  Host bits: the call returns once the upload has
+ * consumed them (the buffer may then be reused).  Device bits must be 16-byte aligned.  All other
+ * arguments as snicit_infer. */
 snicit_status snicit_infer_packed(snicit_network* net, const uint32_t* y0_bits, int64_t batch,
                                   int32_t bits_on_device, float one_value, int64_t row_offset,
                                   int32_t threshold_layer, int32_t centroid_count,
@@ -201,6 +207,13 @@ snicit_status snicit_infer_packed(snicit_network* net, const uint32_t* y0_bits, 
  * the count).  SNICIT_E_STATE before any infer. */
 snicit_status snicit_categories(snicit_network* net, int64_t* rows, int64_t* count,
                                 int32_t rows_on_device);
+
+/* Device-side export of the category set of the last infer for the multi-GPU all-gather (SURVEY
+ * 8(e)): asynchronous on the handle's stream, no host synchronisation.  out (DEVICE pointer, 8-byte
+ * aligned, 1 + capacity int64): out[0] = total number of categories of this shard, out[1 + i] =
+ * row_offset + local row id of the i-th category (ascending), i < min(total, capacity); the rest of
+ * `out` is left untouched.  SNICIT_E_STATE before any infer. */
+snicit_status snicit_categories_device(snicit_network* net, int64_t* out, int64_t capacity);
 
 /* Statistics of the last infer (synchronises the stream). */
 snicit_status snicit_stats(snicit_network* net, snicit_stats_t* out);

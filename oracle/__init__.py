@@ -46,6 +46,10 @@ def lib():
         L.oracle_layers_f32.argtypes = [i32, P, P, P, P, f32, i32, i32, i64, P, P, i32]
         L.oracle_layers_f64.argtypes = [i32, P, P, P, P, f32, i32, i32, i64, P, P, i32]
         L.oracle_layers_circulant_f32.argtypes = [i32, i32, P, P, P, f32, i32, i32, i64, P, P, i32]
+        L.oracle_layers_f32_fast.argtypes = [i32, P, P, P, P, f32, i32, i32, i64, P, P, i32]
+        L.oracle_layers_f32_fast.restype = i64
+        L.oracle_layers_circulant_f32_fast.argtypes = [i32, i32, P, P, P, f32, i32, i32, i64, P, P, i32]
+        L.oracle_layers_circulant_f32_fast.restype = i64
         L.oracle_sum_downsample.argtypes = [i32, i32, i32, P, P]
         L.oracle_prune.argtypes = [i32, i32, P, f32, f32, P]
         L.oracle_prune.restype = i32
@@ -101,6 +105,27 @@ def layers_circulant_f32(cnet, Y: np.ndarray, l0: int = 0, l1: Optional[int] = N
     lib().oracle_layers_circulant_f32(cnet.N, w.shape[1], _p(nu), _p(w), _p(b), cnet.ymax, l0, l1, Y.shape[0],
                                       _p(Y), _p(out), nthreads)
     return out
+
+
+def layers_f32_fast(net, Y: np.ndarray, l0: int = 0, l1: Optional[int] = None, nthreads: int = 0,
+                    return_skipped: bool = False):
+    """Exact fast mode of Eq. (1) (oracle.h): fixed-point rows (all-zero / all-YMAX) whose image under a
+    layer is themselves are not re-evaluated.  Identical to layers_f32 (pinned).  Accepts a CSC Network
+    or a compact CirculantNetwork."""
+    l1 = net.L if l1 is None else l1
+    Y = np.ascontiguousarray(Y, dtype=np.float32)
+    out = np.empty_like(Y)
+    if hasattr(net, "nu"):
+        nu = np.ascontiguousarray(net.nu, dtype=np.int32)
+        w = np.ascontiguousarray(net.w, dtype=np.float32)
+        b = np.ascontiguousarray(net.bias, dtype=np.float32)
+        sk = lib().oracle_layers_circulant_f32_fast(net.N, w.shape[1], _p(nu), _p(w), _p(b), net.ymax, l0, l1,
+                                                    Y.shape[0], _p(Y), _p(out), nthreads)
+    else:
+        ptr, idx, val, bias = _net_arrays(net)
+        sk = lib().oracle_layers_f32_fast(net.N, _p(ptr), _p(idx), _p(val), _p(bias), net.ymax, l0, l1,
+                                          Y.shape[0], _p(Y), _p(out), nthreads)
+    return (out, int(sk)) if return_skipped else out
 
 
 def categories(Y: np.ndarray) -> np.ndarray:

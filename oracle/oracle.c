@@ -103,7 +103,11 @@ static void row_layer_circ_f32(int32_t N, int32_t K, int32_t nu, const float* w,
                                const float* y, float* y_next) {
     for (int32_t j = 0; j < N; ++j) {
         float acc = 0.0f;
-        for (int32_t n = 0; n < K; ++n) acc = fmaf(y[(int32_t)(((int64_t)j + (int64_t)n * nu) % N)], w[n], acc);
+        for (int32_t n = 0; n < K; ++n) {
+            int64_t k = (int64_t)j + (int64_t)n * nu; /* (j + n*nu) mod N */
+            if (k >= N) k %= N;
+            acc = fmaf(y[k], w[n], acc);
+        }
         y_next[j] = sigma_f32(acc + b[j], ymax);
     }
 }
@@ -128,6 +132,101 @@ void oracle_layers_circulant_f32(int32_t N, int32_t K, const int32_t* nu, const 
         free(a);
         free(c);
     }
+}
+
+/* ---- exact fast mode (oracle.h): memoised fixed points of one layer */
+static int row_all_equal(const float* y, int32_t N, float v) {
+    for (int32_t k = 0; k < N; ++k) if (!(y[k] == v)) return 0;
+    return 1;
+}
+
+/* fixed[l - l0]: bit 0 = layer l maps the all-zero row to itself, bit 1 = the all-YMAX row to itself,
+ * decided by evaluating the layer on those two rows with the plain row function */
+static uint8_t* fixed_points(int32_t N, int32_t l0, int32_t l1, float ymax,
+                             void (*eval)(int32_t l, const float* y, float* y_next, const void* ctx),
+                             const void* ctx) {
+    uint8_t* fixed = (uint8_t*)calloc((size_t)(l1 > l0 ? l1 - l0 : 1), 1);
+#pragma omp parallel
+    {
+        float* z = (float*)malloc(sizeof(float) * (size_t)N);
+        float* o = (float*)malloc(sizeof(float) * (size_t)N);
+#pragma omp for schedule(dynamic, 1)
+        for (int32_t l = l0; l < l1; ++l) { /* layers are independent here */
+            uint8_t f = 0;
+            for (int32_t k = 0; k < N; ++k) z[k] = 0.0f;
+            eval(l, z, o, ctx);
+            if (row_all_equal(o, N, 0.0f)) f |= 1;
+            for (int32_t k = 0; k < N; ++k) z[k] = ymax;
+            eval(l, z, o, ctx);
+            if (row_all_equal(o, N, ymax)) f |= 2;
+            fixed[l - l0] = f;
+        }
+        free(z);
+        free(o);
+    }
+    return fixed;
+}
+
+static int64_t layers_fast(int32_t N, float ymax, int32_t l0, int32_t l1, int64_t B, const float* Yin, float* Yout,
+                           int32_t nthreads, void (*eval)(int32_t, const float*, float*, const void*),
+                           const void* ctx) {
+    set_threads(nthreads);
+    uint8_t* fixed = fixed_points(N, l0, l1, ymax, eval, ctx);
+    int64_t skipped = 0;
+#pragma omp parallel reduction(+ : skipped)
+    {
+        float* a = (float*)malloc(sizeof(float) * (size_t)N);
+        float* c = (float*)malloc(sizeof(float) * (size_t)N);
+#pragma omp for schedule(dynamic, 4)
+        for (int64_t r = 0; r < B; ++r) {
+            memcpy(a, Yin + r * N, sizeof(float) * (size_t)N);
+            int kind = -1; /* what `a` is: -1 not yet checked, 0 other, 1 all-zero, 2 all-YMAX */
+            for (int32_t l = l0; l < l1; ++l) {
+                const uint8_t f = fixed[l - l0];
+                if (f && kind < 0)
+                    kind = row_all_equal(a, N, 0.0f) ? 1 : (row_all_equal(a, N, ymax) ? 2 : 0);
+                if (kind > 0 && (f & kind)) {
+                    skipped += 1;  /* the layer maps this row to itself: `a` unchanged, `kind` still holds */
+                    continue;
+                }
+                eval(l, a, c, ctx);
+                float* tmp = a; a = c; c = tmp;
+                kind = -1;
+            }
+            memcpy(Yout + r * N, a, sizeof(float) * (size_t)N);
+        }
+        free(a);
+        free(c);
+    }
+    free(fixed);
+    return skipped;
+}
+
+struct csc_ctx { int32_t N; const int64_t* ptr; const int32_t* idx; const float* val; const float* bias; float ymax; };
+static void eval_csc(int32_t l, const float* y, float* y_next, const void* vctx) {
+    const struct csc_ctx* x = (const struct csc_ctx*)vctx;
+    row_layer_f32(x->N, x->ptr + (int64_t)l * (x->N + 1), x->idx, x->val, x->bias + (int64_t)l * x->N, x->ymax, y,
+                  y_next);
+}
+struct circ_ctx { int32_t N, K; const int32_t* nu; const float* w; const float* bias; float ymax; };
+static void eval_circ(int32_t l, const float* y, float* y_next, const void* vctx) {
+    const struct circ_ctx* x = (const struct circ_ctx*)vctx;
+    row_layer_circ_f32(x->N, x->K, x->nu[l], x->w + (int64_t)l * x->K, x->bias + (int64_t)l * x->N, x->ymax, y,
+                       y_next);
+}
+
+int64_t oracle_layers_f32_fast(int32_t N, const int64_t* ptr, const int32_t* idx, const float* val,
+                               const float* bias, float ymax, int32_t l0, int32_t l1,
+                               int64_t B, const float* Yin, float* Yout, int32_t nthreads) {
+    struct csc_ctx x = {N, ptr, idx, val, bias, ymax};
+    return layers_fast(N, ymax, l0, l1, B, Yin, Yout, nthreads, eval_csc, &x);
+}
+
+int64_t oracle_layers_circulant_f32_fast(int32_t N, int32_t K, const int32_t* nu, const float* w,
+                                         const float* bias, float ymax, int32_t l0, int32_t l1, int64_t B,
+                                         const float* Yin, float* Yout, int32_t nthreads) {
+    struct circ_ctx x = {N, K, nu, w, bias, ymax};
+    return layers_fast(N, ymax, l0, l1, B, Yin, Yout, nthreads, eval_circ, &x);
 }
 
 /* Sum downsampling: "divides the original column into n segments, each containing N/n elements

@@ -46,6 +46,22 @@ void oracle_layers_circulant_f32(int32_t N, int32_t K, const int32_t* nu, const 
                                  float ymax, int32_t l0, int32_t l1, int64_t B, const float* Yin, float* Yout,
                                  int32_t nthreads);
 
+/* ---- Exact fast mode of Eq. (1) (used only to make full-size category parity
+ * affordable).  A layer is a pure function of its input row, so a row equal (==) to a row whose
+ * image was already computed has that image.  Two such rows are memoised per layer: the all-zero row
+ * (its fma chains are +0 whatever the signs of its zeros) and the all-YMAX row.  When the image of
+ * the all-zero (all-YMAX) row under layer l is that row again, every all-zero (all-YMAX) row is left
+ * unchanged by layer l and the evaluation is skipped; every other row is evaluated exactly as by
+ * oracle_layers_f32 / oracle_layers_circulant_f32 (same function calls).  Results are identical to
+ * the plain mode (compared with ==; pinned in tests/test_oracle_pins.py).  Returns the number of
+ * skipped row-layer evaluations. */
+int64_t oracle_layers_f32_fast(int32_t N, const int64_t* ptr, const int32_t* idx, const float* val,
+                               const float* bias, float ymax, int32_t l0, int32_t l1,
+                               int64_t B, const float* Yin, float* Yout, int32_t nthreads);
+int64_t oracle_layers_circulant_f32_fast(int32_t N, int32_t K, const int32_t* nu, const float* w,
+                                         const float* bias, float ymax, int32_t l0, int32_t l1, int64_t B,
+                                         const float* Yin, float* Yout, int32_t nthreads);
+
 /* ---- Sum downsampling, Sec. 3.2.1, Fig. 3a PAPER.md:587-596.
  * rows: s x N (the sampled rows).  F: n x s row-major, F[g*s+q] = sum of rows[q][k] over
  * segment g, segments of floor(N/n) elements, last segment takes the remainder (R15).

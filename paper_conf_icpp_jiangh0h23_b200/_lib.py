@@ -23,7 +23,8 @@ KERNEL_AUTO, KERNEL_ELL, KERNEL_CIRC, KERNEL_CIRC_SMEM = 0, 1, 2, 3
 EXPORTED = ["snicit_default_options", "snicit_load_network", "snicit_set_stream", "snicit_infer",
             "snicit_categories", "snicit_stats", "snicit_debug_clustering", "snicit_debug_layer",
             "snicit_layer_is_circulant", "snicit_free_network", "snicit_last_error", "snicit_abi_version",
-            "snicit_layer_profile", "snicit_load_network_circulant", "snicit_infer_packed"]
+            "snicit_layer_profile", "snicit_load_network_circulant", "snicit_infer_packed",
+            "snicit_categories_device"]
 
 
 class Options(ctypes.Structure):
@@ -80,6 +81,8 @@ def load_library(path: str = LIB_PATH):
     L.snicit_infer_packed.restype = i32
     L.snicit_categories.argtypes = [P, P, ctypes.POINTER(i64), i32]
     L.snicit_categories.restype = i32
+    L.snicit_categories_device.argtypes = [P, P, i64]
+    L.snicit_categories_device.restype = i32
     L.snicit_stats.argtypes = [P, ctypes.POINTER(Stats)]
     L.snicit_stats.restype = i32
     L.snicit_layer_profile.argtypes = [P, i32, P, P, P, P]

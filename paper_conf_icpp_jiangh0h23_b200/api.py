@@ -33,6 +33,29 @@ def pack_rows(Y: np.ndarray, one: float = 1.0) -> np.ndarray:
     return np.ascontiguousarray(by).view("<u4").reshape(B, W)
 
 
+def _check_device(x, device: int, what: str) -> None:
+    if _is_cuda_tensor(x) and int(x.device.index) != int(device):
+        raise ValueError(f"{what} is on cuda:{x.device.index}, the network on cuda:{device}")
+
+
+def _out_arg(y_out, B: int, N: int, device: int):
+    """(on_device, pointer) of a caller-owned B x N fp32 C-contiguous output (None -> not materialised).
+    The library writes B*N*4 bytes there, so shape, dtype and layout are checked first."""
+    if y_out is None:
+        return 0, None
+    if _is_cuda_tensor(y_out):
+        import torch
+        if y_out.dtype != torch.float32 or tuple(y_out.shape) != (B, N) or not y_out.is_contiguous():
+            raise ValueError(f"y_out must be a contiguous float32 tensor of shape ({B}, {N})")
+        _check_device(y_out, device, "y_out")
+        return 1, y_out.data_ptr()
+    ya = y_out.numpy() if hasattr(y_out, "numpy") else y_out
+    if not (isinstance(ya, np.ndarray) and ya.dtype == np.float32 and ya.shape == (B, N) and ya.flags.c_contiguous
+            and ya.flags.writeable):
+        raise ValueError(f"host y_out must be a writeable C-contiguous float32 array of shape ({B}, {N})")
+    return 0, ya.ctypes.data
+
+
 class SnicitNetwork:
     """Owns one `snicit_network*` (device copy of W, b + workspace) on `device`.
 
@@ -56,6 +79,7 @@ class SnicitNetwork:
         check(st, "snicit_load_network")
         self._h = h
         self._last_batch = 0
+        self._last_ns = (0, 1)
         self._stream = None
 
     @classmethod
@@ -76,6 +100,7 @@ class SnicitNetwork:
                                                       ctypes.byref(h)), "snicit_load_network_circulant")
         self._h = h
         self._last_batch = 0
+        self._last_ns = (0, 1)
         self._stream = None
         return self
 
@@ -123,28 +148,27 @@ class SnicitNetwork:
         elif opt_kw:
             raise ValueError("pass either options or keyword options")
         if _is_cuda_tensor(y0):
-            assert y0.dtype.__str__() == "torch.float32" and y0.is_contiguous()
+            import torch
+            if y0.dtype != torch.float32 or not y0.is_contiguous() or y0.dim() != 2:
+                raise ValueError("device y0 must be a contiguous 2-D float32 tensor")
+            _check_device(y0, self.device, "y0")
             B = int(y0.shape[0])
             y0_dev, y0p = 1, y0.data_ptr()
         else:
             arr = y0.numpy() if hasattr(y0, "numpy") else y0
-            if not (isinstance(arr, np.ndarray) and arr.dtype == np.float32 and arr.flags.c_contiguous):
-                raise ValueError("host y0 must be a C-contiguous float32 array")
+            if not (isinstance(arr, np.ndarray) and arr.dtype == np.float32 and arr.flags.c_contiguous
+                    and arr.ndim == 2):
+                raise ValueError("host y0 must be a C-contiguous 2-D float32 array")
             B = int(arr.shape[0])
             y0_dev, y0p = 0, arr.ctypes.data
-        if B and int(y0.shape[1]) != self.N:
+        if int(y0.shape[1]) != self.N:
             raise ValueError(f"y0 must be B x {self.N}")
-        if y_out is None:
-            yo_dev, yop = 0, None
-        elif _is_cuda_tensor(y_out):
-            yo_dev, yop = 1, y_out.data_ptr()
-        else:
-            ya = y_out.numpy() if hasattr(y_out, "numpy") else y_out
-            yo_dev, yop = 0, ya.ctypes.data
+        yo_dev, yop = _out_arg(y_out, B, self.N, self.device)
         st = self._lib.snicit_infer(self._h, y0p, B, y0_dev, int(row_offset), int(t), int(s), ctypes.byref(options),
                                     yop, yo_dev)
         check(st, "snicit_infer")
         self._last_batch = B
+        self._last_ns = (self.N if options.n_segments == 0 else int(options.n_segments), int(s))
         return y_out
 
     def infer_packed(self, bits, t: int, s: int = 32, options: Optional[Options] = None, y_out=None,
@@ -157,25 +181,23 @@ class SnicitNetwork:
             raise ValueError("pass either options or keyword options")
         W = (self.N + 31) // 32
         if _is_cuda_tensor(bits):
-            assert bits.element_size() == 4 and bits.is_contiguous()
+            if bits.element_size() != 4 or not bits.is_contiguous() or bits.dim() != 2:
+                raise ValueError("device bits must be a contiguous 2-D tensor of 32-bit words")
+            _check_device(bits, self.device, "bits")
             B, dev, bp = int(bits.shape[0]), 1, bits.data_ptr()
         else:
             arr = bits.numpy() if hasattr(bits, "numpy") else bits
-            if not (isinstance(arr, np.ndarray) and arr.dtype.itemsize == 4 and arr.flags.c_contiguous):
-                raise ValueError("host bits must be a C-contiguous 32-bit array")
+            if not (isinstance(arr, np.ndarray) and arr.dtype.itemsize == 4 and arr.flags.c_contiguous
+                    and arr.ndim == 2):
+                raise ValueError("host bits must be a C-contiguous 2-D 32-bit array")
             B, dev, bp = int(arr.shape[0]), 0, arr.ctypes.data
-        if B and int(bits.shape[1]) != W:
+        if int(bits.shape[1]) != W:
             raise ValueError(f"bits must be B x {W}")
-        if y_out is None:
-            yo_dev, yop = 0, None
-        elif _is_cuda_tensor(y_out):
-            yo_dev, yop = 1, y_out.data_ptr()
-        else:
-            ya = y_out.numpy() if hasattr(y_out, "numpy") else y_out
-            yo_dev, yop = 0, ya.ctypes.data
+        yo_dev, yop = _out_arg(y_out, B, self.N, self.device)
         check(self._lib.snicit_infer_packed(self._h, bp, B, dev, float(one), int(row_offset), int(t), int(s),
                                             ctypes.byref(options), yop, yo_dev), "snicit_infer_packed")
         self._last_batch = B
+        self._last_ns = (self.N if options.n_segments == 0 else int(options.n_segments), int(s))
         return y_out
 
     def categories(self) -> np.ndarray:
@@ -186,6 +208,17 @@ class SnicitNetwork:
         if n.value:
             check(self._lib.snicit_categories(self._h, out.ctypes.data, ctypes.byref(n), 0), "snicit_categories")
         return out[:n.value]
+
+    def categories_device(self, out) -> None:
+        """snicit_categories_device: out (CUDA int64 tensor of 1 + capacity) <- [count, ids...], queued on
+        the handle's stream (no host synchronisation)."""
+        import torch
+        if not (_is_cuda_tensor(out) and out.dtype == torch.int64 and out.is_contiguous() and out.dim() == 1
+                and out.numel() >= 1):
+            raise ValueError("out must be a contiguous 1-D int64 CUDA tensor of 1 + capacity entries")
+        _check_device(out, self.device, "out")
+        check(self._lib.snicit_categories_device(self._h, out.data_ptr(), int(out.numel()) - 1),
+              "snicit_categories_device")
 
     def num_categories(self) -> int:
         n = ctypes.c_int64(0)
@@ -209,9 +242,15 @@ class SnicitNetwork:
         k = n.value
         return dict(ms=ms[:k].copy(), rows=rows[:k].copy(), bytes=by[:k].copy())
 
-    def debug_clustering(self, n_segments: int = 16, s: int = 32) -> dict:
+    def debug_clustering(self, n_segments: Optional[int] = None, s: Optional[int] = None) -> dict:
+        """Clustering state of the last infer.  The buffers are sized from that infer's n and s (the
+        arguments are accepted for compatibility and must match them if given)."""
         B = self._last_batch
-        n = self.N if n_segments == 0 else n_segments
+        n_last, s_last = self._last_ns
+        if (n_segments is not None and (self.N if n_segments == 0 else n_segments) != n_last) or \
+                (s is not None and s != s_last):
+            raise ValueError(f"last infer used n={n_last}, s={s_last}")
+        n, s = n_last, s_last
         cent = np.empty(max(s, 1), np.int32)
         ncent = ctypes.c_int32(0)
         M = np.empty(max(B, 1), np.int32)

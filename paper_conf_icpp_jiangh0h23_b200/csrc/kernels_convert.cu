@@ -497,4 +497,23 @@ cudaError_t launch_unpack_bits(const uint32_t* bits, int R, int N, float one, fl
     return cudaGetLastError();
 }
 
+// Category export (multi-GPU all-gather): out[0] = total (int64), out[1 + i] = offset +
+// catlist[i] for i < min(total, cap) -- device to device, no host synchronisation
+__global__ void export_categories_kernel(const int* __restrict__ catlist, const int* __restrict__ count,
+                                         long long offset, long long* __restrict__ out, long long cap) {
+    const long long n = *count;
+    const long long m = n < cap ? n : cap;
+    if (blockIdx.x == 0 && threadIdx.x == 0) out[0] = n;
+    for (long long i = (long long)blockIdx.x * blockDim.x + threadIdx.x; i < m; i += (long long)gridDim.x * blockDim.x)
+        out[1 + i] = offset + catlist[i];
+}
+cudaError_t launch_export_categories(const int* catlist, const int* count, long long offset, long long* out,
+                                     long long cap, cudaStream_t st) {
+    long long grid = (cap + 255) / 256;
+    if (grid > 1024) grid = 1024;
+    if (grid < 1) grid = 1;
+    export_categories_kernel<<<(int)grid, 256, 0, st>>>(catlist, count, offset, out, cap);
+    return cudaGetLastError();
+}
+
 }  // namespace snicit

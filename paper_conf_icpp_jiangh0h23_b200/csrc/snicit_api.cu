@@ -58,6 +58,23 @@ struct DevBuf {
     }
 };
 
+// Every entry point that touches the GPU switches to the handle's device and restores the caller's
+// current device on return (the library never leaves the caller's device changed).
+struct DeviceGuard {
+    int prev = -1;
+    cudaError_t status = cudaSuccess;
+    explicit DeviceGuard(int dev) {
+        if (cudaGetDevice(&prev) != cudaSuccess) prev = -1;
+        if (dev >= 0) status = cudaSetDevice(dev);
+    }
+    ~DeviceGuard() {
+        if (prev >= 0) cudaSetDevice(prev);
+    }
+};
+
+// device pointers the kernels access with 16-byte vector / TMA bulk operations
+inline bool misaligned16(const void* p) { return p && (reinterpret_cast<uintptr_t>(p) & 15u) != 0; }
+
 // device counters (one int each)
 enum Counter {
     CNT_LIVE0 = 0, CNT_LIVE1, CNT_LIVE2, CNT_ORD, CNT_RES0, CNT_RES1, CNT_NCENT, CNT_SEFF, CNT_ALL, CNT_NCAT,
@@ -278,7 +295,8 @@ int32_t snicit_abi_version(void) { return SNICIT_ABI_VERSION; }
 
 void snicit_free_network(snicit_network* net) {
     if (!net) return;
-    if (cudaSetDevice(net->device) == cudaSuccess && net->stream) cudaStreamSynchronize(net->stream);
+    DeviceGuard dg(net->device);
+    if (dg.status == cudaSuccess && net->stream) cudaStreamSynchronize(net->stream);
     net->idx16_d.release();
     net->idx32_d.release();
     net->val_d.release();
@@ -331,6 +349,7 @@ snicit_status snicit_load_network(int32_t N, int32_t L, snicit_format fmt, const
                                   snicit_network** out) {
     if (!out) return fail(SNICIT_E_INVALID_ARG, "out is NULL");
     *out = nullptr;
+    DeviceGuard dg(-1);  // net_device_init switches to cuda_device; the caller's device is restored
     if (N < 1 || L < 1) return fail(SNICIT_E_INVALID_ARG, "n_neurons and n_layers must be >= 1");
     if (!ptr || !bias) return fail(SNICIT_E_INVALID_ARG, "ptr/bias NULL");
     if (!(ymax > 0.0f) || std::isnan(ymax)) return fail(SNICIT_E_INVALID_ARG, "ymax must be > 0");
@@ -527,6 +546,7 @@ snicit_status snicit_load_network_circulant(int32_t N, int32_t L, const int32_t*
                                             snicit_network** out) {
     if (!out) return fail(SNICIT_E_INVALID_ARG, "out is NULL");
     *out = nullptr;
+    DeviceGuard dg(-1);
     if (N < 1 || L < 1 || K < 1) return fail(SNICIT_E_INVALID_ARG, "n_neurons, n_layers, K must be >= 1");
     if (!nu || !w || !bias) return fail(SNICIT_E_INVALID_ARG, "nu/w/bias NULL");
     if (!(ymax > 0.0f) || std::isnan(ymax)) return fail(SNICIT_E_INVALID_ARG, "ymax must be > 0");
@@ -666,15 +686,15 @@ static cudaError_t ensure_workspace(snicit_network* net, int64_t R, int s, int n
     if ((e = net->cscratch.ensure((size_t)compact_scratch_ints((int)rows))) != cudaSuccess) return e;
     if (net->segflag.n < rows) {
         if ((e = net->segflag.ensure(rows)) != cudaSuccess) return e;
-        if ((e = cudaMemset(net->segflag.p, 0, rows)) != cudaSuccess) return e;
+        if ((e = cudaMemsetAsync(net->segflag.p, 0, rows, net->stream)) != cudaSuccess) return e;
     }
     if (net->cmin.n < rows) {
         if ((e = net->cmin.ensure(rows)) != cudaSuccess) return e;
-        if ((e = cudaMemset(net->cmin.p, 0xff, rows * sizeof(unsigned))) != cudaSuccess) return e;
+        if ((e = cudaMemsetAsync(net->cmin.p, 0xff, rows * sizeof(unsigned), net->stream)) != cudaSuccess) return e;
     }
     if (net->cmax.n < rows) {
         if ((e = net->cmax.ensure(rows)) != cudaSuccess) return e;
-        if ((e = cudaMemset(net->cmax.p, 0, rows * sizeof(unsigned))) != cudaSuccess) return e;
+        if ((e = cudaMemsetAsync(net->cmax.p, 0, rows * sizeof(unsigned), net->stream)) != cudaSuccess) return e;
     }
     for (auto* b : {&net->clist, &net->clayer})
         if ((e = b->ensure(rows)) != cudaSuccess) return e;
@@ -683,7 +703,7 @@ static cudaError_t ensure_workspace(snicit_network* net, int64_t R, int s, int n
     if ((e = net->rval.ensure(rows)) != cudaSuccess) return e;
     if (net->rowctr.n < rows) {
         if ((e = net->rowctr.ensure(rows)) != cudaSuccess) return e;
-        if ((e = cudaMemset(net->rowctr.p, 0, rows * sizeof(int))) != cudaSuccess) return e;
+        if ((e = cudaMemsetAsync(net->rowctr.p, 0, rows * sizeof(int), net->stream)) != cudaSuccess) return e;
     }
     return cudaSuccess;
 }
@@ -737,6 +757,9 @@ static snicit_status infer_core(snicit_network* net, const float* y0, int64_t ba
     if (t < 0) return fail(SNICIT_E_INVALID_ARG, "threshold_layer < 0");
     if (s < 1) return fail(SNICIT_E_INVALID_ARG, "centroid_count < 1");
     if (row_offset < 0) return fail(SNICIT_E_INVALID_ARG, "row_offset < 0");
+    if ((y0_on_device && misaligned16(y0)) || (y_out_on_device && misaligned16(y_out)) ||
+        (y0_mode == 3 && misaligned16(bits)))
+        return fail(SNICIT_E_INVALID_ARG, "device y0 / y_out / bits must be 16-byte aligned");
     snicit_options opt;
     if (opt_in)
         opt = *opt_in;
@@ -760,7 +783,8 @@ static snicit_status infer_core(snicit_network* net, const float* y0, int64_t ba
     const int tt = std::min(t, L);
     const int n_seg = opt.n_segments == 0 ? N : opt.n_segments;
     const int ne_interval = opt.ne_interval > 0 ? opt.ne_interval : 64;
-    CUDA_TRY(cudaSetDevice(net->device));
+    DeviceGuard dg(net->device);
+    CUDA_TRY(dg.status);
     CUDA_TRY(ensure_workspace(net, R, s, n_seg));
     cudaStream_t st = net->stream;
     int64_t launches = y0_mode == 2 ? 1 : 0;  // + the unpack kernel of snicit_infer_packed (mode 2)
@@ -1200,6 +1224,9 @@ static snicit_status infer_core(snicit_network* net, const float* y0, int64_t ba
         cudaEventElapsedTime(&ms, net->ev[0], net->ev[5]);
         net->stats.t_total_ms = ms;
     }
+    // a host buffer is involved (y0 read by an async H2D copy, y_out filled by an async D2H copy):
+    // return only when the caller may read / reuse it
+    if (y0_mode == 1 || (y_out && !y_out_on_device)) CUDA_TRY(cudaStreamSynchronize(st));
     return SNICIT_OK;
 }
 
@@ -1217,10 +1244,12 @@ snicit_status snicit_infer_packed(snicit_network* net, const uint32_t* y0_bits, 
     if (batch > 0 && !y0_bits) return fail(SNICIT_E_INVALID_ARG, "y0_bits NULL");
     if (!std::isfinite(one_value)) return fail(SNICIT_E_INVALID_ARG, "one_value not finite");
     if (t < 0 || s < 1) return fail(SNICIT_E_INVALID_ARG, "threshold_layer < 0 or centroid_count < 1");
+    if (bits_on_device && misaligned16(y0_bits)) return fail(SNICIT_E_INVALID_ARG, "device y0_bits must be 16-byte aligned");
     const int N = net->N;
     const int R = (int)batch;
     const size_t W = ((size_t)N + 31) / 32;
-    CUDA_TRY(cudaSetDevice(net->device));
+    DeviceGuard dg(net->device);
+    CUDA_TRY(dg.status);
     const int n_seg = (opt && opt->n_segments > 0 && opt->n_segments <= N) ? opt->n_segments : N;
     CUDA_TRY(ensure_workspace(net, R, s, n_seg));
     const uint32_t* bits = y0_bits;
@@ -1285,13 +1314,16 @@ snicit_status snicit_infer_packed(snicit_network* net, const uint32_t* y0_bits, 
     }
     // later work on the handle's stream (and the next upload) is ordered after this upload
     if (streamed) CUDA_TRY(cudaStreamWaitEvent(net->stream, net->cev[1], 0));
+    // host bits are read by asynchronous copies: return once they are consumed
+    if (stt == SNICIT_OK && !bits_on_device && R > 0) CUDA_TRY(cudaStreamSynchronize(net->stream));
     return stt;
 }
 
 snicit_status snicit_categories(snicit_network* net, int64_t* rows, int64_t* count, int32_t rows_on_device) {
     if (!net || !count) return fail(SNICIT_E_INVALID_ARG, "net/count NULL");
     if (!net->have_result) return fail(SNICIT_E_STATE, "no inference result");
-    CUDA_TRY(cudaSetDevice(net->device));
+    DeviceGuard dg(net->device);
+    CUDA_TRY(dg.status);
     int total = 0;
     CUDA_TRY(read_counter(net, CNT_NCAT, &total));
     if (!rows) {
@@ -1314,10 +1346,23 @@ snicit_status snicit_categories(snicit_network* net, int64_t* rows, int64_t* cou
     return SNICIT_OK;
 }
 
+snicit_status snicit_categories_device(snicit_network* net, int64_t* out, int64_t capacity) {
+    if (!net || !out) return fail(SNICIT_E_INVALID_ARG, "net/out NULL");
+    if (capacity < 0) return fail(SNICIT_E_INVALID_ARG, "capacity < 0");
+    if (reinterpret_cast<uintptr_t>(out) & 7u) return fail(SNICIT_E_INVALID_ARG, "out must be 8-byte aligned");
+    if (!net->have_result) return fail(SNICIT_E_STATE, "no inference result");
+    DeviceGuard dg(net->device);
+    CUDA_TRY(dg.status);
+    CUDA_TRY(launch_export_categories(net->catlist.p, net->counters.p + CNT_NCAT, (long long)net->last_offset,
+                                      reinterpret_cast<long long*>(out), (long long)capacity, net->stream));
+    return SNICIT_OK;
+}
+
 snicit_status snicit_stats(snicit_network* net, snicit_stats_t* out) {
     if (!net || !out) return fail(SNICIT_E_INVALID_ARG, "net/out NULL");
     if (!net->have_result) return fail(SNICIT_E_STATE, "no inference result");
-    CUDA_TRY(cudaSetDevice(net->device));
+    DeviceGuard dg(net->device);
+    CUDA_TRY(dg.status);
     int v = 0;
     CUDA_TRY(read_counter(net, net->live_counter, &v));
     net->stats.live_at_t = v;
@@ -1363,7 +1408,8 @@ snicit_status snicit_layer_profile(snicit_network* net, int32_t max, double* ms,
                                    int32_t* n) {
     if (!net) return fail(SNICIT_E_INVALID_ARG, "net NULL");
     if (!net->have_result) return fail(SNICIT_E_STATE, "no inference result");
-    CUDA_TRY(cudaSetDevice(net->device));
+    DeviceGuard dg(net->device);
+    CUDA_TRY(dg.status);
     CUDA_TRY(cudaStreamSynchronize(net->stream));
     const int cnt = std::min<int>(std::max(max, 0), net->prof_layers);
     std::vector<int> h((size_t)std::max(cnt, 1));
@@ -1399,7 +1445,8 @@ snicit_status snicit_debug_clustering(snicit_network* net, int32_t* cent, int32_
                                       double* F, int32_t* n_sampled, uint8_t* live_t) {
     if (!net) return fail(SNICIT_E_INVALID_ARG, "net NULL");
     if (!net->have_result) return fail(SNICIT_E_STATE, "no inference result");
-    CUDA_TRY(cudaSetDevice(net->device));
+    DeviceGuard dg(net->device);
+    CUDA_TRY(dg.status);
     CUDA_TRY(cudaStreamSynchronize(net->stream));
     const int R = (int)net->last_batch;
     int C = 0, se = 0;
@@ -1432,7 +1479,8 @@ snicit_status snicit_debug_layer(snicit_network* net, int32_t layer, const float
     if (kernel < 0 || kernel > SNICIT_KERNEL_CIRC_SMEM) return fail(SNICIT_E_INVALID_ARG, "bad kernel");
     if ((kernel == SNICIT_KERNEL_CIRC || kernel == SNICIT_KERNEL_CIRC_SMEM) && net->plan[layer].kind == 0)
         return fail(SNICIT_E_UNSUPPORTED, "layer is not circulant");
-    CUDA_TRY(cudaSetDevice(net->device));
+    DeviceGuard dg(net->device);
+    CUDA_TRY(dg.status);
     CUDA_TRY(ensure_workspace(net, rows, 1, 1));
     CUDA_TRY(launch_iota(net->list0.p, (int)rows, net->counters.p + CNT_LIVE0, net->stream));
     LayerArgs a = layer_args(net, layer, kernel == SNICIT_KERNEL_ELL);

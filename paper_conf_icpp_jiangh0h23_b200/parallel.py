@@ -1,9 +1,17 @@
 """Row sharding and the one collective of the path.
 
-Rows of the batch are independent (Eq. 1 acts per sample; clustering runs per shard), so each rank
-infers a contiguous block of rows with replicated weights.  The only exchange is the final
-all-gather of the category ids: counts first, then ids padded to the max count
-(torch.distributed: NCCL on GPUs, gloo in the CPU tests).
+Rows of the batch are independent (Eq. 1 acts per sample; clustering runs per shard), so
+each rank infers a contiguous block of rows with replicated weights.  The only exchange is the final
+all-gather of the category ids (torch.distributed: NCCL over NVLink on GPUs, gloo in the CPU tests).
+
+Two forms:
+* ``allgather_categories_padded`` -- the production form: every rank exports [count, ids...] into a
+  fixed-size device buffer (``snicit_categories_device``, no host round trip, capacity = the largest
+  shard) and ONE all_gather of those buffers leaves the whole category set on every rank.  No host
+  synchronisation is needed inside the step; ``assemble_categories`` turns the gathered buffers into the
+  ascending global list when the caller wants it.
+* ``allgather_categories`` -- variable-length ids (counts first, then ids padded to the max count), for
+  callers that already hold a host/device id list.
 """
 from __future__ import annotations
 
@@ -15,6 +23,11 @@ def shard_rows(batch: int, world: int, rank: int) -> Tuple[int, int]:
     base, rem = divmod(batch, world)
     start = rank * base + min(rank, rem)
     return start, start + base + (1 if rank < rem else 0)
+
+
+def shard_capacity(batch: int, world: int) -> int:
+    """Largest shard of `batch` rows over `world` ranks (the padded all-gather's capacity)."""
+    return -(-batch // world) if world > 0 else batch
 
 
 def allgather_categories(local_ids, group=None):
@@ -36,3 +49,29 @@ def allgather_categories(local_ids, group=None):
     parts = [torch.empty_like(padded) for _ in range(world)]
     dist.all_gather(parts, padded, group=group)
     return torch.cat([p[:c] for p, c in zip(parts, cnt)])
+
+
+def allgather_categories_padded(local_buf, group=None):
+    """local_buf: int64 tensor [1 + cap] = [count, ids...] (``SnicitNetwork.categories_device``).
+    Returns the gathered [world, 1 + cap] tensor (same device): row r = rank r's [count, ids...].
+    One collective, no host synchronisation."""
+    import torch
+    import torch.distributed as dist
+
+    world = dist.get_world_size(group)
+    out = torch.empty((world, local_buf.numel()), dtype=local_buf.dtype, device=local_buf.device)
+    dist.all_gather_into_tensor(out, local_buf, group=group)
+    return out
+
+
+def assemble_categories(gathered):
+    """[world, 1 + cap] gathered buffers -> ascending global category ids (int64, same device).
+    Reads the counts (one small device->host copy)."""
+    import torch
+
+    counts = gathered[:, 0].tolist()
+    cap = gathered.shape[1] - 1
+    if any(c > cap for c in counts):
+        raise ValueError("a shard has more categories than the buffer capacity")
+    parts = [gathered[r, 1:1 + int(c)] for r, c in enumerate(counts)]
+    return torch.cat(parts) if parts else gathered.new_empty(0)

@@ -35,7 +35,7 @@ def test_header_symbols_exported(lib):
 
 
 def test_abi_version_and_defaults(lib):
-    assert lib.snicit_abi_version() == 3
+    assert lib.snicit_abi_version() == 4
     o = _lib.default_options()
     # SDGC defaults, P:1038 / P:1138
     assert o.n_segments == 16 and abs(o.eta - 0.03) < 1e-7 and abs(o.eps - 0.03) < 1e-7

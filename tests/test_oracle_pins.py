@@ -386,3 +386,63 @@ def test_circulant_form_equals_csc():
         assert c.nnz == net.nnz
         Y0 = sdgc.gen_inputs(N, 7) * np.float32(3.3)
         assert np.array_equal(oracle.layers_circulant_f32(c, Y0), oracle.layers_f32(net, Y0))
+
+
+# ---------------------------------------------------------------- exact fast mode
+
+def _same(a, b):
+    """Equal under == (reading R19: +0 == -0) -- the comparison every parity test uses."""
+    return a.shape == b.shape and bool(np.all(a == b))
+
+
+@pytest.mark.parametrize("N,L,B", [(1024, 120, 2000)])
+def test_fast_oracle_equals_plain_c1(N, L, B):
+    """Fast mode == plain Eq. (1) on the whole C1 workload (SDGC 1024 x 120, B = 2000), and it skips most
+    row-layers there (rows collapse to all-0 / all-32)."""
+    net = sdgc.gen_network(N, L, "radix")
+    Y0 = sdgc.gen_inputs(N, B)
+    plain = oracle.layers_f32(net, Y0)
+    fast, skipped = oracle.layers_f32_fast(net, Y0, return_skipped=True)
+    assert _same(fast, plain)
+    assert skipped > 0.5 * B * L
+
+
+def test_fast_oracle_equals_plain_c2_rows_and_compact_form():
+    """C2 (4096 x 480) on a row sample, through the CSC and the compact circulant forms."""
+    cn = sdgc.gen_circulant(4096, 480)
+    rs = np.random.RandomState(11)
+    rows = np.sort(rs.choice(60000, 48, replace=False))
+    Y0 = np.concatenate([sdgc.gen_inputs(4096, 1, row0=int(r)) for r in rows])
+    plain = oracle.layers_circulant_f32(cn, Y0)
+    assert _same(oracle.layers_f32_fast(cn, Y0), plain)
+    assert _same(oracle.layers_f32_fast(cn.to_network(), Y0), plain)
+
+
+def test_fast_oracle_degenerate_rows_and_non_fixed_layers():
+    """All-zero, all-YMAX, constant and random rows; layers where the zero row is NOT a fixed point
+    (positive biases) and where YMAX is not (negative weights): fast == plain, bit for bit under ==."""
+    N, L = 64, 9
+    net = tiny_random_net(N, L, 12, 5)
+    rs = np.random.RandomState(2)
+    Y0 = rs.uniform(0, 32, size=(40, N)).astype(np.float32)
+    Y0[0::5] = 0.0
+    Y0[1::5] = 32.0
+    Y0[2::5] = -0.0
+    Y0[3::5] = 7.25
+    assert _same(oracle.layers_f32_fast(net, Y0), oracle.layers_f32(net, Y0))
+    # SDGC layers with one positive-bias layer in the middle (zero rows wake up there)
+    c = sdgc.gen_circulant(1024, 12)
+    c.bias[5 * 1024:6 * 1024] = 0.25
+    Y1 = sdgc.gen_inputs(1024, 300)
+    Y1[::3] = 0.0
+    assert _same(oracle.layers_f32_fast(c, Y1), oracle.layers_circulant_f32(c, Y1))
+    out6 = oracle.layers_f32_fast(c, Y1, 0, 6)
+    assert _same(out6, oracle.layers_circulant_f32(c, Y1, 0, 6))
+    assert (out6[::3] == np.float32(0.25)).all()  # the zero rows were evaluated by the positive-bias layer
+
+
+def test_fast_oracle_equals_plain_c3_rows():
+    """C3 geometry (16384 x 1920, compact form) on a few rows: fast == plain."""
+    cn = sdgc.gen_circulant(16384, 1920)
+    Y0 = np.concatenate([sdgc.gen_inputs(16384, 1, row0=r) for r in (0, 1, 7, 59999)])
+    assert _same(oracle.layers_f32_fast(cn, Y0), oracle.layers_circulant_f32(cn, Y0))
