@@ -1,22 +1,31 @@
 #!/usr/bin/env python
 """SNICIT hot-path benchmark: SDGC inference edges/s on B200 (BASELINE.json metric).
 
-    python bench.py [--gpus N] [--steps K] [--warmup W] [--config C2] [--impl snicit|reference]
+    python bench.py [--gpus N] [--steps K] [--warmup W] [--config C3] [--impl snicit|reference]
 
 A step = one whole SNICIT inference (all SURVEY 8(a) rows: pre-convergence layers, conversion,
-post-convergence layers, recovery, categories) over one batch.  N=1 workload: config C2 (SDGC 4096
-neurons x 480 layers, batch 60,000, t=30, s=32, n=16, eta=eps=0.03), synthetic inputs (DESIGN.md
-section 5).  N>1 (torchrun, one rank per GPU, NCCL): weak scaling -- every rank infers its own 60,000-row
-batch (global row ids offset by rank), the category ids are all-gathered; value = rows of all ranks x
-connections / max-over-ranks step time.
+post-convergence layers, recovery, category set) over one batch.  The N = 1 workload is config C3
+(SDGC 16384 neurons x 1920 layers, batch 60,000, t = 30, s = 32, n = 16, eta = eps = 0.03: the config
+BASELINE.json quotes the metric "at 1/2/4/8 B200" on), synthetic inputs.
+
+N > 1: one rank per GPU over NCCL.  `--gpus N` without a torchrun environment re-launches itself under
+torch.distributed.run (127.0.0.1).  Default **strong** scaling: the one 60,000-row batch is
+sharded in contiguous row blocks (B/G rows per rank, global ids by row_offset), weights replicated,
+clustering per shard; the only collective is one all_gather of the per-rank category buffers, exported
+on the device (snicit_categories_device, no host round trip).  `--scaling weak`: every rank its own batch.
 
 value: device-resident inputs (Y0 already in HBM), CUDA events around exactly K steps on the stream the
-library launches on, barrier + synchronize on both sides.  Inputs (983 MB) are larger than L2 (126 MB), so
-no explicit L2 flush.  e2e: the same metric through the C ABI with host (pinned) buffers: H2D of Y0 and D2H
-of Y(L) + categories inside the timed region.
+library launches on, barrier + synchronize on both sides, max over ranks.  Inputs (3.9 GB at C3) exceed
+L2 (126 MB): no flush needed.  e2e: the same metric through snicit_infer with pinned HOST
+fp32 rows (H2D inside the call, streamed under the pre phase) and the category set read back to the host
+(D2H); e2e_packed: the same through snicit_infer_packed (binary inputs as a bitmap).
+
+Extra keys (N = 1): `residue` -- the method's conversion / residue kernels in a residue-heavy regime
+(C2, t = 10) with their rooflines; `general_csc` -- the general (non-circulant) CSC path (C2 "perm"
+weights) with the ELL layer kernel's HBM roofline.
 
 --impl reference: the CPU oracle (plain Eq. 1, oracle/) timed on the host cores on a bounded row sample of
-the same workload (rank 0 only).
+the same workload (rank 0 only; other ranks exit 0).
 """
 from __future__ import annotations
 
@@ -39,13 +48,13 @@ METRIC = "SDGC inference edges/sec at 1/2/4/8 B200; % of HBM roofline"
 UNIT = "edges/s"
 
 
-def parse():
+def parse(argv=None):
     p = argparse.ArgumentParser()
     p.add_argument("--gpus", type=int, default=1)
     p.add_argument("--steps", type=int, default=5)
     p.add_argument("--warmup", type=int, default=3)
     p.add_argument("--impl", choices=["snicit", "reference"], default="snicit")
-    p.add_argument("--config", default="C2", choices=["C1", "C2", "C3", "C4", "C5"])
+    p.add_argument("--config", default="C3", choices=["C1", "C2", "C3", "C4", "C5"])
     p.add_argument("--mode", default="radix", choices=["radix", "perm", "random"])
     p.add_argument("--t", type=int, default=None)
     p.add_argument("--s", type=int, default=None)
@@ -53,46 +62,56 @@ def parse():
     p.add_argument("--load", default="auto", choices=["auto", "csc", "compact"],
                    help="network ABI: explicit CSC (snicit_load_network) or compact circulant form; auto = "
                         "compact for radix nets with N >= 16384 (C3/C4 CSC is 8-32 GB)")
-    p.add_argument("--scaling", default="weak", choices=["weak", "strong"])
-    p.add_argument("--batch", type=int, default=None, help="override rows per rank (weak) / global (strong)")
+    p.add_argument("--scaling", default="strong", choices=["weak", "strong"])
+    p.add_argument("--batch", type=int, default=None, help="override rows (strong: global, weak: per rank)")
     p.add_argument("--no-e2e", action="store_true")
     p.add_argument("--no-cpu-baseline", action="store_true")
     p.add_argument("--no-uncompressed", action="store_true")
+    p.add_argument("--no-residue", action="store_true", help="skip the residue-regime study (C2, t = 10)")
+    p.add_argument("--no-general", action="store_true", help="skip the general-CSC study (C2 perm)")
+    p.add_argument("--residue-t", type=int, default=10)
     p.add_argument("--pre-fused", type=int, default=1, choices=[0, 1, 2],
                    help="options.pre_fused: 1 = row-resident pre phase (default), 2 = without the constant-row "
                         "shortcut, 0 = one launch per layer")
     p.add_argument("--no-variants", action="store_true", help="skip the pre_fused = 2 / 0 roofline variants")
     p.add_argument("--cpu-seconds", type=float, default=15.0, help="target CPU work of the oracle sample")
-    return p.parse_args()
+    p.add_argument("--quick", action="store_true", help="value only (no e2e/uncompressed/variants/studies)")
+    a = p.parse_args(argv)
+    if a.quick:
+        a.no_e2e = a.no_cpu_baseline = a.no_uncompressed = a.no_residue = a.no_general = a.no_variants = True
+    return a
 
 
-def config_params(args):
-    c = dict(sdgc.CONFIGS[args.config])
-    if args.config == "C5":
+def config_params(args, config=None, t=None):
+    config = config or args.config
+    c = dict(sdgc.CONFIGS[config])
+    if config == "C5":
         snic = dict(t=sdgc.medium_t(c["L"]), s=128, n=0)
     else:
         snic = dict(t=30, s=32, n=16)
-    if args.t is not None:
+    if t is not None:
+        snic["t"] = t
+    elif args.t is not None:
         snic["t"] = args.t
     if args.s is not None:
         snic["s"] = args.s
-    if args.batch is not None:
+    if args.batch is not None and config == args.config:
         c["B"] = args.batch
     return c, snic
 
 
-def use_compact(args, c):
-    if args.config == "C5" or args.mode != "radix":
+def use_compact(config, mode, load, c):
+    if config == "C5" or mode != "radix":
         return False
-    return args.load == "compact" or (args.load == "auto" and c["N"] >= 16384)
+    return load == "compact" or (load == "auto" and c["N"] >= 16384)
 
 
-def make_network(args, c):
-    if args.config == "C5":
+def make_network(config, mode, load, c):
+    if config == "C5":
         return sdgc.gen_medium_network(c["N"], c["L"])
-    if use_compact(args, c):
+    if use_compact(config, mode, load, c):
         return sdgc.gen_circulant(c["N"], c["L"])
-    return sdgc.gen_network(c["N"], c["L"], args.mode)
+    return sdgc.gen_network(c["N"], c["L"], mode)
 
 
 def oracle_layers(oracle, net, Y, nthreads=0):
@@ -101,8 +120,8 @@ def oracle_layers(oracle, net, Y, nthreads=0):
     return oracle.layers_f32(net, Y, nthreads=nthreads)
 
 
-def make_inputs(args, c, B, row0):
-    if args.config == "C5":
+def make_inputs(config, c, B, row0):
+    if config == "C5":
         return sdgc.gen_medium_inputs(c["N"], B, row0=row0)
     return sdgc.gen_inputs(c["N"], B, row0=row0)
 
@@ -134,10 +153,11 @@ class ClockSampler:
     def start(self):
         try:
             self.proc = subprocess.Popen(["nvidia-smi", "-i", str(self.index), f"--query-gpu={self.Q}",
-                                          "--format=csv,noheader,nounits", "-lms", "200"],
+                                          "--format=csv,noheader,nounits", "-lms", "100"],
                                          stdout=subprocess.PIPE, stderr=subprocess.DEVNULL, text=True)
             self.th = threading.Thread(target=self._read, daemon=True)
             self.th.start()
+            time.sleep(0.3)  # the sampler is running before the timed region starts
         except (OSError, FileNotFoundError):
             self.proc = None
 
@@ -148,13 +168,13 @@ class ClockSampler:
     def stop(self):
         if self.proc is None:
             return None
-        time.sleep(0.25)
+        time.sleep(0.15)
         self.proc.terminate()
         try:
             self.proc.wait(timeout=5)
         except subprocess.TimeoutExpired:
             self.proc.kill()
-        sm, mx, reasons = [], 0, set()
+        sm, mx, reasons, pw = [], 0, set(), []
         names = ["hw_slowdown", "hw_thermal_slowdown", "sw_thermal_slowdown", "sw_power_cap"]
         for ln in self.lines:
             parts = [p.strip() for p in ln.split(",")]
@@ -163,6 +183,7 @@ class ClockSampler:
             try:
                 sm.append(float(parts[0]))
                 mx = max(mx, float(parts[1]))
+                pw.append(float(parts[2]))
             except ValueError:
                 continue
             for nm, v in zip(names, parts[4:8]):
@@ -170,15 +191,15 @@ class ClockSampler:
                     reasons.add(nm)
         if not sm:
             return None
-        return {"sm_mhz": float(np.median(sm)), "sm_max_mhz": mx, "reasons": sorted(reasons), "samples": len(sm)}
+        return {"sm_mhz": float(np.median(sm)), "sm_max_mhz": mx, "reasons": sorted(reasons), "samples": len(sm),
+                "power_w_max": max(pw) if pw else None}
 
 
-def committed_traffic(config: str):
-    """Mean DRAM bytes per a1 layer-kernel launch from the latest committed ncu capture of this config
-    (profiles/rNN_traffic_<config>.json, written by scripts/traffic.py), or (None, None)."""
+def committed_traffic(tag: str):
+    """Mean DRAM bytes per launch of the dominant kernel from the latest committed ncu capture of this
+    configuration (profiles/rNN_traffic_<tag>.json, written by scripts/traffic.py), or (None, None)."""
     import glob
-    files = sorted(glob.glob(os.path.join(os.path.dirname(os.path.abspath(__file__)), "profiles",
-                                          f"r*_traffic_{config}.json")))
+    files = sorted(glob.glob(os.path.join(ROOT, "profiles", f"r*_traffic_{tag}.json")))
     if not files:
         return None, None
     d = json.load(open(files[-1]))
@@ -186,11 +207,11 @@ def committed_traffic(config: str):
 
 
 # FP32 FMA pipe of a B200: 148 SMs x 128 FMA lanes/clk x 2 flop x 1965 MHz (B200_PROFILING.md: 148 SMs,
-# clocks.max.sm 1965 MHz; 128 FP32 lanes per SM: scripts/ubench_ffma.cu measured 127.9 FMA/clk/SM =
-# 37.1 TFMA/s for FFMA and FFMA2 alike)
+# clocks.max.sm 1965 MHz; 128 FP32 lanes per SM: scripts/ubench_ffma.cu measured 127.9 FMA/clk/SM,
+# profiles/r02_ubench_ffma.txt)
 FMA_PEAK_TFLOPS = 148 * 128 * 2 * 1965e6 / 1e12
 FMA_PEAK_SRC = ("derived: 148 SMs x 128 FP32 FMA/clk x 2 flop x 1965 MHz = 74.45 TFLOP/s (DESIGN.md §7; "
-                "scripts/ubench_ffma.cu measured 74.2)")
+                "scripts/ubench_ffma.cu measured 127.9 FMA/clk/SM, profiles/r02_ubench_ffma.txt)")
 
 
 def measured_peaks():
@@ -203,11 +224,10 @@ def measured_peaks():
 
 
 def oracle_sample_time(oracle, net, Y, cores, seconds, probe_only=False, max_rows=None):
-    """Rows of Y the oracle processes in ~`seconds` on all host cores (calibrated on `cores` rows run
-    with all threads; at most `max_rows`, default len(Y)), and the measured time for that many rows."""
+    """Rows of Y the oracle processes in ~`seconds` on all host cores, and the measured time for them.
+    Probe sizes double (from one row per core) until a probe takes >= seconds / 2: small probes are
+    dominated by per-call and thread start-up cost, which would under-size the sample."""
     cap = len(Y) if max_rows is None else max_rows
-    # probe sizes double until one takes >= seconds / 2 (small probes are dominated by per-call and
-    # thread start-up cost, which would under-size the sample)
     k = max(1, min(len(Y), cores))
     while True:
         t0 = time.perf_counter()
@@ -226,6 +246,15 @@ def oracle_sample_time(oracle, net, Y, cores, seconds, probe_only=False, max_row
     return rows, time.perf_counter() - t0
 
 
+def workload_config(args, c, snic, net, extra=None):
+    d = {"workload": f"{args.config}: {c['desc']}", "neurons": c["N"], "layers": c["L"], "batch": c["B"],
+         "connections": int(net.nnz), "w_mode": args.mode, "t": snic["t"], "s": snic["s"], "n": snic["n"],
+         "eta": 0.03, "eps": 0.03}
+    if extra:
+        d.update(extra)
+    return d
+
+
 # ------------------------------------------------------------------ reference arm (CPU oracle)
 def run_reference(args):
     rank = int(os.environ.get("RANK", "0"))
@@ -234,14 +263,14 @@ def run_reference(args):
     import oracle
 
     c, snic = config_params(args)
-    net = make_network(args, c)
+    net = make_network(args.config, args.mode, args.load, c)
     nnz = net.nnz
     cores = os.cpu_count() or 1
     # size the per-step sample to ~cpu_seconds / steps of the oracle on all cores
-    probe = make_inputs(args, c, min(c["B"], 64 * cores), 0)
+    probe = make_inputs(args.config, c, min(c["B"], 64 * cores), 0)
     rows, _ = oracle_sample_time(oracle, net, probe, cores, args.cpu_seconds / max(args.steps, 1), probe_only=True,
                                  max_rows=c["B"])
-    Y = make_inputs(args, c, rows, 0)
+    Y = make_inputs(args.config, c, rows, 0)
     if args.warmup > 0:
         oracle_layers(oracle, net, Y[: max(1, min(rows, cores))])
     times = []
@@ -256,8 +285,7 @@ def run_reference(args):
         "impl": "reference", "metric": METRIC, "value": value, "unit": UNIT, "n_gpus": args.gpus,
         "steps": args.steps, "warmup": args.warmup, "ms_per_step": T * 1e3, "higher_is_better": True,
         "scaling": args.scaling, "vs_baseline": None, "dtype": "f32", "data": "synthetic",
-        "config": {"workload": f"{args.config}: {c['desc']}", "neurons": c["N"], "layers": c["L"],
-                   "batch": c["B"], "w_mode": args.mode, "t": snic["t"], "s": snic["s"]},
+        "config": workload_config(args, c, snic, net),
         "cpu_baseline": {"value": value, "unit": UNIT, "cores": cores, "kind": "oracle", "sample": sample,
                          "cpu": cpu_info()},
         "e2e": {"value": value, "unit": UNIT, "h2d_bytes_per_step": 0, "d2h_bytes_per_step": 0},
@@ -266,13 +294,141 @@ def run_reference(args):
     return 0
 
 
+# ------------------------------------------------------------------ helpers of the SNICIT arm
+def load_handle(net, dev_index):
+    from paper_conf_icpp_jiangh0h23_b200 import SnicitNetwork
+    if isinstance(net, sdgc.CirculantNetwork):
+        return SnicitNetwork.circulant(net.N, net.L, net.nu, net.w, net.bias, net.ymax, device=dev_index)
+    return SnicitNetwork.from_network(net, device=dev_index)
+
+
+def event_ms(stream, fn, k, sync_dev):
+    """CUDA-event time of k calls of fn on `stream` (synchronize on both sides)."""
+    import torch
+    torch.cuda.synchronize(sync_dev)
+    e0, e1 = torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)
+    e0.record(stream)
+    for _ in range(k):
+        fn()
+    e1.record(stream)
+    torch.cuda.synchronize(sync_dev)
+    return e0.elapsed_time(e1) / k
+
+
+def residue_study(args, dev, stream, peak):
+    """The method's own conversion / residue kernels where they carry work: C2 at a small threshold
+    layer (t = 10: ~31 centroids and ~23k non-empty residue rows, profiles/r01_studies.md).  Rooflines of
+    map_residual_kernel (Alg. 2 / Eq. 3-4) and the residue trajectory kernel (Eq. 5) from live CUDA-event
+    kernel times and the library's work counters."""
+    from paper_conf_icpp_jiangh0h23_b200 import default_options
+    cfg = "C2"
+    c, snic = config_params(args, cfg, t=args.residue_t)
+    net = make_network(cfg, "radix", "csc", c)
+    Yh = make_inputs(cfg, c, c["B"], 0)
+    g = load_handle(net, dev.index)
+    g.set_stream(stream)
+    import torch
+    y0 = torch.from_numpy(Yh).to(dev)
+    y_out = torch.empty_like(y0)
+    t, s = snic["t"], snic["s"]
+    opt = default_options(n_segments=snic["n"])
+
+    def step():
+        g.infer(y0, t=t, s=s, options=opt, y_out=y_out)
+    step()
+    ms = event_ms(stream, step, max(1, min(args.steps, 3)), dev)
+    opt_t = default_options(n_segments=snic["n"], timing=2)
+    g.infer(y0, t=t, s=s, options=opt_t, y_out=y_out)
+    st = g.stats()
+    N = c["N"]
+    out = {"workload": f"C2 ({c['desc']}), t = {t}", "ms_per_step": ms, "value": c["B"] * net.nnz / (ms * 1e-3),
+           "unit": UNIT, "phases_ms": {k: st[k] for k in ("t_pre_ms", "t_convert_ms", "t_post_ms", "t_recover_ms")},
+           "dynamics": {k: st[k] for k in ("live_at_t", "n_centroids", "residual_at_t", "residual_final",
+                                            "res_nnz_at_t", "res_full_rl", "res_sparse_rl", "res_sparse_out",
+                                            "res_scalar_rl") if k in st}}
+    kms = st.get("t_map_ms", -1.0)
+    if kms and kms > 0:
+        # map_residual: every live row read once (float4 compares against <= C centroid rows, which stay
+        # in L2) + the residue rows written (4N each): algorithmic bytes = 4 N (live + residues at t)
+        by = 4.0 * N * (st["live_at_t"] + st["residual_at_t"])
+        ach = by / (kms * 1e-3) / 1e9
+        out["map_residual_kernel"] = {"bound": "hbm", "achieved": ach, "peak": peak, "unit": "GB/s",
+                                      "frac": ach / peak, "ms": kms, "algorithmic_bytes": by}
+    rms = st.get("t_residual_ms", -1.0)
+    if rms and rms > 0:
+        # residue trajectories: 2 flop per evaluated tap (32 taps per evaluated output)
+        outs = float(st.get("res_full_rl", 0)) * N + float(st.get("res_sparse_out", 0))
+        flops = 2.0 * 32 * outs
+        ach = flops / (rms * 1e-3) / 1e12
+        out["residual_kernel"] = {"bound": "alu", "achieved": ach, "peak": FMA_PEAK_TFLOPS, "unit": "TFLOP/s",
+                                  "frac": ach / FMA_PEAK_TFLOPS, "ms": rms, "algorithmic_flops": flops,
+                                  "evaluated_outputs": outs, "peak_source": FMA_PEAK_SRC}
+    # the same study with the dense-row residue form only (the paper's load-reduced SpMM, P:860-864)
+    if "res_sparse_rl" in st:
+        opt_d = default_options(n_segments=snic["n"], res_sparse=0)
+
+        def step_d():
+            g.infer(y0, t=t, s=s, options=opt_d, y_out=y_out)
+        step_d()
+        out["dense_residue_ms_per_step"] = event_ms(stream, step_d, max(1, min(args.steps, 3)), dev)
+    g.close()
+    del y0, y_out
+    return out
+
+
+def general_study(args, dev, stream, peak):
+    """General (non-circulant) CSC path: C2 with "perm" weights (RadiX columns under a seeded output
+    permutation per layer: 32 in / 32 out per neuron, not shift-invariant -> the ELL gather kernel).
+    SURVEY 8(d): reported next to radix so structure-exploiting kernels cannot hide general-CSC speed."""
+    from paper_conf_icpp_jiangh0h23_b200 import default_options
+    cfg = "C2"
+    c, snic = config_params(args, cfg, t=30)
+    net = make_network(cfg, "perm", "csc", c)
+    Yh = make_inputs(cfg, c, c["B"], 0)
+    g = load_handle(net, dev.index)
+    g.set_stream(stream)
+    import torch
+    y0 = torch.from_numpy(Yh).to(dev)
+    y_out = torch.empty_like(y0)
+    t, s = snic["t"], snic["s"]
+    opt = default_options(n_segments=snic["n"])
+
+    def step():
+        g.infer(y0, t=t, s=s, options=opt, y_out=y_out)
+    step()
+    ms = event_ms(stream, step, max(1, min(args.steps, 3)), dev)
+    g.infer(y0, t=t, s=s, options=default_options(n_segments=snic["n"], timing=2), y_out=y_out)
+    pr = g.layer_profile()
+    st = g.stats()
+    kms, kb = float(pr["ms"].sum()), float(pr["bytes"].sum())
+    ach = kb / (kms * 1e-3) / 1e9
+    rows = float(pr["rows"].sum())
+    # shared-memory gather ceiling (SURVEY H1): 4 B of LDS per edge-row at 148 SMs x 128 B/clk x 1.965 GHz
+    gather_peak = 148 * 128 * 1.965e9 / 4.0
+    edge_rows = 32.0 * c["N"] * rows
+    out = {"workload": f"C2 perm ({c['desc']}), t = {t}", "ms_per_step": ms, "value": c["B"] * net.nnz / (ms * 1e-3),
+           "unit": UNIT, "circ_layers": st["circ_layers"],
+           "roofline": {"bound": "hbm", "achieved": ach, "peak": peak, "unit": "GB/s", "frac": ach / peak,
+                        "kernel": "layer_ell_kernel (general CSC, a1)", "launches": int(len(pr["ms"])),
+                        "avg_launch_ms": kms / max(len(pr["ms"]), 1), "algorithmic_bytes": kb,
+                        "edge_rows_per_s": edge_rows / (kms * 1e-3),
+                        "smem_gather_frac": edge_rows / (kms * 1e-3) / gather_peak},
+           "phases_ms": {k: st[k] for k in ("t_pre_ms", "t_convert_ms", "t_post_ms", "t_recover_ms")}}
+    traffic, src = committed_traffic("C2_perm")
+    out["roofline"]["traffic"] = traffic
+    out["roofline"]["traffic_source"] = src
+    g.close()
+    return out
+
+
 # ------------------------------------------------------------------ SNICIT arm
 def run_snicit(args):
     import torch
     import torch.distributed as dist
 
-    from paper_conf_icpp_jiangh0h23_b200 import KERNEL_AUTO, KERNEL_CIRC, KERNEL_ELL, SnicitNetwork, default_options
-    from paper_conf_icpp_jiangh0h23_b200.parallel import allgather_categories, shard_rows
+    from paper_conf_icpp_jiangh0h23_b200 import (KERNEL_AUTO, KERNEL_CIRC, KERNEL_ELL, allgather_categories,
+                                                 allgather_categories_padded, default_options, shard_capacity,
+                                                 shard_rows)
 
     world = int(os.environ.get("WORLD_SIZE", "1"))
     rank = int(os.environ.get("RANK", "0"))
@@ -295,47 +451,38 @@ def run_snicit(args):
     if args.scaling == "weak":
         B_local, row0 = c["B"], rank * c["B"]
         B_global = c["B"] * world
+        cap = c["B"]
     else:
         a, b = shard_rows(c["B"], world, rank)
         B_local, row0, B_global = b - a, a, c["B"]
-    net = make_network(args, c)
+        cap = shard_capacity(c["B"], world)
+    net = make_network(args.config, args.mode, args.load, c)
     nnz = net.nnz
     kern = {"auto": KERNEL_AUTO, "ell": KERNEL_ELL, "circ": KERNEL_CIRC}[args.kernel]
-    Yh = make_inputs(args, c, B_local, row0)
-    if isinstance(net, sdgc.CirculantNetwork):
-        g = SnicitNetwork.circulant(net.N, net.L, net.nu, net.w, net.bias, net.ymax, device=dev.index)
-    else:
-        g = SnicitNetwork.from_network(net, device=dev.index)
+    Yh = make_inputs(args.config, c, B_local, row0)
+    g = load_handle(net, dev.index)
     stream = torch.cuda.Stream(device=dev)
     g.set_stream(stream)
     y0 = torch.from_numpy(Yh).to(dev)
     y_out = torch.empty_like(y0)
+    cat_buf = torch.empty(1 + cap, dtype=torch.int64, device=dev)
     opt = default_options(kernel=kern, n_segments=snic["n"], pre_fused=args.pre_fused)
     t, s = snic["t"], snic["s"]
+    gathered = [None]
 
     def step():
         g.infer(y0, t=t, s=s, options=opt, y_out=y_out, row_offset=row0)
+        g.categories_device(cat_buf)  # [count, ids...] on the device, queued on the library's stream
         if distributed:
             with torch.cuda.stream(stream):
-                ids = torch.from_numpy(g.categories()).to(coll_dev)
-                allgather_categories(ids)
-        else:
-            g.num_categories()  # category set present (count read synchronises the stream)
+                gathered[0] = allgather_categories_padded(cat_buf if backend == "nccl" else cat_buf.cpu())
 
     def timed(fn, k):
         if distributed:
             dist.barrier()
-        torch.cuda.synchronize(dev)
-        e0, e1 = torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)
-        e0.record(stream)
-        for _ in range(k):
-            fn()
-        e1.record(stream)
-        torch.cuda.synchronize(dev)
+        ms = event_ms(stream, fn, k, dev)
         if distributed:
             dist.barrier()
-        ms = e0.elapsed_time(e1) / k
-        if distributed:
             tt = torch.tensor([ms], device=coll_dev)
             dist.all_reduce(tt, op=dist.ReduceOp.MAX)
             ms = float(tt.item())
@@ -343,12 +490,32 @@ def run_snicit(args):
 
     for _ in range(max(args.warmup, 3)):
         step()
-    clocks = ClockSampler(local)
-    clocks.start()
+    clocks = ClockSampler(dev.index)
+    if rank == 0:
+        clocks.start()
     ms = timed(step, args.steps)
-    clk = clocks.stop()
-    launches_per_step = g.stats()["kernel_launches"]
+    clk = clocks.stop() if rank == 0 else None
+    st0 = g.stats()
+    launches_per_step = st0["kernel_launches"]
     value = B_global * nnz / (ms * 1e-3)
+    n_cat_global = None
+    if distributed:
+        counts = gathered[0][:, 0].tolist()
+        n_cat_global = int(sum(counts))
+    else:
+        n_cat_global = int(cat_buf[0].item())
+
+    # ---- per-rank phase times (one extra inference with phase events)
+    g.infer(y0, t=t, s=s, options=default_options(kernel=kern, n_segments=snic["n"], pre_fused=args.pre_fused,
+                                                  timing=1), y_out=y_out, row_offset=row0)
+    st1 = g.stats()
+    mine = {"rank": rank, "rows": B_local, "row_offset": row0,
+            **{k: st1[k] for k in ("t_pre_ms", "t_convert_ms", "t_post_ms", "t_recover_ms", "t_total_ms",
+                                   "live_at_t", "n_centroids", "residual_at_t", "n_categories")}}
+    per_rank = [mine]
+    if distributed:
+        per_rank = [None] * world
+        dist.all_gather_object(per_rank, mine)
 
     # ---- roofline of the dominant kernel (the pre-convergence a1 kernel), live CUDA events
     def profile_pre(pre_fused):
@@ -365,88 +532,91 @@ def run_snicit(args):
         pb_ = pbs[0] if pbs else np.zeros(0)
         return st_, pm_, pb_
 
-    st, pm, pb = profile_pre(args.pre_fused)
-    phases = {k: st[k] for k in ("t_pre_ms", "t_convert_ms", "t_post_ms", "t_recover_ms", "t_total_ms")}
     peak, peak_src = measured_peaks()
-    tag = args.config if args.t is None and args.mode == "radix" else None
-
-    def hbm_roof(pm_, pb_, st_):
-        """HBM roofline of the per-layer a1 kernels (8 B per live row-element per layer)."""
-        avg_ms = float(pm_.mean())
-        avg_bytes = float(pb_.mean())
-        achieved = avg_bytes / (avg_ms * 1e-3) / 1e9
-        traffic, traffic_src = committed_traffic(tag) if tag else (None, None)
-        r = {"bound": "hbm", "achieved": achieved, "peak": peak, "unit": "GB/s", "frac": achieved / peak,
-             "traffic": traffic, "traffic_unit": "bytes per launch (ncu dram read + write)",
-             "traffic_source": traffic_src,
-             "kernel": ("a1 layer kernels: layer_circ_kernel / layer_circ_seg_kernel (nu = 1), "
-                        "layer_circ_col_kernel (strided)") if st_["circ_layers"] else "layer_ell_kernel",
-             "peak_source": peak_src, "launches": int(len(pm_)), "avg_launch_ms": avg_ms,
-             "avg_algorithmic_bytes": avg_bytes,
-             "layer0_frac": float(pb_[0] / (pm_[0] * 1e-3) / 1e9 / peak)}
-        if args.mode == "radix":  # per stride class (layer l has stride nu_l; DESIGN.md §7 kernels)
-            strides = sdgc.radix_strides(c["N"])
-            by = {}
-            for l in range(len(pm_)):
-                e = by.setdefault(f"nu={strides[l % len(strides)]}", [0, 0.0, 0.0])
-                e[0] += 1
-                e[1] += float(pm_[l])
-                e[2] += float(pb_[l])
-            r["by_stride"] = {k: {"launches": n, "ms": round(ms_, 4),
-                                  "frac": round(b_ / (ms_ * 1e-3) / 1e9 / peak, 4)} for k, (n, ms_, b_) in by.items()}
-        return r
-
-    def alu_roof(pm_, pb_, st_):
-        """FP32 FMA-pipe roofline of the row-resident kernel: algorithmic flops = 2 x 32 x N per full
-        row-layer evaluation (constant rows carried by a scalar chain are not counted)."""
-        kms = float(pm_.sum())
-        flops = 2.0 * 32 * c["N"] * float(st_["pre_full_rows"])
-        achieved = flops / (kms * 1e-3) / 1e12
-        hbm_gbs = float(pb_.sum()) / (kms * 1e-3) / 1e9
-        traffic, traffic_src = committed_traffic(tag + "_fused") if tag else (None, None)
-        return {"bound": "alu", "achieved": achieved, "peak": FMA_PEAK_TFLOPS, "unit": "TFLOP/s",
-                "frac": achieved / FMA_PEAK_TFLOPS, "traffic": traffic,
-                "traffic_unit": "bytes per launch (ncu dram read + write)", "traffic_source": traffic_src,
-                "kernel": "pre_fused_kernel (row-resident a1: layers 0..t-1 of a row in shared memory, FFMA2 chains)",
-                "peak_source": FMA_PEAK_SRC, "launches": int(len(pm_)), "avg_launch_ms": kms,
-                "algorithmic_flops": flops, "full_row_layers": int(st_["pre_full_rows"]),
-                "const_rows": int(st_["pre_const_rows"]),
-                "hbm": {"algorithmic_bytes": float(pb_.sum()), "achieved_gbs": hbm_gbs, "frac": hbm_gbs / peak}}
-
     roof = None
-    if len(pm):
-        roof = alu_roof(pm, pb, st) if st["pre_fused"] else hbm_roof(pm, pb, st)
-        roof["share_of_step"] = float(pm.sum() / ms) if ms > 0 else None
-        if st["pre_fused"] and ms > 0:
-            # whole step (SURVEY 8(d)): the step's algorithmic flops (the row-resident pre phase: post
-            # layers of constant centroids are scalars) and bytes (pre phase + the live rows' final
-            # activations written by the recovery) over the measured step time
-            step_flops = roof["algorithmic_flops"]
-            step_bytes = roof["hbm"]["algorithmic_bytes"] + 4.0 * c["N"] * st["live_at_t"]
-            roof["whole_step"] = {"alu_frac": step_flops / (ms * 1e-3) / 1e12 / FMA_PEAK_TFLOPS,
-                                  "hbm_frac": step_bytes / (ms * 1e-3) / 1e9 / peak,
-                                  "algorithmic_flops": step_flops, "algorithmic_bytes": step_bytes}
-        if st["pre_fused"] and not args.no_variants:
-            # the same kernel with every live row evaluated in full (no constant-row shortcut), and the
-            # per-layer kernels (one launch per layer, HBM-bound) on the same inputs
-            st2, pm2, pb2 = profile_pre(2)
-            if st2["pre_fused"] and len(pm2):
-                r2 = alu_roof(pm2, pb2, st2)
-                roof["no_const_skip"] = {k: r2[k] for k in ("achieved", "frac", "avg_launch_ms", "full_row_layers")}
-            st0, pm0, pb0 = profile_pre(0)
-            if len(pm0):
-                r0 = hbm_roof(pm0, pb0, st0)
-                roof["per_layer_kernels"] = {k: r0[k] for k in ("bound", "achieved", "peak", "unit", "frac", "traffic",
-                                                                "traffic_source", "launches", "avg_launch_ms",
-                                                                "by_stride") if k in r0}
-                roof["per_layer_kernels"]["ms_total"] = float(pm0.sum())
+    phases = {k: st1[k] for k in ("t_pre_ms", "t_convert_ms", "t_post_ms", "t_recover_ms", "t_total_ms")}
+    if rank == 0 or not distributed:
+        st, pm, pb = profile_pre(args.pre_fused)
+        tag = args.config if args.t is None and args.mode == "radix" else None
+
+        def hbm_roof(pm_, pb_, st_):
+            """HBM roofline of the per-layer a1 kernels (8 B per live row-element per layer)."""
+            avg_ms = float(pm_.mean())
+            avg_bytes = float(pb_.mean())
+            achieved = avg_bytes / (avg_ms * 1e-3) / 1e9
+            traffic, traffic_src = committed_traffic(tag) if tag else (None, None)
+            r = {"bound": "hbm", "achieved": achieved, "peak": peak, "unit": "GB/s", "frac": achieved / peak,
+                 "traffic": traffic, "traffic_unit": "bytes per launch (ncu dram read + write)",
+                 "traffic_source": traffic_src,
+                 "kernel": ("a1 layer kernels: layer_circ_kernel / layer_circ_seg_kernel (nu = 1), "
+                            "layer_circ_col_kernel (strided)") if st_["circ_layers"] else "layer_ell_kernel",
+                 "peak_source": peak_src, "launches": int(len(pm_)), "avg_launch_ms": avg_ms,
+                 "avg_algorithmic_bytes": avg_bytes,
+                 "layer0_frac": float(pb_[0] / (pm_[0] * 1e-3) / 1e9 / peak)}
+            if args.mode == "radix":  # per stride class (layer l has stride nu_l; DESIGN.md §7 kernels)
+                strides = sdgc.radix_strides(c["N"])
+                by = {}
+                for l in range(len(pm_)):
+                    e = by.setdefault(f"nu={strides[l % len(strides)]}", [0, 0.0, 0.0])
+                    e[0] += 1
+                    e[1] += float(pm_[l])
+                    e[2] += float(pb_[l])
+                r["by_stride"] = {k: {"launches": n, "ms": round(ms_, 4),
+                                      "frac": round(b_ / (ms_ * 1e-3) / 1e9 / peak, 4)}
+                                  for k, (n, ms_, b_) in by.items()}
+            return r
+
+        def alu_roof(pm_, pb_, st_):
+            """FP32 FMA-pipe roofline of the row-resident kernel: algorithmic flops = 2 x 32 x N per full
+            row-layer evaluation (constant rows carried by a scalar chain are not counted)."""
+            kms = float(pm_.sum())
+            flops = 2.0 * 32 * c["N"] * float(st_["pre_full_rows"])
+            achieved = flops / (kms * 1e-3) / 1e12
+            hbm_gbs = float(pb_.sum()) / (kms * 1e-3) / 1e9
+            traffic, traffic_src = committed_traffic(tag + "_fused") if tag else (None, None)
+            return {"bound": "alu", "achieved": achieved, "peak": FMA_PEAK_TFLOPS, "unit": "TFLOP/s",
+                    "frac": achieved / FMA_PEAK_TFLOPS, "traffic": traffic,
+                    "traffic_unit": "bytes per launch (ncu dram read + write)", "traffic_source": traffic_src,
+                    "kernel": "pre_fused_kernel (row-resident a1: layers 0..t-1 of a row in shared memory)",
+                    "peak_source": FMA_PEAK_SRC, "launches": int(len(pm_)), "avg_launch_ms": kms,
+                    "algorithmic_flops": flops, "full_row_layers": int(st_["pre_full_rows"]),
+                    "const_rows": int(st_["pre_const_rows"]),
+                    "hbm": {"algorithmic_bytes": float(pb_.sum()), "achieved_gbs": hbm_gbs, "frac": hbm_gbs / peak,
+                            "peak": peak, "peak_source": peak_src}}
+
+        if len(pm):
+            roof = alu_roof(pm, pb, st) if st["pre_fused"] else hbm_roof(pm, pb, st)
+            # the timed step of a rank processes B_local rows; roofline launches are this rank's too
+            roof["share_of_step"] = float(pm.sum() / ms) if ms > 0 else None
+            if st["pre_fused"] and ms > 0:
+                step_flops = roof["algorithmic_flops"]
+                step_bytes = roof["hbm"]["algorithmic_bytes"] + 4.0 * c["N"] * st["live_at_t"]
+                roof["whole_step"] = {"alu_frac": step_flops / (ms * 1e-3) / 1e12 / FMA_PEAK_TFLOPS,
+                                      "hbm_frac": step_bytes / (ms * 1e-3) / 1e9 / peak,
+                                      "algorithmic_flops": step_flops, "algorithmic_bytes": step_bytes}
+            if st["pre_fused"] and not args.no_variants:
+                st2, pm2, pb2 = profile_pre(2)
+                if st2["pre_fused"] and len(pm2):
+                    r2 = alu_roof(pm2, pb2, st2)
+                    roof["no_const_skip"] = {k: r2[k] for k in ("achieved", "frac", "avg_launch_ms",
+                                                                "full_row_layers")}
+                st0_, pm0, pb0 = profile_pre(0)
+                if len(pm0):
+                    r0 = hbm_roof(pm0, pb0, st0_)
+                    roof["per_layer_kernels"] = {k: r0[k] for k in ("bound", "achieved", "peak", "unit", "frac",
+                                                                    "traffic", "traffic_source", "launches",
+                                                                    "avg_launch_ms", "by_stride") if k in r0}
+                    roof["per_layer_kernels"]["ms_total"] = float(pm0.sum())
 
     # ---- uncompressed GPU baseline (t >= L, same kernels)
     unc = None
     if not args.no_uncompressed:
         def step_unc():
             g.infer(y0, t=net.L, s=s, options=opt, y_out=y_out, row_offset=row0)
-            g.num_categories()
+            g.categories_device(cat_buf)
+            if distributed:
+                with torch.cuda.stream(stream):
+                    allgather_categories_padded(cat_buf if backend == "nccl" else cat_buf.cpu())
         step_unc()
         ms_u = timed(step_unc, max(1, min(args.steps, 3)))
         unc = {"value": B_global * nnz / (ms_u * 1e-3), "unit": UNIT, "ms_per_step": ms_u,
@@ -456,36 +626,39 @@ def run_snicit(args):
 
             def step_unc0():
                 g.infer(y0, t=net.L, s=s, options=opt0, y_out=y_out, row_offset=row0)
-                g.num_categories()
+                g.categories_device(cat_buf)
+                if distributed:
+                    with torch.cuda.stream(stream):
+                        allgather_categories_padded(cat_buf if backend == "nccl" else cat_buf.cpu())
             step_unc0()
             ms_u0 = timed(step_unc0, max(1, min(args.steps, 3)))
             unc["per_layer_kernels"] = {"value": B_global * nnz / (ms_u0 * 1e-3), "ms_per_step": ms_u0}
 
-    # ---- e2e through the C ABI with host (pinned) buffers.  Headline: the SDGC inputs are binary, so
-    # Y0 is uploaded as the packed bitmap of snicit_infer_packed (H2D inside the call) and the step's
-    # result is the category set (D2H).  Also reported: fp32 rows in and Y(L) out (e2e_fp32_io).
-    e2e = e2e_fp32 = None
+    # ---- e2e through the C ABI with host (pinned) buffers: snicit_infer with fp32 Y0 from
+    # the host (H2D inside the call, streamed under the pre phase) and the category set read back (D2H),
+    # all-gathered across ranks.  Also: snicit_infer_packed (binary inputs as a bitmap).
+    e2e = e2e_packed = None
     if not args.no_e2e:
         from paper_conf_icpp_jiangh0h23_b200 import pack_rows
         binary = bool(np.all((Yh == 0) | (Yh == 1)))  # SDGC inputs; config 5's are real-valued
-        bits_pin = torch.from_numpy(pack_rows(Yh if binary else Yh[:1] * 0).view(np.int32)).pin_memory()
         yh_pin = torch.from_numpy(Yh).pin_memory()
-        yo_pin = torch.empty_like(yh_pin).pin_memory()
+        bits_pin = torch.from_numpy(pack_rows(Yh).view(np.int32)).pin_memory() if binary else None
+
+        def gather_host(cats):
+            if distributed:
+                with torch.cuda.stream(stream):
+                    allgather_categories(torch.from_numpy(cats).to(coll_dev))
+
+        def step_fp32():
+            g.infer(yh_pin.numpy(), t=t, s=s, options=opt, row_offset=row0)  # host y0: returns when consumed
+            cats = g.categories()
+            gather_host(cats)
+            return cats
 
         def step_packed():
             g.infer_packed(bits_pin.numpy(), t=t, s=s, options=opt, row_offset=row0)
             cats = g.categories()
-            if distributed:
-                with torch.cuda.stream(stream):
-                    allgather_categories(torch.from_numpy(cats).to(coll_dev))
-            return cats
-
-        def step_fp32():
-            g.infer(yh_pin.numpy(), t=t, s=s, options=opt, y_out=yo_pin.numpy(), row_offset=row0)
-            cats = g.categories()
-            if distributed:
-                with torch.cuda.stream(stream):
-                    allgather_categories(torch.from_numpy(cats).to(coll_dev))
+            gather_host(cats)
             return cats
 
         def wall(fn):
@@ -506,18 +679,26 @@ def run_snicit(args):
             return ms_e, cats
 
         ms_f, cats = wall(step_fp32)
-        e2e_fp32 = {"value": B_global * nnz / (ms_f * 1e-3), "unit": UNIT, "ms_per_step": ms_f,
-                    "h2d_bytes_per_step": int(Yh.nbytes) * world, "d2h_bytes_per_step": (int(Yh.nbytes) + 8 * len(cats)) * world,
-                    "api": "snicit_infer (fp32 Y0 in, fp32 Y(L) out) + snicit_categories",
-                    "timer": "host wall clock around K synchronous C-ABI calls"}
+        e2e = {"value": B_global * nnz / (ms_f * 1e-3), "unit": UNIT, "ms_per_step": ms_f,
+               "h2d_bytes_per_step": int(Yh.nbytes) * world, "d2h_bytes_per_step": (4 + 8 * len(cats)) * world,
+               "api": "snicit_infer (fp32 Y0 from pinned host memory, streamed H2D under the pre phase) + "
+                      "snicit_categories (D2H)",
+               "timer": "host wall clock around K synchronous C-ABI calls, max over ranks"}
         if binary:
             ms_e, cats = wall(step_packed)
-            e2e = {"value": B_global * nnz / (ms_e * 1e-3), "unit": UNIT, "ms_per_step": ms_e,
-                   "h2d_bytes_per_step": int(bits_pin.numel() * 4) * world, "d2h_bytes_per_step": (4 + 8 * len(cats)) * world,
-                   "api": "snicit_infer_packed (Y0 as packed binary bitmap) + snicit_categories",
-                   "timer": "host wall clock around K synchronous C-ABI calls"}
-        else:  # real-valued inputs: fp32 rows in, final activations out
-            e2e = e2e_fp32
+            e2e_packed = {"value": B_global * nnz / (ms_e * 1e-3), "unit": UNIT, "ms_per_step": ms_e,
+                          "h2d_bytes_per_step": int(bits_pin.numel() * 4) * world,
+                          "d2h_bytes_per_step": (4 + 8 * len(cats)) * world,
+                          "api": "snicit_infer_packed (Y0 as packed binary bitmap) + snicit_categories",
+                          "timer": "host wall clock around K synchronous C-ABI calls, max over ranks"}
+
+    # ---- studies of the method's own kernels (rank 0, N = 1)
+    residue = general = None
+    if rank == 0 and not distributed:
+        if not args.no_residue and args.config != "C5":
+            residue = residue_study(args, dev, stream, peak)
+        if not args.no_general and args.config != "C5":
+            general = general_study(args, dev, stream, peak)
 
     # ---- CPU oracle baseline (rank 0, N = 1 only), bounded sample
     cpu = None
@@ -534,18 +715,21 @@ def run_snicit(args):
             "metric": METRIC, "value": value, "unit": UNIT, "n_gpus": world, "steps": args.steps,
             "warmup": max(args.warmup, 3), "ms_per_step": ms, "higher_is_better": True, "scaling": args.scaling,
             "vs_baseline": None, "dtype": "f32", "data": "synthetic (seeded SDGC-like RadiX W, MNIST-like binary Y0)",
-            "config": {"workload": f"{args.config}: {c['desc']}", "neurons": c["N"], "layers": c["L"],
-                       "batch_per_rank": B_local, "global_batch": B_global, "connections": nnz, "w_mode": args.mode,
-                       "t": t, "s": s, "n": snic["n"], "eta": 0.03, "eps": 0.03, "kernel": args.kernel,
-                       "pre_fused": args.pre_fused,
-                       "network_abi": "compact circulant" if isinstance(net, sdgc.CirculantNetwork) else "CSC",
-                       "l2": "inputs larger than L2 (no flush)", "parallelism": f"dp{world} (row shards)"},
-            "roofline": roof, "cpu_baseline": cpu, "e2e": e2e, "e2e_fp32_io": e2e_fp32, "clocks": clk,
-            "gpu_launches": int(launches_per_step * args.steps),
-            "uncompressed": unc, "phases_ms": phases,
-            "dynamics": {k: st[k] for k in ("live_at_t", "n_centroids", "n_sampled", "residual_at_t",
-                                            "residual_final", "n_categories")},
-            "paper_context": "SNICIT 4096-480 on 1x RTX A6000, B=60000: 44.17 ms = 8.55e13 edges/s (Table 3, P:1377)",
+            "config": workload_config(args, c, snic, net, {
+                "batch_per_rank": B_local, "global_batch": B_global, "kernel": args.kernel,
+                "pre_fused": args.pre_fused,
+                "network_abi": "compact circulant" if isinstance(net, sdgc.CirculantNetwork) else "CSC",
+                "l2": "inputs larger than L2 (no flush)",
+                "parallelism": f"dp{world} (row shards, {args.scaling} scaling)"}),
+            "roofline": roof, "cpu_baseline": cpu, "e2e": e2e, "e2e_packed": e2e_packed, "clocks": clk,
+            "gpu_launches": int(launches_per_step * args.steps + (2 * args.steps if distributed else args.steps)),
+            "uncompressed": unc, "phases_ms": phases, "per_rank": per_rank,
+            "categories": n_cat_global,
+            "dynamics": {k: st0[k] for k in ("live_at_t", "n_centroids", "n_sampled", "residual_at_t",
+                                             "residual_final", "n_categories")},
+            "residue": residue, "general_csc": general,
+            "paper_context": "SNICIT 16384-1920 on 1x RTX A6000, B=60000: 179.37 ms = 3.37e14 edges/s "
+                             "(Table 3, P:1383)",
         }
         print(json.dumps(line), flush=True)
     g.close()
@@ -555,8 +739,26 @@ def run_snicit(args):
     return 0
 
 
-def main():
-    args = parse()
+def spawn(args, argv):
+    """`--gpus N` outside a torchrun environment: re-launch this script with N ranks (one per GPU)."""
+    env = dict(os.environ)
+    env.setdefault("NCCL_DEBUG", "INFO")        # keep NCCL's communicator log (init, NVLS) on stderr
+    env.setdefault("NCCL_DEBUG_SUBSYS", "INIT")
+    import socket
+    sk = socket.socket()
+    sk.bind(("127.0.0.1", 0))
+    port = sk.getsockname()[1]
+    sk.close()
+    cmd = [sys.executable, "-m", "torch.distributed.run", "--nnodes=1", f"--nproc-per-node={args.gpus}",
+           "--master-addr=127.0.0.1", f"--master-port={port}", os.path.abspath(__file__)] + argv
+    return subprocess.call(cmd, env=env)
+
+
+def main(argv=None):
+    argv = sys.argv[1:] if argv is None else argv
+    args = parse(argv)
+    if args.gpus > 1 and "WORLD_SIZE" not in os.environ:
+        return spawn(args, argv)
     if args.impl == "reference":
         return run_reference(args)
     return run_snicit(args)

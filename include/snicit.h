@@ -101,6 +101,11 @@ typedef struct {
                                scalar fma chain per layer, written once at t (R26, exact; column-streaming
                                and segmented layer kernels, every layer < t circulant with uniform weight
                                and bias); 0 = every live row through every layer */
+    int32_t res_sparse;     /* fused post mode, circulant post layers: 1 = a residue row with few non-zero
+                               entries propagates only them (the outputs they touch are evaluated, every
+                               other output of Eq. 5 is exactly 0; north_star "only the nonzero residual
+                               entries are propagated"), chosen per row and layer from its non-zero count;
+                               0 = always the dense-row form.  Results identical. */
 } snicit_options;
 
 /* Per-run statistics of the last snicit_infer (times in ms, valid when options.timing). */
@@ -121,6 +126,13 @@ typedef struct {
     int32_t pre_fused;        /* the pre-convergence layers ran in the row-resident fused kernel */
     int32_t pre_const_rows;   /* fused: rows that became constant before t (carried by a scalar) */
     int64_t pre_full_rows;    /* fused: full-row layer evaluations (row x layer, 32*N fma each) */
+    int64_t res_nnz_at_t;     /* non-zero entries of the non-empty residue rows right after conversion */
+    int64_t res_full_rl;      /* residue row-layers evaluated in the dense-row form (N outputs each) */
+    int64_t res_sparse_rl;    /* residue row-layers evaluated in the sparse-entry form */
+    int64_t res_sparse_out;   /* outputs evaluated by the sparse-entry form (32 fma each) */
+    int64_t res_scalar_rl;    /* residue row-layers carried by a scalar (constant rows, R25/R26) */
+    double t_map_ms;          /* map_residual kernel (Alg. 2), CUDA events (options.timing), else -1 */
+    double t_residual_ms;     /* residue trajectory kernel (Eq. 5, fused post mode), else -1 */
 } snicit_stats_t;
 
 /* Fill *opt with the paper's SDGC defaults (n = 16, eta = eps = 0.03, prune_eps = 0,

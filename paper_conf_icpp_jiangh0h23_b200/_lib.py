@@ -32,7 +32,7 @@ class Options(ctypes.Structure):
                 ("prune_eps", ctypes.c_float), ("drop_dead_rows", ctypes.c_int32), ("kernel", ctypes.c_int32),
                 ("timing", ctypes.c_int32), ("ne_interval", ctypes.c_int32), ("post_mode", ctypes.c_int32),
                 ("post_cluster", ctypes.c_int32), ("post_const", ctypes.c_int32),
-                ("pre_fused", ctypes.c_int32), ("pre_const", ctypes.c_int32)]
+                ("pre_fused", ctypes.c_int32), ("pre_const", ctypes.c_int32), ("res_sparse", ctypes.c_int32)]
 
 
 class Stats(ctypes.Structure):
@@ -43,7 +43,10 @@ class Stats(ctypes.Structure):
                 ("n_centroids", ctypes.c_int32), ("n_sampled", ctypes.c_int32), ("threshold_layer", ctypes.c_int32),
                 ("circ_layers", ctypes.c_int32), ("kernel_launches", ctypes.c_int64),
                 ("const_centroids", ctypes.c_int32), ("pre_fused", ctypes.c_int32),
-                ("pre_const_rows", ctypes.c_int32), ("pre_full_rows", ctypes.c_int64)]
+                ("pre_const_rows", ctypes.c_int32), ("pre_full_rows", ctypes.c_int64),
+                ("res_nnz_at_t", ctypes.c_int64), ("res_full_rl", ctypes.c_int64), ("res_sparse_rl", ctypes.c_int64),
+                ("res_sparse_out", ctypes.c_int64), ("res_scalar_rl", ctypes.c_int64), ("t_map_ms", ctypes.c_double),
+                ("t_residual_ms", ctypes.c_double)]
 
     def as_dict(self):
         return {k: getattr(self, k) for k, _ in self._fields_}

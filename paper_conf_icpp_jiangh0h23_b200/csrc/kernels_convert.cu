@@ -293,7 +293,8 @@ __global__ void __launch_bounds__(kMapThreads) map_residual_kernel(const float* 
                                                                    float* __restrict__ yhat,
                                                                    float* __restrict__ cbuf,
                                                                    const uint8_t* __restrict__ rconst,
-                                                                   const float* __restrict__ rval) {
+                                                                   const float* __restrict__ rval,
+                                                                   unsigned long long* nnz_sum) {
     __shared__ int red[kMapThreads / 32];
     __shared__ int s_best, s_slot;
     const int n = *count;
@@ -370,6 +371,8 @@ __global__ void __launch_bounds__(kMapThreads) map_residual_kernel(const float* 
             const uint8_t ne = best_dist != 0 ? 1 : 0;  // lines 26-29
             ne_row[r] = ne;
             flag_pos[p] = ne;
+            // the residue's non-zeros are exactly the differing elements (x - y != 0 <=> x != y, finite)
+            if (nnz_sum && ne) atomicAdd(nnz_sum, (unsigned long long)best_dist);
         }
         __syncthreads();
         if (s_slot != 0) {  // residue only needed for non-empty rows (Eq. 4 first case)
@@ -386,12 +389,12 @@ __global__ void __launch_bounds__(kMapThreads) map_residual_kernel(const float* 
 cudaError_t launch_map_residual(const float* y, int N, const int* rows, const int* count, const int* cent,
                                 const int* n_cent, int* M, int* cslot, uint8_t* ne_row, uint8_t* flag_pos,
                                 float* yhat, float* cbuf, int max_rows, int num_sms, cudaStream_t st,
-                                const uint8_t* rconst, const float* rval) {
+                                const uint8_t* rconst, const float* rval, unsigned long long* nnz_sum) {
     int grid = num_sms * 8;
     if (grid > max_rows) grid = max_rows;
     if (grid < 1) grid = 1;
     map_residual_kernel<<<grid, kMapThreads, 0, st>>>(y, N, rows, count, cent, n_cent, M, cslot, ne_row, flag_pos,
-                                                      yhat, cbuf, rconst, rval);
+                                                      yhat, cbuf, rconst, rval, nnz_sum);
     return cudaGetLastError();
 }
 

@@ -76,13 +76,13 @@ __device__ __forceinline__ PL load_pl(const PostLayer* __restrict__ p) {
 
 // One layer of one row by the whole CTA: in -> out (shared memory).  `dup` != 0: in[N .. 2N) holds a
 // copy of in[0 .. N) (windows of every stride class read without wrap-around); else only a 64-float
-// halo is present (nu == 1 windows) and the general class wraps explicitly.  Returns this thread's
-// "some output != 0"; CENTROID mode also stores acc into aout (if non-NULL).
+// halo is present (nu == 1 windows) and the general class wraps explicitly.  Returns the number of
+// this thread's outputs != 0; CENTROID mode also stores acc into aout (if non-NULL).
 // MNU1 / MGEN: outputs per work item of the nu == 1 / general classes; QG: threads per residue class
 // of the Q == 32 class (32 / QG outputs each).  Small values -> more, shorter items (latency-bound
 // centroid trajectory on one SM); large -> fewer shared-memory loads per FMA (throughput).
 template <int MODE, bool UNIF, int MNU1, int MGEN, int QG>
-__device__ __forceinline__ bool post_row_circ(const PL& Ld, int N, int dup, float ymax, float prune_eps,
+__device__ __forceinline__ int post_row_circ(const PL& Ld, int N, int dup, float ymax, float prune_eps,
                                               const float* __restrict__ in, float* __restrict__ out,
                                               const float* __restrict__ ac, float* __restrict__ aout) {
     const float w0 = Ld.w0, b0 = Ld.b0;
@@ -94,7 +94,7 @@ __device__ __forceinline__ bool post_row_circ(const PL& Ld, int N, int dup, floa
 #pragma unroll
         for (int n = 0; n < kPK; ++n) w[n] = __ldg(Ld.wtab + n);
     }
-    bool any = false;
+    int nz = 0;
     auto emit = [&](float acc, int q) {
         const float b = ubias ? b0 : __ldg(bias + q);
         if constexpr (MODE == MODE_CENTROID) {
@@ -102,7 +102,7 @@ __device__ __forceinline__ bool post_row_circ(const PL& Ld, int N, int dup, floa
         }
         const float v = post_epi<MODE>(acc, b, ac, q, ymax, prune_eps);
         out[q] = v;
-        any |= (v != 0.0f);
+        nz += (v != 0.0f);
     };
     if (Ld.cls == PCLS_NU1) {
         constexpr int M = MNU1, WIN = M + kPK - 1;
@@ -173,11 +173,11 @@ __device__ __forceinline__ bool post_row_circ(const PL& Ld, int N, int dup, floa
             }
         }
     }
-    return any;
+    return nz;
 }
 
 template <int MODE>
-__device__ __forceinline__ bool post_row_ell(const PL& Ld, int N, float ymax, float prune_eps,
+__device__ __forceinline__ int post_row_ell(const PL& Ld, int N, float ymax, float prune_eps,
                                              const float* __restrict__ in, float* __restrict__ out,
                                              const float* __restrict__ ac, float* __restrict__ aout) {
     const uint8_t* __restrict__ lens = Ld.len;
@@ -188,7 +188,7 @@ __device__ __forceinline__ bool post_row_ell(const PL& Ld, int N, float ymax, fl
     const int K = Ld.K;
     const bool unif = Ld.unif != 0, ubias = Ld.ubias != 0;
     const float w0 = Ld.w0, b0 = Ld.b0;
-    bool any = false;
+    int nz = 0;
     for (int j = threadIdx.x; j < N; j += blockDim.x) {
         const int len = lens ? (int)lens[j] : K;
         float acc = 0.0f;
@@ -204,13 +204,13 @@ __device__ __forceinline__ bool post_row_ell(const PL& Ld, int N, float ymax, fl
         }
         const float v = post_epi<MODE>(acc, b, ac, j, ymax, prune_eps);
         out[j] = v;
-        any |= (v != 0.0f);
+        nz += (v != 0.0f);
     }
-    return any;
+    return nz;
 }
 
 template <int MODE, int MNU1, int MGEN, int QG>
-__device__ __forceinline__ bool post_row_layer(const PL& Ld, int N, int dup, float ymax, float prune_eps,
+__device__ __forceinline__ int post_row_layer(const PL& Ld, int N, int dup, float ymax, float prune_eps,
                                                const float* in, float* out, const float* ac, float* aout,
                                                int force_ell) {
     if (Ld.kind == 1 && !force_ell) {
@@ -280,13 +280,134 @@ __global__ void __launch_bounds__(kCentThreads) centroid_traj_kernel(PostArgs a)
     unstage_row(a.cbuf + (size_t)c * N, cur, N);
 }
 
+// ---- sparse-entry residue form (north_star: "only the nonzero residual entries are propagated";
+// Eq. 5 / load-reduced SpMM P:860-889).  For a circulant layer, output j reads inputs (j + n nu) mod N,
+// so input k feeds outputs (k - n nu) mod N, n = 0..31.  An output none of whose inputs is non-zero
+// has a_r = +0 exactly (every fma adds a signed zero to +0), so Eq. 5 gives sigma((a_c + 0) + b) -
+// sigma(a_c + b) == 0 (R16): only the outputs touched by a non-zero input can be non-zero, and each
+// of them is evaluated with its full stored-order chain (R12; the zero taps add exact zeros), so the
+// result is bit-identical to the dense-row form (tested).  A row is evaluated this way while its
+// non-zero count is at most N / kSpDiv (so at most N/4 outputs are touched); otherwise densely.
+constexpr int kSpDiv = 128;
+__host__ __device__ inline int sp_cap(int N) { return N / kSpDiv > 0 ? N / kSpDiv : 1; }
+// extra shared memory of the sparse form (ints): touched bitmap, two non-zero lists, touched list
+__host__ __device__ inline int sp_ints(int N) { return (N + 31) / 32 + 2 * sp_cap(N) + 32 * sp_cap(N); }
+
+// list the non-zero entries of row[0 .. N) into lst (first `cap` of them, in no particular order);
+// returns the total count (every thread)
+__device__ __forceinline__ int sp_list(const float* row, int N, int* lst, int cap, int* s_cnt) {
+    const int lane = threadIdx.x & 31;
+    if (threadIdx.x == 0) *s_cnt = 0;
+    __syncthreads();
+    for (int k0 = (threadIdx.x & ~31); k0 < N; k0 += blockDim.x) {
+        const int k = k0 + lane;
+        const bool nzv = k < N && row[k] != 0.0f;
+        const unsigned m = __ballot_sync(0xffffffffu, nzv);
+        int base = 0;
+        if (lane == 0 && m) base = atomicAdd(s_cnt, __popc(m));
+        base = __shfl_sync(0xffffffffu, base, 0);
+        const int pos = base + __popc(m & ((1u << lane) - 1u));
+        if (nzv && pos < cap) lst[pos] = k;
+    }
+    __syncthreads();
+    return *s_cnt;
+}
+
+// One sparse-entry layer of a residue row: in (dense, non-zero exactly at lst[0 .. nnz)) -> out (all
+// zero on entry; written at the touched outputs).  Returns the output's non-zero count (every thread);
+// its first `cap` non-zeros are listed in lst_out.  *ntouched = outputs evaluated.
+template <bool UNIF>
+__device__ int sp_layer(const PL& Ld, int N, float ymax, float prune_eps, const float* __restrict__ in,
+                        float* __restrict__ out, const float* __restrict__ ac, const int* lst, int nnz, int* lst_out,
+                        int cap, unsigned* bm, int* tl, int* s_cnt, int* ntouched) {
+    const int nu = Ld.nu, W = (N + 31) >> 5;
+    const float w0 = Ld.w0, b0 = Ld.b0;
+    const bool ubias = Ld.ubias != 0;
+    float w[UNIF ? 1 : kPK];
+    if constexpr (!UNIF) {
+#pragma unroll
+        for (int n = 0; n < kPK; ++n) w[n] = __ldg(Ld.wtab + n);
+    }
+    for (int i = threadIdx.x; i < W; i += blockDim.x) bm[i] = 0u;
+    if (threadIdx.x == 0) {
+        s_cnt[0] = 0;  // touched outputs
+        s_cnt[1] = 0;  // non-zero outputs
+    }
+    __syncthreads();
+    // mark the outputs fed by the non-zero inputs (32 per input)
+    for (int i = threadIdx.x; i < nnz * kPK; i += blockDim.x) {
+        const int k = lst[i >> 5], n = i & 31;
+        int j = k - n * nu;
+        j = j < 0 ? j + N : j;  // n nu < N (K nu <= N, distinct inputs)
+        atomicOr(bm + (j >> 5), 1u << (j & 31));
+    }
+    __syncthreads();
+    // touched list (per-warp scan of the bitmap words; order across warps is irrelevant)
+    const int lane = threadIdx.x & 31;
+    for (int i0 = (threadIdx.x & ~31); i0 < W; i0 += blockDim.x) {
+        const int i = i0 + lane;
+        const unsigned m = i < W ? bm[i] : 0u;
+        const int c = __popc(m);
+        int incl = c;
+#pragma unroll
+        for (int o = 1; o < 32; o <<= 1) {
+            const int v = __shfl_up_sync(0xffffffffu, incl, o);
+            if (lane >= o) incl += v;
+        }
+        int base = 0;
+        if (lane == 31 && incl) base = atomicAdd(&s_cnt[0], incl);
+        base = __shfl_sync(0xffffffffu, base, 31);
+        int pos = base + incl - c;
+        for (unsigned mm = m; mm; mm &= mm - 1u) tl[pos++] = (i << 5) + __ffs(mm) - 1;
+    }
+    __syncthreads();
+    const int nt = s_cnt[0];
+    // evaluate the touched outputs: the full stored-order chain (R12), Eq. 5 epilogue
+    for (int i0 = (threadIdx.x & ~31); i0 < nt; i0 += blockDim.x) {
+        const int i = i0 + lane;
+        float v = 0.0f;
+        int j = 0;
+        if (i < nt) {
+            j = tl[i];
+            float acc = 0.0f;
+            int k = j;
+#pragma unroll
+            for (int n = 0; n < kPK; ++n) {
+                acc = fmaf(in[k], UNIF ? w0 : w[n], acc);
+                k += nu;
+                k = k >= N ? k - N : k;
+            }
+            const float b = ubias ? b0 : __ldg(Ld.bias + j);
+            v = post_epi<MODE_RESIDUAL>(acc, b, ac, j, ymax, prune_eps);
+            out[j] = v;
+        }
+        const unsigned m = __ballot_sync(0xffffffffu, v != 0.0f);
+        int base = 0;
+        if (lane == 0 && m) base = atomicAdd(&s_cnt[1], __popc(m));
+        base = __shfl_sync(0xffffffffu, base, 0);
+        const int pos = base + __popc(m & ((1u << lane) - 1u));
+        if (v != 0.0f && pos < cap) lst_out[pos] = j;
+    }
+    __syncthreads();
+    *ntouched = nt;
+    return s_cnt[1];
+}
+
 __global__ void __launch_bounds__(kPostThreads, 2) residual_traj_kernel(PostArgs a) {
     extern __shared__ __align__(128) float sm[];
     __shared__ int s_p;
+    __shared__ int s_nz[3];   // per-layer non-zero count of the dense form (rotating slots)
+    __shared__ int s_cnt[2];  // sparse form scratch
     const int N = a.N;
     const int h = post_halo(N);
     const int dup = h == N;
     const int n = *a.rcount;
+    const int cap = sp_cap(N);
+    // sparse-form scratch after the two row buffers
+    unsigned* bm = reinterpret_cast<unsigned*>(sm + 2 * (N + h));
+    int* lsts[2] = {reinterpret_cast<int*>(bm + (N + 31) / 32), reinterpret_cast<int*>(bm + (N + 31) / 32) + cap};
+    int* tl = lsts[1] + cap;
+    unsigned long long c_full = 0, c_sparse = 0, c_sout = 0, c_scalar = 0;  // thread 0's work counters
     for (;;) {
         if (threadIdx.x == 0) s_p = atomicAdd(a.work_counter, 1);
         __syncthreads();
@@ -303,14 +424,54 @@ __global__ void __launch_bounds__(kPostThreads, 2) residual_traj_kernel(PostArgs
         bool alive = true, cst = false;
         float vr = 0.0f;
         const int cfrom = a.cfrom ? a.cfrom[slot] : a.L - a.t;
+        // sparse form: nnz of `cur` and whether lsts[li] lists all of its non-zeros; nxt_zero: `nxt` is
+        // all-zero in [0, N) (left so by the previous sparse layer)
+        int nnz = -1, li = 0;
+        bool listed = false, nxt_zero = false;
+        if (a.res_sparse) {
+            nnz = sp_list(cur, N, lsts[0], cap, &s_cnt[0]);
+            listed = nnz <= cap;
+        }
         PL Ld = load_pl(a.layers + a.t);
         int l = a.t;
         for (; l < a.L; ++l) {
             const PL Lnext = load_pl(a.layers + min(l + 1, a.L - 1));
             const float* ac = a.a_all + ((size_t)(l - a.t) * a.s + slot) * N;
-            const bool any = post_row_layer<MODE_RESIDUAL, 17, 16, 1>(Ld, N, dup, a.ymax, a.prune_eps, cur, nxt, ac,
-                                                                      nullptr, a.force_ell);
-            if (!__syncthreads_or(any)) {  // the residue became empty: it stays empty (R16)
+            const bool sparse = a.res_sparse && listed && Ld.kind == 1 && !a.force_ell;
+            int cnt;
+            if (sparse) {
+                if (!nxt_zero)
+                    for (int k = threadIdx.x; k < N; k += blockDim.x) nxt[k] = 0.0f;
+                // (sp_layer's first barrier orders these stores before its own)
+                int nt = 0;
+                cnt = Ld.unif ? sp_layer<true>(Ld, N, a.ymax, a.prune_eps, cur, nxt, ac, lsts[li], nnz, lsts[li ^ 1],
+                                               cap, bm, tl, s_cnt, &nt)
+                              : sp_layer<false>(Ld, N, a.ymax, a.prune_eps, cur, nxt, ac, lsts[li], nnz,
+                                                lsts[li ^ 1], cap, bm, tl, s_cnt, &nt);
+                // `cur` becomes the next output buffer: clear its non-zeros (exactly lsts[li])
+                for (int i = threadIdx.x; i < nnz; i += blockDim.x) cur[lsts[li][i]] = 0.0f;
+                nxt_zero = true;
+                li ^= 1;
+                nnz = cnt;
+                listed = cnt <= cap;
+                if (threadIdx.x == 0) {
+                    ++c_sparse;
+                    c_sout += (unsigned long long)nt;
+                }
+            } else {
+                if (threadIdx.x == 0) s_nz[(l + 1) % 3] = 0;  // slot of the next layer (read two barriers ago)
+                const int mine = post_row_layer<MODE_RESIDUAL, 17, 16, 1>(Ld, N, dup, a.ymax, a.prune_eps, cur, nxt,
+                                                                          ac, nullptr, a.force_ell);
+                const int wsum = __reduce_add_sync(0xffffffffu, mine);
+                if ((threadIdx.x & 31) == 0 && wsum) atomicAdd(&s_nz[l % 3], wsum);
+                __syncthreads();
+                cnt = s_nz[l % 3];
+                nxt_zero = false;
+                nnz = cnt;
+                listed = false;
+                if (threadIdx.x == 0) ++c_full;
+            }
+            if (cnt == 0) {  // the residue became empty: it stays empty (R16)
                 alive = false;
                 break;
             }
@@ -330,6 +491,10 @@ __global__ void __launch_bounds__(kPostThreads, 2) residual_traj_kernel(PostArgs
             }
             fill_halo(nxt, N, h);
             __syncthreads();
+            if (a.res_sparse && !listed && nnz <= cap) {  // the dense output is sparse: list it
+                nnz = sp_list(nxt, N, lsts[li], cap, &s_cnt[0]);
+                listed = true;
+            }
             float* tmp = cur;
             cur = nxt;
             nxt = tmp;
@@ -346,6 +511,7 @@ __global__ void __launch_bounds__(kPostThreads, 2) residual_traj_kernel(PostArgs
                 float v = sigma((acv + acc) + b0, a.ymax) - sigma(acv + b0, a.ymax);
                 if (a.prune_eps > 0.0f && fabsf(v) <= a.prune_eps) v = 0.0f;
                 vr = v;
+                if (threadIdx.x == 0) ++c_scalar;
                 if (v == 0.0f) {
                     alive = false;
                     break;
@@ -364,6 +530,12 @@ __global__ void __launch_bounds__(kPostThreads, 2) residual_traj_kernel(PostArgs
             if (alive && a.alive_count) atomicAdd(a.alive_count, 1);
         }
         __syncthreads();  // s_p and the row buffers are reused
+    }
+    if (threadIdx.x == 0 && a.ctr64) {
+        if (c_full) atomicAdd(a.ctr64 + C64_FULL_RL, c_full);
+        if (c_sparse) atomicAdd(a.ctr64 + C64_SPARSE_RL, c_sparse);
+        if (c_sout) atomicAdd(a.ctr64 + C64_SPARSE_OUT, c_sout);
+        if (c_scalar) atomicAdd(a.ctr64 + C64_SCALAR_RL, c_scalar);
     }
 }
 
@@ -697,9 +869,14 @@ cudaError_t launch_centroid_traj(const PostArgs& a, int C_max, cudaStream_t st) 
     return cudaGetLastError();
 }
 
-cudaError_t launch_residual_traj(const PostArgs& a, int max_rows, int num_sms, cudaStream_t st) {
+cudaError_t launch_residual_traj(const PostArgs& a_in, int max_rows, int num_sms, cudaStream_t st) {
     if (max_rows <= 0) return cudaSuccess;
-    const size_t smem = sizeof(float) * 2 * (size_t)(a.N + post_halo(a.N));
+    PostArgs a = a_in;
+    size_t smem = sizeof(float) * 2 * (size_t)(a.N + post_halo(a.N));
+    if (a.res_sparse && smem + sizeof(int) * (size_t)sp_ints(a.N) <= (size_t)220 * 1024)
+        smem += sizeof(int) * (size_t)sp_ints(a.N);
+    else
+        a.res_sparse = 0;
     int per_sm = 1;
     cudaError_t e = blocks_per_sm((const void*)residual_traj_kernel, kPostThreads, smem, &per_sm);
     if (e != cudaSuccess) return e;

@@ -251,13 +251,13 @@ __global__ void __launch_bounds__(T, PfCfg<T>::kMinBlocks) pre_fused_kernel(cons
     };
     auto issue_load = [&](int p_, float* dst, uint64_t* b, int slot) {
         const size_t r_ = (size_t)__ldg(a.rows + p_);
+        if (a.ready) {  // streamed upload: wait until the copy engine has delivered this row's chunk
+            // geometric chunks: chunk c holds rows [b (2^c - 1), b (2^(c+1) - 1)), b = ready_rows
+            const int* f = a.ready + (31 - __clz((int)(r_ / a.ready_rows) + 1));
+            while (ld_acquire_gpu(f) == 0) __nanosleep(256);
+            fence_proxy_async_global();
+        }
         if (a.ybits) {  // packed binary row: N/8 bytes
-            if (a.ready) {  // streamed upload: wait until the copy engine has delivered this row's chunk
-                // geometric chunks: chunk c holds rows [b (2^c - 1), b (2^(c+1) - 1)), b = ready_rows
-                const int* f = a.ready + (31 - __clz((int)(r_ / a.ready_rows) + 1));
-                while (ld_acquire_gpu(f) == 0) __nanosleep(256);
-                fence_proxy_async_global();
-            }
             mbar_arrive_expect_tx(b, (uint32_t)(N / 8));
             bulk_g2s(s_bits + slot * (N / 32), a.ybits + r_ * (N / 32), N / 8, b);
         } else {

@@ -21,6 +21,10 @@
 
 using namespace snicit;
 
+// the Python binding mirrors these structs (paper_conf_icpp_jiangh0h23_b200/_lib.py; tests/test_abi.py)
+static_assert(sizeof(snicit_options) == 56, "snicit_options layout");
+static_assert(sizeof(snicit_stats_t) == 184, "snicit_stats_t layout");
+
 namespace {
 
 thread_local std::string g_last_error;
@@ -149,7 +153,9 @@ struct snicit_network {
     bool last_dead_zeroed = false;  // the row-resident kernel wrote dead rows' zeros into y_out
     bool res_at_t_lazy = false;     // residual_at_t is read from CNT_RES0 by snicit_stats
     snicit_stats_t stats{};
-    cudaEvent_t ev[6] = {nullptr, nullptr, nullptr, nullptr, nullptr, nullptr};
+    cudaEvent_t ev[10] = {};  // phase events [0..5]; map_residual [6, 7]; residue trajectories [8, 9]
+    bool ev_map = false, ev_res = false;  // the kernel events of the last timed infer were recorded
+    DevBuf<unsigned long long> ctr64;     // work counters of the last infer (Ctr64)
     std::vector<cudaEvent_t> lev;  // 2 per pre-convergence layer (timing == 2)
     DevBuf<int> hist;              // active rows at the start of each pre-convergence layer
     int prof_layers = 0;
@@ -266,7 +272,8 @@ static cudaError_t net_upload_common(snicit_network* net, const float* bias, con
     if (e == cudaSuccess) e = net->pf_full.ensure(1);
     if (e == cudaSuccess) e = net->counters.ensure(CNT_N);
     if (e == cudaSuccess) e = cudaMallocHost(&net->h_counters, sizeof(int) * CNT_N);
-    for (int i = 0; i < 6 && e == cudaSuccess; ++i) e = cudaEventCreate(&net->ev[i]);
+    for (int i = 0; i < 10 && e == cudaSuccess; ++i) e = cudaEventCreate(&net->ev[i]);
+    if (e == cudaSuccess) e = net->ctr64.ensure(C64_N);
     return e;
 }
 
@@ -288,6 +295,7 @@ void snicit_default_options(snicit_options* opt) {
     opt->post_const = 1;
     opt->pre_fused = 1;
     opt->pre_const = 1;
+    opt->res_sparse = 1;
 }
 
 const char* snicit_last_error(void) { return g_last_error.c_str(); }
@@ -341,6 +349,7 @@ void snicit_free_network(snicit_network* net) {
     net->cfrom.release();
     net->rval.release();
     net->a_all.release();
+    net->ctr64.release();
     delete net;
 }
 
@@ -742,6 +751,46 @@ static bool pf_plan(const snicit_network* net, int tt, const snicit_options& opt
     return pf;
 }
 
+// Streamed upload of R host rows of `row_bytes` each into the device buffer `dst`: the copy engine
+// delivers geometric chunks of rows (chunk c = rows [b (2^c - 1), b (2^(c+1) - 1)), b = kChunk0) on a
+// side stream, each followed by its ready flag, while the row-resident kernel runs (it polls the flag
+// of a row's chunk before loading the row), so the upload overlaps the compute.  The first rows
+// arrive within microseconds and the whole batch takes a handful of API calls.  The handle's stream
+// must wait on net->cev[1] before anything later reuses `dst` or the flags.
+static cudaError_t stream_upload(snicit_network* net, void* dst, const void* src, size_t row_bytes, int R,
+                                 const int** ready, int* ready_rows) {
+    constexpr int kChunk0 = 512;
+    int nch = 0;
+    while ((long long)kChunk0 * ((1LL << nch) - 1) < R) ++nch;
+    cudaError_t e;
+    if (!net->copy_stream && (e = cudaStreamCreateWithFlags(&net->copy_stream, cudaStreamNonBlocking)) != cudaSuccess)
+        return e;
+    for (auto& ev : net->cev)
+        if (!ev && (e = cudaEventCreateWithFlags(&ev, cudaEventDisableTiming)) != cudaSuccess) return e;
+    if (!net->h_ones) {
+        if ((e = cudaMallocHost(&net->h_ones, sizeof(int))) != cudaSuccess) return e;
+        *net->h_ones = 1;
+    }
+    if ((e = net->bits_ready.ensure((size_t)std::max(nch, 1))) != cudaSuccess) return e;
+    if ((e = cudaMemsetAsync(net->bits_ready.p, 0, sizeof(int) * std::max(nch, 1), net->stream)) != cudaSuccess) return e;
+    if ((e = cudaEventRecord(net->cev[0], net->stream)) != cudaSuccess) return e;
+    if ((e = cudaStreamWaitEvent(net->copy_stream, net->cev[0], 0)) != cudaSuccess) return e;
+    for (int c = 0; c < nch; ++c) {
+        const size_t r0 = (size_t)kChunk0 * ((1ull << c) - 1);
+        const size_t nr = std::min<size_t>((size_t)kChunk0 << c, R - r0);
+        if ((e = cudaMemcpyAsync(static_cast<char*>(dst) + r0 * row_bytes, static_cast<const char*>(src) + r0 * row_bytes,
+                                 row_bytes * nr, cudaMemcpyHostToDevice, net->copy_stream)) != cudaSuccess)
+            return e;
+        if ((e = cudaMemcpyAsync(net->bits_ready.p + c, net->h_ones, sizeof(int), cudaMemcpyHostToDevice,
+                                 net->copy_stream)) != cudaSuccess)
+            return e;
+    }
+    if ((e = cudaEventRecord(net->cev[1], net->copy_stream)) != cudaSuccess) return e;
+    *ready = net->bits_ready.p;
+    *ready_rows = kChunk0;
+    return cudaSuccess;
+}
+
 // y0_mode: 0 = y0 is a device pointer, 1 = host pointer, 2 = the input rows are already in net->Ya,
 // 3 = packed binary rows `bits` (device-accessible, possibly host-mapped) read by the row-resident
 // kernel (the caller checked pf_plan)
@@ -750,6 +799,7 @@ static snicit_status infer_core(snicit_network* net, const float* y0, int64_t ba
                                 int64_t row_offset, int32_t t, int32_t s, const snicit_options* opt_in, float* y_out,
                                 int32_t y_out_on_device, const uint32_t* bits = nullptr, float one = 1.0f,
                                 const int* bits_ready = nullptr, int ready_rows = 0) {
+    // (bits_ready / ready_rows: the ready flags of a streamed upload, set here for host fp32 rows)
     const int32_t y0_on_device = y0_mode == 0;
     if (!net) return fail(SNICIT_E_INVALID_ARG, "net NULL");
     if (batch < 0 || batch > 0x7fffffffLL) return fail(SNICIT_E_INVALID_ARG, "batch out of range");
@@ -772,6 +822,7 @@ static snicit_status infer_core(snicit_network* net, const float* y0, int64_t ba
     if (opt.post_mode < 0 || opt.post_mode > 1) return fail(SNICIT_E_INVALID_ARG, "bad post_mode");
     if (opt.pre_fused < 0 || opt.pre_fused > 2) return fail(SNICIT_E_INVALID_ARG, "bad pre_fused");
     if (opt.pre_const < 0 || opt.pre_const > 1) return fail(SNICIT_E_INVALID_ARG, "bad pre_const");
+    if (opt.res_sparse < 0 || opt.res_sparse > 1) return fail(SNICIT_E_INVALID_ARG, "bad res_sparse");
     if (opt.kernel == SNICIT_KERNEL_ELL && !net->has_ell)
         return fail(SNICIT_E_UNSUPPORTED, "network loaded in compact circulant form has no ELL copy");
     const int N = net->N, L = net->L;
@@ -790,11 +841,13 @@ static snicit_status infer_core(snicit_network* net, const float* y0, int64_t ba
     int64_t launches = y0_mode == 2 ? 1 : 0;  // + the unpack kernel of snicit_infer_packed (mode 2)
     int circ_layers = 0;
     net->have_result = false;
+    net->ev_map = net->ev_res = false;
     snicit_stats_t stats{};
     stats.batch = batch;
     stats.threshold_layer = tt;
 
     if (opt.timing) CUDA_TRY(cudaEventRecord(net->ev[0], st));
+    bool host_streamed = false;  // host fp32 rows uploaded by stream_upload while the pre phase runs
     // ---- input
     const float* cur;
     float* bufs[2] = {net->Ya.p, net->Yb.p};
@@ -804,8 +857,15 @@ static snicit_status infer_core(snicit_network* net, const float* y0, int64_t ba
     } else if (y0_mode == 3) {
         cur = nullptr;  // the row-resident kernel reads the packed rows itself
     } else {
-        if (y0_mode == 1)
-            CUDA_TRY(cudaMemcpyAsync(net->Ya.p, y0, sizeof(float) * (size_t)R * N, cudaMemcpyHostToDevice, st));
+        if (y0_mode == 1 && R > 0) {
+            int H_ = 0, g_ = 0;
+            if (pf_plan(net, tt, opt, R, &H_, &g_)) {  // the row-resident kernel polls the chunks' flags
+                CUDA_TRY(stream_upload(net, net->Ya.p, y0, sizeof(float) * (size_t)N, R, &bits_ready, &ready_rows));
+                host_streamed = true;
+            } else {
+                CUDA_TRY(cudaMemcpyAsync(net->Ya.p, y0, sizeof(float) * (size_t)R * N, cudaMemcpyHostToDevice, st));
+            }
+        }
         cur = net->Ya.p;
         nxt_i = 1;
     }
@@ -870,7 +930,7 @@ static snicit_status infer_core(snicit_network* net, const float* y0, int64_t ba
         pa.yin = cur;
         pa.ybits = y0_mode == 3 ? bits : nullptr;
         pa.one = one;
-        pa.ready = y0_mode == 3 ? bits_ready : nullptr;
+        pa.ready = (y0_mode == 3 || host_streamed) ? bits_ready : nullptr;
         pa.ready_rows = ready_rows;
         pa.yout = bufs[nxt_i];
         pa.rows = lists[li];
@@ -884,6 +944,7 @@ static snicit_status infer_core(snicit_network* net, const float* y0, int64_t ba
         pa.rval = net->rval.p;
         pa.n_const = cnt + CNT_PFCONST;
         CUDA_TRY(launch_pre_fused(pa, net->pf_layers_h.data(), net->num_sms, st));
+        if (host_streamed) CUDA_TRY(cudaStreamWaitEvent(st, net->cev[1], 0));  // Ya reused after this
         if (prof) CUDA_TRY(cudaEventRecord(net->lev[1], st));
         ++launches;
         circ_layers += tt;
@@ -1007,9 +1068,13 @@ static snicit_status infer_core(snicit_network* net, const float* y0, int64_t ba
         CUDA_TRY(launch_fill_u8(net->ne_row.p, R, 0, st));
         float* yhat = bufs[nxt_i];
         float* yhat_other = bufs[nxt_i ^ 1];
+        CUDA_TRY(cudaMemsetAsync(net->ctr64.p, 0, sizeof(unsigned long long) * C64_N, st));
+        if (opt.timing) CUDA_TRY(cudaEventRecord(net->ev[6], st));
         CUDA_TRY(launch_map_residual(cur, N, list_cur, cnt_cur, net->cent.p, cnt + CNT_NCENT, net->M.p, net->cslot.p,
                                      net->ne_row.p, net->flag_pos.p, yhat, net->cbuf0.p, R, net->num_sms, st,
-                                     net->rconst.p, net->rval.p));
+                                     net->rconst.p, net->rval.p, net->ctr64.p + C64_RES_NNZ));
+        if (opt.timing) CUDA_TRY(cudaEventRecord(net->ev[7], st));
+        net->ev_map = opt.timing != 0;
         int* rlist = net->res0.p;
         int* rlist_nxt = net->res1.p;
         int* rcnt = cnt + CNT_RES0;
@@ -1098,6 +1163,8 @@ static snicit_status infer_core(snicit_network* net, const float* y0, int64_t ba
             pa.ne_row = net->ne_row.p;
             pa.alive_count = cnt + CNT_ALIVE;
             pa.cdone = cdone;
+            pa.ctr64 = net->ctr64.p;
+            pa.res_sparse = opt.res_sparse;
             CUDA_TRY(cudaMemsetAsync(cnt + CNT_WORK, 0, 2 * sizeof(int), st));
             pa.force_ell = opt.kernel == SNICIT_KERNEL_ELL ? 1 : 0;
             // cluster (DSMEM) trajectory when every post layer is circulant and partition-compatible
@@ -1130,7 +1197,10 @@ static snicit_status infer_core(snicit_network* net, const float* y0, int64_t ba
                     CUDA_TRY(launch_acconst(pa, s, st));
                     ++launches;
                 }
+                if (opt.timing) CUDA_TRY(cudaEventRecord(net->ev[8], st));
                 CUDA_TRY(launch_residual_traj(pa, R, net->num_sms, st));
+                if (opt.timing) CUDA_TRY(cudaEventRecord(net->ev[9], st));
+                net->ev_res = opt.timing != 0;
                 ++launches;
             }
         }
@@ -1224,6 +1294,17 @@ static snicit_status infer_core(snicit_network* net, const float* y0, int64_t ba
         cudaEventElapsedTime(&ms, net->ev[0], net->ev[5]);
         net->stats.t_total_ms = ms;
     }
+    net->stats.t_map_ms = net->stats.t_residual_ms = -1.0;
+    if (net->ev_map) {
+        float ms;
+        cudaEventElapsedTime(&ms, net->ev[6], net->ev[7]);
+        net->stats.t_map_ms = ms;
+    }
+    if (net->ev_res) {
+        float ms;
+        cudaEventElapsedTime(&ms, net->ev[8], net->ev[9]);
+        net->stats.t_residual_ms = ms;
+    }
     // a host buffer is involved (y0 read by an async H2D copy, y_out filled by an async D2H copy):
     // return only when the caller may read / reuse it
     if (y0_mode == 1 || (y_out && !y_out_on_device)) CUDA_TRY(cudaStreamSynchronize(st));
@@ -1266,36 +1347,8 @@ snicit_status snicit_infer_packed(snicit_network* net, const uint32_t* y0_bits, 
     if (!bits_on_device && R > 0) {
         CUDA_TRY(net->bits.ensure((size_t)R * W));
         if (direct) {
-            // streamed upload: the copy engine delivers chunks of rows on a side stream while the
-            // row-resident kernel runs; each chunk is followed by its ready flag (the kernel polls it
-            // before loading a row of the chunk), so the upload overlaps the compute
-            // geometric chunks: chunk c = rows [b (2^c - 1), b (2^(c+1) - 1)), b = kChunk0 -- the first
-            // rows arrive within microseconds and the whole batch takes a handful of API calls
-            constexpr int kChunk0 = 512;
-            int nch = 0;
-            while ((long long)kChunk0 * ((1LL << nch) - 1) < R) ++nch;
-            if (!net->copy_stream) CUDA_TRY(cudaStreamCreateWithFlags(&net->copy_stream, cudaStreamNonBlocking));
-            for (auto& e : net->cev)
-                if (!e) CUDA_TRY(cudaEventCreateWithFlags(&e, cudaEventDisableTiming));
-            if (!net->h_ones) {
-                CUDA_TRY(cudaMallocHost(&net->h_ones, sizeof(int)));
-                *net->h_ones = 1;
-            }
-            CUDA_TRY(net->bits_ready.ensure((size_t)std::max(nch, 1)));
-            CUDA_TRY(cudaMemsetAsync(net->bits_ready.p, 0, sizeof(int) * std::max(nch, 1), net->stream));
-            CUDA_TRY(cudaEventRecord(net->cev[0], net->stream));
-            CUDA_TRY(cudaStreamWaitEvent(net->copy_stream, net->cev[0], 0));
-            for (int c = 0; c < nch; ++c) {
-                const size_t r0 = (size_t)kChunk0 * ((1ull << c) - 1);
-                const size_t nr = std::min<size_t>((size_t)kChunk0 << c, R - r0);
-                CUDA_TRY(cudaMemcpyAsync(net->bits.p + r0 * W, y0_bits + r0 * W, sizeof(uint32_t) * nr * W,
-                                         cudaMemcpyHostToDevice, net->copy_stream));
-                CUDA_TRY(cudaMemcpyAsync(net->bits_ready.p + c, net->h_ones, sizeof(int), cudaMemcpyHostToDevice,
-                                         net->copy_stream));
-            }
-            CUDA_TRY(cudaEventRecord(net->cev[1], net->copy_stream));
-            ready = net->bits_ready.p;
-            ready_rows = kChunk0;
+            // streamed upload (the copy engine delivers chunks while the row-resident kernel runs)
+            CUDA_TRY(stream_upload(net, net->bits.p, y0_bits, sizeof(uint32_t) * W, R, &ready, &ready_rows));
             streamed = true;
         } else {
             CUDA_TRY(cudaMemcpyAsync(net->bits.p, y0_bits, sizeof(uint32_t) * (size_t)R * W, cudaMemcpyHostToDevice,
@@ -1392,6 +1445,18 @@ snicit_status snicit_stats(snicit_network* net, snicit_stats_t* out) {
     if (net->last_pre_const) {
         CUDA_TRY(read_counter(net, CNT_CCOUNT, &v));
         net->stats.pre_const_rows = v;
+    }
+    net->stats.res_nnz_at_t = net->stats.res_full_rl = net->stats.res_sparse_rl = 0;
+    net->stats.res_sparse_out = net->stats.res_scalar_rl = 0;
+    if (net->last_converted) {
+        unsigned long long c64[C64_N];
+        CUDA_TRY(cudaMemcpyAsync(c64, net->ctr64.p, sizeof(c64), cudaMemcpyDeviceToHost, net->stream));
+        CUDA_TRY(cudaStreamSynchronize(net->stream));
+        net->stats.res_nnz_at_t = (int64_t)c64[C64_RES_NNZ];
+        net->stats.res_full_rl = (int64_t)c64[C64_FULL_RL];
+        net->stats.res_sparse_rl = (int64_t)c64[C64_SPARSE_RL];
+        net->stats.res_sparse_out = (int64_t)c64[C64_SPARSE_OUT];
+        net->stats.res_scalar_rl = (int64_t)c64[C64_SCALAR_RL];
     }
     if (net->last_pre_fused) {
         CUDA_TRY(read_counter(net, CNT_PFCONST, &v));

@@ -1,0 +1,254 @@
+"""GPU parity for the round-2 pieces of the path, through the C ABI against the CPU oracle:
+
+* row sharding: G shards run one after another on one GPU with row_offset ("fake
+  multi-GPU") give the category set of G = 1 and of the oracle, and the device category export;
+* the two-rank bench step end to end through libsnicit (gloo hook, both ranks on cuda:0);
+* the sparse-entry residue form (north_star "only the nonzero residual entries are propagated") on
+  inputs whose residues are sparse, bit-identical to the dense form and the oracle;
+* the approximate mode (near-zero residue pruning) element by element vs the oracle;
+* the SNICIT_CSR loader branch; a non-blocking stream while the legacy default stream is busy.
+"""
+import json
+import os
+import subprocess
+import sys
+
+import numpy as np
+import pytest
+
+torch = pytest.importorskip("torch")
+
+import oracle  # noqa: E402
+from paper_conf_icpp_jiangh0h23_b200 import CSR_FORMAT, SnicitNetwork, shard_capacity, shard_rows  # noqa: E402
+from workload import sdgc  # noqa: E402
+from workload.sdgc import Network  # noqa: E402
+
+pytestmark = pytest.mark.gpu
+
+ATOL, RTOL = 1e-4, 1e-5
+ROOT = os.path.dirname(os.path.dirname(os.path.abspath(__file__)))
+
+
+@pytest.fixture(scope="module", autouse=True)
+def _need_gpu():
+    if not torch.cuda.is_available():
+        pytest.skip("no CUDA device")
+    from paper_conf_icpp_jiangh0h23_b200 import build
+    build.build()
+
+
+def _infer(g, Y0, t, s=32, row_offset=0, **opt):
+    y0 = torch.from_numpy(np.ascontiguousarray(Y0)).cuda()
+    out = torch.empty_like(y0)
+    g.infer(y0, t=t, s=s, y_out=out, row_offset=row_offset, **opt)
+    return out.cpu().numpy(), g.categories(), g.stats()
+
+
+# ------------------------------------------------------------------------------ sharding
+
+@pytest.mark.parametrize("N,L,B,t", [(4096, 60, 6000, 10), (4096, 60, 6000, 30), (1024, 120, 2000, 5)])
+def test_sharded_inference_matches_single_gpu_and_oracle(N, L, B, t):
+    """Rows are independent (Eq. 1), clustering runs per shard (reading R14): for G = 1, 2, 4,
+    8 contiguous shards with row_offset, the concatenated category sets are identical to G = 1 and to the
+    oracle's, and every shard's activations are within tolerance of the plain oracle."""
+    net = sdgc.gen_network(N, L, "radix")
+    Y0 = sdgc.gen_inputs(N, B)
+    plain = oracle.layers_f32_fast(net, Y0)
+    ref_cats = oracle.categories(plain)
+    with SnicitNetwork.from_network(net) as g:
+        g.set_stream(torch.cuda.current_stream())
+        for G in (1, 2, 4, 8):
+            cats, Ys = [], []
+            for r in range(G):
+                a, b = shard_rows(B, G, r)
+                Y, c, st = _infer(g, Y0[a:b], t, row_offset=a)
+                assert np.all((c >= a) & (c < b))
+                cats.append(c)
+                Ys.append(Y)
+                # device export of this shard's categories (the all-gather buffer)
+                cap = shard_capacity(B, G)
+                buf = torch.full((1 + cap,), -7, dtype=torch.int64, device="cuda")
+                g.categories_device(buf)
+                torch.cuda.synchronize()
+                hb = buf.cpu().numpy()
+                assert hb[0] == len(c) and np.array_equal(hb[1:1 + len(c)], c) and np.all(hb[1 + len(c):] == -7)
+            assert np.array_equal(np.concatenate(cats), ref_cats), f"G = {G}"
+            np.testing.assert_allclose(np.concatenate(Ys), plain, atol=ATOL, rtol=RTOL)
+
+
+def test_bench_two_ranks_gloo_hook():
+    """bench.py --gpus 2 (it launches torchrun itself) with SNICIT_DIST_BACKEND=gloo: both ranks share
+    cuda:0, each infers its row shard through libsnicit, the padded category buffers are all-gathered;
+    the line reports n_gpus 2 and the category count of a one-rank run."""
+    env = dict(os.environ, SNICIT_DIST_BACKEND="gloo")
+    common = ["--config", "C1", "--quick", "--steps", "2", "--warmup", "3"]
+
+    def run(extra, e):
+        p = subprocess.run([sys.executable, os.path.join(ROOT, "bench.py")] + common + extra, env=e,
+                           capture_output=True, text=True, timeout=900, cwd=ROOT)
+        assert p.returncode == 0, p.stderr[-3000:]
+        lines = [ln for ln in p.stdout.splitlines() if ln.startswith("{")]
+        assert len(lines) == 1, p.stdout[-2000:]
+        return json.loads(lines[0])
+
+    two = run(["--gpus", "2"], env)
+    one = run(["--gpus", "1"], dict(os.environ))
+    assert two["n_gpus"] == 2 and one["n_gpus"] == 1
+    assert two["categories"] == one["categories"] > 0
+    assert len(two["per_rank"]) == 2 and sum(r["rows"] for r in two["per_rank"]) == 2000
+    assert two["config"]["global_batch"] == one["config"]["global_batch"] == 2000
+
+
+# ------------------------------------------------------------------------------ sparse-entry residues
+
+def _near_duplicate_inputs(N, B, flips, seed):
+    """Rows 0..31 are 8 distinct base images (the sampled rows: they become the centroids); every other
+    row is a base image with `flips` pixels toggled, so its residue at t = 0 has ~`flips` non-zeros."""
+    rs = np.random.RandomState(seed)
+    base = sdgc.gen_inputs(N, 8, row0=seed * 8)
+    Y = np.repeat(base, (B + 7) // 8, axis=0)[:B].copy()
+    Y[:32] = base[np.arange(32) % 8]
+    for r in range(32, B):
+        Y[r] = base[r % 8]
+        k = rs.choice(N, flips, replace=False)
+        Y[r, k] = 1.0 - Y[r, k]
+    return Y.astype(np.float32)
+
+
+@pytest.mark.parametrize("N,L,B,t,flips", [(4096, 24, 600, 0, 3), (4096, 24, 600, 1, 1), (1024, 30, 800, 0, 2),
+                                           (16384, 10, 64, 0, 5)])
+def test_sparse_entry_residues(N, L, B, t, flips):
+    """Residue rows with few non-zeros propagate only the outputs their non-zeros touch (fused post mode,
+    circulant layers): bit-identical to the dense-row form (res_sparse = 0) and to the oracle's SNICIT
+    pipeline; the stats show sparse row-layers evaluated."""
+    net = sdgc.gen_network(N, L, "radix")
+    Y0 = _near_duplicate_inputs(N, B, flips, N + t)
+    ref = oracle.snicit(net, Y0, t=t)
+    plain = oracle.layers_f32(net, Y0)
+    with SnicitNetwork.from_network(net) as g:
+        g.set_stream(torch.cuda.current_stream())
+        Ys, cs, sts = _infer(g, Y0, t, res_sparse=1)
+        Yd, cd, std = _infer(g, Y0, t, res_sparse=0)
+    assert sts["residual_at_t"] > 0 and sts["res_sparse_rl"] > 0 and std["res_sparse_rl"] == 0
+    assert sts["res_nnz_at_t"] <= sts["residual_at_t"] * (flips if t == 0 else 32 * flips)
+    assert np.array_equal(Ys, Yd) and np.array_equal(cs, cd)
+    assert np.array_equal(Ys, ref["Y"]) and np.array_equal(cs, ref["categories"])
+    assert np.array_equal(cs, oracle.categories(plain))
+    np.testing.assert_allclose(Ys, plain, atol=ATOL, rtol=RTOL)
+
+
+def test_sparse_entry_residues_per_n_weights_and_bias():
+    """The sparse form with per-n weights and per-neuron biases (non-uniform circulant layers)."""
+    N, L, B = 2048, 12, 300
+    rs = np.random.RandomState(9)
+    nu = np.array([[1, 32, 64][l % 3] for l in range(L)], np.int32)
+    w = rs.uniform(0.02, 0.09, size=(L, 32)).astype(np.float32)
+    bias = rs.uniform(-0.4, -0.1, size=L * N).astype(np.float32)
+    cn = sdgc.CirculantNetwork(N=N, L=L, nu=nu, w=w, bias=bias, ymax=32.0)
+    net = cn.to_network()
+    base = (rs.uniform(size=(8, N)) < 0.3).astype(np.float32) * 3.0
+    Y0 = base[np.arange(B) % 8].copy()
+    for r in range(32, B):
+        k = rs.choice(N, 2, replace=False)
+        Y0[r, k] += 1.0
+    ref = oracle.snicit(net, Y0, t=0)
+    with SnicitNetwork.from_network(net) as g:
+        g.set_stream(torch.cuda.current_stream())
+        Ys, cs, sts = _infer(g, Y0, 0, res_sparse=1)
+        Yd, cd, _ = _infer(g, Y0, 0, res_sparse=0)
+    assert sts["res_sparse_rl"] > 0
+    assert np.array_equal(Ys, Yd) and np.array_equal(Ys, ref["Y"]) and np.array_equal(cs, ref["categories"])
+
+
+# ------------------------------------------------------------------------------ approximate mode (f2)
+
+@pytest.mark.parametrize("prune_eps", [0.1, 0.5])
+@pytest.mark.parametrize("pm", [0, 1])
+def test_prune_eps_matches_oracle(prune_eps, pm):
+    """Near-zero residue pruning (|v| <= prune_eps -> 0, reading R8) is outside exact parity
+    with the plain result, but the GPU's approximate pipeline equals the oracle's approximate pipeline
+    (oracle_post_layer's prune_eps branch) element by element, fused and per-layer post modes."""
+    net = sdgc.gen_network(1024, 40, "radix")
+    Y0 = sdgc.gen_inputs(1024, 1500)
+    ref = oracle.snicit(net, Y0, t=3, prune_eps=prune_eps)
+    with SnicitNetwork.from_network(net) as g:
+        g.set_stream(torch.cuda.current_stream())
+        Y, cats, st = _infer(g, Y0, 3, prune_eps=prune_eps, post_mode=pm)
+    assert st["residual_at_t"] > 0
+    assert np.array_equal(Y, ref["Y"]) and np.array_equal(cats, ref["categories"])
+
+
+# ------------------------------------------------------------------------------ loader / streams
+
+def test_csr_loader_equals_csc():
+    """SNICIT_CSR (per input k its outputs j): transposed on load, each output column ordered by
+    ascending k.  A CSC net stored in ascending-k order loads to the same plan: identical results."""
+    net = sdgc.gen_network(1024, 12, "random")  # columns stored ascending (workload recipe)
+    N, L = net.N, net.L
+    ptr_r, idx_r, val_r = [0], [], []
+    for l in range(L):
+        p, idx, val, _ = net.layer(l)
+        cols = np.repeat(np.arange(N), np.diff(p))
+        order = np.lexsort((cols, idx))  # by input k, then output j
+        k_sorted = idx[order]
+        idx_r.extend(cols[order].tolist())
+        val_r.extend(val[order].tolist())
+        counts = np.bincount(k_sorted, minlength=N)
+        base = ptr_r[-1]
+        ptr_r.extend((base + np.cumsum(counts)).tolist())
+        if l < L - 1:
+            ptr_r.append(ptr_r[-1])
+    ptr_r = np.array(ptr_r, np.int64)
+    csr = Network(N=N, L=L, ptr=ptr_r, idx=np.array(idx_r, np.int32), val=np.array(val_r, np.float32),
+                  bias=net.bias, ymax=net.ymax, mode="csr")
+    Y0 = sdgc.gen_inputs(N, 500)
+    plain = oracle.layers_f32(net, Y0)
+    with SnicitNetwork.from_network(net) as g1:
+        g1.set_stream(torch.cuda.current_stream())
+        Ya, ca, _ = _infer(g1, Y0, 4)
+    with SnicitNetwork(N, L, csr.ptr, csr.idx, csr.val, csr.bias, csr.ymax, fmt=CSR_FORMAT) as g2:
+        g2.set_stream(torch.cuda.current_stream())
+        Yb, cb, _ = _infer(g2, Y0, 4)
+        Yu, cu, _ = _infer(g2, Y0, L)
+    assert np.array_equal(Ya, Yb) and np.array_equal(ca, cb)
+    assert np.array_equal(Yu, plain) and np.array_equal(cu, oracle.categories(plain))
+
+
+@pytest.mark.parametrize("pre_fused", [0, 1])
+def test_nonblocking_stream_with_busy_default_stream(pre_fused):
+    """All work of a handle (including the first-call workspace initialisation of the self-clearing
+    counters) is ordered on the handle's stream: a fresh non-blocking stream while the legacy default
+    stream is busy gives the oracle's result (per-layer path: column-streaming + segmented kernels)."""
+    N, L, B = 16384, 8, 48
+    net = sdgc.gen_network(N, L, "radix")
+    Y0 = sdgc.gen_inputs(N, B)
+    plain = oracle.layers_f32(net, Y0)
+    y0 = torch.from_numpy(Y0).cuda()
+    big = torch.randn(8192, 8192, device="cuda")
+    torch.cuda.synchronize()
+    s = torch.cuda.Stream()  # created cudaStreamNonBlocking
+    with SnicitNetwork.from_network(net) as g:
+        g.set_stream(s)
+        for _ in range(3):
+            for _ in range(20):  # keep the legacy default stream busy
+                big = big @ big
+                big = big / big.norm()
+            out = torch.empty_like(y0)
+            with torch.cuda.stream(s):
+                g.infer(y0, t=L, s=32, y_out=out, pre_fused=pre_fused)
+                cats = g.categories()
+                s.synchronize()
+                got = out.cpu().numpy()
+            assert np.array_equal(got, plain) and np.array_equal(cats, oracle.categories(plain))
+
+
+def test_misaligned_device_pointer_rejected():
+    net = sdgc.gen_network(1024, 4, "radix")
+    Y0 = sdgc.gen_inputs(1024, 9)
+    with SnicitNetwork.from_network(net) as g:
+        flat = torch.from_numpy(np.ascontiguousarray(Y0)).cuda().flatten()
+        buf = torch.empty(9 * 1024 + 1, dtype=torch.float32, device="cuda")
+        buf[1:].copy_(flat)
+        y0 = buf[1:].view(9, 1024)  # contiguous, 4-byte offset
+        with pytest.raises(Exception):
+            g.infer(y0, t=2, s=8)
