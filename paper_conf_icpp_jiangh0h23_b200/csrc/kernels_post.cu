@@ -397,7 +397,8 @@ __global__ void __launch_bounds__(kPostThreads, 2) residual_traj_kernel(PostArgs
     extern __shared__ __align__(128) float sm[];
     __shared__ int s_p;
     __shared__ int s_nz[3];   // per-layer non-zero count of the dense form (rotating slots)
-    __shared__ int s_cnt[2];  // sparse form scratch
+    __shared__ int s_cnt[3];  // sparse form: [0], [1] sp_layer's counters, [2] sp_list's (distinct slots:
+                              // sp_layer may follow sp_list with no barrier in between)
     const int N = a.N;
     const int h = post_halo(N);
     const int dup = h == N;
@@ -418,6 +419,7 @@ __global__ void __launch_bounds__(kPostThreads, 2) residual_traj_kernel(PostArgs
         float* cur = sm;
         float* nxt = sm + N + h;
         stage_row(cur, a.yhat + (size_t)row * N, N);
+        if (threadIdx.x < 3) s_nz[threadIdx.x] = 0;
         __syncthreads();
         fill_halo(cur, N, h);
         __syncthreads();
@@ -429,7 +431,7 @@ __global__ void __launch_bounds__(kPostThreads, 2) residual_traj_kernel(PostArgs
         int nnz = -1, li = 0;
         bool listed = false, nxt_zero = false;
         if (a.res_sparse) {
-            nnz = sp_list(cur, N, lsts[0], cap, &s_cnt[0]);
+            nnz = sp_list(cur, N, lsts[0], cap, &s_cnt[2]);
             listed = nnz <= cap;
         }
         PL Ld = load_pl(a.layers + a.t);
@@ -439,6 +441,7 @@ __global__ void __launch_bounds__(kPostThreads, 2) residual_traj_kernel(PostArgs
             const float* ac = a.a_all + ((size_t)(l - a.t) * a.s + slot) * N;
             const bool sparse = a.res_sparse && listed && Ld.kind == 1 && !a.force_ell;
             int cnt;
+            if (threadIdx.x == 0) s_nz[(l + 1) % 3] = 0;  // the next layer's slot (last read two barriers ago)
             if (sparse) {
                 if (!nxt_zero)
                     for (int k = threadIdx.x; k < N; k += blockDim.x) nxt[k] = 0.0f;
@@ -459,7 +462,6 @@ __global__ void __launch_bounds__(kPostThreads, 2) residual_traj_kernel(PostArgs
                     c_sout += (unsigned long long)nt;
                 }
             } else {
-                if (threadIdx.x == 0) s_nz[(l + 1) % 3] = 0;  // slot of the next layer (read two barriers ago)
                 const int mine = post_row_layer<MODE_RESIDUAL, 17, 16, 1>(Ld, N, dup, a.ymax, a.prune_eps, cur, nxt,
                                                                           ac, nullptr, a.force_ell);
                 const int wsum = __reduce_add_sync(0xffffffffu, mine);
@@ -492,7 +494,7 @@ __global__ void __launch_bounds__(kPostThreads, 2) residual_traj_kernel(PostArgs
             fill_halo(nxt, N, h);
             __syncthreads();
             if (a.res_sparse && !listed && nnz <= cap) {  // the dense output is sparse: list it
-                nnz = sp_list(nxt, N, lsts[li], cap, &s_cnt[0]);
+                nnz = sp_list(nxt, N, lsts[li], cap, &s_cnt[2]);
                 listed = true;
             }
             float* tmp = cur;

@@ -60,7 +60,10 @@ def allgather_categories_padded(local_buf, group=None):
 
     world = dist.get_world_size(group)
     out = torch.empty((world, local_buf.numel()), dtype=local_buf.dtype, device=local_buf.device)
-    dist.all_gather_into_tensor(out, local_buf, group=group)
+    if dist.get_backend(group) == "nccl":
+        dist.all_gather_into_tensor(out, local_buf, group=group)
+    else:  # gloo (CPU tests, the shared-GPU hook): list form
+        dist.all_gather(list(out.unbind(0)), local_buf, group=group)
     return out
 
 

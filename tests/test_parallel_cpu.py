@@ -9,7 +9,8 @@ import torch
 import torch.distributed as dist
 import torch.multiprocessing as mp
 
-from paper_conf_icpp_jiangh0h23_b200.parallel import allgather_categories, shard_rows
+from paper_conf_icpp_jiangh0h23_b200.parallel import (allgather_categories, allgather_categories_padded,
+                                                       assemble_categories, shard_capacity, shard_rows)
 
 
 def _free_port():
@@ -27,6 +28,15 @@ def _worker(rank, world, port, B, cats, q):
     a, b = shard_rows(B, world, rank)
     local = torch.tensor([c for c in cats if a <= c < b], dtype=torch.int64)
     got = allgather_categories(local)
+    # the padded device-export form: [count, ids..., junk] per rank, one collective
+    cap = shard_capacity(B, world)
+    buf = torch.full((1 + cap,), -5, dtype=torch.int64)
+    buf[0] = local.numel()
+    buf[1:1 + local.numel()] = local
+    gathered = allgather_categories_padded(buf)
+    assert tuple(gathered.shape) == (world, 1 + cap)
+    got2 = assemble_categories(gathered)
+    assert got2.tolist() == got.tolist()
     q.put((rank, got.tolist(), (a, b)))
     dist.barrier()
     dist.destroy_process_group()
