@@ -70,9 +70,9 @@ def parse(argv=None):
     p.add_argument("--no-residue", action="store_true", help="skip the residue-regime study (C2, t = 10)")
     p.add_argument("--no-general", action="store_true", help="skip the general-CSC study (C2 perm)")
     p.add_argument("--residue-t", type=int, default=10)
-    p.add_argument("--pre-fused", type=int, default=1, choices=[0, 1, 2],
-                   help="options.pre_fused: 1 = row-resident pre phase (default), 2 = without the constant-row "
-                        "shortcut, 0 = one launch per layer")
+    p.add_argument("--pre-fused", type=int, default=1, choices=[0, 1, 2, 3],
+                   help="options.pre_fused: 1 = row-resident pre phase (default; cluster form for N >= 16384), "
+                        "2 = without the constant-row shortcut, 3 = never the cluster form, 0 = one launch per layer")
     p.add_argument("--no-variants", action="store_true", help="skip the pre_fused = 2 / 0 roofline variants")
     p.add_argument("--cpu-seconds", type=float, default=15.0, help="target CPU work of the oracle sample")
     p.add_argument("--quick", action="store_true", help="value only (no e2e/uncompressed/variants/studies)")
@@ -577,7 +577,9 @@ def run_snicit(args):
             return {"bound": "alu", "achieved": achieved, "peak": FMA_PEAK_TFLOPS, "unit": "TFLOP/s",
                     "frac": achieved / FMA_PEAK_TFLOPS, "traffic": traffic,
                     "traffic_unit": "bytes per launch (ncu dram read + write)", "traffic_source": traffic_src,
-                    "kernel": "pre_fused_kernel (row-resident a1: layers 0..t-1 of a row in shared memory)",
+                    "kernel": ("pre_cluster_kernel (row-resident a1, a row split over a cluster of N/8192 CTAs, "
+                               "DSMEM exchange)") if st_["pre_fused"] == 2 else
+                              "pre_fused_kernel (row-resident a1: layers 0..t-1 of a row in shared memory)",
                     "peak_source": FMA_PEAK_SRC, "launches": int(len(pm_)), "avg_launch_ms": kms,
                     "algorithmic_flops": flops, "full_row_layers": int(st_["pre_full_rows"]),
                     "const_rows": int(st_["pre_const_rows"]),

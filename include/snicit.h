@@ -87,14 +87,18 @@ typedef struct {
                                when every post layer is circulant with uniform weights and bias
                                (such a layer maps a constant row to a constant row; bit-identical
                                results); 0 = always the full-row evaluation */
-    int32_t pre_fused;      /* pre-convergence layers 0..t-1 (Eq. 1): 1 = row-resident fused kernel -- a
+    int32_t pre_fused;      /* pre-convergence layers 0..t-1 (Eq. 1): 1 = row-resident fused kernel (rows of
+                               N = 16384 / 32768 / 65536 split over a thread-block cluster of N/8192 CTAs
+                               exchanging layer outputs through distributed shared memory; 3 = the same but
+                               never the cluster form, i.e. one CTA per row where that exists) -- a
                                CTA keeps one row in shared memory for all t layers (Y0 read and Y(t)
                                written once) and carries a row that became constant (all elements
                                equal) by one scalar fma chain per layer (R26, exact); 2 = the same kernel
                                without the constant-row shortcut (every live row evaluated in full);
                                0 = one kernel launch per layer.  Used when every layer < t is circulant
                                with 32 taps, uniform weight and uniform bias, and N/32 is one of
-                               32..512 (N = 1024..16384); otherwise the per-layer kernels run.
+                               32..512 (N = 1024..16384) or the cluster form supports every stride
+                               (N = 16384..65536); otherwise the per-layer kernels run.
                                Results are bit-identical in every mode (tested). */
     int32_t pre_const;      /* per-layer pre-convergence path (pre_fused = 0 or not applicable): 1 = a row
                                whose outputs are all equal leaves the active list and is carried by one
@@ -123,7 +127,9 @@ typedef struct {
     int64_t kernel_launches;  /* kernels launched by this infer */
     int32_t const_centroids;  /* centroids carried through the post layers as constant rows
                                  (options.post_const) */
-    int32_t pre_fused;        /* the pre-convergence layers ran in the row-resident fused kernel */
+    int32_t pre_fused;        /* the pre-convergence layers ran in the row-resident kernel: 1 = one CTA per
+                                 row (kernels_pre_fused.cu), 2 = a cluster of CTAs per row
+                                 (kernels_pre_cluster.cu), 0 = one launch per layer */
     int32_t pre_const_rows;   /* fused: rows that became constant before t (carried by a scalar) */
     int64_t pre_full_rows;    /* fused: full-row layer evaluations (row x layer, 32*N fma each) */
     int64_t res_nnz_at_t;     /* non-zero entries of the non-empty residue rows right after conversion */

@@ -731,10 +731,27 @@ extern "C" {
 
 // Row-resident pre phase applicable?  (kernels_pre_fused.cu: circulant layers < t with 32 taps,
 // uniform weight and bias, N / 32 in 32..512, t <= kPfMaxLayers, smem fits); *H = circular halo
-static bool pf_plan(const snicit_network* net, int tt, const snicit_options& opt, int R, int* H, int* gen) {
+// *cluster: the row is split over a thread-block cluster (kernels_pre_cluster.cu: N = 16384 / 32768 /
+// 65536, every layer's stride supported; pre_fused = 3 keeps the single-CTA kernel where it exists);
+// *bits_ok: packed input rows can be read by the chosen kernel
+static bool pf_plan(const snicit_network* net, int tt, const snicit_options& opt, int R, int* H, int* gen,
+                    bool* cluster = nullptr, bool* bits_ok = nullptr) {
     const int N = net->N;
-    bool pf = opt.pre_fused != 0 && tt > 0 && tt <= kPfMaxLayers && R > 0 && opt.kernel == SNICIT_KERNEL_AUTO &&
-              pre_fused_threads(N) > 0;
+    if (cluster) *cluster = false;
+    if (bits_ok) *bits_ok = true;
+    const bool base_ok = opt.pre_fused != 0 && tt > 0 && tt <= kPfMaxLayers && R > 0 && opt.kernel == SNICIT_KERNEL_AUTO;
+    if (base_ok && opt.pre_fused != 3 && pre_cluster_supported(N)) {
+        bool ok = true;
+        for (int l = 0; l < tt && ok; ++l) ok = net->pf_elig[l] != 0 && pre_cluster_class(N, net->plan[l].nu) >= 0;
+        if (ok) {
+            if (cluster) *cluster = true;
+            if (bits_ok) *bits_ok = N % 128 == 0 && pre_cluster_class(N, net->plan[0].nu) <= 1;  // W partition at layer 0
+            *H = 0;
+            *gen = 0;
+            return true;
+        }
+    }
+    bool pf = base_ok && pre_fused_threads(N) > 0;
     for (int l = 0; l < tt && pf; ++l) pf = net->pf_elig[l] != 0;
     int h = 96, g = 0;  // nu == 1 windows read 47 past an item, head items write 68; STR 31*nu
     if (pf) {
@@ -820,7 +837,7 @@ static snicit_status infer_core(snicit_network* net, const float* y0, int64_t ba
         return fail(SNICIT_E_INVALID_ARG, "bad eta/eps/prune_eps");
     if (opt.kernel < 0 || opt.kernel > SNICIT_KERNEL_CIRC_SMEM) return fail(SNICIT_E_INVALID_ARG, "bad kernel option");
     if (opt.post_mode < 0 || opt.post_mode > 1) return fail(SNICIT_E_INVALID_ARG, "bad post_mode");
-    if (opt.pre_fused < 0 || opt.pre_fused > 2) return fail(SNICIT_E_INVALID_ARG, "bad pre_fused");
+    if (opt.pre_fused < 0 || opt.pre_fused > 3) return fail(SNICIT_E_INVALID_ARG, "bad pre_fused");
     if (opt.pre_const < 0 || opt.pre_const > 1) return fail(SNICIT_E_INVALID_ARG, "bad pre_const");
     if (opt.res_sparse < 0 || opt.res_sparse > 1) return fail(SNICIT_E_INVALID_ARG, "bad res_sparse");
     if (opt.kernel == SNICIT_KERNEL_ELL && !net->has_ell)
@@ -904,12 +921,14 @@ static snicit_status infer_core(snicit_network* net, const float* y0, int64_t ba
     }
     // row-resident fused pre phase (kernels_pre_fused.cu): one launch for layers 0..t-1
     int pf_H = 96, pf_gen = 0;
-    const bool pf = pf_plan(net, tt, opt, R, &pf_H, &pf_gen);
+    bool pf_cluster = false, pf_bits_ok = true;
+    const bool pf = pf_plan(net, tt, opt, R, &pf_H, &pf_gen, &pf_cluster, &pf_bits_ok);
+    if (y0_mode == 3 && pf && !pf_bits_ok) return fail(SNICIT_E_STATE, "packed rows not readable by the pre-phase kernel");
     if (y0_mode == 3 && !pf && R > 0) return fail(SNICIT_E_STATE, "packed rows without the row-resident kernel");
     net->last_pre_fused = pf;
     const int dead_zeroed = (pf && y_out_on_device && y_out && drop) ? 1 : 0;  // y_out rows of dead rows
     net->last_dead_zeroed = dead_zeroed != 0;
-    stats.pre_fused = pf ? 1 : 0;
+    stats.pre_fused = pf ? (pf_cluster ? 2 : 1) : 0;
     if (R > 0) CUDA_TRY(cudaMemsetAsync(net->rconst.p, 0, (size_t)R, st));  // rows constant at t (R26)
     if (pf) {
         if (prof) {
@@ -925,7 +944,7 @@ static snicit_status infer_core(snicit_network* net, const float* y0, int64_t ba
         pa.H = pf_H;
         pa.ymax = net->ymax;
         pa.drop = drop ? 1 : 0;
-        pa.const_skip = opt.pre_fused == 1 ? 1 : 0;
+        pa.const_skip = opt.pre_fused != 2 ? 1 : 0;
         pa.gen_str = pf_gen;
         pa.yin = cur;
         pa.ybits = y0_mode == 3 ? bits : nullptr;
@@ -943,7 +962,10 @@ static snicit_status infer_core(snicit_network* net, const float* y0, int64_t ba
         pa.rconst = net->rconst.p;
         pa.rval = net->rval.p;
         pa.n_const = cnt + CNT_PFCONST;
-        CUDA_TRY(launch_pre_fused(pa, net->pf_layers_h.data(), net->num_sms, st));
+        if (pf_cluster)
+            CUDA_TRY(launch_pre_cluster(pa, net->pf_layers_h.data(), net->num_sms, st));
+        else
+            CUDA_TRY(launch_pre_fused(pa, net->pf_layers_h.data(), net->num_sms, st));
         if (host_streamed) CUDA_TRY(cudaStreamWaitEvent(st, net->cev[1], 0));  // Ya reused after this
         if (prof) CUDA_TRY(cudaEventRecord(net->lev[1], st));
         ++launches;
@@ -1340,7 +1362,8 @@ snicit_status snicit_infer_packed(snicit_network* net, const uint32_t* y0_bits, 
     else
         snicit_default_options(&o);
     int H = 0, gen = 0;
-    const bool direct = N % 128 == 0 && pf_plan(net, std::min(t, net->L), o, R, &H, &gen);
+    bool cl = false, bits_ok = true;
+    const bool direct = N % 128 == 0 && pf_plan(net, std::min(t, net->L), o, R, &H, &gen, &cl, &bits_ok) && bits_ok;
     const int* ready = nullptr;
     int ready_rows = 0;
     bool streamed = false;

@@ -295,6 +295,13 @@ constexpr int kPfMaxLayers = 2000;  // t limit of the row-resident kernel (descr
 // layers: host descriptors of layers 0..t-1
 cudaError_t launch_pre_fused(const PreFusedArgs& a, const PreFusedLayer* layers, int num_sms, cudaStream_t st);
 
+// kernels_pre_cluster.cu: the row-resident pre phase for large rows (N = 16384 / 32768 / 65536), a row
+// split over a cluster of N / 8192 CTAs exchanging layer outputs through distributed shared memory
+int pre_cluster_class(int N, int nu);  // < 0: layer stride not supported
+bool pre_cluster_supported(int N);
+size_t pre_cluster_smem(int N, int Hh);
+cudaError_t launch_pre_cluster(const PreFusedArgs& a, const PreFusedLayer* layers, int num_sms, cudaStream_t st);
+
 // kernels_const.cu: constant rows in the per-layer pre-convergence path (R26)
 cudaError_t launch_const_split(const int* list_in, const int* count_in, unsigned* cmin, unsigned* cmax, int* list_out,
                                int* count_out, int* clist, float* cval, int* clayer, int* ccount, int layer,

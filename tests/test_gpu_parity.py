@@ -391,7 +391,9 @@ def _pf_inputs(N, B, seed):
 
 
 @pytest.mark.parametrize("N,nus,B", [(1024, (1, 32), 301), (2048, (1, 32, 64), 97), (4096, (1, 32, 128), 150),
-                                     (8192, (1, 64, 256, 32), 41), (16384, (1, 32, 512), 23)])
+                                     (8192, (1, 64, 256, 32), 41), (16384, (1, 32, 512), 23),
+                                     (16384, (512, 1, 32, 1), 17), (32768, (1, 32, 1024), 9),
+                                     (65536, (1, 32, 1024, 2048), 9), (65536, (2048, 32, 1, 1024), 5)])
 @pytest.mark.parametrize("drop", [1, 0])
 def test_pre_fused_bit_exact(N, nus, B, drop):
     """Row-resident pre-convergence kernel (every stride class: nu = 1, Q = 32, STR with compile-time
@@ -407,9 +409,12 @@ def test_pre_fused_bit_exact(N, nus, B, drop):
     Y0 = _pf_inputs(N, B, N + B)
     plain = oracle.layers_f32(net, Y0)
     res = {}
-    for pf in (1, 2, 0):
+    cluster = N >= 16384  # rows split over a thread-block cluster (kernels_pre_cluster.cu)
+    for pf in (1, 2, 0, 3):
+        if pf == 3 and N > 16384:
+            continue  # no single-CTA form
         Y, cats, st, _ = run_gpu(net, Y0, t=L, drop_dead_rows=drop, pre_fused=pf)
-        assert st["pre_fused"] == (1 if pf else 0)
+        assert st["pre_fused"] == (0 if pf == 0 else (2 if cluster and pf != 3 else 1)), f"pre_fused={pf}"
         res[pf] = (Y, cats, st)
         assert np.array_equal(Y, plain), f"pre_fused={pf}"
         assert np.array_equal(cats, oracle.categories(plain))
