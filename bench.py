@@ -70,9 +70,9 @@ def parse(argv=None):
     p.add_argument("--no-residue", action="store_true", help="skip the residue-regime study (C2, t = 10)")
     p.add_argument("--no-general", action="store_true", help="skip the general-CSC study (C2 perm)")
     p.add_argument("--residue-t", type=int, default=10)
-    p.add_argument("--pre-fused", type=int, default=1, choices=[0, 1, 2, 3],
-                   help="options.pre_fused: 1 = row-resident pre phase (default; cluster form for N >= 16384), "
-                        "2 = without the constant-row shortcut, 3 = never the cluster form, 0 = one launch per layer")
+    p.add_argument("--pre-fused", type=int, default=1, choices=[0, 1, 2, 4],
+                   help="options.pre_fused: 1 = row-resident pre phase (default), 2 = without the constant-row "
+                        "shortcut, 4 = rows split over a thread-block cluster (N >= 16384), 0 = one launch per layer")
     p.add_argument("--no-variants", action="store_true", help="skip the pre_fused = 2 / 0 roofline variants")
     p.add_argument("--cpu-seconds", type=float, default=15.0, help="target CPU work of the oracle sample")
     p.add_argument("--quick", action="store_true", help="value only (no e2e/uncompressed/variants/studies)")

@@ -87,18 +87,19 @@ typedef struct {
                                when every post layer is circulant with uniform weights and bias
                                (such a layer maps a constant row to a constant row; bit-identical
                                results); 0 = always the full-row evaluation */
-    int32_t pre_fused;      /* pre-convergence layers 0..t-1 (Eq. 1): 1 = row-resident fused kernel (rows of
-                               N = 16384 / 32768 / 65536 split over a thread-block cluster of N/8192 CTAs
-                               exchanging layer outputs through distributed shared memory; 3 = the same but
-                               never the cluster form, i.e. one CTA per row where that exists) -- a
+    int32_t pre_fused;      /* pre-convergence layers 0..t-1 (Eq. 1): 1 = row-resident fused kernel -- a
                                CTA keeps one row in shared memory for all t layers (Y0 read and Y(t)
                                written once) and carries a row that became constant (all elements
                                equal) by one scalar fma chain per layer (R26, exact); 2 = the same kernel
                                without the constant-row shortcut (every live row evaluated in full);
-                               0 = one kernel launch per layer.  Used when every layer < t is circulant
+                               0 = one kernel launch per layer; 3 = as 1; 4 = the row-resident kernel with
+                               each row split over a thread-block cluster of N/8192 CTAs exchanging layer
+                               outputs through distributed shared memory (N = 16384 / 32768 / 65536; the
+                               cluster form of a row that does not fit one CTA at several CTAs per SM).
+                               Used when every layer < t is circulant
                                with 32 taps, uniform weight and uniform bias, and N/32 is one of
-                               32..512 (N = 1024..16384) or the cluster form supports every stride
-                               (N = 16384..65536); otherwise the per-layer kernels run.
+                               32..512 (N = 1024..16384; 4: the cluster form supports every stride);
+                               otherwise the per-layer kernels run.
                                Results are bit-identical in every mode (tested). */
     int32_t pre_const;      /* per-layer pre-convergence path (pre_fused = 0 or not applicable): 1 = a row
                                whose outputs are all equal leaves the active list and is carried by one

@@ -32,6 +32,10 @@ constexpr int kCLS = 13;        // log2(kCS)
 constexpr int kCT = kCS / 32;   // threads per CTA
 constexpr int kCWp = kCT / 32;  // warps per CTA
 constexpr int kCSurv = 32;
+#ifndef SNICIT_CF_MINBLOCKS
+#define SNICIT_CF_MINBLOCKS 3
+#endif
+constexpr int kCfMinBlocks = SNICIT_CF_MINBLOCKS;  // CTAs per SM the register budget is sized for
 
 typedef unsigned long long u64;
 
@@ -248,11 +252,139 @@ __device__ __forceinline__ void cf_body_q32(const float* __restrict__ in, int r,
     }
 }
 
+// ---------------------------------------------------------------------------- specialised routes
+// The transitions of the SDGC stride cycles (N = 16384: nu 1 -> 32 -> 512 -> 1; N = 65536: 1 -> 32 ->
+// 1024 -> 2048 -> 1) with the routing folded into per-thread base addresses and compile-time offsets:
+// for output m of an item the target rank and offset are affine in m (derivations at each body), so a
+// store costs one st.shared::cluster with an immediate offset instead of the generic Router's integer work
+// (measured: the generic routing made the kernel issue-bound, 45% more instructions).
+
+// W, nu = 32 -> C(NNU) (NNU >= 512, nu'/G = NNU/G in [32, 512]).  Item base Qi = Qhi + c with Qhi a
+// multiple of 512 (q0 = r S, a0 32 with a0 a multiple of 16) and c < 32, so with b = Qhi mod NNU (a
+// multiple of 512, hence of nu'/G): output Qi + 32 m (m < 16) has residue b + c + 32 m, owner rank
+// (b >> lnug) + (32 m >> lnug) and offset ((Qhi >> lnu) << lnug) + c + (32 m & (nu'/G - 1)).
+template <int G, int NNU>
+__device__ __forceinline__ void sp_wstr32_c(const float* __restrict__ in, int q0, float w0, float b0, float ymax,
+                                            const uint32_t* nb, float& mn, float& mx) {
+    constexpr int NUG = NNU / G;
+    constexpr int LNU = __builtin_ctz(NNU), LNUG = __builtin_ctz(NUG);
+    constexpr int NB = (16 * 32 + NUG - 1) / NUG;  // ranks one item's 16 outputs span
+    constexpr int P32 = (kCS / 2);                 // second item: + P nu = S / 2
+    const int c = (int)threadIdx.x & 31;
+    const int a0 = ((int)threadIdx.x >> 5) * 16;
+    const float* s = in + a0 * 32 + c;
+    u64 R[47];
+#pragma unroll
+    for (int i = 0; i < 47; ++i) R[i] = f2_pack(s[i * 32], s[i * 32 + P32]);
+    uint32_t B1[NB], B2[NB];
+    {
+        const int Qhi1 = q0 + a0 * 32, Qhi2 = Qhi1 + P32;
+        const int hb1 = (Qhi1 & (NNU - 1)) >> LNUG, hb2 = (Qhi2 & (NNU - 1)) >> LNUG;
+        const uint32_t o1 = 4u * (uint32_t)(((Qhi1 >> LNU) << LNUG) + c), o2 = 4u * (uint32_t)(((Qhi2 >> LNU) << LNUG) + c);
+#pragma unroll
+        for (int k = 0; k < NB; ++k) {
+            B1[k] = nb[hb1 + k] + o1;
+            B2[k] = nb[hb2 + k] + o2;
+        }
+    }
+    const u64 W2 = f2_pack(w0, w0), BB = f2_pack(b0, b0);
+#pragma unroll
+    for (int m = 0; m < 16; ++m) {
+        u64 acc = 0ull;
+#pragma unroll
+        for (int n = 0; n < 32; ++n) acc = f2_fma(R[m + n], W2, acc);
+        float z1, z2;
+        f2_unpack(f2_add(acc, BB), z1, z2);
+        const float o1 = sigma(z1, ymax), o2 = sigma(z2, ymax);
+        st_cl_f32(B1[(32 * m) >> LNUG] + 4u * (uint32_t)((32 * m) & (NUG - 1)), o1);
+        st_cl_f32(B2[(32 * m) >> LNUG] + 4u * (uint32_t)((32 * m) & (NUG - 1)), o2);
+        mn = fminf(mn, fminf(o1, o2));
+        mx = fmaxf(mx, fmaxf(o1, o2));
+    }
+}
+
+// C, Q = 32 (nu = N/32, a multiple of S / 32 ... S is a multiple of nu) -> W.  Output m nu + cg (cg =
+// r nu/G + c' < nu): owner rank (m nu) >> 13, offset (m nu mod S) + cg; halo copy when that offset < Hh.
+template <int N>
+__device__ __forceinline__ void sp_q32_w(const float* __restrict__ in, int r, float w0, float b0, float ymax, int hh,
+                                         const uint32_t* nb, float& mn, float& mx) {
+    constexpr int G = N / kCS, NU = N / 32, T = kCT;
+    const int cp = threadIdx.x;
+    float x[32];
+#pragma unroll
+    for (int k = 0; k < 32; ++k) x[k] = in[k * T + cp];
+    u64 P[32];
+#pragma unroll
+    for (int k = 0; k < 32; ++k) P[k] = f2_pack(x[k], x[(k + 16) & 31]);
+    const u64 W2 = f2_pack(w0, w0), BB = f2_pack(b0, b0);
+    const int cg = r * T + cp;
+    const uint32_t o = 4u * (uint32_t)cg;
+#pragma unroll
+    for (int m = 0; m < 16; ++m) {
+        u64 acc = 0ull;
+#pragma unroll
+        for (int n = 0; n < 32; ++n) acc = f2_fma(P[(m + n) & 31], W2, acc);
+        float z1, z2;
+        f2_unpack(f2_add(acc, BB), z1, z2);
+        const float o1 = sigma(z1, ymax), o2 = sigma(z2, ymax);
+#pragma unroll
+        for (int it = 0; it < 2; ++it) {
+            const int mm = m + 16 * it;
+            const int h = (mm * NU) >> kCLS, off0 = (mm * NU) & (kCS - 1);  // compile-time
+            const float v = it ? o2 : o1;
+            st_cl_f32(nb[h] + o + 4u * (uint32_t)off0, v);
+            if (off0 < 1024 && off0 + cg < hh)  // the previous rank's halo
+                st_cl_f32(nb[(h - 1) & (G - 1)] + o + 4u * (uint32_t)(kCS + off0), v);
+        }
+        mn = fminf(mn, fminf(o1, o2));
+        mx = fmaxf(mx, fmaxf(o1, o2));
+    }
+}
+
+// C, Q = 64 (nu = N/64) -> C(2 nu).  Output (a + m) nu + cg (a in {a0, a0 + 32}, a0 in {0, 16}, cg = r nu/G + c'):
+// residue of 2 nu is (m & 1) nu + cg, so with nu'/G = 2 nu / G the owner rank is (m & 1) (nu >> lnug') +
+// (cg >> lnug') and the offset (((a >> 1) + (m >> 1)) << lnug') + (cg & (nu'/G - 1)).
+template <int N>
+__device__ __forceinline__ void sp_cstr_c2(const float* __restrict__ in, int r, float w0, float b0, float ymax,
+                                           const uint32_t* nb, float& mn, float& mx) {
+    constexpr int G = N / kCS, NU = N / 64, Q = 64;
+    constexpr int NUG = NU / G, LNUG = __builtin_ctz(NUG);
+    constexpr int NUG2 = 2 * NU / G, LNUG2 = __builtin_ctz(NUG2);
+    const int cp = (int)threadIdx.x & (NUG - 1);
+    const int a0 = ((int)threadIdx.x >> LNUG) * 16;
+    const float* sc = in + cp;
+    u64 R[47];
+#pragma unroll
+    for (int i = 0; i < 47; ++i) R[i] = f2_pack(sc[((a0 + i) & (Q - 1)) * NUG], sc[((a0 + 32 + i) & (Q - 1)) * NUG]);
+    const int cg = r * NUG + cp;
+    uint32_t B1[2], B2[2];
+#pragma unroll
+    for (int k = 0; k < 2; ++k) {
+        const uint32_t nbk = nb[k * (NU >> LNUG2) + (cg >> LNUG2)];
+        B1[k] = nbk + 4u * (uint32_t)(((a0 >> 1) << LNUG2) + (cg & (NUG2 - 1)));
+        B2[k] = nbk + 4u * (uint32_t)((((a0 + 32) >> 1) << LNUG2) + (cg & (NUG2 - 1)));
+    }
+    const u64 W2 = f2_pack(w0, w0), BB = f2_pack(b0, b0);
+#pragma unroll
+    for (int m = 0; m < 16; ++m) {
+        u64 acc = 0ull;
+#pragma unroll
+        for (int n = 0; n < 32; ++n) acc = f2_fma(R[m + n], W2, acc);
+        float z1, z2;
+        f2_unpack(f2_add(acc, BB), z1, z2);
+        const float o1 = sigma(z1, ymax), o2 = sigma(z2, ymax);
+        st_cl_f32(B1[m & 1] + 4u * (uint32_t)((m >> 1) << LNUG2), o1);
+        st_cl_f32(B2[m & 1] + 4u * (uint32_t)((m >> 1) << LNUG2), o2);
+        mn = fminf(mn, fminf(o1, o2));
+        mx = fmaxf(mx, fmaxf(o1, o2));
+    }
+}
+
 // ---------------------------------------------------------------------------- the kernel
 // G = N / kCS CTAs per cluster (launched with the cluster dimension set at launch); WUNI: one weight for
 // every layer (read at a constant offset -> uniform-register FFMA2 operand).
 template <int N, bool WUNI>
-__global__ void __launch_bounds__(kCT, 3) pre_cluster_kernel(const __grid_constant__ CfParams p) {
+__global__ void __launch_bounds__(kCT, kCfMinBlocks) pre_cluster_kernel(const __grid_constant__ CfParams p) {
     constexpr int G = N / kCS;
     constexpr int T = kCT;
     constexpr int NU_Q32 = N / 32;
@@ -364,9 +496,14 @@ __global__ void __launch_bounds__(kCT, 3) pre_cluster_kernel(const __grid_consta
                         cf_body_nu1<RT_C>(in, r * kCS, w0, b0, a.ymax, rt, mn, mx);
                 } else if (cls == CF_WSTR) {
                     const int P = (N / nu) / (2 * G);
+                    const int nnu = p.L[l + 1].nu;
                     if (nu == 32) {
                         if (nw)
                             cf_body_wstr<32, RT_LOC>(in, r * kCS, 32, P, w0, b0, a.ymax, rt, mn, mx);
+                        else if (nnu == N / 32 && N / 32 / G >= 32 && N / 32 / G <= 512)
+                            sp_wstr32_c<G, N / 32>(in, r * kCS, w0, b0, a.ymax, rt.base, mn, mx);
+                        else if (nnu == N / 64 && N / 64 / G >= 32 && N / 64 / G <= 512)
+                            sp_wstr32_c<G, N / 64>(in, r * kCS, w0, b0, a.ymax, rt.base, mn, mx);
                         else
                             cf_body_wstr<32, RT_C>(in, r * kCS, 32, P, w0, b0, a.ymax, rt, mn, mx);
                     } else {
@@ -377,11 +514,13 @@ __global__ void __launch_bounds__(kCT, 3) pre_cluster_kernel(const __grid_consta
                     }
                 } else if (cls == CF_Q32) {
                     if (nw)
-                        cf_body_q32<NU_Q32, RT_W>(in, r, w0, b0, a.ymax, rt, mn, mx);
+                        sp_q32_w<N>(in, r, w0, b0, a.ymax, Hh, rt.base, mn, mx);
                     else
                         cf_body_q32<NU_Q32, RT_C>(in, r, w0, b0, a.ymax, rt, mn, mx);
                 } else {
-                    if (nw)
+                    if (!nw && nu == N / 64 && p.L[l + 1].nu == N / 32 && (N / 64) / G >= 4)
+                        sp_cstr_c2<N>(in, r, w0, b0, a.ymax, rt.base, mn, mx);
+                    else if (nw)
                         cf_body_cstr<RT_W>(in, r, nu, N / nu, w0, b0, a.ymax, rt, mn, mx, ilog2i(nu) - ilog2i(G));
                     else
                         cf_body_cstr<RT_C>(in, r, nu, N / nu, w0, b0, a.ymax, rt, mn, mx, ilog2i(nu) - ilog2i(G));

@@ -732,7 +732,8 @@ extern "C" {
 // Row-resident pre phase applicable?  (kernels_pre_fused.cu: circulant layers < t with 32 taps,
 // uniform weight and bias, N / 32 in 32..512, t <= kPfMaxLayers, smem fits); *H = circular halo
 // *cluster: the row is split over a thread-block cluster (kernels_pre_cluster.cu: N = 16384 / 32768 /
-// 65536, every layer's stride supported; pre_fused = 3 keeps the single-CTA kernel where it exists);
+// 65536, every layer's stride supported; only on request, pre_fused = 4: measured slower than the
+// single-CTA kernel at N = 16384 and than the per-layer kernels at N = 65536);
 // *bits_ok: packed input rows can be read by the chosen kernel
 static bool pf_plan(const snicit_network* net, int tt, const snicit_options& opt, int R, int* H, int* gen,
                     bool* cluster = nullptr, bool* bits_ok = nullptr) {
@@ -740,7 +741,7 @@ static bool pf_plan(const snicit_network* net, int tt, const snicit_options& opt
     if (cluster) *cluster = false;
     if (bits_ok) *bits_ok = true;
     const bool base_ok = opt.pre_fused != 0 && tt > 0 && tt <= kPfMaxLayers && R > 0 && opt.kernel == SNICIT_KERNEL_AUTO;
-    if (base_ok && opt.pre_fused != 3 && pre_cluster_supported(N)) {
+    if (base_ok && opt.pre_fused == 4 && pre_cluster_supported(N)) {
         bool ok = true;
         for (int l = 0; l < tt && ok; ++l) ok = net->pf_elig[l] != 0 && pre_cluster_class(N, net->plan[l].nu) >= 0;
         if (ok) {
@@ -751,7 +752,7 @@ static bool pf_plan(const snicit_network* net, int tt, const snicit_options& opt
             return true;
         }
     }
-    bool pf = base_ok && pre_fused_threads(N) > 0;
+    bool pf = base_ok && opt.pre_fused != 4 && pre_fused_threads(N) > 0;
     for (int l = 0; l < tt && pf; ++l) pf = net->pf_elig[l] != 0;
     int h = 96, g = 0;  // nu == 1 windows read 47 past an item, head items write 68; STR 31*nu
     if (pf) {
@@ -837,7 +838,7 @@ static snicit_status infer_core(snicit_network* net, const float* y0, int64_t ba
         return fail(SNICIT_E_INVALID_ARG, "bad eta/eps/prune_eps");
     if (opt.kernel < 0 || opt.kernel > SNICIT_KERNEL_CIRC_SMEM) return fail(SNICIT_E_INVALID_ARG, "bad kernel option");
     if (opt.post_mode < 0 || opt.post_mode > 1) return fail(SNICIT_E_INVALID_ARG, "bad post_mode");
-    if (opt.pre_fused < 0 || opt.pre_fused > 3) return fail(SNICIT_E_INVALID_ARG, "bad pre_fused");
+    if (opt.pre_fused < 0 || opt.pre_fused > 4) return fail(SNICIT_E_INVALID_ARG, "bad pre_fused");
     if (opt.pre_const < 0 || opt.pre_const > 1) return fail(SNICIT_E_INVALID_ARG, "bad pre_const");
     if (opt.res_sparse < 0 || opt.res_sparse > 1) return fail(SNICIT_E_INVALID_ARG, "bad res_sparse");
     if (opt.kernel == SNICIT_KERNEL_ELL && !net->has_ell)

@@ -409,22 +409,29 @@ def test_pre_fused_bit_exact(N, nus, B, drop):
     Y0 = _pf_inputs(N, B, N + B)
     plain = oracle.layers_f32(net, Y0)
     res = {}
-    cluster = N >= 16384  # rows split over a thread-block cluster (kernels_pre_cluster.cu)
-    for pf in (1, 2, 0, 3):
-        if pf == 3 and N > 16384:
-            continue  # no single-CTA form
+    single = N <= 16384  # one CTA per row exists (kernels_pre_fused.cu); pre_fused = 4: cluster form (N >= 16384)
+    for pf in (1, 2, 0, 4):
+        if pf == 4 and N < 16384:
+            continue
         Y, cats, st, _ = run_gpu(net, Y0, t=L, drop_dead_rows=drop, pre_fused=pf)
-        assert st["pre_fused"] == (0 if pf == 0 else (2 if cluster and pf != 3 else 1)), f"pre_fused={pf}"
+        want = 2 if pf == 4 else (0 if pf == 0 or not single else 1)
+        assert st["pre_fused"] == want, f"pre_fused={pf}"
         res[pf] = (Y, cats, st)
         assert np.array_equal(Y, plain), f"pre_fused={pf}"
         assert np.array_equal(cats, oracle.categories(plain))
-    assert res[1][2]["pre_const_rows"] > 0 and res[2][2]["pre_const_rows"] == 0
-    assert res[1][2]["pre_full_rows"] < res[2][2]["pre_full_rows"]
+    if single:
+        assert res[1][2]["pre_const_rows"] > 0 and res[2][2]["pre_const_rows"] == 0
+        assert res[1][2]["pre_full_rows"] < res[2][2]["pre_full_rows"]
+    if 4 in res:
+        assert res[4][2]["pre_const_rows"] > 0 and res[4][2]["live_at_t"] == res[0][2]["live_at_t"]
     assert res[1][2]["live_at_t"] == res[0][2]["live_at_t"] == res[2][2]["live_at_t"]
     # SNICIT pipeline with conversion at t = L // 2: fused pre phase == per-layer pre phase
     Ya, ca, sa, cla = run_gpu(net, Y0, t=L // 2, drop_dead_rows=drop, pre_fused=1)
     Yb, cb, sb, clb = run_gpu(net, Y0, t=L // 2, drop_dead_rows=drop, pre_fused=0)
     assert np.array_equal(Ya, Yb) and np.array_equal(ca, cb)
+    if N >= 16384:
+        Yc, cc, sc, _ = run_gpu(net, Y0, t=L // 2, drop_dead_rows=drop, pre_fused=4)
+        assert sc["pre_fused"] == 2 and np.array_equal(Yc, Yb) and np.array_equal(cc, cb)
     assert np.array_equal(ca, oracle.categories(plain))
     assert np.allclose(Ya, plain, atol=ATOL, rtol=RTOL)
 
