@@ -181,7 +181,8 @@ snicit_status snicit_set_stream(snicit_network* net, void* cuda_stream);
  *  row_offset:      global id of local row 0 (multi-GPU row sharding); category
  *                   ids are row_offset + local row.
  *  threshold_layer: t; t >= L runs the uncompressed plain path.
- *  centroid_count:  s, the sample size and upper bound on cent_cnt; >= 1.
+ *  centroid_count:  s, the sample size and upper bound on cent_cnt; 1 <= s <= 1024
+ *                   (larger: SNICIT_E_UNSUPPORTED).
  *  opt:             NULL = snicit_default_options.
  *  y_out:           batch*N fp32, caller-owned; device pointer if y_out_on_device else host;
  *                   NULL = do not materialise Y(L) (categories are still computed).

@@ -10,6 +10,8 @@
 #include <cuda_runtime.h>
 #include <string.h>
 
+#include <algorithm>
+
 #include "snicit_internal.cuh"
 
 namespace snicit {
@@ -281,120 +283,269 @@ cudaError_t launch_prune(const double* F, const int* count, int s, int n_seg, fl
     return cudaGetLastError();
 }
 
-// Alg. 2 / Eq. 3-4: one CTA per live row.  L0 distance to each centroid (element-wise '!=' counts,
-// Alg. 2 lines 10-12), first minimum over ascending y* wins (strict '<', R6).  Centroid rows are
-// copied to the compact centroid buffer (slot = position in y*), M = -1 and ne = 1 (R7); mapped
-// rows get M = centroid row id, ne = (dist != 0), and their residue Y_r - Y_c written only if ne.
+// Alg. 2 / Eq. 3-4 in two passes.
+//
+// Pass 1 (map_dist_kernel): L0 distances dist[p][c] = #{k : Y[r][k] != Y[cent[c]][k]} (Alg. 2 lines
+// 10-12) of every live row r = rows[p] to every centroid.  A CTA holds a column tile [k0, k0 + TK) of all
+// C centroid rows in shared memory and streams a block of rows through it: lane j of a warp reads
+// element k0 + 32 i + j of the row once (coalesced) and compares it with every centroid's element; a warp
+// ballot + popc turns 32 comparisons into one count (warp-uniform counters, one per centroid).  Tile sums
+// are added to dist (integer atomics: exact, order-free).  Each row element is read from HBM once; the
+// comparisons are bound by the shared-memory read of the centroid values (1 LDS per element-centroid).
+// Pass 2 (map_finish_kernel): one warp per live row: first minimum over ascending y* (strict '<', R6),
+// M, ne, and the residue Y_r - Y_c written only for non-empty rows; centroid rows copied to the compact
+// centroid buffer (slot = position in y*), M = -1, ne = 1 (R7).  Rows constant at t (R26, flags from the
+// pre phase) map to an equal constant centroid without a read (their L0 distance to it is 0 and to any
+// other centroid > 0, so it is Alg. 2's argmin).
 constexpr int kMapThreads = 256;
-__global__ void __launch_bounds__(kMapThreads) map_residual_kernel(const float* __restrict__ y, int N,
-                                                                   const int* rows, const int* count,
-                                                                   const int* cent, const int* n_cent, int* M,
-                                                                   int* cslot, uint8_t* ne_row, uint8_t* flag_pos,
-                                                                   float* __restrict__ yhat,
-                                                                   float* __restrict__ cbuf,
-                                                                   const uint8_t* __restrict__ rconst,
-                                                                   const float* __restrict__ rval,
-                                                                   unsigned long long* nnz_sum) {
-    __shared__ int red[kMapThreads / 32];
-    __shared__ int s_best, s_slot;
+constexpr int kMapSmemFloats = 16384;  // 64 KB of centroid tile
+// columns per tile for C centroids (padded to a multiple of 32): Cp * TK <= kMapSmemFloats
+__host__ __device__ inline int map_tile(int C) {
+    const int Cp = (C + 31) / 32 * 32;
+    return Cp <= 32 ? 512 : (Cp <= 128 ? 128 : 32);
+}
+
+// constant-row shortcut / centroid test of row r (thread-uniform): returns slot >= 0 for a centroid row, else
+// -1; *hit = centroid index of an equal constant centroid (R26) or -1
+__device__ __forceinline__ int map_classify(int r, const int* cent, int C, const uint8_t* rconst, const float* rval,
+                                            int* hit) {
+    int slot = -1;
+    for (int c = 0; c < C; ++c)
+        if (cent[c] == r) slot = c;
+    *hit = -1;
+    if (slot < 0 && rconst && rconst[r]) {
+        const float v = rval[r];
+        for (int c = 0; c < C && *hit < 0; ++c)
+            if (rconst[cent[c]] && rval[cent[c]] == v) *hit = c;
+    }
+    return slot;
+}
+
+// TK: columns per tile (compile-time).  Shared layout [Cp centroids][TK] (float4 rows); lane j of a warp
+// owns the float4 chunks j, j + 32, .. of the tile: it reads its row elements once and compares them with
+// every centroid's elements, keeping one counter per centroid in registers (4 compares per LDS.128); the
+// warp sums each centroid's counters at the end of the tile (shuffles) and lane c adds centroid c's sum to
+// dist.  Centroids are processed in groups of 32 (register counters).
+template <int TK>
+__global__ void __launch_bounds__(kMapThreads) map_dist_kernel(const float* __restrict__ y, int N, const int* rows,
+                                                               const int* count, const int* cent, const int* n_cent,
+                                                               int* __restrict__ dist, int s,
+                                                               const uint8_t* __restrict__ rconst,
+                                                               const float* __restrict__ rval) {
+    extern __shared__ float4 s_c4[];
+    __shared__ float s_cv[1024];  // constant value of centroid c (R26) or NaN
+    constexpr int TK4 = TK / 4, CH = (TK4 + 31) / 32;  // float4 chunks per lane
     const int n = *count;
-    const int C = *n_cent;
-    const int lane = threadIdx.x & 31, wid = threadIdx.x >> 5;
+    const int C = min(*n_cent, s);
+    if (C <= 0 || map_tile(C) != TK) return;  // the launcher starts every TK variant; one matches
+    const int Cp = (C + 31) / 32 * 32;
+    const int ntiles = (N + TK - 1) / TK;
+    if ((int)blockIdx.x >= ((int)gridDim.x / ntiles) * ntiles) return;  // grid remainder
+    const int tile = blockIdx.x % ntiles;
+    const int k0 = tile * TK;
+    const int kl4 = min(TK, N - k0) >> 2;  // N % 4 == 0 (16-byte rows)
+    for (int i = threadIdx.x; i < Cp * TK4; i += blockDim.x) {
+        const int c = i / TK4, k4 = i - c * TK4;
+        s_c4[i] = (c < C && k4 < kl4) ? __ldg(reinterpret_cast<const float4*>(y + (size_t)cent[c] * N + k0) + k4)
+                                      : make_float4(0.f, 0.f, 0.f, 0.f);
+    }
+    for (int c = threadIdx.x; c < C; c += blockDim.x)
+        s_cv[c] = (rconst && rconst[cent[c]]) ? rval[cent[c]] : __int_as_float(0x7fffffff);
+    __syncthreads();
+    const int lane = threadIdx.x & 31, warp = threadIdx.x >> 5;
+    const int nwb = (gridDim.x / ntiles) * (kMapThreads / 32);  // warps over the rows
+    // rows that need distances (a constant row with an equal constant centroid does not)
+    auto needed = [&](int p_) {
+        const int r_ = rows[p_];
+        if (!(rconst && rconst[r_])) return true;
+        const float v = rval[r_];
+        for (int c = 0; c < C; ++c)
+            if (s_cv[c] == v) return false;
+        return true;
+    };
+    auto next_row = [&](int p_) {
+        while (p_ < n && !needed(p_)) p_ += nwb;
+        return p_;
+    };
+    auto load_tile = [&](int p_, float4* v) {
+        const float4* yr4 = reinterpret_cast<const float4*>(y + (size_t)rows[p_] * N + k0);
+#pragma unroll
+        for (int i = 0; i < CH; ++i) {
+            const int k4 = lane + 32 * i;
+            v[i] = k4 < kl4 ? __ldg(yr4 + k4) : make_float4(0.f, 0.f, 0.f, 0.f);
+        }
+    };
+    int p = next_row((blockIdx.x / ntiles) * (kMapThreads / 32) + warp);
+    float4 yn[CH];  // the next row's tile, loaded while this one is compared
+    if (p < n) load_tile(p, yn);
+    while (p < n) {
+        float4 yv[CH];
+#pragma unroll
+        for (int i = 0; i < CH; ++i) yv[i] = yn[i];
+        const int pcur = p;
+        p = next_row(p + nwb);
+        if (p < n) load_tile(p, yn);
+        for (int cg = 0; cg < Cp; cg += 32) {
+            int cnt[32];
+#pragma unroll
+            for (int j = 0; j < 32; ++j) {
+                int c_ = 0;
+                const float4* sc = s_c4 + (size_t)(cg + j) * TK4 + lane;
+#pragma unroll
+                for (int i = 0; i < CH; ++i) {
+                    if (lane + 32 * i < kl4) {
+                        const float4 cv = sc[32 * i];
+                        c_ += (yv[i].x != cv.x) + (yv[i].y != cv.y) + (yv[i].z != cv.z) + (yv[i].w != cv.w);
+                    }
+                }
+                cnt[j] = c_;
+            }
+            // transpose-reduce: after the butterfly lane j holds the warp sum of centroid cg + j
+#pragma unroll
+            for (int o = 16; o > 0; o >>= 1) {
+#pragma unroll
+                for (int j = 0; j < o; ++j) {
+                    // lanes with bit o set keep the upper half, the others the lower half
+                    const bool up = (lane & o) != 0;
+                    const int send = up ? cnt[j] : cnt[j + o];
+                    const int recv = __shfl_xor_sync(0xffffffffu, send, o);
+                    cnt[j] = (up ? cnt[j + o] : cnt[j]) + recv;
+                }
+            }
+            const int mine = cnt[0];
+            if (cg + lane < C && mine) atomicAdd(dist + (size_t)pcur * s + cg + lane, mine);
+        }
+    }
+}
+
+__global__ void __launch_bounds__(kMapThreads) map_finish_kernel(const float* __restrict__ y, int N, const int* rows,
+                                                                 const int* count, const int* cent, const int* n_cent,
+                                                                 const int* __restrict__ dist, int s, int* M, int* cslot,
+                                                                 uint8_t* ne_row, uint8_t* flag_pos,
+                                                                 float* __restrict__ yhat, float* __restrict__ cbuf,
+                                                                 const uint8_t* __restrict__ rconst,
+                                                                 const float* __restrict__ rval,
+                                                                 unsigned long long* nnz_sum, int* rnnz) {
+    const int n = *count;
+    const int C = min(*n_cent, s);
+    const int lane = threadIdx.x & 31;
+    const int warps = (gridDim.x * blockDim.x) >> 5;
     const int N4 = N >> 2;
-    for (int p = blockIdx.x; p < n; p += gridDim.x) {
+    for (int p = (blockIdx.x * blockDim.x + threadIdx.x) >> 5; p < n; p += warps) {
         const int r = rows[p];
         const float4* y4 = reinterpret_cast<const float4*>(y + (size_t)r * N);
-        if (threadIdx.x == 0) {
-            s_slot = -1;
-            for (int c = 0; c < C; ++c)
-                if (cent[c] == r) s_slot = c;
-        }
-        __syncthreads();
-        const int slot = s_slot;
+        int hit;
+        const int slot = map_classify(r, cent, C, rconst, rval, &hit);
         if (slot >= 0) {  // centroid row (Eq. 4 second case)
             float4* d4 = reinterpret_cast<float4*>(cbuf + (size_t)slot * N);
-            for (int k = threadIdx.x; k < N4; k += blockDim.x) d4[k] = y4[k];
-            if (threadIdx.x == 0) {
+            for (int k = lane; k < N4; k += 32) d4[k] = y4[k];
+            if (lane == 0) {
                 M[r] = -1;
                 cslot[r] = slot;
                 ne_row[r] = 1;
                 flag_pos[p] = 0;
             }
-            __syncthreads();
             continue;
         }
-        if (rconst && rconst[r]) {
-            // constant row (R26, flags from the pre phase): its L0 distance to a centroid that is the
-            // same constant is 0 and to any other centroid > 0, so the first such centroid is Alg. 2's
-            // argmin (strict <) -- empty residue, nothing to read or write
-            int hit = -1;
-            const float v = rval[r];
-            for (int c = 0; c < C && hit < 0; ++c)
-                if (rconst[cent[c]] && rval[cent[c]] == v) hit = c;
-            if (hit >= 0) {
-                if (threadIdx.x == 0) {
-                    M[r] = cent[hit];
-                    cslot[r] = hit;
-                    ne_row[r] = 0;
-                    flag_pos[p] = 0;
-                }
-                continue;  // uniform across the CTA: no barrier needed
+        if (hit >= 0) {  // constant row over an equal constant centroid: empty residue
+            if (lane == 0) {
+                M[r] = cent[hit];
+                cslot[r] = hit;
+                ne_row[r] = 0;
+                flag_pos[p] = 0;
             }
+            continue;
         }
-        int best_dist = N + 1, best = 0;  // Alg. 2 line 3 (tracked by thread 0)
-        for (int c = 0; c < C; ++c) {
-            const float4* c4 = reinterpret_cast<const float4*>(y + (size_t)cent[c] * N);
-            int cnt = 0;
-            for (int k = threadIdx.x; k < N4; k += blockDim.x) {
-                const float4 a = y4[k], b = c4[k];
-                cnt += (a.x != b.x) + (a.y != b.y) + (a.z != b.z) + (a.w != b.w);
+        if (C <= 0) {  // no centroid at all
+            if (lane == 0) {
+                M[r] = -2;
+                ne_row[r] = 0;
+                flag_pos[p] = 0;
             }
+            continue;
+        }
+        // first minimum over ascending y* (Alg. 2 lines 14-16, strict '<' from dist = N + 1: R6)
+        int best = 0x7fffffff, bc = 0;
+        for (int c0 = 0; c0 < C; c0 += 32) {
+            const int c = c0 + lane;
+            int d = c < C ? dist[(size_t)p * s + c] : 0x7fffffff;
+            int cc = c;
 #pragma unroll
-            for (int o = 16; o > 0; o >>= 1) cnt += __shfl_down_sync(0xffffffffu, cnt, o);
-            if (lane == 0) red[wid] = cnt;
-            __syncthreads();
-            if (threadIdx.x == 0) {
-                int d = 0;
-                for (int w = 0; w < kMapThreads / 32; ++w) d += red[w];
-                if (d < best_dist) {  // lines 14-16
-                    best_dist = d;
-                    best = c;
+            for (int o = 16; o; o >>= 1) {
+                const int d2 = __shfl_xor_sync(0xffffffffu, d, o), c2 = __shfl_xor_sync(0xffffffffu, cc, o);
+                if (d2 < d || (d2 == d && c2 < cc)) {
+                    d = d2;
+                    cc = c2;
                 }
             }
-            __syncthreads();
+            if (d < best) {
+                best = d;
+                bc = cc;
+            }
         }
-        if (threadIdx.x == 0) {
-            s_best = best;
-            s_slot = best_dist;  // reuse as the distance broadcast
-            M[r] = cent[best];   // line 25
-            cslot[r] = best;
-            const uint8_t ne = best_dist != 0 ? 1 : 0;  // lines 26-29
+        const uint8_t ne = best != 0 ? 1 : 0;  // lines 26-29
+        if (lane == 0) {
+            M[r] = cent[bc];  // line 25
+            cslot[r] = bc;
             ne_row[r] = ne;
             flag_pos[p] = ne;
             // the residue's non-zeros are exactly the differing elements (x - y != 0 <=> x != y, finite)
-            if (nnz_sum && ne) atomicAdd(nnz_sum, (unsigned long long)best_dist);
+            if (nnz_sum && ne) atomicAdd(nnz_sum, (unsigned long long)best);
+            if (rnnz) rnnz[r] = ne ? best : 0;
         }
-        __syncthreads();
-        if (s_slot != 0) {  // residue only needed for non-empty rows (Eq. 4 first case)
-            const float4* c4 = reinterpret_cast<const float4*>(y + (size_t)cent[s_best] * N);
+        if (ne) {  // residue only for non-empty rows (Eq. 4 first case)
+            const float4* c4 = reinterpret_cast<const float4*>(y + (size_t)cent[bc] * N);
             float4* o4 = reinterpret_cast<float4*>(yhat + (size_t)r * N);
-            for (int k = threadIdx.x; k < N4; k += blockDim.x) {
-                const float4 a = y4[k], b = c4[k];
+            for (int k = lane; k < N4; k += 32) {
+                const float4 a = y4[k], b = __ldg(c4 + k);
                 o4[k] = make_float4(a.x - b.x, a.y - b.y, a.z - b.z, a.w - b.w);
             }
         }
-        __syncthreads();
     }
 }
+
 cudaError_t launch_map_residual(const float* y, int N, const int* rows, const int* count, const int* cent,
                                 const int* n_cent, int* M, int* cslot, uint8_t* ne_row, uint8_t* flag_pos,
                                 float* yhat, float* cbuf, int max_rows, int num_sms, cudaStream_t st,
-                                const uint8_t* rconst, const float* rval, unsigned long long* nnz_sum) {
+                                const uint8_t* rconst, const float* rval, unsigned long long* nnz_sum, int* dist,
+                                int s, int* rnnz) {
+    if (max_rows <= 0) return cudaSuccess;
+    cudaError_t e = cudaMemsetAsync(dist, 0, sizeof(int) * (size_t)max_rows * s, st);
+    if (e != cudaSuccess) return e;
+    // pass 1: the tile width depends on the centroid count C <= s, known only on the device: every tile
+    // variant up to the one of C = s is launched and all but the matching one exit at once
+    if (s > 1024) return cudaErrorInvalidValue;  // the widest centroid tile (32 columns) must fit
+    const size_t smem = sizeof(float) * std::max<size_t>(kMapSmemFloats, (size_t)(s + 31) / 32 * 32 * 32);
+    auto one = [&](const void* kern, int TK, auto launch) -> cudaError_t {
+        if (TK < map_tile(s)) return cudaSuccess;  // C <= s never selects a narrower tile
+        int bps = 1;
+        cudaError_t e2 = blocks_per_sm(kern, kMapThreads, smem, &bps);
+        if (e2 != cudaSuccess) return e2;
+        const int T = (N + TK - 1) / TK;
+        int rb = (num_sms * bps + T - 1) / T;  // row blocks: the whole GPU busy
+        const int rb_max = (max_rows + kMapThreads / 32 - 1) / (kMapThreads / 32);
+        if (rb > rb_max) rb = rb_max;
+        if (rb < 1) rb = 1;
+        launch(rb * T);
+        return cudaGetLastError();
+    };
+    e = one((const void*)map_dist_kernel<512>, 512, [&](int g) {
+        map_dist_kernel<512><<<g, kMapThreads, smem, st>>>(y, N, rows, count, cent, n_cent, dist, s, rconst, rval);
+    });
+    if (e == cudaSuccess)
+        e = one((const void*)map_dist_kernel<128>, 128, [&](int g) {
+            map_dist_kernel<128><<<g, kMapThreads, smem, st>>>(y, N, rows, count, cent, n_cent, dist, s, rconst, rval);
+        });
+    if (e == cudaSuccess)
+        e = one((const void*)map_dist_kernel<32>, 32, [&](int g) {
+            map_dist_kernel<32><<<g, kMapThreads, smem, st>>>(y, N, rows, count, cent, n_cent, dist, s, rconst, rval);
+        });
+    if (e != cudaSuccess) return e;
     int grid = num_sms * 8;
-    if (grid > max_rows) grid = max_rows;
+    if (grid > (max_rows + 7) / 8) grid = (max_rows + 7) / 8;
     if (grid < 1) grid = 1;
-    map_residual_kernel<<<grid, kMapThreads, 0, st>>>(y, N, rows, count, cent, n_cent, M, cslot, ne_row, flag_pos,
-                                                      yhat, cbuf, rconst, rval, nnz_sum);
+    map_finish_kernel<<<grid, kMapThreads, 0, st>>>(y, N, rows, count, cent, n_cent, dist, s, M, cslot, ne_row,
+                                                    flag_pos, yhat, cbuf, rconst, rval, nnz_sum, rnnz);
     return cudaGetLastError();
 }
 

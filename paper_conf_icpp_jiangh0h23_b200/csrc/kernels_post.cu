@@ -84,7 +84,8 @@ __device__ __forceinline__ PL load_pl(const PostLayer* __restrict__ p) {
 template <int MODE, bool UNIF, int MNU1, int MGEN, int QG>
 __device__ __forceinline__ int post_row_circ(const PL& Ld, int N, int dup, float ymax, float prune_eps,
                                               const float* __restrict__ in, float* __restrict__ out,
-                                              const float* __restrict__ ac, float* __restrict__ aout) {
+                                              const float* __restrict__ ac, float* __restrict__ aout, float& mn,
+                                              float& mx) {
     const float w0 = Ld.w0, b0 = Ld.b0;
     const bool ubias = Ld.ubias != 0;
     const float* __restrict__ bias = Ld.bias;
@@ -103,6 +104,10 @@ __device__ __forceinline__ int post_row_circ(const PL& Ld, int N, int dup, float
         const float v = post_epi<MODE>(acc, b, ac, q, ymax, prune_eps);
         out[q] = v;
         nz += (v != 0.0f);
+        if constexpr (MODE == MODE_RESIDUAL) {
+            mn = fminf(mn, v);
+            mx = fmaxf(mx, v);
+        }
     };
     if (Ld.cls == PCLS_NU1) {
         constexpr int M = MNU1, WIN = M + kPK - 1;
@@ -179,7 +184,8 @@ __device__ __forceinline__ int post_row_circ(const PL& Ld, int N, int dup, float
 template <int MODE>
 __device__ __forceinline__ int post_row_ell(const PL& Ld, int N, float ymax, float prune_eps,
                                              const float* __restrict__ in, float* __restrict__ out,
-                                             const float* __restrict__ ac, float* __restrict__ aout) {
+                                             const float* __restrict__ ac, float* __restrict__ aout, float& mn,
+                                             float& mx) {
     const uint8_t* __restrict__ lens = Ld.len;
     const uint16_t* __restrict__ i16 = Ld.idx16;
     const int32_t* __restrict__ i32 = Ld.idx32;
@@ -205,6 +211,10 @@ __device__ __forceinline__ int post_row_ell(const PL& Ld, int N, float ymax, flo
         const float v = post_epi<MODE>(acc, b, ac, j, ymax, prune_eps);
         out[j] = v;
         nz += (v != 0.0f);
+        if constexpr (MODE == MODE_RESIDUAL) {
+            mn = fminf(mn, v);
+            mx = fmaxf(mx, v);
+        }
     }
     return nz;
 }
@@ -212,13 +222,13 @@ __device__ __forceinline__ int post_row_ell(const PL& Ld, int N, float ymax, flo
 template <int MODE, int MNU1, int MGEN, int QG>
 __device__ __forceinline__ int post_row_layer(const PL& Ld, int N, int dup, float ymax, float prune_eps,
                                                const float* in, float* out, const float* ac, float* aout,
-                                               int force_ell) {
+                                               int force_ell, float& mn, float& mx) {
     if (Ld.kind == 1 && !force_ell) {
         if (Ld.unif)
-            return post_row_circ<MODE, true, MNU1, MGEN, QG>(Ld, N, dup, ymax, prune_eps, in, out, ac, aout);
-        return post_row_circ<MODE, false, MNU1, MGEN, QG>(Ld, N, dup, ymax, prune_eps, in, out, ac, aout);
+            return post_row_circ<MODE, true, MNU1, MGEN, QG>(Ld, N, dup, ymax, prune_eps, in, out, ac, aout, mn, mx);
+        return post_row_circ<MODE, false, MNU1, MGEN, QG>(Ld, N, dup, ymax, prune_eps, in, out, ac, aout, mn, mx);
     }
-    return post_row_ell<MODE>(Ld, N, ymax, prune_eps, in, out, ac, aout);
+    return post_row_ell<MODE>(Ld, N, ymax, prune_eps, in, out, ac, aout, mn, mx);
 }
 
 __device__ __forceinline__ void stage_row(float* dst, const float* __restrict__ src, int N) {
@@ -268,7 +278,8 @@ __global__ void __launch_bounds__(kCentThreads) centroid_traj_kernel(PostArgs a)
     for (int l = a.t; l < a.L; ++l) {
         const PL Lnext = load_pl(a.layers + min(l + 1, a.L - 1));  // prefetch (serial critical path)
         float* aout = want_a ? a.a_all + ((size_t)(l - a.t) * a.s + c) * N : nullptr;
-        post_row_layer<MODE_CENTROID, 5, 4, 8>(Ld, N, dup, a.ymax, 0.0f, cur, nxt, nullptr, aout, a.force_ell);
+        float dmn = 0.0f, dmx = 0.0f;
+        post_row_layer<MODE_CENTROID, 5, 4, 8>(Ld, N, dup, a.ymax, 0.0f, cur, nxt, nullptr, aout, a.force_ell, dmn, dmx);
         __syncthreads();
         fill_halo(nxt, N, h);
         __syncthreads();
@@ -397,6 +408,7 @@ __global__ void __launch_bounds__(kPostThreads, 2) residual_traj_kernel(PostArgs
     extern __shared__ __align__(128) float sm[];
     __shared__ int s_p;
     __shared__ int s_nz[3];   // per-layer non-zero count of the dense form (rotating slots)
+    __shared__ int s_mn[3], s_mx[3];  // per-layer output range of the dense form (order-preserving int codes)
     __shared__ int s_cnt[3];  // sparse form: [0], [1] sp_layer's counters, [2] sp_list's (distinct slots:
                               // sp_layer may follow sp_list with no barrier in between)
     const int N = a.N;
@@ -419,7 +431,11 @@ __global__ void __launch_bounds__(kPostThreads, 2) residual_traj_kernel(PostArgs
         float* cur = sm;
         float* nxt = sm + N + h;
         stage_row(cur, a.yhat + (size_t)row * N, N);
-        if (threadIdx.x < 3) s_nz[threadIdx.x] = 0;
+        if (threadIdx.x < 3) {
+            s_nz[threadIdx.x] = 0;
+            s_mn[threadIdx.x] = 0x7fffffff;
+            s_mx[threadIdx.x] = (int)0x80000000;
+        }
         __syncthreads();
         fill_halo(cur, N, h);
         __syncthreads();
@@ -431,8 +447,13 @@ __global__ void __launch_bounds__(kPostThreads, 2) residual_traj_kernel(PostArgs
         int nnz = -1, li = 0;
         bool listed = false, nxt_zero = false;
         if (a.res_sparse) {
-            nnz = sp_list(cur, N, lsts[0], cap, &s_cnt[2]);
-            listed = nnz <= cap;
+            const int known = a.rnnz ? a.rnnz[row] : -1;  // non-zeros at t (Alg. 2's distance), if recorded
+            if (known > cap) {
+                nnz = known;
+            } else {
+                nnz = sp_list(cur, N, lsts[0], cap, &s_cnt[2]);
+                listed = nnz <= cap;
+            }
         }
         PL Ld = load_pl(a.layers + a.t);
         int l = a.t;
@@ -441,7 +462,13 @@ __global__ void __launch_bounds__(kPostThreads, 2) residual_traj_kernel(PostArgs
             const float* ac = a.a_all + ((size_t)(l - a.t) * a.s + slot) * N;
             const bool sparse = a.res_sparse && listed && Ld.kind == 1 && !a.force_ell;
             int cnt;
-            if (threadIdx.x == 0) s_nz[(l + 1) % 3] = 0;  // the next layer's slot (last read two barriers ago)
+            bool rowconst = false;  // every output of this layer equal (dense form; a listed sparse row never is)
+            float v0 = 0.0f;
+            if (threadIdx.x == 0) {  // the next layer's slots (last read two barriers ago)
+                s_nz[(l + 1) % 3] = 0;
+                s_mn[(l + 1) % 3] = 0x7fffffff;
+                s_mx[(l + 1) % 3] = (int)0x80000000;
+            }
             if (sparse) {
                 if (!nxt_zero)
                     for (int k = threadIdx.x; k < N; k += blockDim.x) nxt[k] = 0.0f;
@@ -462,12 +489,28 @@ __global__ void __launch_bounds__(kPostThreads, 2) residual_traj_kernel(PostArgs
                     c_sout += (unsigned long long)nt;
                 }
             } else {
+                float mn = __int_as_float(0x7f800000), mx = -__int_as_float(0x7f800000);
                 const int mine = post_row_layer<MODE_RESIDUAL, 17, 16, 1>(Ld, N, dup, a.ymax, a.prune_eps, cur, nxt,
-                                                                          ac, nullptr, a.force_ell);
+                                                                          ac, nullptr, a.force_ell, mn, mx);
                 const int wsum = __reduce_add_sync(0xffffffffu, mine);
-                if ((threadIdx.x & 31) == 0 && wsum) atomicAdd(&s_nz[l % 3], wsum);
+                // order-preserving integer codes of the range (bitwise-equal floats <-> equal codes)
+                auto code = [](float f) {
+                    const int b = __float_as_int(f);
+                    return b ^ ((b >> 31) & 0x7fffffff);
+                };
+                const int wmn = __reduce_min_sync(0xffffffffu, code(mn)), wmx = __reduce_max_sync(0xffffffffu, code(mx));
+                if ((threadIdx.x & 31) == 0) {
+                    if (wsum) atomicAdd(&s_nz[l % 3], wsum);
+                    atomicMin(&s_mn[l % 3], wmn);
+                    atomicMax(&s_mx[l % 3], wmx);
+                }
                 __syncthreads();
                 cnt = s_nz[l % 3];
+                rowconst = s_mn[l % 3] == s_mx[l % 3];
+                if (rowconst) {
+                    const int c0 = s_mn[l % 3];
+                    v0 = __int_as_float(c0 ^ ((c0 >> 31) & 0x7fffffff));
+                }
                 nxt_zero = false;
                 nnz = cnt;
                 listed = false;
@@ -477,19 +520,13 @@ __global__ void __launch_bounds__(kPostThreads, 2) residual_traj_kernel(PostArgs
                 alive = false;
                 break;
             }
-            if (a.scalar_ok && l + 1 < a.L && l + 1 - a.t >= cfrom) {
-                // the centroid row is constant from here on (its a_c rows are): if this residue row is
-                // constant too, Eq. 5 maps it to a constant row every layer -- carry it by a scalar
-                // (R25/R26 argument; bit-identical)
-                const float v0 = nxt[0];
-                bool eq = true;
-                for (int k = threadIdx.x; k < N; k += blockDim.x) eq = eq && nxt[k] == v0;
-                if (__syncthreads_and(eq)) {
-                    cst = true;
-                    vr = v0;
-                    ++l;
-                    break;
-                }
+            if (a.scalar_ok && rowconst && l + 1 < a.L && l + 1 - a.t >= cfrom) {
+                // the centroid row is constant from here on (its a_c rows are) and this residue row is constant
+                // too: Eq. 5 maps it to a constant row every layer -- carry it by a scalar (R25/R26; bit-identical)
+                cst = true;
+                vr = v0;
+                ++l;
+                break;
             }
             fill_halo(nxt, N, h);
             __syncthreads();
@@ -503,10 +540,35 @@ __global__ void __launch_bounds__(kPostThreads, 2) residual_traj_kernel(PostArgs
             Ld = Lnext;
         }
         if (cst) {  // layers l .. L-1: every thread evaluates the same scalar chain
+            // the centroid's pre-activation rows are constant from here on: gather their values (one per
+            // layer) into shared memory first -- the row buffers are free now -- so the serial chain does not
+            // wait on one L2 round trip per layer
+            float* s_acv = sm;       // [L - l] a_c values
+            float2* s_wb = reinterpret_cast<float2*>(sm + ((a.L - l + 1) & ~1));  // [L - l] (w0, b0)
+            const int nl = a.L - l;
+            const bool fits = 3 * nl <= 2 * (N + h);
+            if (fits) {
+                for (int i = threadIdx.x; i < nl; i += blockDim.x) {
+                    s_acv[i] = __ldg(a.a_all + ((size_t)(l + i - a.t) * a.s + slot) * N);
+                    const PostLayer* pl = a.layers + l + i;
+                    s_wb[i] = make_float2(pl->w0, pl->b0);
+                }
+                __syncthreads();
+            }
+            const int l0 = l;
             for (; l < a.L; ++l) {
-                const PostLayer* pl = a.layers + l;
-                const float w0 = pl->w0, b0 = pl->b0;
-                const float acv = __ldg(a.a_all + ((size_t)(l - a.t) * a.s + slot) * N);
+                float w0, b0, acv;
+                if (fits) {
+                    const float2 wb = s_wb[l - l0];
+                    w0 = wb.x;
+                    b0 = wb.y;
+                    acv = s_acv[l - l0];
+                } else {
+                    const PostLayer* pl = a.layers + l;
+                    w0 = pl->w0;
+                    b0 = pl->b0;
+                    acv = __ldg(a.a_all + ((size_t)(l - a.t) * a.s + slot) * N);
+                }
                 float acc = 0.0f;
 #pragma unroll
                 for (int n2 = 0; n2 < kPK; ++n2) acc = fmaf(vr, w0, acc);

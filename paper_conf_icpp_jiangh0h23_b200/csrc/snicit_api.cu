@@ -125,6 +125,8 @@ struct snicit_network {
     DevBuf<int> clist, clayer;    // constant rows of the per-layer pre phase (R26)
     DevBuf<float> cval;
     DevBuf<int> cfrom;        // per centroid: first post layer with a constant a_c row (residual_traj)
+    DevBuf<int> dist;         // [rows][s] L0 distances of Alg. 2 (map_residual pass 1)
+    DevBuf<int> rnnz;         // [rows] non-zeros of each residue row at t
     DevBuf<uint8_t> rconst;   // rows constant at t (R26): flag + value, set by the pre phase
     DevBuf<float> rval;
     bool last_pre_const = false;
@@ -350,6 +352,8 @@ void snicit_free_network(snicit_network* net) {
     net->rval.release();
     net->a_all.release();
     net->ctr64.release();
+    net->dist.release();
+    net->rnnz.release();
     delete net;
 }
 
@@ -692,6 +696,8 @@ static cudaError_t ensure_workspace(snicit_network* net, int64_t R, int s, int n
     if ((e = net->col_idx.ensure(ss)) != cudaSuccess) return e;
     if ((e = net->iota_s.ensure(ss)) != cudaSuccess) return e;
     if ((e = net->F.ensure((size_t)std::max(n, 1) * ss)) != cudaSuccess) return e;
+    if ((e = net->dist.ensure(rows * ss)) != cudaSuccess) return e;
+    if ((e = net->rnnz.ensure(rows)) != cudaSuccess) return e;
     if ((e = net->cscratch.ensure((size_t)compact_scratch_ints((int)rows))) != cudaSuccess) return e;
     if (net->segflag.n < rows) {
         if ((e = net->segflag.ensure(rows)) != cudaSuccess) return e;
@@ -824,6 +830,7 @@ static snicit_status infer_core(snicit_network* net, const float* y0, int64_t ba
     if (batch > 0 && !y0 && y0_mode < 2) return fail(SNICIT_E_INVALID_ARG, "y0 NULL");
     if (t < 0) return fail(SNICIT_E_INVALID_ARG, "threshold_layer < 0");
     if (s < 1) return fail(SNICIT_E_INVALID_ARG, "centroid_count < 1");
+    if (s > 1024) return fail(SNICIT_E_UNSUPPORTED, "centroid_count > 1024");
     if (row_offset < 0) return fail(SNICIT_E_INVALID_ARG, "row_offset < 0");
     if ((y0_on_device && misaligned16(y0)) || (y_out_on_device && misaligned16(y_out)) ||
         (y0_mode == 3 && misaligned16(bits)))
@@ -1095,7 +1102,8 @@ static snicit_status infer_core(snicit_network* net, const float* y0, int64_t ba
         if (opt.timing) CUDA_TRY(cudaEventRecord(net->ev[6], st));
         CUDA_TRY(launch_map_residual(cur, N, list_cur, cnt_cur, net->cent.p, cnt + CNT_NCENT, net->M.p, net->cslot.p,
                                      net->ne_row.p, net->flag_pos.p, yhat, net->cbuf0.p, R, net->num_sms, st,
-                                     net->rconst.p, net->rval.p, net->ctr64.p + C64_RES_NNZ));
+                                     net->rconst.p, net->rval.p, net->ctr64.p + C64_RES_NNZ, net->dist.p, s,
+                                     net->rnnz.p));
         if (opt.timing) CUDA_TRY(cudaEventRecord(net->ev[7], st));
         net->ev_map = opt.timing != 0;
         int* rlist = net->res0.p;
@@ -1188,6 +1196,7 @@ static snicit_status infer_core(snicit_network* net, const float* y0, int64_t ba
             pa.cdone = cdone;
             pa.ctr64 = net->ctr64.p;
             pa.res_sparse = opt.res_sparse;
+            pa.rnnz = net->rnnz.p;
             CUDA_TRY(cudaMemsetAsync(cnt + CNT_WORK, 0, 2 * sizeof(int), st));
             pa.force_ell = opt.kernel == SNICIT_KERNEL_ELL ? 1 : 0;
             // cluster (DSMEM) trajectory when every post layer is circulant and partition-compatible

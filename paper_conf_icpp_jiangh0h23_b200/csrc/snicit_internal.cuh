@@ -234,6 +234,7 @@ struct PostArgs {
     int scalar_ok;       // every post layer circulant with uniform weight and bias: constant residue rows
                          //   over constant centroids are carried by a scalar (residual_traj_kernel)
     int res_sparse;      // 1: sparse-entry residue form for residue rows with few non-zeros (circulant layers)
+    const int* rnnz;     // nullable: non-zeros of each row's residue at t (map_residual), by row id
     unsigned long long* ctr64;  // nullable: work counters (Ctr64)
 };
 // 64-bit work counters of one infer (stats): residue entries at t, residue row-layers by form, outputs
@@ -330,8 +331,8 @@ cudaError_t launch_prune(const double* F, const int* count, int s, int n_seg, fl
 cudaError_t launch_map_residual(const float* y, int N, const int* rows, const int* count, const int* cent,
                                 const int* n_cent, int* M, int* cslot, uint8_t* ne_row, uint8_t* flag_pos,
                                 float* yhat, float* cbuf, int max_rows, int num_sms, cudaStream_t st,
-                                const uint8_t* rconst = nullptr, const float* rval = nullptr,
-                                unsigned long long* nnz_sum = nullptr);
+                                const uint8_t* rconst, const float* rval, unsigned long long* nnz_sum,
+                                int* dist /* [max_rows][s] scratch */, int s, int* rnnz /* nullable, by row */);
 cudaError_t launch_recover(int N, int R, int plain, const float* yfinal, const uint8_t* live_row, const int* M,
                            const int* cslot, const uint8_t* ne_row, const float* cbuf, float* y_out,
                            uint8_t* cat, int num_sms, cudaStream_t st, int dead_zeroed = 0);
