@@ -138,7 +138,9 @@ typedef struct {
     int64_t res_sparse_rl;    /* residue row-layers evaluated in the sparse-entry form */
     int64_t res_sparse_out;   /* outputs evaluated by the sparse-entry form (32 fma each) */
     int64_t res_scalar_rl;    /* residue row-layers carried by a scalar (constant rows, R25/R26) */
-    double t_map_ms;          /* map_residual kernel (Alg. 2), CUDA events (options.timing), else -1 */
+    int64_t map_rows;         /* rows whose L0 distances to every centroid Alg. 2 computed (the others: centroid
+                                 rows and constant rows with an equal constant centroid, R26) */
+    double t_map_ms;          /* map_residual kernels (Alg. 2), CUDA events (options.timing), else -1 */
     double t_residual_ms;     /* residue trajectory kernel (Eq. 5, fused post mode), else -1 */
 } snicit_stats_t;
 

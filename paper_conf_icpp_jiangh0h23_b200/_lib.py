@@ -45,7 +45,8 @@ class Stats(ctypes.Structure):
                 ("const_centroids", ctypes.c_int32), ("pre_fused", ctypes.c_int32),
                 ("pre_const_rows", ctypes.c_int32), ("pre_full_rows", ctypes.c_int64),
                 ("res_nnz_at_t", ctypes.c_int64), ("res_full_rl", ctypes.c_int64), ("res_sparse_rl", ctypes.c_int64),
-                ("res_sparse_out", ctypes.c_int64), ("res_scalar_rl", ctypes.c_int64), ("t_map_ms", ctypes.c_double),
+                ("res_sparse_out", ctypes.c_int64), ("res_scalar_rl", ctypes.c_int64), ("map_rows", ctypes.c_int64),
+                ("t_map_ms", ctypes.c_double),
                 ("t_residual_ms", ctypes.c_double)]
 
     def as_dict(self):

@@ -331,7 +331,8 @@ __global__ void __launch_bounds__(kMapThreads) map_dist_kernel(const float* __re
                                                                const int* count, const int* cent, const int* n_cent,
                                                                int* __restrict__ dist, int s,
                                                                const uint8_t* __restrict__ rconst,
-                                                               const float* __restrict__ rval) {
+                                                               const float* __restrict__ rval,
+                                                               unsigned long long* map_rows) {
     extern __shared__ float4 s_c4[];
     __shared__ float s_cv[1024];  // constant value of centroid c (R26) or NaN
     constexpr int TK4 = TK / 4, CH = (TK4 + 31) / 32;  // float4 chunks per lane
@@ -385,6 +386,7 @@ __global__ void __launch_bounds__(kMapThreads) map_dist_kernel(const float* __re
         const int pcur = p;
         p = next_row(p + nwb);
         if (p < n) load_tile(p, yn);
+        if (map_rows && tile == 0 && lane == 0) atomicAdd(map_rows, 1ull);  // rows whose distances are computed
         for (int cg = 0; cg < Cp; cg += 32) {
             int cnt[32];
 #pragma unroll
@@ -530,15 +532,15 @@ cudaError_t launch_map_residual(const float* y, int N, const int* rows, const in
         return cudaGetLastError();
     };
     e = one((const void*)map_dist_kernel<512>, 512, [&](int g) {
-        map_dist_kernel<512><<<g, kMapThreads, smem, st>>>(y, N, rows, count, cent, n_cent, dist, s, rconst, rval);
+        map_dist_kernel<512><<<g, kMapThreads, smem, st>>>(y, N, rows, count, cent, n_cent, dist, s, rconst, rval, nnz_sum ? nnz_sum + (C64_MAP_ROWS - C64_RES_NNZ) : nullptr);
     });
     if (e == cudaSuccess)
         e = one((const void*)map_dist_kernel<128>, 128, [&](int g) {
-            map_dist_kernel<128><<<g, kMapThreads, smem, st>>>(y, N, rows, count, cent, n_cent, dist, s, rconst, rval);
+            map_dist_kernel<128><<<g, kMapThreads, smem, st>>>(y, N, rows, count, cent, n_cent, dist, s, rconst, rval, nnz_sum ? nnz_sum + (C64_MAP_ROWS - C64_RES_NNZ) : nullptr);
         });
     if (e == cudaSuccess)
         e = one((const void*)map_dist_kernel<32>, 32, [&](int g) {
-            map_dist_kernel<32><<<g, kMapThreads, smem, st>>>(y, N, rows, count, cent, n_cent, dist, s, rconst, rval);
+            map_dist_kernel<32><<<g, kMapThreads, smem, st>>>(y, N, rows, count, cent, n_cent, dist, s, rconst, rval, nnz_sum ? nnz_sum + (C64_MAP_ROWS - C64_RES_NNZ) : nullptr);
         });
     if (e != cudaSuccess) return e;
     int grid = num_sms * 8;

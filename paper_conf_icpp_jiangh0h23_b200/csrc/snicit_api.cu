@@ -23,7 +23,7 @@ using namespace snicit;
 
 // the Python binding mirrors these structs (paper_conf_icpp_jiangh0h23_b200/_lib.py; tests/test_abi.py)
 static_assert(sizeof(snicit_options) == 56, "snicit_options layout");
-static_assert(sizeof(snicit_stats_t) == 184, "snicit_stats_t layout");
+static_assert(sizeof(snicit_stats_t) == 192, "snicit_stats_t layout");
 
 namespace {
 
@@ -1480,7 +1480,7 @@ snicit_status snicit_stats(snicit_network* net, snicit_stats_t* out) {
         net->stats.pre_const_rows = v;
     }
     net->stats.res_nnz_at_t = net->stats.res_full_rl = net->stats.res_sparse_rl = 0;
-    net->stats.res_sparse_out = net->stats.res_scalar_rl = 0;
+    net->stats.res_sparse_out = net->stats.res_scalar_rl = net->stats.map_rows = 0;
     if (net->last_converted) {
         unsigned long long c64[C64_N];
         CUDA_TRY(cudaMemcpyAsync(c64, net->ctr64.p, sizeof(c64), cudaMemcpyDeviceToHost, net->stream));
@@ -1490,6 +1490,7 @@ snicit_status snicit_stats(snicit_network* net, snicit_stats_t* out) {
         net->stats.res_sparse_rl = (int64_t)c64[C64_SPARSE_RL];
         net->stats.res_sparse_out = (int64_t)c64[C64_SPARSE_OUT];
         net->stats.res_scalar_rl = (int64_t)c64[C64_SCALAR_RL];
+        net->stats.map_rows = (int64_t)c64[C64_MAP_ROWS];
     }
     if (net->last_pre_fused) {
         CUDA_TRY(read_counter(net, CNT_PFCONST, &v));

@@ -239,7 +239,7 @@ struct PostArgs {
 };
 // 64-bit work counters of one infer (stats): residue entries at t, residue row-layers by form, outputs
 // evaluated by the sparse-entry form
-enum Ctr64 : int { C64_RES_NNZ = 0, C64_FULL_RL, C64_SPARSE_RL, C64_SPARSE_OUT, C64_SCALAR_RL, C64_N };
+enum Ctr64 : int { C64_RES_NNZ = 0, C64_FULL_RL, C64_SPARSE_RL, C64_SPARSE_OUT, C64_SCALAR_RL, C64_MAP_ROWS, C64_N };
 cudaError_t launch_acconst(const PostArgs& a, int C_max, cudaStream_t st);
 int post_fused_max_n();
 cudaError_t launch_centroid_traj(const PostArgs& a, int C_max, cudaStream_t st);
