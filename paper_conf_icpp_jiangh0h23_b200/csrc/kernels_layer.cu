@@ -167,6 +167,130 @@ __global__ void __launch_bounds__(kEllThreads, 1) layer_ell_kernel(LayerArgs a) 
     if (a.app_list) ell_flush(a, s_surv, &s_nsurv, &s_pos);
 }
 
+// ---- row-interleaved variant (the general-CSC hot path): the RT rows of a tile are stored
+// interleaved, element (k, r) at k RT + r, so one thread (output column j) fetches input k of all RT rows
+// with one 16-byte shared load (RT = 4) or two (RT = 8) instead of RT scattered 4-byte loads, and feeds
+// them to packed FFMA2 pairs (rows r, r + 1).  For RT = 8 the two 16-byte halves of input k are stored
+// in the order h0 = (k >> 2) & 1 first, so the first load of a warp touches chunk (2k + h0) mod 8 -- all
+// eight 16-byte bank groups -- instead of only the even ones.  Rows are loaded with coalesced float4
+// global loads and transposed on the shared-memory store; the next tile's rows are prefetched into L2.
+template <int RT>
+__device__ __forceinline__ int il_pos(int k, int r) {
+    if constexpr (RT == 8) {
+        const int h0 = (k >> 2) & 1;
+        return k * 8 + (((r >> 2) ^ h0) << 2) + (r & 3);
+    } else {
+        return k * RT + r;
+    }
+}
+
+template <int MODE, int RT, bool IDX16, bool UNIF, bool RAGGED>
+__global__ void __launch_bounds__(kEllThreads, 1) layer_ell_il_kernel(LayerArgs a) {
+    static_assert(RT == 2 || RT == 4 || RT == 8, "RT");
+    extern __shared__ __align__(128) unsigned char smem[];
+    const int N = a.N;
+    float* s_in = reinterpret_cast<float*>(smem);
+    int* s_flag = reinterpret_cast<int*>(s_in + (size_t)RT * N);
+    int* s_row = s_flag + RT;
+    int* s_slot = s_row + RT;
+    int* s_surv = s_slot + RT;  // kEllSurvCap surviving row ids (fused dead-row compaction)
+    __shared__ int s_nsurv, s_pos;
+
+    if (blockIdx.x == 0 && threadIdx.x == 0 && a.zero_count) *a.zero_count = 0;
+    if (threadIdx.x == 0) s_nsurv = 0;
+    const int count = *a.count;
+    const int ntiles = (count + RT - 1) / RT;
+    const int N4 = N >> 2;
+    __syncthreads();
+    for (int tile = blockIdx.x; tile < ntiles; tile += gridDim.x) {
+        const int r0 = tile * RT;
+        const int nr = min(RT, count - r0);
+        if (threadIdx.x < RT) {
+            const int row = a.rows[r0 + min((int)threadIdx.x, nr - 1)];
+            s_row[threadIdx.x] = row;
+            s_flag[threadIdx.x] = 0;
+            if constexpr (MODE == MODE_RESIDUAL) s_slot[threadIdx.x] = a.cslot[row];
+        } else if (threadIdx.x < 2 * RT) {  // the next tile's rows -> L2 while this one computes
+            const int nt = tile + gridDim.x, i = threadIdx.x - RT;
+            if (nt < ntiles && nt * RT + i < count)
+                bulk_prefetch_l2(a.yin + (size_t)a.rows[nt * RT + i] * N, (uint32_t)N * 4);
+        }
+        __syncthreads();
+        // transposed load: thread -> (row r, float4 chunk c)
+        for (int t = threadIdx.x; t < RT * N4; t += blockDim.x) {
+            const int r = t % RT, c = t / RT;
+            const float4 v = __ldg(reinterpret_cast<const float4*>(a.yin + (size_t)s_row[r] * N) + c);
+            s_in[il_pos<RT>(4 * c + 0, r)] = v.x;
+            s_in[il_pos<RT>(4 * c + 1, r)] = v.y;
+            s_in[il_pos<RT>(4 * c + 2, r)] = v.z;
+            s_in[il_pos<RT>(4 * c + 3, r)] = v.w;
+        }
+        __syncthreads();
+        int anyr = 0;  // bit r: row r has a non-zero output in this thread's columns
+        for (int j = threadIdx.x; j < N; j += blockDim.x) {
+            const int len = RAGGED ? (int)a.len[j] : a.K;
+            unsigned long long acc[RT / 2];
+#pragma unroll
+            for (int q = 0; q < RT / 2; ++q) acc[q] = 0ull;
+#pragma unroll 4
+            for (int n = 0; n < len; ++n) {
+                const size_t e = (size_t)n * N + j;
+                const int k = IDX16 ? (int)__ldg(a.idx16 + e) : __ldg(a.idx32 + e);
+                const float w = UNIF ? a.w0 : __ldg(a.val + e);
+                const unsigned long long W2 = f2_pack(w, w);
+                if constexpr (RT == 8) {
+                    const int h0 = (k >> 2) & 1;
+                    const float4 lo = *reinterpret_cast<const float4*>(s_in + k * 8 + (h0 << 2));        // rows 0..3
+                    const float4 hi = *reinterpret_cast<const float4*>(s_in + k * 8 + ((h0 ^ 1) << 2));  // rows 4..7
+                    acc[0] = f2_fma(f2_pack(lo.x, lo.y), W2, acc[0]);
+                    acc[1] = f2_fma(f2_pack(lo.z, lo.w), W2, acc[1]);
+                    acc[2] = f2_fma(f2_pack(hi.x, hi.y), W2, acc[2]);
+                    acc[3] = f2_fma(f2_pack(hi.z, hi.w), W2, acc[3]);
+                } else if constexpr (RT == 4) {
+                    const float4 v = *reinterpret_cast<const float4*>(s_in + k * 4);
+                    acc[0] = f2_fma(f2_pack(v.x, v.y), W2, acc[0]);
+                    acc[1] = f2_fma(f2_pack(v.z, v.w), W2, acc[1]);
+                } else {
+                    const float2 v = *reinterpret_cast<const float2*>(s_in + k * 2);
+                    acc[0] = f2_fma(f2_pack(v.x, v.y), W2, acc[0]);
+                }
+            }
+            const float bj = __ldg(a.bias + j);
+#pragma unroll
+            for (int q = 0; q < RT / 2; ++q) {
+                float z[2];
+                f2_unpack(acc[q], z[0], z[1]);
+#pragma unroll
+                for (int h = 0; h < 2; ++h) {
+                    const int r = 2 * q + h;
+                    if (r < nr) {
+                        const int row = s_row[r];
+                        const float v = epilogue<MODE>(a, z[h], bj, j, row, MODE == MODE_RESIDUAL ? s_slot[r] : 0);
+                        a.yout[(size_t)row * N + j] = v;
+                        if (v != 0.0f) anyr |= 1 << r;
+                    }
+                }
+            }
+        }
+#pragma unroll
+        for (int r = 0; r < RT; ++r)
+            if (anyr & (1 << r)) s_flag[r] = 1;
+        __syncthreads();
+        if (threadIdx.x < nr) {
+            const uint8_t f = s_flag[threadIdx.x] ? 1 : 0;
+            if (a.flag_pos) a.flag_pos[r0 + threadIdx.x] = f;
+            if (a.flag_row) a.flag_row[s_row[threadIdx.x]] = f;
+        }
+        if (a.app_list && threadIdx.x == 0) {
+            for (int i = 0; i < nr; ++i)
+                if (s_flag[i]) s_surv[s_nsurv++] = s_row[i];
+        }
+        __syncthreads();
+        if (a.app_list && s_nsurv > kEllSurvCap - RT) ell_flush(a, s_surv, &s_nsurv, &s_pos);
+    }
+    if (a.app_list) ell_flush(a, s_surv, &s_nsurv, &s_pos);
+}
+
 bool ell_smem_ok(int N) { return (size_t)N * 4 * 2 <= 200 * 1024 && N % 4 == 0; }
 
 template <int MODE, int RT, bool SMEM>
@@ -174,8 +298,14 @@ static cudaError_t launch_ell_t(const LayerArgs& a, int max_rows, int num_sms, c
     const size_t smem = (SMEM ? (size_t)RT * a.N * 4 : 0) + 16 + 12 * RT + 16 + 4 * kEllSurvCap;
     const bool i16 = a.idx16 != nullptr, unif = a.val == nullptr, rag = a.len != nullptr;
     void (*kern)(LayerArgs) = nullptr;
-#define SNICIT_PICK(I, U, G) \
-    if (i16 == I && unif == U && rag == G) kern = layer_ell_kernel<MODE, RT, I, U, G, SMEM>;
+    constexpr bool IL = SMEM && (RT == 2 || RT == 4 || RT == 8);  // row-interleaved tile
+#define SNICIT_PICK(I, U, G)                                                                 \
+    if (i16 == I && unif == U && rag == G) {                                                 \
+        if constexpr (IL)                                                                    \
+            kern = layer_ell_il_kernel<MODE, (IL ? RT : 2), I, U, G>;                        \
+        else                                                                                 \
+            kern = layer_ell_kernel<MODE, RT, I, U, G, SMEM>;                                \
+    }
     SNICIT_PICK(true, true, false)
     SNICIT_PICK(true, false, false)
     SNICIT_PICK(true, true, true)

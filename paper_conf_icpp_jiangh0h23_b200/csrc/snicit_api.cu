@@ -1133,8 +1133,10 @@ static snicit_status infer_core(snicit_network* net, const float* y0, int64_t ba
         // weights and bias.  Fused mode: in place, the trajectory kernels skip the carried rows.
         // Per-layer mode (no residues): into cbuf1; the layer loop is skipped when all were carried.
         bool const_ok = opt.post_const != 0 && opt.kernel != SNICIT_KERNEL_ELL;
+        // (any layer whose columns all hold K = 32 entries of one weight, with one bias: every output of a
+        // constant row evaluates the same stored-order chain -- circulant or not, R25)
         for (int l = tt; l < L && const_ok; ++l)
-            const_ok = use_circ(net, l, opt.kernel) && net->plan[l].uniform && net->plan[l].ubias;
+            const_ok = net->plan[l].uniform && net->plan[l].ubias && !net->plan[l].ragged && net->plan[l].K == 32;
         int* cdone = nullptr;
         bool all_const = false;
         if (const_ok && (fused || res_host == 0)) {
