@@ -90,6 +90,7 @@ __global__ void __launch_bounds__(kEllThreads, 1) layer_ell_kernel(LayerArgs a) 
     int* s_slot = s_row + RT;
     int* s_surv = s_slot + RT;  // kEllSurvCap surviving row ids (fused dead-row compaction)
     __shared__ int s_nsurv, s_pos;
+    __shared__ unsigned s_cmn[RT], s_cmx[RT];  // constant-row mode: each row's output range (bits)
 
     if (blockIdx.x == 0 && threadIdx.x == 0 && a.zero_count) *a.zero_count = 0;
     if (threadIdx.x == 0) s_nsurv = 0;
@@ -108,6 +109,8 @@ __global__ void __launch_bounds__(kEllThreads, 1) layer_ell_kernel(LayerArgs a) 
             const int row = a.rows[r0 + min((int)threadIdx.x, nr - 1)];
             s_row[threadIdx.x] = row;
             s_flag[threadIdx.x] = 0;
+            s_cmn[threadIdx.x] = 0xffffffffu;
+            s_cmx[threadIdx.x] = 0u;
             if constexpr (MODE == MODE_RESIDUAL) s_slot[threadIdx.x] = a.cslot[row];
         }
         __syncthreads();
@@ -125,6 +128,12 @@ __global__ void __launch_bounds__(kEllThreads, 1) layer_ell_kernel(LayerArgs a) 
         for (int r = 0; r < RT; ++r)
             base[r] = SMEM ? (s_in + (size_t)(r < nr ? r : 0) * N) : (a.yin + (size_t)s_row[r] * N);
         int anyr = 0;  // bit r: row r has a non-zero output in this thread's columns
+        unsigned rmn[RT], rmx[RT];  // constant-row mode: this thread's output range per row
+#pragma unroll
+        for (int r = 0; r < RT; ++r) {
+            rmn[r] = 0xffffffffu;
+            rmx[r] = 0u;
+        }
         for (int j = threadIdx.x; j < N; j += blockDim.x) {
             const int len = RAGGED ? (int)a.len[j] : a.K;
             float acc[RT];
@@ -145,17 +154,36 @@ __global__ void __launch_bounds__(kEllThreads, 1) layer_ell_kernel(LayerArgs a) 
                     const float v = epilogue<MODE>(a, acc[r], __ldg(a.bias + j), j, row, MODE == MODE_RESIDUAL ? s_slot[r] : 0);
                     a.yout[(size_t)row * N + j] = v;
                     if (v != 0.0f) anyr |= 1 << r;
+                    if (MODE == MODE_PLAIN) {
+                        const unsigned u = __float_as_uint(v + 0.0f);
+                        rmn[r] = min(rmn[r], u);
+                        rmx[r] = max(rmx[r], u);
+                    }
                 }
             }
         }
 #pragma unroll
         for (int r = 0; r < RT; ++r)
             if (anyr & (1 << r)) s_flag[r] = 1;
+        if (MODE == MODE_PLAIN && a.cmin) {  // constant-row mode (R26): each row's range over the tile's outputs
+#pragma unroll
+            for (int r = 0; r < RT; ++r) {
+                const unsigned wmn = __reduce_min_sync(0xffffffffu, rmn[r]), wmx = __reduce_max_sync(0xffffffffu, rmx[r]);
+                if ((threadIdx.x & 31) == 0) {
+                    atomicMin(&s_cmn[r], wmn);
+                    atomicMax(&s_cmx[r], wmx);
+                }
+            }
+        }
         __syncthreads();
         if (threadIdx.x < nr) {
             const uint8_t f = s_flag[threadIdx.x] ? 1 : 0;
             if (a.flag_pos) a.flag_pos[r0 + threadIdx.x] = f;
             if (a.flag_row) a.flag_row[s_row[threadIdx.x]] = f;
+            if (MODE == MODE_PLAIN && a.cmin) {  // the tile holds whole rows: the range is final
+                a.cmin[r0 + threadIdx.x] = s_cmn[threadIdx.x];
+                a.cmax[r0 + threadIdx.x] = s_cmx[threadIdx.x];
+            }
         }
         if (a.app_list && threadIdx.x == 0) {
             for (int i = 0; i < nr; ++i)
@@ -195,6 +223,7 @@ __global__ void __launch_bounds__(kEllThreads, 1) layer_ell_il_kernel(LayerArgs 
     int* s_slot = s_row + RT;
     int* s_surv = s_slot + RT;  // kEllSurvCap surviving row ids (fused dead-row compaction)
     __shared__ int s_nsurv, s_pos;
+    __shared__ unsigned s_cmn[RT], s_cmx[RT];  // constant-row mode: each row's output range (bits)
 
     if (blockIdx.x == 0 && threadIdx.x == 0 && a.zero_count) *a.zero_count = 0;
     if (threadIdx.x == 0) s_nsurv = 0;
@@ -209,6 +238,8 @@ __global__ void __launch_bounds__(kEllThreads, 1) layer_ell_il_kernel(LayerArgs 
             const int row = a.rows[r0 + min((int)threadIdx.x, nr - 1)];
             s_row[threadIdx.x] = row;
             s_flag[threadIdx.x] = 0;
+            s_cmn[threadIdx.x] = 0xffffffffu;
+            s_cmx[threadIdx.x] = 0u;
             if constexpr (MODE == MODE_RESIDUAL) s_slot[threadIdx.x] = a.cslot[row];
         } else if (threadIdx.x < 2 * RT) {  // the next tile's rows -> L2 while this one computes
             const int nt = tile + gridDim.x, i = threadIdx.x - RT;
@@ -227,6 +258,12 @@ __global__ void __launch_bounds__(kEllThreads, 1) layer_ell_il_kernel(LayerArgs 
         }
         __syncthreads();
         int anyr = 0;  // bit r: row r has a non-zero output in this thread's columns
+        unsigned rmn[RT], rmx[RT];  // constant-row mode: this thread's output range per row (bits, +0 for -0)
+#pragma unroll
+        for (int r = 0; r < RT; ++r) {
+            rmn[r] = 0xffffffffu;
+            rmx[r] = 0u;
+        }
         for (int j = threadIdx.x; j < N; j += blockDim.x) {
             const int len = RAGGED ? (int)a.len[j] : a.K;
             unsigned long long acc[RT / 2];
@@ -268,6 +305,11 @@ __global__ void __launch_bounds__(kEllThreads, 1) layer_ell_il_kernel(LayerArgs 
                         const float v = epilogue<MODE>(a, z[h], bj, j, row, MODE == MODE_RESIDUAL ? s_slot[r] : 0);
                         a.yout[(size_t)row * N + j] = v;
                         if (v != 0.0f) anyr |= 1 << r;
+                        if (MODE == MODE_PLAIN) {
+                            const unsigned u = __float_as_uint(v + 0.0f);
+                            rmn[r] = min(rmn[r], u);
+                            rmx[r] = max(rmx[r], u);
+                        }
                     }
                 }
             }
@@ -275,11 +317,25 @@ __global__ void __launch_bounds__(kEllThreads, 1) layer_ell_il_kernel(LayerArgs 
 #pragma unroll
         for (int r = 0; r < RT; ++r)
             if (anyr & (1 << r)) s_flag[r] = 1;
+        if (MODE == MODE_PLAIN && a.cmin) {  // constant-row mode (R26): each row's range over the tile's outputs
+#pragma unroll
+            for (int r = 0; r < RT; ++r) {
+                const unsigned wmn = __reduce_min_sync(0xffffffffu, rmn[r]), wmx = __reduce_max_sync(0xffffffffu, rmx[r]);
+                if ((threadIdx.x & 31) == 0) {
+                    atomicMin(&s_cmn[r], wmn);
+                    atomicMax(&s_cmx[r], wmx);
+                }
+            }
+        }
         __syncthreads();
         if (threadIdx.x < nr) {
             const uint8_t f = s_flag[threadIdx.x] ? 1 : 0;
             if (a.flag_pos) a.flag_pos[r0 + threadIdx.x] = f;
             if (a.flag_row) a.flag_row[s_row[threadIdx.x]] = f;
+            if (MODE == MODE_PLAIN && a.cmin) {  // the tile holds whole rows: the range is final
+                a.cmin[r0 + threadIdx.x] = s_cmn[threadIdx.x];
+                a.cmax[r0 + threadIdx.x] = s_cmx[threadIdx.x];
+            }
         }
         if (a.app_list && threadIdx.x == 0) {
             for (int i = 0; i < nr; ++i)

@@ -671,6 +671,13 @@ static bool use_col(const snicit_network* net, int l, int kernel_opt) {
     return use_circ(net, l, kernel_opt) && kernel_opt != SNICIT_KERNEL_CIRC_SMEM && net->plan[l].col;
 }
 
+// a general (ELL) layer on which a constant row stays constant: one weight, one bias, 32 entries in every
+// column (the chain every output evaluates is the same, R26); the ELL kernels report row output ranges
+static bool ell_const_ok(const snicit_network* net, int l, int kernel_opt) {
+    const LayerPlan& pl = net->plan[l];
+    return !use_circ(net, l, kernel_opt) && net->has_ell && pl.uniform && pl.ubias && !pl.ragged && pl.K == 32;
+}
+
 static cudaError_t run_layer(snicit_network* net, int l, int kernel_opt, int mode, LayerArgs a, int max_rows) {
     if (mode == MODE_PLAIN && use_col(net, l, kernel_opt))
         return launch_layer_circ_col(a, max_rows, net->num_sms, net->stream);
@@ -990,7 +997,8 @@ static snicit_status infer_core(snicit_network* net, const float* y0, int64_t ba
     // uniform weight and bias and run by the column-streaming or segmented kernel
     bool pcst = !pf && opt.pre_const != 0 && tt > 0 && R > 0 && opt.kernel == SNICIT_KERNEL_AUTO;
     for (int l = 0; l < tt && pcst; ++l)
-        pcst = net->pf_elig[l] != 0 && (use_col(net, l, opt.kernel) || use_seg(net, l, opt.kernel));
+        pcst = (net->pf_elig[l] != 0 && (use_col(net, l, opt.kernel) || use_seg(net, l, opt.kernel))) ||
+               ell_const_ok(net, l, opt.kernel);
     net->last_pre_const = pcst;
     if (pcst) CUDA_TRY(cudaMemsetAsync(cnt + CNT_CCOUNT, 0, sizeof(int), st));
     for (int l = 0; l < tt && !pf; ++l) {
@@ -1010,7 +1018,10 @@ static snicit_status infer_core(snicit_network* net, const float* y0, int64_t ba
         a.rows = lists[li];
         a.count = cnt + live_ctr[ci];
         // segmented layers: row flags OR-ed across CTAs + a compaction launch; the others append
-        const bool seg = use_seg(net, l, opt.kernel) && !use_col(net, l, opt.kernel);
+        // segmented layers (and general layers in constant-row mode): per-row flags / output ranges, then a
+        // separate compaction or split launch instead of the fused append
+        const bool seg = (use_seg(net, l, opt.kernel) && !use_col(net, l, opt.kernel)) ||
+                         (pcst && !use_circ(net, l, opt.kernel));
         a.row_ctr = net->rowctr.p;                     // column-streaming kernel: last warp of a row appends
         if (drop_now && !seg) {
             a.app_list = lists[li ^ 1];

@@ -252,3 +252,31 @@ def test_misaligned_device_pointer_rejected():
         y0 = buf[1:].view(9, 1024)  # contiguous, 4-byte offset
         with pytest.raises(Exception):
             g.infer(y0, t=2, s=8)
+
+
+@pytest.mark.parametrize("N,L,B,mode", [(1024, 12, 400, "perm"), (4096, 10, 150, "perm"), (1024, 9, 300, "random")])
+@pytest.mark.parametrize("drop", [1, 0])
+def test_general_layers_constant_rows(N, L, B, mode, drop):
+    """Constant-row mode (R26) of the general (ELL) layer kernels: rows whose outputs are all equal leave
+    the active list and are carried by a scalar chain, bit-identical to evaluating every live row (and
+    to the oracle), uncompressed and SNICIT (t = 4); constant centroid rows likewise (R25)."""
+    net = sdgc.gen_network(N, L, mode)
+    rs = np.random.RandomState(N + L)
+    Y0 = sdgc.gen_inputs(N, B)
+    Y0[1::5] = 0.0
+    Y0[2::5] = np.float32(32.0)
+    Y0[3::5] = np.float32(0.5)
+    plain = oracle.layers_f32(net, Y0)
+    with SnicitNetwork.from_network(net) as g:
+        g.set_stream(torch.cuda.current_stream())
+        for t in (L, 4):
+            Ya, ca, sa = _infer(g, Y0, t, drop_dead_rows=drop, pre_const=1)
+            Yb, cb, sb = _infer(g, Y0, t, drop_dead_rows=drop, pre_const=0, post_const=0)
+            assert np.array_equal(Ya, Yb) and np.array_equal(ca, cb)
+            assert np.array_equal(ca, oracle.categories(plain))
+            if t == L:
+                assert np.array_equal(Ya, plain)
+                if mode == "perm":  # uniform weights, 32 per column: the constant-row mode applies
+                    assert sa["pre_const_rows"] > 0 and sb["pre_const_rows"] == 0
+            else:
+                np.testing.assert_allclose(Ya, plain, atol=ATOL, rtol=RTOL)
