@@ -32,7 +32,8 @@ class Options(ctypes.Structure):
                 ("prune_eps", ctypes.c_float), ("drop_dead_rows", ctypes.c_int32), ("kernel", ctypes.c_int32),
                 ("timing", ctypes.c_int32), ("ne_interval", ctypes.c_int32), ("post_mode", ctypes.c_int32),
                 ("post_cluster", ctypes.c_int32), ("post_const", ctypes.c_int32),
-                ("pre_fused", ctypes.c_int32), ("pre_const", ctypes.c_int32), ("res_sparse", ctypes.c_int32)]
+                ("pre_fused", ctypes.c_int32), ("pre_const", ctypes.c_int32), ("res_sparse", ctypes.c_int32),
+                ("dyn_t", ctypes.c_int32)]
 
 
 class Stats(ctypes.Structure):

@@ -672,4 +672,77 @@ cudaError_t launch_export_categories(const int* catlist, const int* count, long 
     return cudaGetLastError();
 }
 
+// ------------------------------------------------------------------------------ dynamic t (probe)
+// Convergence statistics of the S probe rows after one layer (the dynamic threshold-layer heuristic,
+// SURVEY 8(f) rank 3; the paper's future work): out[0] = live rows (any non-zero),
+// out[1] = 1 if every live row equals the first live row (exact ==, reading R19), out[2] = distinct live
+// rows by a 32-bit hash (a heuristic count: collisions can only lower it).  One CTA.
+__global__ void __launch_bounds__(256) probe_stat_kernel(const float* __restrict__ y, int S, int N, int* out) {
+    __shared__ int s_live[1024];
+    __shared__ unsigned s_hash[1024];
+    __shared__ int s_first, s_ident;
+    const int lane = threadIdx.x & 31, warp = threadIdx.x >> 5, nw = blockDim.x >> 5;
+    for (int i = warp; i < S; i += nw) {  // warp per row: live flag and hash
+        const float* r = y + (size_t)i * N;
+        int any = 0;
+        unsigned h = 0;
+        for (int k = lane; k < N; k += 32) {
+            const float v = r[k];
+            any |= v != 0.0f;
+            const unsigned b = __float_as_uint(v + 0.0f);  // +0 for -0 (== semantics)
+            h += (b ^ (b >> 15)) * (2u * (unsigned)k + 0x9E3779B1u);
+        }
+        any = __any_sync(0xffffffffu, any);
+        h = __reduce_add_sync(0xffffffffu, h);
+        if (lane == 0) {
+            s_live[i] = any;
+            s_hash[i] = h;
+        }
+    }
+    __syncthreads();
+    if (threadIdx.x == 0) {
+        int f = -1, live = 0;
+        for (int i = 0; i < S; ++i)
+            if (s_live[i]) {
+                ++live;
+                if (f < 0) f = i;
+            }
+        s_first = f;
+        s_ident = 1;
+        out[0] = live;
+    }
+    __syncthreads();
+    const int f = s_first;
+    if (f >= 0) {  // exact comparison of every live row with the first one
+        int ok = 1;
+        for (int i = f + 1 + warp; i < S && ok; i += nw) {
+            if (!s_live[i]) continue;
+            const float* a = y + (size_t)f * N;
+            const float* b = y + (size_t)i * N;
+            int eq = 1;
+            for (int k = lane; k < N && eq; k += 32) eq = a[k] == b[k];
+            eq = __all_sync(0xffffffffu, eq);
+            ok = eq;
+        }
+        if (lane == 0 && !ok) s_ident = 0;
+    }
+    __syncthreads();
+    if (threadIdx.x == 0) {
+        int uniq = 0;
+        for (int i = 0; i < S; ++i) {
+            if (!s_live[i]) continue;
+            bool dup = false;
+            for (int j = 0; j < i && !dup; ++j) dup = s_live[j] && s_hash[j] == s_hash[i];
+            uniq += !dup;
+        }
+        out[1] = f < 0 ? 1 : s_ident;
+        out[2] = uniq;
+    }
+}
+cudaError_t launch_probe_stat(const float* y, int S, int N, int* out, cudaStream_t st) {
+    if (S > 1024) return cudaErrorInvalidValue;
+    probe_stat_kernel<<<1, 256, 0, st>>>(y, S, N, out);
+    return cudaGetLastError();
+}
+
 }  // namespace snicit

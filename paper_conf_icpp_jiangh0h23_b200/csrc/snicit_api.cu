@@ -22,7 +22,7 @@
 using namespace snicit;
 
 // the Python binding mirrors these structs (paper_conf_icpp_jiangh0h23_b200/_lib.py; tests/test_abi.py)
-static_assert(sizeof(snicit_options) == 56, "snicit_options layout");
+static_assert(sizeof(snicit_options) == 60, "snicit_options layout");
 static_assert(sizeof(snicit_stats_t) == 192, "snicit_stats_t layout");
 
 namespace {
@@ -82,7 +82,7 @@ inline bool misaligned16(const void* p) { return p && (reinterpret_cast<uintptr_
 // device counters (one int each)
 enum Counter {
     CNT_LIVE0 = 0, CNT_LIVE1, CNT_LIVE2, CNT_ORD, CNT_RES0, CNT_RES1, CNT_NCENT, CNT_SEFF, CNT_ALL, CNT_NCAT,
-    CNT_WORK, CNT_ALIVE, CNT_CDONE, CNT_PFWORK, CNT_PFCONST, CNT_CCOUNT, CNT_N
+    CNT_WORK, CNT_ALIVE, CNT_CDONE, CNT_PFWORK, CNT_PFCONST, CNT_CCOUNT, CNT_PROBE, CNT_N
 };
 
 }  // namespace
@@ -127,6 +127,9 @@ struct snicit_network {
     DevBuf<int> cfrom;        // per centroid: first post layer with a constant a_c row (residual_traj)
     DevBuf<int> dist;         // [rows][s] L0 distances of Alg. 2 (map_residual pass 1)
     DevBuf<int> rnnz;         // [rows] non-zeros of each residue row at t
+    DevBuf<float> probe0, probe1;  // dynamic t: the probe rows (ping-pong)
+    DevBuf<int> pstat;             // dynamic t: per probe layer (live, identical, distinct)
+    int probe_layers = 0;
     DevBuf<uint8_t> rconst;   // rows constant at t (R26): flag + value, set by the pre phase
     DevBuf<float> rval;
     bool last_pre_const = false;
@@ -298,6 +301,7 @@ void snicit_default_options(snicit_options* opt) {
     opt->pre_fused = 1;
     opt->pre_const = 1;
     opt->res_sparse = 1;
+    opt->dyn_t = 0;
 }
 
 const char* snicit_last_error(void) { return g_last_error.c_str(); }
@@ -354,6 +358,9 @@ void snicit_free_network(snicit_network* net) {
     net->ctr64.release();
     net->dist.release();
     net->rnnz.release();
+    net->probe0.release();
+    net->probe1.release();
+    net->pstat.release();
     delete net;
 }
 
@@ -822,6 +829,60 @@ static cudaError_t stream_upload(snicit_network* net, void* dst, const void* src
     return cudaSuccess;
 }
 
+// Dynamic threshold layer ("determine t dynamically" is the paper's future work,
+// P:1619-1621).  Any t gives the plain result, so t only decides the cost.  The first
+// S = min(s, R) rows of the batch -- the rows Alg. 1 samples -- are run layer by layer on the
+// side; t is the first layer after which every live probe row is identical (the clustering then finds
+// one centroid and no residue among them), at most tmax.  If that never happens and more than S/2 of the
+// probe rows are still distinct at tmax, clustering cannot compress the batch and the
+// uncompressed path is taken (t = L).  Statistics are read back every 4 layers.
+static cudaError_t choose_t(snicit_network* net, const float* src, const uint32_t* bits, float one, int R, int s,
+                            int tmax, int* t_out) {
+    const int N = net->N, L = net->L;
+    const int S = std::min(std::min(s, R), 1024);
+    cudaStream_t st = net->stream;
+    cudaError_t e;
+    if ((e = net->probe0.ensure((size_t)S * N)) != cudaSuccess) return e;
+    if ((e = net->probe1.ensure((size_t)S * N)) != cudaSuccess) return e;
+    if ((e = net->pstat.ensure((size_t)3 * (tmax + 1))) != cudaSuccess) return e;
+    if ((e = net->iota_s.ensure((size_t)std::max(S, 1))) != cudaSuccess) return e;
+    if (src)
+        e = cudaMemcpyAsync(net->probe0.p, src, sizeof(float) * (size_t)S * N, cudaMemcpyDeviceToDevice, st);
+    else
+        e = launch_unpack_bits(bits, S, N, one, net->probe0.p, net->num_sms, st);
+    if (e != cudaSuccess) return e;
+    if ((e = launch_iota(net->iota_s.p, S, net->counters.p + CNT_PROBE, st)) != cudaSuccess) return e;
+    std::vector<int> h((size_t)3 * (tmax + 1));
+    float* pin = net->probe0.p;
+    float* pout = net->probe1.p;
+    int done = 0, chosen = -1;
+    net->probe_layers = 0;
+    for (int l = 0; l < tmax && chosen < 0; ++l) {
+        LayerArgs a = layer_args(net, l, false);
+        a.yin = pin;
+        a.yout = pout;
+        a.rows = net->iota_s.p;
+        a.count = net->counters.p + CNT_PROBE;
+        a.row_ctr = net->rowctr.p;
+        if ((e = run_layer(net, l, SNICIT_KERNEL_AUTO, MODE_PLAIN, a, S)) != cudaSuccess) return e;
+        if ((e = launch_probe_stat(pout, S, N, net->pstat.p + 3 * (l + 1), st)) != cudaSuccess) return e;
+        std::swap(pin, pout);
+        net->probe_layers = l + 1;
+        if ((l + 1) % 4 == 0 || l + 1 == tmax) {
+            if ((e = cudaMemcpyAsync(h.data() + 3 * (done + 1), net->pstat.p + 3 * (done + 1),
+                                     sizeof(int) * 3 * (l + 1 - done), cudaMemcpyDeviceToHost, st)) != cudaSuccess)
+                return e;
+            if ((e = cudaStreamSynchronize(st)) != cudaSuccess) return e;
+            for (int k = done + 1; k <= l + 1 && chosen < 0; ++k)
+                if (h[3 * k] == 0 || h[3 * k + 1]) chosen = k;
+            done = l + 1;
+        }
+    }
+    if (chosen < 0) chosen = (2 * h[3 * tmax + 2] > S) ? L : tmax;
+    *t_out = chosen;
+    return cudaSuccess;
+}
+
 // y0_mode: 0 = y0 is a device pointer, 1 = host pointer, 2 = the input rows are already in net->Ya,
 // 3 = packed binary rows `bits` (device-accessible, possibly host-mapped) read by the row-resident
 // kernel (the caller checked pf_plan)
@@ -855,6 +916,7 @@ static snicit_status infer_core(snicit_network* net, const float* y0, int64_t ba
     if (opt.pre_fused < 0 || opt.pre_fused > 4) return fail(SNICIT_E_INVALID_ARG, "bad pre_fused");
     if (opt.pre_const < 0 || opt.pre_const > 1) return fail(SNICIT_E_INVALID_ARG, "bad pre_const");
     if (opt.res_sparse < 0 || opt.res_sparse > 1) return fail(SNICIT_E_INVALID_ARG, "bad res_sparse");
+    if (opt.dyn_t < 0 || opt.dyn_t > 1) return fail(SNICIT_E_INVALID_ARG, "bad dyn_t");
     if (opt.kernel == SNICIT_KERNEL_ELL && !net->has_ell)
         return fail(SNICIT_E_UNSUPPORTED, "network loaded in compact circulant form has no ELL copy");
     const int N = net->N, L = net->L;
@@ -863,7 +925,7 @@ static snicit_status infer_core(snicit_network* net, const float* y0, int64_t ba
             if (net->plan[l].kind == 0)
                 return fail(SNICIT_E_UNSUPPORTED, "layer " + std::to_string(l) + " is not circulant");
     const int R = (int)batch;
-    const int tt = std::min(t, L);
+    int tt = std::min(t, L);
     const int n_seg = opt.n_segments == 0 ? N : opt.n_segments;
     const int ne_interval = opt.ne_interval > 0 ? opt.ne_interval : 64;
     DeviceGuard dg(net->device);
@@ -891,7 +953,7 @@ static snicit_status infer_core(snicit_network* net, const float* y0, int64_t ba
     } else {
         if (y0_mode == 1 && R > 0) {
             int H_ = 0, g_ = 0;
-            if (pf_plan(net, tt, opt, R, &H_, &g_)) {  // the row-resident kernel polls the chunks' flags
+            if (!opt.dyn_t && pf_plan(net, tt, opt, R, &H_, &g_)) {  // the row-resident kernel polls the chunks' flags
                 CUDA_TRY(stream_upload(net, net->Ya.p, y0, sizeof(float) * (size_t)N, R, &bits_ready, &ready_rows));
                 host_streamed = true;
             } else {
@@ -900,6 +962,14 @@ static snicit_status infer_core(snicit_network* net, const float* y0, int64_t ba
         }
         cur = net->Ya.p;
         nxt_i = 1;
+    }
+    // ---- dynamic threshold layer (options.dyn_t): t is chosen from the first s rows before the pre phase
+    if (opt.dyn_t && tt > 0 && R > 0) {
+        int chosen = tt;
+        CUDA_TRY(choose_t(net, cur, y0_mode == 3 ? bits : nullptr, one, R, s, tt, &chosen));
+        tt = chosen;
+        stats.threshold_layer = tt;
+        launches += 2 * net->probe_layers + 2;
     }
     int* cnt = net->counters.p;
     int* scratch = net->cscratch.p;
@@ -1386,7 +1456,8 @@ snicit_status snicit_infer_packed(snicit_network* net, const uint32_t* y0_bits, 
         snicit_default_options(&o);
     int H = 0, gen = 0;
     bool cl = false, bits_ok = true;
-    const bool direct = N % 128 == 0 && pf_plan(net, std::min(t, net->L), o, R, &H, &gen, &cl, &bits_ok) && bits_ok;
+    const bool direct = N % 128 == 0 && !o.dyn_t && pf_plan(net, std::min(t, net->L), o, R, &H, &gen, &cl, &bits_ok) &&
+                        bits_ok;
     const int* ready = nullptr;
     int ready_rows = 0;
     bool streamed = false;

@@ -339,6 +339,8 @@ cudaError_t launch_recover(int N, int R, int plain, const float* yfinal, const u
 // packed binary rows -> fp32 rows: y[r][j] = bit j of row r ? one : 0 (snicit_infer_packed)
 cudaError_t launch_unpack_bits(const uint32_t* bits, int R, int N, float one, float* y, int num_sms, cudaStream_t st);
 cudaError_t launch_mark_rows(const int* rows, const int* count, uint8_t* flag_row, int max_rows, cudaStream_t st);
+// dynamic t: convergence statistics of S probe rows (live, all identical, distinct by hash) -> out[3]
+cudaError_t launch_probe_stat(const float* y, int S, int N, int* out, cudaStream_t st);
 cudaError_t launch_export_categories(const int* catlist, const int* count, long long offset, long long* out,
                                      long long cap, cudaStream_t st);
 

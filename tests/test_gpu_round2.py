@@ -280,3 +280,49 @@ def test_general_layers_constant_rows(N, L, B, mode, drop):
                     assert sa["pre_const_rows"] > 0 and sb["pre_const_rows"] == 0
             else:
                 np.testing.assert_allclose(Ya, plain, atol=ATOL, rtol=RTOL)
+
+
+# ------------------------------------------------------------------------------ dynamic t (f3)
+
+def test_dynamic_threshold_layer():
+    """dyn_t: t is chosen from the first s rows (the first layer after which all live probe rows are
+    identical, at most threshold_layer; the uncompressed path when they stay distinct).  Any t gives the
+    plain result: categories equal the oracle's, activations within tolerance, and the chosen t is the
+    one the rule names on the oracle's own layer-by-layer rows."""
+    net = sdgc.gen_network(1024, 120, "radix")
+    Y0 = sdgc.gen_inputs(1024, 2000)
+    plain = oracle.layers_f32_fast(net, Y0)
+    # the rule on the oracle: first l with every live row among the first 32 identical
+    want = None
+    y = Y0[:32].copy()
+    for l in range(30):
+        y = oracle.layers_f32(net, y, l, l + 1)
+        live = y[(y != 0).any(1)]
+        if len(live) == 0 or (live == live[0]).all():
+            want = l + 1
+            break
+    with SnicitNetwork.from_network(net) as g:
+        g.set_stream(torch.cuda.current_stream())
+        Y, cats, st = _infer(g, Y0, 30, dyn_t=1)
+        assert st["threshold_layer"] == (want if want is not None else 30)
+        assert np.array_equal(cats, oracle.categories(plain))
+        np.testing.assert_allclose(Y, plain, atol=ATOL, rtol=RTOL)
+        # packed input and host input choose the same t
+        from paper_conf_icpp_jiangh0h23_b200 import pack_rows
+        out = torch.empty((2000, 1024), dtype=torch.float32, device="cuda")
+        g.infer_packed(pack_rows(Y0), t=30, s=32, y_out=out, dyn_t=1)
+        assert g.stats()["threshold_layer"] == st["threshold_layer"]
+        assert np.array_equal(g.categories(), cats)
+
+
+def test_dynamic_t_non_converging_net_goes_uncompressed():
+    """A random-init medium net (config 5) never converges: the probe rows stay distinct, so dyn_t takes
+    the uncompressed path (t = L), bit-exact with the oracle."""
+    net = sdgc.gen_medium_network(256, 18)
+    Y0 = sdgc.gen_medium_inputs(256, 3000)
+    plain = oracle.layers_f32(net, Y0)
+    with SnicitNetwork.from_network(net) as g:
+        g.set_stream(torch.cuda.current_stream())
+        Y, cats, st = _infer(g, Y0, sdgc.medium_t(18), s=128, n_segments=0, dyn_t=1)
+    assert st["threshold_layer"] == 18
+    assert np.array_equal(Y, plain) and np.array_equal(cats, oracle.categories(plain))
