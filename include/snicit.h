@@ -112,10 +112,10 @@ typedef struct {
                                entries are propagated"), chosen per row and layer from its non-zero count;
                                0 = always the dense-row form.  Results identical. */
     int32_t dyn_t;          /* 1 = dynamic threshold layer (the paper's future work): the first s
-                               rows of the batch are run layer by layer on the side and t is the first layer
-                               after which all of them that are live are identical (one centroid, no
-                               residue among them), at most threshold_layer; if that never happens and more
-                               than half of them are still distinct, the uncompressed path (t = L) is taken.
+                               rows of the batch are run through the layers on the side; with l* the first
+                               layer after which all of them that are live are identical (one centroid, no
+                               residue among them), t = min(2 l*, threshold_layer); if that never happens and
+                               more than half of them are still distinct, the uncompressed path (t = L).
                                stats.threshold_layer reports the t used.  0 = t as given.  Results are the
                                plain result for any t (within the tolerance of SNICIT's Eq. 5 rounding). */
 } snicit_options;

@@ -291,6 +291,75 @@ __global__ void __launch_bounds__(kCentThreads) centroid_traj_kernel(PostArgs a)
     unstage_row(a.cbuf + (size_t)c * N, cur, N);
 }
 
+// Dynamic-t probe (snicit_api.cu choose_t): probe row b (one CTA each) through layers 0..tmax-1 in
+// shared memory with the same layer arithmetic (Eq. 1); after every layer the row's live flag and a 64-bit
+// hash of its values (+0 for -0, == semantics) go to out[l][b] (hash, live in bit 0 of a second word).
+__global__ void __launch_bounds__(kCentThreads) probe_traj_kernel(PostArgs a, const float* __restrict__ rows, int tmax,
+                                                                  unsigned long long* __restrict__ out) {
+    extern __shared__ __align__(128) float sm[];
+    __shared__ unsigned long long s_h;
+    __shared__ int s_live;
+    const int b = blockIdx.x;
+    const int N = a.N;
+    const int h = post_halo(N);
+    const int dup = h == N;
+    float* cur = sm;
+    float* nxt = sm + N + h;
+    stage_row(cur, rows + (size_t)b * N, N);
+    __syncthreads();
+    fill_halo(cur, N, h);
+    PL Ld = load_pl(a.layers);
+    for (int l = 0; l < tmax; ++l) {
+        if (threadIdx.x == 0) {
+            s_h = 0ull;
+            s_live = 0;
+        }
+        __syncthreads();  // halo filled, slots reset
+        const PL Lnext = load_pl(a.layers + min(l + 1, a.L - 1));
+        float dmn = 0.0f, dmx = 0.0f;
+        post_row_layer<MODE_CENTROID, 5, 4, 8>(Ld, N, dup, a.ymax, 0.0f, cur, nxt, nullptr, nullptr, a.force_ell, dmn,
+                                               dmx);
+        __syncthreads();
+        unsigned long long hh = 0ull;
+        int live = 0;
+        for (int k = threadIdx.x; k < N; k += blockDim.x) {
+            const float v = nxt[k];
+            live |= v != 0.0f;
+            const unsigned long long u = __float_as_uint(v + 0.0f);
+            hh += (u ^ (u << 29) ^ 0x9E3779B97F4A7C15ull) * (2ull * (unsigned long long)k + 0xD1B54A32D192ED03ull);
+        }
+        hh = __reduce_add_sync(0xffffffffu, (unsigned)hh) | ((unsigned long long)__reduce_add_sync(0xffffffffu,
+                                                                                                  (unsigned)(hh >> 32))
+                                                             << 32);
+        live = __any_sync(0xffffffffu, live);
+        if ((threadIdx.x & 31) == 0) {
+            atomicAdd(&s_h, hh);
+            if (live) s_live = 1;
+        }
+        fill_halo(nxt, N, h);
+        __syncthreads();
+        if (threadIdx.x == 0) {
+            out[2 * ((size_t)l * gridDim.x + b)] = s_h;
+            out[2 * ((size_t)l * gridDim.x + b) + 1] = (unsigned long long)s_live;
+        }
+        float* tmp = cur;
+        cur = nxt;
+        nxt = tmp;
+        Ld = Lnext;
+    }
+}
+cudaError_t launch_probe_traj(const PostArgs& a, const float* rows, int S, int tmax, unsigned long long* out,
+                              cudaStream_t st) {
+    if (S <= 0 || tmax <= 0) return cudaSuccess;
+    if (a.N > post_fused_max_n()) return cudaErrorInvalidValue;
+    const size_t smem = sizeof(float) * 2 * (size_t)(a.N + post_halo(a.N));
+    int per_sm = 1;
+    cudaError_t e = blocks_per_sm((const void*)probe_traj_kernel, kCentThreads, smem, &per_sm);
+    if (e != cudaSuccess) return e;
+    probe_traj_kernel<<<S, kCentThreads, smem, st>>>(a, rows, tmax, out);
+    return cudaGetLastError();
+}
+
 // ---- sparse-entry residue form (north_star: "only the nonzero residual entries are propagated";
 // Eq. 5 / load-reduced SpMM P:860-889).  For a circulant layer, output j reads inputs (j + n nu) mod N,
 // so input k feeds outputs (k - n nu) mod N, n = 0..31.  An output none of whose inputs is non-zero

@@ -129,6 +129,7 @@ struct snicit_network {
     DevBuf<int> rnnz;         // [rows] non-zeros of each residue row at t
     DevBuf<float> probe0, probe1;  // dynamic t: the probe rows (ping-pong)
     DevBuf<int> pstat;             // dynamic t: per probe layer (live, identical, distinct)
+    DevBuf<unsigned long long> phash;  // dynamic t: per probe layer and row (hash, live)
     int probe_layers = 0;
     DevBuf<uint8_t> rconst;   // rows constant at t (R26): flag + value, set by the pre phase
     DevBuf<float> rval;
@@ -361,6 +362,7 @@ void snicit_free_network(snicit_network* net) {
     net->probe0.release();
     net->probe1.release();
     net->pstat.release();
+    net->phash.release();
     delete net;
 }
 
@@ -831,11 +833,15 @@ static cudaError_t stream_upload(snicit_network* net, void* dst, const void* src
 
 // Dynamic threshold layer ("determine t dynamically" is the paper's future work,
 // P:1619-1621).  Any t gives the plain result, so t only decides the cost.  The first
-// S = min(s, R) rows of the batch -- the rows Alg. 1 samples -- are run layer by layer on the
-// side; t is the first layer after which every live probe row is identical (the clustering then finds
-// one centroid and no residue among them), at most tmax.  If that never happens and more than S/2 of the
-// probe rows are still distinct at tmax, clustering cannot compress the batch and the
-// uncompressed path is taken (t = L).  Statistics are read back every 4 layers.
+// S = min(s, R) rows of the batch -- the rows Alg. 1 samples -- are run through the layers on
+// the side; l* is the first layer after which every live probe row is identical (the clustering would find
+// one centroid and no residue among them).  The rest of the batch converges later than its first rows
+// do on average, and a late t is cheap (rows that became constant cost a scalar per layer, R26) while an
+// early t leaves residue rows for hundreds of layers, so t = min(2 l*, tmax) (measured on C1/C2/C3:
+// profiles/r02_dyn_t.md).  If the probe rows never become identical and more than S/2 of them are still
+// distinct at tmax, clustering cannot compress the batch: the uncompressed path (t = L).
+// Rows of N <= 24576: one kernel carries each probe row through all tmax layers and records per-layer
+// hashes (one launch, one read-back); larger rows: per-layer launches, statistics read every 4 layers.
 static cudaError_t choose_t(snicit_network* net, const float* src, const uint32_t* bits, float one, int R, int s,
                             int tmax, int* t_out) {
     const int N = net->N, L = net->L;
@@ -852,6 +858,49 @@ static cudaError_t choose_t(snicit_network* net, const float* src, const uint32_
         e = launch_unpack_bits(bits, S, N, one, net->probe0.p, net->num_sms, st);
     if (e != cudaSuccess) return e;
     if ((e = launch_iota(net->iota_s.p, S, net->counters.p + CNT_PROBE, st)) != cudaSuccess) return e;
+    if (N <= post_fused_max_n()) {  // one launch: probe rows through all tmax layers, per-layer hashes
+        if ((e = net->phash.ensure((size_t)2 * tmax * S)) != cudaSuccess) return e;
+        PostArgs pa{};
+        pa.N = N;
+        pa.L = L;
+        pa.t = 0;
+        pa.ymax = net->ymax;
+        pa.layers = net->post_layers_d.p;
+        if ((e = launch_probe_traj(pa, net->probe0.p, S, tmax, net->phash.p, st)) != cudaSuccess) return e;
+        std::vector<unsigned long long> hv((size_t)2 * tmax * S);
+        if ((e = cudaMemcpyAsync(hv.data(), net->phash.p, sizeof(unsigned long long) * hv.size(),
+                                 cudaMemcpyDeviceToHost, st)) != cudaSuccess)
+            return e;
+        if ((e = cudaStreamSynchronize(st)) != cudaSuccess) return e;
+        net->probe_layers = 1;
+        int lstar = -1;
+        for (int l = 0; l < tmax && lstar < 0; ++l) {
+            bool have = false, ident = true;
+            unsigned long long h0 = 0;
+            for (int b = 0; b < S; ++b) {
+                const unsigned long long hb = hv[2 * ((size_t)l * S + b)], live = hv[2 * ((size_t)l * S + b) + 1];
+                if (!live) continue;
+                if (!have) {
+                    have = true;
+                    h0 = hb;
+                } else if (hb != h0) {
+                    ident = false;
+                }
+            }
+            if (!have || ident) lstar = l + 1;
+        }
+        if (lstar > 0) {
+            *t_out = std::min(2 * lstar, tmax);
+        } else {  // distinct live probe rows after layer tmax
+            std::vector<unsigned long long> hs;
+            for (int b = 0; b < S; ++b)
+                if (hv[2 * ((size_t)(tmax - 1) * S + b) + 1]) hs.push_back(hv[2 * ((size_t)(tmax - 1) * S + b)]);
+            std::sort(hs.begin(), hs.end());
+            const int uniq = (int)(std::unique(hs.begin(), hs.end()) - hs.begin());
+            *t_out = 2 * uniq > S ? L : tmax;
+        }
+        return cudaSuccess;
+    }
     std::vector<int> h((size_t)3 * (tmax + 1));
     float* pin = net->probe0.p;
     float* pout = net->probe1.p;
@@ -874,7 +923,7 @@ static cudaError_t choose_t(snicit_network* net, const float* src, const uint32_
                 return e;
             if ((e = cudaStreamSynchronize(st)) != cudaSuccess) return e;
             for (int k = done + 1; k <= l + 1 && chosen < 0; ++k)
-                if (h[3 * k] == 0 || h[3 * k + 1]) chosen = k;
+                if (h[3 * k] == 0 || h[3 * k + 1]) chosen = std::min(2 * k, tmax);
             done = l + 1;
         }
     }

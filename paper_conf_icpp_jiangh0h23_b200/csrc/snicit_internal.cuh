@@ -247,6 +247,9 @@ cudaError_t launch_centroid_traj(const PostArgs& a, int C_max, cudaStream_t st);
 bool centroid_cluster_ok(int N, const int* nu, const int* cls, int t, int L);
 cudaError_t launch_centroid_cluster(const PostArgs& a, int C_max, int win_max, cudaStream_t st);
 cudaError_t launch_residual_traj(const PostArgs& a, int max_rows, int num_sms, cudaStream_t st);
+// dynamic t: S probe rows through layers 0..tmax-1 (one CTA each); out[l][b] = (hash, live) after layer l
+cudaError_t launch_probe_traj(const PostArgs& a, const float* rows, int S, int tmax, unsigned long long* out,
+                              cudaStream_t st);
 // constant centroid rows through layers t..L-1 that are all circulant with uniform weights and bias:
 // one scalar chain per layer (exact, see kernels_post.cu); cout[c] = row at L, a.a_all filled if set,
 // cdone[c] = 1 and ++*ndone for constant rows, cdone[c] = 0 otherwise

@@ -304,7 +304,7 @@ def test_dynamic_threshold_layer():
     with SnicitNetwork.from_network(net) as g:
         g.set_stream(torch.cuda.current_stream())
         Y, cats, st = _infer(g, Y0, 30, dyn_t=1)
-        assert st["threshold_layer"] == (want if want is not None else 30)
+        assert st["threshold_layer"] == (min(2 * want, 30) if want is not None else 30)
         assert np.array_equal(cats, oracle.categories(plain))
         np.testing.assert_allclose(Y, plain, atol=ATOL, rtol=RTOL)
         # packed input and host input choose the same t
