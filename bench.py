@@ -76,6 +76,8 @@ def parse(argv=None):
     p.add_argument("--no-variants", action="store_true", help="skip the pre_fused = 2 / 0 roofline variants")
     p.add_argument("--cpu-seconds", type=float, default=15.0, help="target CPU work of the oracle sample")
     p.add_argument("--quick", action="store_true", help="value only (no e2e/uncompressed/variants/studies)")
+    p.add_argument("--dyn-log", default=os.path.join(ROOT, "gpurun_out", "bench_dynamics_{config}_rank{rank}.jsonl"),
+                   help="per-layer dynamics JSONL of one inference per rank (SURVEY 5); '' = off")
     a = p.parse_args(argv)
     if a.quick:
         a.no_e2e = a.no_cpu_baseline = a.no_uncompressed = a.no_residue = a.no_general = a.no_variants = True
@@ -516,6 +518,11 @@ def run_snicit(args):
     g.infer(y0, t=t, s=s, options=default_options(kernel=kern, n_segments=snic["n"], pre_fused=args.pre_fused,
                                                   timing=1), y_out=y_out, row_offset=row0)
     st1 = g.stats()
+    dyn_path = None
+    if args.dyn_log:
+        dyn_path = args.dyn_log.format(config=args.config, rank=rank)
+        os.makedirs(os.path.dirname(dyn_path) or ".", exist_ok=True)
+        g.write_dynamics_jsonl(dyn_path, {"config": args.config, "rank": rank, "row_offset": row0})
     mine = {"rank": rank, "rows": B_local, "row_offset": row0,
             **{k: st1[k] for k in ("t_pre_ms", "t_convert_ms", "t_post_ms", "t_recover_ms", "t_total_ms",
                                    "live_at_t", "n_centroids", "residual_at_t", "n_categories")}}
@@ -736,7 +743,7 @@ def run_snicit(args):
             "categories": n_cat_global,
             "dynamics": {k: st0[k] for k in ("live_at_t", "n_centroids", "n_sampled", "residual_at_t",
                                              "residual_final", "n_categories")},
-            "residue": residue, "general_csc": general,
+            "residue": residue, "general_csc": general, "dynamics_log": dyn_path,
             "paper_context": "SNICIT 16384-1920 on 1x RTX A6000, B=60000: 179.37 ms = 3.37e14 edges/s "
                              "(Table 3, P:1383)",
         }

@@ -257,6 +257,18 @@ snicit_status snicit_stats(snicit_network* net, snicit_stats_t* out);
 snicit_status snicit_layer_profile(snicit_network* net, int32_t max, double* ms, int64_t* rows, double* bytes,
                                    int32_t* n);
 
+/* Per-layer dynamics of the last infer run with options.timing >= 1 (metrics / logging), for
+ * layers l < *n = min(max, L) (host pointers, any may be NULL; -1 = not recorded for that layer):
+ *  pre_full[l]   (l < t) rows evaluated in full by pre-convergence layer l (the others alive are carried as
+ *                constant rows, R26);
+ *  pre_live[l]   (l < t) rows alive after layer l (not dropped as dead, R23);
+ *  res_alive[l]  (l >= t) non-empty residue rows after post-convergence layer l (ne_idx);
+ *  res_scalar[l] (l >= t) residue rows carried by a scalar from post layer l or earlier.
+ * Recorded by the row-resident pre phase and the fused post mode; the per-layer pre path reports pre_full
+ * / pre_live from its per-layer active counts when options.timing == 2.  Synchronises the stream. */
+snicit_status snicit_dynamics(snicit_network* net, int32_t max, int64_t* pre_full, int64_t* pre_live,
+                              int64_t* res_alive, int64_t* res_scalar, int32_t* n);
+
 /* ---- test hooks (used by tests/ for step-level parity; not needed by applications) ---- */
 
 /* Clustering state of the last infer (t < L): centroid row ids (ascending, <= s entries),

@@ -24,7 +24,7 @@ EXPORTED = ["snicit_default_options", "snicit_load_network", "snicit_set_stream"
             "snicit_categories", "snicit_stats", "snicit_debug_clustering", "snicit_debug_layer",
             "snicit_layer_is_circulant", "snicit_free_network", "snicit_last_error", "snicit_abi_version",
             "snicit_layer_profile", "snicit_load_network_circulant", "snicit_infer_packed",
-            "snicit_categories_device"]
+            "snicit_categories_device", "snicit_dynamics"]
 
 
 class Options(ctypes.Structure):
@@ -90,6 +90,8 @@ def load_library(path: str = LIB_PATH):
     L.snicit_categories_device.restype = i32
     L.snicit_stats.argtypes = [P, ctypes.POINTER(Stats)]
     L.snicit_stats.restype = i32
+    L.snicit_dynamics.argtypes = [P, i32, P, P, P, P, P]
+    L.snicit_dynamics.restype = i32
     L.snicit_layer_profile.argtypes = [P, i32, P, P, P, P]
     L.snicit_layer_profile.restype = i32
     L.snicit_debug_clustering.argtypes = [P, P, P, P, P, P, P, P]

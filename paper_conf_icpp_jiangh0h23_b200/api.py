@@ -242,6 +242,40 @@ class SnicitNetwork:
         k = n.value
         return dict(ms=ms[:k].copy(), rows=rows[:k].copy(), bytes=by[:k].copy())
 
+    def dynamics(self) -> dict:
+        """Per-layer dynamics of the last infer run with options.timing >= 1 (snicit_dynamics): arrays over
+        layers 0..L-1, -1 where not recorded."""
+        L = self.L
+        arrs = {k: np.full(L, -1, np.int64) for k in ("pre_full", "pre_live", "res_alive", "res_scalar")}
+        n = ctypes.c_int32(0)
+        check(self._lib.snicit_dynamics(self._h, L, arrs["pre_full"].ctypes.data, arrs["pre_live"].ctypes.data,
+                                        arrs["res_alive"].ctypes.data, arrs["res_scalar"].ctypes.data,
+                                        ctypes.byref(n)), "snicit_dynamics")
+        return arrs
+
+    def write_dynamics_jsonl(self, path: str, extra: Optional[dict] = None) -> int:
+        """One JSON object per layer (SURVEY 5 per-layer log): layer, phase, live / full / residue counts,
+        plus the run's clustering stats on the first line.  Returns the number of lines written."""
+        import json
+        d = self.dynamics()
+        st = self.stats()
+        t = int(st["threshold_layer"])
+        with open(path, "w") as f:
+            head = {"run": {k: st[k] for k in ("batch", "threshold_layer", "live_at_t", "n_centroids", "n_sampled",
+                                               "residual_at_t", "residual_final", "res_nnz_at_t", "n_categories")}}
+            if extra:
+                head["run"].update(extra)
+            f.write(json.dumps(head) + "\n")
+            for l in range(self.L):
+                rec = {"layer": l, "phase": "pre" if l < t else "post"}
+                if l < t:
+                    rec.update(pre_full=int(d["pre_full"][l]), pre_live=int(d["pre_live"][l]))
+                else:
+                    rec.update(centroids=int(st["n_centroids"]), res_alive=int(d["res_alive"][l]),
+                               res_scalar=int(d["res_scalar"][l]))
+                f.write(json.dumps(rec) + "\n")
+        return self.L + 1
+
     def debug_clustering(self, n_segments: Optional[int] = None, s: Optional[int] = None) -> dict:
         """Clustering state of the last infer.  The buffers are sized from that infer's n and s (the
         arguments are accepted for compatibility and must match them if given)."""

@@ -510,6 +510,7 @@ __global__ void __launch_bounds__(kPostThreads, 2) residual_traj_kernel(PostArgs
         __syncthreads();
         bool alive = true, cst = false;
         float vr = 0.0f;
+        int sc_from = a.L;  // first layer carried by a scalar
         const int cfrom = a.cfrom ? a.cfrom[slot] : a.L - a.t;
         // sparse form: nnz of `cur` and whether lsts[li] lists all of its non-zeros; nxt_zero: `nxt` is
         // all-zero in [0, N) (left so by the previous sparse layer)
@@ -625,6 +626,7 @@ __global__ void __launch_bounds__(kPostThreads, 2) residual_traj_kernel(PostArgs
                 __syncthreads();
             }
             const int l0 = l;
+            sc_from = l;
             for (; l < a.L; ++l) {
                 float w0, b0, acv;
                 if (fits) {
@@ -661,6 +663,11 @@ __global__ void __launch_bounds__(kPostThreads, 2) residual_traj_kernel(PostArgs
         if (threadIdx.x == 0) {
             a.ne_row[row] = alive ? 1 : 0;
             if (alive && a.alive_count) atomicAdd(a.alive_count, 1);
+            if (a.dyn) {  // post layers this residue row stayed non-empty through; scalar start
+                const int nl = a.L - a.t;
+                atomicAdd(a.dyn + (alive ? nl : l - a.t), 1ull);
+                atomicAdd(a.dyn + (nl + 1) + (cst ? sc_from - a.t : nl), 1ull);
+            }
         }
         __syncthreads();  // s_p and the row buffers are reused
     }

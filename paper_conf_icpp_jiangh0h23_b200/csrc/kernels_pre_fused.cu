@@ -307,6 +307,7 @@ __global__ void __launch_bounds__(T, PfCfg<T>::kMinBlocks) pre_fused_kernel(cons
         bool cst = false, dead = false;
         float v = 0.0f;
         int full = 0;
+        int lend = a.t;  // the layer that zeroed the row (dead, R23), or t: alive after layer l <=> lend > l
         for (int l = 0; l < a.t; ++l) {
             // WUNI: one weight for every layer, read at a constant offset -> a uniform register operand
             const float w0 = WUNI ? p.L[0].w0 : p.L[l].w0, b0 = p.L[l].b0;
@@ -352,6 +353,7 @@ __global__ void __launch_bounds__(T, PfCfg<T>::kMinBlocks) pre_fused_kernel(cons
                     if (a.const_skip) cst = true;
                     if (v == 0.0f && a.drop && dead_next) {
                         dead = true;
+                        lend = l;
                         break;
                     }
                 }
@@ -368,6 +370,7 @@ __global__ void __launch_bounds__(T, PfCfg<T>::kMinBlocks) pre_fused_kernel(cons
                 }
                 if (v == 0.0f && a.drop && dead_next) {
                     dead = true;
+                    lend = l;
                     break;
                 }
             }
@@ -403,6 +406,10 @@ __global__ void __launch_bounds__(T, PfCfg<T>::kMinBlocks) pre_fused_kernel(cons
         if (tid == 0) {
             if (a.full_rl) atomicAdd(a.full_rl, (unsigned long long)full);
             if (a.n_const && cst) atomicAdd(a.n_const, 1);
+            if (a.dyn) {  // per-layer dynamics: histograms of the full-evaluation count and of the end layer
+                atomicAdd(a.dyn + full, 1ull);
+                atomicAdd(a.dyn + (a.t + 1) + lend, 1ull);
+            }
         }
         if (NB == 2 && tid == 0) {
             s_pos[2 + (k & 1)] = np;

@@ -130,6 +130,8 @@ struct snicit_network {
     DevBuf<float> probe0, probe1;  // dynamic t: the probe rows (ping-pong)
     DevBuf<int> pstat;             // dynamic t: per probe layer (live, identical, distinct)
     DevBuf<unsigned long long> phash;  // dynamic t: per probe layer and row (hash, live)
+    DevBuf<unsigned long long> dynbuf; // per-layer dynamics histograms (options.timing): pre [2][t + 1], post [2][L - t + 1]
+    bool dyn_pre = false, dyn_post = false;
     int probe_layers = 0;
     DevBuf<uint8_t> rconst;   // rows constant at t (R26): flag + value, set by the pre phase
     DevBuf<float> rval;
@@ -363,6 +365,7 @@ void snicit_free_network(snicit_network* net) {
     net->probe1.release();
     net->pstat.release();
     net->phash.release();
+    net->dynbuf.release();
     delete net;
 }
 
@@ -985,6 +988,7 @@ static snicit_status infer_core(snicit_network* net, const float* y0, int64_t ba
     int circ_layers = 0;
     net->have_result = false;
     net->ev_map = net->ev_res = false;
+    net->dyn_pre = net->dyn_post = false;
     snicit_stats_t stats{};
     stats.batch = batch;
     stats.threshold_layer = tt;
@@ -1096,6 +1100,12 @@ static snicit_status infer_core(snicit_network* net, const float* y0, int64_t ba
         pa.rconst = net->rconst.p;
         pa.rval = net->rval.p;
         pa.n_const = cnt + CNT_PFCONST;
+        if (opt.timing) {
+            CUDA_TRY(net->dynbuf.ensure((size_t)2 * (tt + 1) + 2 * (L + 1)));
+            CUDA_TRY(cudaMemsetAsync(net->dynbuf.p, 0, sizeof(unsigned long long) * 2 * (tt + 1), st));
+            pa.dyn = net->dynbuf.p;
+            net->dyn_pre = true;
+        }
         if (pf_cluster)
             CUDA_TRY(launch_pre_cluster(pa, net->pf_layers_h.data(), net->num_sms, st));
         else
@@ -1329,6 +1339,13 @@ static snicit_status infer_core(snicit_network* net, const float* y0, int64_t ba
             pa.ctr64 = net->ctr64.p;
             pa.res_sparse = opt.res_sparse;
             pa.rnnz = net->rnnz.p;
+            if (opt.timing) {
+                CUDA_TRY(net->dynbuf.ensure((size_t)2 * (tt + 1) + 2 * (L + 1)));
+                unsigned long long* d = net->dynbuf.p + 2 * (tt + 1);
+                CUDA_TRY(cudaMemsetAsync(d, 0, sizeof(unsigned long long) * 2 * (L - tt + 1), st));
+                pa.dyn = d;
+                net->dyn_post = true;
+            }
             CUDA_TRY(cudaMemsetAsync(cnt + CNT_WORK, 0, 2 * sizeof(int), st));
             pa.force_ell = opt.kernel == SNICIT_KERNEL_ELL ? 1 : 0;
             // cluster (DSMEM) trajectory when every post layer is circulant and partition-compatible
@@ -1668,6 +1685,55 @@ snicit_status snicit_layer_profile(snicit_network* net, int32_t max, double* ms,
                 wb = (double)pl.K * net->N * ((net->idx16 ? 2.0 : 4.0) + (pl.uniform ? 0.0 : 4.0));
             bytes[l] = 8.0 * (double)h[l] * net->N + wb + 4.0 * net->N;
         }
+    }
+    if (n) *n = cnt;
+    return SNICIT_OK;
+}
+
+snicit_status snicit_dynamics(snicit_network* net, int32_t max, int64_t* pre_full, int64_t* pre_live,
+                              int64_t* res_alive, int64_t* res_scalar, int32_t* n) {
+    if (!net) return fail(SNICIT_E_INVALID_ARG, "net NULL");
+    if (!net->have_result) return fail(SNICIT_E_STATE, "no inference result");
+    DeviceGuard dg(net->device);
+    CUDA_TRY(dg.status);
+    const int L = net->L, t = net->last_t;
+    const int cnt = std::min<int>(std::max(max, 0), L);
+    std::vector<unsigned long long> h(net->dynbuf.n ? net->dynbuf.n : 1, 0ull);
+    if (net->dyn_pre || net->dyn_post) {
+        CUDA_TRY(cudaMemcpyAsync(h.data(), net->dynbuf.p, sizeof(unsigned long long) * net->dynbuf.n,
+                                 cudaMemcpyDeviceToHost, net->stream));
+        CUDA_TRY(cudaStreamSynchronize(net->stream));
+    }
+    std::vector<int> hist;
+    if (!net->last_pre_fused && net->prof_layers > 0) {  // per-layer pre path with timing == 2: active rows
+        hist.resize((size_t)net->prof_layers);
+        CUDA_TRY(cudaMemcpy(hist.data(), net->hist.p, sizeof(int) * hist.size(), cudaMemcpyDeviceToHost));
+    }
+    const unsigned long long* F = h.data();               // rows by full-evaluation count [t + 1]
+    const unsigned long long* E = h.data() + (t + 1);     // rows by end layer [t + 1]
+    const int nl = L - t;
+    const unsigned long long* A = h.data() + 2 * (t + 1);          // residue rows by layers survived [nl + 1]
+    const unsigned long long* Sc = A + (nl + 1);                    // residue rows by scalar start [nl + 1]
+    for (int l = 0; l < cnt; ++l) {
+        int64_t pf = -1, pl = -1, ra = -1, rs = -1;
+        if (l < t && net->dyn_pre) {
+            pf = pl = 0;
+            for (int f = l + 1; f <= t; ++f) pf += (int64_t)F[f];
+            for (int e = l + 1; e <= t; ++e) pl += (int64_t)E[e];
+        } else if (l < t && l < (int)hist.size()) {
+            pf = hist[l];
+            if (l + 1 < (int)hist.size()) pl = hist[l + 1];
+        }
+        if (l >= t && net->dyn_post) {
+            const int k = l - t;
+            ra = rs = 0;
+            for (int e = k + 1; e <= nl; ++e) ra += (int64_t)A[e];
+            for (int c = 0; c <= k; ++c) rs += (int64_t)Sc[c];
+        }
+        if (pre_full) pre_full[l] = pf;
+        if (pre_live) pre_live[l] = pl;
+        if (res_alive) res_alive[l] = ra;
+        if (res_scalar) res_scalar[l] = rs;
     }
     if (n) *n = cnt;
     return SNICIT_OK;

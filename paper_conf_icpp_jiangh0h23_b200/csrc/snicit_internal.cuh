@@ -235,6 +235,8 @@ struct PostArgs {
                          //   over constant centroids are carried by a scalar (residual_traj_kernel)
     int res_sparse;      // 1: sparse-entry residue form for residue rows with few non-zeros (circulant layers)
     const int* rnnz;     // nullable: non-zeros of each row's residue at t (map_residual), by row id
+    unsigned long long* dyn;  // nullable: [L - t + 1] residue rows by post layers survived, [L - t + 1] by the
+                              //   post layer from which they were carried by a scalar (L - t: never)
     unsigned long long* ctr64;  // nullable: work counters (Ctr64)
 };
 // 64-bit work counters of one infer (stats): residue entries at t, residue row-layers by form, outputs
@@ -289,6 +291,7 @@ struct PreFusedArgs {
     uint8_t* rconst;              // nullable: rconst[row] = 1, rval[row] = v for rows constant at t (R26)
     float* rval;
     unsigned long long* full_rl;  // nullable: += full (non-constant) row-layer evaluations
+    unsigned long long* dyn;      // nullable: [t + 1] rows by full-evaluation count, [t + 1] rows by end layer
     int* n_const;                 // nullable: += rows that became constant
 };
 // 0 if N is not supported (T = N/32 threads must be 32..512)

@@ -326,3 +326,37 @@ def test_dynamic_t_non_converging_net_goes_uncompressed():
         Y, cats, st = _infer(g, Y0, sdgc.medium_t(18), s=128, n_segments=0, dyn_t=1)
     assert st["threshold_layer"] == 18
     assert np.array_equal(Y, plain) and np.array_equal(cats, oracle.categories(plain))
+
+
+# ------------------------------------------------------------------------------ per-layer dynamics log
+
+def test_dynamics_log(tmp_path):
+    """snicit_dynamics (SURVEY 5 per-layer log): pre_live[l] = rows with a non-zero output after layer l,
+    pre_full[l] = rows not yet constant before layer l (both counted on the oracle's layer-by-layer rows);
+    res_alive ends at stats.residual_final and never increases (zero residues are absorbing, R16)."""
+    N, L, B, t = 1024, 40, 600, 6
+    net = sdgc.gen_network(N, L, "radix")
+    Y0 = sdgc.gen_inputs(N, B)
+    with SnicitNetwork.from_network(net) as g:
+        g.set_stream(torch.cuda.current_stream())
+        _infer(g, Y0, t, timing=1)
+        d = g.dynamics()
+        st = g.stats()
+        nlines = g.write_dynamics_jsonl(str(tmp_path / "dyn.jsonl"))
+    y = Y0.copy()
+    const_before = np.zeros(B, bool)  # row constant after the previous layer (carried by a scalar from then on)
+    alive = np.ones(B, bool)
+    for l in range(t):
+        full = alive & ~const_before
+        assert d["pre_full"][l] == int(full.sum()), l
+        y = oracle.layers_f32(net, y, l, l + 1)
+        nz = (y != 0).any(1)
+        alive = alive & nz
+        assert d["pre_live"][l] == int(alive.sum()), l
+        const_before = const_before | (alive & (y == y[:, :1]).all(1))
+    ra = d["res_alive"][t:]
+    assert ra[-1] == st["residual_final"] and np.all(np.diff(ra) <= 0) and ra[0] <= st["residual_at_t"]
+    assert np.all(d["pre_full"][t:] == -1) and np.all(d["res_alive"][:t] == -1)
+    lines = open(tmp_path / "dyn.jsonl").read().splitlines()
+    assert nlines == len(lines) == L + 1
+    assert json.loads(lines[1])["phase"] == "pre" and json.loads(lines[-1])["phase"] == "post"
