@@ -45,4 +45,46 @@ with SnicitNetwork.from_network(net) as g:
     cats = g.categories()
     torch.cuda.synchronize()
 print("packed streamed 4096 12 5000 4 categories", len(cats), "sum", float(out.sum()))
+# round 2: cluster-split row-resident kernel (pre_fused = 4), two-pass Alg. 2, sparse-entry residues,
+# interleaved ELL tiles in constant-row mode, dynamic t probe, device category export
+for N, L, B, t, kw in ((16384, 7, 9, 7, dict(pre_fused=4)), (65536, 5, 3, 5, dict(pre_fused=4))):
+    net = sdgc.gen_network(N, L, "radix")
+    Y0 = torch.from_numpy(sdgc.gen_inputs(N, B)).cuda()
+    out = torch.empty_like(Y0)
+    with SnicitNetwork.from_network(net) as g:
+        g.set_stream(torch.cuda.current_stream())
+        g.infer(Y0, t=t, s=32, y_out=out, **kw)
+        cats = g.categories()
+        torch.cuda.synchronize()
+    print("cluster", N, L, B, t, "categories", len(cats), "sum", float(out.sum()))
+for mode, N, L, B, t, kw in (("radix", 4096, 16, 200, 10, dict(timing=1)), ("perm", 1024, 12, 200, 12, {}),
+                             ("random", 1024, 10, 150, 4, {}), ("radix", 1024, 40, 400, 30, dict(dyn_t=1))):
+    net = sdgc.gen_network(N, L, mode)
+    Y0 = torch.from_numpy(sdgc.gen_inputs(N, B)).cuda()
+    out = torch.empty_like(Y0)
+    with SnicitNetwork.from_network(net) as g:
+        g.set_stream(torch.cuda.current_stream())
+        g.infer(Y0, t=t, s=32, y_out=out, **kw)
+        cats = g.categories()
+        buf = torch.empty(1 + B, dtype=torch.int64, device="cuda")
+        g.categories_device(buf)
+        torch.cuda.synchronize()
+    print(mode, N, L, B, t, kw, "categories", len(cats), "sum", float(out.sum()))
+# sparse residues (near-duplicate rows, t = 0)
+N, L, B = 4096, 8, 120
+base = sdgc.gen_inputs(N, 8)
+Yh = base[np.arange(B) % 8].copy()
+rs = np.random.RandomState(0)
+for r in range(32, B):
+    k = rs.choice(N, 2, replace=False)
+    Yh[r, k] = 1.0 - Yh[r, k]
+net = sdgc.gen_network(N, L, "radix")
+Y0 = torch.from_numpy(Yh).cuda()
+out = torch.empty_like(Y0)
+with SnicitNetwork.from_network(net) as g:
+    g.set_stream(torch.cuda.current_stream())
+    g.infer(Y0, t=0, s=32, y_out=out)
+    st = g.stats()
+    torch.cuda.synchronize()
+print("sparse residues: sparse row-layers", st["res_sparse_rl"], "sum", float(out.sum()))
 print("sanitize run done")
