@@ -330,15 +330,13 @@ template <int TK>
 __global__ void __launch_bounds__(kMapThreads) map_dist_kernel(const float* __restrict__ y, int N, const int* rows,
                                                                const int* count, const int* cent, const int* n_cent,
                                                                int* __restrict__ dist, int s,
-                                                               const uint8_t* __restrict__ rconst,
-                                                               const float* __restrict__ rval,
-                                                               unsigned long long* map_rows) {
+                                                               const int* __restrict__ need,
+                                                               const int* __restrict__ need_count) {
     extern __shared__ float4 s_c4[];
-    __shared__ float s_cv[1024];  // constant value of centroid c (R26) or NaN
     constexpr int TK4 = TK / 4, CH = (TK4 + 31) / 32;  // float4 chunks per lane
-    const int n = *count;
+    const int n = *need_count;  // rows whose distances are needed (map_need_kernel)
     const int C = min(*n_cent, s);
-    if (C <= 0 || map_tile(C) != TK) return;  // the launcher starts every TK variant; one matches
+    if (C <= 0 || n <= 0 || map_tile(C) != TK) return;  // the launcher starts every TK variant; one matches
     const int Cp = (C + 31) / 32 * 32;
     const int ntiles = (N + TK - 1) / TK;
     if ((int)blockIdx.x >= ((int)gridDim.x / ntiles) * ntiles) return;  // grid remainder
@@ -350,26 +348,12 @@ __global__ void __launch_bounds__(kMapThreads) map_dist_kernel(const float* __re
         s_c4[i] = (c < C && k4 < kl4) ? __ldg(reinterpret_cast<const float4*>(y + (size_t)cent[c] * N + k0) + k4)
                                       : make_float4(0.f, 0.f, 0.f, 0.f);
     }
-    for (int c = threadIdx.x; c < C; c += blockDim.x)
-        s_cv[c] = (rconst && rconst[cent[c]]) ? rval[cent[c]] : __int_as_float(0x7fffffff);
     __syncthreads();
     const int lane = threadIdx.x & 31, warp = threadIdx.x >> 5;
     const int nwb = (gridDim.x / ntiles) * (kMapThreads / 32);  // warps over the rows
-    // rows that need distances (a constant row with an equal constant centroid does not)
-    auto needed = [&](int p_) {
-        const int r_ = rows[p_];
-        if (!(rconst && rconst[r_])) return true;
-        const float v = rval[r_];
-        for (int c = 0; c < C; ++c)
-            if (s_cv[c] == v) return false;
-        return true;
-    };
-    auto next_row = [&](int p_) {
-        while (p_ < n && !needed(p_)) p_ += nwb;
-        return p_;
-    };
-    auto load_tile = [&](int p_, float4* v) {
-        const float4* yr4 = reinterpret_cast<const float4*>(y + (size_t)rows[p_] * N + k0);
+    auto next_row = [&](int q_) { return q_; };
+    auto load_tile = [&](int q_, float4* v) {
+        const float4* yr4 = reinterpret_cast<const float4*>(y + (size_t)rows[need[q_]] * N + k0);
 #pragma unroll
         for (int i = 0; i < CH; ++i) {
             const int k4 = lane + 32 * i;
@@ -383,10 +367,9 @@ __global__ void __launch_bounds__(kMapThreads) map_dist_kernel(const float* __re
         float4 yv[CH];
 #pragma unroll
         for (int i = 0; i < CH; ++i) yv[i] = yn[i];
-        const int pcur = p;
+        const int pcur = need[p];  // list position of this row
         p = next_row(p + nwb);
         if (p < n) load_tile(p, yn);
-        if (map_rows && tile == 0 && lane == 0) atomicAdd(map_rows, 1ull);  // rows whose distances are computed
         for (int cg = 0; cg < Cp; cg += 32) {
             int cnt[32];
 #pragma unroll
@@ -417,6 +400,41 @@ __global__ void __launch_bounds__(kMapThreads) map_dist_kernel(const float* __re
             const int mine = cnt[0];
             if (cg + lane < C && mine) atomicAdd(dist + (size_t)pcur * s + cg + lane, mine);
         }
+    }
+}
+
+// Rows whose L0 distances Alg. 2 needs: all live rows except constant rows (R26) with an equal constant
+// centroid (their argmin is that centroid, map_finish).  Appends list positions (unordered) to need.
+__global__ void __launch_bounds__(kMapThreads) map_need_kernel(const int* rows, const int* count, const int* cent,
+                                                               const int* n_cent, int s, const uint8_t* rconst,
+                                                               const float* rval, int* need, int* need_count,
+                                                               unsigned long long* map_rows) {
+    __shared__ float s_cv[1024];  // constant value of centroid c or NaN
+    const int n = *count;
+    const int C = min(*n_cent, s);
+    for (int c = threadIdx.x; c < C; c += blockDim.x)
+        s_cv[c] = (rconst && rconst[cent[c]]) ? rval[cent[c]] : __int_as_float(0x7fffffff);
+    __syncthreads();
+    const int lane = threadIdx.x & 31;
+    for (int p0 = blockIdx.x * blockDim.x; p0 < n; p0 += gridDim.x * blockDim.x) {
+        const int p = p0 + threadIdx.x;
+        bool nd = false;
+        if (p < n && C > 0) {
+            nd = true;
+            const int r = rows[p];
+            if (rconst && rconst[r]) {
+                const float v = rval[r];
+                for (int c = 0; c < C && nd; ++c) nd = !(s_cv[c] == v);
+            }
+        }
+        const unsigned m = __ballot_sync(0xffffffffu, nd);
+        int base = 0;
+        if (lane == 0 && m) {
+            base = atomicAdd(need_count, __popc(m));
+            if (map_rows) atomicAdd(map_rows, (unsigned long long)__popc(m));
+        }
+        base = __shfl_sync(0xffffffffu, base, 0);
+        if (nd) need[base + __popc(m & ((1u << lane) - 1u))] = p;
     }
 }
 
@@ -510,10 +528,18 @@ cudaError_t launch_map_residual(const float* y, int N, const int* rows, const in
                                 const int* n_cent, int* M, int* cslot, uint8_t* ne_row, uint8_t* flag_pos,
                                 float* yhat, float* cbuf, int max_rows, int num_sms, cudaStream_t st,
                                 const uint8_t* rconst, const float* rval, unsigned long long* nnz_sum, int* dist,
-                                int s, int* rnnz) {
+                                int s, int* rnnz, int* need, int* need_count) {
     if (max_rows <= 0) return cudaSuccess;
     cudaError_t e = cudaMemsetAsync(dist, 0, sizeof(int) * (size_t)max_rows * s, st);
     if (e != cudaSuccess) return e;
+    if ((e = cudaMemsetAsync(need_count, 0, sizeof(int), st)) != cudaSuccess) return e;
+    {
+        int g = (max_rows + kMapThreads - 1) / kMapThreads;
+        if (g > num_sms * 4) g = num_sms * 4;
+        map_need_kernel<<<g, kMapThreads, 0, st>>>(rows, count, cent, n_cent, s, rconst, rval, need, need_count,
+                                                   nnz_sum ? nnz_sum + (C64_MAP_ROWS - C64_RES_NNZ) : nullptr);
+        if ((e = cudaGetLastError()) != cudaSuccess) return e;
+    }
     // pass 1: the tile width depends on the centroid count C <= s, known only on the device: every tile
     // variant up to the one of C = s is launched and all but the matching one exit at once
     if (s > 1024) return cudaErrorInvalidValue;  // the widest centroid tile (32 columns) must fit
@@ -532,15 +558,15 @@ cudaError_t launch_map_residual(const float* y, int N, const int* rows, const in
         return cudaGetLastError();
     };
     e = one((const void*)map_dist_kernel<512>, 512, [&](int g) {
-        map_dist_kernel<512><<<g, kMapThreads, smem, st>>>(y, N, rows, count, cent, n_cent, dist, s, rconst, rval, nnz_sum ? nnz_sum + (C64_MAP_ROWS - C64_RES_NNZ) : nullptr);
+        map_dist_kernel<512><<<g, kMapThreads, smem, st>>>(y, N, rows, count, cent, n_cent, dist, s, need, need_count);
     });
     if (e == cudaSuccess)
         e = one((const void*)map_dist_kernel<128>, 128, [&](int g) {
-            map_dist_kernel<128><<<g, kMapThreads, smem, st>>>(y, N, rows, count, cent, n_cent, dist, s, rconst, rval, nnz_sum ? nnz_sum + (C64_MAP_ROWS - C64_RES_NNZ) : nullptr);
+            map_dist_kernel<128><<<g, kMapThreads, smem, st>>>(y, N, rows, count, cent, n_cent, dist, s, need, need_count);
         });
     if (e == cudaSuccess)
         e = one((const void*)map_dist_kernel<32>, 32, [&](int g) {
-            map_dist_kernel<32><<<g, kMapThreads, smem, st>>>(y, N, rows, count, cent, n_cent, dist, s, rconst, rval, nnz_sum ? nnz_sum + (C64_MAP_ROWS - C64_RES_NNZ) : nullptr);
+            map_dist_kernel<32><<<g, kMapThreads, smem, st>>>(y, N, rows, count, cent, n_cent, dist, s, need, need_count);
         });
     if (e != cudaSuccess) return e;
     int grid = num_sms * 8;

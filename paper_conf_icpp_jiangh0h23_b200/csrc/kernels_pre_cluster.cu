@@ -412,6 +412,8 @@ __global__ void __launch_bounds__(kCT, kCfMinBlocks) pre_cluster_kernel(const __
         mbar_init(&bar[1], 1);
         fence_proxy_async_smem();
     }
+    // every CTA of the cluster has started (and initialised its shared memory) before any remote access
+    cluster_barrier();
     // the first row: rank 0 claims it for the cluster
     if (r == 0 && tid == 0) {
         const int p0 = atomicAdd(a.work, 1);

@@ -82,7 +82,7 @@ inline bool misaligned16(const void* p) { return p && (reinterpret_cast<uintptr_
 // device counters (one int each)
 enum Counter {
     CNT_LIVE0 = 0, CNT_LIVE1, CNT_LIVE2, CNT_ORD, CNT_RES0, CNT_RES1, CNT_NCENT, CNT_SEFF, CNT_ALL, CNT_NCAT,
-    CNT_WORK, CNT_ALIVE, CNT_CDONE, CNT_PFWORK, CNT_PFCONST, CNT_CCOUNT, CNT_PROBE, CNT_N
+    CNT_WORK, CNT_ALIVE, CNT_CDONE, CNT_PFWORK, CNT_PFCONST, CNT_CCOUNT, CNT_PROBE, CNT_NEED, CNT_N
 };
 
 }  // namespace
@@ -127,6 +127,7 @@ struct snicit_network {
     DevBuf<int> cfrom;        // per centroid: first post layer with a constant a_c row (residual_traj)
     DevBuf<int> dist;         // [rows][s] L0 distances of Alg. 2 (map_residual pass 1)
     DevBuf<int> rnnz;         // [rows] non-zeros of each residue row at t
+    DevBuf<int> need;         // [rows] list positions whose Alg. 2 distances are computed
     DevBuf<float> probe0, probe1;  // dynamic t: the probe rows (ping-pong)
     DevBuf<int> pstat;             // dynamic t: per probe layer (live, identical, distinct)
     DevBuf<unsigned long long> phash;  // dynamic t: per probe layer and row (hash, live)
@@ -361,6 +362,7 @@ void snicit_free_network(snicit_network* net) {
     net->ctr64.release();
     net->dist.release();
     net->rnnz.release();
+    net->need.release();
     net->probe0.release();
     net->probe1.release();
     net->pstat.release();
@@ -717,6 +719,7 @@ static cudaError_t ensure_workspace(snicit_network* net, int64_t R, int s, int n
     if ((e = net->F.ensure((size_t)std::max(n, 1) * ss)) != cudaSuccess) return e;
     if ((e = net->dist.ensure(rows * ss)) != cudaSuccess) return e;
     if ((e = net->rnnz.ensure(rows)) != cudaSuccess) return e;
+    if ((e = net->need.ensure(rows)) != cudaSuccess) return e;
     if ((e = net->cscratch.ensure((size_t)compact_scratch_ints((int)rows))) != cudaSuccess) return e;
     if (net->segflag.n < rows) {
         if ((e = net->segflag.ensure(rows)) != cudaSuccess) return e;
@@ -1243,7 +1246,7 @@ static snicit_status infer_core(snicit_network* net, const float* y0, int64_t ba
         CUDA_TRY(launch_map_residual(cur, N, list_cur, cnt_cur, net->cent.p, cnt + CNT_NCENT, net->M.p, net->cslot.p,
                                      net->ne_row.p, net->flag_pos.p, yhat, net->cbuf0.p, R, net->num_sms, st,
                                      net->rconst.p, net->rval.p, net->ctr64.p + C64_RES_NNZ, net->dist.p, s,
-                                     net->rnnz.p));
+                                     net->rnnz.p, net->need.p, cnt + CNT_NEED));
         if (opt.timing) CUDA_TRY(cudaEventRecord(net->ev[7], st));
         net->ev_map = opt.timing != 0;
         int* rlist = net->res0.p;

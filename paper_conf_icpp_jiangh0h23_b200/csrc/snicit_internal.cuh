@@ -338,7 +338,8 @@ cudaError_t launch_map_residual(const float* y, int N, const int* rows, const in
                                 const int* n_cent, int* M, int* cslot, uint8_t* ne_row, uint8_t* flag_pos,
                                 float* yhat, float* cbuf, int max_rows, int num_sms, cudaStream_t st,
                                 const uint8_t* rconst, const float* rval, unsigned long long* nnz_sum,
-                                int* dist /* [max_rows][s] scratch */, int s, int* rnnz /* nullable, by row */);
+                                int* dist /* [max_rows][s] scratch */, int s, int* rnnz /* nullable, by row */,
+                                int* need /* [max_rows] scratch */, int* need_count /* device int */);
 cudaError_t launch_recover(int N, int R, int plain, const float* yfinal, const uint8_t* live_row, const int* M,
                            const int* cslot, const uint8_t* ne_row, const float* cbuf, float* y_out,
                            uint8_t* cat, int num_sms, cudaStream_t st, int dead_zeroed = 0);
