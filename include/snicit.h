@@ -95,7 +95,10 @@ typedef struct {
                                0 = one kernel launch per layer; 3 = as 1; 4 = the row-resident kernel with
                                each row split over a thread-block cluster of N/8192 CTAs exchanging layer
                                outputs through distributed shared memory (N = 16384 / 32768 / 65536; the
-                               cluster form of a row that does not fit one CTA at several CTAs per SM).
+                               cluster form of a row that does not fit one CTA at several CTAs per SM);
+                               5 = as 1 with the row stored as pairs (y[p], y[p + N/2]) read by 8-byte
+                               loads (kernels_pre_pair.cu).  4 and 5 are measured alternatives (slower
+                               than 1 on B200), kept selectable and parity-tested.
                                Used when every layer < t is circulant
                                with 32 taps, uniform weight and uniform bias, and N/32 is one of
                                32..512 (N = 1024..16384; 4: the cluster form supports every stride);

@@ -790,7 +790,12 @@ static bool pf_plan(const snicit_network* net, int tt, const snicit_options& opt
                 if (net->pf_layers_h[l].nu != 32) g = 1;
             }
         h = (h + 31) / 32 * 32;
-        if (h > N || pre_fused_smem(N, h) > (size_t)227 * 1024) pf = false;
+        if (opt.pre_fused != 5) {  // the split-layout kernel (kernels_pre_fused.cu)
+            if (h > N || pre_fused_smem(N, h) > (size_t)227 * 1024) pf = false;
+        } else {  // the paired-half layout (kernels_pre_pair.cu), on request
+            const int hp = pre_pair_halo(N, net->pf_layers_h.data(), tt);
+            if (hp < 0 || pre_pair_smem(N, hp) > (size_t)227 * 1024) pf = false;
+        }
     }
     *H = h;
     *gen = g;
@@ -968,7 +973,7 @@ static snicit_status infer_core(snicit_network* net, const float* y0, int64_t ba
         return fail(SNICIT_E_INVALID_ARG, "bad eta/eps/prune_eps");
     if (opt.kernel < 0 || opt.kernel > SNICIT_KERNEL_CIRC_SMEM) return fail(SNICIT_E_INVALID_ARG, "bad kernel option");
     if (opt.post_mode < 0 || opt.post_mode > 1) return fail(SNICIT_E_INVALID_ARG, "bad post_mode");
-    if (opt.pre_fused < 0 || opt.pre_fused > 4) return fail(SNICIT_E_INVALID_ARG, "bad pre_fused");
+    if (opt.pre_fused < 0 || opt.pre_fused > 5) return fail(SNICIT_E_INVALID_ARG, "bad pre_fused");
     if (opt.pre_const < 0 || opt.pre_const > 1) return fail(SNICIT_E_INVALID_ARG, "bad pre_const");
     if (opt.res_sparse < 0 || opt.res_sparse > 1) return fail(SNICIT_E_INVALID_ARG, "bad res_sparse");
     if (opt.dyn_t < 0 || opt.dyn_t > 1) return fail(SNICIT_E_INVALID_ARG, "bad dyn_t");
@@ -1111,6 +1116,8 @@ static snicit_status infer_core(snicit_network* net, const float* y0, int64_t ba
         }
         if (pf_cluster)
             CUDA_TRY(launch_pre_cluster(pa, net->pf_layers_h.data(), net->num_sms, st));
+        else if (opt.pre_fused == 5)
+            CUDA_TRY(launch_pre_pair(pa, net->pf_layers_h.data(), net->num_sms, st));
         else
             CUDA_TRY(launch_pre_fused(pa, net->pf_layers_h.data(), net->num_sms, st));
         if (host_streamed) CUDA_TRY(cudaStreamWaitEvent(st, net->cev[1], 0));  // Ya reused after this

@@ -302,6 +302,11 @@ constexpr int kPfMaxLayers = 2000;  // t limit of the row-resident kernel (descr
 // layers: host descriptors of layers 0..t-1
 cudaError_t launch_pre_fused(const PreFusedArgs& a, const PreFusedLayer* layers, int num_sms, cudaStream_t st);
 
+// kernels_pre_pair.cu: the row-resident pre phase in the paired-half layout (the default form)
+size_t pre_pair_smem(int N, int Hp);
+int pre_pair_halo(int N, const PreFusedLayer* layers, int t);  // < 0: not supported
+cudaError_t launch_pre_pair(const PreFusedArgs& a, const PreFusedLayer* layers, int num_sms, cudaStream_t st);
+
 // kernels_pre_cluster.cu: the row-resident pre phase for large rows (N = 16384 / 32768 / 65536), a row
 // split over a cluster of N / 8192 CTAs exchanging layer outputs through distributed shared memory
 int pre_cluster_class(int N, int nu);  // < 0: layer stride not supported

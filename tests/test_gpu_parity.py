@@ -410,8 +410,8 @@ def test_pre_fused_bit_exact(N, nus, B, drop):
     plain = oracle.layers_f32(net, Y0)
     res = {}
     single = N <= 16384  # one CTA per row exists (kernels_pre_fused.cu); pre_fused = 4: cluster form (N >= 16384)
-    for pf in (1, 2, 0, 4):
-        if pf == 4 and N < 16384:
+    for pf in (1, 2, 0, 5, 4):  # 1/2: split layout, 5: paired-half layout, 4: cluster form, 0: per layer
+        if (pf == 4 and N < 16384) or (pf == 5 and not single):
             continue
         Y, cats, st, _ = run_gpu(net, Y0, t=L, drop_dead_rows=drop, pre_fused=pf)
         want = 2 if pf == 4 else (0 if pf == 0 or not single else 1)
