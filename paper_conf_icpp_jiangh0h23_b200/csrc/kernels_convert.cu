@@ -456,9 +456,7 @@ __global__ void __launch_bounds__(kMapThreads) map_finish_kernel(const float* __
         const float4* y4 = reinterpret_cast<const float4*>(y + (size_t)r * N);
         int hit;
         const int slot = map_classify(r, cent, C, rconst, rval, &hit);
-        if (slot >= 0) {  // centroid row (Eq. 4 second case)
-            float4* d4 = reinterpret_cast<float4*>(cbuf + (size_t)slot * N);
-            for (int k = lane; k < N4; k += 32) d4[k] = y4[k];
+        if (slot >= 0) {  // centroid row (Eq. 4 second case); its row is copied by map_centroids_kernel
             if (lane == 0) {
                 M[r] = -1;
                 cslot[r] = slot;
@@ -524,6 +522,20 @@ __global__ void __launch_bounds__(kMapThreads) map_finish_kernel(const float* __
     }
 }
 
+// centroid rows -> the compact centroid buffer (slot = position in y*), many CTAs per row
+__global__ void __launch_bounds__(256) map_centroids_kernel(const float* __restrict__ y, int N, const int* cent,
+                                                            const int* n_cent, int s, float* __restrict__ cbuf) {
+    const int C = min(*n_cent, s);
+    const int N4 = N >> 2;
+    const int per = (N4 + gridDim.y - 1) / gridDim.y;
+    for (int c = blockIdx.x; c < C; c += gridDim.x) {
+        const float4* src = reinterpret_cast<const float4*>(y + (size_t)cent[c] * N);
+        float4* dst = reinterpret_cast<float4*>(cbuf + (size_t)c * N);
+        const int k0 = blockIdx.y * per, k1 = min(N4, k0 + per);
+        for (int k = k0 + threadIdx.x; k < k1; k += blockDim.x) dst[k] = __ldg(src + k);
+    }
+}
+
 cudaError_t launch_map_residual(const float* y, int N, const int* rows, const int* count, const int* cent,
                                 const int* n_cent, int* M, int* cslot, uint8_t* ne_row, uint8_t* flag_pos,
                                 float* yhat, float* cbuf, int max_rows, int num_sms, cudaStream_t st,
@@ -569,6 +581,11 @@ cudaError_t launch_map_residual(const float* y, int N, const int* rows, const in
             map_dist_kernel<32><<<g, kMapThreads, smem, st>>>(y, N, rows, count, cent, n_cent, dist, s, need, need_count);
         });
     if (e != cudaSuccess) return e;
+    {
+        const int gy = std::max(1, std::min(64, (N / 4 + 1023) / 1024));
+        map_centroids_kernel<<<dim3(std::max(1, std::min(s, 64)), gy), 256, 0, st>>>(y, N, cent, n_cent, s, cbuf);
+        if ((e = cudaGetLastError()) != cudaSuccess) return e;
+    }
     int grid = num_sms * 8;
     if (grid > (max_rows + 7) / 8) grid = (max_rows + 7) / 8;
     if (grid < 1) grid = 1;

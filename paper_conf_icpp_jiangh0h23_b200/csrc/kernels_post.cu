@@ -939,13 +939,30 @@ __global__ void __launch_bounds__(256) centroid_const_kernel(PostArgs a, float* 
         return;
     }
     float* s_acc = reinterpret_cast<float*>(s_wb + nl);
+    // Fixed-point prefix, evaluated in parallel: layer l maps the constant v0 to itself (bitwise) for every
+    // l < lfix, so by induction the row enters each of those layers as v0 (acc_l = chain(v0, w_l)) and
+    // leaves the prefix as v0; the serial chain below starts at lfix (SDGC: YMAX is a fixed point of every
+    // layer, so lfix = L - t and nothing is serial)
+    __shared__ int s_lfix;
+    const float v0 = __uint_as_float(an);
+    if (threadIdx.x == 0) s_lfix = nl;
+    __syncthreads();
+    for (int l = threadIdx.x; l < nl; l += blockDim.x) {
+        const float2 wb = s_wb[l];
+        float acc = 0.0f;
+#pragma unroll
+        for (int n = 0; n < kPK; ++n) acc = fmaf(v0, wb.x, acc);
+        s_acc[l] = acc;
+        if (__float_as_uint(sigma(acc + wb.y, a.ymax)) != an) atomicMin(&s_lfix, l);
+    }
+    __syncthreads();
+    const int lfix = s_lfix;
     if (threadIdx.x == 0) {
-        float v = __uint_as_float(an);
+        float v = v0;
         // the chain is a pure function of (v, w0): reuse the previous layer's value when both repeat
-        // (SDGC: one weight for every layer and a fixed point v = YMAX -> one chain for all layers)
         float pv = 0.0f, pw = 0.0f, pacc = 0.0f;
         bool have = false;
-        for (int l = 0; l < nl; ++l) {
+        for (int l = lfix; l < nl; ++l) {
             const float2 wb = s_wb[l];
             float acc;
             if (have && __float_as_uint(v) == __float_as_uint(pv) && __float_as_uint(wb.x) == __float_as_uint(pw)) {
