@@ -155,11 +155,13 @@ class ClockSampler:
     def start(self):
         try:
             self.proc = subprocess.Popen(["nvidia-smi", "-i", str(self.index), f"--query-gpu={self.Q}",
-                                          "--format=csv,noheader,nounits", "-lms", "100"],
+                                          "--format=csv,noheader,nounits", "-lms", "20"],
                                          stdout=subprocess.PIPE, stderr=subprocess.DEVNULL, text=True)
             self.th = threading.Thread(target=self._read, daemon=True)
             self.th.start()
-            time.sleep(0.3)  # the sampler is running before the timed region starts
+            t0 = time.time()  # the sampler is producing lines before the timed region starts
+            while not self.lines and time.time() - t0 < 10.0 and self.proc.poll() is None:
+                time.sleep(0.02)
         except (OSError, FileNotFoundError):
             self.proc = None
 
@@ -167,10 +169,14 @@ class ClockSampler:
         for line in self.proc.stdout:
             self.lines.append(line.strip())
 
+    def mark(self):
+        """Index of the next sample: samples from here on were taken during the timed region."""
+        self.t_mark = len(self.lines)
+
     def stop(self):
         if self.proc is None:
             return None
-        time.sleep(0.15)
+        time.sleep(0.06)
         self.proc.terminate()
         try:
             self.proc.wait(timeout=5)
@@ -178,7 +184,9 @@ class ClockSampler:
             self.proc.kill()
         sm, mx, reasons, pw = [], 0, set(), []
         names = ["hw_slowdown", "hw_thermal_slowdown", "sw_thermal_slowdown", "sw_power_cap"]
-        for ln in self.lines:
+        # samples of the timed region (plus the one straddling its end); at least the last one taken
+        lines = self.lines[max(0, min(getattr(self, "t_mark", 0), len(self.lines) - 1)):]
+        for ln in lines:
             parts = [p.strip() for p in ln.split(",")]
             if len(parts) < 8:
                 continue
@@ -497,11 +505,13 @@ def run_snicit(args):
             ms = float(tt.item())
         return ms
 
-    for _ in range(max(args.warmup, 3)):
-        step()
     clocks = ClockSampler(dev.index)
     if rank == 0:
-        clocks.start()
+        clocks.start()  # running (and under load through the warm-up) before the timed region
+    for _ in range(max(args.warmup, 3)):
+        step()
+    if rank == 0:
+        clocks.mark()
     ms = timed(step, args.steps)
     clk = clocks.stop() if rank == 0 else None
     st0 = g.stats()

@@ -16,6 +16,7 @@
 //    global memory (L1/L2).
 #include <cuda_runtime.h>
 
+#include <cstdlib>
 #include <map>
 #include <mutex>
 #include <utility>
@@ -212,8 +213,15 @@ __device__ __forceinline__ int il_pos(int k, int r) {
     }
 }
 
+// RT = 4 tiles (64 KB at N = 4096) run 256 threads at three CTAs per SM (other CTAs cover a tile's load);
+// RT = 8 / 2: 512 threads, one CTA per SM
+template <int RT>
+constexpr int kIlThreads = RT == 4 ? 256 : kEllThreads;
+template <int RT>
+constexpr int kIlMinBlocks = RT == 4 ? 3 : 1;
+
 template <int MODE, int RT, bool IDX16, bool UNIF, bool RAGGED>
-__global__ void __launch_bounds__(kEllThreads, 1) layer_ell_il_kernel(LayerArgs a) {
+__global__ void __launch_bounds__(kIlThreads<RT>, kIlMinBlocks<RT>) layer_ell_il_kernel(LayerArgs a) {
     static_assert(RT == 2 || RT == 4 || RT == 8, "RT");
     extern __shared__ __align__(128) unsigned char smem[];
     const int N = a.N;
@@ -372,13 +380,14 @@ static cudaError_t launch_ell_t(const LayerArgs& a, int max_rows, int num_sms, c
     SNICIT_PICK(false, false, true)
 #undef SNICIT_PICK
     int per_sm = 1;
-    cudaError_t e = blocks_per_sm((const void*)kern, kEllThreads, smem, &per_sm);
+    const int threads = IL ? kIlThreads<RT> : kEllThreads;
+    cudaError_t e = blocks_per_sm((const void*)kern, threads, smem, &per_sm);
     if (e != cudaSuccess) return e;
     const int tiles = (max_rows + RT - 1) / RT;
     int grid = num_sms * per_sm;
     if (grid > tiles) grid = tiles;
     if (grid < 1) grid = 1;
-    kern<<<grid, kEllThreads, smem, st>>>(a);
+    kern<<<grid, threads, smem, st>>>(a);
     return cudaGetLastError();
 }
 
@@ -386,6 +395,11 @@ template <int MODE>
 static cudaError_t launch_ell_m(const LayerArgs& a, int max_rows, int num_sms, cudaStream_t st) {
     if (!ell_smem_ok(a.N)) return launch_ell_t<MODE, 4, false>(a, max_rows, num_sms, st);
     const size_t row = (size_t)a.N * 4;
+    static const int force_rt = [] {
+        const char* e = getenv("SNICIT_ELL_RT");  // A/B experiments only
+        return e ? atoi(e) : 0;
+    }();
+    if (force_rt == 4 && max_rows >= 4 && 4 * row <= 70 * 1024) return launch_ell_t<MODE, 4, true>(a, max_rows, num_sms, st);
     if (max_rows >= 8 && 8 * row <= 200 * 1024) return launch_ell_t<MODE, 8, true>(a, max_rows, num_sms, st);
     if (max_rows >= 4 && 4 * row <= 200 * 1024) return launch_ell_t<MODE, 4, true>(a, max_rows, num_sms, st);
     if (max_rows >= 2 && 2 * row <= 200 * 1024) return launch_ell_t<MODE, 2, true>(a, max_rows, num_sms, st);
