@@ -723,6 +723,11 @@ __device__ __forceinline__ int ilog2(int x) { return 31 - __clz(x); }
 __global__ void __cluster_dims__(kCL, 1, 1) __launch_bounds__(kClThreads) centroid_cluster_kernel(PostArgs a) {
     extern __shared__ __align__(128) float sm[];
     __shared__ float* s_rbase[2][kCL];  // peers' slice buffers (cluster-mapped generic pointers)
+    // constant-row detection (R25 from the layer the row becomes constant): each CTA's output range
+    // (bits of sigma outputs, >= 0) pushed to every rank before the layer's cluster barrier
+    __shared__ unsigned s_vmn[2][kCL], s_vmx[2][kCL];
+    __shared__ unsigned s_bmn[2], s_bmx[2];
+    __shared__ unsigned* s_vbase[2][kCL];
     cg::cluster_group cl = cg::this_cluster();
     const int r = (int)cl.block_rank();
     const int cid = blockIdx.x / kCL;
@@ -736,12 +741,22 @@ __global__ void __cluster_dims__(kCL, 1, 1) __launch_bounds__(kClThreads) centro
     if (threadIdx.x < 2 * kCL) {
         const int bsel = threadIdx.x / kCL, o = threadIdx.x % kCL;
         s_rbase[bsel][o] = cl.map_shared_rank(slice[bsel], o);
+        s_vbase[bsel][o] = cl.map_shared_rank(bsel ? &s_vmx[0][0] : &s_vmn[0][0], o);
     }
     for (int i = threadIdx.x; i < S; i += blockDim.x) slice[0][i] = a.cbuf[(size_t)cid * N + r * S + i];
     int prev_part = 0, prev_nu = 1, cur = 0;
+    bool cst = false;
+    float vc = 0.0f;
+    int lc = a.L;
     cl.sync();
     PL Ld = load_pl(a.layers + a.t);
     for (int l = a.t; l < a.L; ++l) {
+        const int par = (l - a.t) & 1;
+        if (threadIdx.x == 0) {
+            s_bmn[par] = 0xffffffffu;
+            s_bmx[par] = 0u;
+        }
+        unsigned umn = 0xffffffffu, umx = 0u;
         const PL Lnext = load_pl(a.layers + min(l + 1, a.L - 1));
         const int nu = Ld.nu, cls = Ld.cls;
         const int shnu = ilog2(nu), Q = N >> shnu;
@@ -801,7 +816,11 @@ __global__ void __cluster_dims__(kCL, 1, 1) __launch_bounds__(kClThreads) centro
         auto emit = [&](float acc, int q, int so) {
             const float b = ubias ? b0 : __ldg(bias + q);
             if (aout) aout[q] = acc;
-            out[so] = sigma(acc + b, a.ymax);
+            const float o = sigma(acc + b, a.ymax);
+            out[so] = o;
+            const unsigned u = __float_as_uint(o + 0.0f);
+            umn = min(umn, u);
+            umx = max(umx, u);
         };
         if (cls == PCLS_NU1) {
             constexpr int M = 5, WIN = M + kPK - 1;  // odd M: conflict-free window loads
@@ -854,11 +873,54 @@ __global__ void __cluster_dims__(kCL, 1, 1) __launch_bounds__(kClThreads) centro
                 }
             }
         }
-        cl.sync();  // outputs of this layer visible cluster-wide; nobody still reads slice[cur]
+        if (a.scalar_ok) {  // this CTA's output range -> every rank
+            umn = __reduce_min_sync(0xffffffffu, umn);
+            umx = __reduce_max_sync(0xffffffffu, umx);
+            if ((threadIdx.x & 31) == 0) {
+                atomicMin(&s_bmn[par], umn);
+                atomicMax(&s_bmx[par], umx);
+            }
+            __syncthreads();
+            if (threadIdx.x < kCL) {
+                s_vbase[0][threadIdx.x][par * kCL + r] = s_bmn[par];
+                s_vbase[1][threadIdx.x][par * kCL + r] = s_bmx[par];
+            }
+        }
+        cl.sync();  // outputs (and ranges) of this layer visible cluster-wide; nobody still reads slice[cur]
         cur ^= 1;
         prev_part = part;
         prev_nu = nu;
         Ld = Lnext;
+        if (a.scalar_ok) {
+            unsigned gmn = 0xffffffffu, gmx = 0u;
+#pragma unroll
+            for (int o = 0; o < kCL; ++o) {
+                gmn = min(gmn, s_vmn[par][o]);
+                gmx = max(gmx, s_vmx[par][o]);
+            }
+            if (gmn == gmx && l + 1 < a.L) {  // the row is the constant v: every later layer maps it to a
+                cst = true;                   // constant row (one weight, one bias, R25)
+                vc = __uint_as_float(gmn);
+                lc = l + 1;
+                break;
+            }
+        }
+    }
+    if (cst) {  // layers lc .. L-1 by one scalar chain; a_c rows (constant) written when residues need them
+        for (int l = lc; l < a.L; ++l) {
+            const PostLayer* pl = a.layers + l;
+            const float w0 = pl->w0, b0 = pl->b0;
+            float acc = 0.0f;
+#pragma unroll
+            for (int n = 0; n < kPK; ++n) acc = fmaf(vc, w0, acc);
+            if (want_a) {
+                float* dst = a.a_all + ((size_t)(l - a.t) * a.s + cid) * N + r * S;
+                for (int i = threadIdx.x; i < S; i += blockDim.x) dst[i] = acc;
+            }
+            vc = sigma(acc + b0, a.ymax);
+        }
+        for (int i = threadIdx.x; i < S; i += blockDim.x) a.cbuf[(size_t)cid * N + r * S + i] = vc;
+        return;
     }
     // ---- the final centroid row back to global memory
     for (int i = threadIdx.x; i < S; i += blockDim.x) {

@@ -1371,6 +1371,11 @@ static snicit_status infer_core(snicit_network* net, const float* y0, int64_t ba
                 }
             }
             const bool use_cluster = opt.post_cluster != 0 && centroid_cluster_ok(N, nus.data(), clss.data(), tt, L);
+            {  // every post layer circulant with one weight and one bias: constant rows stay constant (R25)
+                bool sok = opt.post_const != 0 && opt.kernel == SNICIT_KERNEL_AUTO;
+                for (int l = tt; l < L && sok; ++l) sok = net->pf_elig[l] != 0;
+                pa.scalar_ok = sok ? 1 : 0;
+            }
             net->last_cluster = use_cluster;
             if (use_cluster)
                 CUDA_TRY(launch_centroid_cluster(pa, s, win_max, st));
