@@ -485,21 +485,59 @@ __global__ void __launch_bounds__(kPostThreads, 2) residual_traj_kernel(PostArgs
     const int dup = h == N;
     const int n = *a.rcount;
     const int cap = sp_cap(N);
-    // sparse-form scratch after the two row buffers
-    unsigned* bm = reinterpret_cast<unsigned*>(sm + 2 * (N + h));
+    // three row buffers when they fit (a.smem_floats): the next residue row is loaded by the TMA engine
+    // into the third while this one is processed; otherwise two and a synchronous stage
+    const int nbuf = a.smem_floats >= 3 * (N + h) + (a.res_sparse ? sp_ints(N) : 0) ? 3 : 2;
+    // sparse-form scratch after the row buffers
+    unsigned* bm = reinterpret_cast<unsigned*>(sm + nbuf * (N + h));
     int* lsts[2] = {reinterpret_cast<int*>(bm + (N + 31) / 32), reinterpret_cast<int*>(bm + (N + 31) / 32) + cap};
     int* tl = lsts[1] + cap;
     unsigned long long c_full = 0, c_sparse = 0, c_sout = 0, c_scalar = 0;  // thread 0's work counters
+    __shared__ __align__(8) uint64_t s_bar;
+    __shared__ int s_next;
+    int sb = 0;        // buffer receiving / holding the prefetched row
+    uint32_t ph = 0;
+    if (nbuf == 3 && threadIdx.x == 0) {
+        mbar_init(&s_bar, 1);
+        fence_proxy_async_smem();
+        const int p0 = atomicAdd(a.work_counter, 1);
+        s_next = p0;
+        if (p0 < n) {
+            mbar_arrive_expect_tx(&s_bar, (uint32_t)N * 4);
+            bulk_g2s(sm, a.yhat + (size_t)a.rlist[p0] * N, (uint32_t)N * 4, &s_bar);
+        }
+    }
     for (;;) {
-        if (threadIdx.x == 0) s_p = atomicAdd(a.work_counter, 1);
+        if (nbuf == 2 && threadIdx.x == 0) s_p = atomicAdd(a.work_counter, 1);
         __syncthreads();
-        const int p = s_p;
+        const int p = nbuf == 3 ? s_next : s_p;
         if (p >= n) break;
         const int row = a.rlist[p];
         const int slot = a.cslot[row];
-        float* cur = sm;
-        float* nxt = sm + N + h;
-        stage_row(cur, a.yhat + (size_t)row * N, N);
+        float* cur;
+        float* nxt;
+        if (nbuf == 3) {
+            cur = sm + sb * (N + h);
+            nxt = sm + ((sb + 1) % 3) * (N + h);
+            float* spare = sm + ((sb + 2) % 3) * (N + h);
+            mbar_wait(&s_bar, ph);
+            ph ^= 1u;
+            __syncthreads();  // every thread past the wait before the barrier is re-armed
+            if (threadIdx.x == 0) {  // the next row -> the spare buffer, behind this row's work
+                const int np = atomicAdd(a.work_counter, 1);
+                s_next = np;
+                if (np < n) {
+                    fence_proxy_async_smem();  // the spare buffer's generic accesses (previous rows) first
+                    mbar_arrive_expect_tx(&s_bar, (uint32_t)N * 4);
+                    bulk_g2s(spare, a.yhat + (size_t)a.rlist[np] * N, (uint32_t)N * 4, &s_bar);
+                }
+            }
+            sb = (sb + 2) % 3;  // next row's buffer
+        } else {
+            cur = sm;
+            nxt = sm + N + h;
+            stage_row(cur, a.yhat + (size_t)row * N, N);
+        }
         if (threadIdx.x < 3) {
             s_nz[threadIdx.x] = 0;
             s_mn[threadIdx.x] = 0x7fffffff;
@@ -613,15 +651,15 @@ __global__ void __launch_bounds__(kPostThreads, 2) residual_traj_kernel(PostArgs
             // the centroid's pre-activation rows are constant from here on: gather their values (one per
             // layer) into shared memory first -- the row buffers are free now -- so the serial chain does not
             // wait on one L2 round trip per layer
-            float* s_acv = sm;       // [L - l] a_c values
-            float2* s_wb = reinterpret_cast<float2*>(sm + ((a.L - l + 1) & ~1));  // [L - l] (w0, b0)
+            float* s_acv = nxt;      // [L - l] a_c values (the row buffers are free now; not the spare one)
+            float2* s_wb = reinterpret_cast<float2*>(nxt + ((a.L - l + 1) & ~1));  // [L - l] (w0, b0)
             const int nl = a.L - l;
-            const bool fits = 3 * nl <= 2 * (N + h);
+            const bool fits = 3 * nl <= N + h;
             if (fits) {
-                for (int i = threadIdx.x; i < nl; i += blockDim.x) {
-                    s_acv[i] = __ldg(a.a_all + ((size_t)(l + i - a.t) * a.s + slot) * N);
-                    const PostLayer* pl = a.layers + l + i;
-                    s_wb[i] = make_float2(pl->w0, pl->b0);
+                for (int i = threadIdx.x; i < nl; i += blockDim.x) {  // contiguous copies (acconst_kernel, load time)
+                    s_acv[i] = a.acs ? a.acs[(size_t)slot * (a.L - a.t) + (l - a.t) + i]
+                                     : __ldg(a.a_all + ((size_t)(l + i - a.t) * a.s + slot) * N);
+                    s_wb[i] = a.wb ? a.wb[l + i] : make_float2(a.layers[l + i].w0, a.layers[l + i].b0);
                 }
                 __syncthreads();
             }
@@ -698,6 +736,8 @@ __global__ void __launch_bounds__(256) acconst_kernel(PostArgs a) {
         }
     }
     if (threadIdx.x == 0) a.cfrom[c] = l2;
+    if (a.acs)  // the constant a_c values from cfrom on, contiguous per centroid (the residue rows' scalar tails)
+        for (int i = l2 + threadIdx.x; i < nl; i += blockDim.x) a.acs[(size_t)c * nl + i] = __ldg(a.a_all + ((size_t)i * a.s + c) * N);
 }
 cudaError_t launch_acconst(const PostArgs& a, int C_max, cudaStream_t st) {
     if (C_max <= 0) return cudaSuccess;
@@ -907,17 +947,64 @@ __global__ void __cluster_dims__(kCL, 1, 1) __launch_bounds__(kClThreads) centro
         }
     }
     if (cst) {  // layers lc .. L-1 by one scalar chain; a_c rows (constant) written when residues need them
-        for (int l = lc; l < a.L; ++l) {
-            const PostLayer* pl = a.layers + l;
-            const float w0 = pl->w0, b0 = pl->b0;
-            float acc = 0.0f;
-#pragma unroll
-            for (int n = 0; n < kPK; ++n) acc = fmaf(vc, w0, acc);
-            if (want_a) {
-                float* dst = a.a_all + ((size_t)(l - a.t) * a.s + cid) * N + r * S;
-                for (int i = threadIdx.x; i < S; i += blockDim.x) dst[i] = acc;
+        // the slice / window buffers are free now: (w0, b0) of the remaining layers, gathered in parallel,
+        // then the serial chain (memoised on (v, w0): SDGC repeats one weight and reaches a fixed point),
+        // then the a_c rows written by all threads
+        const int nl = a.L - lc;
+        float2* s_wb2 = reinterpret_cast<float2*>(sm);
+        float* s_ac = reinterpret_cast<float*>(s_wb2 + nl);
+        const bool fits = 3 * nl <= a.smem_floats;
+        __shared__ float s_vfin;
+        if (fits) {
+            __syncthreads();  // every thread is past its reads of the buffers
+            for (int i = threadIdx.x; i < nl; i += blockDim.x) {
+                const PostLayer* pl = a.layers + lc + i;
+                s_wb2[i] = make_float2(pl->w0, pl->b0);
             }
-            vc = sigma(acc + b0, a.ymax);
+            __syncthreads();
+            if (threadIdx.x == 0) {
+                float v = vc, pv = 0.0f, pw = 0.0f, pacc = 0.0f;
+                bool have = false;
+                for (int i = 0; i < nl; ++i) {
+                    const float2 wb = s_wb2[i];
+                    float acc;
+                    if (have && __float_as_uint(v) == __float_as_uint(pv) && __float_as_uint(wb.x) == __float_as_uint(pw)) {
+                        acc = pacc;
+                    } else {
+                        acc = 0.0f;
+#pragma unroll
+                        for (int n = 0; n < kPK; ++n) acc = fmaf(v, wb.x, acc);
+                        pv = v;
+                        pw = wb.x;
+                        pacc = acc;
+                        have = true;
+                    }
+                    s_ac[i] = acc;
+                    v = sigma(acc + wb.y, a.ymax);
+                }
+                s_vfin = v;
+            }
+            __syncthreads();
+            if (want_a)
+                for (int i = 0; i < nl; ++i) {
+                    float* dst = a.a_all + ((size_t)(lc + i - a.t) * a.s + cid) * N + r * S;
+                    const float acc = s_ac[i];
+                    for (int j = threadIdx.x; j < S; j += blockDim.x) dst[j] = acc;
+                }
+            vc = s_vfin;
+        } else {
+            for (int l = lc; l < a.L; ++l) {
+                const PostLayer* pl = a.layers + l;
+                const float w0 = pl->w0, b0 = pl->b0;
+                float acc = 0.0f;
+#pragma unroll
+                for (int n = 0; n < kPK; ++n) acc = fmaf(vc, w0, acc);
+                if (want_a) {
+                    float* dst = a.a_all + ((size_t)(l - a.t) * a.s + cid) * N + r * S;
+                    for (int i = threadIdx.x; i < S; i += blockDim.x) dst[i] = acc;
+                }
+                vc = sigma(acc + b0, a.ymax);
+            }
         }
         for (int i = threadIdx.x; i < S; i += blockDim.x) a.cbuf[(size_t)cid * N + r * S + i] = vc;
         return;
@@ -1068,9 +1155,11 @@ cudaError_t launch_centroid_const(const PostArgs& a, float* cout, int* cdone, in
     return cudaGetLastError();
 }
 
-cudaError_t launch_centroid_cluster(const PostArgs& a, int C_max, int win_max, cudaStream_t st) {
+cudaError_t launch_centroid_cluster(const PostArgs& a_in, int C_max, int win_max, cudaStream_t st) {
     if (C_max <= 0) return cudaSuccess;
+    PostArgs a = a_in;
     const size_t smem = sizeof(float) * (2 * (size_t)(a.N / kCL) + (size_t)win_max);
+    a.smem_floats = (int)(smem / sizeof(float));
     int per_sm = 1;
     cudaError_t e = blocks_per_sm((const void*)centroid_cluster_kernel, kClThreads, smem, &per_sm);
     if (e != cudaSuccess) return e;
@@ -1091,11 +1180,16 @@ cudaError_t launch_centroid_traj(const PostArgs& a, int C_max, cudaStream_t st) 
 cudaError_t launch_residual_traj(const PostArgs& a_in, int max_rows, int num_sms, cudaStream_t st) {
     if (max_rows <= 0) return cudaSuccess;
     PostArgs a = a_in;
-    size_t smem = sizeof(float) * 2 * (size_t)(a.N + post_halo(a.N));
-    if (a.res_sparse && smem + sizeof(int) * (size_t)sp_ints(a.N) <= (size_t)220 * 1024)
-        smem += sizeof(int) * (size_t)sp_ints(a.N);
+    const size_t row = sizeof(float) * (size_t)(a.N + post_halo(a.N));
+    const size_t sp = sizeof(int) * (size_t)sp_ints(a.N);
+    const size_t lim = (size_t)220 * 1024;
+    size_t smem = 2 * row;
+    if (a.res_sparse && smem + sp <= lim)
+        smem += sp;
     else
         a.res_sparse = 0;
+    if (smem + row <= lim) smem += row;  // a third row buffer: the next row is prefetched
+    a.smem_floats = (int)(smem / sizeof(float));
     int per_sm = 1;
     cudaError_t e = blocks_per_sm((const void*)residual_traj_kernel, kPostThreads, smem, &per_sm);
     if (e != cudaSuccess) return e;

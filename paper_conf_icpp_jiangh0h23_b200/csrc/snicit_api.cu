@@ -128,6 +128,8 @@ struct snicit_network {
     DevBuf<int> dist;         // [rows][s] L0 distances of Alg. 2 (map_residual pass 1)
     DevBuf<int> rnnz;         // [rows] non-zeros of each residue row at t
     DevBuf<int> need;         // [rows] list positions whose Alg. 2 distances are computed
+    DevBuf<float> acs;        // [s][L - t] constant centroid pre-activations from cfrom on
+    DevBuf<float2> wb_d;      // [L] (w0, b0) per layer (first bias of the layer)
     DevBuf<float> probe0, probe1;  // dynamic t: the probe rows (ping-pong)
     DevBuf<int> pstat;             // dynamic t: per probe layer (live, identical, distinct)
     DevBuf<unsigned long long> phash;  // dynamic t: per probe layer and row (hash, live)
@@ -278,6 +280,11 @@ static cudaError_t net_upload_common(snicit_network* net, const float* bias, con
         }
         e = upload(net->pf_layers_d, net->pf_layers_h.data(), net->pf_layers_h.size());
     }
+    if (e == cudaSuccess) {
+        std::vector<float2> wb(L);
+        for (int l = 0; l < L; ++l) wb[l] = make_float2(net->plan[l].w0, bias[(int64_t)l * N]);
+        e = upload(net->wb_d, wb.data(), wb.size());
+    }
     if (e == cudaSuccess) e = net->pf_full.ensure(1);
     if (e == cudaSuccess) e = net->counters.ensure(CNT_N);
     if (e == cudaSuccess) e = cudaMallocHost(&net->h_counters, sizeof(int) * CNT_N);
@@ -363,6 +370,8 @@ void snicit_free_network(snicit_network* net) {
     net->dist.release();
     net->rnnz.release();
     net->need.release();
+    net->acs.release();
+    net->wb_d.release();
     net->probe0.release();
     net->probe1.release();
     net->pstat.release();
@@ -1388,7 +1397,10 @@ static snicit_status infer_core(snicit_network* net, const float* y0, int64_t ba
                 for (int l = tt; l < L && sok; ++l) sok = net->pf_elig[l] != 0;
                 if (sok) {  // constant residue rows over constant centroids leave as scalars
                     CUDA_TRY(net->cfrom.ensure((size_t)s));
+                    CUDA_TRY(net->acs.ensure((size_t)s * (L - tt)));
                     pa.cfrom = net->cfrom.p;
+                    pa.acs = net->acs.p;
+                    pa.wb = net->wb_d.p;
                     pa.scalar_ok = 1;
                     CUDA_TRY(launch_acconst(pa, s, st));
                     ++launches;

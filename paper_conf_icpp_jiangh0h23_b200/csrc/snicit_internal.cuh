@@ -235,6 +235,9 @@ struct PostArgs {
                          //   over constant centroids are carried by a scalar (residual_traj_kernel)
     int res_sparse;      // 1: sparse-entry residue form for residue rows with few non-zeros (circulant layers)
     const int* rnnz;     // nullable: non-zeros of each row's residue at t (map_residual), by row id
+    int smem_floats;     // set by the launcher: dynamic shared memory of the kernel (floats)
+    float* acs;          // nullable: [s][L - t] constant a_c values of each centroid from cfrom on (acconst)
+    const float2* wb;    // nullable: [L] (w0, b0) of each layer (uniform layers)
     unsigned long long* dyn;  // nullable: [L - t + 1] residue rows by post layers survived, [L - t + 1] by the
                               //   post layer from which they were carried by a scalar (L - t: never)
     unsigned long long* ctr64;  // nullable: work counters (Ctr64)
