@@ -634,6 +634,19 @@ def run_snicit(args):
                                                                     "avg_launch_ms", "by_stride") if k in r0}
                     roof["per_layer_kernels"]["ms_total"] = float(pm0.sum())
 
+    # ---- dynamic threshold layer (options.dyn_t, DESIGN R28): t chosen from the first s rows, at most t
+    dyn = None
+    if not args.no_uncompressed:
+        opt_d = default_options(kernel=kern, n_segments=snic["n"], pre_fused=args.pre_fused, dyn_t=1)
+
+        def step_dyn():
+            g.infer(y0, t=t, s=s, options=opt_d, y_out=y_out, row_offset=row0)
+            g.categories_device(cat_buf)
+        step_dyn()
+        ms_d = timed(step_dyn, max(1, min(args.steps, 3)))
+        dyn = {"t": int(g.stats()["threshold_layer"]), "t_max": t, "ms_per_step": ms_d,
+               "value": B_global * nnz / (ms_d * 1e-3), "unit": UNIT}
+
     # ---- uncompressed GPU baseline (t >= L, same kernels)
     unc = None
     if not args.no_uncompressed:
@@ -749,7 +762,7 @@ def run_snicit(args):
                 "parallelism": f"dp{world} (row shards, {args.scaling} scaling)"}),
             "roofline": roof, "cpu_baseline": cpu, "e2e": e2e, "e2e_packed": e2e_packed, "clocks": clk,
             "gpu_launches": int(launches_per_step * args.steps + (2 * args.steps if distributed else args.steps)),
-            "uncompressed": unc, "phases_ms": phases, "per_rank": per_rank,
+            "uncompressed": unc, "dynamic_t": dyn, "phases_ms": phases, "per_rank": per_rank,
             "categories": n_cat_global,
             "dynamics": {k: st0[k] for k in ("live_at_t", "n_centroids", "n_sampled", "residual_at_t",
                                              "residual_final", "n_categories")},
