@@ -30,6 +30,7 @@
 // active list at t.  Rows are scheduled dynamically (one atomic per row).
 #include <cuda_runtime.h>
 
+#include <cmath>
 #include <cstring>
 
 #include "snicit_internal.cuh"
@@ -202,7 +203,7 @@ struct PfCfg {
 struct PfLayerParam {
     float w0, b0;
     int nu;
-    int flags;  // cls | dead_next << 4 | ymax_fixed << 5
+    int flags;  // cls | dead_next << 4 | ymax_fixed << 5 | ymax fixed for all later layers < t << 6
 };
 struct PreFusedParams {
     PreFusedArgs a;
@@ -224,8 +225,8 @@ __global__ void __launch_bounds__(T, PfCfg<T>::kMinBlocks) pre_fused_kernel(cons
     uint64_t* bar = reinterpret_cast<uint64_t*>(buf + NB * S);  // [2] row loads, alternating per row
     int* s_pos = reinterpret_cast<int*>(bar + 2);               // [0] first row, [2 + (k & 1)] next row
     constexpr int kWarps = T / 32;
-    float* s_rep = reinterpret_cast<float*>(s_pos + 4);  // [2][kWarps] per-warp reference value
-    int* s_ok = reinterpret_cast<int*>(s_rep + 2 * kWarps);  // [2][kWarps] per-warp "all equal" vote
+    unsigned* s_vmn = reinterpret_cast<unsigned*>(s_pos + 4);  // [2][kWarps] per-warp output minimum (bits)
+    unsigned* s_vmx = s_vmn + 2 * kWarps;                      // [2][kWarps] per-warp output maximum
     const int tid = threadIdx.x;
     const int count = *a.count;
     if (tid == 0) {
@@ -237,7 +238,7 @@ __global__ void __launch_bounds__(T, PfCfg<T>::kMinBlocks) pre_fused_kernel(cons
     __syncthreads();
     int pos = s_pos[0];
     // one row (and its circular halo: a second copy of the row head) -> buffer `dst`, completion on `b`
-    uint32_t* s_bits = reinterpret_cast<uint32_t*>(s_ok + 2 * kWarps);  // [2][N/32] packed rows (a.ybits)
+    uint32_t* s_bits = reinterpret_cast<uint32_t*>(s_vmx + 2 * kWarps);  // [2][N/32] packed rows (a.ybits)
     int* s_surv = reinterpret_cast<int*>(s_bits + 2 * (N / 32));       // [kPfSurv] rows alive at t, batched
     int nsurv = 0;                                                     // (tid 0) entries in s_surv
     // one atomic per kPfSurv survivors (an atomic whose result is waited on stalls the whole CTA at the
@@ -307,6 +308,7 @@ __global__ void __launch_bounds__(T, PfCfg<T>::kMinBlocks) pre_fused_kernel(cons
         bool cst = false, dead = false;
         float v = 0.0f;
         int full = 0;
+        unsigned cmn = 0u, cmx = 0xffffffffu;  // the previous layer's output range (bits)
         int lend = a.t;  // the layer that zeroed the row (dead, R23), or t: alive after layer l <=> lend > l
         for (int l = 0; l < a.t; ++l) {
             // WUNI: one weight for every layer, read at a constant offset -> a uniform register operand
@@ -315,6 +317,23 @@ __global__ void __launch_bounds__(T, PfCfg<T>::kMinBlocks) pre_fused_kernel(cons
             const bool dead_next = (fl >> 4) & 1;
             if (!cst) {
                 float mn = __int_as_float(0x7f800000), mx = -__int_as_float(0x7f800000);
+                // range prediction (exact, one weight w0 >= 0 and one bias for every layer < t): every
+                // output of this layer is an fma chain monotone in each input, so if the previous layer's
+                // minimum already maps to YMAX (>= thr_hi) every output is YMAX, and if its maximum maps to 0
+                // (<= thr_lo) every output is 0 -- the row becomes constant without this layer's evaluation
+                if (a.thr_ok && l > 0) {
+                    const float pmn = __uint_as_float(cmn), pmx = __uint_as_float(cmx);
+                    if (pmn >= a.thr_hi || pmx <= a.thr_lo) {
+                        v = pmn >= a.thr_hi ? a.ymax : 0.0f;
+                        cst = true;
+                        if (v == 0.0f && a.drop && dead_next) {
+                            dead = true;
+                            lend = l;
+                            break;
+                        }
+                        continue;
+                    }
+                }
                 const int cls = fl & 15;
                 if (cls == PF_NU1)
                     pf_body_nu1<T>(in, out, w0, b0, a.ymax, H, mn, mx);
@@ -324,23 +343,25 @@ __global__ void __launch_bounds__(T, PfCfg<T>::kMinBlocks) pre_fused_kernel(cons
                     pf_body_str<T, 0, kPfStrHalo<T>>(in, out, p.L[l].nu, w0, b0, a.ymax, H, mn, mx);
                 else
                     pf_body_str<T, 32, kPfStrHalo<T>>(in, out, 32, w0, b0, a.ymax, H, mn, mx);
-                // "all outputs equal" in one barrier: a warp votes against its lane 0's minimum and
-                // publishes (vote, value) before the barrier; after it every thread combines the warps'
-                // entries (slots double-buffered by layer parity, so no second barrier is needed)
+                // the row's output range in one barrier: each warp publishes its (min, max) (bits of
+                // outputs >= 0, -0 as +0, so bit order is value order and equal bits are equal values); after
+                // the barrier every warp reduces the kWarps entries (slots double-buffered by layer parity)
                 {
-                    const float ref = __shfl_sync(0xffffffffu, mn, 0);
-                    const bool ok = __all_sync(0xffffffffu, mn >= ref && mx <= ref);
+                    const unsigned wmn = __reduce_min_sync(0xffffffffu, __float_as_uint(mn + 0.0f));
+                    const unsigned wmx = __reduce_max_sync(0xffffffffu, __float_as_uint(mx + 0.0f));
                     if ((tid & 31) == 0) {
-                        s_rep[(l & 1) * kWarps + (tid >> 5)] = ref;
-                        s_ok[(l & 1) * kWarps + (tid >> 5)] = ok ? 1 : 0;
+                        s_vmn[(l & 1) * kWarps + (tid >> 5)] = wmn;
+                        s_vmx[(l & 1) * kWarps + (tid >> 5)] = wmx;
                     }
                 }
-                __syncthreads();  // outputs and votes written
-                bool all_eq = true;
-                const float o0 = s_rep[(l & 1) * kWarps];
-#pragma unroll
-                for (int w = 0; w < kWarps; ++w)
-                    all_eq = all_eq && s_ok[(l & 1) * kWarps + w] && s_rep[(l & 1) * kWarps + w] == o0;
+                __syncthreads();  // outputs and ranges written
+                {
+                    const int ln = tid & 31;
+                    cmn = __reduce_min_sync(0xffffffffu, ln < kWarps ? s_vmn[(l & 1) * kWarps + ln] : 0xffffffffu);
+                    cmx = __reduce_max_sync(0xffffffffu, ln < kWarps ? s_vmx[(l & 1) * kWarps + ln] : 0u);
+                }
+                const bool all_eq = cmn == cmx;  // every output equal (R26)
+                const float o0 = __uint_as_float(cmn);
                 ++full;
                 float* tmp = in;
                 in = out;
@@ -373,6 +394,8 @@ __global__ void __launch_bounds__(T, PfCfg<T>::kMinBlocks) pre_fused_kernel(cons
                     lend = l;
                     break;
                 }
+                // fixed point for every remaining layer: nothing more to evaluate (uncompressed path: t = L)
+                if ((v == a.ymax && ((fl >> 6) & 1)) || (v == 0.0f && dead_next)) break;
             }
         }
         if (dead && a.ydead) {  // final activations of a dead row: zeros, written now (the SMs' HBM is idle)
@@ -469,6 +492,53 @@ cudaError_t launch_pre_fused(const PreFusedArgs& a, const PreFusedLayer* layers,
         p.L[l].b0 = layers[l].b0;
         p.L[l].nu = layers[l].nu;
         p.L[l].flags = (layers[l].cls & 15) | (layers[l].dead_next ? 16 : 0) | (layers[l].ymax_fixed ? 32 : 0);
+    }
+    // bit 6: YMAX is a fixed point of every layer l + 1 .. t-1 (a constant YMAX row after layer l needs
+    // no more evaluation)
+    for (int l = a.t - 1, all = 1; l >= 0; --l) {
+        if (all) p.L[l].flags |= 64;
+        all = all && layers[l].ymax_fixed;
+    }
+    // range prediction thresholds (one weight >= 0 and one bias for every layer < t; see the kernel)
+    p.a.thr_ok = 0;
+    {
+        bool same = layers[0].w0 >= 0.0f;
+        for (int l = 1; l < a.t && same; ++l)
+            same = memcmp(&layers[l].w0, &layers[0].w0, sizeof(float)) == 0 &&
+                   memcmp(&layers[l].b0, &layers[0].b0, sizeof(float)) == 0;
+        if (same) {
+            const float w0 = layers[0].w0, b0 = layers[0].b0, ymax = a.ymax;
+            auto out = [&](float m) {  // the kernels' chain for a constant input m, then sigma
+                float acc = 0.0f;
+                for (int n = 0; n < 32; ++n) acc = std::fma(m, w0, acc);
+                const float z = acc + b0;
+                return std::fmin(std::fmax(z, 0.0f), ymax);
+            };
+            auto bits = [](float f) { uint32_t u; memcpy(&u, &f, 4); return u; };
+            auto flt = [](uint32_t u) { float f; memcpy(&f, &u, 4); return f; };
+            // thr_hi = least m in [0, ymax] with out(m) == ymax (out is monotone non-decreasing in m)
+            float hi = INFINITY, lo = -1.0f;
+            if (out(ymax) == ymax) {
+                uint32_t a0 = 0, a1 = bits(ymax);
+                while (a0 < a1) {
+                    const uint32_t mid = a0 + (a1 - a0) / 2;
+                    if (out(flt(mid)) == ymax) a1 = mid; else a0 = mid + 1;
+                }
+                hi = flt(a0);
+            }
+            // thr_lo = greatest m in [0, ymax] with out(m) == 0
+            if (out(0.0f) == 0.0f) {
+                uint32_t a0 = 0, a1 = bits(ymax);
+                while (a0 < a1) {
+                    const uint32_t mid = a0 + (a1 - a0 + 1) / 2;
+                    if (out(flt(mid)) == 0.0f) a0 = mid; else a1 = mid - 1;
+                }
+                lo = flt(a0);
+            }
+            p.a.thr_hi = hi;
+            p.a.thr_lo = lo;
+            p.a.thr_ok = a.const_skip ? 1 : 0;
+        }
     }
     bool wuni = true;
     for (int l = 1; l < a.t; ++l) wuni = wuni && memcmp(&p.L[l].w0, &p.L[0].w0, sizeof(float)) == 0;

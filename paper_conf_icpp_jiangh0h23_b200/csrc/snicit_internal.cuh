@@ -295,6 +295,8 @@ struct PreFusedArgs {
     float* rval;
     unsigned long long* full_rl;  // nullable: += full (non-constant) row-layer evaluations
     unsigned long long* dyn;      // nullable: [t + 1] rows by full-evaluation count, [t + 1] rows by end layer
+    int thr_ok;                   // range prediction on (one weight >= 0, one bias for every layer < t):
+    float thr_hi, thr_lo;         //   min >= thr_hi -> next layer all YMAX; max <= thr_lo -> next layer all 0
     int* n_const;                 // nullable: += rows that became constant
 };
 // 0 if N is not supported (T = N/32 threads must be 32..512)
