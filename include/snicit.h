@@ -264,7 +264,9 @@ snicit_status snicit_layer_profile(snicit_network* net, int32_t max, double* ms,
  * layers l < *n = min(max, L) (host pointers, any may be NULL; -1 = not recorded for that layer):
  *  pre_full[l]   (l < t) rows evaluated in full by pre-convergence layer l (the others alive are carried as
  *                constant rows, R26);
- *  pre_live[l]   (l < t) rows alive after layer l (not dropped as dead, R23);
+ *  pre_live[l]   (l < t) rows alive after layer l: not dropped as dead (R23) -- the row-resident kernel drops a
+ *                row at the layer by which it is proven zero, exactly (all outputs 0) or by the range rule
+ *                (R30: its range bounds Y(t) to zero), so this counts rows not yet proven zero;
  *  res_alive[l]  (l >= t) non-empty residue rows after post-convergence layer l (ne_idx);
  *  res_scalar[l] (l >= t) residue rows carried by a scalar from post layer l or earlier.
  * Recorded by the row-resident pre phase and the fused post mode; the per-layer pre path reports pre_full

@@ -205,8 +205,14 @@ struct PfLayerParam {
     int nu;
     int flags;  // cls | dead_next << 4 | ymax_fixed << 5 | ymax fixed for all later layers < t << 6
 };
+// range prediction (R30): thr_hi[k-1] = least m with out^k(m) == YMAX, thr_lo[k-1] = greatest m with
+// out^k(m) == 0, out(m) = sigma(chain(m) + b0) the layers' map of a constant row (host-evaluated with the
+// kernels' fma order); k > kPfThr uses entry kPfThr (thr_hi non-increasing and thr_lo non-decreasing in
+// k, so the shorter horizon is the stricter test)
+constexpr int kPfThr = 32;
 struct PreFusedParams {
     PreFusedArgs a;
+    float thr_hi[kPfThr], thr_lo[kPfThr];
     PfLayerParam L[kPfMaxLayers];
 };
 static_assert(sizeof(PreFusedParams) <= 32764, "kernel parameter space");
@@ -317,21 +323,30 @@ __global__ void __launch_bounds__(T, PfCfg<T>::kMinBlocks) pre_fused_kernel(cons
             const bool dead_next = (fl >> 4) & 1;
             if (!cst) {
                 float mn = __int_as_float(0x7f800000), mx = -__int_as_float(0x7f800000);
-                // range prediction (exact, one weight w0 >= 0 and one bias for every layer < t): every
-                // output of this layer is an fma chain monotone in each input, so if the previous layer's
-                // minimum already maps to YMAX (>= thr_hi) every output is YMAX, and if its maximum maps to 0
-                // (<= thr_lo) every output is 0 -- the row becomes constant without this layer's evaluation
+                // range prediction (R30, exact; one weight w0 >= 0 and one bias for every layer < t): each
+                // output is an fma chain + sigma, monotone in every input, so after k more layers every
+                // element lies in [out^k(min), out^k(max)] of the previous layer's range.  min >= thr_hi[k-1]
+                // with k = t - l: Y(t) is the constant row YMAX; max <= thr_lo[k-1]: Y(t) is zero (the row is
+                // dropped at layer l - 1 + k, the layer by which it is proven zero).
                 if (a.thr_ok && l > 0) {
+                    const int rem = a.t - l;
+                    const int kh = min(rem, kPfThr), kl = kh;
                     const float pmn = __uint_as_float(cmn), pmx = __uint_as_float(cmx);
-                    if (pmn >= a.thr_hi || pmx <= a.thr_lo) {
-                        v = pmn >= a.thr_hi ? a.ymax : 0.0f;
+                    if (pmn >= p.thr_hi[kh - 1]) {  // YMAX from layer l - 1 + kh on (a fixed point of the rest)
+                        v = a.ymax;
                         cst = true;
-                        if (v == 0.0f && a.drop && dead_next) {
+                        break;
+                    }
+                    if (pmx <= p.thr_lo[kl - 1]) {  // zero from layer l - 1 + kl on (b0 <= 0: absorbing)
+                        v = 0.0f;
+                        cst = true;
+                        if (a.drop && (kl == 1 ? dead_next : a.dead_t)) {
                             dead = true;
-                            lend = l;
+                            lend = l + kl - 1;
                             break;
                         }
-                        continue;
+                        if (kl == 1) continue;
+                        break;
                     }
                 }
                 const int cls = fl & 15;
@@ -499,14 +514,14 @@ cudaError_t launch_pre_fused(const PreFusedArgs& a, const PreFusedLayer* layers,
         if (all) p.L[l].flags |= 64;
         all = all && layers[l].ymax_fixed;
     }
-    // range prediction thresholds (one weight >= 0 and one bias for every layer < t; see the kernel)
+    // range prediction thresholds (R30; one weight >= 0 and one bias for every layer < t; see the kernel)
     p.a.thr_ok = 0;
     {
         bool same = layers[0].w0 >= 0.0f;
         for (int l = 1; l < a.t && same; ++l)
             same = memcmp(&layers[l].w0, &layers[0].w0, sizeof(float)) == 0 &&
                    memcmp(&layers[l].b0, &layers[0].b0, sizeof(float)) == 0;
-        if (same) {
+        if (same && a.const_skip) {
             const float w0 = layers[0].w0, b0 = layers[0].b0, ymax = a.ymax;
             auto out = [&](float m) {  // the kernels' chain for a constant input m, then sigma
                 float acc = 0.0f;
@@ -516,28 +531,37 @@ cudaError_t launch_pre_fused(const PreFusedArgs& a, const PreFusedLayer* layers,
             };
             auto bits = [](float f) { uint32_t u; memcpy(&u, &f, 4); return u; };
             auto flt = [](uint32_t u) { float f; memcpy(&f, &u, 4); return f; };
-            // thr_hi = least m in [0, ymax] with out(m) == ymax (out is monotone non-decreasing in m)
-            float hi = INFINITY, lo = -1.0f;
-            if (out(ymax) == ymax) {
-                uint32_t a0 = 0, a1 = bits(ymax);
-                while (a0 < a1) {
-                    const uint32_t mid = a0 + (a1 - a0) / 2;
-                    if (out(flt(mid)) == ymax) a1 = mid; else a0 = mid + 1;
+            // out is non-decreasing on [0, ymax], so {m : out^k(m) == ymax} = [thr_hi[k-1], ymax] with
+            // thr_hi[k-1] = least m with out(m) >= thr_hi[k-2] (thr_hi[-1] = ymax), and {m : out^k(m) == 0}
+            // = [0, thr_lo[k-1]] with thr_lo[k-1] = greatest m with out(m) <= thr_lo[k-2] (thr_lo[-1] = 0);
+            // bisection over the bit patterns of [0, ymax] (order-preserving for floats >= 0)
+            const bool hi_ok = out(ymax) == ymax, lo_ok = out(0.0f) == 0.0f;
+            float hprev = ymax, lprev = 0.0f;
+            for (int k = 0; k < kPfThr; ++k) {
+                float hi = INFINITY, lo = -1.0f;
+                if (hi_ok) {
+                    uint32_t a0 = 0, a1 = bits(ymax);
+                    while (a0 < a1) {
+                        const uint32_t mid = a0 + (a1 - a0) / 2;
+                        if (out(flt(mid)) >= hprev) a1 = mid; else a0 = mid + 1;
+                    }
+                    hi = flt(a0);
+                    hprev = hi;
                 }
-                hi = flt(a0);
-            }
-            // thr_lo = greatest m in [0, ymax] with out(m) == 0
-            if (out(0.0f) == 0.0f) {
-                uint32_t a0 = 0, a1 = bits(ymax);
-                while (a0 < a1) {
-                    const uint32_t mid = a0 + (a1 - a0 + 1) / 2;
-                    if (out(flt(mid)) == 0.0f) a0 = mid; else a1 = mid - 1;
+                if (lo_ok) {
+                    uint32_t a0 = 0, a1 = bits(ymax);
+                    while (a0 < a1) {
+                        const uint32_t mid = a0 + (a1 - a0 + 1) / 2;
+                        if (out(flt(mid)) <= lprev) a0 = mid; else a1 = mid - 1;
+                    }
+                    lo = flt(a0);
+                    lprev = lo;
                 }
-                lo = flt(a0);
+                p.thr_hi[k] = hi;
+                p.thr_lo[k] = lo;
             }
-            p.a.thr_hi = hi;
-            p.a.thr_lo = lo;
-            p.a.thr_ok = a.const_skip ? 1 : 0;
+            p.a.thr_ok = hi_ok || lo_ok;
+            p.a.dead_t = layers[a.t - 1].dead_next;
         }
     }
     bool wuni = true;

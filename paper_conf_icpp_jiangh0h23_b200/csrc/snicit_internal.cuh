@@ -295,8 +295,8 @@ struct PreFusedArgs {
     float* rval;
     unsigned long long* full_rl;  // nullable: += full (non-constant) row-layer evaluations
     unsigned long long* dyn;      // nullable: [t + 1] rows by full-evaluation count, [t + 1] rows by end layer
-    int thr_ok;                   // range prediction on (one weight >= 0, one bias for every layer < t):
-    float thr_hi, thr_lo;         //   min >= thr_hi -> next layer all YMAX; max <= thr_lo -> next layer all 0
+    int thr_ok;                   // range prediction on (R30; set by launch_pre_fused: one weight >= 0 and
+    int dead_t;                   //   one bias for every layer < t); dead_t = dead_ok[t]
     int* n_const;                 // nullable: += rows that became constant
 };
 // 0 if N is not supported (T = N/32 threads must be 32..512)

@@ -330,10 +330,91 @@ def test_dynamic_t_non_converging_net_goes_uncompressed():
 
 # ------------------------------------------------------------------------------ per-layer dynamics log
 
+def _range_thresholds(w0: float, b0: float, ymax: float, kmax: int = 32):
+    """R30: out(m) = sigma(32-tap chain of the constant m, + b0), the map of a constant row
+    through one uniform circulant layer.  thr_hi[k-1] = least m in [0, ymax] with out^k(m) == ymax,
+    thr_lo[k-1] = greatest m with out^k(m) == 0, found here by direct iteration of out^k over a bisection
+    of the float bit patterns (w0 is a power of two, so m*w0 is exact and the fp32 add is the fma)."""
+    f32 = np.float32
+
+    def out(m):
+        acc = f32(0.0)
+        for _ in range(32):
+            acc = f32(acc + f32(m) * f32(w0))
+        return float(min(max(f32(acc + f32(b0)), f32(0.0)), f32(ymax)))
+
+    def outk(m, k):
+        for _ in range(k):
+            m = out(m)
+        return m
+
+    top = int(np.array(ymax, np.float32).view(np.uint32))
+    flt = lambda u: float(np.array(u, np.uint32).view(np.float32))
+    hi, lo = [], []
+    for k in range(1, kmax + 1):
+        a0, a1 = 0, top
+        if outk(ymax, k) != ymax:
+            hi.append(np.inf)
+        else:
+            while a0 < a1:
+                mid = (a0 + a1) // 2
+                a0, a1 = (a0, mid) if outk(flt(mid), k) == ymax else (mid + 1, a1)
+            hi.append(flt(a0))
+        a0, a1 = 0, top
+        if outk(0.0, k) != 0.0:
+            lo.append(-1.0)
+        else:
+            while a0 < a1:
+                mid = (a0 + a1 + 1) // 2
+                a0, a1 = (mid, a1) if outk(flt(mid), k) == 0.0 else (a0, mid - 1)
+            lo.append(flt(a0))
+    return hi, lo
+
+
+def test_range_thresholds_monotone():
+    """The R30 horizon tables: thr_hi non-increasing, thr_lo non-decreasing in k, never overlapping."""
+    hi, lo = _range_thresholds(sdgc.SDGC_WEIGHT, sdgc.SDGC_BIAS[1024], sdgc.SDGC_YMAX, 12)
+    assert all(a >= b for a, b in zip(hi, hi[1:])) and all(a <= b for a, b in zip(lo, lo[1:]))
+    assert all(l_ < h for l_, h in zip(lo, hi))
+    # out(m) = 2m - 0.3 (32 taps of 1/16): one layer saturates from (32 + 0.3)/2, zeroes up to 0.15
+    assert abs(hi[0] - 16.15) < 1e-5 and abs(lo[0] - 0.15) < 1e-6
+
+
+@pytest.mark.parametrize("N,drop", [(1024, 1), (1024, 0), (4096, 1), (16384, 1)])
+def test_range_prediction_bit_exact(N, drop):
+    """R30 on rows built to sit near the repelling fixed point of out(m) = 2m + b0 (values b0/(1 - 2) +-
+    small noise): rows drift to YMAX or to zero over many layers, so the range test fires at long and short
+    horizons (k up to 32 and the clamped k > 32).  Uncompressed (t = L) and SNICIT (t < L) outputs equal
+    the oracle's bit for bit, and equal the run without the constant-row shortcut (no R26 / R30)."""
+    L, B = 48, 240 if N <= 4096 else 40
+    net = sdgc.gen_network(N, L, "radix")
+    fix = -sdgc.SDGC_BIAS[N]
+    rs = np.random.RandomState(N + drop)
+    base = rs.uniform(fix - 0.05, fix + 0.05, size=(B, 1))
+    Y0 = (base + rs.uniform(-0.03, 0.03, size=(B, N))).clip(0, None).astype(np.float32)
+    Y0[::5] = sdgc.gen_inputs(N, B)[::5]
+    plain = oracle.layers_f32(net, Y0)
+    with SnicitNetwork.from_network(net) as g:
+        g.set_stream(torch.cuda.current_stream())
+        Y1, c1, st1 = _infer(g, Y0, L, drop_dead_rows=drop)
+        Y2, c2, st2 = _infer(g, Y0, L, drop_dead_rows=drop, pre_fused=2)
+        Y3, c3, st3 = _infer(g, Y0, 40, drop_dead_rows=drop)
+        Y4, c4, st4 = _infer(g, Y0, 40, drop_dead_rows=drop, pre_fused=0)
+    assert st1["pre_fused"] == 1 and st2["pre_fused"] == 1
+    assert np.array_equal(Y1, plain) and np.array_equal(Y2, plain)
+    assert st1["pre_full_rows"] < st2["pre_full_rows"]
+    assert np.array_equal(c1, oracle.categories(plain)) and np.array_equal(c3, c1)
+    assert np.array_equal(Y3, Y4) and np.array_equal(c3, c4)
+    assert np.allclose(Y3, plain, atol=ATOL, rtol=RTOL)
+
+
 def test_dynamics_log(tmp_path):
-    """snicit_dynamics (SURVEY 5 per-layer log): pre_live[l] = rows with a non-zero output after layer l,
-    pre_full[l] = rows not yet constant before layer l (both counted on the oracle's layer-by-layer rows);
-    res_alive ends at stats.residual_final and never increases (zero residues are absorbing, R16)."""
+    """snicit_dynamics (SURVEY 5 per-layer log) of the row-resident kernel, modelled row by row on the
+    oracle's layer-by-layer rows: pre_full[l] = rows evaluated in full by layer l (not yet constant, R26,
+    and not predicted by the range rule, R30: before layer l >= 1 with k = min(t - l, 32), min of Y(l) >=
+    thr_hi[k-1] -> YMAX at t, max <= thr_lo[k-1] -> zero at t, dropped at layer l - 1 + k); pre_live[l] =
+    rows not dropped after layer l (all-zero rows drop at once, R23); res_alive ends at
+    stats.residual_final and never increases (zero residues are absorbing, R16)."""
     N, L, B, t = 1024, 40, 600, 6
     net = sdgc.gen_network(N, L, "radix")
     Y0 = sdgc.gen_inputs(N, B)
@@ -343,17 +424,40 @@ def test_dynamics_log(tmp_path):
         d = g.dynamics()
         st = g.stats()
         nlines = g.write_dynamics_jsonl(str(tmp_path / "dyn.jsonl"))
+    hi, lo = _range_thresholds(sdgc.SDGC_WEIGHT, sdgc.SDGC_BIAS[N], sdgc.SDGC_YMAX)
     y = Y0.copy()
-    const_before = np.zeros(B, bool)  # row constant after the previous layer (carried by a scalar from then on)
-    alive = np.ones(B, bool)
+    mn, mx, alleq, allz = [], [], [], []
     for l in range(t):
-        full = alive & ~const_before
-        assert d["pre_full"][l] == int(full.sum()), l
         y = oracle.layers_f32(net, y, l, l + 1)
-        nz = (y != 0).any(1)
-        alive = alive & nz
-        assert d["pre_live"][l] == int(alive.sum()), l
-        const_before = const_before | (alive & (y == y[:, :1]).all(1))
+        mn.append(y.min(1))
+        mx.append(y.max(1))
+        alleq.append((y == y[:, :1]).all(1))
+        allz.append(~(y != 0).any(1))
+    full = np.zeros(B, int)
+    lend = np.full(B, t)
+    n_pred = 0
+    for r in range(B):
+        cst = False
+        for l in range(t):
+            if not cst:
+                if l > 0:
+                    k = min(t - l, 32)
+                    if mn[l - 1][r] >= hi[k - 1]:
+                        n_pred += 1
+                        break
+                    if mx[l - 1][r] <= lo[k - 1]:
+                        n_pred += 1
+                        lend[r] = l + k - 1
+                        break
+                full[r] += 1
+                cst = bool(alleq[l][r])
+            if allz[l][r]:
+                lend[r] = l
+                break
+    assert n_pred > 0  # the workload exercises R30
+    for l in range(t):
+        assert d["pre_full"][l] == int((full > l).sum()), l
+        assert d["pre_live"][l] == int((lend > l).sum()), l
     ra = d["res_alive"][t:]
     assert ra[-1] == st["residual_final"] and np.all(np.diff(ra) <= 0) and ra[0] <= st["residual_at_t"]
     assert np.all(d["pre_full"][t:] == -1) and np.all(d["res_alive"][:t] == -1)
