@@ -278,6 +278,8 @@ __global__ void __launch_bounds__(T, PfCfg<T>::kMinBlocks) pre_fused_kernel(cons
     uint32_t ph = 0;                    // phase bit of bar[0], bar[1]
     if (NB == 3 && tid == 0 && pos < count) issue_load(pos, buf, &bar[0], 0);
     int np = 0;  // tid 0: the next row's list position
+    // NB == 3: the position after that, claimed one row ahead so the atomic's latency is never waited on
+    int nq = (NB == 3 && tid == 0) ? atomicAdd(a.work, 1) : 0;
     for (int k = 0; pos < count; ++k) {
         const int row = __ldg(a.rows + pos);
         if (tid == 0) {
@@ -285,7 +287,12 @@ __global__ void __launch_bounds__(T, PfCfg<T>::kMinBlocks) pre_fused_kernel(cons
                 bulk_wait_read0();  // the previous row's TMA store has finished reading its buffer
                 issue_load(pos, buf, &bar[k & 1], k & 1);
             }
-            np = atomicAdd(a.work, 1);  // next row (NB == 2: consumed at the row end, latency hidden)
+            if (NB == 3) {
+                np = nq;
+                nq = atomicAdd(a.work, 1);  // consumed at the next row's start
+            } else {
+                np = atomicAdd(a.work, 1);  // next row (consumed at the row end, latency hidden)
+            }
             if (NB == 3) {
                 s_pos[2 + (k & 1)] = np;
                 if (np < count) {  // load it now, behind this row's compute
