@@ -70,9 +70,10 @@ def parse(argv=None):
     p.add_argument("--no-residue", action="store_true", help="skip the residue-regime study (C2, t = 10)")
     p.add_argument("--no-general", action="store_true", help="skip the general-CSC study (C2 perm)")
     p.add_argument("--residue-t", type=int, default=10)
-    p.add_argument("--pre-fused", type=int, default=1, choices=[0, 1, 2, 3, 4, 5],
+    p.add_argument("--pre-fused", type=int, default=1, choices=[0, 1, 2, 3, 4, 5, 6],
                    help="options.pre_fused: 1 = row-resident pre phase (default), 2 = without the constant-row "
-                        "shortcut, 4 = rows split over a thread-block cluster (N >= 16384), 0 = one launch per layer")
+                        "shortcut, 6 = without the range prediction (R30), 4 = rows split over a thread-block "
+                        "cluster (N >= 16384), 0 = one launch per layer")
     p.add_argument("--no-variants", action="store_true", help="skip the pre_fused = 2 / 0 roofline variants")
     p.add_argument("--cpu-seconds", type=float, default=15.0, help="target CPU work of the oracle sample")
     p.add_argument("--quick", action="store_true", help="value only (no e2e/uncompressed/variants/studies)")
@@ -625,6 +626,11 @@ def run_snicit(args):
                 if st2["pre_fused"] and len(pm2):
                     r2 = alu_roof(pm2, pb2, st2)
                     roof["no_const_skip"] = {k: r2[k] for k in ("achieved", "frac", "avg_launch_ms",
+                                                                "full_row_layers")}
+                st6, pm6, pb6 = profile_pre(6)
+                if st6["pre_fused"] and len(pm6):
+                    r6 = alu_roof(pm6, pb6, st6)
+                    roof["no_range_pred"] = {k: r6[k] for k in ("achieved", "frac", "avg_launch_ms",
                                                                 "full_row_layers")}
                 st0_, pm0, pb0 = profile_pre(0)
                 if len(pm0):

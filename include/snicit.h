@@ -99,6 +99,9 @@ typedef struct {
                                5 = as 1 with the row stored as pairs (y[p], y[p + N/2]) read by 8-byte
                                loads (kernels_pre_pair.cu).  4 and 5 are measured alternatives (slower
                                than 1 on B200), kept selectable and parity-tested.
+                               6 = as 1 without the range prediction (R30: a row whose output range
+                               bounds Y(t) to the constant row YMAX or to zero leaves early; on in 1), for
+                               measurement.
                                Used when every layer < t is circulant
                                with 32 taps, uniform weight and uniform bias, and N/32 is one of
                                32..512 (N = 1024..16384; 4: the cluster form supports every stride);
@@ -108,7 +111,9 @@ typedef struct {
                                whose outputs are all equal leaves the active list and is carried by one
                                scalar fma chain per layer, written once at t (R26, exact; column-streaming
                                and segmented layer kernels, every layer < t circulant with uniform weight
-                               and bias); 0 = every live row through every layer */
+                               and bias), and with every layer < t sharing one weight and bias a row
+                               whose output range bounds Y(t) to YMAX or to zero leaves at once (R30,
+                               exact); 2 = as 1 without R30; 0 = every live row through every layer */
     int32_t res_sparse;     /* fused post mode, circulant post layers: 1 = a residue row with few non-zero
                                entries propagates only them (the outputs they touch are evaluated, every
                                other output of Eq. 5 is exactly 0; north_star "only the nonzero residual

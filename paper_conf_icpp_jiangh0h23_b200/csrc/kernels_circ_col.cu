@@ -76,11 +76,11 @@ __global__ void __launch_bounds__(kColThreads, 2) layer_circ_col_kernel(LayerArg
     };
     // constant-row mode (a.cmin, R26): rows whose outputs are all equal leave the list for the
     // constant list (row, value, layer); the warps of a row combine (min, max) at cmin/cmax[pos]
-    auto push_const = [&](int row, float v) {
+    auto push_const = [&](int row, float v, int layer) {
         const int p = atomicAdd(a.ccount, 1);
         a.clist[p] = row;
         a.cval[p] = v;
-        a.clayer[p] = a.layer;
+        a.clayer[p] = layer;
     };
     // Constant-row mode walks the units row-major per warp (all G column groups of a row in one warp,
     // see nextu), so a row's output range is combined in registers and decided by that warp alone.
@@ -102,7 +102,11 @@ __global__ void __launch_bounds__(kColThreads, 2) layer_circ_col_kernel(LayerArg
             const int row = (int)(base / (size_t)N);
             if (umn == umx) {
                 const float v = __uint_as_float(umn);
-                if (lane == 0 && !(v == 0.0f && a.dead_drop)) push_const(row, v);
+                if (lane == 0 && !(v == 0.0f && a.dead_drop)) push_const(row, v, a.layer);
+            } else if (__uint_as_float(umn) >= a.thr_hi) {  // range prediction (R30): YMAX at t
+                if (lane == 0) push_const(row, ymax, a.thr_layer);
+            } else if (__uint_as_float(umx) <= a.thr_lo) {  // R30: zero at t (dead, or a constant zero row)
+                if (lane == 0 && !a.thr_dead) push_const(row, 0.0f, a.thr_layer);
             } else {
                 if (lane == nbuf) abuf = row;
                 if (++nbuf == 32) flush();

@@ -9,6 +9,9 @@
 // Exact: results are bit-identical to the full evaluation (tested).
 #include <cuda_runtime.h>
 
+#include <cmath>
+#include <cstring>
+
 #include "snicit_internal.cuh"
 
 namespace snicit {
@@ -18,13 +21,14 @@ namespace snicit {
 // (unordered, R24; warp-aggregated appends).
 __global__ void const_split_kernel(const int* list_in, const int* count_in, unsigned* cmin, unsigned* cmax,
                                    int* list_out, int* count_out, int* clist, float* cval, int* clayer, int* ccount,
-                                   int layer, int dead_drop) {
+                                   int layer, int dead_drop, float thr_hi, float thr_lo, int thr_layer, int thr_dead,
+                                   float ymax) {
     const int n = *count_in;
     const int lane = threadIdx.x & 31;
     for (int i0 = blockIdx.x * blockDim.x; i0 < n; i0 += gridDim.x * blockDim.x) {
         const int i = i0 + threadIdx.x;
         bool keep = false, cst = false;
-        int row = 0;
+        int row = 0, cl = layer;
         float v = 0.0f;
         if (i < n) {
             row = list_in[i];
@@ -34,6 +38,13 @@ __global__ void const_split_kernel(const int* list_in, const int* count_in, unsi
             if (umn == umx) {
                 v = __uint_as_float(umn);
                 cst = !(v == 0.0f && dead_drop);
+            } else if (__uint_as_float(umn) >= thr_hi) {  // R30: YMAX at t
+                v = ymax;
+                cst = true;
+                cl = thr_layer;
+            } else if (__uint_as_float(umx) <= thr_lo) {  // R30: zero at t
+                cst = !thr_dead;
+                cl = thr_layer;
             } else {
                 keep = true;
             }
@@ -47,19 +58,65 @@ __global__ void const_split_kernel(const int* list_in, const int* count_in, unsi
             const int p = atomicAdd(ccount, 1);
             clist[p] = row;
             cval[p] = v;
-            clayer[p] = layer;
+            clayer[p] = cl;
         }
     }
 }
 
 cudaError_t launch_const_split(const int* list_in, const int* count_in, unsigned* cmin, unsigned* cmax, int* list_out,
                                int* count_out, int* clist, float* cval, int* clayer, int* ccount, int layer,
-                               int dead_drop, int max_rows, cudaStream_t st) {
+                               int dead_drop, int max_rows, cudaStream_t st, const LayerArgs* thr) {
     int grid = max_rows > 0 ? (max_rows + 255) / 256 : 1;
     if (grid > 2048) grid = 2048;
     const_split_kernel<<<grid, 256, 0, st>>>(list_in, count_in, cmin, cmax, list_out, count_out, clist, cval, clayer,
-                                             ccount, layer, dead_drop);
+                                             ccount, layer, dead_drop, thr ? thr->thr_hi : INFINITY,
+                                             thr ? thr->thr_lo : -1.0f, thr ? thr->thr_layer : layer,
+                                             thr ? thr->thr_dead : 0, thr ? thr->ymax : 0.0f);
     return cudaGetLastError();
+}
+
+bool range_tables(const PreFusedLayer* layers, int t, float ymax, float* hi, float* lo) {
+    if (t < 1 || !(layers[0].w0 >= 0.0f)) return false;
+    for (int l = 1; l < t; ++l)
+        if (memcmp(&layers[l].w0, &layers[0].w0, sizeof(float)) != 0 ||
+            memcmp(&layers[l].b0, &layers[0].b0, sizeof(float)) != 0)
+            return false;
+    const float w0 = layers[0].w0, b0 = layers[0].b0;
+    auto out = [&](float m) {  // the kernels' chain for a constant input m (acc = fma(m, w0, acc) x 32), + b0, sigma
+        float acc = 0.0f;
+        for (int n = 0; n < 32; ++n) acc = std::fma(m, w0, acc);
+        const float z = acc + b0;
+        return std::fmin(std::fmax(z, 0.0f), ymax);
+    };
+    auto bits = [](float f) { uint32_t u; memcpy(&u, &f, 4); return u; };
+    auto flt = [](uint32_t u) { float f; memcpy(&f, &u, 4); return f; };
+    // out is non-decreasing on [0, ymax], so {m : out^k(m) == ymax} = [hi[k-1], ymax] with hi[k-1] = least m
+    // with out(m) >= hi[k-2] (hi[-1] = ymax), and {m : out^k(m) == 0} = [0, lo[k-1]] with lo[k-1] = greatest
+    // m with out(m) <= lo[k-2] (lo[-1] = 0); bisection over the bit patterns of [0, ymax] (order-preserving
+    // for floats >= 0)
+    const bool hi_ok = out(ymax) == ymax, lo_ok = out(0.0f) == 0.0f;
+    float hprev = ymax, lprev = 0.0f;
+    for (int k = 0; k < kRangeK; ++k) {
+        hi[k] = INFINITY;
+        lo[k] = -1.0f;
+        if (hi_ok) {
+            uint32_t a0 = 0, a1 = bits(ymax);
+            while (a0 < a1) {
+                const uint32_t mid = a0 + (a1 - a0) / 2;
+                if (out(flt(mid)) >= hprev) a1 = mid; else a0 = mid + 1;
+            }
+            hi[k] = hprev = flt(a0);
+        }
+        if (lo_ok) {
+            uint32_t a0 = 0, a1 = bits(ymax);
+            while (a0 < a1) {
+                const uint32_t mid = a0 + (a1 - a0 + 1) / 2;
+                if (out(flt(mid)) <= lprev) a0 = mid; else a1 = mid - 1;
+            }
+            lo[k] = lprev = flt(a0);
+        }
+    }
+    return hi_ok || lo_ok;
 }
 
 // At t: each constant row (value v after layer clayer) through layers clayer + 1 .. t - 1 by one scalar

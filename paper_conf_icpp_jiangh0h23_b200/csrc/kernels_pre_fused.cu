@@ -209,7 +209,7 @@ struct PfLayerParam {
 // out^k(m) == 0, out(m) = sigma(chain(m) + b0) the layers' map of a constant row (host-evaluated with the
 // kernels' fma order); k > kPfThr uses entry kPfThr (thr_hi non-increasing and thr_lo non-decreasing in
 // k, so the shorter horizon is the stricter test)
-constexpr int kPfThr = 32;
+constexpr int kPfThr = kRangeK;
 struct PreFusedParams {
     PreFusedArgs a;
     float thr_hi[kPfThr], thr_lo[kPfThr];
@@ -521,56 +521,9 @@ cudaError_t launch_pre_fused(const PreFusedArgs& a, const PreFusedLayer* layers,
         if (all) p.L[l].flags |= 64;
         all = all && layers[l].ymax_fixed;
     }
-    // range prediction thresholds (R30; one weight >= 0 and one bias for every layer < t; see the kernel)
-    p.a.thr_ok = 0;
-    {
-        bool same = layers[0].w0 >= 0.0f;
-        for (int l = 1; l < a.t && same; ++l)
-            same = memcmp(&layers[l].w0, &layers[0].w0, sizeof(float)) == 0 &&
-                   memcmp(&layers[l].b0, &layers[0].b0, sizeof(float)) == 0;
-        if (same && a.const_skip) {
-            const float w0 = layers[0].w0, b0 = layers[0].b0, ymax = a.ymax;
-            auto out = [&](float m) {  // the kernels' chain for a constant input m, then sigma
-                float acc = 0.0f;
-                for (int n = 0; n < 32; ++n) acc = std::fma(m, w0, acc);
-                const float z = acc + b0;
-                return std::fmin(std::fmax(z, 0.0f), ymax);
-            };
-            auto bits = [](float f) { uint32_t u; memcpy(&u, &f, 4); return u; };
-            auto flt = [](uint32_t u) { float f; memcpy(&f, &u, 4); return f; };
-            // out is non-decreasing on [0, ymax], so {m : out^k(m) == ymax} = [thr_hi[k-1], ymax] with
-            // thr_hi[k-1] = least m with out(m) >= thr_hi[k-2] (thr_hi[-1] = ymax), and {m : out^k(m) == 0}
-            // = [0, thr_lo[k-1]] with thr_lo[k-1] = greatest m with out(m) <= thr_lo[k-2] (thr_lo[-1] = 0);
-            // bisection over the bit patterns of [0, ymax] (order-preserving for floats >= 0)
-            const bool hi_ok = out(ymax) == ymax, lo_ok = out(0.0f) == 0.0f;
-            float hprev = ymax, lprev = 0.0f;
-            for (int k = 0; k < kPfThr; ++k) {
-                float hi = INFINITY, lo = -1.0f;
-                if (hi_ok) {
-                    uint32_t a0 = 0, a1 = bits(ymax);
-                    while (a0 < a1) {
-                        const uint32_t mid = a0 + (a1 - a0) / 2;
-                        if (out(flt(mid)) >= hprev) a1 = mid; else a0 = mid + 1;
-                    }
-                    hi = flt(a0);
-                    hprev = hi;
-                }
-                if (lo_ok) {
-                    uint32_t a0 = 0, a1 = bits(ymax);
-                    while (a0 < a1) {
-                        const uint32_t mid = a0 + (a1 - a0 + 1) / 2;
-                        if (out(flt(mid)) <= lprev) a0 = mid; else a1 = mid - 1;
-                    }
-                    lo = flt(a0);
-                    lprev = lo;
-                }
-                p.thr_hi[k] = hi;
-                p.thr_lo[k] = lo;
-            }
-            p.a.thr_ok = hi_ok || lo_ok;
-            p.a.dead_t = layers[a.t - 1].dead_next;
-        }
-    }
+    // range prediction horizon tables (R30, kernels_const.cu)
+    p.a.thr_ok = a.const_skip && a.range_pred && range_tables(layers, a.t, a.ymax, p.thr_hi, p.thr_lo);
+    p.a.dead_t = layers[a.t - 1].dead_next;
     bool wuni = true;
     for (int l = 1; l < a.t; ++l) wuni = wuni && memcmp(&p.L[l].w0, &p.L[0].w0, sizeof(float)) == 0;
     switch (pre_fused_threads(a.N)) {

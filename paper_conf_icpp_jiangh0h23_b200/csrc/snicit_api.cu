@@ -657,6 +657,8 @@ int32_t snicit_layer_is_circulant(const snicit_network* net, int32_t l) {
 static LayerArgs layer_args(snicit_network* net, int l, bool force_ell) {
     const LayerPlan& pl = net->plan[l];
     LayerArgs a{};
+    a.thr_hi = INFINITY;  // range prediction (R30) off unless the constant-row pre path turns it on
+    a.thr_lo = -1.0f;
     a.N = net->N;
     a.bias = net->bias_d.p + (size_t)l * net->N;
     a.ymax = net->ymax;
@@ -982,8 +984,8 @@ static snicit_status infer_core(snicit_network* net, const float* y0, int64_t ba
         return fail(SNICIT_E_INVALID_ARG, "bad eta/eps/prune_eps");
     if (opt.kernel < 0 || opt.kernel > SNICIT_KERNEL_CIRC_SMEM) return fail(SNICIT_E_INVALID_ARG, "bad kernel option");
     if (opt.post_mode < 0 || opt.post_mode > 1) return fail(SNICIT_E_INVALID_ARG, "bad post_mode");
-    if (opt.pre_fused < 0 || opt.pre_fused > 5) return fail(SNICIT_E_INVALID_ARG, "bad pre_fused");
-    if (opt.pre_const < 0 || opt.pre_const > 1) return fail(SNICIT_E_INVALID_ARG, "bad pre_const");
+    if (opt.pre_fused < 0 || opt.pre_fused > 6) return fail(SNICIT_E_INVALID_ARG, "bad pre_fused");
+    if (opt.pre_const < 0 || opt.pre_const > 2) return fail(SNICIT_E_INVALID_ARG, "bad pre_const");
     if (opt.res_sparse < 0 || opt.res_sparse > 1) return fail(SNICIT_E_INVALID_ARG, "bad res_sparse");
     if (opt.dyn_t < 0 || opt.dyn_t > 1) return fail(SNICIT_E_INVALID_ARG, "bad dyn_t");
     if (opt.kernel == SNICIT_KERNEL_ELL && !net->has_ell)
@@ -1100,6 +1102,7 @@ static snicit_status infer_core(snicit_network* net, const float* y0, int64_t ba
         pa.ymax = net->ymax;
         pa.drop = drop ? 1 : 0;
         pa.const_skip = opt.pre_fused != 2 ? 1 : 0;
+        pa.range_pred = opt.pre_fused != 6 ? 1 : 0;  // R30 (6: R26 alone, for measurement)
         pa.gen_str = pf_gen;
         pa.yin = cur;
         pa.ybits = y0_mode == 3 ? bits : nullptr;
@@ -1149,6 +1152,9 @@ static snicit_status infer_core(snicit_network* net, const float* y0, int64_t ba
                ell_const_ok(net, l, opt.kernel);
     net->last_pre_const = pcst;
     if (pcst) CUDA_TRY(cudaMemsetAsync(cnt + CNT_CCOUNT, 0, sizeof(int), st));
+    // range prediction (R30) in constant-row mode: horizon tables when layers 0..t-1 share weight and bias
+    float thr_hi[kRangeK], thr_lo[kRangeK];
+    const bool thr_ok = pcst && opt.pre_const != 2 && range_tables(net->pf_layers_h.data(), tt, net->ymax, thr_hi, thr_lo);
     for (int l = 0; l < tt && !pf; ++l) {
         // exact dead-row compaction (R23) fused into the layer: rows with a non-zero output are
         // appended (unordered) to the other list; the append counter of the NEXT dropping layer is
@@ -1186,6 +1192,13 @@ static snicit_status infer_core(snicit_network* net, const float* y0, int64_t ba
             a.ccount = cnt + CNT_CCOUNT;
             a.layer = l;
             a.dead_drop = dead_now ? 1 : 0;
+            if (thr_ok && l + 1 < tt) {  // k = t - 1 - l layers follow this one
+                const int k = std::min(tt - 1 - l, kRangeK);
+                a.thr_hi = thr_hi[k - 1];
+                a.thr_lo = thr_lo[k - 1];
+                a.thr_layer = tt - 1;
+                a.thr_dead = (drop && net->dead_ok[tt]) ? 1 : 0;
+            }
         }
         CUDA_TRY(run_layer(net, l, opt.kernel, MODE_PLAIN, a, R));
         if (prof) CUDA_TRY(cudaEventRecord(net->lev[2 * l + 1], st));
@@ -1193,7 +1206,7 @@ static snicit_status infer_core(snicit_network* net, const float* y0, int64_t ba
         if (pcst && seg) {
             CUDA_TRY(launch_const_split(lists[li], cnt + live_ctr[ci], net->cmin.p, net->cmax.p, lists[li ^ 1],
                                         cnt + live_ctr[(ci + 1) % 3], net->clist.p, net->cval.p, net->clayer.p,
-                                        cnt + CNT_CCOUNT, l, dead_now ? 1 : 0, R, st));
+                                        cnt + CNT_CCOUNT, l, dead_now ? 1 : 0, R, st, &a));
             CUDA_TRY(cudaMemsetAsync(cnt + live_ctr[(ci + 2) % 3], 0, sizeof(int), st));
             launches += 1;
         } else if (drop_now && seg) {

@@ -146,6 +146,11 @@ struct LayerArgs {
     int* ccount;
     int layer;              // index of this layer
     int dead_drop;          // an all-zero row after this layer is dead (drop && dead_ok[l + 1])
+    // range prediction (R30) in constant-row mode: a row whose output range after this layer has
+    // min >= thr_hi is the constant row YMAX at t, max <= thr_lo the zero row at t (dead when thr_dead);
+    // it leaves with layer index thr_layer = t - 1.  thr_hi = +inf, thr_lo = -1: off
+    float thr_hi, thr_lo;
+    int thr_layer, thr_dead;
 };
 
 struct LayerPlan {
@@ -272,6 +277,15 @@ struct PreFusedLayer {
                     // the host with the kernel's fma order)
     int pad[2];
 };
+// range prediction (R30, exact): when layers 0..t-1 share one weight w0 >= 0 and one bias b0, every output
+// is a monotone function of every input, so after k more layers each element of a row lies in
+// [out^k(min), out^k(max)], out(m) = sigma(chain(m) + b0) the map of a constant row (host-evaluated with
+// the kernels' fma order).  hi[k-1] = least m with out^k(m) == YMAX (+inf if none), lo[k-1] = greatest m
+// with out^k(m) == 0 (-1 if none), k = 1..kRangeK (longer horizons use entry kRangeK: hi is
+// non-increasing and lo non-decreasing in k, so the shorter horizon is the stricter test).  Returns
+// false (tables off) when the layers differ or w0 < 0.
+constexpr int kRangeK = 32;
+bool range_tables(const PreFusedLayer* layers, int t, float ymax, float* hi, float* lo);
 struct PreFusedArgs {
     int N, t, H;     // H: circular halo (floats) of every staged row, >= 64 and >= 31*nu of STR layers
     float ymax;
@@ -295,6 +309,7 @@ struct PreFusedArgs {
     float* rval;
     unsigned long long* full_rl;  // nullable: += full (non-constant) row-layer evaluations
     unsigned long long* dyn;      // nullable: [t + 1] rows by full-evaluation count, [t + 1] rows by end layer
+    int range_pred;               // caller: allow the range prediction (R30)
     int thr_ok;                   // range prediction on (R30; set by launch_pre_fused: one weight >= 0 and
     int dead_t;                   //   one bias for every layer < t); dead_t = dead_ok[t]
     int* n_const;                 // nullable: += rows that became constant
@@ -322,7 +337,7 @@ cudaError_t launch_pre_cluster(const PreFusedArgs& a, const PreFusedLayer* layer
 // kernels_const.cu: constant rows in the per-layer pre-convergence path (R26)
 cudaError_t launch_const_split(const int* list_in, const int* count_in, unsigned* cmin, unsigned* cmax, int* list_out,
                                int* count_out, int* clist, float* cval, int* clayer, int* ccount, int layer,
-                               int dead_drop, int max_rows, cudaStream_t st);
+                               int dead_drop, int max_rows, cudaStream_t st, const LayerArgs* thr = nullptr);
 cudaError_t launch_const_finish(const int* clist, const float* cval, const int* clayer, const int* ccount,
                                 const PreFusedLayer* layers, int t, float ymax, int drop, int N, float* y, int* live,
                                 int* live_count, int num_sms, cudaStream_t st, uint8_t* rconst = nullptr,

@@ -467,14 +467,15 @@ def test_pre_fused_positive_bias_and_fallbacks():
 @pytest.mark.parametrize("drop", [1, 0])
 def test_pre_const_per_layer(N, L, B, drop):
     """Per-layer pre-convergence path (segmented + column-streaming kernels) in constant-row mode
-    (R26: rows whose outputs are all equal leave the list and are carried by a scalar chain) ==
-    the same path without it == the oracle, bit for bit: uncompressed (t = L) and SNICIT (t = 4)."""
+    (R26: rows whose outputs are all equal leave the list and are carried by a scalar chain; with R30,
+    rows whose range bounds Y(t) leave too) == R26 alone == the path without either == the oracle, bit
+    for bit: uncompressed (t = L) and SNICIT (t = 4)."""
     net = sdgc.gen_network(N, L, "radix")
     Y0 = _pf_inputs(N, B, 3)
     plain = oracle.layers_f32(net, Y0)
     for t in (L, 4):
         res = {}
-        for pc in (1, 0):
+        for pc in (1, 2, 0):  # 2: R26 without the range prediction (R30)
             Y, cats, st, _ = run_gpu(net, Y0, t=t, drop_dead_rows=drop, pre_fused=0, pre_const=pc)
             assert st["pre_fused"] == 0
             res[pc] = (Y, cats, st)
@@ -482,5 +483,6 @@ def test_pre_const_per_layer(N, L, B, drop):
             if t == L:
                 assert np.array_equal(Y, plain), f"pre_const={pc}"
         assert np.array_equal(res[1][0], res[0][0]) and np.array_equal(res[1][1], res[0][1])
+        assert np.array_equal(res[2][0], res[0][0]) and np.array_equal(res[2][1], res[0][1])
         assert res[1][2]["live_at_t"] == res[0][2]["live_at_t"]
         assert res[1][2]["pre_const_rows"] > 0 and res[0][2]["pre_const_rows"] == 0

@@ -380,13 +380,14 @@ def test_range_thresholds_monotone():
     assert abs(hi[0] - 16.15) < 1e-5 and abs(lo[0] - 0.15) < 1e-6
 
 
-@pytest.mark.parametrize("N,drop", [(1024, 1), (1024, 0), (4096, 1), (16384, 1)])
+@pytest.mark.parametrize("N,drop", [(1024, 1), (1024, 0), (4096, 1), (16384, 1), (65536, 1)])
 def test_range_prediction_bit_exact(N, drop):
-    """R30 on rows built to sit near the repelling fixed point of out(m) = 2m + b0 (values b0/(1 - 2) +-
-    small noise): rows drift to YMAX or to zero over many layers, so the range test fires at long and short
-    horizons (k up to 32 and the clamped k > 32).  Uncompressed (t = L) and SNICIT (t < L) outputs equal
-    the oracle's bit for bit, and equal the run without the constant-row shortcut (no R26 / R30)."""
-    L, B = 48, 240 if N <= 4096 else 40
+    """R30 on rows built to sit near the repelling fixed point of out(m) = 2m + b0 (values -b0 +- small
+    noise): rows drift to YMAX or to zero over many layers, so the range test fires at long and short
+    horizons (k up to 32 and the clamped k > 32).  Uncompressed (t = L) outputs equal the oracle's bit for
+    bit in the row-resident kernel (pre_fused 1, and 6 = without R30) and in the per-layer constant-row
+    path (pre_const 1, and 2 = without R30); SNICIT (t < L) outputs agree across the pre paths."""
+    L, B = 48, (240 if N <= 4096 else (40 if N <= 16384 else 8))
     net = sdgc.gen_network(N, L, "radix")
     fix = -sdgc.SDGC_BIAS[N]
     rs = np.random.RandomState(N + drop)
@@ -394,18 +395,25 @@ def test_range_prediction_bit_exact(N, drop):
     Y0 = (base + rs.uniform(-0.03, 0.03, size=(B, N))).clip(0, None).astype(np.float32)
     Y0[::5] = sdgc.gen_inputs(N, B)[::5]
     plain = oracle.layers_f32(net, Y0)
+    want_c = oracle.categories(plain)
+    runs = {}
     with SnicitNetwork.from_network(net) as g:
         g.set_stream(torch.cuda.current_stream())
-        Y1, c1, st1 = _infer(g, Y0, L, drop_dead_rows=drop)
-        Y2, c2, st2 = _infer(g, Y0, L, drop_dead_rows=drop, pre_fused=2)
-        Y3, c3, st3 = _infer(g, Y0, 40, drop_dead_rows=drop)
-        Y4, c4, st4 = _infer(g, Y0, 40, drop_dead_rows=drop, pre_fused=0)
-    assert st1["pre_fused"] == 1 and st2["pre_fused"] == 1
-    assert np.array_equal(Y1, plain) and np.array_equal(Y2, plain)
-    assert st1["pre_full_rows"] < st2["pre_full_rows"]
-    assert np.array_equal(c1, oracle.categories(plain)) and np.array_equal(c3, c1)
-    assert np.array_equal(Y3, Y4) and np.array_equal(c3, c4)
-    assert np.allclose(Y3, plain, atol=ATOL, rtol=RTOL)
+        modes = [("pl1", dict(pre_fused=0, pre_const=1)), ("pl2", dict(pre_fused=0, pre_const=2))]
+        if N <= 16384:
+            modes += [("pf1", dict(pre_fused=1)), ("pf6", dict(pre_fused=6))]
+        for name, kw in modes:
+            runs[name] = _infer(g, Y0, L, drop_dead_rows=drop, **kw)
+            assert np.array_equal(runs[name][0], plain), name
+            assert np.array_equal(runs[name][1], want_c), name
+            runs[name + "_t"] = _infer(g, Y0, 40, drop_dead_rows=drop, **kw)
+    for name, _ in modes:
+        assert np.array_equal(runs[name + "_t"][0], runs["pl2_t"][0]), name
+        assert np.array_equal(runs[name + "_t"][1], runs["pl2_t"][1]), name
+    assert np.allclose(runs["pl1_t"][0], plain, atol=ATOL, rtol=RTOL)
+    if N <= 16384:
+        assert runs["pf1"][2]["pre_fused"] == 1 and runs["pf6"][2]["pre_fused"] == 1
+        assert runs["pf1"][2]["pre_full_rows"] < runs["pf6"][2]["pre_full_rows"]
 
 
 def test_dynamics_log(tmp_path):
