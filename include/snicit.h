@@ -295,6 +295,13 @@ snicit_status snicit_debug_clustering(snicit_network* net, int32_t* cent, int32_
 snicit_status snicit_debug_layer(snicit_network* net, int32_t layer, const float* yin,
                                  float* yout, int64_t rows, int32_t kernel);
 
+/* Range-prediction horizon tables (R30; host computation, no GPU needed): for a layer map of a
+ * constant row out(v) = min(max(chain(v) + b0, 0), ymax), chain = 32 fmas acc = fma(v, w0, acc) from +0,
+ * hi[k-1] = least v in [0, ymax] with out^k(v) == ymax (+inf if none) and lo[k-1] = greatest v with
+ * out^k(v) == 0 (-1 if none), k = 1..kmax (kmax <= 32).  Returns 1 if either table is active, 0 if
+ * neither (or w0 < 0), SNICIT_E_INVALID_ARG for bad arguments.  Host pointers, kmax floats each. */
+int32_t snicit_debug_range_tables(float w0, float b0, float ymax, int32_t kmax, float* hi, float* lo);
+
 /* 1 if layer l is eligible for the circulant kernel, 0 if not, < 0 on error. */
 int32_t snicit_layer_is_circulant(const snicit_network* net, int32_t layer);
 

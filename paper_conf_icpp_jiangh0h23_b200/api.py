@@ -13,6 +13,18 @@ from . import _lib
 from ._lib import Options, SnicitError, Stats, check, default_options, load_library
 
 
+def range_tables(w0: float, b0: float, ymax: float, kmax: int = 32):
+    """snicit_debug_range_tables (R30): (hi, lo, active) horizon tables of the constant-row map
+    out(v) = sigma(chain(v) + b0), k = 1..kmax.  Host computation inside the library (no GPU needed)."""
+    L = load_library()
+    hi = np.empty(kmax, np.float32)
+    lo = np.empty(kmax, np.float32)
+    r = L.snicit_debug_range_tables(float(w0), float(b0), float(ymax), int(kmax), hi.ctypes.data, lo.ctypes.data)
+    if r < 0:
+        check(r, "snicit_debug_range_tables")
+    return hi, lo, bool(r)
+
+
 def _is_cuda_tensor(x) -> bool:
     return hasattr(x, "is_cuda") and bool(x.is_cuda)
 

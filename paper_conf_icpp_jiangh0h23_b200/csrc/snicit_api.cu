@@ -646,6 +646,20 @@ snicit_status snicit_set_stream(snicit_network* net, void* s) {
     return SNICIT_OK;
 }
 
+int32_t snicit_debug_range_tables(float w0, float b0, float ymax, int32_t kmax, float* hi, float* lo) {
+    if (!hi || !lo || kmax < 1 || kmax > kRangeK || !(ymax > 0.0f)) return SNICIT_E_INVALID_ARG;
+    PreFusedLayer d{};
+    d.w0 = w0;
+    d.b0 = b0;
+    float h[kRangeK], l_[kRangeK];
+    const bool ok = range_tables(&d, 1, ymax, h, l_);
+    for (int k = 0; k < kmax; ++k) {
+        hi[k] = ok ? h[k] : INFINITY;
+        lo[k] = ok ? l_[k] : -1.0f;
+    }
+    return ok ? 1 : 0;
+}
+
 int32_t snicit_layer_is_circulant(const snicit_network* net, int32_t l) {
     if (!net || l < 0 || l >= net->L) return -1;
     return net->plan[l].kind != 0 ? 1 : 0;

@@ -99,3 +99,32 @@ def test_null_handle_errors(lib):
 def test_package_exports():
     assert callable(pkg.SnicitNetwork) and callable(pkg.shard_rows)
     assert pkg.shard_rows(10, 3, 0) == (0, 4) and pkg.shard_rows(10, 3, 2) == (7, 10)
+
+
+@pytest.mark.parametrize("b0,kmax", [(-0.3, 32), (-0.4, 32), (-0.45, 12), (0.05, 8), (-40.0, 4)])
+def test_range_tables_match_reference(b0, kmax):
+    """R30 horizon tables computed by the library (composition: hi[k] = least v with out(v) >= hi[k-1])
+    equal an independent direct iteration of out^k (tests/range_ref.py), bit for bit; hi non-increasing,
+    lo non-decreasing, never overlapping; inactive tables are +inf / -1."""
+    from paper_conf_icpp_jiangh0h23_b200 import range_tables
+    from range_ref import range_thresholds
+    w0, ymax = 1.0 / 16.0, 32.0
+    hi, lo, active = range_tables(w0, b0, ymax, kmax)
+    rhi, rlo = range_thresholds(w0, b0, ymax, kmax)
+    assert active
+    assert np.array_equal(hi, np.array(rhi, np.float32)) and np.array_equal(lo, np.array(rlo, np.float32))
+    assert np.all(hi[1:] <= hi[:-1]) and np.all(lo[1:] >= lo[:-1]) and np.all(lo < hi)
+    if b0 > 0:
+        assert np.all(lo == -1.0)  # out(0) = b0 > 0: no row is ever proven zero
+    if b0 == -0.3:  # out(v) = 2v - 0.3: one layer saturates from (32 + 0.3)/2 and zeroes up to 0.15
+        assert abs(hi[0] - 16.15) < 1e-5 and abs(lo[0] - 0.15) < 1e-6
+        assert abs(hi[-1] - 0.3) < 1e-5 and abs(lo[-1] - 0.3) < 1e-5  # both close in on v* = -b0
+    if b0 == -40.0:  # out(v) = 2v - 40 < 32 on [0, 32]: no row reaches YMAX; zero after k layers from
+        assert np.all(np.isinf(hi)) and list(lo) == [20.0, 30.0, 32.0, 32.0]  # v <= 40 - 40/2^k (capped)
+
+
+def test_range_tables_rejects_bad_args():
+    from paper_conf_icpp_jiangh0h23_b200 import range_tables
+    with pytest.raises(Exception):
+        range_tables(0.0625, -0.3, 32.0, 33)
+    assert not range_tables(-0.0625, -0.3, 32.0, 4)[2]  # w0 < 0: outputs not monotone, tables off
