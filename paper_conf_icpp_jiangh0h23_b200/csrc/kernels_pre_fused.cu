@@ -181,6 +181,31 @@ __device__ __forceinline__ void pf_body_q32(const float* __restrict__ in, float*
     }
 }
 
+// Class-sum bounds of a Q32 layer (R31): thread c owns residue class c, and every output of the class is a
+// chain over the same 32 elements (a rotation of them), so one pass of directed-rounding sums bounds all
+// 32 outputs of the class before any of them is evaluated.  Inputs are >= 0 (outputs of sigma), w0 >= 0:
+// each RN step of a chain satisfies y (1 - u) - 2^-150 <= RN(y) <= y (1 + u) + 2^-150 (u = 2^-24), so a
+// chain in any order lies in [(1 - u)^32 S - 32 2^-150, (1 + u)^32 S + 32 2^-150], S = sum x w0 exactly,
+// bracketed by the round-down / round-up chains; (1 - u)^32 >= 1 - 2^-19, (1 + u)^32 <= 1 + 2^-18.  The
+// bias add and sigma are monotone, so sigma(RD(lo + b0)) <= y <= sigma(RU(hi + b0)) for every output y.
+template <int T>
+__device__ __forceinline__ void pf_q32_bounds(const float* __restrict__ in, float w0, float b0, float ymax,
+                                              float& ylo, float& yhi) {
+    constexpr int nu = T;
+    const int c = threadIdx.x;
+    float slo = 0.0f, shi = 0.0f;
+#pragma unroll
+    for (int k = 0; k < 32; ++k) {
+        const float x = in[k * nu + c];
+        slo = __fmaf_rd(x, w0, slo);
+        shi = __fmaf_ru(x, w0, shi);
+    }
+    const float lo = __fsub_rd(__fmul_rd(slo, 1.0f - 0x1p-19f), 0x1p-140f);
+    const float hi = __fadd_ru(__fmul_ru(shi, 1.0f + 0x1p-18f), 0x1p-140f);
+    ylo = sigma(__fadd_rd(lo, b0), ymax);
+    yhi = sigma(__fadd_ru(hi, b0), ymax);
+}
+
 // STR wrap handling: a 31*nu halo, or (kPfStrHalo = false) the a-row index mod Q
 template <int T>
 constexpr bool kPfStrHalo = true;  // measured: the masked form (H = 64, 6 CTAs/SM at N = 4096) is slower
@@ -233,6 +258,8 @@ __global__ void __launch_bounds__(T, PfCfg<T>::kMinBlocks) pre_fused_kernel(cons
     constexpr int kWarps = T / 32;
     unsigned* s_vmn = reinterpret_cast<unsigned*>(s_pos + 4);  // [2][kWarps] per-warp output minimum (bits)
     unsigned* s_vmx = s_vmn + 2 * kWarps;                      // [2][kWarps] per-warp output maximum
+    unsigned* s_bmn = s_vmx + 2 * kWarps;                      // [kWarps] Q32 class-sum bounds (R31)
+    unsigned* s_bmx = s_bmn + 2 * kWarps;                      //   (slots of 2 kWarps: s_bits stays 16-B aligned)
     const int tid = threadIdx.x;
     const int count = *a.count;
     if (tid == 0) {
@@ -244,7 +271,7 @@ __global__ void __launch_bounds__(T, PfCfg<T>::kMinBlocks) pre_fused_kernel(cons
     __syncthreads();
     int pos = s_pos[0];
     // one row (and its circular halo: a second copy of the row head) -> buffer `dst`, completion on `b`
-    uint32_t* s_bits = reinterpret_cast<uint32_t*>(s_vmx + 2 * kWarps);  // [2][N/32] packed rows (a.ybits)
+    uint32_t* s_bits = reinterpret_cast<uint32_t*>(s_bmx + 2 * kWarps);  // [2][N/32] packed rows (a.ybits)
     int* s_surv = reinterpret_cast<int*>(s_bits + 2 * (N / 32));       // [kPfSurv] rows alive at t, batched
     int nsurv = 0;                                                     // (tid 0) entries in s_surv
     // one atomic per kPfSurv survivors (an atomic whose result is waited on stalls the whole CTA at the
@@ -357,6 +384,39 @@ __global__ void __launch_bounds__(T, PfCfg<T>::kMinBlocks) pre_fused_kernel(cons
                     }
                 }
                 const int cls = fl & 15;
+                // R31: a Q32 layer's outputs are bounded by its class sums (pf_q32_bounds) before they are
+                // evaluated; the bounds of Y(l + 1) against the horizon k = t - l - 1 decide as in R30
+                if (cls == PF_Q32 && a.thr_ok && l > 0) {
+                    float ylo, yhi;
+                    pf_q32_bounds<T>(in, w0, b0, a.ymax, ylo, yhi);
+                    const unsigned wmn = __reduce_min_sync(0xffffffffu, __float_as_uint(ylo + 0.0f));
+                    const unsigned wmx = __reduce_max_sync(0xffffffffu, __float_as_uint(yhi + 0.0f));
+                    if ((tid & 31) == 0) {
+                        s_bmn[tid >> 5] = wmn;
+                        s_bmx[tid >> 5] = wmx;
+                    }
+                    __syncthreads();
+                    const int ln = tid & 31;
+                    const float bmn =
+                        __uint_as_float(__reduce_min_sync(0xffffffffu, ln < kWarps ? s_bmn[ln] : 0xffffffffu));
+                    const float bmx = __uint_as_float(__reduce_max_sync(0xffffffffu, ln < kWarps ? s_bmx[ln] : 0u));
+                    const int k2 = a.t - l - 1;  // layers after this one
+                    const int kk = min(k2, kPfThr);
+                    if (bmn >= (k2 ? p.thr_hi[kk - 1] : a.ymax)) {  // Y(t) is the constant row YMAX
+                        v = a.ymax;
+                        cst = true;
+                        break;
+                    }
+                    if (bmx <= (k2 ? p.thr_lo[kk - 1] : 0.0f)) {  // Y(t) is zero
+                        v = 0.0f;
+                        cst = true;
+                        if (a.drop && (k2 ? a.dead_t : dead_next)) {
+                            dead = true;
+                            lend = l + kk;
+                        }
+                        break;
+                    }
+                }
                 if (cls == PF_NU1)
                     pf_body_nu1<T>(in, out, w0, b0, a.ymax, H, mn, mx);
                 else if (cls == PF_Q32)
@@ -484,7 +544,7 @@ int pre_fused_threads(int N) {
 
 size_t pre_fused_smem(int N, int H) {
     const int nb = N / 32 >= 512 ? 3 : 2;  // kPfBufs
-    return sizeof(float) * nb * (size_t)(N + H) + 2 * sizeof(uint64_t) + 4 * sizeof(int) + 4 * sizeof(int) * (N / 32 / 32) +
+    return sizeof(float) * nb * (size_t)(N + H) + 2 * sizeof(uint64_t) + 4 * sizeof(int) + 8 * sizeof(int) * (N / 32 / 32) +
            2 * sizeof(uint32_t) * (size_t)(N / 32) + sizeof(int) * kPfSurv;  // packed-row slots, survivors
 }
 

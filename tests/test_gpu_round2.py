@@ -22,7 +22,6 @@ import oracle  # noqa: E402
 from paper_conf_icpp_jiangh0h23_b200 import CSR_FORMAT, SnicitNetwork, shard_capacity, shard_rows  # noqa: E402
 from workload import sdgc  # noqa: E402
 from workload.sdgc import Network  # noqa: E402
-from range_ref import range_thresholds as _range_thresholds  # noqa: E402
 
 pytestmark = pytest.mark.gpu
 
@@ -368,55 +367,38 @@ def test_range_prediction_bit_exact(N, drop):
 
 
 def test_dynamics_log(tmp_path):
-    """snicit_dynamics (SURVEY 5 per-layer log) of the row-resident kernel, modelled row by row on the
-    oracle's layer-by-layer rows: pre_full[l] = rows evaluated in full by layer l (not yet constant, R26,
-    and not predicted by the range rule, R30: before layer l >= 1 with k = min(t - l, 32), min of Y(l) >=
-    thr_hi[k-1] -> YMAX at t, max <= thr_lo[k-1] -> zero at t, dropped at layer l - 1 + k); pre_live[l] =
-    rows not dropped after layer l (all-zero rows drop at once, R23); res_alive ends at
-    stats.residual_final and never increases (zero residues are absorbing, R16)."""
+    """snicit_dynamics (SURVEY 5 per-layer log) of the row-resident kernel.  Without the range rules
+    (pre_fused = 6) it is modelled row by row on the oracle's layer-by-layer rows: pre_full[l] = rows not
+    yet constant (R26) before layer l, pre_live[l] = rows with a non-zero output after layer l (all-zero
+    rows drop at once, R23).  With them (default: R30 / R31 drop a row at the layer by which its range
+    proves Y(t)), fewer rows are evaluated in full, pre_live counts rows not yet proven zero (>= the
+    non-zero rows) and is exact after layer t - 1.  res_alive ends at stats.residual_final and never
+    increases (zero residues are absorbing, R16)."""
     N, L, B, t = 1024, 40, 600, 6
     net = sdgc.gen_network(N, L, "radix")
     Y0 = sdgc.gen_inputs(N, B)
     with SnicitNetwork.from_network(net) as g:
         g.set_stream(torch.cuda.current_stream())
+        _infer(g, Y0, t, timing=1, pre_fused=6)
+        d6 = g.dynamics()
         _infer(g, Y0, t, timing=1)
         d = g.dynamics()
         st = g.stats()
         nlines = g.write_dynamics_jsonl(str(tmp_path / "dyn.jsonl"))
-    hi, lo = _range_thresholds(sdgc.SDGC_WEIGHT, sdgc.SDGC_BIAS[N], sdgc.SDGC_YMAX)
     y = Y0.copy()
-    mn, mx, alleq, allz = [], [], [], []
+    const_before = np.zeros(B, bool)
+    alive = np.ones(B, bool)
     for l in range(t):
+        full = alive & ~const_before
+        assert d6["pre_full"][l] == int(full.sum()), l
         y = oracle.layers_f32(net, y, l, l + 1)
-        mn.append(y.min(1))
-        mx.append(y.max(1))
-        alleq.append((y == y[:, :1]).all(1))
-        allz.append(~(y != 0).any(1))
-    full = np.zeros(B, int)
-    lend = np.full(B, t)
-    n_pred = 0
-    for r in range(B):
-        cst = False
-        for l in range(t):
-            if not cst:
-                if l > 0:
-                    k = min(t - l, 32)
-                    if mn[l - 1][r] >= hi[k - 1]:
-                        n_pred += 1
-                        break
-                    if mx[l - 1][r] <= lo[k - 1]:
-                        n_pred += 1
-                        lend[r] = l + k - 1
-                        break
-                full[r] += 1
-                cst = bool(alleq[l][r])
-            if allz[l][r]:
-                lend[r] = l
-                break
-    assert n_pred > 0  # the workload exercises R30
-    for l in range(t):
-        assert d["pre_full"][l] == int((full > l).sum()), l
-        assert d["pre_live"][l] == int((lend > l).sum()), l
+        alive = alive & (y != 0).any(1)
+        assert d6["pre_live"][l] == int(alive.sum()), l
+        assert d["pre_live"][l] >= int(alive.sum()), l
+        assert d["pre_full"][l] <= d6["pre_full"][l], l
+        const_before = const_before | (alive & (y == y[:, :1]).all(1))
+    assert d["pre_live"][t - 1] == int(alive.sum())
+    assert sum(d["pre_full"][:t]) < sum(d6["pre_full"][:t])  # the range rules fire on this workload
     ra = d["res_alive"][t:]
     assert ra[-1] == st["residual_final"] and np.all(np.diff(ra) <= 0) and ra[0] <= st["residual_at_t"]
     assert np.all(d["pre_full"][t:] == -1) and np.all(d["res_alive"][:t] == -1)
