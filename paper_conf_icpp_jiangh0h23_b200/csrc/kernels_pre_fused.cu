@@ -41,6 +41,7 @@ constexpr int kPfM1 = 17;  // NU1 outputs per item
 constexpr int kPfM = 16;   // STR / Q32 outputs per item
 constexpr int kPfSurv = 32;  // survivor batch per CTA
 constexpr int kPfW = kPfM + 31;
+constexpr int kPfConstChunk = 1024;  // floats per constant-row TMA store (NB == 3)
 
 typedef unsigned long long u64;
 
@@ -273,6 +274,12 @@ __global__ void __launch_bounds__(T, PfCfg<T>::kMinBlocks) pre_fused_kernel(cons
     // one row (and its circular halo: a second copy of the row head) -> buffer `dst`, completion on `b`
     uint32_t* s_bits = reinterpret_cast<uint32_t*>(s_bmx + 2 * kWarps);  // [2][N/32] packed rows (a.ybits)
     int* s_surv = reinterpret_cast<int*>(s_bits + 2 * (N / 32));       // [kPfSurv] rows alive at t, batched
+    // NB == 3 (one CTA per SM): 4 KB rows of zeros and of YMAX, the sources of the TMA bulk stores that
+    // write dead rows and constant-YMAX rows (16 bulk copies issued by one thread instead of N/4 vector
+    // stores from every warp); written once, never modified
+    float* s_cz = reinterpret_cast<float*>(s_surv + kPfSurv);
+    float* s_cy = s_cz + kPfConstChunk;
+    bool prev_res = false;  // (tid 0, NB == 3) the previous row ended with a TMA store of a row buffer
     int nsurv = 0;                                                     // (tid 0) entries in s_surv
     // one atomic per kPfSurv survivors (an atomic whose result is waited on stalls the whole CTA at the
     // next barrier; per row that was ~1 us)
@@ -301,6 +308,14 @@ __global__ void __launch_bounds__(T, PfCfg<T>::kMinBlocks) pre_fused_kernel(cons
             bulk_g2s(dst + N, g, H * 4, b);
         }
     };
+    if (NB == 3) {
+        for (int i = tid; i < kPfConstChunk; i += T) {
+            s_cz[i] = 0.0f;
+            s_cy[i] = a.ymax;
+        }
+        fence_proxy_async_smem();
+        __syncthreads();
+    }
     int i_in = 0, i_out = 1, i_pf = 2;  // buffer roles (NB == 3: i_pf receives the next row)
     uint32_t ph = 0;                    // phase bit of bar[0], bar[1]
     if (NB == 3 && tid == 0 && pos < count) issue_load(pos, buf, &bar[0], 0);
@@ -323,7 +338,9 @@ __global__ void __launch_bounds__(T, PfCfg<T>::kMinBlocks) pre_fused_kernel(cons
             if (NB == 3) {
                 s_pos[2 + (k & 1)] = np;
                 if (np < count) {  // load it now, behind this row's compute
-                    bulk_wait_read0();
+                    // its buffer held the previous row's result: wait until that row's TMA store has read
+                    // it (older stores were waited for one row earlier; constant-row stores read s_cz/s_cy)
+                    if (prev_res) bulk_wait_read0();
                     issue_load(np, buf + i_pf * S, &bar[(k + 1) & 1], (k + 1) & 1);
                 }
             }
@@ -480,23 +497,43 @@ __global__ void __launch_bounds__(T, PfCfg<T>::kMinBlocks) pre_fused_kernel(cons
                 if ((v == a.ymax && ((fl >> 6) & 1)) || (v == 0.0f && dead_next)) break;
             }
         }
+        if (NB == 3 && tid == 0) prev_res = false;
         if (dead && a.ydead) {  // final activations of a dead row: zeros, written now (the SMs' HBM is idle)
-            float4* dz = reinterpret_cast<float4*>(a.ydead + (size_t)row * N);
+            if (NB == 3) {
+                if (tid == 0) {
+                    float* dz = a.ydead + (size_t)row * N;
+                    for (int i = 0; i < N / kPfConstChunk; ++i) bulk_s2g(dz + i * kPfConstChunk, s_cz, kPfConstChunk * 4);
+                    bulk_commit();
+                }
+            } else {
+                float4* dz = reinterpret_cast<float4*>(a.ydead + (size_t)row * N);
 #pragma unroll
-            for (int i = 0; i < N / 4 / T; ++i) dz[i * T + tid] = make_float4(0.f, 0.f, 0.f, 0.f);
+                for (int i = 0; i < N / 4 / T; ++i) dz[i * T + tid] = make_float4(0.f, 0.f, 0.f, 0.f);
+            }
         }
         if (!dead) {
             float* gout = a.yout + (size_t)row * N;
             if (cst) {
-                const float4 v4 = make_float4(v, v, v, v);
+                const uint32_t vb = __float_as_uint(v);
+                if (NB == 3 && (vb == __float_as_uint(a.ymax) || vb == 0u)) {  // bitwise +0 / YMAX rows
+                    if (tid == 0) {
+                        const float* src = vb == 0u ? s_cz : s_cy;
+                        for (int i = 0; i < N / kPfConstChunk; ++i)
+                            bulk_s2g(gout + i * kPfConstChunk, src, kPfConstChunk * 4);
+                        bulk_commit();
+                    }
+                } else {
+                    const float4 v4 = make_float4(v, v, v, v);
 #pragma unroll
-                for (int i = 0; i < N / 4 / T; ++i) reinterpret_cast<float4*>(gout)[i * T + tid] = v4;
+                    for (int i = 0; i < N / 4 / T; ++i) reinterpret_cast<float4*>(gout)[i * T + tid] = v4;
+                }
             } else {
                 fence_proxy_async_smem();  // generic-proxy writes of `in` -> visible to the TMA engine
                 __syncthreads();
                 if (tid == 0) {
                     bulk_s2g(gout, in, N * 4);
                     bulk_commit();
+                    prev_res = true;
                 }
             }
             if (tid == 0 && a.app_list) {
@@ -545,7 +582,8 @@ int pre_fused_threads(int N) {
 size_t pre_fused_smem(int N, int H) {
     const int nb = N / 32 >= 512 ? 3 : 2;  // kPfBufs
     return sizeof(float) * nb * (size_t)(N + H) + 2 * sizeof(uint64_t) + 4 * sizeof(int) + 8 * sizeof(int) * (N / 32 / 32) +
-           2 * sizeof(uint32_t) * (size_t)(N / 32) + sizeof(int) * kPfSurv;  // packed-row slots, survivors
+           2 * sizeof(uint32_t) * (size_t)(N / 32) + sizeof(int) * kPfSurv +  // packed-row slots, survivors
+           (nb == 3 ? 2 * sizeof(float) * kPfConstChunk : 0);                 // constant-row store sources
 }
 
 template <int T, bool GENSTR, bool WUNI>
