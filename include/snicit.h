@@ -202,7 +202,9 @@ snicit_status snicit_set_stream(snicit_network* net, void* cuda_stream);
  *                   (larger: SNICIT_E_UNSUPPORTED).
  *  opt:             NULL = snicit_default_options.
  *  y_out:           batch*N fp32, caller-owned; device pointer if y_out_on_device else host;
- *                   NULL = do not materialise Y(L) (categories are still computed).
+ *                   NULL = do not materialise Y(L) (categories are still computed).  A device y_out
+ *                   (not overlapping a device y0) also stores Y(t) when the row-resident pre phase runs,
+ *                   so rows whose Y(L) equals their constant Y(t) are written once.
  * Alignment: device y0 / y_out must be 16-byte aligned (TMA bulk copies and float4 accesses);
  * otherwise SNICIT_E_INVALID_ARG.
  * Host synchronisation: when y0 or y_out is a HOST pointer the call returns only after the stream

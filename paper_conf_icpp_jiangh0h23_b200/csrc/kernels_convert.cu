@@ -597,14 +597,20 @@ cudaError_t launch_map_residual(const float* y, int N, const int* rows, const in
 // ------------------------------------------------------------------------------ recovery
 // Eq. 6: Y_r = Yhat_r (centroid); (ne ? Yhat_r : 0) + Yhat_M(r) (mapped, R18); 0 (dead, R23).
 // plain != 0 (t >= L): Y_r = live ? yfinal_r : 0.  cat[r] = any non-zero (R13).  One CTA per row.
+// yt_rconst != NULL: y_out already holds Y(t) (the row-resident kernel wrote it there) and yt_rconst /
+// rval flag the rows constant at t.  Plain: Y(L) = Y(t) is in place (only the flags are computed; a
+// constant row needs no read).  SNICIT: a row that is a centroid (M = -1) or maps to one with an empty
+// residue (Eq. 6: 0 + c) while its Y(t) is the constant v > 0 and its centroid is a constant row carried
+// to L (cdone, R25) with the same value bitwise already holds Y(L) = v: no write.
 constexpr int kRecThreads = 256;
 __global__ void __launch_bounds__(kRecThreads) recover_kernel(int N, int R, int plain,
-                                                              const float* __restrict__ yfinal,
+                                                              const float* yfinal,
                                                               const uint8_t* live_row, const int* M,
                                                               const int* cslot, const uint8_t* ne_row,
                                                               const float* __restrict__ cbuf,
-                                                              float* __restrict__ y_out, uint8_t* cat,
-                                                              int dead_zeroed) {
+                                                              float* y_out, uint8_t* cat,
+                                                              int dead_zeroed, const uint8_t* yt_rconst,
+                                                              const float* rval, const int* cdone) {
     const int N4 = N >> 2;
     for (int r = blockIdx.x; r < R; r += gridDim.x) {
         int mode;  // 0 zero, 1 copy a, 2 a + c, 3 0 + c
@@ -634,8 +640,24 @@ __global__ void __launch_bounds__(kRecThreads) recover_kernel(int N, int R, int 
             if (threadIdx.x == 0) cat[r] = 0;
             continue;  // uniform across the CTA
         }
+        bool in_place = false;
+        if (yt_rconst) {
+            if (plain && mode == 1) {
+                if (yt_rconst[r]) {
+                    if (threadIdx.x == 0) cat[r] = rval[r] != 0.0f ? 1 : 0;
+                    continue;
+                }
+                in_place = true;  // Y(L) = Y(t) already in y_out: read for the flag only
+            } else if (!plain && (mode == 1 || mode == 3) && cdone && yt_rconst[r] && cdone[cslot[r]]) {
+                const float v = rval[r];
+                if (v > 0.0f && __float_as_uint(v) == __float_as_uint(cbuf[(size_t)cslot[r] * N])) {
+                    if (threadIdx.x == 0) cat[r] = 1;
+                    continue;
+                }
+            }
+        }
         int any = 0;
-        float4* o4 = y_out ? reinterpret_cast<float4*>(y_out + (size_t)r * N) : nullptr;
+        float4* o4 = (y_out && !in_place) ? reinterpret_cast<float4*>(y_out + (size_t)r * N) : nullptr;
         for (int k = threadIdx.x; k < N4; k += blockDim.x) {
             float4 v;
             if (mode == 0) {
@@ -658,12 +680,13 @@ __global__ void __launch_bounds__(kRecThreads) recover_kernel(int N, int R, int 
 }
 cudaError_t launch_recover(int N, int R, int plain, const float* yfinal, const uint8_t* live_row, const int* M,
                            const int* cslot, const uint8_t* ne_row, const float* cbuf, float* y_out,
-                           uint8_t* cat, int num_sms, cudaStream_t st, int dead_zeroed) {
+                           uint8_t* cat, int num_sms, cudaStream_t st, int dead_zeroed,
+                           const uint8_t* yt_rconst, const float* rval, const int* cdone) {
     if (R <= 0) return cudaSuccess;
     int grid = num_sms * 8;
     if (grid > R) grid = R;
     recover_kernel<<<grid, kRecThreads, 0, st>>>(N, R, plain, yfinal, live_row, M, cslot, ne_row, cbuf, y_out,
-                                                 cat, dead_zeroed);
+                                                 cat, dead_zeroed, yt_rconst, rval, cdone);
     return cudaGetLastError();
 }
 

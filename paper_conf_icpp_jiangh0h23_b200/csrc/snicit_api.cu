@@ -1098,6 +1098,11 @@ static snicit_status infer_core(snicit_network* net, const float* y0, int64_t ba
     if (y0_mode == 3 && !pf && R > 0) return fail(SNICIT_E_STATE, "packed rows without the row-resident kernel");
     net->last_pre_fused = pf;
     const int dead_zeroed = (pf && y_out_on_device && y_out && drop) ? 1 : 0;  // y_out rows of dead rows
+    // a device y_out holds Y(t) too (the row-resident kernel writes it there): rows whose Y(L) equals
+    // their constant Y(t) are then never rewritten by the recovery (unless y0 overlaps y_out)
+    const bool yt_out = pf && y_out_on_device && y_out &&
+                        !(y0_on_device && y0 && (const char*)y0 < (const char*)(y_out + (size_t)R * N) &&
+                          (const char*)y_out < (const char*)(y0 + (size_t)R * N));
     net->last_dead_zeroed = dead_zeroed != 0;
     stats.pre_fused = pf ? (pf_cluster ? 2 : 1) : 0;
     if (R > 0) CUDA_TRY(cudaMemsetAsync(net->rconst.p, 0, (size_t)R, st));  // rows constant at t (R26)
@@ -1123,7 +1128,7 @@ static snicit_status infer_core(snicit_network* net, const float* y0, int64_t ba
         pa.one = one;
         pa.ready = (y0_mode == 3 || host_streamed) ? bits_ready : nullptr;
         pa.ready_rows = ready_rows;
-        pa.yout = bufs[nxt_i];
+        pa.yout = yt_out ? y_out : bufs[nxt_i];
         pa.rows = lists[li];
         pa.count = cnt + live_ctr[ci];
         pa.app_list = drop ? lists[li ^ 1] : nullptr;
@@ -1151,8 +1156,12 @@ static snicit_status infer_core(snicit_network* net, const float* y0, int64_t ba
         ++launches;
         circ_layers += tt;
         net->last_kernel_circ = true;
-        cur = bufs[nxt_i];
-        nxt_i ^= 1;
+        if (yt_out) {
+            cur = y_out;  // both workspace buffers stay free for the residues
+        } else {
+            cur = bufs[nxt_i];
+            nxt_i ^= 1;
+        }
         if (drop) {
             li ^= 1;
             ci = (ci + 1) % 3;
@@ -1267,7 +1276,8 @@ static snicit_status infer_core(snicit_network* net, const float* y0, int64_t ba
         }
         if (!y_out_on_device && y_out) y_dst = bufs[nxt_i];
         CUDA_TRY(launch_recover(N, R, 1, yfinal, net->live_row.p, nullptr, nullptr, nullptr, nullptr, y_dst,
-                                net->cat.p, net->num_sms, st, y_dst == y_out ? dead_zeroed : 0));
+                                net->cat.p, net->num_sms, st, y_dst == y_out ? dead_zeroed : 0,
+                                yt_out ? net->rconst.p : nullptr, net->rval.p, nullptr));
         ++launches;
     } else {
         // ordered live list: "the first s columns" are the first s live rows by id (R14)
@@ -1491,7 +1501,8 @@ static snicit_status infer_core(snicit_network* net, const float* y0, int64_t ba
         // ---- a6: recovery (Eq. 6)
         if (!y_out_on_device && y_out) y_dst = yh_nxt;  // free buffer
         CUDA_TRY(launch_recover(N, R, 0, yfinal, nullptr, net->M.p, net->cslot.p, net->ne_row.p, cfinal, y_dst,
-                                net->cat.p, net->num_sms, st, y_dst == y_out ? dead_zeroed : 0));
+                                net->cat.p, net->num_sms, st, y_dst == y_out ? dead_zeroed : 0,
+                                (yt_out && y_dst == y_out) ? net->rconst.p : nullptr, net->rval.p, cdone));
         ++launches;
     }
     // categories: ordered compaction of the cat flags over all rows (R13)

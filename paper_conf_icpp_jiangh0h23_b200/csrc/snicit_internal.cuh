@@ -367,7 +367,8 @@ cudaError_t launch_map_residual(const float* y, int N, const int* rows, const in
                                 int* need /* [max_rows] scratch */, int* need_count /* device int */);
 cudaError_t launch_recover(int N, int R, int plain, const float* yfinal, const uint8_t* live_row, const int* M,
                            const int* cslot, const uint8_t* ne_row, const float* cbuf, float* y_out,
-                           uint8_t* cat, int num_sms, cudaStream_t st, int dead_zeroed = 0);
+                           uint8_t* cat, int num_sms, cudaStream_t st, int dead_zeroed = 0,
+                           const uint8_t* yt_rconst = nullptr, const float* rval = nullptr, const int* cdone = nullptr);
 // packed binary rows -> fp32 rows: y[r][j] = bit j of row r ? one : 0 (snicit_infer_packed)
 cudaError_t launch_unpack_bits(const uint32_t* bits, int R, int N, float one, float* y, int num_sms, cudaStream_t st);
 cudaError_t launch_mark_rows(const int* rows, const int* count, uint8_t* flag_row, int max_rows, cudaStream_t st);
