@@ -70,7 +70,7 @@ def parse(argv=None):
     p.add_argument("--no-residue", action="store_true", help="skip the residue-regime study (C2, t = 10)")
     p.add_argument("--no-general", action="store_true", help="skip the general-CSC study (C2 perm)")
     p.add_argument("--residue-t", type=int, default=10)
-    p.add_argument("--pre-fused", type=int, default=1, choices=[0, 1, 2, 3, 4, 5, 6],
+    p.add_argument("--pre-fused", type=int, default=1, choices=[0, 1, 2, 3, 4, 5, 6, 7],
                    help="options.pre_fused: 1 = row-resident pre phase (default), 2 = without the constant-row "
                         "shortcut, 6 = without the range prediction (R30), 4 = rows split over a thread-block "
                         "cluster (N >= 16384), 0 = one launch per layer")

@@ -30,7 +30,7 @@
 extern "C" {
 #endif
 
-#define SNICIT_ABI_VERSION 4
+#define SNICIT_ABI_VERSION 5
 
 typedef struct snicit_network snicit_network; /* opaque: owns device copies of W, b + workspace */
 
@@ -99,9 +99,14 @@ typedef struct {
                                5 = as 1 with the row stored as pairs (y[p], y[p + N/2]) read by 8-byte
                                loads (kernels_pre_pair.cu).  4 and 5 are measured alternatives (slower
                                than 1 on B200), kept selectable and parity-tested.
-                               6 = as 1 without the range prediction (R30: a row whose output range
-                               bounds Y(t) to the constant row YMAX or to zero leaves early; on in 1), for
-                               measurement.
+                               6 = as 1 with fma chains for every non-constant row-layer: without the
+                               range prediction (R30/R31: a row whose output range or class-sum bounds
+                               prove Y(t) the constant row YMAX or zero leaves early) and without the
+                               popcount layer 0 (R32: a stride-1 layer 0 on a row of zeros and one value
+                               is a table lookup by window count); 2 also runs without R32.  For
+                               measurement.  R32 runs on packed rows (snicit_infer_packed: the bitmap is
+                               given); 7 = as 1 with R32 also on fp32 rows of zeros and one value (the
+                               bitmap built by ballots: measured slower on C3).
                                Used when every layer < t is circulant
                                with 32 taps, uniform weight and uniform bias, and N/32 is one of
                                32..512 (N = 1024..16384; 4: the cluster form supports every stride);
@@ -157,6 +162,9 @@ typedef struct {
                                  rows and constant rows with an equal constant centroid, R26) */
     double t_map_ms;          /* map_residual kernels (Alg. 2), CUDA events (options.timing), else -1 */
     double t_residual_ms;     /* residue trajectory kernel (Eq. 5, fused post mode), else -1 */
+    int64_t pre_popc_rows;    /* fused: rows whose layer 0 (stride 1) ran as a popcount table lookup (a row
+                                 of 0 and one value c: each output depends only on the count of c in its
+                                 window, R32) -- not counted in pre_full_rows */
 } snicit_stats_t;
 
 /* Fill *opt with the paper's SDGC defaults (n = 16, eta = eps = 0.03, prune_eps = 0,

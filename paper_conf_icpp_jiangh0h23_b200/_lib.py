@@ -48,7 +48,7 @@ class Stats(ctypes.Structure):
                 ("res_nnz_at_t", ctypes.c_int64), ("res_full_rl", ctypes.c_int64), ("res_sparse_rl", ctypes.c_int64),
                 ("res_sparse_out", ctypes.c_int64), ("res_scalar_rl", ctypes.c_int64), ("map_rows", ctypes.c_int64),
                 ("t_map_ms", ctypes.c_double),
-                ("t_residual_ms", ctypes.c_double)]
+                ("t_residual_ms", ctypes.c_double), ("pre_popc_rows", ctypes.c_int64)]
 
     def as_dict(self):
         return {k: getattr(self, k) for k, _ in self._fields_}

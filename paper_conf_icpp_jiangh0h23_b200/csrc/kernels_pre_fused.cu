@@ -207,6 +207,101 @@ __device__ __forceinline__ void pf_q32_bounds(const float* __restrict__ in, floa
     yhi = sigma(__fadd_ru(hi, b0), ymax);
 }
 
+// R32: layer 0 of stride 1 as a table lookup when the row holds zeros and one value c (checked here for
+// fp32 rows; packed rows are binary with c = one).  Warp w owns the words j = 32 w .. 32 w + 31 of the
+// row's bitmap (bit b of word j = element 32 j + b != 0; lane i holds word 32 w + i, built by one ballot
+// per word for fp32 rows or read from the packed row) and lane i the outputs q = 32 j + e of its word j:
+// window q .. q + 31 = bits e .. e + 31 of (word j + 1 : word j), k = popc of it, output tab[k] (the
+// warp's copy of tab[k] = sigma(chain of k fmas of c from +0, + b0), k = 0..32, in shared memory).  The
+// lanes walk e = (b + lane) mod 32 so the stores of one step hit 32 different banks.  Returns false
+// (nothing written) for a row with two different non-zero values, a NaN or c < 0.
+__device__ __forceinline__ float max_nan(float a, float b) {
+    float r;
+    asm("max.NaN.f32 %0, %1, %2;" : "=f"(r) : "f"(a), "f"(b));
+    return r;
+}
+constexpr int kPfTabStride = 40;  // floats per warp table (33 used)
+template <int T>
+__device__ __forceinline__ bool pf_popc_layer0(const float* __restrict__ in, float* __restrict__ out,
+                                               const uint32_t* pwords, float one, float w0, float b0, float ymax,
+                                               int H, unsigned* s_red, float* s_tabw, float& mn, float& mx) {
+    constexpr int N = 32 * T, W = N / 32, kWarps = T / 32;
+    const int tid = threadIdx.x, lane = tid & 31, warp = tid >> 5;
+    const int j0 = warp * 32;  // W / kWarps == 32 words per warp
+    uint32_t wl, wnext;
+    float c = one;
+    if (pwords) {
+        wl = pwords[j0 + lane];
+        wnext = pwords[(j0 + 32) & (W - 1)];
+    } else {
+        float nzmin = __int_as_float(0x7f800000), nzmax = -__int_as_float(0x7f800000);
+        wl = 0u;
+        const float* src = in + j0 * 32 + lane;
+#pragma unroll 8
+        for (int i = 0; i < 32; ++i) {
+            const float x = src[i * 32];
+            const bool nz = x != 0.0f;
+            const uint32_t bw = __ballot_sync(0xffffffffu, nz);
+            wl = lane == i ? bw : wl;
+            nzmin = fminf(nzmin, nz ? x : __int_as_float(0x7f800000));
+            nzmax = max_nan(nzmax, x);
+        }
+        wnext = __ballot_sync(0xffffffffu, in[((j0 + 32) & (W - 1)) * 32 + lane] != 0.0f);
+#pragma unroll
+        for (int d = 16; d; d >>= 1) {
+            nzmin = fminf(nzmin, __shfl_xor_sync(0xffffffffu, nzmin, d));
+            nzmax = max_nan(nzmax, __shfl_xor_sync(0xffffffffu, nzmax, d));
+        }
+        if (lane == 0) {
+            s_red[warp] = __float_as_uint(nzmin);
+            s_red[kWarps + warp] = __float_as_uint(nzmax);
+        }
+        __syncthreads();
+        float gmin = __int_as_float(0x7f800000), gmax = -__int_as_float(0x7f800000);
+#pragma unroll
+        for (int w = 0; w < kWarps; ++w) {
+            gmin = fminf(gmin, __uint_as_float(s_red[w]));
+            gmax = max_nan(gmax, __uint_as_float(s_red[kWarps + w]));
+        }
+        __syncthreads();  // s_red read by every thread before it is reused
+        // two-valued: every non-zero equals gmax (> 0); all zero: gmax = 0, every count 0
+        if (gmax == 0.0f) c = 0.0f;
+        else if (gmin == gmax && gmax > 0.0f) c = gmax;
+        else return false;
+    }
+    float* tw = s_tabw + warp * kPfTabStride;
+    {
+        float acc = 0.0f;
+        for (int n = 0; n < lane; ++n) acc = fmaf(c, w0, acc);
+        tw[lane] = sigma(acc + b0, ymax);
+        const float acc31 = __shfl_sync(0xffffffffu, acc, 31);
+        if (lane == 0) tw[32] = sigma(fmaf(c, w0, acc31) + b0, ymax);
+    }
+    __syncwarp();
+    const uint32_t wn = __shfl_down_sync(0xffffffffu, wl, 1);
+    const uint32_t wj1 = lane < 31 ? wn : wnext;
+    float* dst = out + (j0 + lane) * 32;
+    const int qb = (j0 + lane) * 32;
+    const bool halo = j0 * 32 < H;  // warp-uniform
+    int kmin = 32, kmax = 0;
+#pragma unroll 8
+    for (int b = 0; b < 32; ++b) {
+        const int e = (b + lane) & 31;
+        const int k = __popc(__funnelshift_r(wl, wj1, e));
+        const float o = tw[k];
+        dst[e] = o;
+        if (halo && qb + e < H) dst[N + e] = o;
+        kmin = min(kmin, k);
+        kmax = max(kmax, k);
+    }
+    // tab is monotone in k (chains of one value c >= 0, sigma monotone): the range is tab[kmin], tab[kmax]
+    kmin = __reduce_min_sync(0xffffffffu, kmin);
+    kmax = __reduce_max_sync(0xffffffffu, kmax);
+    mn = fminf(mn, tw[kmin]);
+    mx = fmaxf(mx, tw[kmax]);
+    return true;
+}
+
 // STR wrap handling: a 31*nu halo, or (kPfStrHalo = false) the a-row index mod Q
 template <int T>
 constexpr bool kPfStrHalo = true;  // measured: the masked form (H = 64, 6 CTAs/SM at N = 4096) is slower
@@ -277,7 +372,8 @@ __global__ void __launch_bounds__(T, PfCfg<T>::kMinBlocks) pre_fused_kernel(cons
     // NB == 3 (one CTA per SM): 4 KB rows of zeros and of YMAX, the sources of the TMA bulk stores that
     // write dead rows and constant-YMAX rows (16 bulk copies issued by one thread instead of N/4 vector
     // stores from every warp); written once, never modified
-    float* s_cz = reinterpret_cast<float*>(s_surv + kPfSurv);
+    float* s_tabw = reinterpret_cast<float*>(s_surv + kPfSurv);  // [kWarps][kPfTabStride] R32 tables
+    float* s_cz = s_tabw + kWarps * kPfTabStride;
     float* s_cy = s_cz + kPfConstChunk;
     bool prev_res = false;  // (tid 0, NB == 3) the previous row ended with a TMA store of a row buffer
     int nsurv = 0;                                                     // (tid 0) entries in s_surv
@@ -347,7 +443,8 @@ __global__ void __launch_bounds__(T, PfCfg<T>::kMinBlocks) pre_fused_kernel(cons
         }
         mbar_wait(&bar[k & 1], (ph >> (k & 1)) & 1u);
         ph ^= 1u << (k & 1);
-        if (a.ybits) {  // expand the bits (value a.one, as snicit_infer_packed's unpack) + the halo copy
+        // packed rows whose layer 0 runs as R32 are never expanded (layer 0 reads the bitmap only)
+        if (a.ybits && !(a.popc0 && (p.L[0].flags & 15) == PF_NU1)) {  // expand the bits (value a.one) + halo
             float* dst = buf + i_in * S;
             const uint32_t* sb = s_bits + (k & 1) * (N / 32);
             const int wq = tid >> 5, lane = tid & 31;
@@ -364,7 +461,8 @@ __global__ void __launch_bounds__(T, PfCfg<T>::kMinBlocks) pre_fused_kernel(cons
         float* out = buf + i_out * S;
         bool cst = false, dead = false;
         float v = 0.0f;
-        int full = 0;
+        int full = 0, full_fma = 0;  // layers evaluated in full; of them by fma chains (not R32)
+        bool popc = false;
         unsigned cmn = 0u, cmx = 0xffffffffu;  // the previous layer's output range (bits)
         int lend = a.t;  // the layer that zeroed the row (dead, R23), or t: alive after layer l <=> lend > l
         for (int l = 0; l < a.t; ++l) {
@@ -401,6 +499,16 @@ __global__ void __launch_bounds__(T, PfCfg<T>::kMinBlocks) pre_fused_kernel(cons
                     }
                 }
                 const int cls = fl & 15;
+                // R32: layer 0 of stride 1 on a row of zeros and one value c.  fma(0, w0, acc) = acc exactly,
+                // so every chain is k fmas of c from +0 (k = count of c in the window, in any order): the
+                // output is tab[k], 33 values; the windows' counts are popcounts of the row's bitmap
+                if (l == 0 && cls == PF_NU1 && (a.popc0 == 1 || (a.popc0 == 2 && a.ybits))) {
+                    if (pf_popc_layer0<T>(in, out, a.ybits ? s_bits + (k & 1) * (N / 32) : nullptr, a.one, w0, b0,
+                                          a.ymax, H, s_bmn, s_tabw, mn, mx)) {
+                        popc = true;
+                        goto layer_done;
+                    }
+                }
                 // R31: a Q32 layer's outputs are bounded by its class sums (pf_q32_bounds) before they are
                 // evaluated; the bounds of Y(l + 1) against the horizon k = t - l - 1 decide as in R30
                 if (cls == PF_Q32 && a.thr_ok && l > 0) {
@@ -442,6 +550,8 @@ __global__ void __launch_bounds__(T, PfCfg<T>::kMinBlocks) pre_fused_kernel(cons
                     pf_body_str<T, 0, kPfStrHalo<T>>(in, out, p.L[l].nu, w0, b0, a.ymax, H, mn, mx);
                 else
                     pf_body_str<T, 32, kPfStrHalo<T>>(in, out, 32, w0, b0, a.ymax, H, mn, mx);
+                ++full_fma;
+            layer_done:
                 // the row's output range in one barrier: each warp publishes its (min, max) (bits of
                 // outputs >= 0, -0 as +0, so bit order is value order and equal bits are equal values); after
                 // the barrier every warp reduces the kWarps entries (slots double-buffered by layer parity)
@@ -546,7 +656,10 @@ __global__ void __launch_bounds__(T, PfCfg<T>::kMinBlocks) pre_fused_kernel(cons
             }
         }
         if (tid == 0) {
-            if (a.full_rl) atomicAdd(a.full_rl, (unsigned long long)full);
+            if (a.full_rl) {
+                atomicAdd(a.full_rl, (unsigned long long)full_fma);
+                if (popc) atomicAdd(a.full_rl + 1, 1ull);
+            }
             if (a.n_const && cst) atomicAdd(a.n_const, 1);
             if (a.dyn) {  // per-layer dynamics: histograms of the full-evaluation count and of the end layer
                 atomicAdd(a.dyn + full, 1ull);
@@ -583,6 +696,7 @@ size_t pre_fused_smem(int N, int H) {
     const int nb = N / 32 >= 512 ? 3 : 2;  // kPfBufs
     return sizeof(float) * nb * (size_t)(N + H) + 2 * sizeof(uint64_t) + 4 * sizeof(int) + 8 * sizeof(int) * (N / 32 / 32) +
            2 * sizeof(uint32_t) * (size_t)(N / 32) + sizeof(int) * kPfSurv +  // packed-row slots, survivors
+           sizeof(float) * kPfTabStride * (N / 32 / 32) +                    // R32 tables
            (nb == 3 ? 2 * sizeof(float) * kPfConstChunk : 0);                 // constant-row store sources
 }
 

@@ -13,6 +13,7 @@
 
 #include <algorithm>
 #include <cmath>
+#include <cstdlib>
 #include <string>
 #include <vector>
 
@@ -23,7 +24,7 @@ using namespace snicit;
 
 // the Python binding mirrors these structs (paper_conf_icpp_jiangh0h23_b200/_lib.py; tests/test_abi.py)
 static_assert(sizeof(snicit_options) == 60, "snicit_options layout");
-static_assert(sizeof(snicit_stats_t) == 192, "snicit_stats_t layout");
+static_assert(sizeof(snicit_stats_t) == 200, "snicit_stats_t layout");
 
 namespace {
 
@@ -285,7 +286,7 @@ static cudaError_t net_upload_common(snicit_network* net, const float* bias, con
         for (int l = 0; l < L; ++l) wb[l] = make_float2(net->plan[l].w0, bias[(int64_t)l * N]);
         e = upload(net->wb_d, wb.data(), wb.size());
     }
-    if (e == cudaSuccess) e = net->pf_full.ensure(1);
+    if (e == cudaSuccess) e = net->pf_full.ensure(2);
     if (e == cudaSuccess) e = net->counters.ensure(CNT_N);
     if (e == cudaSuccess) e = cudaMallocHost(&net->h_counters, sizeof(int) * CNT_N);
     for (int i = 0; i < 10 && e == cudaSuccess; ++i) e = cudaEventCreate(&net->ev[i]);
@@ -998,7 +999,7 @@ static snicit_status infer_core(snicit_network* net, const float* y0, int64_t ba
         return fail(SNICIT_E_INVALID_ARG, "bad eta/eps/prune_eps");
     if (opt.kernel < 0 || opt.kernel > SNICIT_KERNEL_CIRC_SMEM) return fail(SNICIT_E_INVALID_ARG, "bad kernel option");
     if (opt.post_mode < 0 || opt.post_mode > 1) return fail(SNICIT_E_INVALID_ARG, "bad post_mode");
-    if (opt.pre_fused < 0 || opt.pre_fused > 6) return fail(SNICIT_E_INVALID_ARG, "bad pre_fused");
+    if (opt.pre_fused < 0 || opt.pre_fused > 7) return fail(SNICIT_E_INVALID_ARG, "bad pre_fused");
     if (opt.pre_const < 0 || opt.pre_const > 2) return fail(SNICIT_E_INVALID_ARG, "bad pre_const");
     if (opt.res_sparse < 0 || opt.res_sparse > 1) return fail(SNICIT_E_INVALID_ARG, "bad res_sparse");
     if (opt.dyn_t < 0 || opt.dyn_t > 1) return fail(SNICIT_E_INVALID_ARG, "bad dyn_t");
@@ -1113,7 +1114,7 @@ static snicit_status infer_core(snicit_network* net, const float* y0, int64_t ba
             net->prof_layers = 1;
         }
         CUDA_TRY(cudaMemsetAsync(cnt + CNT_PFWORK, 0, 2 * sizeof(int), st));
-        CUDA_TRY(cudaMemsetAsync(net->pf_full.p, 0, sizeof(unsigned long long), st));
+        CUDA_TRY(cudaMemsetAsync(net->pf_full.p, 0, 2 * sizeof(unsigned long long), st));
         PreFusedArgs pa{};
         pa.N = N;
         pa.t = tt;
@@ -1121,7 +1122,9 @@ static snicit_status infer_core(snicit_network* net, const float* y0, int64_t ba
         pa.ymax = net->ymax;
         pa.drop = drop ? 1 : 0;
         pa.const_skip = opt.pre_fused != 2 ? 1 : 0;
-        pa.range_pred = opt.pre_fused != 6 ? 1 : 0;  // R30 (6: R26 alone, for measurement)
+        pa.range_pred = opt.pre_fused != 6 ? 1 : 0;  // R30 / R31 (6: R26 alone, for measurement)
+        // R32: packed rows (1, 3, 5), every two-valued row (7), never (2, 6: fma chains only)
+        pa.popc0 = (opt.pre_fused == 6 || opt.pre_fused == 2) ? 0 : (opt.pre_fused == 7 ? 1 : 2);
         pa.gen_str = pf_gen;
         pa.yin = cur;
         pa.ybits = y0_mode == 3 ? bits : nullptr;
@@ -1690,6 +1693,7 @@ snicit_status snicit_stats(snicit_network* net, snicit_stats_t* out) {
     }
     net->stats.pre_const_rows = 0;
     net->stats.pre_full_rows = 0;
+    net->stats.pre_popc_rows = 0;
     if (net->last_pre_const) {
         CUDA_TRY(read_counter(net, CNT_CCOUNT, &v));
         net->stats.pre_const_rows = v;
@@ -1710,9 +1714,10 @@ snicit_status snicit_stats(snicit_network* net, snicit_stats_t* out) {
     if (net->last_pre_fused) {
         CUDA_TRY(read_counter(net, CNT_PFCONST, &v));
         net->stats.pre_const_rows = v;
-        unsigned long long f = 0;
-        CUDA_TRY(cudaMemcpy(&f, net->pf_full.p, sizeof(f), cudaMemcpyDeviceToHost));
-        net->stats.pre_full_rows = (int64_t)f;
+        unsigned long long f[2] = {0, 0};
+        CUDA_TRY(cudaMemcpy(f, net->pf_full.p, sizeof(f), cudaMemcpyDeviceToHost));
+        net->stats.pre_full_rows = (int64_t)f[0];
+        net->stats.pre_popc_rows = (int64_t)f[1];
     }
     *out = net->stats;
     return SNICIT_OK;

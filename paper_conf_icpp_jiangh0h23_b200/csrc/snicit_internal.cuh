@@ -307,9 +307,12 @@ struct PreFusedArgs {
     float* ydead;                 // nullable: rows found dead (R23) get N zeros here (the caller's y_out)
     uint8_t* rconst;              // nullable: rconst[row] = 1, rval[row] = v for rows constant at t (R26)
     float* rval;
-    unsigned long long* full_rl;  // nullable: += full (non-constant) row-layer evaluations
+    unsigned long long* full_rl;  // nullable: [0] += full (non-constant) row-layer fma evaluations,
+                                  //   [1] += rows whose layer 0 ran as a popcount table (R32)
     unsigned long long* dyn;      // nullable: [t + 1] rows by full-evaluation count, [t + 1] rows by end layer
     int range_pred;               // caller: allow the range prediction (R30)
+    int popc0;                    // layer 0 of stride 1 as a popcount table (R32): 0 off, 1 every two-valued
+                                  //   row, 2 packed rows only (the bitmap is given; measured faster only there)
     int thr_ok;                   // range prediction on (R30; set by launch_pre_fused: one weight >= 0 and
     int dead_t;                   //   one bias for every layer < t); dead_t = dead_ok[t]
     int* n_const;                 // nullable: += rows that became constant

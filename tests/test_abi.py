@@ -35,13 +35,13 @@ def test_header_symbols_exported(lib):
 
 
 def test_abi_version_and_defaults(lib):
-    assert lib.snicit_abi_version() == 4
+    assert lib.snicit_abi_version() == 5
     o = _lib.default_options()
     # SDGC defaults, P:1038 / P:1138
     assert o.n_segments == 16 and abs(o.eta - 0.03) < 1e-7 and abs(o.eps - 0.03) < 1e-7
     assert o.prune_eps == 0.0 and o.drop_dead_rows == 1 and o.kernel == 0 and o.ne_interval == 64
     assert o.post_const == 1 and o.pre_fused == 1 and o.pre_const == 1
-    assert ctypes.sizeof(_lib.Options) == 60 and ctypes.sizeof(_lib.Stats) == 192
+    assert ctypes.sizeof(_lib.Options) == 60 and ctypes.sizeof(_lib.Stats) == 200
 
 
 def _load(lib, N, L, ptr, idx, val, bias, ymax=32.0, fmt=0):

@@ -19,7 +19,7 @@ import pytest
 torch = pytest.importorskip("torch")
 
 import oracle  # noqa: E402
-from paper_conf_icpp_jiangh0h23_b200 import CSR_FORMAT, SnicitNetwork, shard_capacity, shard_rows  # noqa: E402
+from paper_conf_icpp_jiangh0h23_b200 import CSR_FORMAT, SnicitNetwork, pack_rows, shard_capacity, shard_rows  # noqa: E402
 from workload import sdgc  # noqa: E402
 from workload.sdgc import Network  # noqa: E402
 
@@ -364,6 +364,49 @@ def test_range_prediction_bit_exact(N, drop):
     if N <= 16384:
         assert runs["pf1"][2]["pre_fused"] == 1 and runs["pf6"][2]["pre_fused"] == 1
         assert runs["pf1"][2]["pre_full_rows"] < runs["pf6"][2]["pre_full_rows"]
+
+
+@pytest.mark.parametrize("N", [1024, 4096, 16384])
+def test_popcount_layer0_bit_exact(N):
+    """R32: layer 0 (stride 1) of a row of zeros and one value c runs as a table lookup by window count
+    (k fmas of c from +0, in any order); on fp32 rows with pre_fused = 7, on packed rows by default.  Rows with c in {1, 0.3, 1.7, 0.02, YMAX, 1e-39 (subnormal)},
+    all-zero rows, and rows with two different non-zero values (fma chains): the uncompressed outputs equal
+    the oracle's and the run without R32 (pre_fused = 2 / 6) bit for bit; stats.pre_popc_rows counts
+    exactly the two-valued rows; the packed path (binary) runs every row through it."""
+    L = 9
+    B = 70 if N <= 4096 else 21
+    net = sdgc.gen_network(N, L, "radix")
+    rs = np.random.RandomState(N)
+    Y0 = (rs.uniform(size=(B, N)) < 0.3).astype(np.float32)
+    cs = [1.0, 0.3, 1.7, 0.02, 32.0, 1e-39]
+    for r in range(B):
+        if r % 7 < len(cs):
+            Y0[r] *= np.float32(cs[r % 7])
+    Y0[6::7] = 0.0
+    Y0[3::14, 5] = np.float32(0.5)  # a second non-zero value: not two-valued (c = 0.02 rows)
+    two_valued = np.array([len(np.unique(y[y != 0])) <= 1 for y in Y0])
+    assert 0 < two_valued.sum() < B
+    plain = oracle.layers_f32(net, Y0)
+    with SnicitNetwork.from_network(net) as g:
+        g.set_stream(torch.cuda.current_stream())
+        Y1, c1, st1 = _infer(g, Y0, L, pre_fused=7)  # R32 on fp32 rows too
+        assert st1["pre_fused"] == 1 and st1["pre_popc_rows"] == int(two_valued.sum())
+        assert np.array_equal(Y1, plain) and np.array_equal(c1, oracle.categories(plain))
+        for pf in (1, 2, 6):  # 1: R32 on packed rows only
+            Y2, c2, st2 = _infer(g, Y0, L, pre_fused=pf)
+            assert st2["pre_popc_rows"] == 0 and np.array_equal(Y2, plain), pf
+        # SNICIT path (t < L) agrees with the per-layer pre phase
+        Y3, c3, _ = _infer(g, Y0, 4, pre_fused=7)
+        Y4, c4, _ = _infer(g, Y0, 4, pre_fused=0)
+        assert np.array_equal(Y3, Y4) and np.array_equal(c3, c4)
+        # packed binary rows: every row takes R32, outputs equal the fp32 binary rows'
+        Yb = (Y0 != 0).astype(np.float32)
+        bits = torch.from_numpy(pack_rows(Yb).view(np.int32)).cuda()
+        outp = torch.empty((B, N), dtype=torch.float32, device="cuda")
+        g.infer_packed(bits, t=L, s=32, y_out=outp)
+        stp = g.stats()
+        assert stp["pre_popc_rows"] == B
+        assert np.array_equal(outp.cpu().numpy(), oracle.layers_f32(net, Yb))
 
 
 def test_dynamics_log(tmp_path):
