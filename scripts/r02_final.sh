@@ -11,6 +11,11 @@ echo "pytest rc=$?" >> gpurun_out/${tag}_pytest_gpu.txt
 timeout 300 python -c "import __graft_entry__ as g; g.smoke()" > gpurun_out/${tag}_smoke.txt 2>&1
 timeout 900 python bench.py > gpurun_out/${tag}_bench.json 2> gpurun_out/${tag}_bench.err
 timeout 600 python bench.py --impl reference --steps 2 --warmup 1 > gpurun_out/${tag}_ref.json 2> gpurun_out/${tag}_ref.err
+for c in C1 C2 C4 C5; do
+  timeout 600 python bench.py --config $c --no-cpu-baseline > gpurun_out/${tag}_bench_$c.json 2> gpurun_out/${tag}_bench_$c.err
+done
+timeout 300 python scripts/popc_timing.py > gpurun_out/${tag}_popc_C3.txt 2>&1
+timeout 300 python scripts/popc_timing.py --config C2 > gpurun_out/${tag}_popc_C2.txt 2>&1
 P="python scripts/profile_step.py"
 ncu --metrics gpu__time_duration.sum --clock-control none --profile-from-start off --csv \
     --log-file gpurun_out/${tag}_launches_C3.csv $P --config C3 > /dev/null 2>&1

@@ -87,4 +87,24 @@ with SnicitNetwork.from_network(net) as g:
     st = g.stats()
     torch.cuda.synchronize()
 print("sparse residues: sparse row-layers", st["res_sparse_rl"], "sum", float(out.sum()))
+# round 2 (late): range prediction (R30/R31) near the fixed point, popcount layer 0 (R32) on packed and fp32
+# rows, TMA stores of constant rows, Y(t) kept in y_out (recovery skip), per-layer path with R30
+for N, B, kw in ((16384, 24, {}), (16384, 24, dict(pre_fused=7)), (4096, 200, dict(pre_fused=7)),
+                 (65536, 6, {}), (1024, 300, dict(pre_fused=0, pre_const=1))):
+    net = sdgc.gen_network(N, 40, "radix")
+    rs = np.random.RandomState(N)
+    Yh = (-sdgc.SDGC_BIAS[N] + rs.uniform(-0.05, 0.05, size=(B, 1)) + rs.uniform(-0.03, 0.03, size=(B, N)))
+    Yh = Yh.clip(0, None).astype(np.float32)
+    Yh[::3] = sdgc.gen_inputs(N, B)[::3]
+    Y0 = torch.from_numpy(Yh).cuda()
+    out = torch.empty_like(Y0)
+    with SnicitNetwork.from_network(net) as g:
+        g.set_stream(torch.cuda.current_stream())
+        g.infer(Y0, t=30, s=32, y_out=out, **kw)
+        cats = g.categories()
+        bits = torch.from_numpy(pack_rows((Yh != 0).astype(np.float32)).view(np.int32)).cuda()
+        g.infer_packed(bits, t=30, s=32, y_out=out)
+        cats2 = g.categories()
+        torch.cuda.synchronize()
+    print("range/popc", N, B, kw, "categories", len(cats), len(cats2), "sum", float(out.sum()))
 print("sanitize run done")
