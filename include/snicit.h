@@ -30,7 +30,7 @@
 extern "C" {
 #endif
 
-#define SNICIT_ABI_VERSION 5
+#define SNICIT_ABI_VERSION 6
 
 typedef struct snicit_network snicit_network; /* opaque: owns device copies of W, b + workspace */
 
@@ -311,6 +311,16 @@ snicit_status snicit_debug_layer(snicit_network* net, int32_t layer, const float
  * out^k(v) == 0 (-1 if none), k = 1..kmax (kmax <= 32).  Returns 1 if either table is active, 0 if
  * neither (or w0 < 0), SNICIT_E_INVALID_ARG for bad arguments.  Host pointers, kmax floats each. */
 int32_t snicit_debug_range_tables(float w0, float b0, float ymax, int32_t kmax, float* hi, float* lo);
+
+/* Test hook (host only, no GPU needed): the load-time schedule of the general-CSC row-interleaved kernel
+ * (kernels_gen.cu) for one layer of n_neurons outputs with K inputs each.
+ * cols: n_neurons * K input indices, column-major per output (entry n of output j at j * K + n, chain
+ * order).  Writes the number of outputs one warp instruction covers for this N (G = 2, 4 or
+ * 16 -- tiles of 128 / G rows -- or 0 = kernel not used) to *rows_per_tile and the mean number of
+ * shared-memory wavefronts per quarter-warp tap of the schedule to *cost (1.0 = conflict-free; G = 2 and
+ * G = 4 read whole lines and are always 1.0).  Returns SNICIT_OK or SNICIT_E_INVALID_ARG. */
+snicit_status snicit_debug_gen_schedule(int32_t n_neurons, int32_t K, const int32_t* cols, int32_t* rows_per_tile,
+                                        double* cost);
 
 /* 1 if layer l is eligible for the circulant kernel, 0 if not, < 0 on error. */
 int32_t snicit_layer_is_circulant(const snicit_network* net, int32_t layer);

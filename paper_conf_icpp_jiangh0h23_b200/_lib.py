@@ -24,7 +24,8 @@ EXPORTED = ["snicit_default_options", "snicit_load_network", "snicit_set_stream"
             "snicit_categories", "snicit_stats", "snicit_debug_clustering", "snicit_debug_layer",
             "snicit_layer_is_circulant", "snicit_free_network", "snicit_last_error", "snicit_abi_version",
             "snicit_layer_profile", "snicit_load_network_circulant", "snicit_infer_packed",
-            "snicit_categories_device", "snicit_dynamics", "snicit_debug_range_tables"]
+            "snicit_categories_device", "snicit_dynamics", "snicit_debug_range_tables",
+            "snicit_debug_gen_schedule"]
 
 
 class Options(ctypes.Structure):
@@ -100,6 +101,8 @@ def load_library(path: str = LIB_PATH):
     L.snicit_debug_layer.restype = i32
     L.snicit_debug_range_tables.argtypes = [f32, f32, f32, i32, P, P]
     L.snicit_debug_range_tables.restype = i32
+    L.snicit_debug_gen_schedule.argtypes = [i32, i32, P, P, P]
+    L.snicit_debug_gen_schedule.restype = i32
     L.snicit_layer_is_circulant.argtypes = [P, i32]
     L.snicit_layer_is_circulant.restype = i32
     L.snicit_free_network.argtypes = [P]

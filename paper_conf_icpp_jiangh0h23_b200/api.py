@@ -25,6 +25,21 @@ def range_tables(w0: float, b0: float, ymax: float, kmax: int = 32):
     return hi, lo, bool(r)
 
 
+def gen_schedule(cols: np.ndarray):
+    """snicit_debug_gen_schedule (general-CSC kernel): (rows_per_tile, cost) of the
+    load-time quad schedule for one layer given as an N x K array of input indices (chain order per
+    output).  cost = mean shared-memory wavefronts per tap (1.0 = conflict-free).  Host only."""
+    L = load_library()
+    c = np.ascontiguousarray(cols, dtype=np.int32)
+    if c.ndim != 2:
+        raise ValueError("cols must be N x K")
+    rl = ctypes.c_int32(0)
+    cost = ctypes.c_double(0.0)
+    check(L.snicit_debug_gen_schedule(int(c.shape[0]), int(c.shape[1]), c.ctypes.data, ctypes.byref(rl),
+                                      ctypes.byref(cost)), "snicit_debug_gen_schedule")
+    return int(rl.value), float(cost.value)
+
+
 def _is_cuda_tensor(x) -> bool:
     return hasattr(x, "is_cuda") and bool(x.is_cuda)
 

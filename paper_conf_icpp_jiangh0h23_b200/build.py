@@ -7,7 +7,7 @@ import subprocess
 HERE = os.path.dirname(os.path.abspath(__file__))
 CSRC = os.path.join(HERE, "csrc")
 OUT = os.path.join(HERE, "lib", "libsnicit.so")
-SOURCES = ["snicit_api.cu", "kernels_layer.cu", "kernels_pre_fused.cu", "kernels_pre_pair.cu", "kernels_pre_cluster.cu", "kernels_const.cu", "kernels_circ.cu", "kernels_circ_seg.cu", "kernels_circ_col.cu", "kernels_post.cu", "kernels_convert.cu"]
+SOURCES = ["snicit_api.cu", "kernels_layer.cu", "kernels_gen.cu", "kernels_pre_fused.cu", "kernels_pre_pair.cu", "kernels_pre_cluster.cu", "kernels_const.cu", "kernels_circ.cu", "kernels_circ_seg.cu", "kernels_circ_col.cu", "kernels_post.cu", "kernels_convert.cu"]
 HEADERS = ["snicit_internal.cuh", os.path.join("..", "..", "include", "snicit.h")]
 NVCC_FLAGS = ["-gencode", "arch=compute_100a,code=sm_100a", "-O3", "-lineinfo", "-std=c++17",
               "-Xcompiler", "-fPIC", "-shared"]

@@ -406,8 +406,17 @@ static cudaError_t launch_ell_m(const LayerArgs& a, int max_rows, int num_sms, c
     return launch_ell_t<MODE, 1, true>(a, max_rows, num_sms, st);
 }
 
+bool gen_enabled() {
+    static const bool on = [] {
+        const char* e = getenv("SNICIT_GEN");  // "0": the previous ELL kernels (A/B experiments only)
+        return !(e && e[0] == '0');
+    }();
+    return on;
+}
+
 cudaError_t launch_layer_ell(const LayerArgs& a, int mode, int max_rows, int num_sms, cudaStream_t st) {
     if (max_rows <= 0) return cudaSuccess;
+    if (a.gidx && gen_enabled()) return launch_layer_gen(a, mode, max_rows, num_sms, st);
     switch (mode) {
         case MODE_PLAIN: return launch_ell_m<MODE_PLAIN>(a, max_rows, num_sms, st);
         case MODE_CENTROID: return launch_ell_m<MODE_CENTROID>(a, max_rows, num_sms, st);

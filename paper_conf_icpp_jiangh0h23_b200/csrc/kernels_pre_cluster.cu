@@ -46,11 +46,13 @@ struct CfLayer {
     int nu;
     int flags;  // cls | dead_next << 4 | ymax_fixed << 5
 };
+constexpr int kCfMaxLayers = kPfMaxLayers - 20;  // (parameter space: the R30 tables below)
 struct CfParams {
     PreFusedArgs a;
     int Hh;        // W-partition halo (floats)
     int pad;
-    CfLayer L[kPfMaxLayers + 1];  // L[t]: sentinel (the output of layer t-1 is stored in the W partition)
+    float thr_hi[kRangeK], thr_lo[kRangeK];  // R30 horizon tables (kernels_const.cu range_tables)
+    CfLayer L[kCfMaxLayers + 1];  // L[t]: sentinel (the output of layer t-1 is stored in the W partition)
 };
 static_assert(sizeof(CfParams) <= 32764, "kernel parameter space");
 
@@ -396,9 +398,9 @@ __global__ void __launch_bounds__(kCT, kCfMinBlocks) pre_cluster_kernel(const __
     uint64_t* bar = reinterpret_cast<uint64_t*>(buf + 2 * BS);          // [2] row loads
     uint32_t* s_bits = reinterpret_cast<uint32_t*>(bar + 2);            // [(kCS + 1024) / 32] packed row (16 B aligned)
     int* s_pos = reinterpret_cast<int*>(s_bits + (kCS + 1024) / 32);    // [2] row position by row parity
-    int* s_ok = s_pos + 2;                                              // [2][G * kCWp] warp votes
-    float* s_ref = reinterpret_cast<float*>(s_ok + 2 * G * kCWp);       // [2][G * kCWp] warp references
-    uint32_t* s_base = reinterpret_cast<uint32_t*>(s_ref + 2 * G * kCWp);  // [2][G] buffer b of rank h
+    unsigned* s_vmn = reinterpret_cast<unsigned*>(s_pos + 2);           // [2][G * kCWp] warp output minima (bits)
+    unsigned* s_vmx = s_vmn + 2 * G * kCWp;                             // [2][G * kCWp] warp output maxima
+    uint32_t* s_base = reinterpret_cast<uint32_t*>(s_vmx + 2 * G * kCWp);  // [2][G] buffer b of rank h
     int* s_surv = reinterpret_cast<int*>(s_base + 2 * G);               // [kCSurv]
     const int tid = threadIdx.x;
     const int r = (int)cluster_ctarank();
@@ -527,31 +529,56 @@ __global__ void __launch_bounds__(kCT, kCfMinBlocks) pre_cluster_kernel(const __
                     else
                         cf_body_cstr<RT_C>(in, r, nu, N / nu, w0, b0, a.ymax, rt, mn, mx, ilog2i(nu) - ilog2i(G));
                 }
-                // "all outputs equal" over the whole row: every warp publishes (vote, value) to every rank
+                // the row's output range: every warp publishes its (min, max) (bits of outputs >= 0, -0 as
+                // +0: bit order is value order, equal bits are equal values) to every rank
                 {
-                    const float ref = __shfl_sync(0xffffffffu, mn, 0);
-                    const bool ok = __all_sync(0xffffffffu, mn >= ref && mx <= ref);
+                    const unsigned wmn = __reduce_min_sync(0xffffffffu, __float_as_uint(mn + 0.0f));
+                    const unsigned wmx = __reduce_max_sync(0xffffffffu, __float_as_uint(mx + 0.0f));
                     if ((tid & 31) == 0) {
                         const int slot = (l & 1) * G * kCWp + r * kCWp + (tid >> 5);
                         for (int h = 0; h < G; ++h) {
-                            st_cl_u32(mapa_u32(smem_u32(s_ok + slot), (uint32_t)h), ok ? 1u : 0u);
-                            st_cl_f32(mapa_u32(smem_u32(s_ref + slot), (uint32_t)h), ref);
+                            st_cl_u32(mapa_u32(smem_u32(s_vmn + slot), (uint32_t)h), wmn);
+                            st_cl_u32(mapa_u32(smem_u32(s_vmx + slot), (uint32_t)h), wmx);
                         }
                     }
                 }
-                cluster_barrier();  // every rank's outputs, votes (and the next row position) delivered
-                bool all_eq = true;
-                const float o0 = s_ref[(l & 1) * G * kCWp];
-#pragma unroll 8
-                for (int w = 0; w < G * kCWp; ++w)
-                    all_eq = all_eq && s_ok[(l & 1) * G * kCWp + w] && s_ref[(l & 1) * G * kCWp + w] == o0;
+                cluster_barrier();  // every rank's outputs, ranges (and the next row position) delivered
+                unsigned rmn, rmx;
+                {
+                    const int ln = tid & 31;
+                    unsigned m0 = 0xffffffffu, m1 = 0u;
+                    for (int w = ln; w < G * kCWp; w += 32) {
+                        m0 = min(m0, s_vmn[(l & 1) * G * kCWp + w]);
+                        m1 = max(m1, s_vmx[(l & 1) * G * kCWp + w]);
+                    }
+                    rmn = __reduce_min_sync(0xffffffffu, m0);
+                    rmx = __reduce_max_sync(0xffffffffu, m1);
+                }
                 ++full;
                 cur ^= 1;
-                if (all_eq) {
-                    v = o0;
+                if (rmn == rmx) {  // constant row (R26) or dead (R23)
+                    v = __uint_as_float(rmn);
                     if (a.const_skip) cst = true;
                     if (v == 0.0f && a.drop && dead_next) {
                         dead = true;
+                        break;
+                    }
+                }
+                // range prediction (R30, exact; kernels_pre_fused.cu): after k = t - l - 1 more layers every
+                // element lies in [out^k(min), out^k(max)]; min >= thr_hi[k-1]: Y(t) is the constant row YMAX,
+                // max <= thr_lo[k-1]: Y(t) is zero
+                const int k2 = a.t - l - 1;
+                if (a.thr_ok && k2 > 0) {
+                    const int kk = min(k2, kRangeK);
+                    if (__uint_as_float(rmn) >= p.thr_hi[kk - 1]) {
+                        v = a.ymax;
+                        cst = true;
+                        break;
+                    }
+                    if (__uint_as_float(rmx) <= p.thr_lo[kk - 1]) {
+                        v = 0.0f;
+                        cst = true;
+                        if (a.drop && a.dead_t) dead = true;
                         break;
                     }
                 }
@@ -674,7 +701,7 @@ static cudaError_t launch_cl(const CfParams& p, int num_sms, cudaStream_t st) {
 }
 
 cudaError_t launch_pre_cluster(const PreFusedArgs& a, const PreFusedLayer* layers, int num_sms, cudaStream_t st) {
-    if (a.t < 1 || a.t > kPfMaxLayers || !pre_cluster_supported(a.N)) return cudaErrorInvalidValue;
+    if (a.t < 1 || a.t > kCfMaxLayers || !pre_cluster_supported(a.N)) return cudaErrorInvalidValue;
     static thread_local CfParams p;  // 32 KB: not on the stack
     p.a = a;
     int Hh = 64;
@@ -688,6 +715,9 @@ cudaError_t launch_pre_cluster(const PreFusedArgs& a, const PreFusedLayer* layer
         if (cls == CF_WSTR) Hh = Hh > 31 * layers[l].nu ? Hh : 31 * layers[l].nu;
     }
     p.L[a.t] = CfLayer{0.f, 0.f, 1, CF_NU1};
+    // range prediction horizon tables (R30, kernels_const.cu), as launch_pre_fused
+    p.a.thr_ok = a.const_skip && a.range_pred && range_tables(layers, a.t, a.ymax, p.thr_hi, p.thr_lo);
+    p.a.dead_t = layers[a.t - 1].dead_next;
     p.Hh = (Hh + 127) / 128 * 128;  // bulk copies of the halo (fp32 and packed bits) in 16-byte multiples
     if (p.Hh > 1024) return cudaErrorInvalidValue;
     if (a.ybits && !((p.L[0].flags & 15) == CF_NU1 || (p.L[0].flags & 15) == CF_WSTR)) return cudaErrorInvalidValue;

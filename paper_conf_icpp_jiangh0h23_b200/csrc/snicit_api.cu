@@ -105,6 +105,12 @@ struct snicit_network {
     DevBuf<uint8_t> len_d;
     DevBuf<float> wtab_d;
     std::vector<float> wtab_h;  // host copy (weights passed as kernel parameters)
+    // general-CSC row-interleaved kernel schedules (kernels_gen.cu), per layer with plan[l].gen
+    int grl = 0;                  // outputs per warp instruction G (1 / 4 / 16), 0 = kernel unavailable
+    DevBuf<uint16_t> gidx_d;
+    DevBuf<float> gval_d;
+    DevBuf<uint16_t> gsched_d;
+    double gen_cost = 0.0;        // mean shared-memory wavefronts per tap of the schedules (1 = none lost)
     DevBuf<float> bias_d;
     DevBuf<PostLayer> post_layers_d;  // per-layer descriptors for the fused post-convergence kernels
     DevBuf<PreFusedLayer> pf_layers_d;  // per-layer descriptors of the row-resident pre-convergence kernel
@@ -328,6 +334,9 @@ void snicit_free_network(snicit_network* net) {
     net->val_d.release();
     net->len_d.release();
     net->wtab_d.release();
+    net->gidx_d.release();
+    net->gval_d.release();
+    net->gsched_d.release();
     net->bias_d.release();
     net->Ya.release();
     net->Yb.release();
@@ -418,6 +427,13 @@ snicit_status snicit_load_network(int32_t N, int32_t L, snicit_format fmt, const
     std::vector<std::vector<uint8_t>> lay_len(L);
     std::vector<float> wtab;
     std::vector<uint8_t> mark(N, 0);
+    net->grl = gen_rows_per_tile(N);
+    size_t gen_total = 0;
+    int gen_layers = 0;
+    double gen_cost_sum = 0.0;
+    std::vector<uint16_t> g_idx;
+    std::vector<float> g_val;
+    std::vector<uint16_t> g_sched;
     for (int l = 0; l < L; ++l) {
         const int64_t* p = ptr + (int64_t)l * (N + 1);
         if (l > 0 && p[0] != ptr[(int64_t)l * (N + 1) - 1]) {
@@ -527,6 +543,23 @@ snicit_status snicit_load_network(int32_t N, int32_t L, snicit_format fmt, const
             }
             if (ragged) lay_len[l][j] = (uint8_t)cidx[j].size();
         }
+        // general-CSC kernel schedule: every non-circulant layer; circulant layers too while the arrays stay
+        // small (SNICIT_KERNEL_ELL runs them through the same kernel in tests)
+        pl.gen = false;
+        if (net->grl > 0 && (pl.kind == 0 || (size_t)L * N * 32 <= ((size_t)16 << 20))) {
+            pl.gen = true;
+            pl.gkp = (K + 3) & ~3;
+            if (pl.gkp == 0) pl.gkp = 4;
+            pl.gen_off = gen_total;
+            gen_total += (size_t)N * ((pl.gkp + 7) & ~7);
+            g_idx.resize(gen_total);
+            if (!pl.uniform) g_val.resize(gen_total);
+            if (net->grl == 16) g_sched.resize((size_t)(gen_layers + 1) * N);
+            uint16_t* sch = net->grl == 16 ? g_sched.data() + (size_t)gen_layers * N : nullptr;
+            gen_cost_sum += gen_build_layer(N, net->grl, pl.gkp, cidx, cval, g_idx.data() + pl.gen_off,
+                                            pl.uniform ? nullptr : g_val.data() + pl.gen_off, sch);
+            ++gen_layers;
+        }
     }
     net_bias_flags(net, bias);
     // ---- device (validation above needs no GPU, so bad input is reported on any host)
@@ -568,6 +601,18 @@ snicit_status snicit_load_network(int32_t N, int32_t L, snicit_format fmt, const
                 if (net->plan[l].ragged) std::copy(lay_len[l].begin(), lay_len[l].end(), alll.begin() + (size_t)l * N);
             e = up(net->len_d, alll.data(), alll.size());
         }
+    }
+    if (e == cudaSuccess && gen_layers > 0) {
+        net->gen_cost = gen_cost_sum / gen_layers;
+        // weights of non-uniform layers: fill uniform layers' ranges too (one array for all layers)
+        if (!g_val.empty()) g_val.resize(gen_total, 0.0f);
+        e = up(net->gidx_d, g_idx.data(), gen_total);
+        if (e == cudaSuccess && !g_val.empty()) e = up(net->gval_d, g_val.data(), gen_total);
+        if (e == cudaSuccess && !g_sched.empty()) e = up(net->gsched_d, g_sched.data(), g_sched.size());
+        // per-layer schedule slot (sched arrays are indexed by the order of gen layers)
+        int gi = 0;
+        for (int l = 0; l < L; ++l)
+            if (net->plan[l].gen) net->plan[l].gsched_idx = gi++;
     }
     if (e == cudaSuccess) e = net_upload_common(net, bias, wtab);
     if (e != cudaSuccess) {
@@ -661,6 +706,30 @@ int32_t snicit_debug_range_tables(float w0, float b0, float ymax, int32_t kmax, 
     return ok ? 1 : 0;
 }
 
+snicit_status snicit_debug_gen_schedule(int32_t N, int32_t K, const int32_t* cols, int32_t* rows_per_tile,
+                                        double* cost) {
+    if (N < 1 || K < 1 || K > 255 || !cols || !rows_per_tile || !cost)
+        return fail(SNICIT_E_INVALID_ARG, "bad arguments");
+    std::vector<std::vector<int32_t>> cidx(N);
+    std::vector<std::vector<float>> cval(N);
+    for (int j = 0; j < N; ++j)
+        for (int n = 0; n < K; ++n) {
+            const int32_t k = cols[(size_t)j * K + n];
+            if (k < 0 || k >= N) return fail(SNICIT_E_INVALID_ARG, "index out of range");
+            cidx[j].push_back(k);
+            cval[j].push_back(1.0f);
+        }
+    const int rl = gen_rows_per_tile(N);
+    *rows_per_tile = rl;
+    *cost = 0.0;
+    if (rl == 0) return SNICIT_OK;
+    const int kp = (K + 3) & ~3;
+    std::vector<uint16_t> idx((size_t)N * ((kp + 7) & ~7));
+    std::vector<uint16_t> sched(N);
+    *cost = gen_build_layer(N, rl, kp, cidx, cval, idx.data(), nullptr, sched.data());
+    return SNICIT_OK;
+}
+
 int32_t snicit_layer_is_circulant(const snicit_network* net, int32_t l) {
     if (!net || l < 0 || l >= net->L) return -1;
     return net->plan[l].kind != 0 ? 1 : 0;
@@ -685,6 +754,13 @@ static LayerArgs layer_args(snicit_network* net, int l, bool force_ell) {
             a.idx32 = net->idx32_d.p + pl.ell_off;
         a.val = pl.uniform ? nullptr : net->val_d.p + pl.ell_off;
         a.len = pl.ragged ? net->len_d.p + (size_t)l * net->N : nullptr;
+    }
+    if (pl.gen && net->grl > 0) {
+        a.gidx = net->gidx_d.p + pl.gen_off;
+        a.gval = pl.uniform ? nullptr : net->gval_d.p + pl.gen_off;
+        a.gsched = net->grl == 16 ? net->gsched_d.p + (size_t)pl.gsched_idx * net->N : nullptr;
+        a.grl = net->grl;
+        a.gkp = pl.gkp;
     }
     a.w0 = pl.w0;
     a.uniform_bias = pl.ubias ? 1 : 0;
@@ -1319,7 +1395,11 @@ static snicit_status infer_core(snicit_network* net, const float* y0, int64_t ba
         float* c_nxt = net->cbuf1.p;
         float* yh_cur = yhat;
         float* yh_nxt = yhat_other;
-        const bool fused = opt.post_mode == 0 && N <= post_fused_max_n();
+        // general (non-circulant) post layers with a general-CSC kernel schedule run per layer: the tiled
+        // kernel (kernels_gen.cu) beats the fused trajectory kernels' per-row gathers on them
+        bool gen_post = false;
+        for (int l = tt; l < L; ++l) gen_post |= !use_circ(net, l, opt.kernel) && net->plan[l].gen && net->grl > 0;
+        const bool fused = opt.post_mode == 0 && N <= post_fused_max_n() && !(gen_post && gen_enabled());
         // fused mode: no host read of the residue count (the kernels read it on the device and the
         // a_c rows are written only when residue rows exist), so the stream is never stalled here;
         // res_host = 1 means "maybe"

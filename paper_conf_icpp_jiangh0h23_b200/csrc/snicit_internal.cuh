@@ -151,6 +151,12 @@ struct LayerArgs {
     // it leaves with layer index thr_layer = t - 1.  thr_hi = +inf, thr_lo = -1: off
     float thr_hi, thr_lo;
     int thr_layer, thr_dead;
+    // general-CSC row-interleaved kernel (kernels_gen.cu): load-time schedule of this layer, or goff NULL
+    const uint16_t* gidx;   // per-tap input ids (N * gkp, padded taps -> the zero slot N)
+    const float* gval;      // per-tap weights in the same layout (NULL: uniform w0)
+    const uint16_t* gsched; // G = 16: output id of each quad slot
+    int grl;                // outputs per warp instruction G (2, 4, 16)
+    int gkp;                // taps per column, padded to a multiple of 4 (arrays hold ceil(gkp / 8) blocks)
 };
 
 struct LayerPlan {
@@ -164,6 +170,10 @@ struct LayerPlan {
     float w0;
     size_t ell_off; // element offset of this layer in the ELL arrays
     size_t w_off;   // offset in the per-n weight table
+    bool gen;       // has a schedule for the general-CSC row-interleaved kernel (kernels_gen.cu)
+    int gkp;        // its taps per column (K padded to a multiple of 4)
+    size_t gen_off; // entry offset of this layer in the schedule arrays (N * gkp entries)
+    int gsched_idx; // RL = 8: index of this layer's N-entry block of quad slots
 };
 
 // Epilogue of one output q of one row (acc = the fma chain, b = bias[q]).  `valid` == false marks a
@@ -189,6 +199,12 @@ cudaError_t blocks_per_sm(const void* kern, int threads, size_t smem, int* out);
 
 // launchers (kernels_circ.cu / kernels_layer.cu); return cudaError_t of the launch
 cudaError_t launch_layer_ell(const LayerArgs& a, int mode, int max_rows, int num_sms, cudaStream_t st);
+// general-CSC row-interleaved kernel (kernels_gen.cu)
+int gen_rows_per_tile(int N);
+bool gen_enabled();  // SNICIT_GEN != "0" (A/B switch)
+double gen_build_layer(int N, int G, int Kp, const std::vector<std::vector<int32_t>>& cidx,
+                       const std::vector<std::vector<float>>& cval, uint16_t* idx, float* w, uint16_t* sched);
+cudaError_t launch_layer_gen(const LayerArgs& a, int mode, int max_rows, int num_sms, cudaStream_t st);
 cudaError_t launch_layer_circ(const LayerArgs& a, int mode, int max_rows, int num_sms, cudaStream_t st);
 bool circ_supported(int N, int K, int nu);
 // segmented circulant kernel (rows too large for kernels_circ.cu), kernels_circ_seg.cu

@@ -26,18 +26,25 @@ p.add_argument("--pre-fused", type=int, default=1)
 a = p.parse_args()
 c = sdgc.CONFIGS[a.config]
 B = a.batch or c["B"]
-Y0 = sdgc.gen_inputs(c["N"], B)
-if a.mode == "radix" and c["N"] >= 16384:  # compact circulant ABI (the CSC would be 8-32 GB)
+extra = {}
+if a.config == "C5":  # config 5: medium MLP (random K = 26 columns, per-entry weights), s = 128, n = N
+    Y0 = sdgc.gen_medium_inputs(c["N"], B)
+    g = SnicitNetwork.from_network(sdgc.gen_medium_network(c["N"], c["L"]))
+    extra = dict(n_segments=0)
+    a.s = 128
+elif a.mode == "radix" and c["N"] >= 16384:  # compact circulant ABI (the CSC would be 8-32 GB)
+    Y0 = sdgc.gen_inputs(c["N"], B)
     cn = sdgc.gen_circulant(c["N"], c["L"])
     g = SnicitNetwork.circulant(cn.N, cn.L, cn.nu, cn.w, cn.bias, cn.ymax)
 else:
+    Y0 = sdgc.gen_inputs(c["N"], B)
     net = sdgc.gen_network(c["N"], c["L"], a.mode)
     g = SnicitNetwork.from_network(net)
 st = torch.cuda.Stream()
 g.set_stream(st)
 y0 = torch.from_numpy(Y0).cuda()
 out = torch.empty_like(y0)
-opt = default_options(kernel={"auto": KERNEL_AUTO, "ell": KERNEL_ELL, "circ": KERNEL_CIRC}[a.kernel], pre_fused=a.pre_fused)
+opt = default_options(kernel={"auto": KERNEL_AUTO, "ell": KERNEL_ELL, "circ": KERNEL_CIRC}[a.kernel], pre_fused=a.pre_fused, **extra)
 for _ in range(2):
     g.infer(y0, t=a.t, s=a.s, options=opt, y_out=out)
     g.num_categories()

@@ -35,7 +35,7 @@ def test_header_symbols_exported(lib):
 
 
 def test_abi_version_and_defaults(lib):
-    assert lib.snicit_abi_version() == 5
+    assert lib.snicit_abi_version() == 6
     o = _lib.default_options()
     # SDGC defaults, P:1038 / P:1138
     assert o.n_segments == 16 and abs(o.eta - 0.03) < 1e-7 and abs(o.eps - 0.03) < 1e-7
@@ -128,3 +128,52 @@ def test_range_tables_rejects_bad_args():
     with pytest.raises(Exception):
         range_tables(0.0625, -0.3, 32.0, 33)
     assert not range_tables(-0.0625, -0.3, 32.0, 4)[2]  # w0 < 0: outputs not monotone, tables off
+
+
+def _quad_cost(cols: np.ndarray) -> float:
+    """Mean shared-memory wavefronts per tap when outputs 4i..4i+3 share a warp instruction and input k
+    lives in bank group k % 4 (the RL = 8 tile), identical inputs broadcast: the unscheduled baseline."""
+    N, K = cols.shape
+    tot = 0
+    for g in range(N // 4):
+        for n in range(K):
+            ks = set(int(k) for k in cols[4 * g:4 * g + 4, n])
+            m = [0, 0, 0, 0]
+            for k in ks:
+                m[k % 4] += 1
+            tot += max(m)
+    return tot / (N // 4 * K)
+
+
+def _layer_cols(net, l):
+    N = net.N
+    p = net.ptr[l * (N + 1):(l + 1) * (N + 1)]
+    return np.stack([net.idx[p[j]:p[j + 1]] for j in range(N)]).astype(np.int32)
+
+
+def test_gen_schedule_quads(lib):
+    """General-CSC kernel schedule: the tile shape follows N, whole-line reads
+    (G = 2, 4) never conflict, shift-structured layers get conflict-free quads (radix: inputs of the outputs
+    of a quad differ mod 4 at every tap), a random permutation of them (perm) nearly so, and unstructured
+    random columns beat the unscheduled quads."""
+    from paper_conf_icpp_jiangh0h23_b200.api import gen_schedule
+    from workload import sdgc
+    assert gen_schedule(np.zeros((256, 4), np.int32))[0] == 2
+    assert gen_schedule(np.zeros((1024, 4), np.int32)) == (4, 1.0)
+    for N, mode in [(2048, "radix"), (4096, "radix"), (4096, "perm"), (2048, "random")]:
+        net = sdgc.gen_network(N, 3, mode)
+        for l in range(3):
+            cols = _layer_cols(net, l)
+            rl, cost = gen_schedule(cols)
+            assert rl == 16, (N, rl)
+            base = _quad_cost(cols)
+            if mode == "radix":
+                assert cost == 1.0
+            elif mode == "perm":
+                assert cost < 1.25 and cost < base - 0.5, (cost, base)
+            else:
+                assert cost < base - 0.2, (cost, base)
+    rl, cost = gen_schedule(_layer_cols(sdgc.gen_medium_network(256, 2), 0))
+    assert rl == 2 and cost == 1.0
+    with pytest.raises(Exception):
+        gen_schedule(np.full((64, 3), 64, np.int32))  # index out of range
