@@ -206,6 +206,33 @@ class ClockSampler:
                 "power_w_max": max(pw) if pw else None}
 
 
+def gen_kernel_info(net):
+    """(G, wavefronts per tap) of the general-CSC kernel for this network (kernels_gen.cu, DESIGN.md section
+    7): G = outputs per warp instruction (0: the previous ELL kernels; SNICIT_GEN=0 forces those), and the
+    load-time schedule's mean shared-memory wavefronts per quarter-warp tap over the first layers."""
+    if os.environ.get("SNICIT_GEN", "1") == "0":
+        return 0, None
+    from paper_conf_icpp_jiangh0h23_b200.api import gen_schedule
+    N = net.N
+    costs, G = [], 0
+    for l in range(min(3, net.L)):
+        p = net.ptr[l * (N + 1):(l + 1) * (N + 1)]
+        lens = np.diff(p)
+        if lens.min() != lens.max():
+            break
+        cols = net.idx[p[0]:p[-1]].reshape(N, -1)
+        G, cst = gen_schedule(cols)
+        costs.append(cst)
+    return G, (float(np.mean(costs)) if costs else None)
+
+
+def gen_kernel_label(G):
+    if G:
+        return (f"layer_gen_kernel (general CSC, a1: row-interleaved tile of {128 // G} rows, "
+                f"{G} outputs x 4 rows per lane group per warp instruction)")
+    return "layer_ell_kernel (general CSC, a1)"
+
+
 def committed_traffic(tag: str):
     """Mean DRAM bytes per launch of the dominant kernel from the latest committed ncu capture of this
     configuration (profiles/rNN_traffic_<tag>.json, written by scripts/traffic.py), or (None, None)."""
@@ -421,16 +448,20 @@ def general_study(args, dev, stream, peak):
     kms, kb = float(pr["ms"].sum()), float(pr["bytes"].sum())
     ach = kb / (kms * 1e-3) / 1e9
     rows = float(pr["rows"].sum())
-    # shared-memory gather ceiling: 4 B of LDS per edge-row at 148 SMs x 128 B/clk x 1.965 GHz
+    # shared-memory gather ceiling: every fma needs its 4-byte input delivered from shared
+    # memory to its lane; the L1 / shared data pipe delivers 128 B/clk/SM (148 SMs x 1.965 GHz)
     gather_peak = 148 * 128 * 1.965e9 / 4.0
     edge_rows = 32.0 * c["N"] * rows
+    G, cost = gen_kernel_info(net)
     out = {"workload": f"C2 perm ({c['desc']}), t = {t}", "ms_per_step": ms, "value": c["B"] * net.nnz / (ms * 1e-3),
            "unit": UNIT, "circ_layers": st["circ_layers"],
            "roofline": {"bound": "hbm", "achieved": ach, "peak": peak, "unit": "GB/s", "frac": ach / peak,
-                        "kernel": "layer_ell_kernel (general CSC, a1)", "launches": int(len(pr["ms"])),
+                        "kernel": gen_kernel_label(G), "launches": int(len(pr["ms"])),
                         "avg_launch_ms": kms / max(len(pr["ms"]), 1), "algorithmic_bytes": kb,
                         "edge_rows_per_s": edge_rows / (kms * 1e-3),
-                        "smem_gather_frac": edge_rows / (kms * 1e-3) / gather_peak},
+                        "smem_gather_frac": edge_rows / (kms * 1e-3) / gather_peak,
+                        "smem_peak_gbs": gather_peak * 4 / 1e9, "schedule_wavefronts_per_tap": cost,
+                        "hbm_ceiling_at_smem_peak": gather_peak * 4 / 1e9 / 16.0 / peak},
            "phases_ms": {k: st[k] for k in ("t_pre_ms", "t_convert_ms", "t_post_ms", "t_recover_ms")}}
     traffic, src = committed_traffic("C2_perm")
     out["roofline"]["traffic"] = traffic
@@ -475,6 +506,7 @@ def run_snicit(args):
         B_local, row0, B_global = b - a, a, c["B"]
         cap = shard_capacity(c["B"], world)
     net = make_network(args.config, args.mode, args.load, c)
+    gen_G = gen_kernel_info(net)[0] if isinstance(net, sdgc.Network) else 0
     nnz = net.nnz
     kern = {"auto": KERNEL_AUTO, "ell": KERNEL_ELL, "circ": KERNEL_CIRC}[args.kernel]
     Yh = make_inputs(args.config, c, B_local, row0)
@@ -574,7 +606,7 @@ def run_snicit(args):
                  "traffic": traffic, "traffic_unit": "bytes per launch (ncu dram read + write)",
                  "traffic_source": traffic_src,
                  "kernel": ("a1 layer kernels: layer_circ_kernel / layer_circ_seg_kernel (nu = 1), "
-                            "layer_circ_col_kernel (strided)") if st_["circ_layers"] else "layer_ell_kernel",
+                            "layer_circ_col_kernel (strided)") if st_["circ_layers"] else gen_kernel_label(gen_G),
                  "peak_source": peak_src, "launches": int(len(pm_)), "avg_launch_ms": avg_ms,
                  "avg_algorithmic_bytes": avg_bytes,
                  "layer0_frac": float(pb_[0] / (pm_[0] * 1e-3) / 1e9 / peak)}

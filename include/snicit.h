@@ -97,8 +97,10 @@ typedef struct {
                                outputs through distributed shared memory (N = 16384 / 32768 / 65536; the
                                cluster form of a row that does not fit one CTA at several CTAs per SM);
                                5 = as 1 with the row stored as pairs (y[p], y[p + N/2]) read by 8-byte
-                               loads (kernels_pre_pair.cu).  4 and 5 are measured alternatives (slower
-                               than 1 on B200), kept selectable and parity-tested.
+                               loads (kernels_pre_pair.cu).  1 uses the cluster form of 4 for rows one CTA
+                               cannot hold (N = 32768 / 65536); at N <= 16384, 4 and 5 are measured
+                               alternatives (slower than 1 on B200), kept selectable
+                               and parity-tested.
                                6 = as 1 with fma chains for every non-constant row-layer: without the
                                range prediction (R30/R31: a row whose output range or class-sum bounds
                                prove Y(t) the constant row YMAX or zero leaves early) and without the
@@ -109,7 +111,8 @@ typedef struct {
                                bitmap built by ballots: measured slower on C3).
                                Used when every layer < t is circulant
                                with 32 taps, uniform weight and uniform bias, and N/32 is one of
-                               32..512 (N = 1024..16384; 4: the cluster form supports every stride);
+                               32..512 (N = 1024..16384) or N = 32768 / 65536 (cluster form, every
+                               stride);
                                otherwise the per-layer kernels run.
                                Results are bit-identical in every mode (tested). */
     int32_t pre_const;      /* per-layer pre-convergence path (pre_fused = 0 or not applicable): 1 = a row

@@ -402,6 +402,8 @@ __global__ void __launch_bounds__(kCT, kCfMinBlocks) pre_cluster_kernel(const __
     unsigned* s_vmx = s_vmn + 2 * G * kCWp;                             // [2][G * kCWp] warp output maxima
     uint32_t* s_base = reinterpret_cast<uint32_t*>(s_vmx + 2 * G * kCWp);  // [2][G] buffer b of rank h
     int* s_surv = reinterpret_cast<int*>(s_base + 2 * G);               // [kCSurv]
+    unsigned* s_bmn = reinterpret_cast<unsigned*>(s_surv + kCSurv);      // [G * kCWp] Q32 class-sum bounds (R31)
+    unsigned* s_bmx = s_bmn + G * kCWp;
     const int tid = threadIdx.x;
     const int r = (int)cluster_ctarank();
     const int count = *a.count;
@@ -493,6 +495,52 @@ __global__ void __launch_bounds__(kCT, kCfMinBlocks) pre_cluster_kernel(const __
                 float mn = __int_as_float(0x7f800000), mx = -__int_as_float(0x7f800000);
                 const int cls = fl & 15;
                 const int nu = p.L[l].nu;
+                // R31 (kernels_pre_fused.cu pf_q32_bounds): in the C partition of a Q32 layer thread c owns
+                // residue class r T + c, whose 32 outputs all sum its 32 inputs (buffer a T + c); directed-
+                // rounding chains bound every output before any is evaluated, one extra cluster barrier
+                // gathers the bounds, and the horizon k = t - l - 1 decides as in R30
+                if (cls == CF_Q32 && a.thr_ok && l > 0 && NU_Q32 / G == T) {
+                    float slo = 0.0f, shi = 0.0f;
+#pragma unroll 8
+                    for (int kq = 0; kq < 32; ++kq) {
+                        const float x = in[kq * T + tid];
+                        slo = __fmaf_rd(x, w0, slo);
+                        shi = __fmaf_ru(x, w0, shi);
+                    }
+                    const float blo = __fsub_rd(__fmul_rd(slo, 1.0f - 0x1p-19f), 0x1p-140f);
+                    const float bhi = __fadd_ru(__fmul_ru(shi, 1.0f + 0x1p-18f), 0x1p-140f);
+                    const float ylo = sigma(__fadd_rd(blo, b0), a.ymax), yhi = sigma(__fadd_ru(bhi, b0), a.ymax);
+                    const unsigned wmn = __reduce_min_sync(0xffffffffu, __float_as_uint(ylo + 0.0f));
+                    const unsigned wmx = __reduce_max_sync(0xffffffffu, __float_as_uint(yhi + 0.0f));
+                    if ((tid & 31) == 0) {
+                        const int slot = r * kCWp + (tid >> 5);
+                        for (int h = 0; h < G; ++h) {
+                            st_cl_u32(mapa_u32(smem_u32(s_bmn + slot), (uint32_t)h), wmn);
+                            st_cl_u32(mapa_u32(smem_u32(s_bmx + slot), (uint32_t)h), wmx);
+                        }
+                    }
+                    cluster_barrier();
+                    unsigned m0 = 0xffffffffu, m1 = 0u;
+                    for (int w = tid & 31; w < G * kCWp; w += 32) {
+                        m0 = min(m0, s_bmn[w]);
+                        m1 = max(m1, s_bmx[w]);
+                    }
+                    const float bmn = __uint_as_float(__reduce_min_sync(0xffffffffu, m0));
+                    const float bmx = __uint_as_float(__reduce_max_sync(0xffffffffu, m1));
+                    const int k2 = a.t - l - 1;
+                    const int kk = min(k2, kRangeK);
+                    if (bmn >= (k2 ? p.thr_hi[kk - 1] : a.ymax)) {  // Y(t) is the constant row YMAX
+                        v = a.ymax;
+                        cst = true;
+                        break;
+                    }
+                    if (bmx <= (k2 ? p.thr_lo[kk - 1] : 0.0f)) {  // Y(t) is zero
+                        v = 0.0f;
+                        cst = true;
+                        if (a.drop && (k2 ? a.dead_t : dead_next)) dead = true;
+                        break;
+                    }
+                }
                 if (cls == CF_NU1) {
                     if (nw)
                         cf_body_nu1<RT_LOC>(in, r * kCS, w0, b0, a.ymax, rt, mn, mx);
@@ -666,7 +714,8 @@ size_t pre_cluster_smem(int N, int Hh) {
     const int G = N / kCS;
     return sizeof(float) * 2 * (size_t)(kCS + Hh) + 2 * sizeof(uint64_t) + 2 * sizeof(int) +
            2 * (size_t)G * kCWp * (sizeof(int) + sizeof(float)) + 2 * (size_t)G * sizeof(uint32_t) +
-           sizeof(uint32_t) * (size_t)((kCS + 1024) / 32) + sizeof(int) * kCSurv;
+           sizeof(uint32_t) * (size_t)((kCS + 1024) / 32) + sizeof(int) * kCSurv +
+           2 * (size_t)G * kCWp * sizeof(unsigned);
 }
 
 template <int N, bool WUNI>

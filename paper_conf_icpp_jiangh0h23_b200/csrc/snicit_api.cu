@@ -862,8 +862,9 @@ extern "C" {
 // Row-resident pre phase applicable?  (kernels_pre_fused.cu: circulant layers < t with 32 taps,
 // uniform weight and bias, N / 32 in 32..512, t <= kPfMaxLayers, smem fits); *H = circular halo
 // *cluster: the row is split over a thread-block cluster (kernels_pre_cluster.cu: N = 16384 / 32768 /
-// 65536, every layer's stride supported; only on request, pre_fused = 4: measured slower than the
-// single-CTA kernel at N = 16384 and than the per-layer kernels at N = 65536);
+// 65536, every layer's stride supported): the default for rows a single CTA cannot hold (N > 16384; C4
+// 31.8 -> 29.3 ms with R30 / R31 in the cluster kernel, round 3), on request (pre_fused = 4) at N = 16384,
+// where the single-CTA kernel is faster;
 // *bits_ok: packed input rows can be read by the chosen kernel
 static bool pf_plan(const snicit_network* net, int tt, const snicit_options& opt, int R, int* H, int* gen,
                     bool* cluster = nullptr, bool* bits_ok = nullptr) {
@@ -871,7 +872,8 @@ static bool pf_plan(const snicit_network* net, int tt, const snicit_options& opt
     if (cluster) *cluster = false;
     if (bits_ok) *bits_ok = true;
     const bool base_ok = opt.pre_fused != 0 && tt > 0 && tt <= kPfMaxLayers && R > 0 && opt.kernel == SNICIT_KERNEL_AUTO;
-    if (base_ok && opt.pre_fused == 4 && pre_cluster_supported(N)) {
+    const bool want_cluster = opt.pre_fused == 4 || (opt.pre_fused == 1 && N > 16384);
+    if (base_ok && want_cluster && pre_cluster_supported(N)) {
         bool ok = true;
         for (int l = 0; l < tt && ok; ++l) ok = net->pf_elig[l] != 0 && pre_cluster_class(N, net->plan[l].nu) >= 0;
         if (ok) {

@@ -108,3 +108,34 @@ for N, B, kw in ((16384, 24, {}), (16384, 24, dict(pre_fused=7)), (4096, 200, di
         torch.cuda.synchronize()
     print("range/popc", N, B, kw, "categories", len(cats), len(cats2), "sum", float(out.sum()))
 print("sanitize run done")
+# round 3: general-CSC row-interleaved kernel (kernels_gen.cu: G = 2 / 4 / 16 tiles, padded and ragged
+# columns, PLAIN with constant-row ranges, CENTROID / RESIDUAL in the per-layer post phase) and the
+# cluster pre kernel with R30 / R31 (the default for N = 65536)
+sys.path.insert(0, os.path.join(os.path.dirname(os.path.dirname(os.path.abspath(__file__))), "tests"))
+from test_gpu_round3 import random_k_net  # noqa: E402
+for N, K, B in ((256, 26, 300), (1024, 30, 70), (4096, 32, 20)):
+    net = random_k_net(N, 4, K, seed=N)
+    Y0 = torch.rand(B, N, device="cuda") * 8
+    out = torch.empty_like(Y0)
+    with SnicitNetwork.from_network(net) as g:
+        g.set_stream(torch.cuda.current_stream())
+        g.infer(Y0, t=2, s=32, y_out=out)
+        cats = g.categories()
+        torch.cuda.synchronize()
+    print("gen", N, K, B, "categories", len(cats), "sum", float(out.sum()))
+net = sdgc.gen_medium_network(256, 18)
+Y0 = torch.from_numpy(sdgc.gen_medium_inputs(256, 700)).cuda()
+out = torch.empty_like(Y0)
+with SnicitNetwork.from_network(net) as g:
+    g.set_stream(torch.cuda.current_stream())
+    g.infer(Y0, t=8, s=128, n_segments=0, y_out=out)
+    torch.cuda.synchronize()
+print("gen medium post per-layer sum", float(out.sum()))
+net = sdgc.gen_network(65536, 6, "radix")
+Y0 = torch.from_numpy(sdgc.gen_inputs(65536, 4)).cuda()
+out = torch.empty_like(Y0)
+with SnicitNetwork.from_network(net) as g:
+    g.set_stream(torch.cuda.current_stream())
+    g.infer(Y0, t=6, s=32, y_out=out)
+    torch.cuda.synchronize()
+print("cluster R30/R31 65536 sum", float(out.sum()))

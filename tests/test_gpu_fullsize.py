@@ -107,10 +107,12 @@ def test_full_c3_every_row():
                                oracle.layers_circulant_f32(cn, Y0s), atol=ATOL, rtol=RTOL)
 
 
-def test_c4_quarter_rows_packed():
-    """C4 (SDGC 65536 x 1920, B = 60000, t = 30) through the compact loader and the packed-input call
-    (per-layer pre phase: a row does not fit one SM): every 4th row (15000 rows) against the oracle,
-    and at every size the category set = the non-zero rows of the returned activations."""
+@pytest.mark.parametrize("pf,step", [(1, 4), (0, 16)])
+def test_c4_quarter_rows_packed(pf, step):
+    """C4 (SDGC 65536 x 1920, B = 60000, t = 30) through the compact loader and the packed-input call, with
+    the default pre phase (pf = 1: a row split over an 8-CTA cluster, R26/R30/R31) and the per-layer
+    kernels (pf = 0): every `step`-th row against the oracle, and at every size the category set = the
+    non-zero rows of the returned activations."""
     c = sdgc.CONFIGS["C4"]
     N, L, B = c["N"], c["L"], c["B"]
     cn = sdgc.gen_circulant(N, L)
@@ -118,10 +120,11 @@ def test_c4_quarter_rows_packed():
     with SnicitNetwork.circulant(cn.N, cn.L, cn.nu, cn.w, cn.bias, cn.ymax) as g:
         g.set_stream(torch.cuda.current_stream())
         out = torch.empty((B, N), dtype=torch.float32, device="cuda")
-        g.infer_packed(torch.from_numpy(bits.view(np.int32)).cuda(), t=30, s=32, y_out=out)
+        g.infer_packed(torch.from_numpy(bits.view(np.int32)).cuda(), t=30, s=32, y_out=out, pre_fused=pf)
+        assert g.stats()["pre_fused"] == (2 if pf else 0)
         cats = g.categories()
         nzrows = torch.nonzero((out != 0).any(1)).flatten().cpu().numpy()
-        rows = np.arange(0, B, 4)
+        rows = np.arange(0, B, step)
         ref_cats = _check_rows(cn, out, rows, "C4")
         del out
     assert np.array_equal(cats, nzrows)
