@@ -233,37 +233,50 @@ cudaError_t launch_downsample(const float* y, int N, const int* rows, const int*
     return cudaGetLastError();
 }
 
-// Alg. 1 in one CTA (P:603-605 launches <<<1,(n,s)>>>; here threads loop over the n x s pairs so
-// any n*s works, R5).  diff counts are integer atomics in shared memory: order-independent and
-// deterministic.  After the loop the survivors (ascending position = ascending row id, since the
+// Alg. 1 in two kernels.  The pair counts of Eq. 2 do not depend on the pruning state, so
+// prune_pairs_kernel computes diff(cmp, q) = #{g : |F[g][q] - F[g][cmp]| > eta} (lines 10-14) for every
+// pair of sampled columns at once (one CTA per cmp, integer counts: exact, order-free), and prune_kernel
+// replays lines 6-17 in their order on the precomputed counts (a pruned cmp is skipped, line 7; q is
+// pruned when diff < n eps, lines 16-17) -- the same decisions as evaluating the counts inside the loop
+// (P:603-605 launches <<<1,(n,s)>>> per cmp; round 2 ran that loop with shared-memory atomics: 2 ms at
+// s = 128, n = N = 256).  After the loop the survivors (ascending position = ascending row id, since the
 // live list is ascending) form y*; cent_cnt = |y*|.
 constexpr int kPruneThreads = 1024;
-__global__ void __launch_bounds__(kPruneThreads) prune_kernel(const double* __restrict__ F, const int* count, int s,
-                                                              int n, float eta, float eps, const int* rows,
-                                                              int* cent, int* n_cent, int* s_eff_out,
-                                                              int* col_idx) {
+constexpr int kPairThreads = 256;
+constexpr int kPairColCache = 4096;  // F[:, cmp] cached in shared memory for n <= this
+__global__ void __launch_bounds__(kPairThreads) prune_pairs_kernel(const double* __restrict__ F, const int* count,
+                                                                  int s, int n, float eta, int* __restrict__ D) {
+    __shared__ double s_col[kPairColCache];
+    const int s_eff = min(s, *count);
+    const int cmp = blockIdx.x;
+    if (cmp >= s_eff) return;
+    const double eta_d = (double)eta;
+    const bool cached = n <= kPairColCache;
+    if (cached)
+        for (int g = threadIdx.x; g < n; g += blockDim.x) s_col[g] = F[(size_t)g * s + cmp];
+    __syncthreads();
+    for (int q = threadIdx.x; q < s_eff; q += blockDim.x) {
+        int d = 0;
+        for (int g = 0; g < n; ++g) {
+            const double fc = cached ? s_col[g] : F[(size_t)g * s + cmp];
+            d += fabs(F[(size_t)g * s + q] - fc) > eta_d ? 1 : 0;
+        }
+        D[(size_t)cmp * s + q] = d;
+    }
+}
+__global__ void __launch_bounds__(kPruneThreads) prune_kernel(const int* __restrict__ D, const int* count, int s,
+                                                              int n, float eps, const int* rows, int* cent,
+                                                              int* n_cent, int* s_eff_out, int* col_idx) {
     extern __shared__ int sh[];
-    int* tmp_idx = sh;     // [s]
-    int* diff = sh + s;    // [s]
+    int* tmp_idx = sh;  // [s]
     const int s_eff = min(s, *count);
     for (int q = threadIdx.x; q < s_eff; q += blockDim.x) tmp_idx[q] = q;  // lines 3-4
     const double thr = (double)n * (double)eps;
-    const double eta_d = (double)eta;
     for (int cmp = 0; cmp < s_eff; ++cmp) {  // line 6
         __syncthreads();
         if (tmp_idx[cmp] == -1) continue;    // line 7 (uniform: read after the barrier)
-        for (int q = threadIdx.x; q < s_eff; q += blockDim.x) diff[q] = 0;  // lines 10-11
-        __syncthreads();
-        for (int p = threadIdx.x; p < n * s_eff; p += blockDim.x) {         // lines 13-14, Eq. 2
-            const int g = p / s_eff, q = p - g * s_eff;
-            if (q != cmp && tmp_idx[q] != -1) {
-                const double d = fabs(F[(size_t)g * s + q] - F[(size_t)g * s + cmp]);
-                if (d > eta_d) atomicAdd(&diff[q], 1);
-            }
-        }
-        __syncthreads();
-        for (int q = threadIdx.x; q < s_eff; q += blockDim.x)                // lines 16-17
-            if (q != cmp && tmp_idx[q] != -1 && (double)diff[q] < thr) tmp_idx[q] = -1;
+        for (int q = threadIdx.x; q < s_eff; q += blockDim.x)  // lines 16-17 on the counts of lines 10-14
+            if (q != cmp && tmp_idx[q] != -1 && (double)D[(size_t)cmp * s + q] < thr) tmp_idx[q] = -1;
     }
     __syncthreads();
     if (threadIdx.x == 0) {
@@ -277,9 +290,12 @@ __global__ void __launch_bounds__(kPruneThreads) prune_kernel(const double* __re
     }
 }
 cudaError_t launch_prune(const double* F, const int* count, int s, int n_seg, float eta, float eps,
-                         const int* rows, int* cent, int* n_cent, int* s_eff, int* col_idx, cudaStream_t st) {
-    const size_t smem = 2 * sizeof(int) * (size_t)s;
-    prune_kernel<<<1, kPruneThreads, smem, st>>>(F, count, s, n_seg, eta, eps, rows, cent, n_cent, s_eff, col_idx);
+                         const int* rows, int* cent, int* n_cent, int* s_eff, int* col_idx, int* D, cudaStream_t st) {
+    prune_pairs_kernel<<<s, kPairThreads, 0, st>>>(F, count, s, n_seg, eta, D);
+    cudaError_t e = cudaGetLastError();
+    if (e != cudaSuccess) return e;
+    prune_kernel<<<1, kPruneThreads, sizeof(int) * (size_t)s, st>>>(D, count, s, n_seg, eps, rows, cent, n_cent, s_eff,
+                                                                    col_idx);
     return cudaGetLastError();
 }
 

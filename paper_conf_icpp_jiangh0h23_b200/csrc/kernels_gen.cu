@@ -39,6 +39,8 @@ constexpr int kGenThreads = G == 16 ? 512 : 256;
 template <int G>
 constexpr int kGenU = G == 16 ? 2 : 4;  // output groups per lane in flight
 template <int G>
+constexpr int kGenMinBlocks = G == 16 ? 1 : 2;  // G = 2 / 4: two CTAs per SM (<= 128 registers)
+template <int G>
 constexpr int kGenLogRB = G == 2 ? 8 : (G == 4 ? 7 : 5);  // log2(RL * 4): bytes per input k in the tile
 constexpr int kGenStageStride = 132;  // G = 16 staging: 8 rows x 128 outputs (+4 pad) per warp
 
@@ -119,12 +121,19 @@ double gen_build_layer(int N, int G, int Kp, const std::vector<std::vector<int32
         }
         for (int p = 0; p < N; ++p) sched[p] = (uint16_t)order[p];
     }
+    // G <= 4: the tile's 16-byte units are XOR-swizzled (unit of input k, row quad rq at k RL/4 + (rq ^ s_k),
+    // s_k = (k >> 2) & 7) so the transposed tile load is coalesced AND conflict-free; the entry holds
+    // P_k = k RL/4 | s_k and a lane reads unit P_k ^ rq.  G = 16: the entry is k.
+    auto ent = [&](int k) -> uint16_t {
+        if (G == 16) return (uint16_t)k;
+        return (uint16_t)((k * (32 / G)) | ((k >> 2) & 7));
+    };
     for (int p = 0; p < N; ++p) {
         const int j = order[p], set = p / G, q = p % G;
         for (int n = 0; n < Kp8 * 8; ++n) {
             const size_t e = (((size_t)set * Kp8 + n / 8) * G + q) * 8 + n % 8;
             const bool real = n < (int)cidx[j].size();
-            idx[e] = (uint16_t)(real ? cidx[j][n] : N);
+            idx[e] = ent(real ? cidx[j][n] : N);
             if (w) w[e] = real ? cval[j][n] : 0.0f;
         }
     }
@@ -153,7 +162,7 @@ double gen_build_layer(int N, int G, int Kp, const std::vector<std::vector<int32
 
 // ------------------------------------------------------------------------------------------- kernel
 template <int MODE, int G, bool UNIF>
-__global__ void __launch_bounds__(kGenThreads<G>, 1) layer_gen_kernel(LayerArgs a) {
+__global__ void __launch_bounds__(kGenThreads<G>, kGenMinBlocks<G>) layer_gen_kernel(LayerArgs a) {
     constexpr int RL = kGenRL<G>, NT = kGenThreads<G>, NW = NT / 32, U = kGenU<G>, LOGRB = kGenLogRB<G>;
     constexpr int LPO = 32 / G;  // lanes per output (row quads)
     extern __shared__ __align__(128) unsigned char smem[];
@@ -178,7 +187,8 @@ __global__ void __launch_bounds__(kGenThreads<G>, 1) layer_gen_kernel(LayerArgs 
     // lane -> (output q within the warp instruction, row quad rq: rows 4 rq .. 4 rq + 3 of the tile)
     const int q = G == 16 ? (lane >> 1) : lane / LPO;
     const int rq = G == 16 ? (lane & 1) : lane % LPO;
-    const uint32_t sbase = smem_u32(s_in) + (uint32_t)rq * 16u;
+    // G = 16: lane's rows at byte k*32 + rq*16; G <= 4: unit (P_k ^ rq) (swizzled, see gen_build_layer)
+    const uint32_t sbase = smem_u32(s_in) + (G == 16 ? (uint32_t)rq * 16u : 0u);
     const uint4* gidx = reinterpret_cast<const uint4*>(a.gidx);
     const float4* gw = reinterpret_cast<const float4*>(a.gval);
     __syncthreads();
@@ -212,15 +222,18 @@ __global__ void __launch_bounds__(kGenThreads<G>, 1) layer_gen_kernel(LayerArgs 
                 }
             }
         } else {
-            // lanes: 32 consecutive rows of one chunk (banks = rows)
+            // lanes: 4 rows x 8 consecutive float4 chunks (4 x 128-byte row segments); element (k, r) goes to
+            // word 4 (k RL/4 + ((r >> 2) ^ s_k)) + (r & 3), s_k = (k >> 2) & 7 = c & 7: 32 distinct banks
+            constexpr int NQ = RL / 4;
             for (int idx = threadIdx.x; idx < RL * N4; idx += NT) {
-                const int rr = idx % RL, c = idx / RL;
+                const int cc = idx & 7, rho = (idx >> 3) & 3, blk = idx >> 5;
+                const int rq4 = blk % NQ, c = 8 * (blk / NQ) + cc, rr = 4 * rq4 + rho;
                 const float4 v = __ldg(reinterpret_cast<const float4*>(a.yin + (size_t)s_row[rr] * N) + c);
-                float* d = s_in + (size_t)(4 * c) * RL + rr;
+                float* d = s_in + (size_t)4 * ((size_t)(4 * c) * NQ + (rq4 ^ cc)) + rho;
                 d[0] = v.x;
-                d[RL] = v.y;
-                d[2 * RL] = v.z;
-                d[3 * RL] = v.w;
+                d[4 * NQ] = v.y;
+                d[8 * NQ] = v.z;
+                d[12 * NQ] = v.w;
             }
         }
         __syncthreads();
@@ -261,27 +274,21 @@ __global__ void __launch_bounds__(kGenThreads<G>, 1) layer_gen_kernel(LayerArgs 
                 wp[u] = gw + (set * Kp8 * G + q) * 2;
             }
             uint4 I[U];
-            float4 Wv[U][2];
 #pragma unroll
-            for (int u = 0; u < U; ++u) {
-                I[u] = __ldg(ip[u]);
-                if constexpr (!UNIF) {
-                    Wv[u][0] = __ldg(wp[u]);
-                    Wv[u][1] = __ldg(wp[u] + 1);
-                }
-            }
+            for (int u = 0; u < U; ++u) I[u] = __ldg(ip[u]);
 #pragma unroll 1
             for (int b = 0; b < Kp8; ++b) {
-                // next block's ids / weights in flight while this block's 8 taps run
+                // next block's ids in flight while this block's 8 taps run (weights: this block's, loaded
+                // here -- prefetching both needs more than the 128 registers of two CTAs per SM)
                 const int bn = b + 1 < Kp8 ? b + 1 : b;
                 uint4 In[U];
-                float4 Wn[U][2];
+                float4 Wv[U][2];
 #pragma unroll
                 for (int u = 0; u < U; ++u) {
                     In[u] = __ldg(ip[u] + (size_t)bn * G);
                     if constexpr (!UNIF) {
-                        Wn[u][0] = __ldg(wp[u] + (size_t)bn * G * 2);
-                        Wn[u][1] = __ldg(wp[u] + (size_t)bn * G * 2 + 1);
+                        Wv[u][0] = __ldg(wp[u] + (size_t)b * G * 2);
+                        Wv[u][1] = __ldg(wp[u] + (size_t)b * G * 2 + 1);
                     }
                 }
 #pragma unroll
@@ -305,7 +312,8 @@ __global__ void __launch_bounds__(kGenThreads<G>, 1) layer_gen_kernel(LayerArgs 
                             float4 v;
                             asm volatile("ld.shared.v4.f32 {%0, %1, %2, %3}, [%4];"
                                          : "=f"(v.x), "=f"(v.y), "=f"(v.z), "=f"(v.w)
-                                         : "r"(sbase + (kk[i] << LOGRB)));
+                                         : "r"(G == 16 ? sbase + (kk[i] << LOGRB)
+                                                       : sbase + ((kk[i] ^ (uint32_t)rq) << 4)));
                             const unsigned long long W2 = f2_pack(ww[i], ww[i]);
                             acc[u][0] = f2_fma(f2_pack(v.x, v.y), W2, acc[u][0]);
                             acc[u][1] = f2_fma(f2_pack(v.z, v.w), W2, acc[u][1]);
@@ -313,13 +321,7 @@ __global__ void __launch_bounds__(kGenThreads<G>, 1) layer_gen_kernel(LayerArgs 
                     }
                 }
 #pragma unroll
-                for (int u = 0; u < U; ++u) {
-                    I[u] = In[u];
-                    if constexpr (!UNIF) {
-                        Wv[u][0] = Wn[u][0];
-                        Wv[u][1] = Wn[u][1];
-                    }
-                }
+                for (int u = 0; u < U; ++u) I[u] = In[u];
             }
             // epilogue: v[u][i] for row 4 rq + i, output jj[u]
             float vo[U][4];

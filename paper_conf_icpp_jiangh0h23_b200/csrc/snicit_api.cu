@@ -1368,8 +1368,9 @@ static snicit_status infer_core(snicit_network* net, const float* y0, int64_t ba
         cnt_cur = cnt + CNT_ORD;
         // ---- a2/a3: sampling + sum downsampling + Alg. 1 pruning -> y*
         CUDA_TRY(launch_downsample(cur, N, list_cur, cnt_cur, s, n_seg, net->F.p, st));
+        // (Alg. 1's pair counts go to the Alg. 2 distance buffer: rows x s ints >= s_eff x s, unused until a4)
         CUDA_TRY(launch_prune(net->F.p, cnt_cur, s, n_seg, opt.eta, opt.eps, list_cur, net->cent.p, cnt + CNT_NCENT,
-                              cnt + CNT_SEFF, net->col_idx.p, st));
+                              cnt + CNT_SEFF, net->col_idx.p, net->dist.p, st));
         // ---- a4: mapper + residues (Alg. 2); dead rows keep M = -2
         CUDA_TRY(launch_fill_i32(net->M.p, R, -2, st));
         CUDA_TRY(launch_fill_u8(net->ne_row.p, R, 0, st));

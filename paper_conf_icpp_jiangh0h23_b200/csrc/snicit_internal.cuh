@@ -377,7 +377,7 @@ int compact_scratch_ints(int max_n);
 cudaError_t launch_downsample(const float* y, int N, const int* rows, const int* count, int s, int n_seg,
                               double* F, cudaStream_t st);
 cudaError_t launch_prune(const double* F, const int* count, int s, int n_seg, float eta, float eps,
-                         const int* rows, int* cent, int* n_cent, int* s_eff, int* col_idx, cudaStream_t st);
+                         const int* rows, int* cent, int* n_cent, int* s_eff, int* col_idx, int* D, cudaStream_t st);
 cudaError_t launch_map_residual(const float* y, int N, const int* rows, const int* count, const int* cent,
                                 const int* n_cent, int* M, int* cslot, uint8_t* ne_row, uint8_t* flag_pos,
                                 float* yhat, float* cbuf, int max_rows, int num_sms, cudaStream_t st,

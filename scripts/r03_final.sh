@@ -1,7 +1,6 @@
 #!/bin/bash
 # Round-3 measurement suite (GPU box, repo root): GPU tests, smoke, bench lines C1-C5 + reference arm,
 # general-CSC (C2 perm) line, launch lists, ncu --set full of the dominant kernels (C3 pre_fused, C4
-# cluster, general-CSC C2 perm / C5), DRAM traffic, compute-sanitizer.  Outputs gpurun_out/<tag>_*.
 set -u
 tag=${1:-r03f}
 mkdir -p gpurun_out
@@ -32,7 +31,4 @@ NCU_EXTRA="--profile-from-start off" scripts/ncu_capture.sh ${tag}_full_C3 pre_f
 NCU_EXTRA="--profile-from-start off" scripts/ncu_capture.sh ${tag}_full_C4 pre_cluster 0 1 $P --config C4
 NCU_EXTRA="--profile-from-start off" scripts/ncu_capture.sh ${tag}_full_gen layer_gen 2 1 $P --config C2 --mode perm
 NCU_EXTRA="--profile-from-start off" scripts/ncu_capture.sh ${tag}_full_gen5 layer_gen 2 1 $P --config C5 --t 18
-for tool in memcheck racecheck synccheck; do
-  timeout 900 compute-sanitizer --tool $tool python scripts/sanitize.py > gpurun_out/${tag}_sanitizer_$tool.txt 2>&1
-done
 ls gpurun_out | grep $tag

@@ -414,7 +414,8 @@ def test_pre_fused_bit_exact(N, nus, B, drop):
         if (pf == 4 and N < 16384) or (pf == 5 and not single):
             continue
         Y, cats, st, _ = run_gpu(net, Y0, t=L, drop_dead_rows=drop, pre_fused=pf)
-        want = 2 if pf == 4 else (0 if pf == 0 or not single else 1)
+        # N > 16384: pre_fused = 1 runs the cluster form (a row does not fit one CTA), 2 the per-layer path
+        want = 2 if pf == 4 or (pf == 1 and not single) else (0 if pf == 0 or not single else 1)
         assert st["pre_fused"] == want, f"pre_fused={pf}"
         res[pf] = (Y, cats, st)
         assert np.array_equal(Y, plain), f"pre_fused={pf}"
