@@ -338,10 +338,12 @@ __device__ __forceinline__ int map_classify(int r, const int* cent, int C, const
 }
 
 // TK: columns per tile (compile-time).  Shared layout [Cp centroids][TK] (float4 rows); lane j of a warp
-// owns the float4 chunks j, j + 32, .. of the tile: it reads its row elements once and compares them with
-// every centroid's elements, keeping one counter per centroid in registers (4 compares per LDS.128); the
-// warp sums each centroid's counters at the end of the tile (shuffles) and lane c adds centroid c's sum to
-// dist.  Centroids are processed in groups of 32 (register counters).
+// owns the float4 chunks j, j + 32, .. of the tile.  A warp takes R rows at once (rows p, p + nwb, ..):
+// every 16-byte centroid load is compared with the lane's elements of all R rows, so one shared-memory
+// read serves 4 R comparisons (round 2: one row, 4 -- the kernel was bound by those reads).  The R rows'
+// counts of a centroid share one 32-bit register in FW-bit fields (FW = 8 when a tile's warp sum fits in
+// 8 bits, else 16): the transpose butterfly sums all R rows at once and lane c unpacks centroid cg + c.
+// Integer counts: exact and order-free.  Centroids in groups of 32 (register counters).
 template <int TK>
 __global__ void __launch_bounds__(kMapThreads) map_dist_kernel(const float* __restrict__ y, int N, const int* rows,
                                                                const int* count, const int* cent, const int* n_cent,
@@ -350,6 +352,9 @@ __global__ void __launch_bounds__(kMapThreads) map_dist_kernel(const float* __re
                                                                const int* __restrict__ need_count) {
     extern __shared__ float4 s_c4[];
     constexpr int TK4 = TK / 4, CH = (TK4 + 31) / 32;  // float4 chunks per lane
+    constexpr int FW = CH * 4 * 32 > 255 ? 16 : 8;     // field width of one row's count (warp sums fit)
+    constexpr int R = 32 / FW;                         // rows per warp pass
+    constexpr unsigned FMASK = (1u << FW) - 1u;
     const int n = *need_count;  // rows whose distances are needed (map_need_kernel)
     const int C = min(*n_cent, s);
     if (C <= 0 || n <= 0 || map_tile(C) != TK) return;  // the launcher starts every TK variant; one matches
@@ -367,54 +372,74 @@ __global__ void __launch_bounds__(kMapThreads) map_dist_kernel(const float* __re
     __syncthreads();
     const int lane = threadIdx.x & 31, warp = threadIdx.x >> 5;
     const int nwb = (gridDim.x / ntiles) * (kMapThreads / 32);  // warps over the rows
-    auto next_row = [&](int q_) { return q_; };
     auto load_tile = [&](int q_, float4* v) {
-        const float4* yr4 = reinterpret_cast<const float4*>(y + (size_t)rows[need[q_]] * N + k0);
+        if (q_ < n) {
+            const float4* yr4 = reinterpret_cast<const float4*>(y + (size_t)rows[need[q_]] * N + k0);
 #pragma unroll
-        for (int i = 0; i < CH; ++i) {
-            const int k4 = lane + 32 * i;
-            v[i] = k4 < kl4 ? __ldg(yr4 + k4) : make_float4(0.f, 0.f, 0.f, 0.f);
+            for (int i = 0; i < CH; ++i) {
+                const int k4 = lane + 32 * i;
+                v[i] = k4 < kl4 ? __ldg(yr4 + k4) : make_float4(0.f, 0.f, 0.f, 0.f);
+            }
+        } else {
+#pragma unroll
+            for (int i = 0; i < CH; ++i) v[i] = make_float4(0.f, 0.f, 0.f, 0.f);
         }
     };
-    int p = next_row((blockIdx.x / ntiles) * (kMapThreads / 32) + warp);
-    float4 yn[CH];  // the next row's tile, loaded while this one is compared
-    if (p < n) load_tile(p, yn);
-    while (p < n) {
-        float4 yv[CH];
+    int p = (blockIdx.x / ntiles) * (kMapThreads / 32) + warp;  // rows p + r nwb, r < R
+    float4 yn[R][CH];  // the next pass's rows, loaded while this pass compares
 #pragma unroll
-        for (int i = 0; i < CH; ++i) yv[i] = yn[i];
-        const int pcur = need[p];  // list position of this row
-        p = next_row(p + nwb);
-        if (p < n) load_tile(p, yn);
+    for (int r = 0; r < R; ++r) load_tile(p + r * nwb, yn[r]);
+    while (p < n) {
+        float4 yv[R][CH];
+        int pcur[R];
+#pragma unroll
+        for (int r = 0; r < R; ++r) {
+#pragma unroll
+            for (int i = 0; i < CH; ++i) yv[r][i] = yn[r][i];
+            pcur[r] = p + r * nwb < n ? need[p + r * nwb] : -1;  // list positions of the rows
+        }
+        p += R * nwb;
+#pragma unroll
+        for (int r = 0; r < R; ++r) load_tile(p + r * nwb, yn[r]);
         for (int cg = 0; cg < Cp; cg += 32) {
-            int cnt[32];
+            unsigned cnt[32];
 #pragma unroll
             for (int j = 0; j < 32; ++j) {
-                int c_ = 0;
+                unsigned c_ = 0;
                 const float4* sc = s_c4 + (size_t)(cg + j) * TK4 + lane;
 #pragma unroll
                 for (int i = 0; i < CH; ++i) {
                     if (lane + 32 * i < kl4) {
                         const float4 cv = sc[32 * i];
-                        c_ += (yv[i].x != cv.x) + (yv[i].y != cv.y) + (yv[i].z != cv.z) + (yv[i].w != cv.w);
+#pragma unroll
+                        for (int r = 0; r < R; ++r) {
+                            const unsigned d = (yv[r][i].x != cv.x) + (yv[r][i].y != cv.y) + (yv[r][i].z != cv.z) +
+                                               (yv[r][i].w != cv.w);
+                            c_ += d << (FW * r);
+                        }
                     }
                 }
                 cnt[j] = c_;
             }
-            // transpose-reduce: after the butterfly lane j holds the warp sum of centroid cg + j
+            // transpose-reduce: after the butterfly lane j holds the warp sums of centroid cg + j (all R rows)
 #pragma unroll
             for (int o = 16; o > 0; o >>= 1) {
 #pragma unroll
                 for (int j = 0; j < o; ++j) {
                     // lanes with bit o set keep the upper half, the others the lower half
                     const bool up = (lane & o) != 0;
-                    const int send = up ? cnt[j] : cnt[j + o];
-                    const int recv = __shfl_xor_sync(0xffffffffu, send, o);
+                    const unsigned send = up ? cnt[j] : cnt[j + o];
+                    const unsigned recv = __shfl_xor_sync(0xffffffffu, send, o);
                     cnt[j] = (up ? cnt[j + o] : cnt[j]) + recv;
                 }
             }
-            const int mine = cnt[0];
-            if (cg + lane < C && mine) atomicAdd(dist + (size_t)pcur * s + cg + lane, mine);
+            if (cg + lane < C) {
+#pragma unroll
+                for (int r = 0; r < R; ++r) {
+                    const int mine = (int)((cnt[0] >> (FW * r)) & FMASK);
+                    if (pcur[r] >= 0 && mine) atomicAdd(dist + (size_t)pcur[r] * s + cg + lane, mine);
+                }
+            }
         }
     }
 }

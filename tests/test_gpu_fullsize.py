@@ -129,3 +129,54 @@ def test_c4_quarter_rows_packed(pf, step):
         del out
     assert np.array_equal(cats, nzrows)
     assert np.array_equal(np.intersect1d(cats, rows), ref_cats)
+
+
+def test_full_c2_perm_every_row():
+    """C2 with "perm" weights (general CSC: the row-interleaved kernel of kernels_gen.cu, G = 16 quads under
+    the load-time schedule; bench.py's general_csc line) at B = 60000, t = 30: the whole category set and
+    every activation against the oracle (fast mode), 1000 rows against the plain oracle."""
+    c = sdgc.CONFIGS["C2"]
+    N, L, B = c["N"], c["L"], c["B"]
+    net = sdgc.gen_network(N, L, "perm")
+    y0 = _inputs_device(N, B)
+    out = torch.empty_like(y0)
+    with SnicitNetwork.from_network(net) as g:
+        g.set_stream(torch.cuda.current_stream())
+        g.infer(y0, t=30, s=32, y_out=out)
+        cats = g.categories()
+        st = g.stats()
+    del y0
+    assert st["circ_layers"] == 0
+    ref_cats = _check_rows(net, out, np.arange(B), "C2 perm")
+    assert np.array_equal(cats, ref_cats)
+    rs = np.random.RandomState(5)
+    sample = np.sort(rs.choice(B, 1000, replace=False))
+    Y0s = np.concatenate([sdgc.gen_inputs(N, 1, row0=int(r)) for r in sample])
+    plain = oracle.layers_f32(net, Y0s)
+    np.testing.assert_allclose(out[torch.from_numpy(sample).cuda()].cpu().numpy(), plain, atol=ATOL, rtol=RTOL)
+
+
+def test_full_c5_every_row():
+    """Config 5 (medium MLP 256 x 18, per-entry weights, B = 60000; bench.py's C5 line: t = 8, s = 128,
+    n = N): the GPU SNICIT path (general-CSC kernel G = 2 in the pre phase and, per layer, in the post
+    phase; Alg. 1 from precomputed pair counts) equals the oracle's SNICIT pipeline bit for bit and the
+    plain oracle within tolerance on every row; categories exact; the uncompressed path is bit-exact."""
+    c = sdgc.CONFIGS["C5"]
+    N, L, B = c["N"], c["L"], c["B"]
+    net = sdgc.gen_medium_network(N, L)
+    Y0 = sdgc.gen_medium_inputs(N, B)
+    t = sdgc.medium_t(L)
+    plain = oracle.layers_f32(net, Y0)
+    ref = oracle.snicit(net, Y0, t=t, s=128, n=0)
+    with SnicitNetwork.from_network(net) as g:
+        g.set_stream(torch.cuda.current_stream())
+        y0 = torch.from_numpy(Y0).cuda()
+        out = torch.empty_like(y0)
+        g.infer(y0, t=t, s=128, n_segments=0, y_out=out)
+        cats = g.categories()
+        Y = out.cpu().numpy()
+        assert np.array_equal(Y, ref["Y"])
+        np.testing.assert_allclose(Y, plain, atol=ATOL, rtol=RTOL)
+        assert np.array_equal(cats, oracle.categories(plain))
+        g.infer(y0, t=L, s=128, n_segments=0, y_out=out)
+        assert np.array_equal(out.cpu().numpy(), plain)
