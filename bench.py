@@ -387,17 +387,22 @@ def residue_study(args, dev, stream, peak):
     kms = st.get("t_map_ms", -1.0)
     if kms and kms > 0:
         # map_residual (Alg. 2): the L0 distance of every mapped row to every centroid is map_rows x C x N
-        # element comparisons; each reads one centroid element from shared memory (the centroid tiles), so
-        # the bound is the shared-memory read bandwidth (148 SMs x 128 B/clk x 1.965 GHz); HBM moves
-        # 4 N per row read + 4 N per residue written (the fraction of HBM is reported alongside)
+        # element comparisons.  Round 3 compares each centroid element read from shared memory with 2-4 rows
+        # (map_dist_kernel), so the bound is the ALU issue of a comparison -- a compare and an add per
+        # element, 2 lane-ops: 148 SMs x 128 lanes x 1.965 GHz / 2 comparisons/s; `smem_equiv` keeps the
+        # round-2 reading (one 4-byte shared read per comparison against 148 x 128 B/clk x 1.965 GHz).  HBM
+        # moves 4 N per row read + 4 N per residue written (fraction reported alongside)
         comps = float(st.get("map_rows", 0)) * st["n_centroids"] * N
+        cmp_peak = 148 * 128 * 1.965e9 / 2.0 / 1e12  # Tcomparisons/s
+        ach_c = comps / (kms * 1e-3) / 1e12
         smem_peak = 148 * 128 * 1.965e9 / 1e9  # GB/s
         ach_s = 4.0 * comps / (kms * 1e-3) / 1e9
         by = 4.0 * N * (st["live_at_t"] + st["residual_at_t"])
         ach = by / (kms * 1e-3) / 1e9
-        out["map_residual_kernel"] = {"bound": "smem", "achieved": ach_s, "peak": smem_peak, "unit": "GB/s",
-                                      "frac": ach_s / smem_peak, "ms": kms, "comparisons": comps,
-                                      "peak_source": "derived: 148 SMs x 128 B/clk x 1965 MHz shared-memory reads",
+        out["map_residual_kernel"] = {"bound": "alu", "achieved": ach_c, "peak": cmp_peak, "unit": "Tcomparisons/s",
+                                      "frac": ach_c / cmp_peak, "ms": kms, "comparisons": comps,
+                                      "peak_source": "derived: 148 SMs x 128 lanes x 1965 MHz / 2 lane-ops per comparison",
+                                      "smem_equiv": {"achieved_gbs": ach_s, "peak_gbs": smem_peak, "frac": ach_s / smem_peak},
                                       "hbm": {"algorithmic_bytes": by, "achieved_gbs": ach, "frac": ach / peak}}
     rms = st.get("t_residual_ms", -1.0)
     if rms and rms > 0:
