@@ -609,10 +609,9 @@ __global__ void __launch_bounds__(T, PfCfg<T>::kMinBlocks) pre_fused_kernel(cons
         }
         if (NB == 3 && tid == 0) prev_res = false;
         if (dead && a.ydead) {  // final activations of a dead row: zeros, written now (the SMs' HBM is idle)
-            if (NB == 3) {
-                if (tid == 0) {
-                    float* dz = a.ydead + (size_t)row * N;
-                    for (int i = 0; i < N / kPfConstChunk; ++i) bulk_s2g(dz + i * kPfConstChunk, s_cz, kPfConstChunk * 4);
+            if (NB == 3) {  // one 4 KB bulk store per lane of warp 0 (issued in parallel, not by one thread)
+                if (tid < N / kPfConstChunk) {
+                    bulk_s2g(a.ydead + (size_t)row * N + tid * kPfConstChunk, s_cz, kPfConstChunk * 4);
                     bulk_commit();
                 }
             } else {
@@ -626,10 +625,8 @@ __global__ void __launch_bounds__(T, PfCfg<T>::kMinBlocks) pre_fused_kernel(cons
             if (cst) {
                 const uint32_t vb = __float_as_uint(v);
                 if (NB == 3 && (vb == __float_as_uint(a.ymax) || vb == 0u)) {  // bitwise +0 / YMAX rows
-                    if (tid == 0) {
-                        const float* src = vb == 0u ? s_cz : s_cy;
-                        for (int i = 0; i < N / kPfConstChunk; ++i)
-                            bulk_s2g(gout + i * kPfConstChunk, src, kPfConstChunk * 4);
+                    if (tid < N / kPfConstChunk) {  // one 4 KB bulk store per lane of warp 0
+                        bulk_s2g(gout + tid * kPfConstChunk, vb == 0u ? s_cz : s_cy, kPfConstChunk * 4);
                         bulk_commit();
                     }
                 } else {
@@ -683,7 +680,7 @@ __global__ void __launch_bounds__(T, PfCfg<T>::kMinBlocks) pre_fused_kernel(cons
         }
     }
     if (a.app_list) flush_surv(true);
-    if (tid == 0) bulk_wait0();
+    if (tid < 32) bulk_wait0();  // every lane that issued bulk stores (constant rows: warp 0's lanes)
 }
 
 int pre_fused_threads(int N) {
