@@ -323,18 +323,57 @@ __global__ void __launch_bounds__(kGenThreads<G>, kGenMinBlocks<G>) layer_gen_ke
 #pragma unroll
                 for (int u = 0; u < U; ++u) I[u] = In[u];
             }
-            // epilogue: v[u][i] for row 4 rq + i, output jj[u]
+            // epilogue: v[u][i] for row 4 rq + i, output jj[u].  G = 2 / 4: a lane's U = 4 outputs are
+            // consecutive, so bias, a_c (RESIDUAL) and a_out (CENTROID) move as one float4 per row
             float vo[U][4];
+            float bv[U];
+            float acv[4][U];  // RESIDUAL, G <= 4: a_c of row i, outputs jj[0..3]
+            if constexpr (G != 16) {
+                if (a.uniform_bias) {
+#pragma unroll
+                    for (int u = 0; u < U; ++u) bv[u] = __ldg(a.bias);
+                } else {
+                    const float4 b4 = __ldg(reinterpret_cast<const float4*>(a.bias + jj[0]));
+                    bv[0] = b4.x;
+                    bv[1] = b4.y;
+                    bv[2] = b4.z;
+                    bv[3] = b4.w;
+                }
+                if constexpr (MODE == MODE_RESIDUAL) {
+#pragma unroll
+                    for (int i = 0; i < 4; ++i) {
+                        const float4 c4 = __ldg(reinterpret_cast<const float4*>(a.a_c + (size_t)my_slot[i] * N + jj[0]));
+                        acv[i][0] = c4.x;
+                        acv[i][1] = c4.y;
+                        acv[i][2] = c4.z;
+                        acv[i][3] = c4.w;
+                    }
+                }
+            } else {
+#pragma unroll
+                for (int u = 0; u < U; ++u) bv[u] = a.uniform_bias ? __ldg(a.bias) : __ldg(a.bias + jj[u]);
+            }
+            float zc[4][U];  // CENTROID, G <= 4: pre-activations kept for one float4 store per row
 #pragma unroll
             for (int u = 0; u < U; ++u) {
                 const int j = jj[u];
-                const float bj = a.uniform_bias ? __ldg(a.bias) : __ldg(a.bias + j);
+                const float bj = bv[u];
                 float z[4];
                 f2_unpack(acc[u][0], z[0], z[1]);
                 f2_unpack(acc[u][1], z[2], z[3]);
 #pragma unroll
                 for (int i = 0; i < 4; ++i) {
-                    const float v = epilogue<MODE>(a, z[i], bj, j, my_row[i], my_slot[i], my_valid[i]);
+                    float v;
+                    if constexpr (G != 16 && MODE == MODE_RESIDUAL) {  // Eq. 5 second case (as epilogue<>)
+                        const float c = acv[i][u];
+                        v = sigma((c + z[i]) + bj, a.ymax) - sigma(c + bj, a.ymax);
+                        if (a.prune_eps > 0.0f && fabsf(v) <= a.prune_eps) v = 0.0f;
+                    } else if constexpr (G != 16 && MODE == MODE_CENTROID) {  // Eq. 5 first case, a_c kept
+                        zc[i][u] = z[i];
+                        v = sigma(z[i] + bj, a.ymax);
+                    } else {
+                        v = epilogue<MODE>(a, z[i], bj, j, my_row[i], my_slot[i], my_valid[i]);
+                    }
                     vo[u][i] = v;
                     if (my_valid[i]) {
                         if (v != 0.0f) anyr |= 1u << i;
@@ -365,9 +404,13 @@ __global__ void __launch_bounds__(kGenThreads<G>, kGenMinBlocks<G>) layer_gen_ke
                 // U = 4 consecutive outputs per lane: one float4 per row
 #pragma unroll
                 for (int i = 0; i < 4; ++i)
-                    if (my_valid[i])
+                    if (my_valid[i]) {
                         *reinterpret_cast<float4*>(a.yout + (size_t)my_row[i] * N + u0 + q * U) =
                             make_float4(vo[0][i], vo[1][i], vo[2][i], vo[3][i]);
+                        if constexpr (MODE == MODE_CENTROID)
+                            *reinterpret_cast<float4*>(a.a_out + (size_t)my_row[i] * N + u0 + q * U) =
+                                make_float4(zc[i][0], zc[i][1], zc[i][2], zc[i][3]);
+                    }
             }
         }
         // per-row aggregates: lanes of the same row quad combine, then one shared atomic per row
