@@ -568,9 +568,6 @@ __global__ void __launch_bounds__(kPostThreads, 2) residual_traj_kernel(PostArgs
         for (; l < a.L; ++l) {
             const PL Lnext = load_pl(a.layers + min(l + 1, a.L - 1));
             const float* ac = a.a_all + ((size_t)(l - a.t) * a.s + slot) * N;
-            // the next layer's a_c row -> L2 while this layer runs (its reads were latency-bound, round 3)
-            if (threadIdx.x == 0 && l + 1 < a.L)
-                bulk_prefetch_l2(a.a_all + ((size_t)(l + 1 - a.t) * a.s + slot) * N, (uint32_t)N * 4);
             const bool sparse = a.res_sparse && listed && Ld.kind == 1 && !a.force_ell;
             int cnt;
             bool rowconst = false;  // every output of this layer equal (dense form; a listed sparse row never is)

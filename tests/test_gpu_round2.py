@@ -352,6 +352,10 @@ def test_range_prediction_bit_exact(N, drop):
         modes = [("pl1", dict(pre_fused=0, pre_const=1)), ("pl2", dict(pre_fused=0, pre_const=2))]
         if N <= 16384:
             modes += [("pf1", dict(pre_fused=1)), ("pf6", dict(pre_fused=6))]
+        else:  # a row does not fit one CTA: pre_fused = 1 is the cluster form (R26/R30/R31, round 3)
+            modes += [("pf1", dict(pre_fused=1))]
+        if N >= 16384:
+            modes += [("pf4", dict(pre_fused=4))]
         for name, kw in modes:
             runs[name] = _infer(g, Y0, L, drop_dead_rows=drop, **kw)
             assert np.array_equal(runs[name][0], plain), name
@@ -364,6 +368,42 @@ def test_range_prediction_bit_exact(N, drop):
     if N <= 16384:
         assert runs["pf1"][2]["pre_fused"] == 1 and runs["pf6"][2]["pre_fused"] == 1
         assert runs["pf1"][2]["pre_full_rows"] < runs["pf6"][2]["pre_full_rows"]
+    else:
+        assert runs["pf1"][2]["pre_fused"] == 2
+    if N >= 16384:
+        assert runs["pf4"][2]["pre_fused"] == 2
+
+
+@pytest.mark.parametrize("t", [7, 5])
+def test_cluster_positive_bias_and_horizons(t):
+    """Cluster pre kernel (the default at N = 65536) on a net with a positive-bias layer: a zero row is not
+    absorbing before it (no dead-row drop, R23) and the range tables cover only layers that share one
+    bias (R30 off here: the layers < t do not), so rows are carried by the constant-row rule and full
+    evaluation alone; outputs equal the oracle's bit for bit and the per-layer path's."""
+    N, L, B = 65536, 7, 6
+    nu = np.array([1, 32, 1024, 2048, 1, 32, 1024], np.int32)
+    w = np.full((L, 32), 1.0 / 16.0, np.float32)
+    bias = np.full(L * N, -0.45, np.float32)
+    bias[4 * N:5 * N] = 0.05
+    cn = sdgc.CirculantNetwork(N=N, L=L, nu=nu, w=w, bias=bias, ymax=32.0)
+    net = cn.to_network()
+    rs = np.random.RandomState(t)
+    Y0 = sdgc.gen_inputs(N, B)
+    Y0[1] = np.float32(32.0)
+    Y0[2] = 0.0
+    Y0[3] = rs.uniform(0.4, 0.5, size=N).astype(np.float32)
+    plain = oracle.layers_f32(net, Y0)
+    with SnicitNetwork.from_network(net) as g:
+        g.set_stream(torch.cuda.current_stream())
+        a = _infer(g, Y0, t)
+        b = _infer(g, Y0, t, pre_fused=0)
+    assert a[2]["pre_fused"] == 2 and b[2]["pre_fused"] == 0
+    assert np.array_equal(a[0], b[0]) and np.array_equal(a[1], b[1])
+    assert np.array_equal(a[1], oracle.categories(plain))
+    if t == L:
+        assert np.array_equal(a[0], plain)
+    else:
+        np.testing.assert_allclose(a[0], plain, atol=ATOL, rtol=RTOL)
 
 
 @pytest.mark.parametrize("N", [1024, 4096, 16384])
