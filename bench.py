@@ -387,7 +387,7 @@ def residue_study(args, dev, stream, peak):
     kms = st.get("t_map_ms", -1.0)
     if kms and kms > 0:
         # map_residual (Alg. 2): the L0 distance of every mapped row to every centroid is map_rows x C x N
-        # element comparisons.  Round 3 compares each centroid element read from shared memory with 2-4 rows
+        # element comparisons.  Round 2 (r02c) compares each centroid element read from shared memory with 2-4 rows
         # (map_dist_kernel), so the bound is the ALU issue of a comparison -- a compare and an add per
         # element, 2 lane-ops: 148 SMs x 128 lanes x 1.965 GHz / 2 comparisons/s; `smem_equiv` keeps the
         # round-2 reading (one 4-byte shared read per comparison against 148 x 128 B/clk x 1.965 GHz).  HBM

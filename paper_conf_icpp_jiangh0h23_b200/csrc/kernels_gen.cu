@@ -5,7 +5,7 @@
 // (random gathers).  Every fma of a gather kernel needs one input value delivered from shared
 // memory to its lane, and the L1 / shared-memory data pipe delivers 128 B per clock per SM -- so the
 // roofline is 32 fmas/clk/SM (a quarter of the FP32 pipe), and EVERY byte a lane receives counts: a
-// 16-byte per-lane index load costs as many pipe cycles as a 16-byte data load (ncu, round 3: the first
+// 16-byte per-lane index load costs as many pipe cycles as a 16-byte data load (ncu, round 2 (r02c): the first
 // version of this kernel spent half of its data-pipe wavefronts on index loads).  Hence:
 //  * a tile holds RL rows interleaved (element (k, r) at k RL + r) and every lane owns FOUR consecutive
 //    rows: one 16-byte shared load (LDS.128) feeds two packed FFMA2 of the same tap, so an index (u16,

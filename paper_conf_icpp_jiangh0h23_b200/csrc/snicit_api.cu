@@ -863,7 +863,7 @@ extern "C" {
 // uniform weight and bias, N / 32 in 32..512, t <= kPfMaxLayers, smem fits); *H = circular halo
 // *cluster: the row is split over a thread-block cluster (kernels_pre_cluster.cu: N = 16384 / 32768 /
 // 65536, every layer's stride supported): the default for rows a single CTA cannot hold (N > 16384; C4
-// 31.8 -> 29.3 ms with R30 / R31 in the cluster kernel, round 3), on request (pre_fused = 4) at N = 16384,
+// 31.8 -> 29.3 ms with R30 / R31 in the cluster kernel, round 2 (r02c)), on request (pre_fused = 4) at N = 16384,
 // where the single-CTA kernel is faster;
 // *bits_ok: packed input rows can be read by the chosen kernel
 static bool pf_plan(const snicit_network* net, int tt, const snicit_options& opt, int R, int* H, int* gen,

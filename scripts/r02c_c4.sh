@@ -1,9 +1,9 @@
 #!/bin/bash
-# Round 3: general-CSC kernel + cluster R30 check (GPU box, repo root).  Outputs gpurun_out/<tag>_*.
+# Round 2 (r02c): general-CSC kernel + cluster R30 check (GPU box, repo root).  Outputs gpurun_out/<tag>_*.
 set -u
-tag=${1:-r03j}
+tag=${1:-r02cj}
 mkdir -p gpurun_out
-timeout 900 python -m pytest tests/test_gpu_round3.py tests/test_gpu_parity.py tests/test_gpu_round2.py -q -x -k "gen or ell or perm or medium or ragged or random or uncompressed or post_modes or pre_fused or range or cluster" > gpurun_out/${tag}_pytest.txt 2>&1
+timeout 900 python -m pytest tests/test_gpu_round2c.py tests/test_gpu_parity.py tests/test_gpu_round2.py -q -x -k "gen or ell or perm or medium or ragged or random or uncompressed or post_modes or pre_fused or range or cluster" > gpurun_out/${tag}_pytest.txt 2>&1
 echo "pytest rc=$?" >> gpurun_out/${tag}_pytest.txt
 timeout 300 python bench.py --config C2 --mode perm --quick --no-cpu-baseline > gpurun_out/${tag}_C2perm.json 2> gpurun_out/${tag}_C2perm.err
 timeout 300 python bench.py --config C5 --t 18 --quick --no-cpu-baseline > gpurun_out/${tag}_C5u.json 2> gpurun_out/${tag}_C5u.err

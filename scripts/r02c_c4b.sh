@@ -1,6 +1,6 @@
 #!/bin/bash
 set -u
-tag=${1:-r03k}
+tag=${1:-r02ck}
 mkdir -p gpurun_out
 timeout 900 python -m pytest tests/test_gpu_parity.py tests/test_gpu_round2.py -q -x -k "pre_fused or range or cluster" > gpurun_out/${tag}_pytest.txt 2>&1
 echo "pytest rc=$?" >> gpurun_out/${tag}_pytest.txt

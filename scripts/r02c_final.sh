@@ -2,7 +2,7 @@
 # Round-3 measurement suite (GPU box, repo root): GPU tests, smoke, bench lines C1-C5 + reference arm,
 # general-CSC (C2 perm) line, launch lists, ncu --set full of the dominant kernels (C3 pre_fused, C4
 set -u
-tag=${1:-r03f}
+tag=${1:-r02cf}
 mkdir -p gpurun_out
 nvidia-smi --query-gpu=name,clocks.sm,clocks.max.sm,power.draw --format=csv > gpurun_out/${tag}_smi.txt 2>&1
 timeout 1500 python -m pytest tests -m gpu -q --durations=15 > gpurun_out/${tag}_pytest_gpu.txt 2>&1

@@ -1,9 +1,9 @@
 #!/bin/bash
-# Round 3: general-CSC kernel check (GPU box, repo root).  Outputs gpurun_out/<tag>_*.
+# Round 2 (r02c): general-CSC kernel check (GPU box, repo root).  Outputs gpurun_out/<tag>_*.
 set -u
-tag=${1:-r03g}
+tag=${1:-r02cg}
 mkdir -p gpurun_out
-timeout 600 python -m pytest tests/test_gpu_round3.py tests/test_gpu_parity.py -q -x -k "gen or ell or perm or medium or ragged or random or uncompressed or post_modes" > gpurun_out/${tag}_pytest.txt 2>&1
+timeout 600 python -m pytest tests/test_gpu_round2c.py tests/test_gpu_parity.py -q -x -k "gen or ell or perm or medium or ragged or random or uncompressed or post_modes" > gpurun_out/${tag}_pytest.txt 2>&1
 echo "pytest rc=$?" >> gpurun_out/${tag}_pytest.txt
 for g in 1 0; do
   SNICIT_GEN=$g timeout 300 python bench.py --config C2 --mode perm --quick --no-cpu-baseline > gpurun_out/${tag}_C2perm_gen$g.json 2> gpurun_out/${tag}_C2perm_gen$g.err

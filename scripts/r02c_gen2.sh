@@ -1,8 +1,8 @@
 #!/bin/bash
 set -u
-tag=${1:-r03m}
+tag=${1:-r02cm}
 mkdir -p gpurun_out
-timeout 900 python -m pytest tests/test_gpu_round3.py tests/test_gpu_parity.py -q -x -k "gen or ell or perm or medium or ragged or random or uncompressed or post_modes or c1_vs or pre_fused" > gpurun_out/${tag}_pytest.txt 2>&1
+timeout 900 python -m pytest tests/test_gpu_round2c.py tests/test_gpu_parity.py -q -x -k "gen or ell or perm or medium or ragged or random or uncompressed or post_modes or c1_vs or pre_fused" > gpurun_out/${tag}_pytest.txt 2>&1
 echo "pytest rc=$?" >> gpurun_out/${tag}_pytest.txt
 timeout 300 python bench.py --config C5 --quick --no-cpu-baseline > gpurun_out/${tag}_C5.json 2> gpurun_out/${tag}_C5.err
 timeout 300 python bench.py --config C5 --t 18 --quick --no-cpu-baseline > gpurun_out/${tag}_C5u.json 2> gpurun_out/${tag}_C5u.err

@@ -1,8 +1,8 @@
 #!/bin/bash
 set -u
-tag=${1:-r03p}
+tag=${1:-r02cp}
 mkdir -p gpurun_out
-timeout 900 python -m pytest tests/test_gpu_parity.py tests/test_gpu_round2.py tests/test_gpu_round3.py -q -x -k "c1_vs or medium or perm or post_modes or residue or sparse or cluster_centroid or shard or gen" > gpurun_out/${tag}_pytest.txt 2>&1
+timeout 900 python -m pytest tests/test_gpu_parity.py tests/test_gpu_round2.py tests/test_gpu_round2c.py -q -x -k "c1_vs or medium or perm or post_modes or residue or sparse or cluster_centroid or shard or gen" > gpurun_out/${tag}_pytest.txt 2>&1
 echo "pytest rc=$?" >> gpurun_out/${tag}_pytest.txt
 timeout 600 python -m pytest tests/test_gpu_fullsize.py -q -k "c5 or c2_every" >> gpurun_out/${tag}_pytest.txt 2>&1
 echo "pytest2 rc=$?" >> gpurun_out/${tag}_pytest.txt

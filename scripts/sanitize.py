@@ -108,11 +108,11 @@ for N, B, kw in ((16384, 24, {}), (16384, 24, dict(pre_fused=7)), (4096, 200, di
         torch.cuda.synchronize()
     print("range/popc", N, B, kw, "categories", len(cats), len(cats2), "sum", float(out.sum()))
 print("sanitize run done")
-# round 3: general-CSC row-interleaved kernel (kernels_gen.cu: G = 2 / 4 / 16 tiles, padded and ragged
+# round 2 (r02c): general-CSC row-interleaved kernel (kernels_gen.cu: G = 2 / 4 / 16 tiles, padded and ragged
 # columns, PLAIN with constant-row ranges, CENTROID / RESIDUAL in the per-layer post phase) and the
 # cluster pre kernel with R30 / R31 (the default for N = 65536)
 sys.path.insert(0, os.path.join(os.path.dirname(os.path.dirname(os.path.abspath(__file__))), "tests"))
-from test_gpu_round3 import random_k_net  # noqa: E402
+from test_gpu_round2c import random_k_net  # noqa: E402
 for N, K, B in ((256, 26, 300), (1024, 30, 70), (4096, 32, 20)):
     net = random_k_net(N, 4, K, seed=N)
     Y0 = torch.rand(B, N, device="cuda") * 8

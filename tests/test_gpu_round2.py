@@ -352,7 +352,7 @@ def test_range_prediction_bit_exact(N, drop):
         modes = [("pl1", dict(pre_fused=0, pre_const=1)), ("pl2", dict(pre_fused=0, pre_const=2))]
         if N <= 16384:
             modes += [("pf1", dict(pre_fused=1)), ("pf6", dict(pre_fused=6))]
-        else:  # a row does not fit one CTA: pre_fused = 1 is the cluster form (R26/R30/R31, round 3)
+        else:  # a row does not fit one CTA: pre_fused = 1 is the cluster form (R26/R30/R31, round 2 (r02c))
             modes += [("pf1", dict(pre_fused=1))]
         if N >= 16384:
             modes += [("pf4", dict(pre_fused=4))]

@@ -1,4 +1,4 @@
-"""Round 3 GPU parity: the general-CSC row-interleaved kernel (kernels_gen.cu) against
+"""Round 2 (r02c) GPU parity: the general-CSC row-interleaved kernel (kernels_gen.cu) against
 the oracle, bit-exact (Eq. 1 P:435-438 evaluated in stored order, R12), over both tile shapes (RL = 32
 lanes over rows, RL = 8 quads of outputs), ragged tiles (row counts not a multiple of RL), ragged and
 padded columns (K not a multiple of 4), non-uniform weights and biases, and the whole SNICIT path on
