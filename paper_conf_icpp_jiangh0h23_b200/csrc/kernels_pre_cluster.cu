@@ -454,6 +454,15 @@ __global__ void __launch_bounds__(kCT, kCfMinBlocks) pre_cluster_kernel(const __
         }
     };
     uint32_t ph = 0;
+    // The row-end cluster barrier is needed only when the next row's layer 0 writes into peers' row areas:
+    // when layers 0 and 1 are both W-partitioned (the SDGC cycles), layer 0 writes remote HALOS only, which
+    // no rank reads while it finishes a row (its result store reads [0, kCS)), so a rank may start the next
+    // row at once (round 2 (r02c)).  Votes use a running layer-instance parity (gl) so the slots of a row's
+    // last layer and the next row's first layer differ; a rank is never more than one row ahead of a peer
+    // (it cannot pass the next row's layer-0 barrier alone).
+    const int cls1 = a.t > 1 ? (p.L[1].flags & 15) : CF_NU1;
+    const bool end_barrier = !(w0part && (cls1 == CF_NU1 || cls1 == CF_WSTR));
+    int gl = 0;  // evaluated layer instances (vote slot parity)
     for (int k = 0; pos < count; ++k) {
         const int row = __ldg(a.rows + pos);
         if (tid == 0) issue_load(pos, &bar[0]);
@@ -583,7 +592,7 @@ __global__ void __launch_bounds__(kCT, kCfMinBlocks) pre_cluster_kernel(const __
                     const unsigned wmn = __reduce_min_sync(0xffffffffu, __float_as_uint(mn + 0.0f));
                     const unsigned wmx = __reduce_max_sync(0xffffffffu, __float_as_uint(mx + 0.0f));
                     if ((tid & 31) == 0) {
-                        const int slot = (l & 1) * G * kCWp + r * kCWp + (tid >> 5);
+                        const int slot = (gl & 1) * G * kCWp + r * kCWp + (tid >> 5);
                         for (int h = 0; h < G; ++h) {
                             st_cl_u32(mapa_u32(smem_u32(s_vmn + slot), (uint32_t)h), wmn);
                             st_cl_u32(mapa_u32(smem_u32(s_vmx + slot), (uint32_t)h), wmx);
@@ -596,13 +605,14 @@ __global__ void __launch_bounds__(kCT, kCfMinBlocks) pre_cluster_kernel(const __
                     const int ln = tid & 31;
                     unsigned m0 = 0xffffffffu, m1 = 0u;
                     for (int w = ln; w < G * kCWp; w += 32) {
-                        m0 = min(m0, s_vmn[(l & 1) * G * kCWp + w]);
-                        m1 = max(m1, s_vmx[(l & 1) * G * kCWp + w]);
+                        m0 = min(m0, s_vmn[(gl & 1) * G * kCWp + w]);
+                        m1 = max(m1, s_vmx[(gl & 1) * G * kCWp + w]);
                     }
                     rmn = __reduce_min_sync(0xffffffffu, m0);
                     rmx = __reduce_max_sync(0xffffffffu, m1);
                 }
                 ++full;
+                ++gl;
                 cur ^= 1;
                 if (rmn == rmx) {  // constant row (R26) or dead (R23)
                     v = __uint_as_float(rmn);
@@ -682,10 +692,12 @@ __global__ void __launch_bounds__(kCT, kCfMinBlocks) pre_cluster_kernel(const __
             if (a.full_rl) atomicAdd(a.full_rl, (unsigned long long)full);
             if (a.n_const && cst) atomicAdd(a.n_const, 1);
         }
-        // every rank is done with this row's buffers before any rank writes the next row's outputs
-        cluster_barrier();
+        // every rank is done with this row's buffers before any rank writes the next row's outputs (unless
+        // the next row's first writes are halo-only, see end_barrier)
+        if (end_barrier) cluster_barrier();
         pos = s_pos[(k + 1) & 1];
     }
+    cluster_barrier();  // no CTA leaves while a peer may still access its shared memory
     if (r == 0 && tid == 0 && a.app_list && nsurv > 0) {
         const int p0 = atomicAdd(a.app_count, nsurv);
         for (int i = 0; i < nsurv; ++i) a.app_list[p0 + i] = s_surv[i];
