@@ -413,6 +413,13 @@ __global__ void __launch_bounds__(T, PfCfg<T>::kMinBlocks) pre_fused_kernel(cons
         __syncthreads();
     }
     int i_in = 0, i_out = 1, i_pf = 2;  // buffer roles (NB == 3: i_pf receives the next row)
+    // NB == 3, fp32 rows without the forced R32 pass: no CTA barrier at the row end.  The next row's first
+    // layer writes only the buffer its predecessor's last layer READ (finished before that layer's barrier),
+    // its position slot differs from the one being read, and the range slots use a running layer-instance
+    // parity (gl), so warps may start the next row while warp 0 finishes the bookkeeping (round 2 (r02c));
+    // R32 shares the R31 scratch (s_bmn) and keeps the barrier
+    const bool end_sync = NB != 3 || a.ybits != nullptr || a.popc0 == 1;
+    int gl = 0;  // evaluated layer instances (range slot parity)
     uint32_t ph = 0;                    // phase bit of bar[0], bar[1]
     if (NB == 3 && tid == 0 && pos < count) issue_load(pos, buf, &bar[0], 0);
     int np = 0;  // tid 0: the next row's list position
@@ -559,15 +566,16 @@ __global__ void __launch_bounds__(T, PfCfg<T>::kMinBlocks) pre_fused_kernel(cons
                     const unsigned wmn = __reduce_min_sync(0xffffffffu, __float_as_uint(mn + 0.0f));
                     const unsigned wmx = __reduce_max_sync(0xffffffffu, __float_as_uint(mx + 0.0f));
                     if ((tid & 31) == 0) {
-                        s_vmn[(l & 1) * kWarps + (tid >> 5)] = wmn;
-                        s_vmx[(l & 1) * kWarps + (tid >> 5)] = wmx;
+                        s_vmn[(gl & 1) * kWarps + (tid >> 5)] = wmn;
+                        s_vmx[(gl & 1) * kWarps + (tid >> 5)] = wmx;
                     }
                 }
                 __syncthreads();  // outputs and ranges written
                 {
                     const int ln = tid & 31;
-                    cmn = __reduce_min_sync(0xffffffffu, ln < kWarps ? s_vmn[(l & 1) * kWarps + ln] : 0xffffffffu);
-                    cmx = __reduce_max_sync(0xffffffffu, ln < kWarps ? s_vmx[(l & 1) * kWarps + ln] : 0u);
+                    cmn = __reduce_min_sync(0xffffffffu, ln < kWarps ? s_vmn[(gl & 1) * kWarps + ln] : 0xffffffffu);
+                    cmx = __reduce_max_sync(0xffffffffu, ln < kWarps ? s_vmx[(gl & 1) * kWarps + ln] : 0u);
+                    ++gl;
                 }
                 const bool all_eq = cmn == cmx;  // every output equal (R26)
                 const float o0 = __uint_as_float(cmn);
@@ -668,7 +676,7 @@ __global__ void __launch_bounds__(T, PfCfg<T>::kMinBlocks) pre_fused_kernel(cons
             if (np < count && a.l2_prefetch && !a.ybits)  // pull it into L2: its load is short
                 bulk_prefetch_l2(a.yin + (size_t)__ldg(a.rows + np) * N, N * 4);
         }
-        __syncthreads();  // buffers free, next position visible
+        if (end_sync) __syncthreads();  // buffers free, next position visible
         pos = s_pos[2 + (k & 1)];
         if (NB == 3) {  // the prefetched row becomes the input; the result buffer (store pending) the target
             const int ti = i_in;
