@@ -413,18 +413,21 @@ __global__ void __launch_bounds__(T, PfCfg<T>::kMinBlocks) pre_fused_kernel(cons
         __syncthreads();
     }
     int i_in = 0, i_out = 1, i_pf = 2;  // buffer roles (NB == 3: i_pf receives the next row)
-    // NB == 3, fp32 rows without the forced R32 pass: no CTA barrier at the row end.  The next row's first
+    // No CTA barrier at the row end (except pre_fused = 7).  The next row's first
     // layer writes only the buffer its predecessor's last layer READ (finished before that layer's barrier),
     // its position slot differs from the one being read, and the range slots use a running layer-instance
-    // parity (gl), so warps may start the next row while warp 0 finishes the bookkeeping (round 2 (r02c));
-    // R32 shares the R31 scratch (s_bmn) and keeps the barrier
-    const bool end_sync = NB != 3 || a.ybits != nullptr || a.popc0 == 1;
+    // parity (gl), so warps may start the next row while warp 0 finishes the bookkeeping (round 2 (r02c))
+    // (NB == 2 likewise since r02c: its next position is also claimed a row ahead and published at the
+    // row start, and its next load is issued only after the previous result's TMA store was read)
+    // (packed rows too: R32 on a given bitmap uses no shared scratch; the fp32-row R32 of pre_fused = 7
+    // reduces through s_bmn, the R31 scratch a slow warp may still read, and keeps the barrier)
+    const bool end_sync = a.popc0 == 1;
     int gl = 0;  // evaluated layer instances (range slot parity)
     uint32_t ph = 0;                    // phase bit of bar[0], bar[1]
     if (NB == 3 && tid == 0 && pos < count) issue_load(pos, buf, &bar[0], 0);
     int np = 0;  // tid 0: the next row's list position
-    // NB == 3: the position after that, claimed one row ahead so the atomic's latency is never waited on
-    int nq = (NB == 3 && tid == 0) ? atomicAdd(a.work, 1) : 0;
+    // the position after that, claimed one row ahead so the atomic's latency is never waited on
+    int nq = tid == 0 ? atomicAdd(a.work, 1) : 0;
     for (int k = 0; pos < count; ++k) {
         const int row = __ldg(a.rows + pos);
         if (tid == 0) {
@@ -432,14 +435,12 @@ __global__ void __launch_bounds__(T, PfCfg<T>::kMinBlocks) pre_fused_kernel(cons
                 bulk_wait_read0();  // the previous row's TMA store has finished reading its buffer
                 issue_load(pos, buf, &bar[k & 1], k & 1);
             }
+            np = nq;
+            nq = atomicAdd(a.work, 1);  // consumed at the next row's start
+            s_pos[2 + (k & 1)] = np;    // read at this row's end (visible after its first layer barrier)
+            if (NB == 2 && np < count && a.l2_prefetch && !a.ybits)  // pull it into L2: its load is short
+                bulk_prefetch_l2(a.yin + (size_t)__ldg(a.rows + np) * N, N * 4);
             if (NB == 3) {
-                np = nq;
-                nq = atomicAdd(a.work, 1);  // consumed at the next row's start
-            } else {
-                np = atomicAdd(a.work, 1);  // next row (consumed at the row end, latency hidden)
-            }
-            if (NB == 3) {
-                s_pos[2 + (k & 1)] = np;
                 if (np < count) {  // load it now, behind this row's compute
                     // its buffer held the previous row's result: wait until that row's TMA store has read
                     // it (older stores were waited for one row earlier; constant-row stores read s_cz/s_cy)
@@ -670,11 +671,6 @@ __global__ void __launch_bounds__(T, PfCfg<T>::kMinBlocks) pre_fused_kernel(cons
                 atomicAdd(a.dyn + full, 1ull);
                 atomicAdd(a.dyn + (a.t + 1) + lend, 1ull);
             }
-        }
-        if (NB == 2 && tid == 0) {
-            s_pos[2 + (k & 1)] = np;
-            if (np < count && a.l2_prefetch && !a.ybits)  // pull it into L2: its load is short
-                bulk_prefetch_l2(a.yin + (size_t)__ldg(a.rows + np) * N, N * 4);
         }
         if (end_sync) __syncthreads();  // buffers free, next position visible
         pos = s_pos[2 + (k & 1)];
