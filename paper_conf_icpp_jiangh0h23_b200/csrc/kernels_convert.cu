@@ -241,7 +241,6 @@ cudaError_t launch_downsample(const float* y, int N, const int* rows, const int*
 // (P:603-605 launches <<<1,(n,s)>>> per cmp; round 2 ran that loop with shared-memory atomics: 2 ms at
 // s = 128, n = N = 256).  After the loop the survivors (ascending position = ascending row id, since the
 // live list is ascending) form y*; cent_cnt = |y*|.
-constexpr int kPruneThreads = 1024;
 constexpr int kPairThreads = 256;
 constexpr int kPairColCache = 4096;  // F[:, cmp] cached in shared memory for n <= this
 __global__ void __launch_bounds__(kPairThreads) prune_pairs_kernel(const double* __restrict__ F, const int* count,
@@ -264,27 +263,52 @@ __global__ void __launch_bounds__(kPairThreads) prune_pairs_kernel(const double*
         D[(size_t)cmp * s + q] = d;
     }
 }
-__global__ void __launch_bounds__(kPruneThreads) prune_kernel(const int* __restrict__ D, const int* count, int s,
-                                                              int n, float eps, const int* rows, int* cent,
-                                                              int* n_cent, int* s_eff_out, int* col_idx) {
-    extern __shared__ int sh[];
-    int* tmp_idx = sh;  // [s]
+// Lines 6-17 replayed by ONE warp: the pruning state of sampled column q = lane + 32 m is bit m of the
+// lane's mask, a pruned cmp is skipped (line 7) after a shuffle from its owner lane, and no CTA barrier
+// separates the s sequential iterations (round 2 (r02c): 1024 threads with two barriers per cmp took
+// 88 us at s = 128; s <= 1024 so 32 bits per lane suffice).  For s <= kPruneSmemS the whole count matrix
+// is first copied to shared memory by the CTA (the loop's reads are then short-latency).
+constexpr int kPruneThreads = 1024;
+constexpr int kPruneSmemS = 128;
+__global__ void __launch_bounds__(kPruneThreads) prune_kernel(const int* __restrict__ D, const int* count, int s, int n,
+                                                              float eps, const int* rows, int* cent, int* n_cent,
+                                                              int* s_eff_out, int* col_idx) {
+    extern __shared__ int s_D[];
     const int s_eff = min(s, *count);
-    for (int q = threadIdx.x; q < s_eff; q += blockDim.x) tmp_idx[q] = q;  // lines 3-4
-    const double thr = (double)n * (double)eps;
-    for (int cmp = 0; cmp < s_eff; ++cmp) {  // line 6
+    const bool staged = s <= kPruneSmemS;
+    if (staged) {
+        for (int i = threadIdx.x; i < s_eff * s; i += blockDim.x) s_D[i] = D[i];
         __syncthreads();
-        if (tmp_idx[cmp] == -1) continue;    // line 7 (uniform: read after the barrier)
-        for (int q = threadIdx.x; q < s_eff; q += blockDim.x)  // lines 16-17 on the counts of lines 10-14
-            if (q != cmp && tmp_idx[q] != -1 && (double)D[(size_t)cmp * s + q] < thr) tmp_idx[q] = -1;
     }
-    __syncthreads();
-    if (threadIdx.x == 0) {
-        int C = 0;
-        for (int q = 0; q < s_eff; ++q) {
-            col_idx[q] = tmp_idx[q];
-            if (tmp_idx[q] != -1) cent[C++] = rows[q];
+    if (threadIdx.x >= 32) return;
+    const int* Dm = staged ? s_D : D;
+    const int lane = threadIdx.x;
+    const double thr = (double)n * (double)eps;
+    unsigned alive = 0u;  // lines 3-4: every sampled column valid
+    for (int m = 0; 32 * m + lane < s_eff; ++m) alive |= 1u << m;
+    for (int cmp = 0; cmp < s_eff; ++cmp) {  // line 6
+        const unsigned own = __shfl_sync(0xffffffffu, alive, cmp & 31);
+        if (!((own >> (cmp >> 5)) & 1u)) continue;  // line 7 (uniform)
+        const int* Dc = Dm + (size_t)cmp * s;
+        for (int m = 0; 32 * m < s_eff; ++m) {  // lines 16-17 on the counts of lines 10-14
+            const int q = 32 * m + lane;
+            if (q < s_eff && q != cmp && ((alive >> m) & 1u) && (double)Dc[q] < thr) alive &= ~(1u << m);
         }
+    }
+    for (int m = 0; 32 * m + lane < s_eff; ++m) {
+        const int q = 32 * m + lane;
+        col_idx[q] = ((alive >> m) & 1u) ? q : -1;
+    }
+    // y*: survivors in ascending q (ballot prefix per 32-column block)
+    int C = 0;
+    for (int m = 0; 32 * m < s_eff; ++m) {
+        const int q = 32 * m + lane;
+        const bool keep = q < s_eff && ((alive >> m) & 1u);
+        const unsigned bal = __ballot_sync(0xffffffffu, keep);
+        if (keep) cent[C + __popc(bal & ((1u << lane) - 1u))] = rows[q];
+        C += __popc(bal);
+    }
+    if (lane == 0) {
         *n_cent = C;
         *s_eff_out = s_eff;
     }
@@ -294,8 +318,11 @@ cudaError_t launch_prune(const double* F, const int* count, int s, int n_seg, fl
     prune_pairs_kernel<<<s, kPairThreads, 0, st>>>(F, count, s, n_seg, eta, D);
     cudaError_t e = cudaGetLastError();
     if (e != cudaSuccess) return e;
-    prune_kernel<<<1, kPruneThreads, sizeof(int) * (size_t)s, st>>>(D, count, s, n_seg, eps, rows, cent, n_cent, s_eff,
-                                                                    col_idx);
+    const size_t smem = s <= kPruneSmemS ? sizeof(int) * (size_t)s * s : 0;
+    int bps = 0;
+    e = blocks_per_sm((const void*)prune_kernel, kPruneThreads, smem, &bps);  // (sets the smem attribute)
+    if (e != cudaSuccess) return e;
+    prune_kernel<<<1, kPruneThreads, smem, st>>>(D, count, s, n_seg, eps, rows, cent, n_cent, s_eff, col_idx);
     return cudaGetLastError();
 }
 
