@@ -46,12 +46,14 @@ def _infer(g, Y0, t, s=32, row_offset=0, **opt):
 
 # ------------------------------------------------------------------------------ sharding
 
-@pytest.mark.parametrize("N,L,B,t", [(4096, 60, 6000, 10), (4096, 60, 6000, 30), (1024, 120, 2000, 5)])
-def test_sharded_inference_matches_single_gpu_and_oracle(N, L, B, t):
+@pytest.mark.parametrize("N,L,B,t,mode", [(4096, 60, 6000, 10, "radix"), (4096, 60, 6000, 30, "radix"),
+                                          (1024, 120, 2000, 5, "radix"), (1024, 40, 2000, 6, "perm")])
+def test_sharded_inference_matches_single_gpu_and_oracle(N, L, B, t, mode):
     """Rows are independent (Eq. 1), clustering runs per shard (reading R14): for G = 1, 2, 4,
     8 contiguous shards with row_offset, the concatenated category sets are identical to G = 1 and to the
-    oracle's, and every shard's activations are within tolerance of the plain oracle."""
-    net = sdgc.gen_network(N, L, "radix")
+    oracle's, and every shard's activations are within tolerance of the plain oracle (perm: the general-CSC
+    kernel on every shard, ragged tiles included)."""
+    net = sdgc.gen_network(N, L, mode)
     Y0 = sdgc.gen_inputs(N, B)
     plain = oracle.layers_f32_fast(net, Y0)
     ref_cats = oracle.categories(plain)
