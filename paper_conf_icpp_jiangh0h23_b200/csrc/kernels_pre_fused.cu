@@ -207,6 +207,49 @@ __device__ __forceinline__ void pf_q32_bounds(const float* __restrict__ in, floa
     yhi = sigma(__fadd_ru(hi, b0), ymax);
 }
 
+// R34 (exact): bounds of a stride-1 layer's outputs before it is evaluated.  Output q = sigma(chain over
+// x[q..q+31] + b0); with inputs >= 0 and w0 >= 0 the chain in any order lies in [(1 - 2^-19) S w0 -
+// 2^-140, (1 + 2^-18) S w0 + 2^-140] (R31), S = the exact window sum.  A thread bounds S for its item-1
+// and item-2 windows (pf_body_nu1's mapping: conflict-free loads) by sliding directed sums -- lo' =
+// RD(RD(lo + x_new) - x_old) <= S' whenever lo <= S (and the RU mirror) -- and returns the min / max
+// output bounds over its windows.
+template <int T>
+__device__ __forceinline__ void pf_nu1_bounds(const float* __restrict__ in, float w0, float b0, float ymax,
+                                              float& ylo, float& yhi) {
+    constexpr int M2 = 15;
+    const int i1 = threadIdx.x;
+    float smin = __int_as_float(0x7f800000), smax = 0.0f;
+#pragma unroll
+    for (int it = 0; it < 2; ++it) {
+        const float* src = it == 0 ? in + kPfM1 * i1 : in + kPfM1 * T + M2 * i1;
+        const int M = it == 0 ? kPfM1 : M2;
+        float lo = 0.0f, hi = 0.0f;
+#pragma unroll
+        for (int n = 0; n < 32; ++n) {
+            const float x = src[n];
+            lo = __fadd_rd(lo, x);
+            hi = __fadd_ru(hi, x);
+        }
+        smin = fminf(smin, lo);
+        smax = fmaxf(smax, hi);
+#pragma unroll
+        for (int m = 1; m < kPfM1; ++m) {
+            if (m < M) {
+                const float xn = src[m + 31], xo = src[m - 1];
+                lo = __fsub_rd(__fadd_rd(lo, xn), xo);
+                hi = __fsub_ru(__fadd_ru(hi, xn), xo);
+                smin = fminf(smin, lo);
+                smax = fmaxf(smax, hi);
+            }
+        }
+    }
+    smin = fmaxf(smin, 0.0f);  // S >= 0
+    const float clo = __fsub_rd(__fmul_rd(__fmul_rd(smin, w0), 1.0f - 0x1p-19f), 0x1p-140f);
+    const float chi = __fadd_ru(__fmul_ru(__fmul_ru(smax, w0), 1.0f + 0x1p-18f), 0x1p-140f);
+    ylo = sigma(__fadd_rd(clo, b0), ymax);
+    yhi = sigma(__fadd_ru(chi, b0), ymax);
+}
+
 // R32: layer 0 of stride 1 as a table lookup when the row holds zeros and one value c (checked here for
 // fp32 rows; packed rows are binary with c = one).  Warp w owns the words j = 32 w .. 32 w + 31 of the
 // row's bitmap (bit b of word j = element 32 j + b != 0; lane i holds word 32 w + i, built by one ballot
@@ -471,6 +514,7 @@ __global__ void __launch_bounds__(T, PfCfg<T>::kMinBlocks) pre_fused_kernel(cons
         float v = 0.0f;
         int full = 0, full_fma = 0;  // layers evaluated in full; of them by fma chains (not R32)
         bool popc = false;
+        bool r31_failed = false;  // R31 ran on this row without deciding it (R34 then runs at stride-1 layers)
         unsigned cmn = 0u, cmx = 0xffffffffu;  // the previous layer's output range (bits)
         int lend = a.t;  // the layer that zeroed the row (dead, R23), or t: alive after layer l <=> lend > l
         for (int l = 0; l < a.t; ++l) {
@@ -518,10 +562,17 @@ __global__ void __launch_bounds__(T, PfCfg<T>::kMinBlocks) pre_fused_kernel(cons
                     }
                 }
                 // R31: a Q32 layer's outputs are bounded by its class sums (pf_q32_bounds) before they are
-                // evaluated; the bounds of Y(l + 1) against the horizon k = t - l - 1 decide as in R30
-                if (cls == PF_Q32 && a.thr_ok && l > 0) {
+                // evaluated; R34: a stride-1 layer's by sliding window sums (pf_nu1_bounds; only after a
+                // failed R31: the rows that reach such a layer late); the bounds of Y(l + 1) against the
+                // horizon k = t - l - 1 decide as in R30
+                if ((cls == PF_Q32 || (cls == PF_NU1 && a.win_bounds && r31_failed)) && a.thr_ok && l > 0) {
                     float ylo, yhi;
-                    pf_q32_bounds<T>(in, w0, b0, a.ymax, ylo, yhi);
+                    if (cls == PF_Q32) {
+                        pf_q32_bounds<T>(in, w0, b0, a.ymax, ylo, yhi);
+                        r31_failed = true;  // (if they decide the row it ends here)
+                    } else {
+                        pf_nu1_bounds<T>(in, w0, b0, a.ymax, ylo, yhi);
+                    }
                     const unsigned wmn = __reduce_min_sync(0xffffffffu, __float_as_uint(ylo + 0.0f));
                     const unsigned wmx = __reduce_max_sync(0xffffffffu, __float_as_uint(yhi + 0.0f));
                     if ((tid & 31) == 0) {

@@ -1201,6 +1201,13 @@ static snicit_status infer_core(snicit_network* net, const float* y0, int64_t ba
         pa.drop = drop ? 1 : 0;
         pa.const_skip = opt.pre_fused != 2 ? 1 : 0;
         pa.range_pred = opt.pre_fused != 6 ? 1 : 0;  // R30 / R31 (6: R26 alone, for measurement)
+        {  // R34 with R30 / R31 (SNICIT_WINB=0: off, for A/B measurement)
+            static const bool winb_off = [] {
+                const char* e = getenv("SNICIT_WINB");
+                return e && e[0] == '0';
+            }();
+            pa.win_bounds = pa.range_pred && !winb_off ? 1 : 0;
+        }
         // R32: packed rows (1, 3, 5), every two-valued row (7), never (2, 6: fma chains only)
         pa.popc0 = (opt.pre_fused == 6 || opt.pre_fused == 2) ? 0 : (opt.pre_fused == 7 ? 1 : 2);
         pa.gen_str = pf_gen;

@@ -327,6 +327,7 @@ struct PreFusedArgs {
                                   //   [1] += rows whose layer 0 ran as a popcount table (R32)
     unsigned long long* dyn;      // nullable: [t + 1] rows by full-evaluation count, [t + 1] rows by end layer
     int range_pred;               // caller: allow the range prediction (R30)
+    int win_bounds;               // caller: R34 window-sum bounds at stride-1 layers after a failed R31
     int popc0;                    // layer 0 of stride 1 as a popcount table (R32): 0 off, 1 every two-valued
                                   //   row, 2 packed rows only (the bitmap is given; measured faster only there)
     int thr_ok;                   // range prediction on (R30; set by launch_pre_fused: one weight >= 0 and
