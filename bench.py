@@ -629,10 +629,13 @@ def run_snicit(args):
             return r
 
         def alu_roof(pm_, pb_, st_):
-            """FP32 FMA-pipe roofline of the row-resident kernel: algorithmic flops = 2 x 32 x N per full
-            row-layer evaluation (constant rows carried by a scalar chain are not counted)."""
+            """FP32 FMA-pipe roofline of the row-resident kernel: algorithmic flops = 2 x 32 x N (Eq. 1) per
+            evaluated row-layer -- by fma chains, or by the popcount table of R32 (the layer is evaluated
+            exactly, its Eq. 1 work counted however it is done); row-layers skipped by the exact shortcuts
+            (constant rows R26, range prediction R30, bounds R31 / R34) are not evaluated and not counted."""
             kms = float(pm_.sum())
-            flops = 2.0 * 32 * c["N"] * float(st_["pre_full_rows"])
+            popc_rl = float(st_.get("pre_popc_rows", 0))
+            flops = 2.0 * 32 * c["N"] * (float(st_["pre_full_rows"]) + popc_rl)
             achieved = flops / (kms * 1e-3) / 1e12
             hbm_gbs = float(pb_.sum()) / (kms * 1e-3) / 1e9
             traffic, traffic_src = committed_traffic(tag + "_fused") if tag else (None, None)
@@ -644,6 +647,7 @@ def run_snicit(args):
                               "pre_fused_kernel (row-resident a1: layers 0..t-1 of a row in shared memory)",
                     "peak_source": FMA_PEAK_SRC, "launches": int(len(pm_)), "avg_launch_ms": kms,
                     "algorithmic_flops": flops, "full_row_layers": int(st_["pre_full_rows"]),
+                    "popcount_row_layers": int(popc_rl),
                     "const_rows": int(st_["pre_const_rows"]),
                     "hbm": {"algorithmic_bytes": float(pb_.sum()), "achieved_gbs": hbm_gbs, "frac": hbm_gbs / peak,
                             "peak": peak, "peak_source": peak_src}}
