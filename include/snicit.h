@@ -107,8 +107,8 @@ typedef struct {
                                popcount layer 0 (R32: a stride-1 layer 0 on a row of zeros and one value
                                is a table lookup by window count); 2 also runs without R32.  For
                                measurement.  R32 runs on packed rows (snicit_infer_packed: the bitmap is
-                               given) and, with 1, on fp32 rows of zeros and one value when N <= 4096
-                               (the bitmap built by ballots: faster there, slower at N = 16384); 7 = as 1
+                               given) and, with 1, on fp32 rows of zeros and one value when N = 2048..4096
+                               (the bitmap built by ballots: faster there, slower at N = 1024 / 16384); 7 = as 1
                                with R32 on such fp32 rows at every N.  1 also uses
                                R34 (window-sum bounds of stride-1 layers) with R30 / R31.
                                Used when every layer < t is circulant

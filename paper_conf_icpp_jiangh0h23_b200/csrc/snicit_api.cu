@@ -1209,10 +1209,11 @@ static snicit_status infer_core(snicit_network* net, const float* y0, int64_t ba
             pa.win_bounds = pa.range_pred && !winb_off ? 1 : 0;
         }
         // R32: packed rows (1, 3, 5), every two-valued row (7), never (2, 6: fma chains only)
-        // (1 also by default for fp32 rows at N <= 4096: several CTAs per SM hide the bitmap build and its
-        // barriers -- C2 1.26 -> 1.15 ms; at N = 16384, one CTA per SM, it is slower: 3.91 -> 4.47 ms)
+        // (1 also by default for fp32 rows at N = 2048..4096: several CTAs per SM hide the bitmap build and its
+        // barriers -- C2 1.26 -> 1.15 ms; at N = 16384, one CTA per SM, it is slower: 3.91 -> 4.47 ms, and
+        // at N = 1024 (C1, 2000 rows) 0.30 -> 0.33 ms)
         pa.popc0 = (opt.pre_fused == 6 || opt.pre_fused == 2) ? 0
-                   : (opt.pre_fused == 7 || (opt.pre_fused == 1 && N <= 4096)) ? 1 : 2;
+                   : (opt.pre_fused == 7 || (opt.pre_fused == 1 && N >= 2048 && N <= 4096)) ? 1 : 2;
         pa.gen_str = pf_gen;
         pa.yin = cur;
         pa.ybits = y0_mode == 3 ? bits : nullptr;

@@ -411,7 +411,7 @@ def test_cluster_positive_bias_and_horizons(t):
 @pytest.mark.parametrize("N", [1024, 4096, 16384])
 def test_popcount_layer0_bit_exact(N):
     """R32: layer 0 (stride 1) of a row of zeros and one value c runs as a table lookup by window count
-    (k fmas of c from +0, in any order); on fp32 rows with pre_fused = 7 (and by default at N <= 4096), on
+    (k fmas of c from +0, in any order); on fp32 rows with pre_fused = 7 (and by default at N = 2048..4096), on
     packed rows by default.  Rows with c in {1, 0.3, 1.7, 0.02, YMAX, 1e-39 (subnormal)},
     all-zero rows, and rows with two different non-zero values (fma chains): the uncompressed outputs equal
     the oracle's and the run without R32 (pre_fused = 2 / 6) bit for bit; stats.pre_popc_rows counts
@@ -435,9 +435,9 @@ def test_popcount_layer0_bit_exact(N):
         Y1, c1, st1 = _infer(g, Y0, L, pre_fused=7)  # R32 on fp32 rows too
         assert st1["pre_fused"] == 1 and st1["pre_popc_rows"] == int(two_valued.sum())
         assert np.array_equal(Y1, plain) and np.array_equal(c1, oracle.categories(plain))
-        for pf in (1, 2, 6):  # 1: R32 on fp32 rows too at N <= 4096 (several CTAs per SM), else packed only
+        for pf in (1, 2, 6):  # 1: R32 on fp32 rows too at N = 2048..4096 (several CTAs per SM), else packed only
             Y2, c2, st2 = _infer(g, Y0, L, pre_fused=pf)
-            want = int(two_valued.sum()) if (pf == 1 and N <= 4096) else 0
+            want = int(two_valued.sum()) if (pf == 1 and 2048 <= N <= 4096) else 0
             assert st2["pre_popc_rows"] == want and np.array_equal(Y2, plain), pf
         # SNICIT path (t < L) agrees with the per-layer pre phase
         Y3, c3, _ = _infer(g, Y0, 4, pre_fused=7)
