@@ -410,7 +410,8 @@ __global__ void __launch_bounds__(T, PfCfg<T>::kMinBlocks) pre_fused_kernel(cons
     __syncthreads();
     int pos = s_pos[0];
     // one row (and its circular halo: a second copy of the row head) -> buffer `dst`, completion on `b`
-    uint32_t* s_bits = reinterpret_cast<uint32_t*>(s_bmx + 2 * kWarps);  // [2][N/32] packed rows (a.ybits)
+    unsigned* s_red = s_bmx + 2 * kWarps;  // [4 kWarps] R32's fp32-row reduction (its own: no row-end barrier)
+    uint32_t* s_bits = reinterpret_cast<uint32_t*>(s_red + 4 * kWarps);  // [2][N/32] packed rows (a.ybits)
     int* s_surv = reinterpret_cast<int*>(s_bits + 2 * (N / 32));       // [kPfSurv] rows alive at t, batched
     // NB == 3 (one CTA per SM): 4 KB rows of zeros and of YMAX, the sources of the TMA bulk stores that
     // write dead rows and constant-YMAX rows (16 bulk copies issued by one thread instead of N/4 vector
@@ -456,15 +457,12 @@ __global__ void __launch_bounds__(T, PfCfg<T>::kMinBlocks) pre_fused_kernel(cons
         __syncthreads();
     }
     int i_in = 0, i_out = 1, i_pf = 2;  // buffer roles (NB == 3: i_pf receives the next row)
-    // No CTA barrier at the row end (except pre_fused = 7).  The next row's first
-    // layer writes only the buffer its predecessor's last layer READ (finished before that layer's barrier),
-    // its position slot differs from the one being read, and the range slots use a running layer-instance
-    // parity (gl), so warps may start the next row while warp 0 finishes the bookkeeping (round 2 (r02c))
-    // (NB == 2 likewise since r02c: its next position is also claimed a row ahead and published at the
-    // row start, and its next load is issued only after the previous result's TMA store was read)
-    // (packed rows too: R32 on a given bitmap uses no shared scratch; the fp32-row R32 of pre_fused = 7
-    // reduces through s_bmn, the R31 scratch a slow warp may still read, and keeps the barrier)
-    const bool end_sync = a.popc0 == 1;
+    // No CTA barrier at the row end.  The next row's first layer writes only the buffer its predecessor's
+    // last layer READ (finished before that layer's barrier), its position slot (claimed a row ahead,
+    // published at the row start) differs from the one being read, the range slots use a running
+    // layer-instance parity (gl), R32 reduces through its own scratch, and a row buffer is reloaded only
+    // after its TMA store was read -- so warps may start the next row while warp 0 finishes the bookkeeping
+    // (round 2 (r02c))
     int gl = 0;  // evaluated layer instances (range slot parity)
     uint32_t ph = 0;                    // phase bit of bar[0], bar[1]
     if (NB == 3 && tid == 0 && pos < count) issue_load(pos, buf, &bar[0], 0);
@@ -556,7 +554,7 @@ __global__ void __launch_bounds__(T, PfCfg<T>::kMinBlocks) pre_fused_kernel(cons
                 // output is tab[k], 33 values; the windows' counts are popcounts of the row's bitmap
                 if (l == 0 && cls == PF_NU1 && (a.popc0 == 1 || (a.popc0 == 2 && a.ybits))) {
                     if (pf_popc_layer0<T>(in, out, a.ybits ? s_bits + (k & 1) * (N / 32) : nullptr, a.one, w0, b0,
-                                          a.ymax, H, s_bmn, s_tabw, mn, mx)) {
+                                          a.ymax, H, s_red, s_tabw, mn, mx)) {
                         popc = true;
                         goto layer_done;
                     }
@@ -723,7 +721,6 @@ __global__ void __launch_bounds__(T, PfCfg<T>::kMinBlocks) pre_fused_kernel(cons
                 atomicAdd(a.dyn + (a.t + 1) + lend, 1ull);
             }
         }
-        if (end_sync) __syncthreads();  // buffers free, next position visible
         pos = s_pos[2 + (k & 1)];
         if (NB == 3) {  // the prefetched row becomes the input; the result buffer (store pending) the target
             const int ti = i_in;
@@ -746,7 +743,7 @@ int pre_fused_threads(int N) {
 
 size_t pre_fused_smem(int N, int H) {
     const int nb = N / 32 >= 512 ? 3 : 2;  // kPfBufs
-    return sizeof(float) * nb * (size_t)(N + H) + 2 * sizeof(uint64_t) + 4 * sizeof(int) + 8 * sizeof(int) * (N / 32 / 32) +
+    return sizeof(float) * nb * (size_t)(N + H) + 2 * sizeof(uint64_t) + 4 * sizeof(int) + 12 * sizeof(int) * (N / 32 / 32) +
            2 * sizeof(uint32_t) * (size_t)(N / 32) + sizeof(int) * kPfSurv +  // packed-row slots, survivors
            sizeof(float) * kPfTabStride * (N / 32 / 32) +                    // R32 tables
            (nb == 3 ? 2 * sizeof(float) * kPfConstChunk : 0);                 // constant-row store sources
