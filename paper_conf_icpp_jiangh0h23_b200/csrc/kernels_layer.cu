@@ -416,7 +416,9 @@ bool gen_enabled() {
 
 cudaError_t launch_layer_ell(const LayerArgs& a, int mode, int max_rows, int num_sms, cudaStream_t st) {
     if (max_rows <= 0) return cudaSuccess;
-    if (a.gidx && gen_enabled()) return launch_layer_gen(a, mode, max_rows, num_sms, st);
+    // few rows (the centroid rows of the post phase): the tiled kernel would occupy a handful of CTAs, the
+    // thread-per-output kernel below spreads them over more (C5: 128 centroid rows per post layer)
+    if (a.gidx && gen_enabled() && max_rows > 256) return launch_layer_gen(a, mode, max_rows, num_sms, st);
     switch (mode) {
         case MODE_PLAIN: return launch_ell_m<MODE_PLAIN>(a, max_rows, num_sms, st);
         case MODE_CENTROID: return launch_ell_m<MODE_CENTROID>(a, max_rows, num_sms, st);
